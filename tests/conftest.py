@@ -1,0 +1,21 @@
+import os
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+
+def pytest_configure(config):
+    config.addinivalue_line("markers", "gpu: needs a B200 (sm_100a) and the built libtsv.so")
+    config.addinivalue_line("markers", "slow: long-running CPU test")
+
+
+@pytest.fixture(scope="session")
+def tt_layers():
+    """torchtitan's mirror of BFL's public FLUX layers: an independent library implementation
+    of the architecture, used only as a pin for the oracle."""
+    layers = pytest.importorskip("torchtitan.experiments.flux.model.layers")
+    return layers
