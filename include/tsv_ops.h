@@ -1,0 +1,66 @@
+/*
+ * tsv_ops.h — kernel-level C-ABI of libtsv.so (device pointers), used by the parity tests and
+ * the kernel micro-benchmarks.  Each entry launches exactly the kernel the step uses for that
+ * operation; no host computation.  All pointers are device pointers owned by the caller;
+ * `stream` is a cudaStream_t (NULL = legacy default stream).  Asynchronous; errors are launch
+ * errors (TSV_E_CUDA) or argument errors (TSV_E_INVAL) with tsv_last_error() set.
+ *
+ * Citations: S:§8(a) rows of SURVEY.md (the hot-path scope table); TT = public FLUX.1 code
+ * (architecture facts; the paper cites FLUX.1-dev without equations).
+ */
+#ifndef TSV_OPS_H_
+#define TSV_OPS_H_
+
+#include <stdint.h>
+#include "tsv.h"
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* GEMM epilogue modes (y = A W^T + bias, fp32 accumulate, S:§8(a) a1/a3/a8/a9/a11/a12) */
+enum {
+  TSV_EPI_STORE_BF16 = 0, /* out0 bf16 [M, ld0] = y */
+  TSV_EPI_GELU_BF16 = 1,  /* out0 = gelu_tanh(y) */
+  TSV_EPI_SILU_BF16 = 2,  /* out0 = silu(y) */
+  TSV_EPI_SPLIT_GELU = 3, /* n < n_split: out0[m, n] = y; else out1[m, n - n_split] = gelu_tanh(y) */
+  TSV_EPI_RESID_GATE = 4, /* out0 fp32 [m, n] += gate[n] * y */
+  TSV_EPI_STORE_F32 = 5,  /* out0 fp32 = y */
+  TSV_EPI_ACCUM_F32 = 6,  /* out0 fp32 += y */
+  TSV_EPI_EULER = 7       /* out1 fp32 (optional) = y; out0 fp32 += (*scalar) * y */
+};
+
+/* A [M, K] bf16 (row stride lda elements), W [N, K] bf16 (nn.Linear layout, row stride ldw),
+ * bias [N] bf16 or NULL, gate [N] fp32, scalar: device fp32.  K % 64 == 0, N % 64 == 0, 16-byte
+ * aligned operands and row strides.  force_bn in {0 (auto), 64, 128, 256}. */
+tsv_status tsv_op_gemm(const void* A, int64_t lda, const void* W, int64_t ldw, int M, int N, int K, int mode,
+                       void* out0, int64_t ld0, void* out1, int64_t ld1, int n_split, const void* bias,
+                       const float* gate, const float* scalar, int force_bn, void* stream);
+
+/* a2: u[m, :] = bf16(LN(x[m, :]) * (1 + scale) + shift); x fp32, LN without affine, eps 1e-6. */
+tsv_status tsv_op_ln_mod(const float* x, int64_t ldx, void* u, int64_t ldu, const float* shift,
+                         const float* scale, int M, int h, void* stream);
+
+/* a4: on qkv bf16 [rows, 3*H*D] (columns "(K H D)"), q and k of every head become
+ * RoPE(RMSNorm(x) * g) (eps 1e-6; pair (2j, 2j+1) rotated by the per-row table angle j).
+ * Rows < n_first use gains gq0/gk0, the others gq1/gk1 (bf16 [D]).  cos/sin: fp32 [rows, D/2].
+ * pack == NULL: in place.  Otherwise q, k, v are written to pack laid out
+ * [k_sp][rows][3][H/k_sp][D] (the Ulysses send buffer) and qkv is not modified. */
+tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int H, int D, const void* gq0,
+                               const void* gk0, const void* gq1, const void* gk1, const float* cosb,
+                               const float* sinb, void* pack, int k_sp, void* stream);
+
+/* a6: O = softmax(q k^T / sqrt(D)) v, non-causal, per head h < H; q(l, h) at q + l*ldq + h*D
+ * (bf16, same for k, v, o).  D in {64, 128}. */
+tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
+                            void* o, int64_t ldo, int L, int H, int D, void* stream);
+
+/* SYNTH-1 on device: n values of (seed, tensor_id) starting at element idx0.
+ * kind 0: bf16 rne(r*c); 1: bf16 rne(1 + r*c); 2: fp32 r*c. */
+tsv_status tsv_op_synth(void* dst, uint64_t seed, uint32_t tensor_id, uint64_t idx0, int64_t n, int kind, float c,
+                        void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TSV_OPS_H_ */

@@ -1,0 +1,239 @@
+"""B200-native step-level-SP DiT step (TetriServe's hot path): Python binding of libtsv.so.
+
+The functions below keep the C-ABI's names (without the ``tsv_`` prefix) and only marshal
+arguments; every step runs in libtsv.so's sm_100a kernels.  ``Engine`` is a thin owner of an
+engine handle with the same methods.
+"""
+from __future__ import annotations
+
+import ctypes as C
+
+import numpy as np
+
+from ._lib import EPI, EXPORTED, LIB_PATH, ModelDesc, TsvError, check, last_error, lib  # noqa: F401
+
+__all__ = ["Engine", "ModelDesc", "TsvError", "model_preset", "shard_range", "reshard_plan", "nccl_unique_id",
+           "op_gemm", "op_ln_mod", "op_qk_norm_rope", "op_attention", "op_synth", "EPI", "LIB_PATH"]
+
+
+def model_preset(name: str) -> ModelDesc:
+    d = ModelDesc()
+    check(lib.tsv_model_preset(name.encode(), C.byref(d)))
+    return d
+
+
+def shard_range(n_rows: int, k: int, rank: int) -> tuple[int, int]:
+    b, e = C.c_int64(), C.c_int64()
+    check(lib.tsv_shard_range(n_rows, k, rank, C.byref(b), C.byref(e)))
+    return b.value, e.value
+
+
+def reshard_plan(n_rows: int, k_src: int, k_dst: int):
+    buf = (C.c_int64 * (5 * (k_src + k_dst)))()
+    n = C.c_int()
+    check(lib.tsv_reshard_plan(n_rows, k_src, k_dst, buf, k_src + k_dst, C.byref(n)))
+    return [tuple(buf[5 * i:5 * i + 5]) for i in range(n.value)]
+
+
+def nccl_unique_id() -> bytes:
+    buf = (C.c_uint8 * 128)()
+    check(lib.tsv_nccl_unique_id(buf))
+    return bytes(buf)
+
+
+def _f32p(a: np.ndarray):
+    assert a.dtype == np.float32 and a.flags.c_contiguous
+    return a.ctypes.data_as(C.POINTER(C.c_float))
+
+
+def _u16p(a: np.ndarray):
+    assert a.dtype == np.uint16 and a.flags.c_contiguous
+    return a.ctypes.data_as(C.POINTER(C.c_uint16))
+
+
+class Engine:
+    """Owns a tsv_engine*.  ``devices[i]`` hosts global rank ``rank_base + i``."""
+
+    def __init__(self, model: str | ModelDesc = "flux", devices=(0,), rank_base: int = 0,
+                 world_size: int | None = None, weight_seed: int = 0x7E7125E7):
+        desc = model_preset(model) if isinstance(model, str) else model
+        self.desc = desc
+        devs = (C.c_int * len(devices))(*devices)
+        self.n_local = len(devices)
+        self.world_size = world_size if world_size is not None else rank_base + len(devices)
+        h = C.c_void_p()
+        check(lib.tsv_engine_create(C.byref(desc), devs, len(devices), rank_base, self.world_size, weight_seed,
+                                    C.byref(h)))
+        self.h = h
+        self._groups: dict[tuple, int] = {}
+
+    def close(self):
+        if self.h:
+            lib.tsv_engine_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # --------------------------------------------------------------- groups
+    def init_world(self, nccl_id: bytes):
+        check(lib.tsv_engine_init_world(self.h, (C.c_uint8 * 128).from_buffer_copy(nccl_id)))
+
+    def group_create(self, ranks, nccl_id: bytes | None = None) -> int:
+        ranks = tuple(int(r) for r in ranks)
+        if ranks in self._groups and nccl_id is None:
+            return self._groups[ranks]
+        arr = (C.c_int * len(ranks))(*ranks)
+        g = C.c_int32()
+        idp = (C.c_uint8 * 128).from_buffer_copy(nccl_id) if nccl_id is not None else None
+        check(lib.tsv_group_create(self.h, arr, len(ranks), idp, C.byref(g)))
+        self._groups[ranks] = g.value
+        return g.value
+
+    # --------------------------------------------------------------- requests
+    def request_create(self, height: int, width: int, num_steps: int = 20, seed: int = 1000,
+                       guidance: float = 3.5) -> int:
+        r = C.c_int64()
+        check(lib.tsv_request_create(self.h, height, width, num_steps, seed, guidance, C.byref(r)))
+        return r.value
+
+    def request_set_inputs(self, req: int, x=None, T_bits=None, y_bits=None):
+        check(lib.tsv_request_set_inputs(self.h, req, _f32p(x) if x is not None else None,
+                                         _u16p(T_bits) if T_bits is not None else None,
+                                         _u16p(y_bits) if y_bits is not None else None))
+
+    def request_step(self, req: int, step: int, group: int) -> int:
+        ev = C.c_int64(-1)
+        check(lib.tsv_request_step(self.h, req, step, group, C.byref(ev)))
+        return ev.value
+
+    def request_reshard(self, req: int, group: int) -> int:
+        ev = C.c_int64(-1)
+        check(lib.tsv_request_reshard(self.h, req, group, C.byref(ev)))
+        return ev.value
+
+    def event_wait(self, ev: int):
+        check(lib.tsv_event_wait(self.h, ev))
+
+    def event_query(self, ev: int) -> bool:
+        d = C.c_int()
+        check(lib.tsv_event_query(self.h, ev, C.byref(d)))
+        return bool(d.value)
+
+    def group_record(self, group: int) -> int:
+        ev = C.c_int64()
+        check(lib.tsv_group_record(self.h, group, C.byref(ev)))
+        return ev.value
+
+    def event_elapsed_ms(self, a: int, b: int) -> float:
+        ms = C.c_float()
+        check(lib.tsv_event_elapsed_ms(self.h, a, b, C.byref(ms)))
+        return ms.value
+
+    def request_info(self, req: int):
+        ns, g, li = C.c_int(), C.c_int32(), C.c_int64()
+        check(lib.tsv_request_info(self.h, req, C.byref(ns), C.byref(g), C.byref(li)))
+        return ns.value, g.value, li.value
+
+    def read_latent(self, req: int, row0: int = 0, nrows: int | None = None, out: np.ndarray | None = None):
+        li = self.request_info(req)[2]
+        nrows = li - row0 if nrows is None else nrows
+        out = np.empty((nrows, self.desc.in_ch), np.float32) if out is None else out
+        check(lib.tsv_request_read_latent(self.h, req, row0, nrows, _f32p(out)))
+        return out
+
+    def write_latent(self, req: int, x: np.ndarray, row0: int = 0):
+        x = np.ascontiguousarray(x, dtype=np.float32)
+        check(lib.tsv_request_write_latent(self.h, req, row0, x.shape[0], _f32p(x)))
+
+    def read_velocity(self, req: int, row0: int = 0, nrows: int | None = None):
+        li = self.request_info(req)[2]
+        nrows = li - row0 if nrows is None else nrows
+        out = np.empty((nrows, self.desc.in_ch), np.float32)
+        check(lib.tsv_request_read_velocity(self.h, req, row0, nrows, _f32p(out)))
+        return out
+
+    def request_destroy(self, req: int):
+        check(lib.tsv_request_destroy(self.h, req))
+
+    def latency_table(self, res_px, ks, warmup: int = 3, iters: int = 20):
+        res_px, ks = list(res_px), list(ks)
+        ms = (C.c_double * (len(res_px) * len(ks)))()
+        cv = (C.c_double * (len(res_px) * len(ks)))()
+        check(lib.tsv_latency_table(self.h, (C.c_int * len(res_px))(*res_px), len(res_px),
+                                    (C.c_int * len(ks))(*ks), len(ks), warmup, iters, ms, cv))
+        return (np.array(ms[:]).reshape(len(res_px), len(ks)), np.array(cv[:]).reshape(len(res_px), len(ks)))
+
+    def debug_read_weight(self, tensor_id: int, n: int) -> np.ndarray:
+        out = np.empty(n, np.uint16)
+        check(lib.tsv_debug_read_weight(self.h, tensor_id, _u16p(out), n))
+        return out
+
+    PROF_CLASSES = ("gemm", "attention", "ln_mod", "qk_norm_rope", "a2a", "other")
+
+    def profile(self, enable: bool = True):
+        check(lib.tsv_engine_profile(self.h, int(enable)))
+
+    def profile_read(self) -> dict:
+        n = len(self.PROF_CLASSES)
+        ms, fl, by = (C.c_double * n)(), (C.c_double * n)(), (C.c_double * n)()
+        la = (C.c_int64 * n)()
+        check(lib.tsv_engine_profile_read(self.h, ms, la, fl, by))
+        return {c: dict(ms=ms[i], launches=la[i], flops=fl[i], bytes=by[i]) for i, c in enumerate(self.PROF_CLASSES)}
+
+    def kernel_count(self) -> int:
+        c = C.c_int64()
+        check(lib.tsv_engine_kernel_count(self.h, C.byref(c)))
+        return c.value
+
+
+# ------------------------------------------------------------------- kernel-level ops (device pointers)
+def _ptr(t):
+    if t is None:
+        return None
+    return C.c_void_p(t.data_ptr() if hasattr(t, "data_ptr") else int(t))
+
+
+def _stream(stream):
+    if stream is None:
+        import torch
+        return C.c_void_p(torch.cuda.current_stream().cuda_stream)
+    return C.c_void_p(int(stream))
+
+
+def op_gemm(A, W, mode, out0, out1=None, bias=None, gate=None, scalar=None, n_split=0, M=None, N=None, K=None,
+            lda=None, ldw=None, ld0=None, ld1=None, force_bn=0, stream=None):
+    M = A.shape[0] if M is None else M
+    K = A.shape[1] if K is None else K
+    N = W.shape[0] if N is None else N
+    lda = A.stride(0) if lda is None else lda
+    ldw = W.stride(0) if ldw is None else ldw
+    ld0 = out0.stride(0) if ld0 is None else ld0
+    ld1 = (out1.stride(0) if out1 is not None else 0) if ld1 is None else ld1
+    check(lib.tsv_op_gemm(_ptr(A), lda, _ptr(W), ldw, M, N, K, EPI[mode] if isinstance(mode, str) else mode,
+                          _ptr(out0), ld0, _ptr(out1), ld1, n_split, _ptr(bias), _ptr(gate), _ptr(scalar), force_bn,
+                          _stream(stream)))
+
+
+def op_ln_mod(x, u, shift, scale, stream=None):
+    M, h = x.shape
+    check(lib.tsv_op_ln_mod(_ptr(x), x.stride(0), _ptr(u), u.stride(0), _ptr(shift), _ptr(scale), M, h,
+                            _stream(stream)))
+
+
+def op_qk_norm_rope(qkv, n_first, H, D, gq0, gk0, gq1, gk1, cosb, sinb, pack=None, k_sp=1, stream=None):
+    rows = qkv.shape[0]
+    check(lib.tsv_op_qk_norm_rope(_ptr(qkv), qkv.stride(0), rows, n_first, H, D, _ptr(gq0), _ptr(gk0), _ptr(gq1),
+                                  _ptr(gk1), _ptr(cosb), _ptr(sinb), _ptr(pack), k_sp, _stream(stream)))
+
+
+def op_attention(q, k, v, o, L, H, D, ldq=None, ldk=None, ldv=None, ldo=None, stream=None):
+    check(lib.tsv_op_attention(_ptr(q), ldq or q.stride(0), _ptr(k), ldk or k.stride(0), _ptr(v), ldv or v.stride(0),
+                               _ptr(o), ldo or o.stride(0), L, H, D, _stream(stream)))
+
+
+def op_synth(dst, seed, tensor_id, n, kind, c, idx0=0, stream=None):
+    check(lib.tsv_op_synth(_ptr(dst), seed, tensor_id, idx0, n, kind, float(c), _stream(stream)))

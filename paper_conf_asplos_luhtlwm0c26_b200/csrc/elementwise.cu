@@ -1,0 +1,271 @@
+// HBM-bound kernels of the step (S:§8(a) a2, a4, Ulysses pack/unpack) plus the SYNTH-1 generator.
+// Vectorised 16-byte accesses, one warp per row (LN) or per (row, head) (QK-norm + RoPE).
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace tsv {
+
+// ------------------------------------------------------------------ a2: LN-modulate
+// u = LN(x) (no affine, biased variance, eps 1e-6) * (1 + scale) + shift   -> bf16
+template <int NV>  // float4 per lane: h = 128 * NV
+__global__ void __launch_bounds__(256) ln_mod_kernel(const float* __restrict__ x, long long ldx, bf16* __restrict__ u,
+                                                     long long ldu, const float* __restrict__ shift,
+                                                     const float* __restrict__ scale, int M) {
+  const int row = blockIdx.x * 8 + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (row >= M) return;
+  constexpr int h = 128 * NV;
+  const float4* xr = reinterpret_cast<const float4*>(x + (long long)row * ldx);
+  float4 v[NV];
+  float s = 0.f;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    v[i] = __ldcs(xr + i * 32 + lane);
+    s += (v[i].x + v[i].y) + (v[i].z + v[i].w);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  const float mean = s * (1.0f / h);
+  float q = 0.f;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    float a = v[i].x - mean, b = v[i].y - mean, c = v[i].z - mean, d = v[i].w - mean;
+    q += (a * a + b * b) + (c * c + d * d);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
+  const float rstd = rsqrtf(q * (1.0f / h) + 1e-6f);
+  uint2* ur = reinterpret_cast<uint2*>(u + (long long)row * ldu);
+  const float4* sh4 = reinterpret_cast<const float4*>(shift);
+  const float4* sc4 = reinterpret_cast<const float4*>(scale);
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const int c = i * 32 + lane;
+    float4 sh = __ldg(sh4 + c), sc = __ldg(sc4 + c);
+    float a = (v[i].x - mean) * rstd * (1.f + sc.x) + sh.x;
+    float b = (v[i].y - mean) * rstd * (1.f + sc.y) + sh.y;
+    float cc = (v[i].z - mean) * rstd * (1.f + sc.z) + sh.z;
+    float d = (v[i].w - mean) * rstd * (1.f + sc.w) + sh.w;
+    ur[c] = make_uint2(pack_bf16x2(a, b), pack_bf16x2(cc, d));
+  }
+}
+
+// generic fallback (h multiple of 128): two passes over global memory
+__global__ void __launch_bounds__(256) ln_mod_generic(const float* __restrict__ x, long long ldx, bf16* __restrict__ u,
+                                                      long long ldu, const float* __restrict__ shift,
+                                                      const float* __restrict__ scale, int M, int h) {
+  const int row = blockIdx.x * 8 + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (row >= M) return;
+  const float* xr = x + (long long)row * ldx;
+  float s = 0.f;
+  for (int c = lane; c < h; c += 32) s += xr[c];
+  for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  const float mean = s / h;
+  float q = 0.f;
+  for (int c = lane; c < h; c += 32) { float a = xr[c] - mean; q += a * a; }
+  for (int o = 16; o; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
+  const float rstd = rsqrtf(q / h + 1e-6f);
+  for (int c = lane; c < h; c += 32)
+    u[(long long)row * ldu + c] = __float2bfloat16_rn((xr[c] - mean) * rstd * (1.f + scale[c]) + shift[c]);
+}
+
+void ln_mod_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift, const float* scale,
+                   int M, int h, cudaStream_t s) {
+  if (M <= 0) return;
+  dim3 grid((M + 7) / 8);
+  switch (h) {
+    case 3072: ln_mod_kernel<24><<<grid, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
+    case 1536: ln_mod_kernel<12><<<grid, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
+    case 256: ln_mod_kernel<2><<<grid, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
+    default: ln_mod_generic<<<grid, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M, h); break;
+  }
+}
+
+// ------------------------------------------------------------------ a4: QK-RMSNorm + RoPE (+ Ulysses pack)
+// One warp per (row, head).  Lane l holds D/32 consecutive elements (pairs 2 per 4 elements).
+template <int D>
+__global__ void __launch_bounds__(256) qk_norm_rope_kernel(bf16* __restrict__ qkv, long long ld, int rows, int n_first,
+                                                           int H, const bf16* __restrict__ gq0,
+                                                           const bf16* __restrict__ gk0, const bf16* __restrict__ gq1,
+                                                           const bf16* __restrict__ gk1, const float* __restrict__ cosb,
+                                                           const float* __restrict__ sinb, bf16* __restrict__ pack,
+                                                           int k_sp) {
+  constexpr int E = D / 32;  // elements per lane (4 for D=128, 2 for D=64)
+  const long long gw = (long long)blockIdx.x * 8 + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (gw >= (long long)rows * H) return;
+  const int row = (int)(gw / H), head = (int)(gw % H);
+  const bool first = row < n_first;
+  const bf16* gq = first ? gq0 : gq1;
+  const bf16* gk = first ? gk0 : gk1;
+  const int hD = H * D;
+  bf16* base = qkv + (long long)row * ld;
+  const float* cr = cosb + (long long)row * (D / 2);
+  const float* sr = sinb + (long long)row * (D / 2);
+  const int d0 = lane * E;
+  float cs[E / 2], sn[E / 2];
+#pragma unroll
+  for (int p = 0; p < E / 2; ++p) {
+    cs[p] = __ldg(cr + d0 / 2 + p);
+    sn[p] = __ldg(sr + d0 / 2 + p);
+  }
+  bf16* dst_base = nullptr;
+  int hk = H / k_sp;
+  if (pack) {
+    const int dst = head / hk, hl = head % hk;
+    dst_base = pack + (((long long)dst * rows + row) * 3) * hk * D + (long long)hl * D;
+  }
+#pragma unroll
+  for (int part = 0; part < 2; ++part) {
+    bf16* src = base + part * hD + head * D + d0;
+    float x[E];
+    if constexpr (E == 4) {
+      uint2 u = *reinterpret_cast<const uint2*>(src);
+      float2 a = unpack_bf16x2(u.x), b = unpack_bf16x2(u.y);
+      x[0] = a.x; x[1] = a.y; x[2] = b.x; x[3] = b.y;
+    } else {
+      uint32_t u = *reinterpret_cast<const uint32_t*>(src);
+      float2 a = unpack_bf16x2(u);
+      x[0] = a.x; x[1] = a.y;
+    }
+    float ss = 0.f;
+#pragma unroll
+    for (int e = 0; e < E; ++e) ss += x[e] * x[e];
+#pragma unroll
+    for (int o = 16; o; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
+    const float r = rsqrtf(ss * (1.0f / D) + 1e-6f);
+    const bf16* g = part == 0 ? gq : gk;
+    float y[E];
+#pragma unroll
+    for (int e = 0; e < E; ++e) y[e] = x[e] * r * __bfloat162float(g[d0 + e]);
+    float z[E];
+#pragma unroll
+    for (int p = 0; p < E / 2; ++p) {
+      z[2 * p] = cs[p] * y[2 * p] - sn[p] * y[2 * p + 1];
+      z[2 * p + 1] = sn[p] * y[2 * p] + cs[p] * y[2 * p + 1];
+    }
+    bf16* dst = pack ? dst_base + part * hk * D + d0 : src;
+    if constexpr (E == 4) {
+      *reinterpret_cast<uint2*>(dst) = make_uint2(pack_bf16x2(z[0], z[1]), pack_bf16x2(z[2], z[3]));
+    } else {
+      *reinterpret_cast<uint32_t*>(dst) = pack_bf16x2(z[0], z[1]);
+    }
+  }
+  if (pack) {  // v: plain copy into the send layout
+    const bf16* src = base + 2 * hD + head * D + d0;
+    bf16* dst = dst_base + 2 * hk * D + d0;
+    if constexpr (E == 4) *reinterpret_cast<uint2*>(dst) = *reinterpret_cast<const uint2*>(src);
+    else *reinterpret_cast<uint32_t*>(dst) = *reinterpret_cast<const uint32_t*>(src);
+  }
+}
+
+void qk_norm_rope_launch(bf16* qkv, long long ld, int rows, int n_first, int H, int D, const bf16* gq0,
+                         const bf16* gk0, const bf16* gq1, const bf16* gk1, const float* cosb, const float* sinb,
+                         bf16* pack_out, int k_sp, cudaStream_t s) {
+  if (rows <= 0) return;
+  const long long warps = (long long)rows * H;
+  dim3 grid((unsigned)((warps + 7) / 8));
+  if (D == 128)
+    qk_norm_rope_kernel<128><<<grid, 256, 0, s>>>(qkv, ld, rows, n_first, H, gq0, gk0, gq1, gk1, cosb, sinb,
+                                                  pack_out, k_sp);
+  else
+    qk_norm_rope_kernel<64><<<grid, 256, 0, s>>>(qkv, ld, rows, n_first, H, gq0, gk0, gq1, gk1, cosb, sinb,
+                                                 pack_out, k_sp);
+}
+
+// ------------------------------------------------------------------ small conversions
+__global__ void f32_to_bf16_kernel(const float* __restrict__ src, long long lds, bf16* __restrict__ dst,
+                                   long long ldd, int M, int C, int act) {
+  long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  long long n = (long long)M * C;
+  for (; i < n; i += (long long)gridDim.x * blockDim.x) {
+    int m = (int)(i / C), c = (int)(i % C);
+    float v = src[(long long)m * lds + c];
+    if (act == 1) v = silu(v);
+    dst[(long long)m * ldd + c] = __float2bfloat16_rn(v);
+  }
+}
+void f32_to_bf16_launch(const float* src, long long lds, bf16* dst, long long ldd, int M, int C, cudaStream_t s) {
+  if (M <= 0 || C <= 0) return;
+  long long n = (long long)M * C;
+  int blocks = (int)((n + 255) / 256);
+  if (blocks > 4096) blocks = 4096;
+  f32_to_bf16_kernel<<<blocks, 256, 0, s>>>(src, lds, dst, ldd, M, C, 0);
+}
+void silu_bf16_launch(const float* src, long long lds, bf16* dst, long long ldd, int M, int C, cudaStream_t s) {
+  if (M <= 0 || C <= 0) return;
+  long long n = (long long)M * C;
+  int blocks = (int)((n + 255) / 256);
+  if (blocks > 4096) blocks = 4096;
+  f32_to_bf16_kernel<<<blocks, 256, 0, s>>>(src, lds, dst, ldd, M, C, 1);
+}
+
+// rows x cols bf16, cols multiple of 8, strides multiple of 8 elements
+__global__ void copy2d_bf16_kernel(const uint4* __restrict__ src, long long lds8, uint4* __restrict__ dst,
+                                   long long ldd8, int rows, int cols8) {
+  long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  long long n = (long long)rows * cols8;
+  for (; i < n; i += (long long)gridDim.x * blockDim.x) {
+    int r = (int)(i / cols8), c = (int)(i % cols8);
+    dst[r * ldd8 + c] = src[r * lds8 + c];
+  }
+}
+void copy2d_bf16_launch(const bf16* src, long long lds, bf16* dst, long long ldd, int rows, int cols, cudaStream_t s) {
+  if (rows <= 0 || cols <= 0) return;
+  long long n = (long long)rows * (cols / 8);
+  int blocks = (int)((n + 255) / 256);
+  if (blocks > 8192) blocks = 8192;
+  copy2d_bf16_kernel<<<blocks, 256, 0, s>>>(reinterpret_cast<const uint4*>(src), lds / 8,
+                                            reinterpret_cast<uint4*>(dst), ldd / 8, rows, cols / 8);
+}
+
+__global__ void select_row_kernel(const float* __restrict__ src, long long stride, const int* __restrict__ idx,
+                                  float* __restrict__ dst, long long n) {
+  const float* s = src + (long long)(*idx) * stride;
+  long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long n4 = n / 4;
+  for (; i < n4; i += (long long)gridDim.x * blockDim.x)
+    reinterpret_cast<float4*>(dst)[i] = reinterpret_cast<const float4*>(s)[i];
+  if (blockIdx.x == 0 && threadIdx.x < (n & 3)) dst[n4 * 4 + threadIdx.x] = s[n4 * 4 + threadIdx.x];
+}
+void select_row_launch(const float* src, long long stride, const int* idx_dev, float* dst, long long n,
+                       cudaStream_t s) {
+  if (n <= 0) return;
+  int blocks = (int)((n / 4 + 255) / 256);
+  if (blocks < 1) blocks = 1;
+  if (blocks > 2048) blocks = 2048;
+  select_row_kernel<<<blocks, 256, 0, s>>>(src, stride, idx_dev, dst, n);
+}
+
+// ------------------------------------------------------------------ SYNTH-1 (see include/tsv.h)
+__device__ __forceinline__ uint64_t splitmix64_mix(uint64_t z) {
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+__global__ void synth_kernel(void* dst, uint64_t seed, uint32_t tid, uint64_t idx0, long long n, int kind, float c) {
+  const uint64_t key = seed ^ ((uint64_t)tid << 48);
+  long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  for (; i < n; i += (long long)gridDim.x * blockDim.x) {
+    const uint64_t h = splitmix64_mix(((idx0 + (uint64_t)i) ^ key) + 0x9E3779B97F4A7C15ull);
+    const int u = (int)(h >> 40);
+    const float r = (float)(u - (1 << 23)) * 1.1920928955078125e-07f;  // exact: 24-bit int * 2^-23
+    float v = __fmul_rn(r, c);
+    if (kind == 2) {
+      reinterpret_cast<float*>(dst)[i] = v;
+    } else {
+      if (kind == 1) v = __fadd_rn(1.0f, v);
+      reinterpret_cast<bf16*>(dst)[i] = __float2bfloat16_rn(v);
+    }
+  }
+}
+void synth_launch(void* dst, uint64_t seed, uint32_t tensor_id, uint64_t idx0, long long n, int kind, float c,
+                  cudaStream_t s) {
+  if (n <= 0) return;
+  long long blocks = (n + 255) / 256;
+  if (blocks > 148 * 64) blocks = 148 * 64;
+  synth_kernel<<<(unsigned)blocks, 256, 0, s>>>(dst, seed, tensor_id, idx0, n, kind, c);
+}
+
+}  // namespace tsv

@@ -1,0 +1,1435 @@
+// libtsv.so engine: weights, GPU groups, requests, the denoising step under Ulysses SP, reshard,
+// events and the step-latency table.  Implements include/tsv.h.
+//
+// Step (S:§8(a), per rank r of a group of k; rows of rank r = [txt_r ; img_r]):
+//   a1 embed      img = x_s W_img^T + b (latent cast to bf16), txt = T W_txt^T + b    -> x fp32
+//   double j      per stream: a2 LN-mod -> a3 QKV GEMM -> a4 QK-RMSNorm+RoPE(+pack) ->
+//                 a5 a2a #1 -> a6 attention -> a7 a2a #2 -> (unpack) -> a8 proj + gated residual
+//                 -> a9 LN-mod -> fc1+GELU -> fc2 + gated residual
+//   single j      a2 LN-mod -> linear1 (qkv | GELU(mlp)) -> a4 -> a5 -> a6 -> a7 -> linear2 + gated residual
+//   final         a2 LN-mod(img rows) -> a11 linear -> a12 Euler x += dt v (GEMM epilogue)
+// Conditioning (a0) runs once per (request, GPU): vec_s for all steps, then the modulation table
+// mod[s] = W_mod SiLU(vec_s) + b as one [S, n_mod] GEMM.
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include "../../include/tsv.h"
+#include "../../include/tsv_ops.h"
+#include "kernels.h"
+#include "model.h"
+
+namespace tsv {
+
+// ------------------------------------------------------------------ errors
+static thread_local std::string g_err;
+static tsv_status fail(tsv_status s, const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return s;
+}
+#define CK(call)                                                                                  \
+  do {                                                                                            \
+    cudaError_t e_ = (call);                                                                      \
+    if (e_ != cudaSuccess)                                                                        \
+      return fail(e_ == cudaErrorMemoryAllocation ? TSV_E_OOM : TSV_E_CUDA, "%s:%d %s: %s", __FILE__, \
+                  __LINE__, #call, cudaGetErrorString(e_));                                       \
+  } while (0)
+#define NK(call)                                                                                   \
+  do {                                                                                             \
+    ncclResult_t r_ = (call);                                                                      \
+    if (r_ != ncclSuccess)                                                                         \
+      return fail(TSV_E_NCCL, "%s:%d %s: %s", __FILE__, __LINE__, #call, ncclGetErrorString(r_)); \
+  } while (0)
+#define TRY(expr)                 \
+  do {                            \
+    tsv_status s_ = (expr);       \
+    if (s_ != TSV_OK) return s_;  \
+  } while (0)
+
+static int64_t shard_begin(int64_t n, int k, int r) { return (int64_t)r * (n / k) + std::min<int64_t>(r, n % k); }
+
+// ------------------------------------------------------------------ SYNTH-1 on the host (request inputs)
+static inline uint64_t sm64_mix(uint64_t z) {
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+static inline float synth_r(uint64_t seed, uint32_t tid, uint64_t idx) {
+  const uint64_t h = sm64_mix((idx ^ (seed ^ ((uint64_t)tid << 48))) + 0x9E3779B97F4A7C15ull);
+  return (float)((int)(h >> 40) - (1 << 23)) * (1.0f / 8388608.0f);
+}
+static inline uint16_t f32_to_bf16_bits(float f) {
+  uint32_t b;
+  memcpy(&b, &f, 4);
+  b = (b + 0x7FFFu + ((b >> 16) & 1u)) >> 16;
+  return (uint16_t)b;
+}
+static inline float bf16_bits_to_f32(uint16_t u) {
+  uint32_t b = (uint32_t)u << 16;
+  float f;
+  memcpy(&f, &b, 4);
+  return f;
+}
+
+// ------------------------------------------------------------------ device buffers
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  int device = -1;
+  void release() {
+    if (p) {
+      int cur;
+      cudaGetDevice(&cur);
+      cudaSetDevice(device);
+      cudaFree(p);
+      cudaSetDevice(cur);
+    }
+    p = nullptr;
+    bytes = 0;
+  }
+};
+static tsv_status dev_alloc(DevBuf& b, int device, size_t bytes) {
+  if (b.p && b.bytes >= bytes && b.device == device) return TSV_OK;
+  b.release();
+  if (bytes == 0) return TSV_OK;
+  CK(cudaSetDevice(device));
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, bytes);
+  if (e != cudaSuccess) return fail(TSV_E_OOM, "cudaMalloc(%zu) on device %d: %s", bytes, device, cudaGetErrorString(e));
+  b.p = p;
+  b.bytes = bytes;
+  b.device = device;
+  return TSV_OK;
+}
+
+struct DeviceState {
+  int device = -1;
+  int num_sms = 148;
+  DevBuf weights;  // bf16 blob
+};
+
+struct Workspace {
+  DevBuf x, u, qkv, cat, hbuf, latb, pack, recv, obuf, orecv;
+};
+
+struct Slot {
+  int rank = -1;
+  int device = -1;
+  DeviceState* ds = nullptr;
+  cudaStream_t stream = nullptr;
+  Workspace ws;
+  DevBuf scratch;  // conditioning temporaries
+};
+
+// per (request, slot): state that depends only on the request
+struct ReqDev {
+  DevBuf mod;       // fp32 [S, n_mod]
+  DevBuf dt;        // fp32 [S]
+  bool ready = false;
+};
+// per (request, slot, shard): state that depends on the group position
+struct ReqShard {
+  int rank_in_group = 0, k = 1;
+  int64_t t0 = 0, nt = 0, i0 = 0, ni = 0;  // txt rows [t0, t0+nt), img rows [i0, i0+ni)
+  DevBuf lat, vel, T, cosb, sinb;
+};
+
+struct Group {
+  std::vector<int> ranks;  // global ranks, position = group rank
+  int k = 1;
+  bool all_local = true;
+  std::vector<int> local_slots;      // slot index per local member (same order as ranks filtered)
+  std::vector<int> local_positions;  // group rank of each local member
+  ncclComm_t comm = nullptr;         // multi-process transport (one local rank)
+  std::vector<cudaEvent_t> ev_a, ev_b;  // per local member, for in-process all-to-all ordering
+};
+
+struct Request {
+  int height = 0, width = 0, S = 0;
+  uint64_t seed = 0;
+  float guidance = 3.5f;
+  int64_t Li = 0, Lt = 0;
+  int next_step = 0;
+  int group = -1;
+  std::vector<float> x_host;      // [Li, in] until the first landing
+  std::vector<uint16_t> T_host;   // [Lt, ctx] bf16 bits
+  std::vector<uint16_t> y_host;   // [vec] bf16 bits
+  std::vector<double> ts;         // t_0..t_S
+  std::map<int, ReqDev> dev;      // by slot
+  std::map<int, ReqShard> shard;  // by slot (current group)
+  std::map<int, cudaEvent_t> last;  // by slot: completion of the last submitted work
+  bool has_velocity = false;
+};
+
+struct EventRec {
+  std::vector<std::pair<int, cudaEvent_t>> evs;  // (slot, event)
+};
+
+}  // namespace tsv
+
+using namespace tsv;
+
+struct tsv_engine {
+  Model model;
+  uint64_t weight_seed = 0;
+  int rank_base = 0, n_local = 0, world = 0;
+  std::vector<Slot> slots;
+  std::map<int, std::unique_ptr<DeviceState>> devs;
+  std::vector<Group> groups;
+  std::map<int64_t, Request> requests;
+  int64_t next_req = 1;
+  std::vector<EventRec> events;
+  ncclComm_t world_comm = nullptr;
+  int64_t kernel_count = 0;
+  // per-kernel-class profiling (tsv_engine_profile)
+  bool prof = false;
+  struct ProfRec { int cls; int device; cudaEvent_t a, b; };
+  std::vector<ProfRec> prof_recs;
+  std::map<int, std::vector<cudaEvent_t>> ev_pool;  // by device
+  double prof_flops[8] = {0}, prof_bytes[8] = {0};
+  int64_t prof_launch[8] = {0};
+
+  int slot_of_rank(int rank) const {
+    int i = rank - rank_base;
+    return (i >= 0 && i < n_local) ? i : -1;
+  }
+  const bf16* W(const Slot& s, int id) const {
+    return reinterpret_cast<const bf16*>(s.ds->weights.p) + model.find(id)->offset;
+  }
+};
+
+namespace tsv {
+
+// ------------------------------------------------------------------ launch helpers (count + profile kernels)
+enum KClass { KC_GEMM = 0, KC_ATTN = 1, KC_LNMOD = 2, KC_QKROPE = 3, KC_A2A = 4, KC_OTHER = 5, KC_N = 6 };
+
+static cudaEvent_t pool_event(tsv_engine* e, int device) {
+  auto& v = e->ev_pool[device];
+  if (!v.empty()) { cudaEvent_t ev = v.back(); v.pop_back(); return ev; }
+  cudaEvent_t ev = nullptr;
+  cudaEventCreate(&ev);
+  return ev;
+}
+
+// Counts one launch of class `cls` (kernels = number of CUDA kernels it launches) and, when
+// profiling is on, brackets it with CUDA events on the launching stream.
+struct ProfScope {
+  tsv_engine* e;
+  Slot* s;
+  int cls;
+  cudaEvent_t a = nullptr;
+  ProfScope(tsv_engine* e_, Slot& s_, int cls_, double flops, double bytes, int kernels = 1)
+      : e(e_), s(&s_), cls(cls_) {
+    e->kernel_count += kernels;
+    if (!e->prof) return;
+    e->prof_flops[cls] += flops;
+    e->prof_bytes[cls] += bytes;
+    e->prof_launch[cls] += 1;
+    a = pool_event(e, s->device);
+    cudaEventRecord(a, s->stream);
+  }
+  ~ProfScope() {
+    if (!a) return;
+    cudaEvent_t b = pool_event(e, s->device);
+    cudaEventRecord(b, s->stream);
+    e->prof_recs.push_back({cls, s->device, a, b});
+  }
+};
+
+static tsv_status gemm(tsv_engine* e, Slot& s, const bf16* A, long long lda, const bf16* Wt, long long ldw, int M,
+                       int N, int K, const GemmEpi& epi) {
+  if (M <= 0) return TSV_OK;
+  GemmPlan p;
+  const char* err = nullptr;
+  if (gemm_plan(&p, A, lda, Wt, ldw, M, N, K, epi, s.ds->num_sms, &err))
+    return fail(TSV_E_INVAL, "%s (M=%d N=%d K=%d)", err, M, N, K);
+  const double out_b = (epi.mode <= EPI_SPLIT_GELU) ? 2.0 : (epi.mode == EPI_STORE_F32 ? 4.0 : 8.0);
+  ProfScope ps(e, s, KC_GEMM, 2.0 * M * N * (double)K,
+               2.0 * ((double)M * K + (double)N * K) + out_b * (double)M * N);
+  gemm_launch(p, s.stream);
+  return TSV_OK;
+}
+static void lnmod(tsv_engine* e, Slot& s, const float* x, bf16* u, const float* shift, const float* scale, int n) {
+  const int h = e->model.h;
+  ProfScope ps(e, s, KC_LNMOD, 0.0, (double)n * h * 6.0 + 8.0 * h);
+  ln_mod_launch(x, h, u, h, shift, scale, n, h, s.stream);
+}
+
+static GemmEpi epi_of(int mode, void* out0, long long ld0, const bf16* bias, const float* gate = nullptr,
+                      void* out1 = nullptr, long long ld1 = 0, int n_split = 0, const float* scalar = nullptr) {
+  GemmEpi g;
+  g.mode = mode; g.out0 = out0; g.ld0 = ld0; g.bias = bias; g.gate = gate; g.out1 = out1; g.ld1 = ld1;
+  g.n_split = n_split; g.scalar = scalar;
+  return g;
+}
+
+// ------------------------------------------------------------------ weights
+static tsv_status init_weights(tsv_engine* e, DeviceState& ds) {
+  const Model& m = e->model;
+  TRY(dev_alloc(ds.weights, ds.device, m.total * 2));
+  CK(cudaSetDevice(ds.device));
+  CK(cudaMemset(ds.weights.p, 0, m.total * 2));
+  for (const auto& t : m.tensors) {
+    synth_launch(reinterpret_cast<bf16*>(ds.weights.p) + t.offset, e->weight_seed, (uint32_t)t.id, 0, t.numel(),
+                 t.kind, t.c, nullptr);
+    e->kernel_count++;  // init-time (not a step kernel)
+  }
+  CK(cudaGetLastError());
+  CK(cudaDeviceSynchronize());
+  return TSV_OK;
+}
+
+// ------------------------------------------------------------------ per-request state on a slot
+static tsv_status ensure_reqdev(tsv_engine* e, Request& R, int si) {
+  ReqDev& rd = R.dev[si];
+  if (rd.ready) return TSV_OK;
+  Slot& s = e->slots[si];
+  const Model& m = e->model;
+  const int h = m.h, S = R.S;
+  CK(cudaSetDevice(s.device));
+  TRY(dev_alloc(rd.mod, s.device, (size_t)S * m.n_mod * 4));
+  TRY(dev_alloc(rd.dt, s.device, (size_t)S * 4));
+  // host-side: sinusoidal embeddings e(t_s), e(g) (fp64 -> bf16), y (bf16), dt
+  const int Sp = S;
+  std::vector<uint16_t> et((size_t)Sp * 256), eg((size_t)Sp * 256), ey((size_t)Sp * m.vec);
+  auto emb = [](double t, uint16_t* out) {
+    for (int j = 0; j < 128; ++j) {
+      double f = std::exp(-std::log(10000.0) * j / 128.0);
+      double a = 1000.0 * t * f;
+      out[j] = f32_to_bf16_bits((float)std::cos(a));
+      out[128 + j] = f32_to_bf16_bits((float)std::sin(a));
+    }
+  };
+  std::vector<float> dt(S);
+  for (int i = 0; i < S; ++i) {
+    emb(R.ts[i], &et[(size_t)i * 256]);
+    emb((double)R.guidance, &eg[(size_t)i * 256]);
+    memcpy(&ey[(size_t)i * m.vec], R.y_host.data(), m.vec * 2);
+    dt[i] = (float)(R.ts[i + 1] - R.ts[i]);
+  }
+  // scratch: et, eg, ey (bf16 [S,256],[S,256],[S,vec]); hid bf16 [S,h]; vec f32 [S,h]; asilu bf16 [S,h]
+  const size_t o_et = 0, o_eg = o_et + (size_t)S * 256 * 2, o_ey = o_eg + (size_t)S * 256 * 2;
+  const size_t o_hid = (o_ey + (size_t)S * m.vec * 2 + 255) & ~size_t(255);
+  const size_t o_vec = (o_hid + (size_t)S * h * 2 + 255) & ~size_t(255);
+  const size_t o_as = (o_vec + (size_t)S * h * 4 + 255) & ~size_t(255);
+  const size_t total = o_as + (size_t)S * h * 2;
+  TRY(dev_alloc(s.scratch, s.device, total));
+  uint8_t* sc = reinterpret_cast<uint8_t*>(s.scratch.p);
+  CK(cudaMemcpyAsync(sc + o_et, et.data(), et.size() * 2, cudaMemcpyHostToDevice, s.stream));
+  CK(cudaMemcpyAsync(sc + o_eg, eg.data(), eg.size() * 2, cudaMemcpyHostToDevice, s.stream));
+  CK(cudaMemcpyAsync(sc + o_ey, ey.data(), ey.size() * 2, cudaMemcpyHostToDevice, s.stream));
+  CK(cudaMemcpyAsync(rd.dt.p, dt.data(), S * 4, cudaMemcpyHostToDevice, s.stream));
+  bf16* hid = reinterpret_cast<bf16*>(sc + o_hid);
+  float* vec = reinterpret_cast<float*>(sc + o_vec);
+  bf16* as = reinterpret_cast<bf16*>(sc + o_as);
+  // vec = MLP_t(e(t)) + MLP_g(e(g)) + MLP_y(y)   (TT:model.py:119-120 + FLUX-dev guidance_in)
+  struct MlpIds { size_t off; int K; int w1, b1, w2, b2; bool on; };
+  MlpIds mlps[3] = {{o_et, 256, 4, 5, 6, 7, true}, {o_eg, 256, 8, 9, 10, 11, m.d.guidance_embed != 0},
+                    {o_ey, m.vec, 12, 13, 14, 15, true}};
+  bool first = true;
+  for (auto& ml : mlps) {
+    if (!ml.on) continue;
+    TRY(gemm(e, s, reinterpret_cast<bf16*>(sc + ml.off), ml.K, e->W(s, ml.w1), ml.K, S, h, ml.K,
+             epi_of(EPI_SILU_BF16, hid, h, e->W(s, ml.b1))));
+    TRY(gemm(e, s, hid, h, e->W(s, ml.w2), h, S, h, h,
+             epi_of(first ? EPI_STORE_F32 : EPI_ACCUM_F32, vec, h, e->W(s, ml.b2))));
+    first = false;
+  }
+  {
+    ProfScope ps(e, s, KC_OTHER, 0.0, (double)S * h * 6.0);
+    silu_bf16_launch(vec, h, as, h, S, h, s.stream);
+  }
+  // modulation table for all steps: [S, n_mod] = SiLU(vec) W_mod^T + b   (TT:layers.py:142)
+  const bf16* wb = reinterpret_cast<const bf16*>(s.ds->weights.p);
+  TRY(gemm(e, s, as, h, wb + m.modw_off, h, S, (int)m.n_mod, h,
+           epi_of(EPI_STORE_F32, rd.mod.p, m.n_mod, wb + m.modb_off)));
+  CK(cudaGetLastError());
+  rd.ready = true;
+  return TSV_OK;
+}
+
+// RoPE tables for the rows of one shard (fp64 angles -> fp32 cos/sin, S22)
+static void rope_rows(const Model& m, const Request& R, int64_t t0, int64_t nt, int64_t i0, int64_t ni,
+                      std::vector<float>& c, std::vector<float>& s) {
+  const int half = m.D / 2;
+  c.assign((size_t)(nt + ni) * half, 1.0f);
+  s.assign((size_t)(nt + ni) * half, 0.0f);
+  const int64_t wp = R.width / 16;
+  for (int64_t r = 0; r < ni; ++r) {
+    const int64_t p = i0 + r;
+    const double ids[3] = {0.0, (double)(p / wp), (double)(p % wp)};
+    int pair = 0;
+    for (int a = 0; a < 3; ++a) {
+      const int da = m.d.axes_dim[a];
+      for (int j = 0; j < da / 2; ++j, ++pair) {
+        const double omega = 1.0 / std::pow((double)m.d.theta, (2.0 * j) / da);
+        const double ang = ids[a] * omega;
+        c[(size_t)(nt + r) * half + pair] = (float)std::cos(ang);
+        s[(size_t)(nt + r) * half + pair] = (float)std::sin(ang);
+      }
+    }
+  }
+}
+
+static tsv_status setup_shard(tsv_engine* e, Request& R, int si, int rank_in_group, int k, ReqShard& sh) {
+  Slot& s = e->slots[si];
+  const Model& m = e->model;
+  sh.rank_in_group = rank_in_group;
+  sh.k = k;
+  sh.t0 = shard_begin(R.Lt, k, rank_in_group);
+  sh.nt = shard_begin(R.Lt, k, rank_in_group + 1) - sh.t0;
+  sh.i0 = shard_begin(R.Li, k, rank_in_group);
+  sh.ni = shard_begin(R.Li, k, rank_in_group + 1) - sh.i0;
+  CK(cudaSetDevice(s.device));
+  TRY(dev_alloc(sh.lat, s.device, std::max<size_t>(1, sh.ni) * m.in * 4));
+  TRY(dev_alloc(sh.vel, s.device, std::max<size_t>(1, sh.ni) * m.in * 4));
+  TRY(dev_alloc(sh.T, s.device, std::max<size_t>(1, sh.nt) * m.ctx * 2));
+  const size_t rows = sh.nt + sh.ni;
+  TRY(dev_alloc(sh.cosb, s.device, std::max<size_t>(1, rows) * (m.D / 2) * 4));
+  TRY(dev_alloc(sh.sinb, s.device, std::max<size_t>(1, rows) * (m.D / 2) * 4));
+  if (sh.nt)
+    CK(cudaMemcpyAsync(sh.T.p, R.T_host.data() + sh.t0 * m.ctx, sh.nt * m.ctx * 2, cudaMemcpyHostToDevice, s.stream));
+  std::vector<float> c, sn;
+  rope_rows(m, R, sh.t0, sh.nt, sh.i0, sh.ni, c, sn);
+  if (rows) {
+    CK(cudaMemcpyAsync(sh.cosb.p, c.data(), c.size() * 4, cudaMemcpyHostToDevice, s.stream));
+    CK(cudaMemcpyAsync(sh.sinb.p, sn.data(), sn.size() * 4, cudaMemcpyHostToDevice, s.stream));
+    CK(cudaStreamSynchronize(s.stream));  // host vectors go out of scope
+  }
+  return TSV_OK;
+}
+
+static tsv_status ensure_workspace(tsv_engine* e, Slot& s, int64_t rows, int64_t L, int k) {
+  const Model& m = e->model;
+  const int64_t h = m.h, F = m.F;
+  Workspace& w = s.ws;
+  const int64_t r = std::max<int64_t>(rows, 1);
+  TRY(dev_alloc(w.x, s.device, r * h * 4));
+  TRY(dev_alloc(w.u, s.device, r * h * 2));
+  TRY(dev_alloc(w.qkv, s.device, r * 3 * h * 2));
+  TRY(dev_alloc(w.cat, s.device, r * (h + F) * 2));
+  TRY(dev_alloc(w.hbuf, s.device, r * F * 2));
+  TRY(dev_alloc(w.latb, s.device, r * m.in * 2));
+  if (k > 1) {
+    TRY(dev_alloc(w.pack, s.device, r * 3 * h * 2));
+    TRY(dev_alloc(w.recv, s.device, L * 3 * (h / k) * 2));
+    TRY(dev_alloc(w.obuf, s.device, L * (h / k) * 2));
+    TRY(dev_alloc(w.orecv, s.device, r * h * 2));
+  }
+  return TSV_OK;
+}
+
+// ------------------------------------------------------------------ the step
+struct RankCtx {
+  int si;                 // slot index
+  Slot* s;
+  ReqShard* sh;
+  ReqDev* rd;
+  int64_t nt, ni, rows;   // local rows: [txt (nt) ; img (ni)]
+  float* x;
+  bf16 *u, *qkv, *cat, *hbuf, *latb, *pack, *recv, *obuf, *orecv;
+  const float* mod;       // this step's modulation row
+};
+
+struct StepEnv {
+  tsv_engine* e;
+  Request* R;
+  Group* g;
+  int step;
+  std::vector<RankCtx> rc;
+  // global layout for the all-to-alls
+  std::vector<int64_t> t_off, t_cnt, i_off, i_cnt;  // per group rank
+};
+
+// in-process all-to-all #1: pack_r[d] ([rows_r][3h/k]) -> recv_d rows (global order)
+static tsv_status a2a_qkv(StepEnv& E) {
+  tsv_engine* e = E.e;
+  const Model& m = e->model;
+  Group& g = *E.g;
+  const int k = g.k;
+  const int64_t w = 3 * (int64_t)m.h / k;  // bf16 per row per destination
+  const int64_t Lt = E.R->Lt;
+  if (g.comm) {
+    RankCtx& c = E.rc[0];
+    const int r = g.local_positions[0];
+    CK(cudaSetDevice(c.s->device));
+    ProfScope ps(e, *c.s, KC_A2A, 0.0, 2.0 * c.rows * 3 * m.h * (k - 1) / k);
+    NK(ncclGroupStart());
+    for (int p = 0; p < k; ++p) {
+      const bf16* sendp = c.pack + (int64_t)p * c.rows * w;
+      if (E.t_cnt[r]) NK(ncclSend(sendp, E.t_cnt[r] * w, ncclBfloat16, p, g.comm, c.s->stream));
+      if (E.i_cnt[r]) NK(ncclSend(sendp + E.t_cnt[r] * w, E.i_cnt[r] * w, ncclBfloat16, p, g.comm, c.s->stream));
+      if (E.t_cnt[p]) NK(ncclRecv(c.recv + E.t_off[p] * w, E.t_cnt[p] * w, ncclBfloat16, p, g.comm, c.s->stream));
+      if (E.i_cnt[p])
+        NK(ncclRecv(c.recv + (Lt + E.i_off[p]) * w, E.i_cnt[p] * w, ncclBfloat16, p, g.comm, c.s->stream));
+    }
+    NK(ncclGroupEnd());
+    return TSV_OK;
+  }
+  // in-process: all k ranks are local (rc indexed by group rank)
+  for (int r = 0; r < k; ++r) CK(cudaEventRecord(g.ev_a[r], E.rc[r].s->stream));
+  for (int d = 0; d < k; ++d) {
+    RankCtx& dst = E.rc[d];
+    ProfScope ps(e, *dst.s, KC_A2A, 0.0, 2.0 * dst.rows * 3 * m.h * (k - 1) / k, 0);
+    for (int r = 0; r < k; ++r) CK(cudaStreamWaitEvent(dst.s->stream, g.ev_a[r], 0));
+    for (int r = 0; r < k; ++r) {
+      RankCtx& src = E.rc[r];
+      const bf16* sp = src.pack + (int64_t)d * src.rows * w;
+      if (E.t_cnt[r])
+        CK(cudaMemcpyPeerAsync(dst.recv + E.t_off[r] * w, dst.s->device, sp, src.s->device, E.t_cnt[r] * w * 2,
+                               dst.s->stream));
+      if (E.i_cnt[r])
+        CK(cudaMemcpyPeerAsync(dst.recv + (Lt + E.i_off[r]) * w, dst.s->device, sp + E.t_cnt[r] * w, src.s->device,
+                               E.i_cnt[r] * w * 2, dst.s->stream));
+    }
+    CK(cudaEventRecord(g.ev_b[d], dst.s->stream));
+  }
+  for (int r = 0; r < k; ++r)
+    for (int d = 0; d < k; ++d) CK(cudaStreamWaitEvent(E.rc[r].s->stream, g.ev_b[d], 0));
+  return TSV_OK;
+}
+
+// all-to-all #2: obuf_d ([L][h/k], global rows) -> orecv_r[d] ([rows_r][h/k]), then unpack into cat[:, d*h/k]
+static tsv_status a2a_o(StepEnv& E) {
+  tsv_engine* e = E.e;
+  const Model& m = e->model;
+  Group& g = *E.g;
+  const int k = g.k;
+  const int64_t w = (int64_t)m.h / k;
+  const int64_t Lt = E.R->Lt;
+  if (g.comm) {
+    RankCtx& c = E.rc[0];
+    const int r = g.local_positions[0];
+    CK(cudaSetDevice(c.s->device));
+    ProfScope ps(e, *c.s, KC_A2A, 0.0, 2.0 * c.rows * m.h * (k - 1) / k);
+    NK(ncclGroupStart());
+    for (int p = 0; p < k; ++p) {
+      if (E.t_cnt[p]) NK(ncclSend(c.obuf + E.t_off[p] * w, E.t_cnt[p] * w, ncclBfloat16, p, g.comm, c.s->stream));
+      if (E.i_cnt[p])
+        NK(ncclSend(c.obuf + (Lt + E.i_off[p]) * w, E.i_cnt[p] * w, ncclBfloat16, p, g.comm, c.s->stream));
+      bf16* rp = c.orecv + (int64_t)p * c.rows * w;
+      if (E.t_cnt[r]) NK(ncclRecv(rp, E.t_cnt[r] * w, ncclBfloat16, p, g.comm, c.s->stream));
+      if (E.i_cnt[r]) NK(ncclRecv(rp + E.t_cnt[r] * w, E.i_cnt[r] * w, ncclBfloat16, p, g.comm, c.s->stream));
+    }
+    NK(ncclGroupEnd());
+  } else {
+    for (int d = 0; d < k; ++d) CK(cudaEventRecord(g.ev_a[d], E.rc[d].s->stream));
+    for (int r = 0; r < k; ++r) {
+      RankCtx& dst = E.rc[r];
+      ProfScope ps(e, *dst.s, KC_A2A, 0.0, 2.0 * dst.rows * m.h * (k - 1) / k, 0);
+      for (int d = 0; d < k; ++d) CK(cudaStreamWaitEvent(dst.s->stream, g.ev_a[d], 0));
+      for (int d = 0; d < k; ++d) {
+        RankCtx& src = E.rc[d];
+        bf16* rp = dst.orecv + (int64_t)d * dst.rows * w;
+        if (E.t_cnt[r])
+          CK(cudaMemcpyPeerAsync(rp, dst.s->device, src.obuf + E.t_off[r] * w, src.s->device, E.t_cnt[r] * w * 2,
+                                 dst.s->stream));
+        if (E.i_cnt[r])
+          CK(cudaMemcpyPeerAsync(rp + E.t_cnt[r] * w, dst.s->device, src.obuf + (Lt + E.i_off[r]) * w, src.s->device,
+                                 E.i_cnt[r] * w * 2, dst.s->stream));
+      }
+      CK(cudaEventRecord(g.ev_b[r], dst.s->stream));
+    }
+    for (int r = 0; r < k; ++r)
+      for (int d = 0; d < k; ++d) CK(cudaStreamWaitEvent(E.rc[r].s->stream, g.ev_b[d], 0));
+  }
+  // unpack: cat[i, d*w + c] = orecv[d][i][c]
+  for (auto& c : E.rc) {
+    CK(cudaSetDevice(c.s->device));
+    for (int d = 0; d < k; ++d) {
+      ProfScope ps(e, *c.s, KC_OTHER, 0.0, 4.0 * c.rows * w);
+      copy2d_bf16_launch(c.orecv + (int64_t)d * c.rows * w, w, c.cat + d * w, m.h + m.F, (int)c.rows, (int)w,
+                         c.s->stream);
+    }
+  }
+  return TSV_OK;
+}
+
+// attention for all local ranks (after a2a #1); output into cat[:, :h] (k = 1) or obuf (k > 1)
+static tsv_status attention_all(StepEnv& E) {
+  tsv_engine* e = E.e;
+  const Model& m = e->model;
+  const int k = E.g->k;
+  const int64_t L = E.R->Lt + E.R->Li;
+  for (auto& c : E.rc) {
+    CK(cudaSetDevice(c.s->device));
+    const double Lq = k == 1 ? (double)c.rows : (double)L;
+    ProfScope ps(e, *c.s, KC_ATTN, 4.0 * Lq * Lq * m.D * (m.H / k), 8.0 * Lq * m.D * (m.H / k));
+    if (k == 1) {
+      attention_launch(c.qkv, 3 * m.h, c.qkv + m.h, 3 * m.h, c.qkv + 2 * m.h, 3 * m.h, c.cat, m.h + m.F, (int)c.rows,
+                       m.H, m.D, c.s->stream);
+    } else {
+      const int64_t w = 3 * (int64_t)m.h / k;
+      attention_launch(c.recv, w, c.recv + m.h / k, w, c.recv + 2 * m.h / k, w, c.obuf, m.h / k, (int)L, m.H / k,
+                       m.D, c.s->stream);
+    }
+  }
+  return TSV_OK;
+}
+
+// QK-RMSNorm + RoPE on the local qkv rows (in place for k = 1, into the send buffer for k > 1)
+static void qk_rope(StepEnv& E, RankCtx& c, const bf16* gq0, const bf16* gk0, const bf16* gq1, const bf16* gk1) {
+  const Model& m = E.e->model;
+  const int k = E.g->k;
+  ProfScope ps(E.e, *c.s, KC_QKROPE, 0.0,
+               (double)c.rows * m.H * m.D * (k > 1 ? 12.0 : 8.0) + (double)c.rows * m.D * 4.0);
+  qk_norm_rope_launch(c.qkv, 3 * m.h, (int)c.rows, (int)c.nt, m.H, m.D, gq0, gk0, gq1, gk1,
+                      reinterpret_cast<const float*>(c.sh->cosb.p), reinterpret_cast<const float*>(c.sh->sinb.p),
+                      k > 1 ? c.pack : nullptr, k, c.s->stream);
+}
+
+static tsv_status run_step(StepEnv& E) {
+  tsv_engine* e = E.e;
+  const Model& m = e->model;
+  const int h = m.h, F = m.F;
+  const int64_t ldc = h + F;
+  // a1: embeddings
+  for (auto& c : E.rc) {
+    Slot& s = *c.s;
+    CK(cudaSetDevice(s.device));
+    if (c.ni) {
+      {
+        ProfScope ps(e, s, KC_OTHER, 0.0, 6.0 * c.ni * m.in);
+        f32_to_bf16_launch(reinterpret_cast<float*>(c.sh->lat.p), m.in, c.latb, m.in, (int)c.ni, m.in, s.stream);
+      }
+      TRY(gemm(e, s, c.latb, m.in, e->W(s, 0), m.in, (int)c.ni, h, m.in,
+               epi_of(EPI_STORE_F32, c.x + c.nt * h, h, e->W(s, 1))));
+    }
+    if (c.nt)
+      TRY(gemm(e, s, reinterpret_cast<bf16*>(c.sh->T.p), m.ctx, e->W(s, 2), m.ctx, (int)c.nt, h, m.ctx,
+               epi_of(EPI_STORE_F32, c.x, h, e->W(s, 3))));
+  }
+  // double-stream blocks
+  for (int j = 0; j < m.d.n_double; ++j) {
+    for (auto& c : E.rc) {
+      Slot& s = *c.s;
+      CK(cudaSetDevice(s.device));
+      for (int st = 0; st < 2; ++st) {  // 0 = img, 1 = txt
+        const int base = double_base(j, st);
+        const int64_t r0 = st == 0 ? c.nt : 0, n = st == 0 ? c.ni : c.nt;
+        if (!n) continue;
+        const float* md = c.mod + m.mod_double(j, st);
+        lnmod(e, s, c.x + r0 * h, c.u + r0 * h, md + 0 * h, md + 1 * h, (int)n);
+        TRY(gemm(e, s, c.u + r0 * h, h, e->W(s, base + 2), h, (int)n, 3 * h, h,
+                 epi_of(EPI_STORE_BF16, c.qkv + r0 * 3 * h, 3 * h, e->W(s, base + 3))));
+      }
+      qk_rope(E, c, e->W(s, double_base(j, 1) + 4), e->W(s, double_base(j, 1) + 5), e->W(s, double_base(j, 0) + 4),
+              e->W(s, double_base(j, 0) + 5));
+    }
+    if (E.g->k > 1) TRY(a2a_qkv(E));
+    TRY(attention_all(E));
+    if (E.g->k > 1) TRY(a2a_o(E));
+    for (auto& c : E.rc) {
+      Slot& s = *c.s;
+      CK(cudaSetDevice(s.device));
+      for (int st = 0; st < 2; ++st) {
+        const int base = double_base(j, st);
+        const int64_t r0 = st == 0 ? c.nt : 0, n = st == 0 ? c.ni : c.nt;
+        if (!n) continue;
+        const float* md = c.mod + m.mod_double(j, st);
+        float* x = c.x + r0 * h;
+        TRY(gemm(e, s, c.cat + r0 * ldc, ldc, e->W(s, base + 6), h, (int)n, h, h,
+                 epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 7), md + 2 * h)));
+        lnmod(e, s, x, c.u + r0 * h, md + 3 * h, md + 4 * h, (int)n);
+        TRY(gemm(e, s, c.u + r0 * h, h, e->W(s, base + 8), h, (int)n, F, h,
+                 epi_of(EPI_GELU_BF16, c.hbuf + r0 * F, F, e->W(s, base + 9))));
+        TRY(gemm(e, s, c.hbuf + r0 * F, F, e->W(s, base + 10), F, (int)n, h, F,
+                 epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 11), md + 5 * h)));
+      }
+    }
+  }
+  // single-stream blocks on x = [txt; img] (zero-copy join, a10)
+  for (int j = 0; j < m.d.n_single; ++j) {
+    const int base = single_base(j);
+    for (auto& c : E.rc) {
+      Slot& s = *c.s;
+      CK(cudaSetDevice(s.device));
+      if (!c.rows) continue;
+      const float* md = c.mod + m.mod_single(j);
+      lnmod(e, s, c.x, c.u, md, md + h, (int)c.rows);
+      TRY(gemm(e, s, c.u, h, e->W(s, base + 2), h, (int)c.rows, 3 * h + F, h,
+               epi_of(EPI_SPLIT_GELU, c.qkv, 3 * h, e->W(s, base + 3), nullptr, c.cat + h, ldc, 3 * h)));
+      qk_rope(E, c, e->W(s, base + 4), e->W(s, base + 5), e->W(s, base + 4), e->W(s, base + 5));
+    }
+    if (E.g->k > 1) TRY(a2a_qkv(E));
+    TRY(attention_all(E));
+    if (E.g->k > 1) TRY(a2a_o(E));
+    for (auto& c : E.rc) {
+      Slot& s = *c.s;
+      CK(cudaSetDevice(s.device));
+      if (!c.rows) continue;
+      const float* md = c.mod + m.mod_single(j);
+      TRY(gemm(e, s, c.cat, ldc, e->W(s, base + 6), ldc, (int)c.rows, h, h + F,
+               epi_of(EPI_RESID_GATE, c.x, h, e->W(s, base + 7), md + 2 * h)));
+    }
+  }
+  // final layer + Euler (a11, a12)
+  for (auto& c : E.rc) {
+    Slot& s = *c.s;
+    CK(cudaSetDevice(s.device));
+    if (!c.ni) continue;
+    const float* md = c.mod + m.mod_final();
+    lnmod(e, s, c.x + c.nt * h, c.u, md, md + h, (int)c.ni);
+    TRY(gemm(e, s, c.u, h, e->W(s, 18), h, (int)c.ni, m.in, h,
+             epi_of(EPI_EULER, c.sh->lat.p, m.in, e->W(s, 19), nullptr, c.sh->vel.p, m.in, 0,
+                    reinterpret_cast<const float*>(c.rd->dt.p) + E.step)));
+  }
+  for (auto& c : E.rc) CK(cudaGetLastError());
+  return TSV_OK;
+}
+
+// ------------------------------------------------------------------ landing / reshard
+static tsv_status record_last(tsv_engine* e, Request& R, int si) {
+  Slot& s = e->slots[si];
+  CK(cudaSetDevice(s.device));
+  auto it = R.last.find(si);
+  if (it == R.last.end()) {
+    cudaEvent_t ev;
+    CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+    it = R.last.emplace(si, ev).first;
+  }
+  CK(cudaEventRecord(it->second, s.stream));
+  return TSV_OK;
+}
+
+// Move the request to group gi.  First landing: latent rows come from the host inputs.
+static tsv_status move_request(tsv_engine* e, Request& R, int gi) {
+  Group& g = e->groups[gi];
+  const Model& m = e->model;
+  std::map<int, ReqShard> next;
+  for (size_t q = 0; q < g.local_slots.size(); ++q) {
+    const int si = g.local_slots[q];
+    TRY(setup_shard(e, R, si, g.local_positions[q], g.k, next[si]));
+    TRY(ensure_reqdev(e, R, si));
+  }
+  if (R.group < 0) {
+    for (auto& kv : next) {
+      Slot& s = e->slots[kv.first];
+      ReqShard& sh = kv.second;
+      CK(cudaSetDevice(s.device));
+      if (sh.ni)
+        CK(cudaMemcpyAsync(sh.lat.p, R.x_host.data() + sh.i0 * m.in, sh.ni * m.in * 4, cudaMemcpyHostToDevice,
+                           s.stream));
+      CK(cudaStreamSynchronize(s.stream));
+    }
+  } else {
+    Group& og = e->groups[R.group];
+    const int ks = og.k, kd = g.k;
+    if (!og.all_local || !g.all_local) {
+      // multi-process: exchange rows over the world communicator
+      if (!e->world_comm) return fail(TSV_E_STATE, "reshard across processes needs tsv_engine_init_world");
+      NK(ncclGroupStart());
+      for (int sr = 0; sr < ks; ++sr) {
+        const int64_t a0 = shard_begin(R.Li, ks, sr), a1 = shard_begin(R.Li, ks, sr + 1);
+        for (int dr = 0; dr < kd; ++dr) {
+          const int64_t b0 = shard_begin(R.Li, kd, dr), b1 = shard_begin(R.Li, kd, dr + 1);
+          const int64_t lo = std::max(a0, b0), hi = std::min(a1, b1);
+          if (hi <= lo) continue;
+          const int src_rank = og.ranks[sr], dst_rank = g.ranks[dr];
+          const int ss = e->slot_of_rank(src_rank), ds = e->slot_of_rank(dst_rank);
+          if (ss >= 0 && ds >= 0) {
+            CK(cudaStreamWaitEvent(e->slots[ds].stream, R.last[ss], 0));
+            CK(cudaMemcpyPeerAsync(reinterpret_cast<float*>(next[ds].lat.p) + (lo - b0) * m.in, e->slots[ds].device,
+                                   reinterpret_cast<float*>(R.shard[ss].lat.p) + (lo - a0) * m.in,
+                                   e->slots[ss].device, (hi - lo) * m.in * 4, e->slots[ds].stream));
+          } else if (ss >= 0) {
+            NK(ncclSend(reinterpret_cast<float*>(R.shard[ss].lat.p) + (lo - a0) * m.in, (hi - lo) * m.in, ncclFloat32,
+                        dst_rank, e->world_comm, e->slots[ss].stream));
+          } else if (ds >= 0) {
+            NK(ncclRecv(reinterpret_cast<float*>(next[ds].lat.p) + (lo - b0) * m.in, (hi - lo) * m.in, ncclFloat32,
+                        src_rank, e->world_comm, e->slots[ds].stream));
+          }
+        }
+      }
+      NK(ncclGroupEnd());
+    } else {
+      for (int sr = 0; sr < ks; ++sr) {
+        const int64_t a0 = shard_begin(R.Li, ks, sr), a1 = shard_begin(R.Li, ks, sr + 1);
+        const int ss = e->slot_of_rank(og.ranks[sr]);
+        for (int dr = 0; dr < kd; ++dr) {
+          const int64_t b0 = shard_begin(R.Li, kd, dr), b1 = shard_begin(R.Li, kd, dr + 1);
+          const int64_t lo = std::max(a0, b0), hi = std::min(a1, b1);
+          if (hi <= lo) continue;
+          const int ds = e->slot_of_rank(g.ranks[dr]);
+          Slot& dslot = e->slots[ds];
+          CK(cudaSetDevice(dslot.device));
+          CK(cudaStreamWaitEvent(dslot.stream, R.last[ss], 0));
+          CK(cudaMemcpyPeerAsync(reinterpret_cast<float*>(next[ds].lat.p) + (lo - b0) * m.in, dslot.device,
+                                 reinterpret_cast<float*>(R.shard[ss].lat.p) + (lo - a0) * m.in, e->slots[ss].device,
+                                 (hi - lo) * m.in * 4, dslot.stream));
+        }
+      }
+    }
+    // old buffers: wait until every copy finished before freeing
+    for (auto& kv : next) TRY(record_last(e, R, kv.first));
+    for (auto& kv : next) CK(cudaEventSynchronize(R.last[kv.first]));
+    for (auto& kv : R.shard) {
+      kv.second.lat.release(); kv.second.vel.release(); kv.second.T.release();
+      kv.second.cosb.release(); kv.second.sinb.release();
+    }
+  }
+  R.shard.swap(next);
+  R.group = gi;
+  R.has_velocity = false;
+  for (auto& kv : R.shard) TRY(record_last(e, R, kv.first));
+  return TSV_OK;
+}
+
+static tsv_status new_event(tsv_engine* e, const std::vector<int>& slots_, tsv_event* out) {
+  EventRec rec;
+  for (int si : slots_) {
+    Slot& s = e->slots[si];
+    CK(cudaSetDevice(s.device));
+    cudaEvent_t ev;
+    CK(cudaEventCreate(&ev));
+    CK(cudaEventRecord(ev, s.stream));
+    rec.evs.push_back({si, ev});
+  }
+  e->events.push_back(std::move(rec));
+  if (out) *out = (tsv_event)e->events.size() - 1;
+  return TSV_OK;
+}
+
+static tsv_status do_step(tsv_engine* e, Request& R, int step, int gi, tsv_event* done) {
+  Group& g = e->groups[gi];
+  if (g.local_slots.empty()) {
+    if (done) *done = -1;
+    R.next_step = step + 1;
+    return TSV_OK;
+  }
+  if (R.group != gi) TRY(move_request(e, R, gi));
+  const Model& m = e->model;
+  StepEnv E;
+  E.e = e; E.R = &R; E.g = &g; E.step = step;
+  const int k = g.k;
+  E.t_off.resize(k); E.t_cnt.resize(k); E.i_off.resize(k); E.i_cnt.resize(k);
+  for (int r = 0; r < k; ++r) {
+    E.t_off[r] = shard_begin(R.Lt, k, r);
+    E.t_cnt[r] = shard_begin(R.Lt, k, r + 1) - E.t_off[r];
+    E.i_off[r] = shard_begin(R.Li, k, r);
+    E.i_cnt[r] = shard_begin(R.Li, k, r + 1) - E.i_off[r];
+  }
+  const int64_t L = R.Lt + R.Li;
+  for (size_t q = 0; q < g.local_slots.size(); ++q) {
+    const int si = g.local_slots[q];
+    Slot& s = e->slots[si];
+    ReqShard& sh = R.shard[si];
+    TRY(ensure_workspace(e, s, sh.nt + sh.ni, L, k));
+    RankCtx c;
+    c.si = si; c.s = &s; c.sh = &sh; c.rd = &R.dev[si];
+    c.nt = sh.nt; c.ni = sh.ni; c.rows = sh.nt + sh.ni;
+    c.x = reinterpret_cast<float*>(s.ws.x.p);
+    c.u = reinterpret_cast<bf16*>(s.ws.u.p);
+    c.qkv = reinterpret_cast<bf16*>(s.ws.qkv.p);
+    c.cat = reinterpret_cast<bf16*>(s.ws.cat.p);
+    c.hbuf = reinterpret_cast<bf16*>(s.ws.hbuf.p);
+    c.latb = reinterpret_cast<bf16*>(s.ws.latb.p);
+    c.pack = reinterpret_cast<bf16*>(s.ws.pack.p);
+    c.recv = reinterpret_cast<bf16*>(s.ws.recv.p);
+    c.obuf = reinterpret_cast<bf16*>(s.ws.obuf.p);
+    c.orecv = reinterpret_cast<bf16*>(s.ws.orecv.p);
+    c.mod = reinterpret_cast<const float*>(c.rd->mod.p) + (int64_t)step * m.n_mod;
+    E.rc.push_back(c);
+  }
+  // each slot's stream must follow the request's previous work on that slot
+  for (auto& c : E.rc) {
+    auto it = R.last.find(c.si);
+    if (it != R.last.end()) {
+      CK(cudaSetDevice(c.s->device));
+      CK(cudaStreamWaitEvent(c.s->stream, it->second, 0));
+    }
+  }
+  TRY(run_step(E));
+  for (auto& c : E.rc) TRY(record_last(e, R, c.si));
+  R.next_step = step + 1;
+  R.has_velocity = true;
+  if (done) TRY(new_event(e, g.local_slots, done));
+  return TSV_OK;
+}
+
+}  // namespace tsv
+
+// ================================================================== C ABI
+extern "C" {
+
+const char* tsv_last_error(void) { return g_err.c_str(); }
+
+tsv_status tsv_model_preset(const char* name, tsv_model_desc* out) {
+  if (!name || !out) return fail(TSV_E_INVAL, "null argument");
+  tsv_model_desc d{};
+  std::string n(name);
+  if (n == "flux") {
+    d = {3072, 24, 128, 12288, 19, 38, 64, 4096, 768, 512, {16, 56, 56}, 10000.f, 1};
+  } else if (n == "tiny" || n == "tiny_s" || n == "tiny2") {
+    d = {256, 4, 64, 1024, 1, 0, 64, 512, 256, 64, {8, 28, 28}, 10000.f, 1};
+    if (n == "tiny_s") d.n_single = 1;
+    if (n == "tiny2") { d.n_double = 2; d.n_single = 2; }
+  } else {
+    return fail(TSV_E_INVAL, "unknown preset '%s'", name);
+  }
+  *out = d;
+  return TSV_OK;
+}
+
+tsv_status tsv_engine_create(const tsv_model_desc* model, const int* devices, int n_local, int rank_base,
+                             int world_size, uint64_t weight_seed, tsv_engine** out) {
+  if (!model || !devices || !out || n_local <= 0 || rank_base < 0 || world_size < rank_base + n_local)
+    return fail(TSV_E_INVAL, "tsv_engine_create: bad arguments");
+  int ndev = 0;
+  CK(cudaGetDeviceCount(&ndev));
+  for (int i = 0; i < n_local; ++i)
+    if (devices[i] < 0 || devices[i] >= ndev) return fail(TSV_E_INVAL, "device %d out of range (%d)", devices[i], ndev);
+  auto e = std::make_unique<tsv_engine>();
+  std::string err;
+  if (!build_model(*model, &e->model, &err)) return fail(TSV_E_INVAL, "%s", err.c_str());
+  e->weight_seed = weight_seed;
+  e->rank_base = rank_base;
+  e->n_local = n_local;
+  e->world = world_size;
+  e->slots.resize(n_local);
+  for (int i = 0; i < n_local; ++i) {
+    Slot& s = e->slots[i];
+    s.rank = rank_base + i;
+    s.device = devices[i];
+    auto it = e->devs.find(s.device);
+    if (it == e->devs.end()) {
+      auto ds = std::make_unique<DeviceState>();
+      ds->device = s.device;
+      CK(cudaSetDevice(s.device));
+      CK(cudaDeviceGetAttribute(&ds->num_sms, cudaDevAttrMultiProcessorCount, s.device));
+      TRY(init_weights(e.get(), *ds));
+      it = e->devs.emplace(s.device, std::move(ds)).first;
+    }
+    s.ds = it->second.get();
+    CK(cudaSetDevice(s.device));
+    CK(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+  }
+  // peer access between distinct local devices (in-process all-to-all and reshard)
+  for (auto& a : e->devs)
+    for (auto& b : e->devs) {
+      if (a.first == b.first) continue;
+      int can = 0;
+      cudaDeviceCanAccessPeer(&can, a.first, b.first);
+      if (can) {
+        cudaSetDevice(a.first);
+        cudaError_t r = cudaDeviceEnablePeerAccess(b.first, 0);
+        if (r != cudaSuccess && r != cudaErrorPeerAccessAlreadyEnabled) return fail(TSV_E_CUDA, "peer access");
+        cudaGetLastError();
+      }
+    }
+  *out = e.release();
+  return TSV_OK;
+}
+
+void tsv_engine_destroy(tsv_engine* e) {
+  if (!e) return;
+  for (auto& s : e->slots) {
+    cudaSetDevice(s.device);
+    cudaStreamSynchronize(s.stream);
+  }
+  for (auto& kv : e->requests) {
+    for (auto& d : kv.second.dev) { d.second.mod.release(); d.second.dt.release(); }
+    for (auto& sh : kv.second.shard) {
+      sh.second.lat.release(); sh.second.vel.release(); sh.second.T.release();
+      sh.second.cosb.release(); sh.second.sinb.release();
+    }
+    for (auto& l : kv.second.last) cudaEventDestroy(l.second);
+  }
+  for (auto& g : e->groups) {
+    if (g.comm) ncclCommDestroy(g.comm);
+    for (auto ev : g.ev_a) cudaEventDestroy(ev);
+    for (auto ev : g.ev_b) cudaEventDestroy(ev);
+  }
+  if (e->world_comm) ncclCommDestroy(e->world_comm);
+  for (auto& rec : e->events)
+    for (auto& p : rec.evs) cudaEventDestroy(p.second);
+  for (auto& s : e->slots) {
+    Workspace& w = s.ws;
+    for (DevBuf* b : {&w.x, &w.u, &w.qkv, &w.cat, &w.hbuf, &w.latb, &w.pack, &w.recv, &w.obuf, &w.orecv, &s.scratch})
+      b->release();
+    cudaSetDevice(s.device);
+    cudaStreamDestroy(s.stream);
+  }
+  for (auto& d : e->devs) d.second->weights.release();
+  delete e;
+}
+
+tsv_status tsv_nccl_unique_id(uint8_t out[128]) {
+  if (!out) return fail(TSV_E_INVAL, "null argument");
+  ncclUniqueId id;
+  NK(ncclGetUniqueId(&id));
+  static_assert(sizeof(id) == 128, "ncclUniqueId size");
+  memcpy(out, &id, 128);
+  return TSV_OK;
+}
+
+tsv_status tsv_engine_init_world(tsv_engine* e, const uint8_t nccl_id[128]) {
+  if (!e || !nccl_id) return fail(TSV_E_INVAL, "null argument");
+  if (e->n_local != 1) return fail(TSV_E_UNSUPPORTED, "world communicator needs one local rank per process");
+  if (e->world_comm) return TSV_OK;
+  ncclUniqueId id;
+  memcpy(&id, nccl_id, 128);
+  CK(cudaSetDevice(e->slots[0].device));
+  NK(ncclCommInitRank(&e->world_comm, e->world, id, e->rank_base));
+  return TSV_OK;
+}
+
+tsv_status tsv_group_create(tsv_engine* e, const int* ranks, int k, const uint8_t* nccl_id, tsv_group* out) {
+  if (!e || !ranks || !out) return fail(TSV_E_INVAL, "null argument");
+  if (k < 1 || (k & (k - 1))) return fail(TSV_E_INVAL, "k = %d is not a power of two (P:225)", k);
+  if (k > e->world) return fail(TSV_E_INVAL, "k = %d exceeds the world size %d", k, e->world);
+  for (int i = 0; i < k; ++i) {
+    if (ranks[i] < 0 || ranks[i] >= e->world) return fail(TSV_E_INVAL, "rank %d outside the world", ranks[i]);
+    for (int j = 0; j < i; ++j)
+      if (ranks[j] == ranks[i]) return fail(TSV_E_INVAL, "duplicate rank %d", ranks[i]);
+  }
+  if (e->model.H % k) return fail(TSV_E_UNSUPPORTED, "k = %d does not divide the head count %d (S24)", k, e->model.H);
+  if ((e->model.h / k) % 64) return fail(TSV_E_UNSUPPORTED, "hidden/k must be a multiple of 64");
+  Group g;
+  g.ranks.assign(ranks, ranks + k);
+  g.k = k;
+  for (int i = 0; i < k; ++i) {
+    const int si = e->slot_of_rank(ranks[i]);
+    if (si >= 0) { g.local_slots.push_back(si); g.local_positions.push_back(i); }
+    else g.all_local = false;
+  }
+  if (!g.all_local && !g.local_slots.empty()) {
+    if (g.local_slots.size() != 1) return fail(TSV_E_UNSUPPORTED, "mixed local/remote groups need one local rank");
+    Slot& s = e->slots[g.local_slots[0]];
+    CK(cudaSetDevice(s.device));
+    if (nccl_id) {
+      ncclUniqueId id;
+      memcpy(&id, nccl_id, 128);
+      NK(ncclCommInitRank(&g.comm, k, id, g.local_positions[0]));
+    } else {
+      if (!e->world_comm) return fail(TSV_E_STATE, "group across processes needs nccl_id or init_world");
+      NK(ncclCommSplit(e->world_comm, 1, g.local_positions[0], &g.comm, nullptr));
+    }
+    // warm the communicator once
+    DevBuf tmp;
+    TRY(dev_alloc(tmp, s.device, 256 * k));
+    NK(ncclGroupStart());
+    for (int p = 0; p < k; ++p) {
+      NK(ncclSend(reinterpret_cast<uint8_t*>(tmp.p) + 0, 64, ncclUint8, p, g.comm, s.stream));
+      NK(ncclRecv(reinterpret_cast<uint8_t*>(tmp.p) + 128 + 0, 64, ncclUint8, p, g.comm, s.stream));
+    }
+    NK(ncclGroupEnd());
+    CK(cudaStreamSynchronize(s.stream));
+    tmp.release();
+  } else if (!g.all_local && g.local_slots.empty() && !nccl_id && e->world_comm) {
+    ncclComm_t none = nullptr;
+    NK(ncclCommSplit(e->world_comm, NCCL_SPLIT_NOCOLOR, 0, &none, nullptr));
+  }
+  if (g.all_local) {
+    // order local_slots by group rank (already in group order); events for the in-process a2a
+    for (int i = 0; i < k; ++i) {
+      Slot& s = e->slots[g.local_slots[i]];
+      CK(cudaSetDevice(s.device));
+      cudaEvent_t a, b;
+      CK(cudaEventCreateWithFlags(&a, cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&b, cudaEventDisableTiming));
+      g.ev_a.push_back(a);
+      g.ev_b.push_back(b);
+    }
+  }
+  e->groups.push_back(std::move(g));
+  *out = (tsv_group)e->groups.size() - 1;
+  return TSV_OK;
+}
+
+tsv_status tsv_request_create(tsv_engine* e, int height, int width, int num_steps, uint64_t seed, float guidance,
+                              tsv_request* out) {
+  if (!e || !out) return fail(TSV_E_INVAL, "null argument");
+  if (height <= 0 || width <= 0 || height % 16 || width % 16)
+    return fail(TSV_E_INVAL, "height and width must be positive multiples of 16 (P:442)");
+  if (num_steps < 1) return fail(TSV_E_INVAL, "num_steps must be >= 1");
+  const Model& m = e->model;
+  Request R;
+  R.height = height; R.width = width; R.S = num_steps; R.seed = seed; R.guidance = guidance;
+  R.Li = (int64_t)(height / 16) * (width / 16);
+  R.Lt = m.Lt;
+  R.x_host.resize((size_t)R.Li * m.in);
+  for (size_t i = 0; i < R.x_host.size(); ++i) R.x_host[i] = synth_r(seed, 1, i) * synth_scale(1.0);
+  R.T_host.resize((size_t)R.Lt * m.ctx);
+  const float c1 = synth_scale(1.0);
+  for (size_t i = 0; i < R.T_host.size(); ++i) R.T_host[i] = f32_to_bf16_bits(synth_r(seed, 2, i) * c1);
+  R.y_host.resize(m.vec);
+  for (size_t i = 0; i < R.y_host.size(); ++i) R.y_host[i] = f32_to_bf16_bits(synth_r(seed, 3, i) * c1);
+  // schedule t_j = sigma(1 - j/S), sigma(u) = e^mu / (e^mu + (1/u - 1)), mu linear in L_i
+  const double mu = 0.5 + (1.15 - 0.5) / (4096.0 - 256.0) * ((double)R.Li - 256.0);
+  R.ts.resize(num_steps + 1);
+  for (int j = 0; j <= num_steps; ++j) {
+    const double u = 1.0 - (double)j / num_steps;
+    R.ts[j] = u > 0 ? std::exp(mu) / (std::exp(mu) + (1.0 / u - 1.0)) : 0.0;
+  }
+  R.ts[0] = 1.0;
+  const int64_t id = e->next_req++;
+  e->requests.emplace(id, std::move(R));
+  *out = id;
+  return TSV_OK;
+}
+
+static Request* get_req(tsv_engine* e, tsv_request r) {
+  auto it = e->requests.find(r);
+  return it == e->requests.end() ? nullptr : &it->second;
+}
+
+tsv_status tsv_request_set_inputs(tsv_engine* e, tsv_request r, const float* x, const uint16_t* T, const uint16_t* y) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  Request* R = get_req(e, r);
+  if (!R) return fail(TSV_E_INVAL, "unknown request %lld", (long long)r);
+  if (R->group >= 0 || R->next_step > 0) return fail(TSV_E_STATE, "inputs can only be set before the first step");
+  if (x) memcpy(R->x_host.data(), x, R->x_host.size() * 4);
+  if (T) memcpy(R->T_host.data(), T, R->T_host.size() * 2);
+  if (y) memcpy(R->y_host.data(), y, R->y_host.size() * 2);
+  return TSV_OK;
+}
+
+tsv_status tsv_request_step(tsv_engine* e, tsv_request r, int step, tsv_group gi, tsv_event* done) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  Request* R = get_req(e, r);
+  if (!R) return fail(TSV_E_INVAL, "unknown request %lld", (long long)r);
+  if (gi < 0 || gi >= (int)e->groups.size()) return fail(TSV_E_INVAL, "unknown group %d", gi);
+  if (step != R->next_step)
+    return fail(TSV_E_STATE, "step %d requested but the next step is %d (step dependency, P:235-239)", step,
+                R->next_step);
+  if (step >= R->S) return fail(TSV_E_STATE, "request has only %d steps", R->S);
+  return do_step(e, *R, step, gi, done);
+}
+
+tsv_status tsv_request_reshard(tsv_engine* e, tsv_request r, tsv_group gi, tsv_event* done) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  Request* R = get_req(e, r);
+  if (!R) return fail(TSV_E_INVAL, "unknown request %lld", (long long)r);
+  if (gi < 0 || gi >= (int)e->groups.size()) return fail(TSV_E_INVAL, "unknown group %d", gi);
+  if (R->group != gi) TRY(move_request(e, *R, gi));
+  if (done) TRY(new_event(e, e->groups[gi].local_slots, done));
+  return TSV_OK;
+}
+
+tsv_status tsv_group_record(tsv_engine* e, tsv_group gi, tsv_event* out) {
+  if (!e || !out) return fail(TSV_E_INVAL, "null argument");
+  if (gi < 0 || gi >= (int)e->groups.size()) return fail(TSV_E_INVAL, "unknown group %d", gi);
+  return new_event(e, e->groups[gi].local_slots, out);
+}
+
+tsv_status tsv_event_wait(tsv_engine* e, tsv_event ev) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  if (ev == -1) return TSV_OK;
+  if (ev < 0 || ev >= (int64_t)e->events.size()) return fail(TSV_E_INVAL, "unknown event");
+  for (auto& p : e->events[ev].evs) CK(cudaEventSynchronize(p.second));
+  return TSV_OK;
+}
+
+tsv_status tsv_event_query(tsv_engine* e, tsv_event ev, int* done) {
+  if (!e || !done) return fail(TSV_E_INVAL, "null argument");
+  if (ev == -1) { *done = 1; return TSV_OK; }
+  if (ev < 0 || ev >= (int64_t)e->events.size()) return fail(TSV_E_INVAL, "unknown event");
+  *done = 1;
+  for (auto& p : e->events[ev].evs) {
+    cudaError_t q = cudaEventQuery(p.second);
+    if (q == cudaErrorNotReady) { *done = 0; cudaGetLastError(); }
+    else if (q != cudaSuccess) return fail(TSV_E_CUDA, "event query: %s", cudaGetErrorString(q));
+  }
+  return TSV_OK;
+}
+
+tsv_status tsv_event_elapsed_ms(tsv_engine* e, tsv_event a, tsv_event b, float* ms) {
+  if (!e || !ms) return fail(TSV_E_INVAL, "null argument");
+  if (a < 0 || b < 0 || a >= (int64_t)e->events.size() || b >= (int64_t)e->events.size())
+    return fail(TSV_E_INVAL, "unknown event");
+  auto& ea = e->events[a].evs;
+  auto& eb = e->events[b].evs;
+  if (ea.size() != eb.size()) return fail(TSV_E_INVAL, "events of different groups");
+  float mx = 0.f;
+  for (size_t i = 0; i < ea.size(); ++i) {
+    if (ea[i].first != eb[i].first) return fail(TSV_E_INVAL, "events of different groups");
+    CK(cudaEventSynchronize(eb[i].second));
+    float t = 0.f;
+    CK(cudaEventElapsedTime(&t, ea[i].second, eb[i].second));
+    mx = std::max(mx, t);
+  }
+  *ms = mx;
+  return TSV_OK;
+}
+
+static tsv_status latent_io(tsv_engine* e, tsv_request r, int64_t row0, int64_t nrows, float* host, bool write,
+                            bool velocity) {
+  if (!e || !host) return fail(TSV_E_INVAL, "null argument");
+  Request* R = get_req(e, r);
+  if (!R) return fail(TSV_E_INVAL, "unknown request %lld", (long long)r);
+  const int in = e->model.in;
+  if (row0 < 0 || nrows < 0 || row0 + nrows > R->Li) return fail(TSV_E_INVAL, "rows out of range");
+  if (velocity && !R->has_velocity) return fail(TSV_E_STATE, "no completed step");
+  if (R->group < 0) {
+    if (velocity) return fail(TSV_E_STATE, "no completed step");
+    if (write) memcpy(R->x_host.data() + row0 * in, host, nrows * in * 4);
+    else memcpy(host, R->x_host.data() + row0 * in, nrows * in * 4);
+    return TSV_OK;
+  }
+  // rows must be covered by local shards
+  int64_t covered = 0;
+  for (auto& kv : R->shard) {
+    ReqShard& sh = kv.second;
+    const int64_t lo = std::max(row0, sh.i0), hi = std::min(row0 + nrows, sh.i0 + sh.ni);
+    if (hi <= lo) continue;
+    covered += hi - lo;
+    Slot& s = e->slots[kv.first];
+    CK(cudaSetDevice(s.device));
+    float* dev = reinterpret_cast<float*>(velocity ? sh.vel.p : sh.lat.p) + (lo - sh.i0) * in;
+    float* hp = host + (lo - row0) * in;
+    CK(cudaStreamWaitEvent(s.stream, R->last[kv.first], 0));
+    if (write) CK(cudaMemcpyAsync(dev, hp, (hi - lo) * in * 4, cudaMemcpyHostToDevice, s.stream));
+    else CK(cudaMemcpyAsync(hp, dev, (hi - lo) * in * 4, cudaMemcpyDeviceToHost, s.stream));
+    CK(cudaStreamSynchronize(s.stream));
+    TRY(record_last(e, *R, kv.first));
+  }
+  if (covered != nrows) return fail(TSV_E_INVAL, "rows [%lld, %lld) are not all held by local ranks", (long long)row0,
+                                    (long long)(row0 + nrows));
+  return TSV_OK;
+}
+
+tsv_status tsv_request_read_latent(tsv_engine* e, tsv_request r, int64_t row0, int64_t nrows, float* host) {
+  return latent_io(e, r, row0, nrows, host, false, false);
+}
+tsv_status tsv_request_write_latent(tsv_engine* e, tsv_request r, int64_t row0, int64_t nrows, const float* host) {
+  return latent_io(e, r, row0, nrows, const_cast<float*>(host), true, false);
+}
+tsv_status tsv_request_read_velocity(tsv_engine* e, tsv_request r, int64_t row0, int64_t nrows, float* host) {
+  return latent_io(e, r, row0, nrows, host, false, true);
+}
+
+tsv_status tsv_request_info(tsv_engine* e, tsv_request r, int* next_step, tsv_group* group, int64_t* li) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  Request* R = get_req(e, r);
+  if (!R) return fail(TSV_E_INVAL, "unknown request %lld", (long long)r);
+  if (next_step) *next_step = R->next_step;
+  if (group) *group = R->group;
+  if (li) *li = R->Li;
+  return TSV_OK;
+}
+
+tsv_status tsv_request_destroy(tsv_engine* e, tsv_request r) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  auto it = e->requests.find(r);
+  if (it == e->requests.end()) return fail(TSV_E_INVAL, "unknown request %lld", (long long)r);
+  Request& R = it->second;
+  for (auto& l : R.last) { cudaEventSynchronize(l.second); cudaEventDestroy(l.second); }
+  for (auto& d : R.dev) { d.second.mod.release(); d.second.dt.release(); }
+  for (auto& sh : R.shard) {
+    sh.second.lat.release(); sh.second.vel.release(); sh.second.T.release();
+    sh.second.cosb.release(); sh.second.sinb.release();
+  }
+  e->requests.erase(it);
+  return TSV_OK;
+}
+
+tsv_status tsv_latency_table(tsv_engine* e, const int* res_px, int n_res, const int* ks, int n_k, int warmup,
+                             int iters, double* ms_out, double* cv_out) {
+  if (!e || !res_px || !ks || !ms_out || n_res <= 0 || n_k <= 0 || iters < 1 || warmup < 0)
+    return fail(TSV_E_INVAL, "bad arguments");
+  const bool multi = e->n_local < e->world;
+  if (multi && !e->world_comm) return fail(TSV_E_STATE, "multi-process latency table needs tsv_engine_init_world");
+  for (int i = 0; i < n_res; ++i)
+    for (int j = 0; j < n_k; ++j) {
+      const int k = ks[j];
+      double& out_ms = ms_out[i * n_k + j];
+      double* out_cv = cv_out ? &cv_out[i * n_k + j] : nullptr;
+      if (k > e->world || k < 1 || (k & (k - 1)) || e->model.H % k) {
+        out_ms = -1;
+        if (out_cv) *out_cv = -1;
+        continue;
+      }
+      std::vector<int> ranks(k);
+      for (int q = 0; q < k; ++q) ranks[q] = q;
+      tsv_group g;
+      TRY(tsv_group_create(e, ranks.data(), k, nullptr, &g));
+      tsv_request rq;
+      TRY(tsv_request_create(e, res_px[i], res_px[i], warmup + iters, 1000 + i, 3.5f, &rq));
+      std::vector<double> times;
+      for (int st = 0; st < warmup + iters; ++st) {
+        tsv_event a = -1, b = -1;
+        if (st == 0) TRY(tsv_request_reshard(e, rq, g, nullptr));
+        if (!e->groups[g].local_slots.empty()) TRY(tsv_group_record(e, g, &a));
+        TRY(tsv_request_step(e, rq, st, g, &b));
+        float ms = 0.f;
+        if (b >= 0) TRY(tsv_event_elapsed_ms(e, a, b, &ms));
+        if (multi) {
+          // max over ranks
+          Slot& s = e->slots[0];
+          DevBuf tb;
+          TRY(dev_alloc(tb, s.device, 4));
+          CK(cudaMemcpyAsync(tb.p, &ms, 4, cudaMemcpyHostToDevice, s.stream));
+          NK(ncclAllReduce(tb.p, tb.p, 1, ncclFloat32, ncclMax, e->world_comm, s.stream));
+          CK(cudaMemcpyAsync(&ms, tb.p, 4, cudaMemcpyDeviceToHost, s.stream));
+          CK(cudaStreamSynchronize(s.stream));
+          tb.release();
+        }
+        if (st >= warmup) times.push_back(ms);
+      }
+      TRY(tsv_request_destroy(e, rq));
+      std::vector<double> sorted = times;
+      std::sort(sorted.begin(), sorted.end());
+      const size_t n = sorted.size();
+      out_ms = n % 2 ? sorted[n / 2] : 0.5 * (sorted[n / 2 - 1] + sorted[n / 2]);
+      double mean = 0, var = 0;
+      for (double t : times) mean += t;
+      mean /= n;
+      for (double t : times) var += (t - mean) * (t - mean);
+      var = n > 1 ? var / (n - 1) : 0.0;
+      if (out_cv) *out_cv = mean > 0 ? std::sqrt(var) / mean : 0.0;
+    }
+  return TSV_OK;
+}
+
+tsv_status tsv_shard_range(int64_t n, int k, int r, int64_t* b, int64_t* en) {
+  if (!b || !en || n < 0 || k < 1 || r < 0 || r >= k) return fail(TSV_E_INVAL, "bad shard arguments");
+  *b = shard_begin(n, k, r);
+  *en = shard_begin(n, k, r + 1);
+  return TSV_OK;
+}
+
+tsv_status tsv_reshard_plan(int64_t n, int ks, int kd, int64_t* out, int max_copies, int* n_copies) {
+  if (!n_copies || n < 0 || ks < 1 || kd < 1 || (max_copies > 0 && !out)) return fail(TSV_E_INVAL, "bad arguments");
+  int c = 0;
+  for (int s = 0; s < ks; ++s) {
+    const int64_t a0 = shard_begin(n, ks, s), a1 = shard_begin(n, ks, s + 1);
+    for (int d = 0; d < kd; ++d) {
+      const int64_t b0 = shard_begin(n, kd, d), b1 = shard_begin(n, kd, d + 1);
+      const int64_t lo = std::max(a0, b0), hi = std::min(a1, b1);
+      if (hi <= lo) continue;
+      if (c < max_copies) {
+        int64_t* o = out + 5 * c;
+        o[0] = s; o[1] = lo - a0; o[2] = d; o[3] = lo - b0; o[4] = hi - lo;
+      }
+      ++c;
+    }
+  }
+  *n_copies = c;
+  if (c > max_copies) return fail(TSV_E_INVAL, "plan has %d copies, buffer holds %d", c, max_copies);
+  return TSV_OK;
+}
+
+tsv_status tsv_debug_read_weight(tsv_engine* e, int id, uint16_t* host, size_t n) {
+  if (!e || !host) return fail(TSV_E_INVAL, "null argument");
+  const TensorInfo* t = e->model.find(id);
+  if (!t) return fail(TSV_E_INVAL, "unknown tensor id %d", id);
+  if (n != (size_t)t->numel()) return fail(TSV_E_INVAL, "tensor %d has %lld elements", id, (long long)t->numel());
+  Slot& s = e->slots[0];
+  CK(cudaSetDevice(s.device));
+  CK(cudaMemcpy(host, reinterpret_cast<const bf16*>(s.ds->weights.p) + t->offset, n * 2, cudaMemcpyDeviceToHost));
+  return TSV_OK;
+}
+
+tsv_status tsv_engine_profile(tsv_engine* e, int enable) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  for (auto& r : e->prof_recs) {
+    e->ev_pool[r.device].push_back(r.a);
+    e->ev_pool[r.device].push_back(r.b);
+  }
+  e->prof_recs.clear();
+  for (int i = 0; i < 8; ++i) { e->prof_flops[i] = 0; e->prof_bytes[i] = 0; e->prof_launch[i] = 0; }
+  e->prof = enable != 0;
+  return TSV_OK;
+}
+
+tsv_status tsv_engine_profile_read(tsv_engine* e, double* ms, int64_t* launches, double* flops, double* bytes) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  double acc[8] = {0};
+  for (auto& r : e->prof_recs) {
+    CK(cudaSetDevice(r.device));
+    CK(cudaEventSynchronize(r.b));
+    float t = 0.f;
+    CK(cudaEventElapsedTime(&t, r.a, r.b));
+    acc[r.cls] += t;
+  }
+  for (int i = 0; i < KC_N; ++i) {
+    if (ms) ms[i] = acc[i];
+    if (launches) launches[i] = e->prof_launch[i];
+    if (flops) flops[i] = e->prof_flops[i];
+    if (bytes) bytes[i] = e->prof_bytes[i];
+  }
+  return TSV_OK;
+}
+
+tsv_status tsv_engine_kernel_count(tsv_engine* e, int64_t* count) {
+  if (!e || !count) return fail(TSV_E_INVAL, "null argument");
+  *count = e->kernel_count;
+  return TSV_OK;
+}
+
+// ------------------------------------------------------------------ kernel-level ops (tsv_ops.h)
+tsv_status tsv_op_gemm(const void* A, int64_t lda, const void* Wt, int64_t ldw, int M, int N, int K, int mode,
+                       void* out0, int64_t ld0, void* out1, int64_t ld1, int n_split, const void* bias,
+                       const float* gate, const float* scalar, int force_bn, void* stream) {
+  if (mode < 0 || mode > EPI_EULER) return fail(TSV_E_INVAL, "bad epilogue mode %d", mode);
+  if (force_bn && force_bn != 64 && force_bn != 128 && force_bn != 256) return fail(TSV_E_INVAL, "bad force_bn");
+  int dev = 0, sms = 148;
+  CK(cudaGetDevice(&dev));
+  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  GemmPlan p;
+  const char* err = nullptr;
+  GemmEpi epi = epi_of(mode, out0, ld0, reinterpret_cast<const bf16*>(bias), gate, out1, ld1, n_split, scalar);
+  if (gemm_plan(&p, reinterpret_cast<const bf16*>(A), lda, reinterpret_cast<const bf16*>(Wt), ldw, M, N, K, epi, sms,
+                &err, force_bn))
+    return fail(TSV_E_INVAL, "%s", err);
+  gemm_launch(p, reinterpret_cast<cudaStream_t>(stream));
+  CK(cudaGetLastError());
+  return TSV_OK;
+}
+
+tsv_status tsv_op_ln_mod(const float* x, int64_t ldx, void* u, int64_t ldu, const float* shift, const float* scale,
+                         int M, int h, void* stream) {
+  if (h % 128) return fail(TSV_E_INVAL, "h must be a multiple of 128");
+  ln_mod_launch(x, ldx, reinterpret_cast<bf16*>(u), ldu, shift, scale, M, h, reinterpret_cast<cudaStream_t>(stream));
+  CK(cudaGetLastError());
+  return TSV_OK;
+}
+
+tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int H, int D, const void* gq0,
+                               const void* gk0, const void* gq1, const void* gk1, const float* cosb,
+                               const float* sinb, void* pack, int k_sp, void* stream) {
+  if (D != 64 && D != 128) return fail(TSV_E_INVAL, "D must be 64 or 128");
+  if (k_sp < 1 || H % k_sp) return fail(TSV_E_INVAL, "k_sp must divide H");
+  qk_norm_rope_launch(reinterpret_cast<bf16*>(qkv), ld, rows, n_first, H, D, reinterpret_cast<const bf16*>(gq0),
+                      reinterpret_cast<const bf16*>(gk0), reinterpret_cast<const bf16*>(gq1),
+                      reinterpret_cast<const bf16*>(gk1), cosb, sinb, reinterpret_cast<bf16*>(pack), k_sp,
+                      reinterpret_cast<cudaStream_t>(stream));
+  CK(cudaGetLastError());
+  return TSV_OK;
+}
+
+tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
+                            void* o, int64_t ldo, int L, int H, int D, void* stream) {
+  if (D != 64 && D != 128) return fail(TSV_E_INVAL, "D must be 64 or 128");
+  attention_launch(reinterpret_cast<const bf16*>(q), ldq, reinterpret_cast<const bf16*>(k), ldk,
+                   reinterpret_cast<const bf16*>(v), ldv, reinterpret_cast<bf16*>(o), ldo, L, H, D,
+                   reinterpret_cast<cudaStream_t>(stream));
+  CK(cudaGetLastError());
+  return TSV_OK;
+}
+
+tsv_status tsv_op_synth(void* dst, uint64_t seed, uint32_t tid, uint64_t idx0, int64_t n, int kind, float c,
+                        void* stream) {
+  if (kind < 0 || kind > 2) return fail(TSV_E_INVAL, "bad kind");
+  synth_launch(dst, seed, tid, idx0, n, kind, c, reinterpret_cast<cudaStream_t>(stream));
+  CK(cudaGetLastError());
+  return TSV_OK;
+}
+
+}  // extern "C"

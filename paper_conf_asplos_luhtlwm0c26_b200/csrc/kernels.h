@@ -1,0 +1,86 @@
+// Host-side launchers of the sm_100a kernels (internal to libtsv.so; the public C-ABI is in
+// include/tsv.h and include/tsv_ops.h).
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+namespace tsv {
+
+using bf16 = __nv_bfloat16;
+
+// ------------------------------------------------------------------ GEMM  y = A W^T (+ bias) -> epilogue
+enum EpiMode : int {
+  EPI_STORE_BF16 = 0,   // out0[m,n] = bf16(acc + b)
+  EPI_GELU_BF16 = 1,    // out0[m,n] = bf16(gelu_tanh(acc + b))
+  EPI_SILU_BF16 = 2,    // out0[m,n] = bf16(silu(acc + b))
+  EPI_SPLIT_GELU = 3,   // n < n_split: out0[m,n] = bf16(acc+b); else out1[m,n-n_split] = bf16(gelu(acc+b))
+  EPI_RESID_GATE = 4,   // out0 (fp32) [m,n] += gate[n] * (acc + b)
+  EPI_STORE_F32 = 5,    // out0 (fp32) [m,n] = acc + b
+  EPI_ACCUM_F32 = 6,    // out0 (fp32) [m,n] += acc + b
+  EPI_EULER = 7,        // v = acc + b; out1 (fp32, optional) [m,n] = v; out0 (fp32) [m,n] += (*scalar) * v
+};
+
+struct GemmEpi {
+  int mode = EPI_STORE_BF16;
+  void* out0 = nullptr;
+  long long ld0 = 0;  // elements
+  void* out1 = nullptr;
+  long long ld1 = 0;
+  int n_split = 0;
+  const bf16* bias = nullptr;   // [N]
+  const float* gate = nullptr;  // [N]
+  const float* scalar = nullptr;
+};
+
+struct GemmPlan {
+  CUtensorMap tmA, tmB;
+  int M = 0, N = 0, K = 0;
+  int BN = 256;
+  int grid = 0;
+  GemmEpi epi;
+};
+
+// A: [M, K] bf16 row stride lda (elements); W: [N, K] bf16 row stride ldw. K % 64 == 0, N % 64 == 0.
+// Returns 0 on success, nonzero (and sets *err) on invalid arguments.
+int gemm_plan(GemmPlan* p, const bf16* A, long long lda, const bf16* W, long long ldw, int M, int N, int K,
+              const GemmEpi& epi, int num_sms, const char** err, int force_bn = 0);
+void gemm_launch(const GemmPlan& p, cudaStream_t s);
+
+// ------------------------------------------------------------------ elementwise / norm kernels
+// u[m, :] = bf16( LN(x[m, :]) * (1 + scale) + shift ), x fp32 row stride ldx, u row stride ldu
+void ln_mod_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift, const float* scale,
+                   int M, int h, cudaStream_t s);
+
+// In-place on a qkv buffer [rows, 3*H*D] (row stride ld): q,k <- RoPE(RMSNorm(.) * g).
+// Rows [0, n_first) use gains (gq0, gk0), rows [n_first, rows) use (gq1, gk1).
+// cos/sin tables: [rows, D/2] fp32.
+// If pack_out != null the result for all of q, k, v is instead written to the Ulysses send
+// buffer pack_out laid out [k_sp][rows][3][H/k_sp][D] (bf16), and qkv is left unchanged.
+void qk_norm_rope_launch(bf16* qkv, long long ld, int rows, int n_first, int H, int D, const bf16* gq0,
+                         const bf16* gk0, const bf16* gq1, const bf16* gk1, const float* cosb, const float* sinb,
+                         bf16* pack_out, int k_sp, cudaStream_t s);
+
+// Joint attention, non-causal: O[l, h*D + d] = softmax(q k^T / sqrt(D)) v for heads h in [0, H).
+// q(l, h) at q + l*ldq + h*D (same for k, v, o). L rows.
+void attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
+                      bf16* o, long long ldo, int L, int H, int D, cudaStream_t s);
+
+// dst[m, c] = bf16(src[m, c]) (fp32 -> bf16), row strides in elements
+void f32_to_bf16_launch(const float* src, long long lds, bf16* dst, long long ldd, int M, int C, cudaStream_t s);
+// dst[m, c] = bf16(silu(src[m, c]))
+void silu_bf16_launch(const float* src, long long lds, bf16* dst, long long ldd, int M, int C, cudaStream_t s);
+// dst[r, :] = src[r, :] copies of rows, 2D strided bf16 (used by Ulysses unpack)
+void copy2d_bf16_launch(const bf16* src, long long lds, bf16* dst, long long ldd, int rows, int cols, cudaStream_t s);
+// dst[m] = src[*idx_dev * stride + m] for m < n (fp32): per-step row selection inside a graph
+void select_row_launch(const float* src, long long stride, const int* idx_dev, float* dst, long long n,
+                       cudaStream_t s);
+
+// ------------------------------------------------------------------ SYNTH-1 generator
+// kind: 0 'w'/'b'/'x' (bf16 = rne(r*c)), 1 'g' (bf16 = rne(1 + r*c)), 2 'f' (fp32 = r*c)
+void synth_launch(void* dst, uint64_t seed, uint32_t tensor_id, uint64_t idx0, long long n, int kind, float c,
+                  cudaStream_t s);
+
+}  // namespace tsv

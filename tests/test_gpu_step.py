@@ -1,0 +1,181 @@
+"""Step-level parity (GPU) through the C-ABI: the full denoising step against the float64 oracle,
+SP=k vs SP=1 on one GPU (k virtual ranks), bit-exact reshard, and the API's error model."""
+import os
+
+import numpy as np
+import pytest
+
+from oracle import flux as F
+from oracle.config import MODELS
+from oracle.weights import Weights, request_inputs
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+TOL_REL, TOL_COS = 2e-2, 0.999   # BASELINE.json north_star: max rel error 2e-2, cosine >= 0.999
+
+
+@pytest.fixture(scope="module")
+def tsv():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import paper_conf_asplos_luhtlwm0c26_b200 as m
+    return m
+
+
+def _metrics(g, o):
+    rel = float(np.max(np.abs(g - o)) / np.max(np.abs(o)))
+    cos = float(np.sum(g * o) / np.linalg.norm(g) / np.linalg.norm(o))
+    return rel, cos
+
+
+@pytest.mark.parametrize("model,res,steps,step", [("tiny", (256, 256), 1, 0), ("tiny_s", (256, 256), 4, 0),
+                                                  ("tiny2", (320, 192), 20, 0)])
+def test_step_vs_oracle(tsv, model, res, steps, step):
+    cfg = MODELS[model]
+    H, Wd = res
+    eng = tsv.Engine(model, devices=[0])
+    g = eng.group_create([0])
+    req = eng.request_create(H, Wd, num_steps=steps, seed=1000, guidance=3.5)
+    x0 = eng.read_latent(req)
+    x, T, y = request_inputs(cfg, H, Wd, 1000)
+    assert np.array_equal(x0, x.astype(np.float32))          # host SYNTH-1 inputs are bit-exact
+    eng.event_wait(eng.request_step(req, 0, g))
+    v, x1 = eng.read_velocity(req), eng.read_latent(req)
+    vo, xo = F.request_step(cfg, Weights(cfg), x, T, y, 0, steps, 3.5, H, Wd)
+    for got, ref in ((v, vo), (x1, xo)):
+        rel, cos = _metrics(got.astype(np.float64), ref)
+        assert rel <= TOL_REL and cos >= TOL_COS, (rel, cos)
+    eng.close()
+
+
+def test_multi_step_trajectory(tsv):
+    """Three consecutive steps: each step's output feeds the next (state stays on the GPU)."""
+    cfg = MODELS["tiny2"]
+    eng = tsv.Engine("tiny2", devices=[0])
+    g = eng.group_create([0])
+    req = eng.request_create(256, 256, num_steps=3, seed=1001)
+    x, T, y = request_inputs(cfg, 256, 256, 1001)
+    W = Weights(cfg)
+    xo = x
+    for s in range(3):
+        eng.request_step(req, s, g)
+        _, xo = F.request_step(cfg, W, xo, T, y, s, 3, 3.5, 256, 256)
+    rel, cos = _metrics(eng.read_latent(req).astype(np.float64), xo)
+    assert rel <= TOL_REL and cos >= TOL_COS
+    eng.close()
+
+
+@pytest.mark.parametrize("k", [2, 4])
+def test_sp_invariance_virtual_ranks(tsv, k):
+    """SP=k on k virtual ranks of one GPU (in-process all-to-all) vs SP=1 (S:§8(c) P9)."""
+    eng = tsv.Engine("tiny2", devices=[0] * 4)
+    g1 = eng.group_create([0])
+    gk = eng.group_create(list(range(k)))
+    r1 = eng.request_create(320, 192, num_steps=4, seed=1002)
+    rk = eng.request_create(320, 192, num_steps=4, seed=1002)
+    for s in range(2):
+        eng.request_step(r1, s, g1)
+        eng.request_step(rk, s, gk)
+    a, b = eng.read_latent(r1).astype(np.float64), eng.read_latent(rk).astype(np.float64)
+    print(f"SP={k} vs SP=1 bitwise equal: {np.array_equal(a, b)}")   # diagnostic (S19), not a gate
+    rel, cos = _metrics(b, a)
+    assert rel <= 1e-2 and cos >= 0.9999, (rel, cos)
+    eng.close()
+
+
+def test_sp_k_vs_oracle_uneven_text(tsv):
+    """k = 4 with 64 text + 195 image tokens (uneven image shards 49/49/49/48) vs the oracle."""
+    cfg = MODELS["tiny2"]
+    eng = tsv.Engine("tiny2", devices=[0] * 4)
+    g = eng.group_create([3, 1, 0, 2])      # arbitrary rank order (S14)
+    req = eng.request_create(208, 240, num_steps=2, seed=1003)
+    eng.event_wait(eng.request_step(req, 0, g))
+    x, T, y = request_inputs(cfg, 208, 240, 1003)
+    vo, xo = F.request_step(cfg, Weights(cfg), x, T, y, 0, 2, 3.5, 208, 240)
+    rel, cos = _metrics(eng.read_velocity(req).astype(np.float64), vo)
+    assert rel <= TOL_REL and cos >= TOL_COS, (rel, cos)
+    eng.close()
+
+
+def test_reshard_bitwise_and_step_level_sp(tsv):
+    """Config-4 shape of schedule on virtual ranks: k changes between steps, every reshard is a
+    bit-exact move (S:§8(c) P10), and the trajectory matches an all-k=1 run within tolerance."""
+    eng = tsv.Engine("tiny2", devices=[0] * 4)
+    groups = {k: eng.group_create(list(range(k))) for k in (1, 2, 4)}
+    g23 = eng.group_create([2, 3])
+    plan = [groups[2], groups[4], g23, groups[1], groups[4]]
+    ra = eng.request_create(256, 256, num_steps=5, seed=1004)
+    rb = eng.request_create(256, 256, num_steps=5, seed=1004)
+    for s, g in enumerate(plan):
+        if s > 0:
+            before = eng.read_latent(ra)
+            eng.event_wait(eng.request_reshard(ra, g))
+            assert np.array_equal(before, eng.read_latent(ra))
+        eng.request_step(ra, s, g)
+        eng.request_step(rb, s, groups[1])
+    rel, cos = _metrics(eng.read_latent(ra).astype(np.float64), eng.read_latent(rb).astype(np.float64))
+    assert rel <= 1e-2 and cos >= 0.9999
+    eng.close()
+
+
+def test_api_errors(tsv):
+    eng = tsv.Engine("tiny", devices=[0, 0])
+    with pytest.raises(tsv.TsvError) as e:
+        eng.group_create([0, 1, 0])
+    assert e.value.status == -1   # k = 3 is not a power of two
+    with pytest.raises(tsv.TsvError) as e:
+        eng.group_create([0, 0])
+    assert e.value.status == -1   # duplicate rank
+    with pytest.raises(tsv.TsvError) as e:
+        eng.request_create(250, 256)
+    assert e.value.status == -1
+    g = eng.group_create([0])
+    req = eng.request_create(256, 256, num_steps=2)
+    with pytest.raises(tsv.TsvError) as e:
+        eng.request_step(req, 1, g)    # step dependency
+    assert e.value.status == -2
+    eng.request_step(req, 0, g)
+    eng.request_step(req, 1, g)
+    with pytest.raises(tsv.TsvError) as e:
+        eng.request_step(req, 2, g)
+    assert e.value.status == -2
+    with pytest.raises(tsv.TsvError) as e:
+        eng.request_set_inputs(req, x=np.zeros((256, 64), np.float32))
+    assert e.value.status == -2
+    eng.close()
+    eng8 = tsv.Engine("tiny", devices=[0] * 8)
+    with pytest.raises(tsv.TsvError) as e:
+        eng8.group_create(list(range(8)))   # 8 does not divide the 4 tiny heads (S24)
+    assert e.value.status == -6
+    eng8.close()
+
+
+def test_latency_table_small(tsv):
+    eng = tsv.Engine("tiny2", devices=[0, 0])
+    ms, cv = eng.latency_table([256, 512], [1, 2, 4], warmup=2, iters=5)
+    assert np.all(ms[:, :2] > 0) and np.all(ms[:, 2] == -1)   # k = 4 > world size 2
+    eng.close()
+
+
+def _golden(name):
+    p = os.path.join(ROOT, "tests", "golden", name)
+    if not os.path.exists(p):
+        pytest.skip(f"golden {name} not generated (tools/make_golden.py)")
+    return np.load(p)
+
+
+def test_flux_512_step_vs_golden(tsv):
+    """BASELINE config 2: full 57-block FLUX.1-dev-shaped step at 512x512 (1024 + 512 tokens),
+    SP=1, the launch configuration bench.py times, vs the float64 oracle.  The golden is written
+    by tools/make_golden.py, which calls only oracle/ (request seed 1000, S = 1: t 1 -> 0)."""
+    gold = _golden("flux512_seed1000_S1.npz")
+    eng = tsv.Engine("flux", devices=[0])
+    g = eng.group_create([0])
+    req = eng.request_create(512, 512, num_steps=1, seed=1000)
+    eng.event_wait(eng.request_step(req, 0, g))
+    v, x1 = eng.read_velocity(req).astype(np.float64), eng.read_latent(req).astype(np.float64)
+    for got, ref in ((v, gold["v"]), (x1, gold["x_next"])):
+        rel, cos = _metrics(got, ref)
+        assert rel <= TOL_REL and cos >= TOL_COS, (rel, cos)
+    eng.close()
