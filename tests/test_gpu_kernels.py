@@ -198,7 +198,7 @@ def test_qk_norm_rope(tsv, H, D, rows, n_first):
     # pack layout [k_sp][rows][3][H/k][D] equals the in-place result permuted, bit for bit
     for k_sp in (2, 4):
         t2 = _bf16(qkv)
-        pack = torch.zeros(k_sp * rows * 3 * h, dtype=torch.bfloat16, device="cuda")
+        pack = torch.zeros(rows * 3 * h, dtype=torch.bfloat16, device="cuda")
         tsv.op_qk_norm_rope(t2, n_first, H, D, gt[0], gt[1], gt[2], gt[3], _f32(cosb), _f32(sinb), pack=pack, k_sp=k_sp)
         torch.cuda.synchronize()
         p = pack.view(k_sp, rows, 3, H // k_sp, D).permute(1, 2, 0, 3, 4).reshape(rows, 3, H, D)
