@@ -51,9 +51,11 @@ tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int
                                const float* sinb, void* pack, int k_sp, void* stream);
 
 /* a6: O = softmax(q k^T / sqrt(D)) v, non-causal, per head h < H; q(l, h) at q + l*ldq + h*D
- * (bf16, same for k, v, o).  D in {64, 128}. */
+ * (bf16, same for k, v, o).  D in {64, 128}.  Operands and row strides 16-byte aligned.
+ * impl 0: the tcgen05/TMEM kernel the step uses; impl 1: the mma.sync (FA2-style) baseline,
+ * kept only for comparison. */
 tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
-                            void* o, int64_t ldo, int L, int H, int D, void* stream);
+                            void* o, int64_t ldo, int L, int H, int D, int impl, void* stream);
 
 /* SYNTH-1 on device: n values of (seed, tensor_id) starting at element idx0.
  * kind 0: bf16 rne(r*c); 1: bf16 rne(1 + r*c); 2: fp32 r*c. */

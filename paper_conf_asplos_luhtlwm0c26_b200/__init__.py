@@ -230,9 +230,10 @@ def op_qk_norm_rope(qkv, n_first, H, D, gq0, gk0, gq1, gk1, cosb, sinb, pack=Non
                                   _ptr(gk1), _ptr(cosb), _ptr(sinb), _ptr(pack), k_sp, _stream(stream)))
 
 
-def op_attention(q, k, v, o, L, H, D, ldq=None, ldk=None, ldv=None, ldo=None, stream=None):
+def op_attention(q, k, v, o, L, H, D, ldq=None, ldk=None, ldv=None, ldo=None, impl=0, stream=None):
+    """impl 0: tcgen05 kernel (the step's); impl 1: mma.sync baseline (comparison only)."""
     check(lib.tsv_op_attention(_ptr(q), ldq or q.stride(0), _ptr(k), ldk or k.stride(0), _ptr(v), ldv or v.stride(0),
-                               _ptr(o), ldo or o.stride(0), L, H, D, _stream(stream)))
+                               _ptr(o), ldo or o.stride(0), L, H, D, impl, _stream(stream)))
 
 
 def op_synth(dst, seed, tensor_id, n, kind, c, idx0=0, stream=None):

@@ -213,7 +213,7 @@ __global__ void __launch_bounds__(ATT_WARPS * 32) attention_mma_kernel(const bf1
   }
 }
 
-void attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
+void attention_mma_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
                       bf16* o, long long ldo, int L, int H, int D, cudaStream_t s) {
   if (L <= 0 || H <= 0) return;
   dim3 grid((L + ATT_BQ - 1) / ATT_BQ, H);

@@ -1,0 +1,343 @@
+// Joint text+image attention on the 5th-gen tensor cores (S:§8(a) a6):
+//   O = softmax(q k^T / sqrt(D)) v, non-causal, per head, fp32 online softmax, bf16 operands.
+//
+// One CTA = one (head, 128-query tile).  Warp roles:
+//   warp 0      TMA producer: Q once, then K/V tiles of 128 keys into a 2-stage ring
+//               (3-D tensor maps [rows][heads][D] -> one map serves every head and layout);
+//   warp 1      single-thread tcgen05.mma issuer:  S_j = Q K_j^T into one of two TMEM S buffers
+//               (issued one tile ahead), then O += P_j V_j (V consumed MN-major straight from the
+//               TMA tile, no transpose);
+//   warps 4-7   softmax: thread i owns query row i (TMEM lane i): tcgen05.ld of its 128 scores,
+//               row max / exp2 / row sum in registers, P_j as bf16 into a 128B-swizzled K-major
+//               smem tile (double-buffered), conditional O rescale (only when the running max grows
+//               by more than 2^8, so P stays <= 256 and rescales are rare), final 1/l and store.
+// TMEM: S0 | S1 | O  (128 + 128 + D fp32 columns).
+#include <cfloat>
+#include <cudaTypedefs.h>
+
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace tsv {
+
+namespace {
+
+constexpr int AT_BM = 128;     // queries per CTA
+constexpr int AT_BN = 128;     // keys per tile
+constexpr int AT_THREADS = 256;
+constexpr float RESCALE_THRESHOLD = 8.0f;  // log2 domain
+
+template <int D>
+struct AttnCfg {
+  static constexpr int NSUB = D / 64;                  // 64-wide sub-tiles of the head dim
+  static constexpr int Q_BYTES = AT_BM * D * 2;
+  static constexpr int KV_TILE = AT_BN * D * 2;         // one K (or V) tile
+  static constexpr int P_BYTES = AT_BM * AT_BN * 2;     // 2 sub-tiles of 64 keys
+  static constexpr int OFF_Q = 0;
+  static constexpr int OFF_K = OFF_Q + Q_BYTES;              // 2 stages
+  static constexpr int OFF_V = OFF_K + 2 * KV_TILE;          // 2 stages
+  static constexpr int OFF_P = OFF_V + 2 * KV_TILE;          // 2 buffers
+  static constexpr int OFF_BAR = OFF_P + 2 * P_BYTES;
+  static constexpr int SMEM = OFF_BAR + 256 + 1024;
+  static constexpr int TMEM_COLS = 512;
+  static constexpr int O_COL = 256;
+};
+
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], "
+      "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+      "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+      "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]), "r"(r[8]),
+      "r"(r[9]), "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15]), "r"(r[16]), "r"(r[17]),
+      "r"(r[18]), "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]), "r"(r[24]), "r"(r[25]), "r"(r[26]),
+      "r"(r[27]), "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31]));
+}
+__device__ __forceinline__ void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+
+// MN-major, 128B-swizzled B operand (rows = K, 64 N-elements per 128-byte row):
+// SBO = 1024 B between 8-row K atoms, LBO = byte distance between 64-wide N blocks.
+__device__ __forceinline__ uint64_t make_sw128_mn_desc(uint32_t smem_addr, uint32_t lbo_bytes) {
+  uint64_t lo = ((smem_addr & 0x3FFFFu) >> 4) | ((uint64_t)((lbo_bytes >> 4) & 0x3FFFu) << 16);
+  uint64_t hi = (1024u >> 4) | (1u << 14) | (2u << 29);
+  return lo | (hi << 32);
+}
+
+__host__ __device__ constexpr uint32_t make_idesc_bf16_bmn(int M, int N) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+
+}  // namespace
+
+template <int D>
+__global__ void __launch_bounds__(AT_THREADS, 1)
+    attention_tc_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
+                        const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
+                        float scale_log2) {
+  using C = AttnCfg<D>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
+  uint64_t* q_full = bars + 0;
+  uint64_t* kv_full = bars + 1;    // [2]
+  uint64_t* kv_empty = bars + 3;   // [2]
+  uint64_t* s_full = bars + 5;     // [2]
+  uint64_t* s_free = bars + 7;     // [2]
+  uint64_t* p_full = bars + 9;     // [2]
+  uint64_t* pv_done = bars + 11;   // [2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 14);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int head = blockIdx.y;
+  const int q0 = blockIdx.x * AT_BM;
+  const int n_tiles = (L + AT_BN - 1) / AT_BN;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmQ);
+    tma_prefetch_desc(&tmK);
+    tma_prefetch_desc(&tmV);
+    mbar_init(q_full, 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&kv_full[i], 1);
+      mbar_init(&kv_empty[i], 1);
+      mbar_init(&s_full[i], 1);
+      mbar_init(&s_free[i], 128);
+      mbar_init(&p_full[i], 128);
+      mbar_init(&pv_done[i], 1);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 2) tmem_alloc<C::TMEM_COLS>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // ---------------------------------------------------------------- producer
+      mbar_arrive_expect_tx(q_full, C::Q_BYTES);
+      for (int s = 0; s < C::NSUB; ++s)
+        tma_load_3d(&tmQ, q_full, sm + C::OFF_Q + s * (AT_BM * 128), s * 64, head, q0);
+      for (int j = 0; j < n_tiles; ++j) {
+        const int st = j & 1;
+        if (j >= 2) mbar_wait(&kv_empty[st], ((j - 2) >> 1) & 1);
+        mbar_arrive_expect_tx(&kv_full[st], 2 * C::KV_TILE);
+        for (int s = 0; s < C::NSUB; ++s) {
+          tma_load_3d(&tmK, &kv_full[st], sm + C::OFF_K + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
+                      j * AT_BN);
+          tma_load_3d(&tmV, &kv_full[st], sm + C::OFF_V + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
+                      j * AT_BN);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // ---------------------------------------------------------------- MMA issuer
+      constexpr uint32_t idesc_s = make_idesc_bf16(AT_BM, AT_BN);
+      constexpr uint32_t idesc_o = make_idesc_bf16_bmn(AT_BM, D);
+      const uint32_t sQ = smem_u32(sm + C::OFF_Q);
+      mbar_wait(q_full, 0);
+      auto issue_s = [&](int j) {
+        const int st = j & 1;
+        mbar_wait(&kv_full[st], (j >> 1) & 1);
+        if (j >= 2) mbar_wait(&s_free[st], ((j - 2) >> 1) & 1);
+        tc_fence_after();
+        const uint32_t sK = smem_u32(sm + C::OFF_K + st * C::KV_TILE);
+#pragma unroll
+        for (int kk = 0; kk < D / 16; ++kk) {
+          const uint32_t off = (kk >> 2) * (AT_BM * 128) + (kk & 3) * 32;
+          const uint32_t offk = (kk >> 2) * (AT_BN * 128) + (kk & 3) * 32;
+          umma_bf16_ss(tmem + st * 128, make_sw128_desc(sQ + off), make_sw128_desc(sK + offk), idesc_s, kk > 0);
+        }
+        umma_commit(&s_full[st]);
+      };
+      issue_s(0);
+      for (int j = 0; j < n_tiles; ++j) {
+        if (j + 1 < n_tiles) issue_s(j + 1);
+        const int st = j & 1;
+        mbar_wait(&p_full[st], (j >> 1) & 1);
+        tc_fence_after();
+        const uint32_t sP = smem_u32(sm + C::OFF_P + st * C::P_BYTES);
+        const uint32_t sV = smem_u32(sm + C::OFF_V + st * C::KV_TILE);
+#pragma unroll
+        for (int kk = 0; kk < AT_BN / 16; ++kk) {
+          const uint32_t offp = (kk >> 2) * (AT_BM * 128) + (kk & 3) * 32;
+          umma_bf16_ss(tmem + C::O_COL, make_sw128_desc(sP + offp),
+                       make_sw128_mn_desc(sV + kk * 2048, AT_BN * 128), idesc_o, (j | kk) != 0);
+        }
+        umma_commit(&pv_done[st]);
+        umma_commit(&kv_empty[st]);
+      }
+    }
+  } else if (warp >= 4) {
+    // ---------------------------------------------------------------- softmax (thread = query row)
+    const int wq = warp - 4;
+    const int row = wq * 32 + lane;
+    const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
+    float m_ref = -FLT_MAX, l_sum = 0.f;
+    for (int j = 0; j < n_tiles; ++j) {
+      const int st = j & 1;
+      mbar_wait(&s_full[st], (j >> 1) & 1);
+      tc_fence_after();
+      uint32_t sr[4][32];
+#pragma unroll
+      for (int c = 0; c < 4; ++c) tmem_ld32(tmem + lane_base + st * 128 + c * 32, sr[c]);
+      tmem_ld_wait();
+      tc_fence_before();
+      mbar_arrive(&s_free[st]);
+      const int kbase = j * AT_BN;
+      float mt = -FLT_MAX;
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int i = 0; i < 32; ++i) {
+          float x = __uint_as_float(sr[c][i]) * scale_log2;
+          if (kbase + c * 32 + i >= L) x = -INFINITY;
+          sr[c][i] = __float_as_uint(x);
+          mt = fmaxf(mt, x);
+        }
+      bool rescale = false;
+      float alpha = 1.f;
+      if (j == 0) {
+        m_ref = mt;
+      } else if (mt > m_ref + RESCALE_THRESHOLD) {
+        rescale = true;
+        alpha = exp2f(m_ref - mt);
+        m_ref = mt;
+      }
+      l_sum *= alpha;
+      // P = exp2(x - m_ref) -> bf16, packed in pairs
+      uint32_t pk[64];
+      float ls = 0.f;
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int i = 0; i < 32; i += 2) {
+          const float p0 = exp2f(__uint_as_float(sr[c][i]) - m_ref);
+          const float p1 = exp2f(__uint_as_float(sr[c][i + 1]) - m_ref);
+          ls += p0 + p1;
+          pk[c * 16 + i / 2] = pack_bf16x2(p0, p1);
+        }
+      l_sum += ls;
+      if (j >= 2) mbar_wait(&pv_done[st], ((j - 2) >> 1) & 1);  // P buffer st free
+      if (rescale) {
+        mbar_wait(&pv_done[st ^ 1], ((j - 1) >> 1) & 1);         // O holds tiles < j
+        tc_fence_after();
+#pragma unroll
+        for (int c = 0; c < D / 32; ++c) {
+          uint32_t ov[32];
+          tmem_ld32(tmem + lane_base + C::O_COL + c * 32, ov);
+          tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 32; ++i) ov[i] = __float_as_uint(__uint_as_float(ov[i]) * alpha);
+          tmem_st32(tmem + lane_base + C::O_COL + c * 32, ov);
+        }
+        tmem_st_wait();
+      }
+      // write P row into the K-major SW128 tile: sub-tile t (keys 64t..), atom row/8, chunk ^ (row & 7)
+      uint8_t* pbase = sm + C::OFF_P + st * C::P_BYTES + (row >> 3) * 1024 + (row & 7) * 128;
+#pragma unroll
+      for (int t = 0; t < 2; ++t)
+#pragma unroll
+        for (int ch = 0; ch < 8; ++ch) {
+          const int q = t * 32 + ch * 4;  // index into pk (pairs)
+          uint4 v = make_uint4(pk[q], pk[q + 1], pk[q + 2], pk[q + 3]);
+          *reinterpret_cast<uint4*>(pbase + t * (AT_BM * 128) + ((ch ^ (row & 7)) << 4)) = v;
+        }
+      fence_proxy_async();
+      tc_fence_before();
+      mbar_arrive(&p_full[st]);
+    }
+    // epilogue: O / l -> bf16
+    const int jl = n_tiles - 1;
+    mbar_wait(&pv_done[jl & 1], (jl >> 1) & 1);
+    tc_fence_after();
+    const float inv = 1.f / l_sum;
+    const int grow = q0 + row;
+#pragma unroll
+    for (int c = 0; c < D / 32; ++c) {
+      uint32_t ov[32];
+      tmem_ld32(tmem + lane_base + C::O_COL + c * 32, ov);
+      tmem_ld_wait();
+      if (grow < L) {
+        uint4* dst = reinterpret_cast<uint4*>(o + (long long)grow * ldo + head * D + c * 32);
+#pragma unroll
+        for (int qd = 0; qd < 4; ++qd) {
+          uint4 v;
+          v.x = pack_bf16x2(__uint_as_float(ov[qd * 8 + 0]) * inv, __uint_as_float(ov[qd * 8 + 1]) * inv);
+          v.y = pack_bf16x2(__uint_as_float(ov[qd * 8 + 2]) * inv, __uint_as_float(ov[qd * 8 + 3]) * inv);
+          v.z = pack_bf16x2(__uint_as_float(ov[qd * 8 + 4]) * inv, __uint_as_float(ov[qd * 8 + 5]) * inv);
+          v.w = pack_bf16x2(__uint_as_float(ov[qd * 8 + 6]) * inv, __uint_as_float(ov[qd * 8 + 7]) * inv);
+          dst[qd] = v;
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 2) tmem_dealloc<C::TMEM_COLS>(tmem);
+}
+
+// ------------------------------------------------------------------ host
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    cudaDriverEntryPointQueryResult q;
+    void* p = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  }
+  return fn;
+}
+
+// [rows][heads][D] view of a strided activation: element (r, h, d) at base + r*ld + h*D + d
+static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L, long long ld) {
+  auto enc = encode_fn();
+  if (!enc) return -1;
+  cuuint64_t dims[3] = {(cuuint64_t)D, (cuuint64_t)H, (cuuint64_t)L};
+  cuuint64_t strides[2] = {(cuuint64_t)D * 2, (cuuint64_t)ld * 2};
+  cuuint32_t box[3] = {64, 1, 128};
+  cuuint32_t es[3] = {1, 1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(base), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? 0 : -2;
+}
+
+template <int D>
+static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv, bf16* o,
+                     long long ldo, int L, int H, cudaStream_t s) {
+  using C = AttnCfg<D>;
+  CUtensorMap tq, tk, tv;
+  if (make_tmap_heads(&tq, q, D, H, L, ldq) || make_tmap_heads(&tk, k, D, H, L, ldk) ||
+      make_tmap_heads(&tv, v, D, H, L, ldv))
+    return -1;
+  static unsigned long long done = 0;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!(done >> dev & 1ull)) {
+    cudaFuncSetAttribute(attention_tc_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+    done |= 1ull << dev;
+  }
+  const float scale_log2 = (1.0f / sqrtf((float)D)) * 1.4426950408889634f;
+  dim3 grid((L + AT_BM - 1) / AT_BM, H);
+  attention_tc_kernel<D><<<grid, AT_THREADS, C::SMEM, s>>>(tq, tk, tv, o, ldo, L, scale_log2);
+  return 0;
+}
+
+// returns 0 if the tensor-core path was launched, nonzero if the layout is unsupported by TMA
+int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
+                        bf16* o, long long ldo, int L, int H, int D, cudaStream_t s) {
+  if (L <= 0 || H <= 0) return 0;
+  if (((ldq | ldk | ldv) * 2) % 16 || ((reinterpret_cast<uintptr_t>(q) | reinterpret_cast<uintptr_t>(k) |
+                                        reinterpret_cast<uintptr_t>(v)) & 15))
+    return -1;
+  if (D == 128) return launch_tc<128>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, s);
+  if (D == 64) return launch_tc<64>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, s);
+  return -1;
+}
+
+}  // namespace tsv

@@ -570,14 +570,16 @@ static tsv_status attention_all(StepEnv& E) {
     CK(cudaSetDevice(c.s->device));
     const double Lq = k == 1 ? (double)c.rows : (double)L;
     ProfScope ps(e, *c.s, KC_ATTN, 4.0 * Lq * Lq * m.D * (m.H / k), 8.0 * Lq * m.D * (m.H / k));
+    int rc;
     if (k == 1) {
-      attention_launch(c.qkv, 3 * m.h, c.qkv + m.h, 3 * m.h, c.qkv + 2 * m.h, 3 * m.h, c.cat, m.h + m.F, (int)c.rows,
-                       m.H, m.D, c.s->stream);
+      rc = attention_launch(c.qkv, 3 * m.h, c.qkv + m.h, 3 * m.h, c.qkv + 2 * m.h, 3 * m.h, c.cat, m.h + m.F,
+                            (int)c.rows, m.H, m.D, c.s->stream);
     } else {
       const int64_t w = 3 * (int64_t)m.h / k;
-      attention_launch(c.recv, w, c.recv + m.h / k, w, c.recv + 2 * m.h / k, w, c.obuf, m.h / k, (int)L, m.H / k,
-                       m.D, c.s->stream);
+      rc = attention_launch(c.recv, w, c.recv + m.h / k, w, c.recv + 2 * m.h / k, w, c.obuf, m.h / k, (int)L,
+                            m.H / k, m.D, c.s->stream);
     }
+    if (rc) return fail(TSV_E_CUDA, "attention: tensor map creation failed");
   }
   return TSV_OK;
 }
@@ -1415,11 +1417,17 @@ tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int
 }
 
 tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
-                            void* o, int64_t ldo, int L, int H, int D, void* stream) {
+                            void* o, int64_t ldo, int L, int H, int D, int impl, void* stream) {
   if (D != 64 && D != 128) return fail(TSV_E_INVAL, "D must be 64 or 128");
-  attention_launch(reinterpret_cast<const bf16*>(q), ldq, reinterpret_cast<const bf16*>(k), ldk,
-                   reinterpret_cast<const bf16*>(v), ldv, reinterpret_cast<bf16*>(o), ldo, L, H, D,
-                   reinterpret_cast<cudaStream_t>(stream));
+  if (impl == 1) {
+    attention_mma_launch(reinterpret_cast<const bf16*>(q), ldq, reinterpret_cast<const bf16*>(k), ldk,
+                         reinterpret_cast<const bf16*>(v), ldv, reinterpret_cast<bf16*>(o), ldo, L, H, D,
+                         reinterpret_cast<cudaStream_t>(stream));
+  } else if (attention_launch(reinterpret_cast<const bf16*>(q), ldq, reinterpret_cast<const bf16*>(k), ldk,
+                              reinterpret_cast<const bf16*>(v), ldv, reinterpret_cast<bf16*>(o), ldo, L, H, D,
+                              reinterpret_cast<cudaStream_t>(stream))) {
+    return fail(TSV_E_INVAL, "attention: operands must be 16-byte aligned with 16-byte row strides");
+  }
   CK(cudaGetLastError());
   return TSV_OK;
 }

@@ -64,9 +64,13 @@ void qk_norm_rope_launch(bf16* qkv, long long ld, int rows, int n_first, int H, 
                          bf16* pack_out, int k_sp, cudaStream_t s);
 
 // Joint attention, non-causal: O[l, h*D + d] = softmax(q k^T / sqrt(D)) v for heads h in [0, H).
+// attention_launch: tcgen05/TMEM kernel (returns nonzero if the layout is not TMA-compatible).
+// attention_mma_launch: the mma.sync (FA2-style) baseline kept for comparison.
 // q(l, h) at q + l*ldq + h*D (same for k, v, o). L rows.
-void attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
-                      bf16* o, long long ldo, int L, int H, int D, cudaStream_t s);
+int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
+                     bf16* o, long long ldo, int L, int H, int D, cudaStream_t s);
+void attention_mma_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
+                          bf16* o, long long ldo, int L, int H, int D, cudaStream_t s);
 
 // dst[m, c] = bf16(src[m, c]) (fp32 -> bf16), row strides in elements
 void f32_to_bf16_launch(const float* src, long long lds, bf16* dst, long long ldd, int M, int C, cudaStream_t s);

@@ -207,9 +207,10 @@ def test_qk_norm_rope(tsv, H, D, rows, n_first):
 
 
 # ----------------------------------------------------------------------------- attention
+@pytest.mark.parametrize("impl", [0, 1])
 @pytest.mark.parametrize("L,H,D", [(1, 2, 64), (63, 4, 64), (320, 4, 64), (1000, 3, 128), (1536, 2, 128),
                                    (4700, 1, 128)])
-def test_attention(tsv, L, H, D):
+def test_attention(tsv, L, H, D, impl):
     rng = np.random.default_rng(L + H + D)
     qkv = rng.standard_normal((L, 3, H, D)).astype(np.float32) * np.float32(1.5)
     qkv = synth.bf16_bits_to_f32(synth.bf16_rne_bits(qkv)).astype(np.float64)
@@ -217,7 +218,7 @@ def test_attention(tsv, L, H, D):
     t = _bf16(qkv.reshape(L, 3 * H * D))
     o = torch.zeros(L, 2 * H * D, dtype=torch.bfloat16, device="cuda")   # strided output (row stride 2HD)
     ld = 3 * H * D
-    tsv.op_attention(t, t[:, H * D:], t[:, 2 * H * D:], o, L, H, D, ldq=ld, ldk=ld, ldv=ld)
+    tsv.op_attention(t, t[:, H * D:], t[:, 2 * H * D:], o, L, H, D, ldq=ld, ldk=ld, ldv=ld, impl=impl)
     torch.cuda.synchronize()
     got = _np(o)[:, :H * D].reshape(L, H, D)
     assert _rel(got, ref) < 1.5e-2
@@ -239,3 +240,21 @@ def test_attention_special_cases(tsv):
     torch.cuda.synchronize()
     ref = np.repeat(v.mean(axis=0, keepdims=True), L, axis=0)
     assert np.max(np.abs(_np(o).reshape(L, H, D) - ref)) < 2e-2
+
+
+def test_attention_rescale_path(tsv):
+    """Scores growing along the key axis force the conditional O rescale (max grows by > 2^8)."""
+    L, H, D = 700, 1, 128
+    rng = np.random.default_rng(9)
+    q = np.ones((L, H, D)) * 0.5
+    k = rng.standard_normal((L, H, D)) * 0.1 + np.linspace(0, 3, L)[:, None, None]
+    v = rng.standard_normal((L, H, D))
+    ref = F.attention(q, k, v)
+    o = torch.zeros(L, H * D, dtype=torch.bfloat16, device="cuda")
+    tsv.op_attention(_bf16(q.reshape(L, -1)), _bf16(k.reshape(L, -1)), _bf16(v.reshape(L, -1)), o, L, H, D)
+    torch.cuda.synchronize()
+    # compare against the oracle on the bf16-rounded inputs
+    qb, kb, vb = (synth.bf16_bits_to_f32(synth.bf16_rne_bits(a.astype(np.float32))).astype(np.float64)
+                  for a in (q, k, v))
+    ref = F.attention(qb, kb, vb)
+    assert _rel(_np(o).reshape(L, H, D), ref) < 2e-2

@@ -1,0 +1,86 @@
+"""Kernel micro-benchmarks through the kernel-level C-ABI (CUDA events, warm, L2-resident inputs
+unless stated).  Prints one JSON line per case.
+
+  python tools/microbench.py [gemm] [attn] [ln] [qk]
+"""
+import json
+import math
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch  # noqa: E402
+
+import paper_conf_asplos_luhtlwm0c26_b200 as tsv  # noqa: E402
+
+
+def timeit(fn, iters=20, warm=3):
+    for _ in range(warm):
+        fn()
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    s.record()
+    for _ in range(iters):
+        fn()
+    e.record()
+    torch.cuda.synchronize()
+    return s.elapsed_time(e) / iters
+
+
+def gemm_cases():
+    # FLUX 512^2 (M = 1024 img / 512 txt / 1536 joint) and 2048^2 k=8 shapes
+    shapes = [(1024, 9216, 3072), (512, 9216, 3072), (1024, 3072, 3072), (1024, 12288, 3072), (1024, 3072, 12288),
+              (1536, 21504, 3072), (1536, 3072, 15360), (4096, 12288, 3072), (8192, 3072, 12288)]
+    for M, N, K in shapes:
+        A = torch.randn(M, K, device="cuda").to(torch.bfloat16)
+        W = (torch.randn(N, K, device="cuda") / math.sqrt(K)).to(torch.bfloat16)
+        o = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
+        for bn in (0, 64, 128, 256):
+            if N % (bn or 64):
+                continue
+            ms = timeit(lambda: tsv.op_gemm(A, W, "STORE_BF16", o, force_bn=bn))
+            print(json.dumps({"op": "gemm", "M": M, "N": N, "K": K, "bn": bn, "ms": round(ms, 4),
+                              "tflops": round(2 * M * N * K / ms / 1e9, 1)}), flush=True)
+        ref = timeit(lambda: torch.matmul(A, W.t(), out=o))
+        print(json.dumps({"op": "gemm_cublas_ref", "M": M, "N": N, "K": K, "ms": round(ref, 4),
+                          "tflops": round(2 * M * N * K / ref / 1e9, 1)}), flush=True)
+
+
+def attn_cases():
+    for L, H, D in ((1536, 24, 128), (4608, 24, 128), (16896, 24, 128), (16896, 3, 128), (4608, 24, 64)):
+        qkv = torch.randn(L, 3 * H * D, device="cuda").to(torch.bfloat16)
+        o = torch.empty(L, H * D, dtype=torch.bfloat16, device="cuda")
+        ld = 3 * H * D
+        for impl in (0, 1):
+            f = lambda: tsv.op_attention(qkv, qkv[:, H * D:], qkv[:, 2 * H * D:], o, L, H, D, ldq=ld, ldk=ld,
+                                         ldv=ld, impl=impl)
+            ms = timeit(f, iters=5 if L > 8000 else 20)
+            print(json.dumps({"op": "attention", "impl": ["tcgen05", "mma.sync"][impl], "L": L, "H": H, "D": D,
+                              "ms": round(ms, 4), "tflops": round(4 * L * L * D * H / ms / 1e9, 1)}), flush=True)
+
+
+def ln_cases():
+    for M, h in ((1024, 3072), (1536, 3072), (16896, 3072)):
+        x = torch.randn(M, h, device="cuda")
+        u = torch.empty(M, h, dtype=torch.bfloat16, device="cuda")
+        sh, sc = torch.randn(h, device="cuda"), torch.randn(h, device="cuda")
+        ms = timeit(lambda: tsv.op_ln_mod(x, u, sh, sc))
+        print(json.dumps({"op": "ln_mod", "M": M, "h": h, "ms": round(ms, 4),
+                          "GBps": round(M * h * 6 / ms / 1e6, 1)}), flush=True)
+
+
+def qk_cases():
+    for rows, H, D in ((1536, 24, 128), (16896, 24, 128)):
+        qkv = torch.randn(rows, 3 * H * D, device="cuda").to(torch.bfloat16)
+        g = torch.ones(D, device="cuda").to(torch.bfloat16)
+        cs = torch.randn(rows, D // 2, device="cuda")
+        ms = timeit(lambda: tsv.op_qk_norm_rope(qkv, 0, H, D, g, g, g, g, cs, cs))
+        print(json.dumps({"op": "qk_norm_rope", "rows": rows, "ms": round(ms, 4),
+                          "GBps": round(rows * H * D * 8 / ms / 1e6, 1)}), flush=True)
+
+
+if __name__ == "__main__":
+    which = sys.argv[1:] or ["gemm", "attn", "ln", "qk"]
+    for w in which:
+        {"gemm": gemm_cases, "attn": attn_cases, "ln": ln_cases, "qk": qk_cases}[w]()
