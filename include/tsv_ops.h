@@ -37,6 +37,16 @@ tsv_status tsv_op_gemm(const void* A, int64_t lda, const void* W, int64_t ldw, i
                        void* out0, int64_t ld0, void* out1, int64_t ld1, int n_split, const void* bias,
                        const float* gate, const float* scalar, int force_bn, void* stream);
 
+/* a3 + a4 fused (the step's QKV / linear1 GEMM): y = A W^T + bias with columns "(K H D)" =
+ * [q | k | v] over [0, 3h) (+ GELU columns >= 3h into out1 when mode = TSV_EPI_SPLIT_GELU,
+ * n_split = 3h).  q and k heads become RoPE(RMSNorm(y) * g) (eps 1e-6; gq/gk bf16 [D]; cos/sin fp32
+ * [M][D/2] indexed by GEMM row); v passes through.  k_sp = 1: written to out0 [M, ld0];
+ * k_sp > 1: written to pack laid out [k_sp][pack_rows][3][H/k_sp][D] at row pack_row0 + m. */
+tsv_status tsv_op_gemm_qkv(const void* A, int64_t lda, const void* W, int64_t ldw, int M, int N, int K, int mode,
+                           void* out0, int64_t ld0, void* out1, int64_t ld1, const void* bias, int h, int D,
+                           const void* gq, const void* gk, const float* cosb, const float* sinb, int k_sp,
+                           void* pack, int pack_rows, int pack_row0, void* stream);
+
 /* a2: u[m, :] = bf16(LN(x[m, :]) * (1 + scale) + shift); x fp32, LN without affine, eps 1e-6. */
 tsv_status tsv_op_ln_mod(const float* x, int64_t ldx, void* u, int64_t ldu, const float* shift,
                          const float* scale, int M, int h, void* stream);

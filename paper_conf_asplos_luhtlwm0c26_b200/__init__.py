@@ -218,6 +218,16 @@ def op_gemm(A, W, mode, out0, out1=None, bias=None, gate=None, scalar=None, n_sp
                           _stream(stream)))
 
 
+def op_gemm_qkv(A, W, out0, h, D, gq, gk, cosb, sinb, bias=None, mode="STORE_BF16", out1=None, ld1=None,
+                k_sp=1, pack=None, pack_rows=0, pack_row0=0, stream=None):
+    M, K = A.shape
+    N = W.shape[0]
+    check(lib.tsv_op_gemm_qkv(_ptr(A), A.stride(0), _ptr(W), W.stride(0), M, N, K, EPI[mode], _ptr(out0),
+                              out0.stride(0), _ptr(out1), (ld1 or (out1.stride(0) if out1 is not None else 0)),
+                              _ptr(bias), h, D, _ptr(gq), _ptr(gk), _ptr(cosb), _ptr(sinb), k_sp, _ptr(pack),
+                              pack_rows, pack_row0, _stream(stream)))
+
+
 def op_ln_mod(x, u, shift, scale, stream=None):
     M, h = x.shape
     check(lib.tsv_op_ln_mod(_ptr(x), x.stride(0), _ptr(u), u.stride(0), _ptr(shift), _ptr(scale), M, h,

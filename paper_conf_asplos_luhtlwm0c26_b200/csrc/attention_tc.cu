@@ -221,7 +221,9 @@ __global__ void __launch_bounds__(AT_THREADS, 1)
         }
       l_sum += ls;
       if (j >= 2) mbar_wait(&pv_done[st], ((j - 2) >> 1) & 1);  // P buffer st free
-      if (rescale) {
+      // tcgen05.ld/st are warp-collective (.sync.aligned): rescale the whole warp's rows together
+      // (alpha = 1 for rows that did not need it).
+      if (__any_sync(0xffffffffu, rescale)) {
         mbar_wait(&pv_done[st ^ 1], ((j - 1) >> 1) & 1);         // O holds tiles < j
         tc_fence_after();
 #pragma unroll

@@ -7,40 +7,53 @@ namespace tsv {
 
 // ------------------------------------------------------------------ a2: LN-modulate
 // u = LN(x) (no affine, biased variance, eps 1e-6) * (1 + scale) + shift   -> bf16
-template <int NV>  // float4 per lane: h = 128 * NV
-__global__ void __launch_bounds__(256) ln_mod_kernel(const float* __restrict__ x, long long ldx, bf16* __restrict__ u,
-                                                     long long ldu, const float* __restrict__ shift,
-                                                     const float* __restrict__ scale, int M) {
-  const int row = blockIdx.x * 8 + (threadIdx.x >> 5);
-  const int lane = threadIdx.x & 31;
-  if (row >= M) return;
-  constexpr int h = 128 * NV;
+// One CTA of T threads per row, NV float4 per thread (h = 4 * T * NV): the row stays in registers,
+// two block reductions (mean, then centred sum of squares), ~10 CTAs resident per SM.
+template <int T>
+__device__ __forceinline__ float block_sum(float v, float* red) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  if (T == 32) return v;
+  const int w = threadIdx.x >> 5;
+  __syncthreads();  // red[] reuse
+  if ((threadIdx.x & 31) == 0) red[w] = v;
+  __syncthreads();
+  float s = 0.f;
+#pragma unroll
+  for (int i = 0; i < T / 32; ++i) s += red[i];
+  return s;
+}
+
+template <int T, int NV>
+__global__ void __launch_bounds__(T) ln_mod_kernel(const float* __restrict__ x, long long ldx, bf16* __restrict__ u,
+                                                   long long ldu, const float* __restrict__ shift,
+                                                   const float* __restrict__ scale, int M) {
+  __shared__ float red[T / 32];
+  const int row = blockIdx.x;
+  const int t = threadIdx.x;
+  constexpr int h = 4 * T * NV;
   const float4* xr = reinterpret_cast<const float4*>(x + (long long)row * ldx);
   float4 v[NV];
   float s = 0.f;
 #pragma unroll
   for (int i = 0; i < NV; ++i) {
-    v[i] = __ldcs(xr + i * 32 + lane);
+    v[i] = xr[i * T + t];
     s += (v[i].x + v[i].y) + (v[i].z + v[i].w);
   }
-#pragma unroll
-  for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-  const float mean = s * (1.0f / h);
+  const float mean = block_sum<T>(s, red) * (1.0f / h);
   float q = 0.f;
 #pragma unroll
   for (int i = 0; i < NV; ++i) {
     float a = v[i].x - mean, b = v[i].y - mean, c = v[i].z - mean, d = v[i].w - mean;
     q += (a * a + b * b) + (c * c + d * d);
   }
-#pragma unroll
-  for (int o = 16; o; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
-  const float rstd = rsqrtf(q * (1.0f / h) + 1e-6f);
+  const float rstd = rsqrtf(block_sum<T>(q, red) * (1.0f / h) + 1e-6f);
   uint2* ur = reinterpret_cast<uint2*>(u + (long long)row * ldu);
   const float4* sh4 = reinterpret_cast<const float4*>(shift);
   const float4* sc4 = reinterpret_cast<const float4*>(scale);
 #pragma unroll
   for (int i = 0; i < NV; ++i) {
-    const int c = i * 32 + lane;
+    const int c = i * T + t;
     float4 sh = __ldg(sh4 + c), sc = __ldg(sc4 + c);
     float a = (v[i].x - mean) * rstd * (1.f + sc.x) + sh.x;
     float b = (v[i].y - mean) * rstd * (1.f + sc.y) + sh.y;
@@ -73,12 +86,11 @@ __global__ void __launch_bounds__(256) ln_mod_generic(const float* __restrict__ 
 void ln_mod_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift, const float* scale,
                    int M, int h, cudaStream_t s) {
   if (M <= 0) return;
-  dim3 grid((M + 7) / 8);
   switch (h) {
-    case 3072: ln_mod_kernel<24><<<grid, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
-    case 1536: ln_mod_kernel<12><<<grid, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
-    case 256: ln_mod_kernel<2><<<grid, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
-    default: ln_mod_generic<<<grid, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M, h); break;
+    case 3072: ln_mod_kernel<128, 6><<<M, 128, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
+    case 1536: ln_mod_kernel<128, 3><<<M, 128, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
+    case 256: ln_mod_kernel<32, 2><<<M, 32, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
+    default: ln_mod_generic<<<(M + 7) / 8, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M, h); break;
   }
 }
 

@@ -264,6 +264,28 @@ static tsv_status gemm(tsv_engine* e, Slot& s, const bf16* A, long long lda, con
   gemm_launch(p, s.stream);
   return TSV_OK;
 }
+// Up to two problems with the same N, K in one persistent launch (the img and txt streams of a
+// double block): better wave quantization than two launches of half the tiles each.
+static tsv_status gemm_multi(tsv_engine* e, Slot& s, const GemmProblem* probs, int np, int N, int K) {
+  GemmProblem nz[2];
+  int n = 0;
+  for (int i = 0; i < np; ++i)
+    if (probs[i].M > 0) nz[n++] = probs[i];
+  if (!n) return TSV_OK;
+  GemmPlan p;
+  const char* err = nullptr;
+  if (gemm_plan_multi(&p, nz, n, N, K, s.ds->num_sms, &err))
+    return fail(TSV_E_INVAL, "%s (N=%d K=%d)", err, N, K);
+  double fl = 0, by = 2.0 * N * K * n;
+  for (int i = 0; i < n; ++i) {
+    const double out_b = (nz[i].epi.mode <= EPI_SPLIT_GELU) ? 2.0 : (nz[i].epi.mode == EPI_STORE_F32 ? 4.0 : 8.0);
+    fl += 2.0 * nz[i].M * N * (double)K;
+    by += 2.0 * nz[i].M * K + out_b * nz[i].M * N;
+  }
+  ProfScope ps(e, s, KC_GEMM, fl, by);
+  gemm_launch(p, s.stream);
+  return TSV_OK;
+}
 static void lnmod(tsv_engine* e, Slot& s, const float* x, bf16* u, const float* shift, const float* scale, int n) {
   const int h = e->model.h;
   ProfScope ps(e, s, KC_LNMOD, 0.0, (double)n * h * 6.0 + 8.0 * h);
@@ -584,15 +606,21 @@ static tsv_status attention_all(StepEnv& E) {
   return TSV_OK;
 }
 
-// QK-RMSNorm + RoPE on the local qkv rows (in place for k = 1, into the send buffer for k > 1)
-static void qk_rope(StepEnv& E, RankCtx& c, const bf16* gq0, const bf16* gk0, const bf16* gq1, const bf16* gk1) {
+// a4 fused into the QKV GEMM epilogue: QK-RMSNorm + RoPE on rows [r0, r0 + n) of this rank, written
+// in place (k = 1) or straight into the Ulysses send buffer (k > 1).
+static GemmEpi qk_fused(StepEnv& E, RankCtx& c, GemmEpi epi, int64_t r0, const bf16* gq, const bf16* gk) {
   const Model& m = E.e->model;
-  const int k = E.g->k;
-  ProfScope ps(E.e, *c.s, KC_QKROPE, 0.0,
-               (double)c.rows * m.H * m.D * (k > 1 ? 12.0 : 8.0) + (double)c.rows * m.D * 4.0);
-  qk_norm_rope_launch(c.qkv, 3 * m.h, (int)c.rows, (int)c.nt, m.H, m.D, gq0, gk0, gq1, gk1,
-                      reinterpret_cast<const float*>(c.sh->cosb.p), reinterpret_cast<const float*>(c.sh->sinb.p),
-                      k > 1 ? c.pack : nullptr, k, c.s->stream);
+  epi.qk_h = m.h;
+  epi.qk_D = m.D;
+  epi.gq = gq;
+  epi.gk = gk;
+  epi.cosb = reinterpret_cast<const float*>(c.sh->cosb.p) + r0 * (m.D / 2);
+  epi.sinb = reinterpret_cast<const float*>(c.sh->sinb.p) + r0 * (m.D / 2);
+  epi.k_sp = E.g->k;
+  epi.pack = E.g->k > 1 ? c.pack : nullptr;
+  epi.pack_rows = (int)c.rows;
+  epi.pack_row0 = (int)r0;
+  return epi;
 }
 
 static tsv_status run_step(StepEnv& E) {
@@ -621,17 +649,17 @@ static tsv_status run_step(StepEnv& E) {
     for (auto& c : E.rc) {
       Slot& s = *c.s;
       CK(cudaSetDevice(s.device));
+      GemmProblem pq[2];
       for (int st = 0; st < 2; ++st) {  // 0 = img, 1 = txt
         const int base = double_base(j, st);
         const int64_t r0 = st == 0 ? c.nt : 0, n = st == 0 ? c.ni : c.nt;
-        if (!n) continue;
         const float* md = c.mod + m.mod_double(j, st);
-        lnmod(e, s, c.x + r0 * h, c.u + r0 * h, md + 0 * h, md + 1 * h, (int)n);
-        TRY(gemm(e, s, c.u + r0 * h, h, e->W(s, base + 2), h, (int)n, 3 * h, h,
-                 epi_of(EPI_STORE_BF16, c.qkv + r0 * 3 * h, 3 * h, e->W(s, base + 3))));
+        if (n) lnmod(e, s, c.x + r0 * h, c.u + r0 * h, md + 0 * h, md + 1 * h, (int)n);
+        pq[st] = {c.u + r0 * h, h, e->W(s, base + 2), h, (int)n,
+                  qk_fused(E, c, epi_of(EPI_STORE_BF16, c.qkv + r0 * 3 * h, 3 * h, e->W(s, base + 3)), r0,
+                           e->W(s, base + 4), e->W(s, base + 5))};
       }
-      qk_rope(E, c, e->W(s, double_base(j, 1) + 4), e->W(s, double_base(j, 1) + 5), e->W(s, double_base(j, 0) + 4),
-              e->W(s, double_base(j, 0) + 5));
+      TRY(gemm_multi(e, s, pq, 2, 3 * h, h));   // a3 + a4 for both streams in one launch
     }
     if (E.g->k > 1) TRY(a2a_qkv(E));
     TRY(attention_all(E));
@@ -639,20 +667,27 @@ static tsv_status run_step(StepEnv& E) {
     for (auto& c : E.rc) {
       Slot& s = *c.s;
       CK(cudaSetDevice(s.device));
+      GemmProblem pp[2], p1[2], p2[2];
       for (int st = 0; st < 2; ++st) {
         const int base = double_base(j, st);
         const int64_t r0 = st == 0 ? c.nt : 0, n = st == 0 ? c.ni : c.nt;
-        if (!n) continue;
         const float* md = c.mod + m.mod_double(j, st);
         float* x = c.x + r0 * h;
-        TRY(gemm(e, s, c.cat + r0 * ldc, ldc, e->W(s, base + 6), h, (int)n, h, h,
-                 epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 7), md + 2 * h)));
-        lnmod(e, s, x, c.u + r0 * h, md + 3 * h, md + 4 * h, (int)n);
-        TRY(gemm(e, s, c.u + r0 * h, h, e->W(s, base + 8), h, (int)n, F, h,
-                 epi_of(EPI_GELU_BF16, c.hbuf + r0 * F, F, e->W(s, base + 9))));
-        TRY(gemm(e, s, c.hbuf + r0 * F, F, e->W(s, base + 10), F, (int)n, h, F,
-                 epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 11), md + 5 * h)));
+        pp[st] = {c.cat + r0 * ldc, ldc, e->W(s, base + 6), h, (int)n,
+                  epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 7), md + 2 * h)};
+        p1[st] = {c.u + r0 * h, h, e->W(s, base + 8), h, (int)n,
+                  epi_of(EPI_GELU_BF16, c.hbuf + r0 * F, F, e->W(s, base + 9))};
+        p2[st] = {c.hbuf + r0 * F, F, e->W(s, base + 10), F, (int)n,
+                  epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 11), md + 5 * h)};
       }
+      TRY(gemm_multi(e, s, pp, 2, h, h));        // a8: out-proj + gated residual, both streams
+      for (int st = 0; st < 2; ++st) {           // a9: LN-modulate both streams
+        const int64_t r0 = st == 0 ? c.nt : 0, n = st == 0 ? c.ni : c.nt;
+        const float* md = c.mod + m.mod_double(j, st);
+        if (n) lnmod(e, s, c.x + r0 * h, c.u + r0 * h, md + 3 * h, md + 4 * h, (int)n);
+      }
+      TRY(gemm_multi(e, s, p1, 2, F, h));        // fc1 + GELU
+      TRY(gemm_multi(e, s, p2, 2, h, F));        // fc2 + gated residual
     }
   }
   // single-stream blocks on x = [txt; img] (zero-copy join, a10)
@@ -665,8 +700,8 @@ static tsv_status run_step(StepEnv& E) {
       const float* md = c.mod + m.mod_single(j);
       lnmod(e, s, c.x, c.u, md, md + h, (int)c.rows);
       TRY(gemm(e, s, c.u, h, e->W(s, base + 2), h, (int)c.rows, 3 * h + F, h,
-               epi_of(EPI_SPLIT_GELU, c.qkv, 3 * h, e->W(s, base + 3), nullptr, c.cat + h, ldc, 3 * h)));
-      qk_rope(E, c, e->W(s, base + 4), e->W(s, base + 5), e->W(s, base + 4), e->W(s, base + 5));
+               qk_fused(E, c, epi_of(EPI_SPLIT_GELU, c.qkv, 3 * h, e->W(s, base + 3), nullptr, c.cat + h, ldc, 3 * h),
+                        0, e->W(s, base + 4), e->W(s, base + 5))));
     }
     if (E.g->k > 1) TRY(a2a_qkv(E));
     TRY(attention_all(E));
@@ -1389,6 +1424,36 @@ tsv_status tsv_op_gemm(const void* A, int64_t lda, const void* Wt, int64_t ldw, 
   GemmEpi epi = epi_of(mode, out0, ld0, reinterpret_cast<const bf16*>(bias), gate, out1, ld1, n_split, scalar);
   if (gemm_plan(&p, reinterpret_cast<const bf16*>(A), lda, reinterpret_cast<const bf16*>(Wt), ldw, M, N, K, epi, sms,
                 &err, force_bn))
+    return fail(TSV_E_INVAL, "%s", err);
+  gemm_launch(p, reinterpret_cast<cudaStream_t>(stream));
+  CK(cudaGetLastError());
+  return TSV_OK;
+}
+
+tsv_status tsv_op_gemm_qkv(const void* A, int64_t lda, const void* Wt, int64_t ldw, int M, int N, int K, int mode,
+                           void* out0, int64_t ld0, void* out1, int64_t ld1, const void* bias, int h, int D,
+                           const void* gq, const void* gk, const float* cosb, const float* sinb, int k_sp,
+                           void* pack, int pack_rows, int pack_row0, void* stream) {
+  if (mode != EPI_STORE_BF16 && mode != EPI_SPLIT_GELU) return fail(TSV_E_INVAL, "mode must be STORE_BF16 or SPLIT_GELU");
+  int dev = 0, sms = 148;
+  CK(cudaGetDevice(&dev));
+  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  GemmEpi epi = epi_of(mode, out0, ld0, reinterpret_cast<const bf16*>(bias), nullptr, out1, ld1,
+                       mode == EPI_SPLIT_GELU ? 3 * h : 0, nullptr);
+  epi.qk_h = h;
+  epi.qk_D = D;
+  epi.gq = reinterpret_cast<const bf16*>(gq);
+  epi.gk = reinterpret_cast<const bf16*>(gk);
+  epi.cosb = cosb;
+  epi.sinb = sinb;
+  epi.k_sp = k_sp;
+  epi.pack = reinterpret_cast<bf16*>(pack);
+  epi.pack_rows = pack_rows;
+  epi.pack_row0 = pack_row0;
+  GemmPlan p;
+  const char* err = nullptr;
+  if (gemm_plan(&p, reinterpret_cast<const bf16*>(A), lda, reinterpret_cast<const bf16*>(Wt), ldw, M, N, K, epi, sms,
+                &err, 0))
     return fail(TSV_E_INVAL, "%s", err);
   gemm_launch(p, reinterpret_cast<cudaStream_t>(stream));
   CK(cudaGetLastError());

@@ -33,15 +33,115 @@ struct GemmCfg {
   static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
 };
 
+// Up to two problems with the same N and K (e.g. the img and txt streams of a double block)
+// share one persistent launch: tiles [0, tile0[1]) belong to problem 0, the rest to problem 1.
 struct GemmArgs {
-  int M, N, K;
-  int num_m, num_n, num_tiles;
-  GemmEpi epi;
+  int N, K, num_n, num_tiles, nprob;
+  int M[2], num_m[2], tile0[2];
+  GemmEpi epi[2];
+};
+struct GemmMaps {
+  CUtensorMap A[2];
+  CUtensorMap B[2];
 };
 
-template <int BN>
-__device__ __forceinline__ void epilogue_chunk(const GemmArgs& a, int row, int n0, const uint32_t (&r)[32]) {
-  const GemmEpi& e = a.epi;
+__device__ __forceinline__ void decode_tile(const GemmArgs& a, int t, int& p, int& m_blk, int& n_blk) {
+  p = (a.nprob > 1 && t >= a.tile0[1]) ? 1 : 0;
+  const int lt = t - a.tile0[p];
+  m_blk = lt % a.num_m[p];
+  n_blk = lt / a.num_m[p];
+}
+
+__device__ __forceinline__ void add_bias32(const bf16* bias, int n0, float (&v)[32]) {
+  const uint4* bp = reinterpret_cast<const uint4*>(bias + n0);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint4 u = __ldg(bp + q);
+    float2 f0 = unpack_bf16x2(u.x), f1 = unpack_bf16x2(u.y), f2 = unpack_bf16x2(u.z), f3 = unpack_bf16x2(u.w);
+    v[q * 8 + 0] += f0.x; v[q * 8 + 1] += f0.y; v[q * 8 + 2] += f1.x; v[q * 8 + 3] += f1.y;
+    v[q * 8 + 4] += f2.x; v[q * 8 + 5] += f2.y; v[q * 8 + 6] += f3.x; v[q * 8 + 7] += f3.y;
+  }
+}
+
+__device__ __forceinline__ void store_bf16x32(bf16* ob, const float (&v)[32]) {
+  uint4* dst = reinterpret_cast<uint4*>(ob);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint4 u;
+    u.x = pack_bf16x2(v[q * 8 + 0], v[q * 8 + 1]);
+    u.y = pack_bf16x2(v[q * 8 + 2], v[q * 8 + 3]);
+    u.z = pack_bf16x2(v[q * 8 + 4], v[q * 8 + 5]);
+    u.w = pack_bf16x2(v[q * 8 + 6], v[q * 8 + 7]);
+    dst[q] = u;
+  }
+}
+
+// destination of qkv column n (in [0, 3h)) of GEMM row `row` (plain [M, ld0] or Ulysses pack)
+__device__ __forceinline__ bf16* qkv_dst(const GemmEpi& e, int row, int n) {
+  if (e.k_sp <= 1) return reinterpret_cast<bf16*>(e.out0) + (long long)row * e.ld0 + n;
+  const int h = e.qk_h, D = e.qk_D;
+  const int part = n / h, hd = (n - part * h) / D, d = n % D;
+  const int hk = h / D / e.k_sp;
+  const int dst = hd / hk, hl = hd - dst * hk;
+  return e.pack + ((((long long)dst * e.pack_rows + e.pack_row0 + row) * 3 + part) * hk + hl) * D + d;
+}
+
+// Fused a3 + a4: one thread = one row; a head of D columns is D/32 TMEM chunks.  Pass 1 sums the
+// squares of y = acc + b over the head, pass 2 re-reads TMEM and writes RoPE(y * rsqrt(ms + eps) * g).
+__device__ __forceinline__ void epilogue_qk_head(const GemmEpi& e, int M, int row, int col0, uint32_t tcol) {
+  const int D = e.qk_D;
+  const bool norm = col0 < 2 * e.qk_h;
+  float rn = 1.f;
+  if (norm) {
+    float ss = 0.f;
+    for (int c = 0; c < D / 32; ++c) {
+      uint32_t r[32];
+      tmem_ld32(tcol + c * 32, r);
+      tmem_ld_wait();
+      float v[32];
+#pragma unroll
+      for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+      if (e.bias) add_bias32(e.bias, col0 + c * 32, v);
+#pragma unroll
+      for (int i = 0; i < 32; ++i) ss += v[i] * v[i];
+    }
+    rn = rsqrtf(ss / (float)D + 1e-6f);
+  }
+  const bf16* g = col0 < e.qk_h ? e.gq : e.gk;
+  for (int c = 0; c < D / 32; ++c) {
+    uint32_t r[32];
+    tmem_ld32(tcol + c * 32, r);
+    tmem_ld_wait();
+    float v[32];
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+    if (e.bias) add_bias32(e.bias, col0 + c * 32, v);
+    if (row >= M) continue;
+    if (norm) {
+      const uint4* gp = reinterpret_cast<const uint4*>(g + c * 32);
+      const float4* cp = reinterpret_cast<const float4*>(e.cosb + (long long)row * (D / 2) + c * 16);
+      const float4* sp = reinterpret_cast<const float4*>(e.sinb + (long long)row * (D / 2) + c * 16);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        uint4 gu = __ldg(gp + q);
+        float2 g0 = unpack_bf16x2(gu.x), g1 = unpack_bf16x2(gu.y), g2 = unpack_bf16x2(gu.z), g3 = unpack_bf16x2(gu.w);
+        float gg[8] = {g0.x, g0.y, g1.x, g1.y, g2.x, g2.y, g3.x, g3.y};
+        const float4 c4 = __ldg(cp + q), s4 = __ldg(sp + q);  // pairs 4q..4q+3 of this chunk
+        const float cs[4] = {c4.x, c4.y, c4.z, c4.w}, sn[4] = {s4.x, s4.y, s4.z, s4.w};
+#pragma unroll
+        for (int p = 0; p < 4; ++p) {
+          const float cc = cs[p], ss_ = sn[p];
+          const float y0 = v[q * 8 + 2 * p] * rn * gg[2 * p], y1 = v[q * 8 + 2 * p + 1] * rn * gg[2 * p + 1];
+          v[q * 8 + 2 * p] = cc * y0 - ss_ * y1;
+          v[q * 8 + 2 * p + 1] = ss_ * y0 + cc * y1;
+        }
+      }
+    }
+    store_bf16x32(qkv_dst(e, row, col0 + c * 32), v);
+  }
+}
+
+__device__ __forceinline__ void epilogue_chunk(const GemmEpi& e, int M, int row, int n0, const uint32_t (&r)[32]) {
   float v[32];
 #pragma unroll
   for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
@@ -55,7 +155,7 @@ __device__ __forceinline__ void epilogue_chunk(const GemmArgs& a, int row, int n
       v[q * 8 + 4] += f2.x; v[q * 8 + 5] += f2.y; v[q * 8 + 6] += f3.x; v[q * 8 + 7] += f3.y;
     }
   }
-  if (row >= a.M) return;
+  if (row >= M) return;
   int mode = e.mode;
   bf16* ob = nullptr;
   if (mode == EPI_SPLIT_GELU) {
@@ -133,8 +233,7 @@ __device__ __forceinline__ void epilogue_chunk(const GemmArgs& a, int row, int n
 
 template <int BN>
 __global__ void __launch_bounds__(GEMM_THREADS, 1)
-    gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                   const __grid_constant__ GemmArgs args) {
+    gemm_tc_kernel(const __grid_constant__ GemmMaps maps, const __grid_constant__ GemmArgs args) {
   using C = GemmCfg<BN>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -152,8 +251,10 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   const int num_k = args.K / BK;
 
   if (warp == 0 && lane == 0) {
-    tma_prefetch_desc(&tmA);
-    tma_prefetch_desc(&tmB);
+    for (int q = 0; q < args.nprob; ++q) {
+      tma_prefetch_desc(&maps.A[q]);
+      tma_prefetch_desc(&maps.B[q]);
+    }
     for (int s = 0; s < C::STAGES; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], 1);
@@ -176,12 +277,15 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       int stage = 0;
       uint32_t phase = 0;
       for (int t = blockIdx.x; t < args.num_tiles; t += gridDim.x) {
-        const int m_blk = t % args.num_m, n_blk = t / args.num_m;
+        int pr, m_blk, n_blk;
+        decode_tile(args, t, pr, m_blk, n_blk);
+        const CUtensorMap* tA = &maps.A[pr];
+        const CUtensorMap* tB = &maps.B[pr];
         for (int kb = 0; kb < num_k; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
-          tma_load_2d(&tmA, &full[stage], sA + stage * C::A_BYTES, kb * BK, m_blk * BM);
-          tma_load_2d(&tmB, &full[stage], sB + stage * C::B_BYTES, kb * BK, n_blk * BN);
+          tma_load_2d(tA, &full[stage], sA + stage * C::A_BYTES, kb * BK, m_blk * BM);
+          tma_load_2d(tB, &full[stage], sB + stage * C::B_BYTES, kb * BK, n_blk * BN);
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
       }
@@ -220,19 +324,28 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
     const int wq = warp - 4;
     int it = 0;
     for (int t = blockIdx.x; t < args.num_tiles; t += gridDim.x, ++it) {
-      const int m_blk = t % args.num_m, n_blk = t / args.num_m;
+      int pr, m_blk, n_blk;
+      decode_tile(args, t, pr, m_blk, n_blk);
+      const GemmEpi& epi = args.epi[pr];
+      const int Mp = args.M[pr];
       const int acc = it & 1;
       const uint32_t acc_phase = (it >> 1) & 1;
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
       const int row = m_blk * BM + wq * 32 + lane;
       const uint32_t tbase = tmem_base + ((uint32_t)(wq * 32) << 16) + acc * BN;
+      if (epi.qk_h > 0 && n_blk * BN < 3 * epi.qk_h) {
 #pragma unroll 1
-      for (int c = 0; c < BN / 32; ++c) {
-        uint32_t r[32];
-        tmem_ld32(tbase + c * 32, r);
-        tmem_ld_wait();
-        epilogue_chunk<BN>(args, row, n_blk * BN + c * 32, r);
+        for (int hd = 0; hd < BN / epi.qk_D; ++hd)
+          epilogue_qk_head(epi, Mp, row, n_blk * BN + hd * epi.qk_D, tbase + hd * epi.qk_D);
+      } else {
+#pragma unroll 1
+        for (int c = 0; c < BN / 32; ++c) {
+          uint32_t r[32];
+          tmem_ld32(tbase + c * 32, r);
+          tmem_ld_wait();
+          epilogue_chunk(epi, Mp, row, n_blk * BN + c * 32, r);
+        }
       }
       tc_fence_before();
       mbar_arrive(&tempty[acc]);
@@ -271,31 +384,69 @@ static int make_tmap_2d(CUtensorMap* m, const void* base, uint64_t inner, uint64
   return r == CUDA_SUCCESS ? 0 : -2;
 }
 
-int gemm_plan(GemmPlan* p, const bf16* A, long long lda, const bf16* W, long long ldw, int M, int N, int K,
-              const GemmEpi& epi, int num_sms, const char** err, int force_bn) {
+static const char* check_epi(const GemmEpi& epi, int bn) {
+  if (!epi.qk_h) return nullptr;
+  if (epi.qk_D != 64 && epi.qk_D != 128) return "gemm: fused QK-norm needs D in {64, 128}";
+  if (bn % epi.qk_D || epi.qk_h % epi.qk_D || (epi.qk_h / epi.qk_D) % epi.k_sp)
+    return "gemm: fused QK-norm needs D | BN, D | h and k_sp | heads";
+  if (epi.mode != EPI_STORE_BF16 && epi.mode != EPI_SPLIT_GELU) return "gemm: fused QK-norm needs a bf16 store";
+  if (epi.mode == EPI_SPLIT_GELU && epi.n_split != 3 * epi.qk_h) return "gemm: split must be at 3h";
+  if (!epi.gq || !epi.gk || !epi.cosb || !epi.sinb || (epi.k_sp > 1 && !epi.pack))
+    return "gemm: fused QK-norm needs gains, RoPE tables (and the pack buffer)";
+  return nullptr;
+}
+
+int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int K, int num_sms, const char** err,
+                    int force_bn) {
   *err = nullptr;
-  if (M <= 0 || N <= 0 || K <= 0) { *err = "gemm: empty shape"; return -1; }
+  if (nprob < 1 || nprob > 2) { *err = "gemm: 1 or 2 problems per launch"; return -1; }
+  if (N <= 0 || K <= 0) { *err = "gemm: empty shape"; return -1; }
   if (K % BK) { *err = "gemm: K must be a multiple of 64"; return -1; }
   if (N % 64) { *err = "gemm: N must be a multiple of 64"; return -1; }
-  if ((lda * 2) % 16 || (ldw * 2) % 16) { *err = "gemm: row strides must be 16-byte multiples"; return -1; }
-  if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(W)) & 15) {
-    *err = "gemm: operands must be 16-byte aligned"; return -1;
+  long long nm_total = 0;
+  int qk_D = 0;
+  for (int q = 0; q < nprob; ++q) {
+    const GemmProblem& g = probs[q];
+    if (g.M <= 0) { *err = "gemm: empty problem"; return -1; }
+    if ((g.lda * 2) % 16 || (g.ldw * 2) % 16) { *err = "gemm: row strides must be 16-byte multiples"; return -1; }
+    if ((reinterpret_cast<uintptr_t>(g.A) | reinterpret_cast<uintptr_t>(g.W)) & 15) {
+      *err = "gemm: operands must be 16-byte aligned"; return -1;
+    }
+    nm_total += (g.M + BM - 1) / BM;
+    if (g.epi.qk_h) qk_D = g.epi.qk_D > qk_D ? g.epi.qk_D : qk_D;
   }
   int bn = force_bn;
   if (!bn) {
-    const int nm = (M + BM - 1) / BM;
-    if (N % 256 == 0 && (long long)nm * (N / 256) >= num_sms * 3 / 4) bn = 256;
-    else if (N % 128 == 0 && (long long)nm * (N / 128) >= num_sms * 3 / 4) bn = 128;
-    else if (N % 256 == 0 && N >= 4096) bn = 256;
-    else bn = (N % 128 == 0 && nm * (N / 128) >= num_sms / 2) ? 128 : 64;
+    // Widest tile: measured on B200 (tools/microbench.py), 128x256 beats 128x128 even at 0.65
+    // waves (e.g. 1024x3072x12288: 968 vs 768 TFLOP/s) — narrower tiles are smem-bandwidth bound.
+    (void)nm_total;
+    bn = (N % 256 == 0) ? 256 : (N % 128 == 0 ? 128 : 64);
+    if (bn < qk_D) bn = qk_D;  // a head must sit inside one tile
   }
   if (N % bn) { *err = "gemm: N not a multiple of the tile width"; return -1; }
-  p->M = M; p->N = N; p->K = K; p->BN = bn; p->epi = epi;
-  if (make_tmap_2d(&p->tmA, A, K, M, lda * 2, BK, BM)) { *err = "gemm: cuTensorMapEncodeTiled(A) failed"; return -1; }
-  if (make_tmap_2d(&p->tmB, W, K, N, ldw * 2, BK, bn)) { *err = "gemm: cuTensorMapEncodeTiled(W) failed"; return -1; }
-  const int tiles = ((M + BM - 1) / BM) * (N / bn);
+  p->nprob = nprob; p->N = N; p->K = K; p->BN = bn;
+  int tiles = 0;
+  for (int q = 0; q < nprob; ++q) {
+    const GemmProblem& g = probs[q];
+    if ((*err = check_epi(g.epi, bn))) return -1;
+    p->Mq[q] = g.M;
+    p->epiq[q] = g.epi;
+    p->tile0[q] = tiles;
+    tiles += ((g.M + BM - 1) / BM) * (N / bn);
+    if (make_tmap_2d(&p->tmAq[q], g.A, K, g.M, g.lda * 2, BK, BM)) { *err = "gemm: cuTensorMapEncodeTiled(A) failed"; return -1; }
+    if (make_tmap_2d(&p->tmBq[q], g.W, K, N, g.ldw * 2, BK, bn)) { *err = "gemm: cuTensorMapEncodeTiled(W) failed"; return -1; }
+  }
+  p->tiles = tiles;
   p->grid = tiles < num_sms ? tiles : num_sms;
+  p->M = probs[0].M;
+  p->epi = probs[0].epi;
   return 0;
+}
+
+int gemm_plan(GemmPlan* p, const bf16* A, long long lda, const bf16* W, long long ldw, int M, int N, int K,
+              const GemmEpi& epi, int num_sms, const char** err, int force_bn) {
+  GemmProblem g{A, lda, W, ldw, M, epi};
+  return gemm_plan_multi(p, &g, 1, N, K, num_sms, err, force_bn);
 }
 
 template <int BN>
@@ -309,12 +460,18 @@ static void launch_bn(const GemmPlan& p, cudaStream_t s) {
     attr_done |= 1ull << dev;
   }
   GemmArgs a;
-  a.M = p.M; a.N = p.N; a.K = p.K;
-  a.num_m = (p.M + BM - 1) / BM;
-  a.num_n = p.N / BN;
-  a.num_tiles = a.num_m * a.num_n;
-  a.epi = p.epi;
-  gemm_tc_kernel<BN><<<p.grid, GEMM_THREADS, C::SMEM_BYTES, s>>>(p.tmA, p.tmB, a);
+  GemmMaps maps;
+  a.N = p.N; a.K = p.K; a.num_n = p.N / BN; a.num_tiles = p.tiles; a.nprob = p.nprob;
+  for (int q = 0; q < 2; ++q) {
+    const int qq = q < p.nprob ? q : 0;
+    a.M[q] = p.Mq[qq];
+    a.num_m[q] = (p.Mq[qq] + BM - 1) / BM;
+    a.tile0[q] = p.tile0[qq];
+    a.epi[q] = p.epiq[qq];
+    maps.A[q] = p.tmAq[qq];
+    maps.B[q] = p.tmBq[qq];
+  }
+  gemm_tc_kernel<BN><<<p.grid, GEMM_THREADS, C::SMEM_BYTES, s>>>(maps, a);
 }
 
 void gemm_launch(const GemmPlan& p, cudaStream_t s) {

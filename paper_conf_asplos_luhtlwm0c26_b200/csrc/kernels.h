@@ -33,13 +33,39 @@ struct GemmEpi {
   const bf16* bias = nullptr;   // [N]
   const float* gate = nullptr;  // [N]
   const float* scalar = nullptr;
+  // Fused a4 (QK-RMSNorm + RoPE, Ulysses pack) for a QKV-producing GEMM (modes STORE_BF16 /
+  // SPLIT_GELU): columns [0, 3*qk_h) are "(K H D)" q|k|v; q and k heads get
+  // RoPE(RMSNorm(y) * g), v passes through.  qk_h = 0 disables.
+  int qk_h = 0;
+  int qk_D = 0;
+  const bf16* gq = nullptr;
+  const bf16* gk = nullptr;
+  const float* cosb = nullptr;  // [M][qk_D/2], indexed by GEMM row
+  const float* sinb = nullptr;
+  // k_sp > 1: q|k|v columns are written to pack[dst][pack_rows][3][H/k_sp][D] at row pack_row0 + m
+  int k_sp = 1;
+  bf16* pack = nullptr;
+  int pack_rows = 0;
+  int pack_row0 = 0;
+};
+
+struct GemmProblem {
+  const bf16* A;
+  long long lda;
+  const bf16* W;
+  long long ldw;
+  int M;
+  GemmEpi epi;
 };
 
 struct GemmPlan {
-  CUtensorMap tmA, tmB;
+  int nprob = 1;
+  CUtensorMap tmAq[2], tmBq[2];
+  int Mq[2] = {0, 0}, tile0[2] = {0, 0};
+  GemmEpi epiq[2];
   int M = 0, N = 0, K = 0;
   int BN = 256;
-  int grid = 0;
+  int tiles = 0, grid = 0;
   GemmEpi epi;
 };
 
@@ -47,6 +73,9 @@ struct GemmPlan {
 // Returns 0 on success, nonzero (and sets *err) on invalid arguments.
 int gemm_plan(GemmPlan* p, const bf16* A, long long lda, const bf16* W, long long ldw, int M, int N, int K,
               const GemmEpi& epi, int num_sms, const char** err, int force_bn = 0);
+// One launch for up to two problems sharing N and K (persistent tile loop over both).
+int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int K, int num_sms, const char** err,
+                    int force_bn = 0);
 void gemm_launch(const GemmPlan& p, cudaStream_t s);
 
 // ------------------------------------------------------------------ elementwise / norm kernels
