@@ -205,7 +205,7 @@ def _stream(stream):
 
 
 def op_gemm(A, W, mode, out0, out1=None, bias=None, gate=None, scalar=None, n_split=0, M=None, N=None, K=None,
-            lda=None, ldw=None, ld0=None, ld1=None, force_bn=0, stream=None):
+            lda=None, ldw=None, ld0=None, ld1=None, force_bn=0, force_pair=-1, stream=None):
     M = A.shape[0] if M is None else M
     K = A.shape[1] if K is None else K
     N = W.shape[0] if N is None else N
@@ -214,7 +214,7 @@ def op_gemm(A, W, mode, out0, out1=None, bias=None, gate=None, scalar=None, n_sp
     ld0 = out0.stride(0) if ld0 is None else ld0
     ld1 = (out1.stride(0) if out1 is not None else 0) if ld1 is None else ld1
     check(lib.tsv_op_gemm(_ptr(A), lda, _ptr(W), ldw, M, N, K, EPI[mode] if isinstance(mode, str) else mode,
-                          _ptr(out0), ld0, _ptr(out1), ld1, n_split, _ptr(bias), _ptr(gate), _ptr(scalar), force_bn,
+                          _ptr(out0), ld0, _ptr(out1), ld1, n_split, _ptr(bias), _ptr(gate), _ptr(scalar), force_bn, force_pair,
                           _stream(stream)))
 
 

@@ -1413,7 +1413,7 @@ tsv_status tsv_engine_kernel_count(tsv_engine* e, int64_t* count) {
 // ------------------------------------------------------------------ kernel-level ops (tsv_ops.h)
 tsv_status tsv_op_gemm(const void* A, int64_t lda, const void* Wt, int64_t ldw, int M, int N, int K, int mode,
                        void* out0, int64_t ld0, void* out1, int64_t ld1, int n_split, const void* bias,
-                       const float* gate, const float* scalar, int force_bn, void* stream) {
+                       const float* gate, const float* scalar, int force_bn, int force_pair, void* stream) {
   if (mode < 0 || mode > EPI_EULER) return fail(TSV_E_INVAL, "bad epilogue mode %d", mode);
   if (force_bn && force_bn != 64 && force_bn != 128 && force_bn != 256) return fail(TSV_E_INVAL, "bad force_bn");
   int dev = 0, sms = 148;
@@ -1423,7 +1423,7 @@ tsv_status tsv_op_gemm(const void* A, int64_t lda, const void* Wt, int64_t ldw, 
   const char* err = nullptr;
   GemmEpi epi = epi_of(mode, out0, ld0, reinterpret_cast<const bf16*>(bias), gate, out1, ld1, n_split, scalar);
   if (gemm_plan(&p, reinterpret_cast<const bf16*>(A), lda, reinterpret_cast<const bf16*>(Wt), ldw, M, N, K, epi, sms,
-                &err, force_bn))
+                &err, force_bn, force_pair))
     return fail(TSV_E_INVAL, "%s", err);
   gemm_launch(p, reinterpret_cast<cudaStream_t>(stream));
   CK(cudaGetLastError());

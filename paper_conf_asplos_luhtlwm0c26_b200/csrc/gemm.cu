@@ -357,6 +357,147 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   if (warp == 2) tmem_dealloc<C::TMEM_COLS>(tmem_base);
 }
 
+// ------------------------------------------------------------------ CTA-pair (cta_group::2) variant
+// A cluster of 2 CTAs on one TPC computes a 256 x 256 tile: CTA r loads rows [128r, 128r+128) of the
+// A tile and rows [128r, 128r+128) of the B (weight) tile; the even CTA issues
+// tcgen05.mma.cta_group::2 (M = 256, N = 256), which reads A and B from both CTAs' shared memory
+// at the same offsets and leaves CTA r's 128 output rows in CTA r's TMEM.  Per SM this halves the
+// operand bytes read from shared memory per MMA compared with the 1-CTA 128 x 256 tile.
+struct Gemm2Cfg {
+  static constexpr int BN = 256;
+  static constexpr int A_BYTES = 128 * BK * 2;
+  static constexpr int B_BYTES = (BN / 2) * BK * 2;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int STAGES = 6;
+  static constexpr int TMEM_COLS = 2 * BN;
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+};
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
+    gemm_tc2_kernel(const __grid_constant__ GemmMaps maps, const __grid_constant__ GemmArgs args) {
+  using C = Gemm2Cfg;
+  constexpr int BN = C::BN;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + C::STAGES * C::A_BYTES;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES);
+  uint64_t* full = bars;
+  uint64_t* empty = bars + C::STAGES;
+  uint64_t* tfull = bars + 2 * C::STAGES;
+  uint64_t* tempty = bars + 2 * C::STAGES + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * C::STAGES + 4);
+
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_ctarank();
+  const bool leader = rank == 0;
+  const int cid = blockIdx.x >> 1, ncl = gridDim.x >> 1;
+  const int num_k = args.K / BK;
+
+  if (warp == 0 && lane == 0) {
+    for (int q = 0; q < args.nprob; ++q) {
+      tma_prefetch_desc(&maps.A[q]);
+      tma_prefetch_desc(&maps.B[q]);
+    }
+    for (int s = 0; s < C::STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&tfull[i], 1);
+      mbar_init(&tempty[i], 2 * 128);  // both CTAs' epilogue threads drain before reuse
+    }
+    fence_mbar_init();
+  }
+  if (warp == 2) tmem_alloc_pair<C::TMEM_COLS>(tmem_slot);
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int t = cid; t < args.num_tiles; t += ncl) {
+        int pr, m_blk, n_blk;
+        decode_tile(args, t, pr, m_blk, n_blk);
+        const CUtensorMap* tA = &maps.A[pr];
+        const CUtensorMap* tB = &maps.B[pr];
+        for (int kb = 0; kb < num_k; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          if (leader) mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
+          tma_load_2d_pair(tA, &full[stage], sA + stage * C::A_BYTES, kb * BK, m_blk * 256 + (int)rank * 128);
+          tma_load_2d_pair(tB, &full[stage], sB + stage * C::B_BYTES, kb * BK, n_blk * BN + (int)rank * (BN / 2));
+          if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && leader) {
+      constexpr uint32_t idesc = make_idesc_bf16(256, BN);
+      int stage = 0;
+      uint32_t phase = 0;
+      int it = 0;
+      for (int t = cid; t < args.num_tiles; t += ncl, ++it) {
+        const int acc = it & 1;
+        const uint32_t acc_phase = (it >> 1) & 1;
+        mbar_wait(&tempty[acc], acc_phase ^ 1);
+        tc_fence_after();
+        const uint32_t d_tmem = tmem_base + acc * BN;
+        for (int kb = 0; kb < num_k; ++kb) {
+          mbar_wait(&full[stage], phase);
+          tc_fence_after();
+          const uint32_t a_addr = smem_u32(sA + stage * C::A_BYTES);
+          const uint32_t b_addr = smem_u32(sB + stage * C::B_BYTES);
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k)
+            umma_bf16_ss_pair(d_tmem, make_sw128_desc(a_addr + k * 32), make_sw128_desc(b_addr + k * 32), idesc,
+                              (kb | k) != 0);
+          umma_commit_pair(&empty[stage]);
+          if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+        }
+        umma_commit_pair(&tfull[acc]);
+      }
+    }
+  } else if (warp >= 4) {
+    const int wq = warp - 4;
+    int it = 0;
+    for (int t = cid; t < args.num_tiles; t += ncl, ++it) {
+      int pr, m_blk, n_blk;
+      decode_tile(args, t, pr, m_blk, n_blk);
+      const GemmEpi& epi = args.epi[pr];
+      const int Mp = args.M[pr];
+      const int acc = it & 1;
+      const uint32_t acc_phase = (it >> 1) & 1;
+      mbar_wait(&tfull[acc], acc_phase);
+      tc_fence_after();
+      const int row = m_blk * 256 + (int)rank * 128 + wq * 32 + lane;
+      const uint32_t tbase = tmem_base + ((uint32_t)(wq * 32) << 16) + acc * BN;
+      if (epi.qk_h > 0 && n_blk * BN < 3 * epi.qk_h) {
+#pragma unroll 1
+        for (int hd = 0; hd < BN / epi.qk_D; ++hd)
+          epilogue_qk_head(epi, Mp, row, n_blk * BN + hd * epi.qk_D, tbase + hd * epi.qk_D);
+      } else {
+#pragma unroll 1
+        for (int c = 0; c < BN / 32; ++c) {
+          uint32_t r[32];
+          tmem_ld32(tbase + c * 32, r);
+          tmem_ld_wait();
+          epilogue_chunk(epi, Mp, row, n_blk * BN + c * 32, r);
+        }
+      }
+      tc_fence_before();
+      mbar_arrive_remote(&tempty[acc], 0);
+    }
+  }
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  if (warp == 2) tmem_dealloc_pair<C::TMEM_COLS>(tmem_base);
+}
+
 // ------------------------------------------------------------------ host side
 static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -397,7 +538,7 @@ static const char* check_epi(const GemmEpi& epi, int bn) {
 }
 
 int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int K, int num_sms, const char** err,
-                    int force_bn) {
+                    int force_bn, int force_pair) {
   *err = nullptr;
   if (nprob < 1 || nprob > 2) { *err = "gemm: 1 or 2 problems per launch"; return -1; }
   if (N <= 0 || K <= 0) { *err = "gemm: empty shape"; return -1; }
@@ -424,7 +565,12 @@ int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int
     if (bn < qk_D) bn = qk_D;  // a head must sit inside one tile
   }
   if (N % bn) { *err = "gemm: N not a multiple of the tile width"; return -1; }
-  p->nprob = nprob; p->N = N; p->K = K; p->BN = bn;
+  int maxM = 0;
+  for (int q = 0; q < nprob; ++q) maxM = probs[q].M > maxM ? probs[q].M : maxM;
+  // CTA pairs (256 x 256 tiles, cta_group::2) whenever a 256-wide tile is used on more than 128 rows
+  const bool pair = force_pair >= 0 ? (force_pair > 0 && bn == 256) : (bn == 256 && maxM > 128);
+  const int bm = pair ? 256 : BM;
+  p->nprob = nprob; p->N = N; p->K = K; p->BN = bn; p->pair = pair;
   int tiles = 0;
   for (int q = 0; q < nprob; ++q) {
     const GemmProblem& g = probs[q];
@@ -432,21 +578,28 @@ int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int
     p->Mq[q] = g.M;
     p->epiq[q] = g.epi;
     p->tile0[q] = tiles;
-    tiles += ((g.M + BM - 1) / BM) * (N / bn);
+    tiles += ((g.M + bm - 1) / bm) * (N / bn);
     if (make_tmap_2d(&p->tmAq[q], g.A, K, g.M, g.lda * 2, BK, BM)) { *err = "gemm: cuTensorMapEncodeTiled(A) failed"; return -1; }
-    if (make_tmap_2d(&p->tmBq[q], g.W, K, N, g.ldw * 2, BK, bn)) { *err = "gemm: cuTensorMapEncodeTiled(W) failed"; return -1; }
+    if (make_tmap_2d(&p->tmBq[q], g.W, K, N, g.ldw * 2, BK, pair ? bn / 2 : bn)) {
+      *err = "gemm: cuTensorMapEncodeTiled(W) failed"; return -1;
+    }
   }
   p->tiles = tiles;
-  p->grid = tiles < num_sms ? tiles : num_sms;
+  if (pair) {
+    const int clusters = tiles < num_sms / 2 ? tiles : num_sms / 2;
+    p->grid = 2 * clusters;
+  } else {
+    p->grid = tiles < num_sms ? tiles : num_sms;
+  }
   p->M = probs[0].M;
   p->epi = probs[0].epi;
   return 0;
 }
 
 int gemm_plan(GemmPlan* p, const bf16* A, long long lda, const bf16* W, long long ldw, int M, int N, int K,
-              const GemmEpi& epi, int num_sms, const char** err, int force_bn) {
+              const GemmEpi& epi, int num_sms, const char** err, int force_bn, int force_pair) {
   GemmProblem g{A, lda, W, ldw, M, epi};
-  return gemm_plan_multi(p, &g, 1, N, K, num_sms, err, force_bn);
+  return gemm_plan_multi(p, &g, 1, N, K, num_sms, err, force_bn, force_pair);
 }
 
 template <int BN>
@@ -461,17 +614,27 @@ static void launch_bn(const GemmPlan& p, cudaStream_t s) {
   }
   GemmArgs a;
   GemmMaps maps;
+  const int bm = p.pair ? 256 : BM;
   a.N = p.N; a.K = p.K; a.num_n = p.N / BN; a.num_tiles = p.tiles; a.nprob = p.nprob;
   for (int q = 0; q < 2; ++q) {
     const int qq = q < p.nprob ? q : 0;
     a.M[q] = p.Mq[qq];
-    a.num_m[q] = (p.Mq[qq] + BM - 1) / BM;
+    a.num_m[q] = (p.Mq[qq] + bm - 1) / bm;
     a.tile0[q] = p.tile0[qq];
     a.epi[q] = p.epiq[qq];
     maps.A[q] = p.tmAq[qq];
     maps.B[q] = p.tmBq[qq];
   }
-  gemm_tc_kernel<BN><<<p.grid, GEMM_THREADS, C::SMEM_BYTES, s>>>(maps, a);
+  if (p.pair) {
+    static unsigned long long attr2 = 0;
+    if (!(attr2 >> dev & 1ull)) {
+      cudaFuncSetAttribute(gemm_tc2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, Gemm2Cfg::SMEM_BYTES);
+      attr2 |= 1ull << dev;
+    }
+    gemm_tc2_kernel<<<p.grid, GEMM_THREADS, Gemm2Cfg::SMEM_BYTES, s>>>(maps, a);
+  } else {
+    gemm_tc_kernel<BN><<<p.grid, GEMM_THREADS, C::SMEM_BYTES, s>>>(maps, a);
+  }
 }
 
 void gemm_launch(const GemmPlan& p, cudaStream_t s) {

@@ -66,16 +66,17 @@ struct GemmPlan {
   int M = 0, N = 0, K = 0;
   int BN = 256;
   int tiles = 0, grid = 0;
+  bool pair = false;  // CTA-pair (cta_group::2) 256 x 256 tiles
   GemmEpi epi;
 };
 
 // A: [M, K] bf16 row stride lda (elements); W: [N, K] bf16 row stride ldw. K % 64 == 0, N % 64 == 0.
 // Returns 0 on success, nonzero (and sets *err) on invalid arguments.
 int gemm_plan(GemmPlan* p, const bf16* A, long long lda, const bf16* W, long long ldw, int M, int N, int K,
-              const GemmEpi& epi, int num_sms, const char** err, int force_bn = 0);
+              const GemmEpi& epi, int num_sms, const char** err, int force_bn = 0, int force_pair = -1);
 // One launch for up to two problems sharing N and K (persistent tile loop over both).
 int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int K, int num_sms, const char** err,
-                    int force_bn = 0);
+                    int force_bn = 0, int force_pair = -1);
 void gemm_launch(const GemmPlan& p, cudaStream_t s);
 
 // ------------------------------------------------------------------ elementwise / norm kernels

@@ -72,8 +72,8 @@ GEMM_SHAPES = [(1, 64, 64), (100, 256, 128), (128, 768, 256), (300, 1024, 256), 
 
 
 @pytest.mark.parametrize("M,N,K", GEMM_SHAPES)
-@pytest.mark.parametrize("bn", [0, 64, 128, 256])
-def test_gemm_integer_exact(tsv, M, N, K, bn):
+@pytest.mark.parametrize("bn,pair", [(0, -1), (64, 0), (128, 0), (256, 0), (256, 1)])
+def test_gemm_integer_exact(tsv, M, N, K, bn, pair):
     if bn and N % bn:
         pytest.skip("N not a multiple of the tile")
     rng = np.random.default_rng(M * 7 + N + K + bn)
@@ -82,11 +82,11 @@ def test_gemm_integer_exact(tsv, M, N, K, bn):
     b = rng.integers(-4, 5, N).astype(np.float32)
     exact = A.astype(np.float64) @ W.astype(np.float64).T + b   # |sums| < 2^24: exact in fp32
     out = torch.zeros(M, N, dtype=torch.float32, device="cuda")
-    tsv.op_gemm(_bf16(A), _bf16(W), "STORE_F32", out, bias=_bf16(b), force_bn=bn)
+    tsv.op_gemm(_bf16(A), _bf16(W), "STORE_F32", out, bias=_bf16(b), force_bn=bn, force_pair=pair)
     torch.cuda.synchronize()
     assert np.array_equal(out.cpu().numpy().astype(np.float64), exact)
     outb = torch.zeros(M, N, dtype=torch.bfloat16, device="cuda")
-    tsv.op_gemm(_bf16(A), _bf16(W), "STORE_BF16", outb, bias=_bf16(b), force_bn=bn)
+    tsv.op_gemm(_bf16(A), _bf16(W), "STORE_BF16", outb, bias=_bf16(b), force_bn=bn, force_pair=pair)
     torch.cuda.synchronize()
     ref_b = torch.from_numpy(exact.astype(np.float32)).to(torch.bfloat16)
     assert torch.equal(outb.cpu(), ref_b)

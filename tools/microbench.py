@@ -36,11 +36,11 @@ def gemm_cases():
         A = torch.randn(M, K, device="cuda").to(torch.bfloat16)
         W = (torch.randn(N, K, device="cuda") / math.sqrt(K)).to(torch.bfloat16)
         o = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
-        for bn in (0, 64, 128, 256):
+        for bn, pair in ((0, -1), (128, 0), (256, 0), (256, 1)):
             if N % (bn or 64):
                 continue
-            ms = timeit(lambda: tsv.op_gemm(A, W, "STORE_BF16", o, force_bn=bn))
-            print(json.dumps({"op": "gemm", "M": M, "N": N, "K": K, "bn": bn, "ms": round(ms, 4),
+            ms = timeit(lambda: tsv.op_gemm(A, W, "STORE_BF16", o, force_bn=bn, force_pair=pair))
+            print(json.dumps({"op": "gemm", "M": M, "N": N, "K": K, "bn": bn, "pair": pair, "ms": round(ms, 4),
                               "tflops": round(2 * M * N * K / ms / 1e9, 1)}), flush=True)
         ref = timeit(lambda: torch.matmul(A, W.t(), out=o))
         print(json.dumps({"op": "gemm_cublas_ref", "M": M, "N": N, "K": K, "ms": round(ref, 4),
