@@ -53,6 +53,11 @@ __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&r)[32
       "r"(r[18]), "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]), "r"(r[24]), "r"(r[25]), "r"(r[26]),
       "r"(r[27]), "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31]));
 }
+__device__ __forceinline__ float fast_exp2(float x) {  // MUFU.EX2; ex2(-inf) = +0
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
 __device__ __forceinline__ void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 // MN-major, 128B-swizzled B operand (rows = K, 64 N-elements per 128-byte row):
@@ -187,16 +192,26 @@ __global__ void __launch_bounds__(AT_THREADS, 1)
       tc_fence_before();
       mbar_arrive(&s_free[st]);
       const int kbase = j * AT_BN;
-      float mt = -FLT_MAX;
+      // row max on the raw scores (scale > 0); keys >= L only exist in the last tile
+      float mr0 = -FLT_MAX, mr1 = -FLT_MAX;
+      if (kbase + AT_BN <= L) {
 #pragma unroll
-      for (int c = 0; c < 4; ++c)
+        for (int c = 0; c < 4; ++c)
 #pragma unroll
-        for (int i = 0; i < 32; ++i) {
-          float x = __uint_as_float(sr[c][i]) * scale_log2;
-          if (kbase + c * 32 + i >= L) x = -INFINITY;
-          sr[c][i] = __float_as_uint(x);
-          mt = fmaxf(mt, x);
-        }
+          for (int i = 0; i < 32; i += 2) {
+            mr0 = fmaxf(mr0, __uint_as_float(sr[c][i]));
+            mr1 = fmaxf(mr1, __uint_as_float(sr[c][i + 1]));
+          }
+      } else {
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+#pragma unroll
+          for (int i = 0; i < 32; ++i) {
+            if (kbase + c * 32 + i >= L) sr[c][i] = __float_as_uint(-INFINITY);
+            mr0 = fmaxf(mr0, __uint_as_float(sr[c][i]));
+          }
+      }
+      const float mt = fmaxf(mr0, mr1) * scale_log2;
       bool rescale = false;
       float alpha = 1.f;
       if (j == 0) {
@@ -208,18 +223,21 @@ __global__ void __launch_bounds__(AT_THREADS, 1)
       }
       l_sum *= alpha;
       // P = exp2(x - m_ref) -> bf16, packed in pairs
+      // P = 2^(s * scale_log2 - m_ref): one FFMA + one MUFU.EX2 per score
       uint32_t pk[64];
-      float ls = 0.f;
+      float ls0 = 0.f, ls1 = 0.f;
+      const float neg_m = -m_ref;
 #pragma unroll
       for (int c = 0; c < 4; ++c)
 #pragma unroll
         for (int i = 0; i < 32; i += 2) {
-          const float p0 = exp2f(__uint_as_float(sr[c][i]) - m_ref);
-          const float p1 = exp2f(__uint_as_float(sr[c][i + 1]) - m_ref);
-          ls += p0 + p1;
+          const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
+          const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
+          ls0 += p0;
+          ls1 += p1;
           pk[c * 16 + i / 2] = pack_bf16x2(p0, p1);
         }
-      l_sum += ls;
+      l_sum += ls0 + ls1;
       if (j >= 2) mbar_wait(&pv_done[st], ((j - 2) >> 1) & 1);  // P buffer st free
       // tcgen05.ld/st are warp-collective (.sync.aligned): rescale the whole warp's rows together
       // (alpha = 1 for rows that did not need it).

@@ -567,8 +567,14 @@ int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int
   if (N % bn) { *err = "gemm: N not a multiple of the tile width"; return -1; }
   int maxM = 0;
   for (int q = 0; q < nprob; ++q) maxM = probs[q].M > maxM ? probs[q].M : maxM;
-  // CTA pairs (256 x 256 tiles, cta_group::2) whenever a 256-wide tile is used on more than 128 rows
-  const bool pair = force_pair >= 0 ? (force_pair > 0 && bn == 256) : (bn == 256 && maxM > 128);
+  // CTA pairs (256 x 256 tiles, cta_group::2): faster per tile (half the smem operand traffic per
+  // SM) but half as many tiles.  Measured (tools/microbench.py): pairs win for long K (>= 8192) or
+  // when the pair tiles still fill ~half the SM pairs; e.g. 1024x3072x3072 (48 pair tiles) is
+  // faster as 96 single-CTA tiles.
+  long long pair_tiles = 0;
+  for (int q = 0; q < nprob; ++q) pair_tiles += (long long)((probs[q].M + 255) / 256) * (N / 256);
+  const bool pair_auto = bn == 256 && maxM > 128 && (K >= 8192 || pair_tiles * 2 >= (long long)num_sms * 9 / 10);
+  const bool pair = force_pair >= 0 ? (force_pair > 0 && bn == 256) : pair_auto;
   const int bm = pair ? 256 : BM;
   p->nprob = nprob; p->N = N; p->K = K; p->BN = bn; p->pair = pair;
   int tiles = 0;
