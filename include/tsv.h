@@ -180,6 +180,15 @@ tsv_status tsv_latency_table(tsv_engine* eng, const int* res_px, int n_res, cons
 tsv_status tsv_shard_range(int64_t n_rows, int k, int rank, int64_t* begin, int64_t* end);
 tsv_status tsv_reshard_plan(int64_t n_rows, int k_src, int k_dst, int64_t* out, int max_copies, int* n_copies);
 
+/* Ulysses all-to-all plan of rank `rank` in a group of k (S:§8(a) a5/a7), as the step
+ * executes it: up to max_ops entries of 4 int64 (peer, is_send, row0, rows).  which = 1 (seq ->
+ * head): sends read the pack buffer [k][rows_rank] rows, receives write the [L] rows of the
+ * attention input in global order [txt_0..txt_{k-1}; img_0..img_{k-1}]; which = 2 (head -> seq):
+ * sends read the [L] attention-output rows, receives write [k][rows_rank].  Sends and receives
+ * between two ranks match in plan order.  Row widths: 3h/k (which = 1), h/k (which = 2). */
+tsv_status tsv_a2a_plan(int which, int64_t text_rows, int64_t image_rows, int k, int rank, int64_t* out, int max_ops,
+                        int* n_ops);
+
 /* Debug / parity: copy weight tensor `tensor_id` (bf16 bits) from the device of local slot 0. */
 tsv_status tsv_debug_read_weight(tsv_engine* eng, int tensor_id, uint16_t* host, size_t n);
 /* Per-kernel-class device-time profiling: when enabled, every launch is bracketed by CUDA events

@@ -35,6 +35,15 @@ def reshard_plan(n_rows: int, k_src: int, k_dst: int):
     return [tuple(buf[5 * i:5 * i + 5]) for i in range(n.value)]
 
 
+def a2a_plan(which: int, text_rows: int, image_rows: int, k: int, rank: int):
+    """[(peer, is_send, row0, rows)] of the step's Ulysses all-to-all #which for `rank` (tsv_a2a_plan)."""
+    cap = 4 * k
+    buf = (C.c_int64 * (4 * cap))()
+    n = C.c_int()
+    check(lib.tsv_a2a_plan(which, text_rows, image_rows, k, rank, buf, cap, C.byref(n)))
+    return [tuple(buf[4 * i:4 * i + 4]) for i in range(n.value)]
+
+
 def nccl_unique_id() -> bytes:
     buf = (C.c_uint8 * 128)()
     check(lib.tsv_nccl_unique_id(buf))

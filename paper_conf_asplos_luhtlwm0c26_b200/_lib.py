@@ -64,7 +64,8 @@ _SIGS = {
     "tsv_latency_table": (_i32, [_p, _P(_i32), _i32, _P(_i32), _i32, _i32, _i32, _P(C.c_double), _P(C.c_double)]),
     "tsv_shard_range": (_i32, [_i64, _i32, _i32, _P(_i64), _P(_i64)]),
     "tsv_reshard_plan": (_i32, [_i64, _i32, _i32, _P(_i64), _i32, _P(_i32)]),
-    "tsv_debug_read_weight": (_i32, [_p, _i32, _P(C.c_uint16), C.c_size_t]),
+    "tsv_a2a_plan": (_i32, [_i32, _i64, _i64, _i32, _i32, _P(_i64), _i32, _P(_i32)]),
+    "tsv_debug_read_weight":(_i32, [_p, _i32, _P(C.c_uint16), C.c_size_t]),
     "tsv_engine_kernel_count": (_i32, [_p, _P(_i64)]),
     "tsv_engine_profile": (_i32, [_p, _i32]),
     "tsv_engine_profile_read": (_i32, [_p, _P(C.c_double), _P(_i64), _P(C.c_double), _P(C.c_double)]),

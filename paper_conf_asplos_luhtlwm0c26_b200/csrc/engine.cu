@@ -478,46 +478,85 @@ struct StepEnv {
   std::vector<int64_t> t_off, t_cnt, i_off, i_cnt;  // per group rank
 };
 
-// in-process all-to-all #1: pack_r[d] ([rows_r][3h/k]) -> recv_d rows (global order)
-static tsv_status a2a_qkv(StepEnv& E) {
+// ------------------------------------------------------------------ Ulysses all-to-alls (a5, a7)
+// A plan entry is one contiguous block of `rows` rows (of the all-to-all's row width) exchanged
+// with `peer`: sent from / received into the caller's buffer at row `row0`.  Sends and receives
+// between a pair of ranks are matched in plan order (NCCL point-to-point semantics); the same plan
+// drives the NCCL path and the in-process peer-copy path (and is exported as tsv_a2a_plan).
+struct A2AOp {
+  int peer, send;
+  int64_t row0, rows;
+};
+
+// which = 1 (seq -> head): send buffer = pack [k][rows_r] rows (chunk p = peer p's heads),
+//                          recv buffer = recv [L] rows in global order [txt_0..txt_k-1; img_0..img_k-1].
+// which = 2 (head -> seq): send buffer = obuf [L] rows, recv buffer = orecv [k][rows_r] rows.
+static void a2a_plan(int which, int64_t Lt, int64_t Li, int k, int r, std::vector<A2AOp>& ops) {
+  ops.clear();
+  auto tb = [&](int q) { return shard_begin(Lt, k, q); };
+  auto tc = [&](int q) { return shard_begin(Lt, k, q + 1) - shard_begin(Lt, k, q); };
+  auto ib = [&](int q) { return shard_begin(Li, k, q); };
+  auto ic = [&](int q) { return shard_begin(Li, k, q + 1) - shard_begin(Li, k, q); };
+  const int64_t rows_r = tc(r) + ic(r);
+  for (int p = 0; p < k; ++p) {
+    if (which == 1) {
+      if (tc(r)) ops.push_back({p, 1, p * rows_r, tc(r)});
+      if (ic(r)) ops.push_back({p, 1, p * rows_r + tc(r), ic(r)});
+      if (tc(p)) ops.push_back({p, 0, tb(p), tc(p)});
+      if (ic(p)) ops.push_back({p, 0, Lt + ib(p), ic(p)});
+    } else {
+      if (tc(p)) ops.push_back({p, 1, tb(p), tc(p)});
+      if (ic(p)) ops.push_back({p, 1, Lt + ib(p), ic(p)});
+      if (tc(r)) ops.push_back({p, 0, p * rows_r, tc(r)});
+      if (ic(r)) ops.push_back({p, 0, p * rows_r + tc(r), ic(r)});
+    }
+  }
+}
+
+static tsv_status a2a_exec(StepEnv& E, int which) {
   tsv_engine* e = E.e;
   const Model& m = e->model;
   Group& g = *E.g;
   const int k = g.k;
-  const int64_t w = 3 * (int64_t)m.h / k;  // bf16 per row per destination
-  const int64_t Lt = E.R->Lt;
+  const int64_t w = (which == 1 ? 3 : 1) * (int64_t)m.h / k;  // bf16 per row
+  auto sendbuf = [&](RankCtx& c) { return which == 1 ? c.pack : c.obuf; };
+  auto recvbuf = [&](RankCtx& c) { return which == 1 ? c.recv : c.orecv; };
+  std::vector<A2AOp> ops;
   if (g.comm) {
     RankCtx& c = E.rc[0];
     const int r = g.local_positions[0];
     CK(cudaSetDevice(c.s->device));
-    ProfScope ps(e, *c.s, KC_A2A, 0.0, 2.0 * c.rows * 3 * m.h * (k - 1) / k);
+    ProfScope ps(e, *c.s, KC_A2A, 0.0, 2.0 * c.rows * w * (k - 1));
+    a2a_plan(which, E.R->Lt, E.R->Li, k, r, ops);
     NK(ncclGroupStart());
-    for (int p = 0; p < k; ++p) {
-      const bf16* sendp = c.pack + (int64_t)p * c.rows * w;
-      if (E.t_cnt[r]) NK(ncclSend(sendp, E.t_cnt[r] * w, ncclBfloat16, p, g.comm, c.s->stream));
-      if (E.i_cnt[r]) NK(ncclSend(sendp + E.t_cnt[r] * w, E.i_cnt[r] * w, ncclBfloat16, p, g.comm, c.s->stream));
-      if (E.t_cnt[p]) NK(ncclRecv(c.recv + E.t_off[p] * w, E.t_cnt[p] * w, ncclBfloat16, p, g.comm, c.s->stream));
-      if (E.i_cnt[p])
-        NK(ncclRecv(c.recv + (Lt + E.i_off[p]) * w, E.i_cnt[p] * w, ncclBfloat16, p, g.comm, c.s->stream));
+    for (const A2AOp& o : ops) {
+      if (o.send) NK(ncclSend(sendbuf(c) + o.row0 * w, o.rows * w, ncclBfloat16, o.peer, g.comm, c.s->stream));
+      else NK(ncclRecv(recvbuf(c) + o.row0 * w, o.rows * w, ncclBfloat16, o.peer, g.comm, c.s->stream));
     }
     NK(ncclGroupEnd());
     return TSV_OK;
   }
-  // in-process: all k ranks are local (rc indexed by group rank)
+  // in-process: all k ranks are local (rc indexed by group rank); receiver streams pull.
+  std::vector<std::vector<A2AOp>> plans(k);
+  for (int r = 0; r < k; ++r) a2a_plan(which, E.R->Lt, E.R->Li, k, r, plans[r]);
   for (int r = 0; r < k; ++r) CK(cudaEventRecord(g.ev_a[r], E.rc[r].s->stream));
   for (int d = 0; d < k; ++d) {
     RankCtx& dst = E.rc[d];
-    ProfScope ps(e, *dst.s, KC_A2A, 0.0, 2.0 * dst.rows * 3 * m.h * (k - 1) / k, 0);
+    CK(cudaSetDevice(dst.s->device));
+    ProfScope ps(e, *dst.s, KC_A2A, 0.0, 2.0 * dst.rows * w * (k - 1), 0);
     for (int r = 0; r < k; ++r) CK(cudaStreamWaitEvent(dst.s->stream, g.ev_a[r], 0));
-    for (int r = 0; r < k; ++r) {
-      RankCtx& src = E.rc[r];
-      const bf16* sp = src.pack + (int64_t)d * src.rows * w;
-      if (E.t_cnt[r])
-        CK(cudaMemcpyPeerAsync(dst.recv + E.t_off[r] * w, dst.s->device, sp, src.s->device, E.t_cnt[r] * w * 2,
-                               dst.s->stream));
-      if (E.i_cnt[r])
-        CK(cudaMemcpyPeerAsync(dst.recv + (Lt + E.i_off[r]) * w, dst.s->device, sp + E.t_cnt[r] * w, src.s->device,
-                               E.i_cnt[r] * w * 2, dst.s->stream));
+    std::vector<int> nth_recv(k, 0);
+    for (const A2AOp& o : plans[d]) {
+      if (o.send) continue;
+      const int p = o.peer;
+      int idx = nth_recv[p]++, seen = 0;
+      const A2AOp* match = nullptr;
+      for (const A2AOp& so : plans[p])
+        if (so.send && so.peer == d && seen++ == idx) { match = &so; break; }
+      if (!match || match->rows != o.rows) return fail(TSV_E_STATE, "all-to-all plan mismatch");
+      RankCtx& src = E.rc[p];
+      CK(cudaMemcpyPeerAsync(recvbuf(dst) + o.row0 * w, dst.s->device, sendbuf(src) + match->row0 * w, src.s->device,
+                             o.rows * w * 2, dst.s->stream));
     }
     CK(cudaEventRecord(g.ev_b[d], dst.s->stream));
   }
@@ -526,51 +565,15 @@ static tsv_status a2a_qkv(StepEnv& E) {
   return TSV_OK;
 }
 
-// all-to-all #2: obuf_d ([L][h/k], global rows) -> orecv_r[d] ([rows_r][h/k]), then unpack into cat[:, d*h/k]
+static tsv_status a2a_qkv(StepEnv& E) { return a2a_exec(E, 1); }
+
+// all-to-all #2 then unpack: cat[i, d*h/k + c] = orecv[d][i][c]
 static tsv_status a2a_o(StepEnv& E) {
   tsv_engine* e = E.e;
   const Model& m = e->model;
-  Group& g = *E.g;
-  const int k = g.k;
+  const int k = E.g->k;
   const int64_t w = (int64_t)m.h / k;
-  const int64_t Lt = E.R->Lt;
-  if (g.comm) {
-    RankCtx& c = E.rc[0];
-    const int r = g.local_positions[0];
-    CK(cudaSetDevice(c.s->device));
-    ProfScope ps(e, *c.s, KC_A2A, 0.0, 2.0 * c.rows * m.h * (k - 1) / k);
-    NK(ncclGroupStart());
-    for (int p = 0; p < k; ++p) {
-      if (E.t_cnt[p]) NK(ncclSend(c.obuf + E.t_off[p] * w, E.t_cnt[p] * w, ncclBfloat16, p, g.comm, c.s->stream));
-      if (E.i_cnt[p])
-        NK(ncclSend(c.obuf + (Lt + E.i_off[p]) * w, E.i_cnt[p] * w, ncclBfloat16, p, g.comm, c.s->stream));
-      bf16* rp = c.orecv + (int64_t)p * c.rows * w;
-      if (E.t_cnt[r]) NK(ncclRecv(rp, E.t_cnt[r] * w, ncclBfloat16, p, g.comm, c.s->stream));
-      if (E.i_cnt[r]) NK(ncclRecv(rp + E.t_cnt[r] * w, E.i_cnt[r] * w, ncclBfloat16, p, g.comm, c.s->stream));
-    }
-    NK(ncclGroupEnd());
-  } else {
-    for (int d = 0; d < k; ++d) CK(cudaEventRecord(g.ev_a[d], E.rc[d].s->stream));
-    for (int r = 0; r < k; ++r) {
-      RankCtx& dst = E.rc[r];
-      ProfScope ps(e, *dst.s, KC_A2A, 0.0, 2.0 * dst.rows * m.h * (k - 1) / k, 0);
-      for (int d = 0; d < k; ++d) CK(cudaStreamWaitEvent(dst.s->stream, g.ev_a[d], 0));
-      for (int d = 0; d < k; ++d) {
-        RankCtx& src = E.rc[d];
-        bf16* rp = dst.orecv + (int64_t)d * dst.rows * w;
-        if (E.t_cnt[r])
-          CK(cudaMemcpyPeerAsync(rp, dst.s->device, src.obuf + E.t_off[r] * w, src.s->device, E.t_cnt[r] * w * 2,
-                                 dst.s->stream));
-        if (E.i_cnt[r])
-          CK(cudaMemcpyPeerAsync(rp + E.t_cnt[r] * w, dst.s->device, src.obuf + (Lt + E.i_off[r]) * w, src.s->device,
-                                 E.i_cnt[r] * w * 2, dst.s->stream));
-      }
-      CK(cudaEventRecord(g.ev_b[r], dst.s->stream));
-    }
-    for (int r = 0; r < k; ++r)
-      for (int d = 0; d < k; ++d) CK(cudaStreamWaitEvent(E.rc[r].s->stream, g.ev_b[d], 0));
-  }
-  // unpack: cat[i, d*w + c] = orecv[d][i][c]
+  TRY(a2a_exec(E, 2));
   for (auto& c : E.rc) {
     CK(cudaSetDevice(c.s->device));
     for (int d = 0; d < k; ++d) {
@@ -1359,6 +1362,23 @@ tsv_status tsv_reshard_plan(int64_t n, int ks, int kd, int64_t* out, int max_cop
   }
   *n_copies = c;
   if (c > max_copies) return fail(TSV_E_INVAL, "plan has %d copies, buffer holds %d", c, max_copies);
+  return TSV_OK;
+}
+
+tsv_status tsv_a2a_plan(int which, int64_t Lt, int64_t Li, int k, int rank, int64_t* out, int max_ops, int* n_ops) {
+  if (!n_ops || (which != 1 && which != 2) || Lt < 0 || Li < 0 || k < 1 || rank < 0 || rank >= k ||
+      (max_ops > 0 && !out))
+    return fail(TSV_E_INVAL, "bad arguments");
+  std::vector<A2AOp> ops;
+  a2a_plan(which, Lt, Li, k, rank, ops);
+  *n_ops = (int)ops.size();
+  if ((int)ops.size() > max_ops) return fail(TSV_E_INVAL, "plan has %d ops, buffer holds %d", (int)ops.size(), max_ops);
+  for (size_t i = 0; i < ops.size(); ++i) {
+    out[4 * i + 0] = ops[i].peer;
+    out[4 * i + 1] = ops[i].send;
+    out[4 * i + 2] = ops[i].row0;
+    out[4 * i + 3] = ops[i].rows;
+  }
   return TSV_OK;
 }
 
