@@ -300,6 +300,241 @@ __global__ void __launch_bounds__(AT_THREADS, 1)
   if (warp == 2) tmem_dealloc<C::TMEM_COLS>(tmem);
 }
 
+// ------------------------------------------------------------------ v3: two query tiles per CTA
+// One CTA = one head x 256 queries as two 128-query tiles t = 0, 1 that share every K/V tile
+// (half the K/V traffic per query).  Two softmax warpgroups (warps 4-7: tile 0, 8-11: tile 1)
+// ping-pong with the tensor core: while WG0 turns S0_j into P0_j, the single MMA thread runs
+// PV1_{j-1} and S1_j, and vice versa.  P_j is written back into the S_t TMEM columns as bf16
+// (tcgen05.st) and consumed from TMEM by the PV MMA (A operand in TMEM), so no shared-memory P.
+// Because S_t{j+1} overwrites P_t{j} in TMEM, the MMA thread issues PV_t{j} before S_t{j+1}; the
+// in-order tcgen05 pipe makes "S_t{j} complete" imply "O_t holds tiles < j", so a rare rescale
+// of O (running max grew by > 2^8) needs no extra wait.
+// TMEM: S0 | S1 | O0 | O1 (128 + 128 + D + D fp32 columns).  Smem: Q0, Q1, 2 K/V stages.
+template <int D>
+struct FaCfg {
+  static constexpr int NSUB = D / 64;
+  static constexpr int Q_TILE = AT_BM * D * 2;
+  static constexpr int KV_TILE = AT_BN * D * 2;
+  static constexpr int OFF_Q = 0;                        // 2 tiles
+  static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // 2 stages
+  static constexpr int OFF_V = OFF_K + 2 * KV_TILE;      // 2 stages
+  static constexpr int OFF_BAR = OFF_V + 2 * KV_TILE;
+  static constexpr int SMEM = OFF_BAR + 256 + 1024;
+  static constexpr int O_COL = 256;
+};
+constexpr int FA_THREADS = 384;
+
+template <int D>
+__global__ void __launch_bounds__(FA_THREADS, 1)
+    attention_fa_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
+                        const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
+                        float scale_log2) {
+  using C = FaCfg<D>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
+  uint64_t* q_full = bars + 0;
+  uint64_t* kv_full = bars + 1;    // [2 stages]
+  uint64_t* kv_empty = bars + 3;   // [2 stages]
+  uint64_t* s_full = bars + 5;     // [2 q-tiles]
+  uint64_t* p_full = bars + 7;     // [2 q-tiles]
+  uint64_t* o_done = bars + 9;     // [2 q-tiles]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 12);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int head = blockIdx.y;
+  const int q0 = blockIdx.x * 2 * AT_BM;
+  const int n_tiles = (L + AT_BN - 1) / AT_BN;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmQ);
+    tma_prefetch_desc(&tmK);
+    tma_prefetch_desc(&tmV);
+    mbar_init(q_full, 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&kv_full[i], 1);
+      mbar_init(&kv_empty[i], 1);
+      mbar_init(&s_full[i], 1);
+      mbar_init(&p_full[i], 128);
+      mbar_init(&o_done[i], 1);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 2) tmem_alloc<512>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // ---------------------------------------------------------------- producer
+      mbar_arrive_expect_tx(q_full, 2 * C::Q_TILE);
+      for (int t = 0; t < 2; ++t)
+        for (int s = 0; s < C::NSUB; ++s)
+          tma_load_3d(&tmQ, q_full, sm + C::OFF_Q + t * C::Q_TILE + s * (AT_BM * 128), s * 64, head,
+                      q0 + t * AT_BM);
+      for (int j = 0; j < n_tiles; ++j) {
+        const int st = j & 1;
+        if (j >= 2) mbar_wait(&kv_empty[st], ((j - 2) >> 1) & 1);
+        mbar_arrive_expect_tx(&kv_full[st], 2 * C::KV_TILE);
+        for (int s = 0; s < C::NSUB; ++s) {
+          tma_load_3d(&tmK, &kv_full[st], sm + C::OFF_K + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
+                      j * AT_BN);
+          tma_load_3d(&tmV, &kv_full[st], sm + C::OFF_V + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
+                      j * AT_BN);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // ---------------------------------------------------------------- MMA issuer
+      constexpr uint32_t idesc_s = make_idesc_bf16(AT_BM, AT_BN);
+      constexpr uint32_t idesc_o = make_idesc_bf16_bmn(AT_BM, D);
+      mbar_wait(q_full, 0);
+      auto issue_s = [&](int t, int j) {
+        const uint32_t sQ = smem_u32(sm + C::OFF_Q + t * C::Q_TILE);
+        const uint32_t sK = smem_u32(sm + C::OFF_K + (j & 1) * C::KV_TILE);
+#pragma unroll
+        for (int kk = 0; kk < D / 16; ++kk) {
+          const uint32_t off = (kk >> 2) * (AT_BM * 128) + (kk & 3) * 32;
+          umma_bf16_ss(tmem + t * 128, make_sw128_desc(sQ + off), make_sw128_desc(sK + off), idesc_s, kk > 0);
+        }
+        umma_commit(&s_full[t]);
+      };
+      auto issue_pv = [&](int t, int j) {
+        mbar_wait(&p_full[t], j & 1);
+        tc_fence_after();
+        const uint32_t sV = smem_u32(sm + C::OFF_V + (j & 1) * C::KV_TILE);
+#pragma unroll
+        for (int kk = 0; kk < AT_BN / 16; ++kk)
+          umma_bf16_ts(tmem + C::O_COL + t * D, tmem + t * 128 + kk * 8,
+                       make_sw128_mn_desc(sV + kk * 2048, AT_BN * 128), idesc_o, (j | kk) != 0);
+      };
+      for (int j = 0; j < n_tiles; ++j) {
+        mbar_wait(&kv_full[j & 1], (j >> 1) & 1);
+        tc_fence_after();
+        for (int t = 0; t < 2; ++t) {
+          if (j > 0) {
+            issue_pv(t, j - 1);
+            if (t == 1) umma_commit(&kv_empty[(j - 1) & 1]);
+          }
+          issue_s(t, j);
+        }
+      }
+      for (int t = 0; t < 2; ++t) {
+        issue_pv(t, n_tiles - 1);
+        umma_commit(&o_done[t]);
+      }
+    }
+  } else if (warp >= 4) {
+    // ---------------------------------------------------------------- softmax WG t (thread = query row)
+    const int t = (warp - 4) >> 2;
+    const int wq = (warp - 4) & 3;
+    const int row = wq * 32 + lane;
+    const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
+    const uint32_t s_col = tmem + lane_base + t * 128;
+    const uint32_t o_col = tmem + lane_base + C::O_COL + t * D;
+    float m_ref = -FLT_MAX, l_sum = 0.f;
+    for (int j = 0; j < n_tiles; ++j) {
+      mbar_wait(&s_full[t], j & 1);
+      tc_fence_after();
+      uint32_t sr[4][32];
+#pragma unroll
+      for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
+      tmem_ld_wait();
+      const int kbase = j * AT_BN;
+      float mr0 = -FLT_MAX, mr1 = -FLT_MAX;
+      if (kbase + AT_BN <= L) {
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+#pragma unroll
+          for (int i = 0; i < 32; i += 2) {
+            mr0 = fmaxf(mr0, __uint_as_float(sr[c][i]));
+            mr1 = fmaxf(mr1, __uint_as_float(sr[c][i + 1]));
+          }
+      } else {
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+#pragma unroll
+          for (int i = 0; i < 32; ++i) {
+            if (kbase + c * 32 + i >= L) sr[c][i] = __float_as_uint(-INFINITY);
+            mr0 = fmaxf(mr0, __uint_as_float(sr[c][i]));
+          }
+      }
+      const float mt = fmaxf(mr0, mr1) * scale_log2;
+      bool rescale = false;
+      float alpha = 1.f;
+      if (j == 0) {
+        m_ref = mt;
+      } else if (mt > m_ref + RESCALE_THRESHOLD) {
+        rescale = true;
+        alpha = exp2f(m_ref - mt);
+        m_ref = mt;
+      }
+      l_sum *= alpha;
+      // P = 2^(s * scale_log2 - m_ref) as packed bf16 pairs, in place of S (columns 0..63 of S_t)
+      float ls0 = 0.f, ls1 = 0.f;
+      const float neg_m = -m_ref;
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int i = 0; i < 32; i += 2) {
+          const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
+          const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
+          ls0 += p0;
+          ls1 += p1;
+          sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);  // packed P overwrites consumed S
+        }
+      l_sum += ls0 + ls1;
+      // S_t{j} complete => PV_t{j-1} complete (in-order pipe): O_t can be rescaled right away
+      if (__any_sync(0xffffffffu, rescale)) {
+#pragma unroll
+        for (int c = 0; c < D / 32; ++c) {
+          uint32_t ov[32];
+          tmem_ld32(o_col + c * 32, ov);
+          tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 32; ++i) ov[i] = __float_as_uint(__uint_as_float(ov[i]) * alpha);
+          tmem_st32(o_col + c * 32, ov);
+        }
+      }
+      tmem_st32(s_col, sr[0]);
+      tmem_st32(s_col + 32, sr[1]);
+      tmem_st_wait();
+      tc_fence_before();
+      mbar_arrive(&p_full[t]);
+    }
+    // epilogue: O_t / l -> bf16
+    mbar_wait(&o_done[t], 0);
+    tc_fence_after();
+    const float inv = 1.f / l_sum;
+    const int grow = q0 + t * AT_BM + row;
+#pragma unroll
+    for (int c = 0; c < D / 32; ++c) {
+      uint32_t ov[32];
+      tmem_ld32(o_col + c * 32, ov);
+      tmem_ld_wait();
+      if (grow < L) {
+        uint4* dst = reinterpret_cast<uint4*>(o + (long long)grow * ldo + head * D + c * 32);
+#pragma unroll
+        for (int qd = 0; qd < 4; ++qd) {
+          uint4 v;
+          v.x = pack_bf16x2(__uint_as_float(ov[qd * 8 + 0]) * inv, __uint_as_float(ov[qd * 8 + 1]) * inv);
+          v.y = pack_bf16x2(__uint_as_float(ov[qd * 8 + 2]) * inv, __uint_as_float(ov[qd * 8 + 3]) * inv);
+          v.z = pack_bf16x2(__uint_as_float(ov[qd * 8 + 4]) * inv, __uint_as_float(ov[qd * 8 + 5]) * inv);
+          v.w = pack_bf16x2(__uint_as_float(ov[qd * 8 + 6]) * inv, __uint_as_float(ov[qd * 8 + 7]) * inv);
+          dst[qd] = v;
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 2) tmem_dealloc<512>(tmem);
+}
+
 // ------------------------------------------------------------------ host
 static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -329,8 +564,7 @@ static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L
 
 template <int D>
 static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv, bf16* o,
-                     long long ldo, int L, int H, cudaStream_t s) {
-  using C = AttnCfg<D>;
+                     long long ldo, int L, int H, int version, cudaStream_t s) {
   CUtensorMap tq, tk, tv;
   if (make_tmap_heads(&tq, q, D, H, L, ldq) || make_tmap_heads(&tk, k, D, H, L, ldk) ||
       make_tmap_heads(&tv, v, D, H, L, ldv))
@@ -339,24 +573,32 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
   int dev = 0;
   cudaGetDevice(&dev);
   if (!(done >> dev & 1ull)) {
-    cudaFuncSetAttribute(attention_tc_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+    cudaFuncSetAttribute(attention_tc_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, AttnCfg<D>::SMEM);
+    cudaFuncSetAttribute(attention_fa_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, FaCfg<D>::SMEM);
     done |= 1ull << dev;
   }
   const float scale_log2 = (1.0f / sqrtf((float)D)) * 1.4426950408889634f;
-  dim3 grid((L + AT_BM - 1) / AT_BM, H);
-  attention_tc_kernel<D><<<grid, AT_THREADS, C::SMEM, s>>>(tq, tk, tv, o, ldo, L, scale_log2);
+  if (version == 2) {
+    dim3 grid((L + AT_BM - 1) / AT_BM, H);
+    attention_tc_kernel<D><<<grid, AT_THREADS, AttnCfg<D>::SMEM, s>>>(tq, tk, tv, o, ldo, L, scale_log2);
+  } else {
+    dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H);
+    attention_fa_kernel<D><<<grid, FA_THREADS, FaCfg<D>::SMEM, s>>>(tq, tk, tv, o, ldo, L, scale_log2);
+  }
   return 0;
 }
 
-// returns 0 if the tensor-core path was launched, nonzero if the layout is unsupported by TMA
+// returns 0 if the tensor-core path was launched, nonzero if the layout is unsupported by TMA.
+// version 3: two query tiles per CTA, P in TMEM (the step's kernel); version 2: one query tile,
+// P in shared memory (kept for comparison).
 int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
-                        bf16* o, long long ldo, int L, int H, int D, cudaStream_t s) {
+                     bf16* o, long long ldo, int L, int H, int D, cudaStream_t s, int version) {
   if (L <= 0 || H <= 0) return 0;
   if (((ldq | ldk | ldv) * 2) % 16 || ((reinterpret_cast<uintptr_t>(q) | reinterpret_cast<uintptr_t>(k) |
                                         reinterpret_cast<uintptr_t>(v)) & 15))
     return -1;
-  if (D == 128) return launch_tc<128>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, s);
-  if (D == 64) return launch_tc<64>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, s);
+  if (D == 128) return launch_tc<128>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, s);
+  if (D == 64) return launch_tc<64>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, s);
   return -1;
 }
 

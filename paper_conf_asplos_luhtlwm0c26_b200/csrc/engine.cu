@@ -1510,7 +1510,7 @@ tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t l
                          reinterpret_cast<cudaStream_t>(stream));
   } else if (attention_launch(reinterpret_cast<const bf16*>(q), ldq, reinterpret_cast<const bf16*>(k), ldk,
                               reinterpret_cast<const bf16*>(v), ldv, reinterpret_cast<bf16*>(o), ldo, L, H, D,
-                              reinterpret_cast<cudaStream_t>(stream))) {
+                              reinterpret_cast<cudaStream_t>(stream), impl == 2 ? 2 : 3)) {
     return fail(TSV_E_INVAL, "attention: operands must be 16-byte aligned with 16-byte row strides");
   }
   CK(cudaGetLastError());

@@ -45,11 +45,21 @@ struct GemmMaps {
   CUtensorMap B[2];
 };
 
+// Rasterisation: groups of GROUP_N weight-column tiles; inside a group the n index varies fastest,
+// then m.  A wave of 148 concurrent tiles therefore touches <= GROUP_N weight tiles and
+// ~148/GROUP_N activation row-blocks, both L2-resident, so activations are streamed from HBM about
+// num_n / GROUP_N times instead of num_n times (measured: 2.8 GB -> algorithmic for 2048^2 fc1).
+constexpr int GROUP_N = 8;
 __device__ __forceinline__ void decode_tile(const GemmArgs& a, int t, int& p, int& m_blk, int& n_blk) {
   p = (a.nprob > 1 && t >= a.tile0[1]) ? 1 : 0;
   const int lt = t - a.tile0[p];
-  m_blk = lt % a.num_m[p];
-  n_blk = lt / a.num_m[p];
+  const int nm = a.num_m[p];
+  const int group = lt / (GROUP_N * nm);
+  const int first_n = group * GROUP_N;
+  const int gsize = min(GROUP_N, a.num_n - first_n);
+  const int r = lt - group * GROUP_N * nm;
+  m_blk = r / gsize;
+  n_blk = first_n + r % gsize;
 }
 
 __device__ __forceinline__ void add_bias32(const bf16* bias, int n0, float (&v)[32]) {

@@ -98,7 +98,7 @@ void qk_norm_rope_launch(bf16* qkv, long long ld, int rows, int n_first, int H, 
 // attention_mma_launch: the mma.sync (FA2-style) baseline kept for comparison.
 // q(l, h) at q + l*ldq + h*D (same for k, v, o). L rows.
 int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
-                     bf16* o, long long ldo, int L, int H, int D, cudaStream_t s);
+                     bf16* o, long long ldo, int L, int H, int D, cudaStream_t s, int version = 3);
 void attention_mma_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
                           bf16* o, long long ldo, int L, int H, int D, cudaStream_t s);
 
