@@ -33,13 +33,18 @@ __global__ void __launch_bounds__(T) ln_mod_kernel(const float* __restrict__ x, 
   const int t = threadIdx.x;
   constexpr int h = 4 * T * NV;
   const float4* xr = reinterpret_cast<const float4*>(x + (long long)row * ldx);
-  float4 v[NV];
-  float s = 0.f;
+  float4 v[NV], shv[NV], scv[NV];
+#pragma unroll
+  for (int i = 0; i < NV; ++i) v[i] = xr[i * T + t];
+  // the modulation vectors are independent of the row statistics: issue their loads up front
 #pragma unroll
   for (int i = 0; i < NV; ++i) {
-    v[i] = xr[i * T + t];
-    s += (v[i].x + v[i].y) + (v[i].z + v[i].w);
+    shv[i] = __ldg(reinterpret_cast<const float4*>(shift) + i * T + t);
+    scv[i] = __ldg(reinterpret_cast<const float4*>(scale) + i * T + t);
   }
+  float s = 0.f;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) s += (v[i].x + v[i].y) + (v[i].z + v[i].w);
   const float mean = block_sum<T>(s, red) * (1.0f / h);
   float q = 0.f;
 #pragma unroll
@@ -49,12 +54,10 @@ __global__ void __launch_bounds__(T) ln_mod_kernel(const float* __restrict__ x, 
   }
   const float rstd = rsqrtf(block_sum<T>(q, red) * (1.0f / h) + 1e-6f);
   uint2* ur = reinterpret_cast<uint2*>(u + (long long)row * ldu);
-  const float4* sh4 = reinterpret_cast<const float4*>(shift);
-  const float4* sc4 = reinterpret_cast<const float4*>(scale);
 #pragma unroll
   for (int i = 0; i < NV; ++i) {
     const int c = i * T + t;
-    float4 sh = __ldg(sh4 + c), sc = __ldg(sc4 + c);
+    const float4 sh = shv[i], sc = scv[i];
     float a = (v[i].x - mean) * rstd * (1.f + sc.x) + sh.x;
     float b = (v[i].y - mean) * rstd * (1.f + sc.y) + sh.y;
     float cc = (v[i].z - mean) * rstd * (1.f + sc.z) + sh.z;
@@ -87,7 +90,7 @@ void ln_mod_launch(const float* x, long long ldx, bf16* u, long long ldu, const 
                    int M, int h, cudaStream_t s) {
   if (M <= 0) return;
   switch (h) {
-    case 3072: ln_mod_kernel<128, 6><<<M, 128, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
+    case 3072: ln_mod_kernel<256, 3><<<M, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
     case 1536: ln_mod_kernel<128, 3><<<M, 128, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
     case 256: ln_mod_kernel<32, 2><<<M, 32, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
     default: ln_mod_generic<<<(M + 7) / 8, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M, h); break;
