@@ -198,6 +198,11 @@ tsv_status tsv_debug_read_weight(tsv_engine* eng, int tensor_id, uint16_t* host,
  * summed device ms, launches, algorithmic FLOPs and algorithmic HBM bytes per class. */
 #define TSV_PROF_CLASSES 6
 tsv_status tsv_engine_profile(tsv_engine* eng, int enable);
+/* When a group has exactly one rank in this process, each step is captured once as a CUDA graph
+ * (per request, group and buffer set) and replayed for later steps; the step index is read from
+ * device memory, so one graph serves every step.  enable = 0 launches kernels directly.  Default
+ * on; profiling (tsv_engine_profile) always launches directly. */
+tsv_status tsv_engine_set_graphs(tsv_engine* eng, int enable);
 tsv_status tsv_engine_profile_read(tsv_engine* eng, double* ms, int64_t* launches, double* flops, double* bytes);
 /* Number of kernels this engine launched so far (all slots). */
 tsv_status tsv_engine_kernel_count(tsv_engine* eng, int64_t* count);

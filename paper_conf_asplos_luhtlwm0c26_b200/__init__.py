@@ -183,6 +183,9 @@ class Engine:
 
     PROF_CLASSES = ("gemm", "attention", "ln_mod", "qk_norm_rope", "a2a", "other")
 
+    def set_graphs(self, enable: bool = True):
+        check(lib.tsv_engine_set_graphs(self.h, int(enable)))
+
     def profile(self, enable: bool = True):
         check(lib.tsv_engine_profile(self.h, int(enable)))
 

@@ -140,7 +140,13 @@ struct Slot {
 struct ReqDev {
   DevBuf mod;       // fp32 [S, n_mod]
   DevBuf dt;        // fp32 [S]
+  DevBuf cur;       // fp32 [n_mod + 1]: this step's modulation row and dt (selected on device)
+  DevBuf step;      // int: the step index the next launch runs
   bool ready = false;
+  // CUDA graph of the whole step for this (request, slot, group, buffers); replayed every step
+  cudaGraphExec_t gexec = nullptr;
+  uint64_t gkey = 0;
+  int64_t gkernels = 0;
 };
 // per (request, slot, shard): state that depends on the group position
 struct ReqShard {
@@ -198,6 +204,7 @@ struct tsv_engine {
   int64_t kernel_count = 0;
   // per-kernel-class profiling (tsv_engine_profile)
   bool prof = false;
+  bool graphs = true;  // replay each step as a CUDA graph when a group has one local rank
   struct ProfRec { int cls; int device; cudaEvent_t a, b; };
   std::vector<ProfRec> prof_recs;
   std::map<int, std::vector<cudaEvent_t>> ev_pool;  // by device
@@ -326,6 +333,8 @@ static tsv_status ensure_reqdev(tsv_engine* e, Request& R, int si) {
   CK(cudaSetDevice(s.device));
   TRY(dev_alloc(rd.mod, s.device, (size_t)S * m.n_mod * 4));
   TRY(dev_alloc(rd.dt, s.device, (size_t)S * 4));
+  TRY(dev_alloc(rd.cur, s.device, ((size_t)m.n_mod + 4) * 4));
+  TRY(dev_alloc(rd.step, s.device, 16));
   // host-side: sinusoidal embeddings e(t_s), e(g) (fp64 -> bf16), y (bf16), dt
   const int Sp = S;
   std::vector<uint16_t> et((size_t)Sp * 256), eg((size_t)Sp * 256), ey((size_t)Sp * m.vec);
@@ -631,6 +640,17 @@ static tsv_status run_step(StepEnv& E) {
   const Model& m = e->model;
   const int h = m.h, F = m.F;
   const int64_t ldc = h + F;
+  // this step's modulation row and dt, selected on the device from the step index (so one
+  // captured graph serves every step of the request)
+  for (auto& c : E.rc) {
+    Slot& s = *c.s;
+    CK(cudaSetDevice(s.device));
+    ProfScope ps(e, s, KC_OTHER, 0.0, 8.0 * m.n_mod, 2);
+    const int* step_dev = reinterpret_cast<const int*>(c.rd->step.p);
+    float* cur = reinterpret_cast<float*>(c.rd->cur.p);
+    select_row_launch(reinterpret_cast<const float*>(c.rd->mod.p), m.n_mod, step_dev, cur, m.n_mod, s.stream);
+    select_row_launch(reinterpret_cast<const float*>(c.rd->dt.p), 1, step_dev, cur + m.n_mod, 1, s.stream);
+  }
   // a1: embeddings
   for (auto& c : E.rc) {
     Slot& s = *c.s;
@@ -727,7 +747,7 @@ static tsv_status run_step(StepEnv& E) {
     lnmod(e, s, c.x + c.nt * h, c.u, md, md + h, (int)c.ni);
     TRY(gemm(e, s, c.u, h, e->W(s, 18), h, (int)c.ni, m.in, h,
              epi_of(EPI_EULER, c.sh->lat.p, m.in, e->W(s, 19), nullptr, c.sh->vel.p, m.in, 0,
-                    reinterpret_cast<const float*>(c.rd->dt.p) + E.step)));
+                    reinterpret_cast<const float*>(c.rd->cur.p) + m.n_mod)));
   }
   for (auto& c : E.rc) CK(cudaGetLastError());
   return TSV_OK;
@@ -883,23 +903,66 @@ static tsv_status do_step(tsv_engine* e, Request& R, int step, int gi, tsv_event
     c.recv = reinterpret_cast<bf16*>(s.ws.recv.p);
     c.obuf = reinterpret_cast<bf16*>(s.ws.obuf.p);
     c.orecv = reinterpret_cast<bf16*>(s.ws.orecv.p);
-    c.mod = reinterpret_cast<const float*>(c.rd->mod.p) + (int64_t)step * m.n_mod;
+    c.mod = reinterpret_cast<const float*>(c.rd->cur.p);
     E.rc.push_back(c);
   }
-  // each slot's stream must follow the request's previous work on that slot
+  // each slot's stream must follow the request's previous work on that slot; then publish the
+  // step index (pageable source: staged at call time, so the host value can change right after)
   for (auto& c : E.rc) {
+    CK(cudaSetDevice(c.s->device));
     auto it = R.last.find(c.si);
-    if (it != R.last.end()) {
-      CK(cudaSetDevice(c.s->device));
-      CK(cudaStreamWaitEvent(c.s->stream, it->second, 0));
-    }
+    if (it != R.last.end()) CK(cudaStreamWaitEvent(c.s->stream, it->second, 0));
+    int st = step;
+    CK(cudaMemcpyAsync(c.rd->step.p, &st, sizeof(int), cudaMemcpyHostToDevice, c.s->stream));
   }
-  TRY(run_step(E));
+  if (e->graphs && E.rc.size() == 1 && !e->prof) {
+    // one local rank: replay (or capture once) the whole step as a CUDA graph
+    RankCtx& c = E.rc[0];
+    ReqDev& rd = *c.rd;
+    uint64_t key = 1469598103934665603ull;
+    auto mix = [&](uint64_t v) { key = (key ^ v) * 1099511628211ull; };
+    const void* ptrs[] = {c.x, c.u, c.qkv, c.cat, c.hbuf, c.latb, c.pack, c.recv, c.obuf, c.orecv,
+                          c.sh->lat.p, c.sh->vel.p, c.sh->T.p, c.sh->cosb.p, c.sh->sinb.p, rd.mod.p, rd.cur.p,
+                          rd.step.p};
+    for (const void* p : ptrs) mix(reinterpret_cast<uintptr_t>(p));
+    mix((uint64_t)gi);
+    mix((uint64_t)c.rows);
+    if (!rd.gexec || rd.gkey != key) {
+      if (rd.gexec) { cudaGraphExecDestroy(rd.gexec); rd.gexec = nullptr; }
+      CK(cudaSetDevice(c.s->device));
+      const int64_t k0 = e->kernel_count;
+      CK(cudaStreamBeginCapture(c.s->stream, cudaStreamCaptureModeThreadLocal));
+      tsv_status st = run_step(E);
+      cudaGraph_t graph = nullptr;
+      cudaError_t ce = cudaStreamEndCapture(c.s->stream, &graph);
+      if (st != TSV_OK) { if (graph) cudaGraphDestroy(graph); return st; }
+      if (ce != cudaSuccess) return fail(TSV_E_CUDA, "step capture: %s", cudaGetErrorString(ce));
+      ce = cudaGraphInstantiate(&rd.gexec, graph, 0);
+      cudaGraphDestroy(graph);
+      if (ce != cudaSuccess) { rd.gexec = nullptr; return fail(TSV_E_CUDA, "graph instantiate: %s", cudaGetErrorString(ce)); }
+      rd.gkey = key;
+      rd.gkernels = e->kernel_count - k0;
+      e->kernel_count = k0;
+    }
+    CK(cudaGraphLaunch(rd.gexec, c.s->stream));
+    e->kernel_count += rd.gkernels;
+  } else {
+    TRY(run_step(E));
+  }
   for (auto& c : E.rc) TRY(record_last(e, R, c.si));
   R.next_step = step + 1;
   R.has_velocity = true;
   if (done) TRY(new_event(e, g.local_slots, done));
   return TSV_OK;
+}
+
+static void release_reqdev(ReqDev& d) {
+  if (d.gexec) cudaGraphExecDestroy(d.gexec);
+  d.gexec = nullptr;
+  d.mod.release();
+  d.dt.release();
+  d.cur.release();
+  d.step.release();
 }
 
 }  // namespace tsv
@@ -983,7 +1046,7 @@ void tsv_engine_destroy(tsv_engine* e) {
     cudaStreamSynchronize(s.stream);
   }
   for (auto& kv : e->requests) {
-    for (auto& d : kv.second.dev) { d.second.mod.release(); d.second.dt.release(); }
+    for (auto& d : kv.second.dev) release_reqdev(d.second);
     for (auto& sh : kv.second.shard) {
       sh.second.lat.release(); sh.second.vel.release(); sh.second.T.release();
       sh.second.cosb.release(); sh.second.sinb.release();
@@ -1270,7 +1333,7 @@ tsv_status tsv_request_destroy(tsv_engine* e, tsv_request r) {
   if (it == e->requests.end()) return fail(TSV_E_INVAL, "unknown request %lld", (long long)r);
   Request& R = it->second;
   for (auto& l : R.last) { cudaEventSynchronize(l.second); cudaEventDestroy(l.second); }
-  for (auto& d : R.dev) { d.second.mod.release(); d.second.dt.release(); }
+  for (auto& d : R.dev) release_reqdev(d.second);
   for (auto& sh : R.shard) {
     sh.second.lat.release(); sh.second.vel.release(); sh.second.T.release();
     sh.second.cosb.release(); sh.second.sinb.release();
@@ -1390,6 +1453,12 @@ tsv_status tsv_debug_read_weight(tsv_engine* e, int id, uint16_t* host, size_t n
   Slot& s = e->slots[0];
   CK(cudaSetDevice(s.device));
   CK(cudaMemcpy(host, reinterpret_cast<const bf16*>(s.ds->weights.p) + t->offset, n * 2, cudaMemcpyDeviceToHost));
+  return TSV_OK;
+}
+
+tsv_status tsv_engine_set_graphs(tsv_engine* e, int enable) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  e->graphs = enable != 0;
   return TSV_OK;
 }
 
