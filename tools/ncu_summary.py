@@ -43,21 +43,29 @@ def launches(path):
     rows = list(csv.reader(open(path)))
     hi = [i for i, r in enumerate(rows) if "Kernel Name" in r][0]
     h, data = rows[hi], rows[hi + 1:]
-    ki, vi, ui = h.index("Kernel Name"), h.index("Metric Value"), h.index("Metric Unit")
-    tot, cnt = collections.defaultdict(float), collections.Counter()
+    ii, ki, mi, vi, ui = (h.index(c) for c in ("ID", "Kernel Name", "Metric Name", "Metric Value", "Metric Unit"))
+    recs = collections.defaultdict(dict)
     for r in data:
         if len(r) <= vi:
             continue
         v = float(r[vi].replace(",", ""))
-        v *= {"ns": 1e-3, "nsecond": 1e-3, "us": 1.0, "usecond": 1.0, "ms": 1e3, "msecond": 1e3}.get(r[ui], 1.0)
-        c = classify(r[ki])
-        tot[c] += v
+        unit = r[ui]
+        v *= {"ns": 1e-3, "nsecond": 1e-3, "us": 1.0, "usecond": 1.0, "ms": 1e3, "msecond": 1e3,
+              "byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1.0)
+        recs[r[ii]]["name"] = r[ki]
+        recs[r[ii]][r[mi]] = v
+    tot, cnt, dram = collections.defaultdict(float), collections.Counter(), collections.defaultdict(float)
+    for rec in recs.values():
+        c = classify(rec["name"])
+        tot[c] += rec.get("gpu__time_duration.sum", 0.0)
+        dram[c] += rec.get("dram__bytes_read.sum", 0.0) + rec.get("dram__bytes_write.sum", 0.0)
         cnt[c] += 1
     s = sum(tot.values())
-    print(f"{'class':24s} {'launches':>8s} {'us':>12s} {'share':>7s}")
+    print(f"{'class':24s} {'launches':>8s} {'us':>12s} {'share':>7s} {'DRAM MB/launch':>15s}")
     for k, v in sorted(tot.items(), key=lambda x: -x[1]):
-        print(f"{k:24s} {cnt[k]:8d} {v:12.1f} {100 * v / s:6.1f}%")
+        print(f"{k:24s} {cnt[k]:8d} {v:12.1f} {100 * v / s:6.1f}% {dram[k] / cnt[k] / 1e6:15.2f}")
     print(f"{'total (serialised, cold)':24s} {sum(cnt.values()):8d} {s:12.1f}")
+    return tot, cnt, dram
 
 
 def report(path):

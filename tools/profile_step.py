@@ -20,6 +20,7 @@ ap.add_argument("--steps", type=int, default=1)
 ap.add_argument("--model", default="flux")
 a = ap.parse_args()
 eng = tsv.Engine(a.model, devices=[0] * a.k)
+eng.set_graphs(False)   # direct launches: one ncu record per kernel
 g = eng.group_create(list(range(a.k)))
 req = eng.request_create(a.res, a.res, num_steps=2 + a.steps, seed=1000)
 for s in range(2):
