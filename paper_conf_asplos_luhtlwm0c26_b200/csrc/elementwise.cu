@@ -26,11 +26,16 @@ __device__ __forceinline__ float block_sum(float v, float* red) {
 
 template <int T, int NV>
 __global__ void __launch_bounds__(T) ln_mod_kernel(const float* __restrict__ x, long long ldx, bf16* __restrict__ u,
-                                                   long long ldu, const float* __restrict__ shift,
-                                                   const float* __restrict__ scale, int M) {
+                                                   long long ldu, const float* __restrict__ shift0,
+                                                   const float* __restrict__ scale0, const float* __restrict__ shift1,
+                                                   const float* __restrict__ scale1, int n_first) {
   __shared__ float red[T / 32];
   const int row = blockIdx.x;
   const int t = threadIdx.x;
+  // rows [0, n_first) take (shift0, scale0), the others (shift1, scale1): both streams of a
+  // double block in one launch
+  const float* shift = row < n_first ? shift0 : shift1;
+  const float* scale = row < n_first ? scale0 : scale1;
   constexpr int h = 4 * T * NV;
   const float4* xr = reinterpret_cast<const float4*>(x + (long long)row * ldx);
   float4 v[NV], shv[NV], scv[NV];
@@ -68,11 +73,15 @@ __global__ void __launch_bounds__(T) ln_mod_kernel(const float* __restrict__ x, 
 
 // generic fallback (h multiple of 128): two passes over global memory
 __global__ void __launch_bounds__(256) ln_mod_generic(const float* __restrict__ x, long long ldx, bf16* __restrict__ u,
-                                                      long long ldu, const float* __restrict__ shift,
-                                                      const float* __restrict__ scale, int M, int h) {
+                                                      long long ldu, const float* __restrict__ shift0,
+                                                      const float* __restrict__ scale0,
+                                                      const float* __restrict__ shift1,
+                                                      const float* __restrict__ scale1, int n_first, int M, int h) {
   const int row = blockIdx.x * 8 + (threadIdx.x >> 5);
   const int lane = threadIdx.x & 31;
   if (row >= M) return;
+  const float* shift = row < n_first ? shift0 : shift1;
+  const float* scale = row < n_first ? scale0 : scale1;
   const float* xr = x + (long long)row * ldx;
   float s = 0.f;
   for (int c = lane; c < h; c += 32) s += xr[c];
@@ -86,15 +95,29 @@ __global__ void __launch_bounds__(256) ln_mod_generic(const float* __restrict__ 
     u[(long long)row * ldu + c] = __float2bfloat16_rn((xr[c] - mean) * rstd * (1.f + scale[c]) + shift[c]);
 }
 
-void ln_mod_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift, const float* scale,
-                   int M, int h, cudaStream_t s) {
+void ln_mod2_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift0,
+                    const float* scale0, const float* shift1, const float* scale1, int n_first, int M, int h,
+                    cudaStream_t s) {
   if (M <= 0) return;
   switch (h) {
-    case 3072: ln_mod_kernel<256, 3><<<M, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
-    case 1536: ln_mod_kernel<128, 3><<<M, 128, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
-    case 256: ln_mod_kernel<32, 2><<<M, 32, 0, s>>>(x, ldx, u, ldu, shift, scale, M); break;
-    default: ln_mod_generic<<<(M + 7) / 8, 256, 0, s>>>(x, ldx, u, ldu, shift, scale, M, h); break;
+    case 3072:
+      ln_mod_kernel<256, 3><<<M, 256, 0, s>>>(x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
+      break;
+    case 1536:
+      ln_mod_kernel<128, 3><<<M, 128, 0, s>>>(x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
+      break;
+    case 256:
+      ln_mod_kernel<32, 2><<<M, 32, 0, s>>>(x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
+      break;
+    default:
+      ln_mod_generic<<<(M + 7) / 8, 256, 0, s>>>(x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first, M, h);
+      break;
   }
+}
+
+void ln_mod_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift, const float* scale,
+                   int M, int h, cudaStream_t s) {
+  ln_mod2_launch(x, ldx, u, ldu, shift, scale, shift, scale, M, M, h, s);
 }
 
 // ------------------------------------------------------------------ a4: QK-RMSNorm + RoPE (+ Ulysses pack)

@@ -299,6 +299,10 @@ static void lnmod(tsv_engine* e, Slot& s, const float* x, bf16* u, const float* 
   ln_mod_launch(x, h, u, h, shift, scale, n, h, s.stream);
 }
 
+struct StepEnv;
+struct RankCtx;
+static void lnmod2(StepEnv& E, RankCtx& c, int64_t mod_txt, int64_t mod_img, int chunk);
+
 static GemmEpi epi_of(int mode, void* out0, long long ld0, const bf16* bias, const float* gate = nullptr,
                       void* out1 = nullptr, long long ld1 = 0, int n_split = 0, const float* scalar = nullptr) {
   GemmEpi g;
@@ -635,6 +639,18 @@ static GemmEpi qk_fused(StepEnv& E, RankCtx& c, GemmEpi epi, int64_t r0, const b
   return epi;
 }
 
+// a2 / a9 of a double block for both streams in one launch: rows [0, nt) use the txt stream's
+// (shift, scale) = modulation chunks (chunk, chunk + 1), rows [nt, rows) the img stream's.
+static void lnmod2(StepEnv& E, RankCtx& c, int64_t mod_txt, int64_t mod_img, int chunk) {
+  tsv_engine* e = E.e;
+  const int h = e->model.h;
+  if (!c.rows) return;
+  const float* mt = c.mod + mod_txt + (int64_t)chunk * h;
+  const float* mi = c.mod + mod_img + (int64_t)chunk * h;
+  ProfScope ps(e, *c.s, KC_LNMOD, 0.0, (double)c.rows * h * 6.0 + 16.0 * h);
+  ln_mod2_launch(c.x, h, c.u, h, mt, mt + h, mi, mi + h, (int)c.nt, (int)c.rows, h, c.s->stream);
+}
+
 static tsv_status run_step(StepEnv& E) {
   tsv_engine* e = E.e;
   const Model& m = e->model;
@@ -673,11 +689,10 @@ static tsv_status run_step(StepEnv& E) {
       Slot& s = *c.s;
       CK(cudaSetDevice(s.device));
       GemmProblem pq[2];
+      lnmod2(E, c, m.mod_double(j, 1), m.mod_double(j, 0), 0);   // a2 for both streams: rows [txt; img]
       for (int st = 0; st < 2; ++st) {  // 0 = img, 1 = txt
         const int base = double_base(j, st);
         const int64_t r0 = st == 0 ? c.nt : 0, n = st == 0 ? c.ni : c.nt;
-        const float* md = c.mod + m.mod_double(j, st);
-        if (n) lnmod(e, s, c.x + r0 * h, c.u + r0 * h, md + 0 * h, md + 1 * h, (int)n);
         pq[st] = {c.u + r0 * h, h, e->W(s, base + 2), h, (int)n,
                   qk_fused(E, c, epi_of(EPI_STORE_BF16, c.qkv + r0 * 3 * h, 3 * h, e->W(s, base + 3)), r0,
                            e->W(s, base + 4), e->W(s, base + 5))};
@@ -704,11 +719,7 @@ static tsv_status run_step(StepEnv& E) {
                   epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 11), md + 5 * h)};
       }
       TRY(gemm_multi(e, s, pp, 2, h, h));        // a8: out-proj + gated residual, both streams
-      for (int st = 0; st < 2; ++st) {           // a9: LN-modulate both streams
-        const int64_t r0 = st == 0 ? c.nt : 0, n = st == 0 ? c.ni : c.nt;
-        const float* md = c.mod + m.mod_double(j, st);
-        if (n) lnmod(e, s, c.x + r0 * h, c.u + r0 * h, md + 3 * h, md + 4 * h, (int)n);
-      }
+      lnmod2(E, c, m.mod_double(j, 1), m.mod_double(j, 0), 3);   // a9: LN-modulate both streams
       TRY(gemm_multi(e, s, p1, 2, F, h));        // fc1 + GELU
       TRY(gemm_multi(e, s, p2, 2, h, F));        // fc2 + gated residual
     }

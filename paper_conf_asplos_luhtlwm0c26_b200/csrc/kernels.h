@@ -83,6 +83,10 @@ void gemm_launch(const GemmPlan& p, cudaStream_t s);
 // u[m, :] = bf16( LN(x[m, :]) * (1 + scale) + shift ), x fp32 row stride ldx, u row stride ldu
 void ln_mod_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift, const float* scale,
                    int M, int h, cudaStream_t s);
+// same, rows [0, n_first) modulated by (shift0, scale0), rows [n_first, M) by (shift1, scale1)
+void ln_mod2_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift0,
+                    const float* scale0, const float* shift1, const float* scale1, int n_first, int M, int h,
+                    cudaStream_t s);
 
 // In-place on a qkv buffer [rows, 3*H*D] (row stride ld): q,k <- RoPE(RMSNorm(.) * g).
 // Rows [0, n_first) use gains (gq0, gk0), rows [n_first, rows) use (gq1, gk1).
