@@ -30,7 +30,7 @@ struct GemmCfg {
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int STAGES = (BN == 256) ? 4 : (BN == 128 ? 6 : 8);
   static constexpr int TMEM_COLS = 2 * BN;  // power of two >= 32
-  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ + 4 * 32 * 36 * 4;
 };
 
 // Up to two problems with the same N and K (e.g. the img and txt streams of a double block)
@@ -96,10 +96,35 @@ __device__ __forceinline__ bf16* qkv_dst(const GemmEpi& e, int row, int n) {
   return e.pack + ((((long long)dst * e.pack_rows + e.pack_row0 + row) * 3 + part) * hk + hl) * D + d;
 }
 
+// ------------------------------------------------------------------ epilogue (coalesced via smem)
+// A tcgen05.ld 32x32b chunk gives thread i the 32 columns of row i.  Writing those straight to
+// global memory makes every warp store touch 32 rows (one 16-byte piece per row).  Instead each
+// epilogue warp stages its 32 x 32 fp32 block in shared memory and re-reads it so that 8 lanes
+// cover one row: every global load/store of the epilogue is a full 128-byte (fp32) or 64-byte
+// (bf16) row segment.
+constexpr int STG_PITCH = 36;                  // floats per staged row (16-byte aligned, spreads banks)
+constexpr int STG_FLOATS = 32 * STG_PITCH;     // per epilogue warp
+constexpr int STG_BYTES = 4 * STG_FLOATS * 4;  // 4 epilogue warps
+
+__device__ __forceinline__ void stage_write(float* stg, int lane, const float (&v)[32]) {
+  float4* rowp = reinterpret_cast<float4*>(stg + lane * STG_PITCH);
+#pragma unroll
+  for (int q = 0; q < 8; ++q) rowp[q] = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+}
+__device__ __forceinline__ float4 stage_read(const float* stg, int rr, int c4) {
+  return *reinterpret_cast<const float4*>(stg + rr * STG_PITCH + c4 * 4);
+}
+__device__ __forceinline__ uint2 pack4_bf16(float4 a) {
+  return make_uint2(pack_bf16x2(a.x, a.y), pack_bf16x2(a.z, a.w));
+}
+
 // Fused a3 + a4: one thread = one row; a head of D columns is D/32 TMEM chunks.  Pass 1 sums the
-// squares of y = acc + b over the head, pass 2 re-reads TMEM and writes RoPE(y * rsqrt(ms + eps) * g).
-__device__ __forceinline__ void epilogue_qk_head(const GemmEpi& e, int M, int row, int col0, uint32_t tcol) {
+// squares of y = acc + b over the head, pass 2 re-reads TMEM, computes RoPE(y * rsqrt(ms + eps) * g)
+// per row and stores through the staging tile.  row0 = tile row of lane 0 of this warp.
+__device__ __forceinline__ void epilogue_qk_head(const GemmEpi& e, int M, int row0, int col0, uint32_t tcol,
+                                                 float* stg, int lane) {
   const int D = e.qk_D;
+  const int row = row0 + lane;
   const bool norm = col0 < 2 * e.qk_h;
   float rn = 1.f;
   if (norm) {
@@ -126,8 +151,7 @@ __device__ __forceinline__ void epilogue_qk_head(const GemmEpi& e, int M, int ro
 #pragma unroll
     for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
     if (e.bias) add_bias32(e.bias, col0 + c * 32, v);
-    if (row >= M) continue;
-    if (norm) {
+    if (norm && row < M) {
       const uint4* gp = reinterpret_cast<const uint4*>(g + c * 32);
       const float4* cp = reinterpret_cast<const float4*>(e.cosb + (long long)row * (D / 2) + c * 16);
       const float4* sp = reinterpret_cast<const float4*>(e.sinb + (long long)row * (D / 2) + c * 16);
@@ -147,98 +171,82 @@ __device__ __forceinline__ void epilogue_qk_head(const GemmEpi& e, int M, int ro
         }
       }
     }
-    store_bf16x32(qkv_dst(e, row, col0 + c * 32), v);
+    stage_write(stg, lane, v);
+    __syncwarp();
+    const int c4 = lane & 7;
+#pragma unroll
+    for (int it = 0; it < 8; ++it) {
+      const int rr = it * 4 + (lane >> 3);
+      if (row0 + rr < M)
+        *reinterpret_cast<uint2*>(qkv_dst(e, row0 + rr, col0 + c * 32 + c4 * 4)) = pack4_bf16(stage_read(stg, rr, c4));
+    }
+    __syncwarp();
   }
 }
 
-__device__ __forceinline__ void epilogue_chunk(const GemmEpi& e, int M, int row, int n0, const uint32_t (&r)[32]) {
+__device__ __forceinline__ void epilogue_chunk(const GemmEpi& e, int M, int row0, int n0, const uint32_t (&r)[32],
+                                               float* stg, int lane) {
   float v[32];
 #pragma unroll
   for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+  stage_write(stg, lane, v);
+  __syncwarp();
+  const int c4 = lane & 7;
+  const int col = n0 + c4 * 4;  // this lane's 4 columns for all 8 row groups
+  float4 b = make_float4(0.f, 0.f, 0.f, 0.f);
   if (e.bias) {
-    const uint4* bp = reinterpret_cast<const uint4*>(e.bias + n0);
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      uint4 u = __ldg(bp + q);
-      float2 f0 = unpack_bf16x2(u.x), f1 = unpack_bf16x2(u.y), f2 = unpack_bf16x2(u.z), f3 = unpack_bf16x2(u.w);
-      v[q * 8 + 0] += f0.x; v[q * 8 + 1] += f0.y; v[q * 8 + 2] += f1.x; v[q * 8 + 3] += f1.y;
-      v[q * 8 + 4] += f2.x; v[q * 8 + 5] += f2.y; v[q * 8 + 6] += f3.x; v[q * 8 + 7] += f3.y;
-    }
+    const uint2 bu = __ldg(reinterpret_cast<const uint2*>(e.bias + col));
+    const float2 b0 = unpack_bf16x2(bu.x), b1 = unpack_bf16x2(bu.y);
+    b = make_float4(b0.x, b0.y, b1.x, b1.y);
   }
-  if (row >= M) return;
   int mode = e.mode;
   bf16* ob = nullptr;
-  if (mode == EPI_SPLIT_GELU) {
+  long long ldb = e.ld0;
+  if (mode == EPI_SPLIT_GELU) {  // n0 (and the whole 32-column chunk) is on one side of the split
     if (n0 >= e.n_split) {
       mode = EPI_GELU_BF16;
-      ob = reinterpret_cast<bf16*>(e.out1) + (long long)row * e.ld1 + (n0 - e.n_split);
+      ob = reinterpret_cast<bf16*>(e.out1) + (col - e.n_split);
+      ldb = e.ld1;
     } else {
       mode = EPI_STORE_BF16;
-      ob = reinterpret_cast<bf16*>(e.out0) + (long long)row * e.ld0 + n0;
+      ob = reinterpret_cast<bf16*>(e.out0) + col;
     }
   } else if (mode <= EPI_SILU_BF16) {
-    ob = reinterpret_cast<bf16*>(e.out0) + (long long)row * e.ld0 + n0;
+    ob = reinterpret_cast<bf16*>(e.out0) + col;
   }
-  if (mode <= EPI_SILU_BF16) {
-    if (mode == EPI_GELU_BF16) {
+  float4 g = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (mode == EPI_RESID_GATE) g = __ldg(reinterpret_cast<const float4*>(e.gate + col));
+  const float dt = mode == EPI_EULER ? *e.scalar : 0.f;
 #pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] = gelu_tanh(v[i]);
-    } else if (mode == EPI_SILU_BF16) {
-#pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] = silu(v[i]);
+  for (int it = 0; it < 8; ++it) {
+    const int rr = it * 4 + (lane >> 3);
+    const int grow = row0 + rr;
+    float4 a = stage_read(stg, rr, c4);
+    a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
+    if (grow >= M) continue;
+    if (mode <= EPI_SILU_BF16) {
+      if (mode == EPI_GELU_BF16) { a.x = gelu_tanh(a.x); a.y = gelu_tanh(a.y); a.z = gelu_tanh(a.z); a.w = gelu_tanh(a.w); }
+      else if (mode == EPI_SILU_BF16) { a.x = silu(a.x); a.y = silu(a.y); a.z = silu(a.z); a.w = silu(a.w); }
+      *reinterpret_cast<uint2*>(ob + (long long)grow * ldb) = pack4_bf16(a);
+      continue;
     }
-    uint4* dst = reinterpret_cast<uint4*>(ob);
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      uint4 u;
-      u.x = pack_bf16x2(v[q * 8 + 0], v[q * 8 + 1]);
-      u.y = pack_bf16x2(v[q * 8 + 2], v[q * 8 + 3]);
-      u.z = pack_bf16x2(v[q * 8 + 4], v[q * 8 + 5]);
-      u.w = pack_bf16x2(v[q * 8 + 6], v[q * 8 + 7]);
-      dst[q] = u;
-    }
-    return;
-  }
-  float* of = reinterpret_cast<float*>(e.out0) + (long long)row * e.ld0 + n0;
-  float4* d4 = reinterpret_cast<float4*>(of);
-  if (mode == EPI_STORE_F32) {
-#pragma unroll
-    for (int q = 0; q < 8; ++q) d4[q] = make_float4(v[q * 4], v[q * 4 + 1], v[q * 4 + 2], v[q * 4 + 3]);
-  } else if (mode == EPI_ACCUM_F32) {
-#pragma unroll
-    for (int q = 0; q < 8; ++q) {
-      float4 x = d4[q];
-      d4[q] = make_float4(x.x + v[q * 4], x.y + v[q * 4 + 1], x.z + v[q * 4 + 2], x.w + v[q * 4 + 3]);
-    }
-  } else if (mode == EPI_RESID_GATE) {
-    const float4* g4 = reinterpret_cast<const float4*>(e.gate + n0);
-#pragma unroll
-    for (int q = 0; q < 8; ++q) {
-      float4 x = d4[q];
-      float4 g = __ldg(g4 + q);
-      x.x += g.x * v[q * 4 + 0];
-      x.y += g.y * v[q * 4 + 1];
-      x.z += g.z * v[q * 4 + 2];
-      x.w += g.w * v[q * 4 + 3];
-      d4[q] = x;
-    }
-  } else if (mode == EPI_EULER) {
-    const float dt = *e.scalar;
-    if (e.out1) {
-      float4* v4 = reinterpret_cast<float4*>(reinterpret_cast<float*>(e.out1) + (long long)row * e.ld1 + n0);
-#pragma unroll
-      for (int q = 0; q < 8; ++q) v4[q] = make_float4(v[q * 4], v[q * 4 + 1], v[q * 4 + 2], v[q * 4 + 3]);
-    }
-#pragma unroll
-    for (int q = 0; q < 8; ++q) {
-      float4 x = d4[q];
-      x.x += dt * v[q * 4 + 0];
-      x.y += dt * v[q * 4 + 1];
-      x.z += dt * v[q * 4 + 2];
-      x.w += dt * v[q * 4 + 3];
-      d4[q] = x;
+    float4* xp = reinterpret_cast<float4*>(reinterpret_cast<float*>(e.out0) + (long long)grow * e.ld0 + col);
+    if (mode == EPI_STORE_F32) {
+      *xp = a;
+    } else if (mode == EPI_ACCUM_F32) {
+      float4 x = *xp;
+      *xp = make_float4(x.x + a.x, x.y + a.y, x.z + a.z, x.w + a.w);
+    } else if (mode == EPI_RESID_GATE) {
+      float4 x = *xp;
+      *xp = make_float4(x.x + g.x * a.x, x.y + g.y * a.y, x.z + g.z * a.z, x.w + g.w * a.w);
+    } else if (mode == EPI_EULER) {
+      if (e.out1)
+        *reinterpret_cast<float4*>(reinterpret_cast<float*>(e.out1) + (long long)grow * e.ld1 + col) = a;
+      float4 x = *xp;
+      *xp = make_float4(x.x + dt * a.x, x.y + dt * a.y, x.z + dt * a.z, x.w + dt * a.w);
     }
   }
+  __syncwarp();
 }
 
 template <int BN>
@@ -255,6 +263,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   uint64_t* tfull = bars + 2 * C::STAGES;
   uint64_t* tempty = bars + 2 * C::STAGES + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * C::STAGES + 4);
+  float* stg_all = reinterpret_cast<float*>(smem + C::STAGES * C::STAGE_BYTES + 256);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -332,6 +341,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   } else if (warp >= 4) {
     // ---------------- epilogue: warp (4..7) owns TMEM lanes [32*(warp-4), +32)
     const int wq = warp - 4;
+    float* stg = stg_all + wq * STG_FLOATS;
     int it = 0;
     for (int t = blockIdx.x; t < args.num_tiles; t += gridDim.x, ++it) {
       int pr, m_blk, n_blk;
@@ -342,19 +352,19 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       const uint32_t acc_phase = (it >> 1) & 1;
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
-      const int row = m_blk * BM + wq * 32 + lane;
+      const int row0 = m_blk * BM + wq * 32;
       const uint32_t tbase = tmem_base + ((uint32_t)(wq * 32) << 16) + acc * BN;
       if (epi.qk_h > 0 && n_blk * BN < 3 * epi.qk_h) {
 #pragma unroll 1
         for (int hd = 0; hd < BN / epi.qk_D; ++hd)
-          epilogue_qk_head(epi, Mp, row, n_blk * BN + hd * epi.qk_D, tbase + hd * epi.qk_D);
+          epilogue_qk_head(epi, Mp, row0, n_blk * BN + hd * epi.qk_D, tbase + hd * epi.qk_D, stg, lane);
       } else {
 #pragma unroll 1
         for (int c = 0; c < BN / 32; ++c) {
           uint32_t r[32];
           tmem_ld32(tbase + c * 32, r);
           tmem_ld_wait();
-          epilogue_chunk(epi, Mp, row, n_blk * BN + c * 32, r);
+          epilogue_chunk(epi, Mp, row0, n_blk * BN + c * 32, r, stg, lane);
         }
       }
       tc_fence_before();
@@ -380,7 +390,7 @@ struct Gemm2Cfg {
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int STAGES = 6;
   static constexpr int TMEM_COLS = 2 * BN;
-  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + 4 * 32 * 36 * 4;
 };
 
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
@@ -397,6 +407,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
   uint64_t* tfull = bars + 2 * C::STAGES;
   uint64_t* tempty = bars + 2 * C::STAGES + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * C::STAGES + 4);
+  float* stg_all = reinterpret_cast<float*>(smem + C::STAGES * C::STAGE_BYTES + 256);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -473,6 +484,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
     }
   } else if (warp >= 4) {
     const int wq = warp - 4;
+    float* stg = stg_all + wq * STG_FLOATS;
     int it = 0;
     for (int t = cid; t < args.num_tiles; t += ncl, ++it) {
       int pr, m_blk, n_blk;
@@ -483,19 +495,19 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
       const uint32_t acc_phase = (it >> 1) & 1;
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
-      const int row = m_blk * 256 + (int)rank * 128 + wq * 32 + lane;
+      const int row0 = m_blk * 256 + (int)rank * 128 + wq * 32;
       const uint32_t tbase = tmem_base + ((uint32_t)(wq * 32) << 16) + acc * BN;
       if (epi.qk_h > 0 && n_blk * BN < 3 * epi.qk_h) {
 #pragma unroll 1
         for (int hd = 0; hd < BN / epi.qk_D; ++hd)
-          epilogue_qk_head(epi, Mp, row, n_blk * BN + hd * epi.qk_D, tbase + hd * epi.qk_D);
+          epilogue_qk_head(epi, Mp, row0, n_blk * BN + hd * epi.qk_D, tbase + hd * epi.qk_D, stg, lane);
       } else {
 #pragma unroll 1
         for (int c = 0; c < BN / 32; ++c) {
           uint32_t r[32];
           tmem_ld32(tbase + c * 32, r);
           tmem_ld_wait();
-          epilogue_chunk(epi, Mp, row, n_blk * BN + c * 32, r);
+          epilogue_chunk(epi, Mp, row0, n_blk * BN + c * 32, r, stg, lane);
         }
       }
       tc_fence_before();
