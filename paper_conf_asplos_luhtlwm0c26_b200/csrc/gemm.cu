@@ -214,39 +214,55 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpi& e, int M, int row0
   } else if (mode <= EPI_SILU_BF16) {
     ob = reinterpret_cast<bf16*>(e.out0) + col;
   }
-  float4 g = make_float4(0.f, 0.f, 0.f, 0.f);
-  if (mode == EPI_RESID_GATE) g = __ldg(reinterpret_cast<const float4*>(e.gate + col));
-  const float dt = mode == EPI_EULER ? *e.scalar : 0.f;
+  float4 a[8];
 #pragma unroll
   for (int it = 0; it < 8; ++it) {
-    const int rr = it * 4 + (lane >> 3);
-    const int grow = row0 + rr;
-    float4 a = stage_read(stg, rr, c4);
-    a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
-    if (grow >= M) continue;
-    if (mode <= EPI_SILU_BF16) {
-      if (mode == EPI_GELU_BF16) { a.x = gelu_tanh(a.x); a.y = gelu_tanh(a.y); a.z = gelu_tanh(a.z); a.w = gelu_tanh(a.w); }
-      else if (mode == EPI_SILU_BF16) { a.x = silu(a.x); a.y = silu(a.y); a.z = silu(a.z); a.w = silu(a.w); }
-      *reinterpret_cast<uint2*>(ob + (long long)grow * ldb) = pack4_bf16(a);
-      continue;
+    a[it] = stage_read(stg, it * 4 + (lane >> 3), c4);
+    a[it].x += b.x; a[it].y += b.y; a[it].z += b.z; a[it].w += b.w;
+  }
+  __syncwarp();  // the staging tile may be overwritten by the next chunk from here on
+  const int rbase = row0 + (lane >> 3);
+  if (mode <= EPI_SILU_BF16) {
+#pragma unroll
+    for (int it = 0; it < 8; ++it) {
+      float4 y = a[it];
+      if (mode == EPI_GELU_BF16) { y.x = gelu_tanh(y.x); y.y = gelu_tanh(y.y); y.z = gelu_tanh(y.z); y.w = gelu_tanh(y.w); }
+      else if (mode == EPI_SILU_BF16) { y.x = silu(y.x); y.y = silu(y.y); y.z = silu(y.z); y.w = silu(y.w); }
+      if (rbase + it * 4 < M) *reinterpret_cast<uint2*>(ob + (long long)(rbase + it * 4) * ldb) = pack4_bf16(y);
     }
-    float4* xp = reinterpret_cast<float4*>(reinterpret_cast<float*>(e.out0) + (long long)grow * e.ld0 + col);
-    if (mode == EPI_STORE_F32) {
-      *xp = a;
-    } else if (mode == EPI_ACCUM_F32) {
-      float4 x = *xp;
-      *xp = make_float4(x.x + a.x, x.y + a.y, x.z + a.z, x.w + a.w);
-    } else if (mode == EPI_RESID_GATE) {
-      float4 x = *xp;
-      *xp = make_float4(x.x + g.x * a.x, x.y + g.y * a.y, x.z + g.z * a.z, x.w + g.w * a.w);
-    } else if (mode == EPI_EULER) {
-      if (e.out1)
-        *reinterpret_cast<float4*>(reinterpret_cast<float*>(e.out1) + (long long)grow * e.ld1 + col) = a;
-      float4 x = *xp;
-      *xp = make_float4(x.x + dt * a.x, x.y + dt * a.y, x.z + dt * a.z, x.w + dt * a.w);
+    return;
+  }
+  float* out = reinterpret_cast<float*>(e.out0) + col;
+  if (mode == EPI_STORE_F32) {
+#pragma unroll
+    for (int it = 0; it < 8; ++it)
+      if (rbase + it * 4 < M) *reinterpret_cast<float4*>(out + (long long)(rbase + it * 4) * e.ld0) = a[it];
+    return;
+  }
+  // read-modify-write of the fp32 stream: issue all 8 loads before any store (independent rows)
+  float4 x[8];
+#pragma unroll
+  for (int it = 0; it < 8; ++it)
+    x[it] = rbase + it * 4 < M ? *reinterpret_cast<const float4*>(out + (long long)(rbase + it * 4) * e.ld0)
+                               : make_float4(0.f, 0.f, 0.f, 0.f);
+  float4 g = make_float4(1.f, 1.f, 1.f, 1.f);
+  if (mode == EPI_RESID_GATE) g = __ldg(reinterpret_cast<const float4*>(e.gate + col));
+  if (mode == EPI_EULER) {
+    const float dt = *e.scalar;
+    g = make_float4(dt, dt, dt, dt);
+    if (e.out1) {
+      float* vout = reinterpret_cast<float*>(e.out1) + col;
+#pragma unroll
+      for (int it = 0; it < 8; ++it)
+        if (rbase + it * 4 < M) *reinterpret_cast<float4*>(vout + (long long)(rbase + it * 4) * e.ld1) = a[it];
     }
   }
-  __syncwarp();
+#pragma unroll
+  for (int it = 0; it < 8; ++it) {
+    const float4 y = make_float4(x[it].x + g.x * a[it].x, x[it].y + g.y * a[it].y, x[it].z + g.z * a[it].z,
+                                 x[it].w + g.w * a[it].w);
+    if (rbase + it * 4 < M) *reinterpret_cast<float4*>(out + (long long)(rbase + it * 4) * e.ld0) = y;
+  }
 }
 
 template <int BN>
