@@ -58,6 +58,19 @@ __device__ __forceinline__ float fast_exp2(float x) {  // MUFU.EX2; ex2(-inf) = 
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
   return y;
 }
+// 2^x without the MUFU: x = n + f (n = round(x), |f| <= 1/2), 2^f by a cubic (Taylor of e^(f ln2),
+// rel. error <= 7e-4 on |f| <= 1/2), 2^n added to the exponent field.  x is clamped at -126 so the
+// exponent add cannot wrap (the true value is < 2^-126 there).  Finite x only.
+__device__ __forceinline__ float poly_exp2(float x) {
+  x = fmaxf(x, -126.0f);
+  const float t = x + 12582912.0f;          // 1.5 * 2^23: round(x) lands in the low mantissa bits
+  const float n = t - 12582912.0f;
+  const float f = x - n;
+  float p = fmaf(0.0555041086648216f, f, 0.2402265069591007f);
+  p = fmaf(p, f, 0.6931471805599453f);
+  p = fmaf(p, f, 1.0f);
+  return __int_as_float(__float_as_int(p) + (__float_as_int(t) << 23));
+}
 __device__ __forceinline__ void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 // MN-major, 128B-swizzled B operand (rows = K, 64 N-elements per 128-byte row):
@@ -476,16 +489,39 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       // P = 2^(s * scale_log2 - m_ref) as packed bf16 pairs, in place of S (columns 0..63 of S_t)
       float ls0 = 0.f, ls1 = 0.f;
       const float neg_m = -m_ref;
+      if (kbase + AT_BN <= L) {
+        // MUFU.EX2 throughput equals the MMA rate here, so 1 pair in 4 is evaluated on the FMA/ALU
+        // pipes instead (Cody-Waite split + cubic, rel. error < 1e-3 << bf16 ulp of P).
 #pragma unroll
-      for (int c = 0; c < 4; ++c)
+        for (int c = 0; c < 4; ++c)
 #pragma unroll
-        for (int i = 0; i < 32; i += 2) {
-          const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
-          const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
-          ls0 += p0;
-          ls1 += p1;
-          sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);  // packed P overwrites consumed S
-        }
+          for (int i = 0; i < 32; i += 2) {
+            const float x0 = fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m);
+            const float x1 = fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m);
+            float p0, p1;
+            if ((i & 6) == 6) {
+              p0 = poly_exp2(x0);
+              p1 = poly_exp2(x1);
+            } else {
+              p0 = fast_exp2(x0);
+              p1 = fast_exp2(x1);
+            }
+            ls0 += p0;
+            ls1 += p1;
+            sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);  // packed P overwrites consumed S
+          }
+      } else {
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+#pragma unroll
+          for (int i = 0; i < 32; i += 2) {
+            const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
+            const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
+            ls0 += p0;
+            ls1 += p1;
+            sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);
+          }
+      }
       l_sum += ls0 + ls1;
       // S_t{j} complete => PV_t{j-1} complete (in-order pipe): O_t can be rescaled right away
       if (__any_sync(0xffffffffu, rescale)) {
