@@ -206,25 +206,23 @@ __global__ void __launch_bounds__(AT_THREADS, 1)
       mbar_arrive(&s_free[st]);
       const int kbase = j * AT_BN;
       // row max on the raw scores (scale > 0); keys >= L only exist in the last tile
-      float mr0 = -FLT_MAX, mr1 = -FLT_MAX;
-      if (kbase + AT_BN <= L) {
+      // row max with 8 independent accumulators (a single chain would be 128 dependent FMNMX)
+      float mx[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) mx[q] = -FLT_MAX;
+      if (kbase + AT_BN > L) {
 #pragma unroll
         for (int c = 0; c < 4; ++c)
 #pragma unroll
-          for (int i = 0; i < 32; i += 2) {
-            mr0 = fmaxf(mr0, __uint_as_float(sr[c][i]));
-            mr1 = fmaxf(mr1, __uint_as_float(sr[c][i + 1]));
-          }
-      } else {
-#pragma unroll
-        for (int c = 0; c < 4; ++c)
-#pragma unroll
-          for (int i = 0; i < 32; ++i) {
+          for (int i = 0; i < 32; ++i)
             if (kbase + c * 32 + i >= L) sr[c][i] = __float_as_uint(-INFINITY);
-            mr0 = fmaxf(mr0, __uint_as_float(sr[c][i]));
-          }
       }
-      const float mt = fmaxf(mr0, mr1) * scale_log2;
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int i = 0; i < 32; ++i) mx[i & 7] = fmaxf(mx[i & 7], __uint_as_float(sr[c][i]));
+      const float mt = fmaxf(fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3])),
+                             fmaxf(fmaxf(mx[4], mx[5]), fmaxf(mx[6], mx[7]))) * scale_log2;
       bool rescale = false;
       float alpha = 1.f;
       if (j == 0) {
@@ -457,25 +455,23 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
       tmem_ld_wait();
       const int kbase = j * AT_BN;
-      float mr0 = -FLT_MAX, mr1 = -FLT_MAX;
-      if (kbase + AT_BN <= L) {
+      // row max with 8 independent accumulators (a single chain would be 128 dependent FMNMX)
+      float mx[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) mx[q] = -FLT_MAX;
+      if (kbase + AT_BN > L) {
 #pragma unroll
         for (int c = 0; c < 4; ++c)
 #pragma unroll
-          for (int i = 0; i < 32; i += 2) {
-            mr0 = fmaxf(mr0, __uint_as_float(sr[c][i]));
-            mr1 = fmaxf(mr1, __uint_as_float(sr[c][i + 1]));
-          }
-      } else {
-#pragma unroll
-        for (int c = 0; c < 4; ++c)
-#pragma unroll
-          for (int i = 0; i < 32; ++i) {
+          for (int i = 0; i < 32; ++i)
             if (kbase + c * 32 + i >= L) sr[c][i] = __float_as_uint(-INFINITY);
-            mr0 = fmaxf(mr0, __uint_as_float(sr[c][i]));
-          }
       }
-      const float mt = fmaxf(mr0, mr1) * scale_log2;
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int i = 0; i < 32; ++i) mx[i & 7] = fmaxf(mx[i & 7], __uint_as_float(sr[c][i]));
+      const float mt = fmaxf(fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3])),
+                             fmaxf(fmaxf(mx[4], mx[5]), fmaxf(mx[6], mx[7]))) * scale_log2;
       bool rescale = false;
       float alpha = 1.f;
       if (j == 0) {
@@ -490,6 +486,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       float ls0 = 0.f, ls1 = 0.f;
       const float neg_m = -m_ref;
       if (kbase + AT_BN <= L) {
+        float lsum[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
         // MUFU.EX2 throughput equals the MMA rate here, so 1 pair in 4 is evaluated on the FMA/ALU
         // pipes instead (Cody-Waite split + cubic, rel. error < 1e-3 << bf16 ulp of P).
 #pragma unroll
@@ -506,10 +503,11 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
               p0 = fast_exp2(x0);
               p1 = fast_exp2(x1);
             }
-            ls0 += p0;
-            ls1 += p1;
+            lsum[(i >> 1) & 3] += p0;       // 8 independent partial sums
+            lsum[4 + ((i >> 1) & 3)] += p1;
             sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);  // packed P overwrites consumed S
           }
+        ls0 = ((lsum[0] + lsum[1]) + (lsum[2] + lsum[3])) + ((lsum[4] + lsum[5]) + (lsum[6] + lsum[7]));
       } else {
 #pragma unroll
         for (int c = 0; c < 4; ++c)
