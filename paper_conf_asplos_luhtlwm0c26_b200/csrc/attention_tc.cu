@@ -71,6 +71,21 @@ __device__ __forceinline__ float poly_exp2(float x) {
   p = fmaf(p, f, 1.0f);
   return __int_as_float(__float_as_int(p) + (__float_as_int(t) << 23));
 }
+// The same on a pair, with the sm_100 paired FP32 ops (FADD2 / FFMA2: two lanes per instruction).
+__device__ __forceinline__ float2 poly_exp2_x2(float2 x) {
+  x.x = fmaxf(x.x, -126.0f);
+  x.y = fmaxf(x.y, -126.0f);
+  const float2 magic = make_float2(12582912.0f, 12582912.0f);
+  const float2 t = __fadd2_rn(x, magic);
+  const float2 n = __fadd2_rn(t, make_float2(-12582912.0f, -12582912.0f));
+  const float2 f = __ffma2_rn(n, make_float2(-1.0f, -1.0f), x);
+  float2 p = __ffma2_rn(make_float2(0.0555041086648216f, 0.0555041086648216f), f,
+                        make_float2(0.2402265069591007f, 0.2402265069591007f));
+  p = __ffma2_rn(p, f, make_float2(0.6931471805599453f, 0.6931471805599453f));
+  p = __ffma2_rn(p, f, make_float2(1.0f, 1.0f));
+  return make_float2(__int_as_float(__float_as_int(p.x) + (__float_as_int(t.x) << 23)),
+                     __int_as_float(__float_as_int(p.y) + (__float_as_int(t.y) << 23)));
+}
 __device__ __forceinline__ void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 // MN-major, 128B-swizzled B operand (rows = K, 64 N-elements per 128-byte row):
@@ -376,7 +391,6 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
-
   if (warp == 0) {
     if (lane == 0) {
       // ---------------------------------------------------------------- producer
@@ -486,28 +500,28 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       float ls0 = 0.f, ls1 = 0.f;
       const float neg_m = -m_ref;
       if (kbase + AT_BN <= L) {
-        float lsum[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
-        // MUFU.EX2 throughput equals the MMA rate here, so 1 pair in 4 is evaluated on the FMA/ALU
-        // pipes instead (Cody-Waite split + cubic, rel. error < 1e-3 << bf16 ulp of P).
+        // Per tile each softmax warpgroup must finish inside the ~1024-cycle window in which the
+        // tensor core works on the other query tile.  MUFU.EX2 alone needs 1024 cycles per tile
+        // (16/clk/SM), so 3 pairs in 8 are evaluated on the FMA/ALU pipes (Cody-Waite split +
+        // cubic, rel. error < 1e-3 << bf16 ulp of P), and the arithmetic uses paired FP32 ops.
+        const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(neg_m, neg_m);
+        float2 lsum[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f),
+                          make_float2(0.f, 0.f)};
 #pragma unroll
         for (int c = 0; c < 4; ++c)
 #pragma unroll
           for (int i = 0; i < 32; i += 2) {
-            const float x0 = fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m);
-            const float x1 = fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m);
-            float p0, p1;
-            if ((i & 6) == 6) {
-              p0 = poly_exp2(x0);
-              p1 = poly_exp2(x1);
-            } else {
-              p0 = fast_exp2(x0);
-              p1 = fast_exp2(x1);
-            }
-            lsum[(i >> 1) & 3] += p0;       // 8 independent partial sums
-            lsum[4 + ((i >> 1) & 3)] += p1;
-            sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);  // packed P overwrites consumed S
+            const float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2,
+                                        nm2);
+            float2 p;
+            if (((i >> 1) & 7) >= 5) p = poly_exp2_x2(x);
+            else p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
+            lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], p);     // 8 independent partial sums
+            sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);  // packed P overwrites consumed S
           }
-        ls0 = ((lsum[0] + lsum[1]) + (lsum[2] + lsum[3])) + ((lsum[4] + lsum[5]) + (lsum[6] + lsum[7]));
+        const float2 l01 = __fadd2_rn(lsum[0], lsum[1]), l23 = __fadd2_rn(lsum[2], lsum[3]);
+        const float2 l4 = __fadd2_rn(l01, l23);
+        ls0 = l4.x + l4.y;
       } else {
 #pragma unroll
         for (int c = 0; c < 4; ++c)
