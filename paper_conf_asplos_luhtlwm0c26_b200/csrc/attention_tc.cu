@@ -345,14 +345,10 @@ struct FaCfg {
   static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // 2 stages
   static constexpr int OFF_V = OFF_K + 2 * KV_TILE;      // 2 stages
   static constexpr int OFF_BAR = OFF_V + 2 * KV_TILE;
-  static constexpr int OFF_RED = OFF_BAR + 256;            // [2 tiles][2 halves][128 rows] fp32
-  static constexpr int SMEM = OFF_RED + 2 * 2 * 128 * 4 + 1024;
+  static constexpr int SMEM = OFF_BAR + 256 + 1024;
   static constexpr int O_COL = 256;
 };
-// warps 0-3: TMA producer, MMA issuer, TMEM allocator, idle; warps 4-11: softmax of query tile 0,
-// warps 12-19: softmax of query tile 1.  Two warps share each TMEM lane quadrant of a tile and
-// split its 128 score columns (64 each), so every SM sub-partition runs 2 softmax warps per tile.
-constexpr int FA_THREADS = 640;
+constexpr int FA_THREADS = 384;
 
 template <int D>
 __global__ void __launch_bounds__(FA_THREADS, 1)
@@ -385,7 +381,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       mbar_init(&kv_full[i], 1);
       mbar_init(&kv_empty[i], 1);
       mbar_init(&s_full[i], 1);
-      mbar_init(&p_full[i], 256);
+      mbar_init(&p_full[i], 128);
       mbar_init(&o_done[i], 1);
     }
     fence_mbar_init();
@@ -457,46 +453,39 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       }
     }
   } else if (warp >= 4) {
-    // ---------------------------------------------------------------- softmax (thread = half a query row)
-    const int wi = warp - 4;
-    const int t = wi >> 3;          // query tile
-    const int hf = (wi >> 2) & 1;   // score columns [64 hf, 64 hf + 64) and O columns [D/2 hf, ...)
-    const int wq = warp & 3;        // TMEM lane quadrant (hardware: warp % 4)
+    // ---------------------------------------------------------------- softmax WG t (thread = query row)
+    const int t = (warp - 4) >> 2;
+    const int wq = (warp - 4) & 3;
     const int row = wq * 32 + lane;
     const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
     const uint32_t s_col = tmem + lane_base + t * 128;
-    const uint32_t o_col = tmem + lane_base + C::O_COL + t * D + hf * (D / 2);
-    float* red = reinterpret_cast<float*>(sm + C::OFF_RED) + t * 256;   // [half][row]
-    const int bar_id = 1 + t * 4 + wq;                                   // the 2 warps of (t, wq)
+    const uint32_t o_col = tmem + lane_base + C::O_COL + t * D;
     float m_ref = -FLT_MAX, l_sum = 0.f;
     for (int j = 0; j < n_tiles; ++j) {
       mbar_wait(&s_full[t], j & 1);
       tc_fence_after();
-      uint32_t sr[2][32];
+      uint32_t sr[4][32];
 #pragma unroll
-      for (int c = 0; c < 2; ++c) tmem_ld32(s_col + hf * 64 + c * 32, sr[c]);
+      for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
       tmem_ld_wait();
-      const int kbase = j * AT_BN + hf * 64;
-      if (kbase + 64 > L) {
+      const int kbase = j * AT_BN;
+      // row max with 8 independent accumulators (a single chain would be 128 dependent FMNMX)
+      float mx[8];
 #pragma unroll
-        for (int c = 0; c < 2; ++c)
+      for (int q = 0; q < 8; ++q) mx[q] = -FLT_MAX;
+      if (kbase + AT_BN > L) {
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
 #pragma unroll
           for (int i = 0; i < 32; ++i)
             if (kbase + c * 32 + i >= L) sr[c][i] = __float_as_uint(-INFINITY);
       }
-      float mx[8];
 #pragma unroll
-      for (int q = 0; q < 8; ++q) mx[q] = -FLT_MAX;
-#pragma unroll
-      for (int c = 0; c < 2; ++c)
+      for (int c = 0; c < 4; ++c)
 #pragma unroll
         for (int i = 0; i < 32; ++i) mx[i & 7] = fmaxf(mx[i & 7], __uint_as_float(sr[c][i]));
-      const float pm = fmaxf(fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3])), fmaxf(fmaxf(mx[4], mx[5]), fmaxf(mx[6], mx[7])));
-      // row max across the two halves (the partner's previous value was consumed before it could
-      // arrive on p_full, which S_{j} waited for, so the slot is free here)
-      red[hf * 128 + row] = pm;
-      asm volatile("bar.sync %0, 64;" ::"r"(bar_id) : "memory");
-      const float mt = fmaxf(pm, red[(hf ^ 1) * 128 + row]) * scale_log2;
+      const float mt = fmaxf(fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3])),
+                             fmaxf(fmaxf(mx[4], mx[5]), fmaxf(mx[6], mx[7]))) * scale_log2;
       bool rescale = false;
       float alpha = 1.f;
       if (j == 0) {
@@ -507,29 +496,49 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         m_ref = mt;
       }
       l_sum *= alpha;
-      // P = 2^(s * scale_log2 - m_ref) as packed bf16 pairs into P columns [32 hf, 32 hf + 32) of S_t
-      // (the partner finished reading its S columns before the barrier above)
+      // P = 2^(s * scale_log2 - m_ref) as packed bf16 pairs, in place of S (columns 0..63 of S_t)
+      float ls0 = 0.f, ls1 = 0.f;
       const float neg_m = -m_ref;
-      const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(neg_m, neg_m);
-      float2 lsum[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
-      uint32_t pk[32];
+      if (kbase + AT_BN <= L) {
+        // Per tile each softmax warpgroup must finish inside the ~1024-cycle window in which the
+        // tensor core works on the other query tile.  MUFU.EX2 alone needs 1024 cycles per tile
+        // (16/clk/SM), so 3 pairs in 8 are evaluated on the FMA/ALU pipes (Cody-Waite split +
+        // cubic, rel. error < 1e-3 << bf16 ulp of P), and the arithmetic uses paired FP32 ops.
+        const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(neg_m, neg_m);
+        float2 lsum[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f),
+                          make_float2(0.f, 0.f)};
 #pragma unroll
-      for (int c = 0; c < 2; ++c)
+        for (int c = 0; c < 4; ++c)
 #pragma unroll
-        for (int i = 0; i < 32; i += 2) {
-          const float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2, nm2);
-          float2 p;
-          if (((i >> 1) & 7) >= 5 && kbase + 64 <= L) p = poly_exp2_x2(x);   // 3 of 8 pairs off the MUFU
-          else p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
-          lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], p);
-          pk[c * 16 + i / 2] = pack_bf16x2(p.x, p.y);
-        }
-      const float2 l4 = __fadd2_rn(__fadd2_rn(lsum[0], lsum[1]), __fadd2_rn(lsum[2], lsum[3]));
-      l_sum += l4.x + l4.y;
+          for (int i = 0; i < 32; i += 2) {
+            const float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2,
+                                        nm2);
+            float2 p;
+            if (((i >> 1) & 7) >= 5) p = poly_exp2_x2(x);
+            else p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
+            lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], p);     // 8 independent partial sums
+            sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);  // packed P overwrites consumed S
+          }
+        const float2 l01 = __fadd2_rn(lsum[0], lsum[1]), l23 = __fadd2_rn(lsum[2], lsum[3]);
+        const float2 l4 = __fadd2_rn(l01, l23);
+        ls0 = l4.x + l4.y;
+      } else {
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+#pragma unroll
+          for (int i = 0; i < 32; i += 2) {
+            const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
+            const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
+            ls0 += p0;
+            ls1 += p1;
+            sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);
+          }
+      }
+      l_sum += ls0 + ls1;
       // S_t{j} complete => PV_t{j-1} complete (in-order pipe): O_t can be rescaled right away
       if (__any_sync(0xffffffffu, rescale)) {
 #pragma unroll
-        for (int c = 0; c < D / 64; ++c) {
+        for (int c = 0; c < D / 32; ++c) {
           uint32_t ov[32];
           tmem_ld32(o_col + c * 32, ov);
           tmem_ld_wait();
@@ -538,25 +547,24 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
           tmem_st32(o_col + c * 32, ov);
         }
       }
-      tmem_st32(s_col + hf * 32, pk);
+      tmem_st32(s_col, sr[0]);
+      tmem_st32(s_col + 32, sr[1]);
       tmem_st_wait();
       tc_fence_before();
       mbar_arrive(&p_full[t]);
     }
-    // epilogue: O_t / l -> bf16; l is the sum of the two halves' partial sums
+    // epilogue: O_t / l -> bf16
     mbar_wait(&o_done[t], 0);
     tc_fence_after();
-    red[hf * 128 + row] = l_sum;
-    asm volatile("bar.sync %0, 64;" ::"r"(bar_id) : "memory");
-    const float inv = 1.f / (l_sum + red[(hf ^ 1) * 128 + row]);
+    const float inv = 1.f / l_sum;
     const int grow = q0 + t * AT_BM + row;
 #pragma unroll
-    for (int c = 0; c < D / 64; ++c) {
+    for (int c = 0; c < D / 32; ++c) {
       uint32_t ov[32];
       tmem_ld32(o_col + c * 32, ov);
       tmem_ld_wait();
       if (grow < L) {
-        uint4* dst = reinterpret_cast<uint4*>(o + (long long)grow * ldo + head * D + hf * (D / 2) + c * 32);
+        uint4* dst = reinterpret_cast<uint4*>(o + (long long)grow * ldo + head * D + c * 32);
 #pragma unroll
         for (int qd = 0; qd < 4; ++qd) {
           uint4 v;
