@@ -145,6 +145,7 @@ __global__ void __launch_bounds__(AT_THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  grid_dep_wait();
 
   if (warp == 0) {
     if (lane == 0) {
@@ -391,6 +392,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  grid_dep_wait();
   if (warp == 0) {
     if (lane == 0) {
       // ---------------------------------------------------------------- producer
@@ -577,6 +579,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       }
     }
   }
+  grid_dep_launch();
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -631,7 +634,7 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     attention_tc_kernel<D><<<grid, AT_THREADS, AttnCfg<D>::SMEM, s>>>(tq, tk, tv, o, ldo, L, scale_log2);
   } else {
     dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H);
-    attention_fa_kernel<D><<<grid, FA_THREADS, FaCfg<D>::SMEM, s>>>(tq, tk, tv, o, ldo, L, scale_log2);
+    launch_pdl(attention_fa_kernel<D>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo, L, scale_log2);
   }
   return 0;
 }

@@ -32,6 +32,7 @@ __global__ void __launch_bounds__(T) ln_mod_kernel(const float* __restrict__ x, 
   __shared__ float red[T / 32];
   const int row = blockIdx.x;
   const int t = threadIdx.x;
+  grid_dep_wait();
   // rows [0, n_first) take (shift0, scale0), the others (shift1, scale1): both streams of a
   // double block in one launch
   const float* shift = row < n_first ? shift0 : shift1;
@@ -79,6 +80,8 @@ __global__ void __launch_bounds__(256) ln_mod_generic(const float* __restrict__ 
                                                       const float* __restrict__ scale1, int n_first, int M, int h) {
   const int row = blockIdx.x * 8 + (threadIdx.x >> 5);
   const int lane = threadIdx.x & 31;
+  grid_dep_wait();
+  grid_dep_launch();
   if (row >= M) return;
   const float* shift = row < n_first ? shift0 : shift1;
   const float* scale = row < n_first ? scale0 : scale1;
@@ -101,16 +104,17 @@ void ln_mod2_launch(const float* x, long long ldx, bf16* u, long long ldu, const
   if (M <= 0) return;
   switch (h) {
     case 3072:
-      ln_mod_kernel<256, 3><<<M, 256, 0, s>>>(x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
+      launch_pdl(ln_mod_kernel<256, 3>, dim3(M), dim3(256), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
       break;
     case 1536:
-      ln_mod_kernel<128, 3><<<M, 128, 0, s>>>(x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
+      launch_pdl(ln_mod_kernel<128, 3>, dim3(M), dim3(128), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
       break;
     case 256:
-      ln_mod_kernel<32, 2><<<M, 32, 0, s>>>(x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
+      launch_pdl(ln_mod_kernel<32, 2>, dim3(M), dim3(32), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
       break;
     default:
-      ln_mod_generic<<<(M + 7) / 8, 256, 0, s>>>(x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first, M, h);
+      launch_pdl(ln_mod_generic, dim3((M + 7) / 8), dim3(256), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1,
+                 n_first, M, h);
       break;
   }
 }
@@ -215,6 +219,8 @@ void qk_norm_rope_launch(bf16* qkv, long long ld, int rows, int n_first, int H, 
 // ------------------------------------------------------------------ small conversions
 __global__ void f32_to_bf16_kernel(const float* __restrict__ src, long long lds, bf16* __restrict__ dst,
                                    long long ldd, int M, int C, int act) {
+  grid_dep_wait();
+  grid_dep_launch();
   long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   long long n = (long long)M * C;
   for (; i < n; i += (long long)gridDim.x * blockDim.x) {
@@ -229,19 +235,21 @@ void f32_to_bf16_launch(const float* src, long long lds, bf16* dst, long long ld
   long long n = (long long)M * C;
   int blocks = (int)((n + 255) / 256);
   if (blocks > 4096) blocks = 4096;
-  f32_to_bf16_kernel<<<blocks, 256, 0, s>>>(src, lds, dst, ldd, M, C, 0);
+  launch_pdl(f32_to_bf16_kernel, dim3(blocks), dim3(256), 0, s, src, lds, dst, ldd, M, C, 0);
 }
 void silu_bf16_launch(const float* src, long long lds, bf16* dst, long long ldd, int M, int C, cudaStream_t s) {
   if (M <= 0 || C <= 0) return;
   long long n = (long long)M * C;
   int blocks = (int)((n + 255) / 256);
   if (blocks > 4096) blocks = 4096;
-  f32_to_bf16_kernel<<<blocks, 256, 0, s>>>(src, lds, dst, ldd, M, C, 1);
+  launch_pdl(f32_to_bf16_kernel, dim3(blocks), dim3(256), 0, s, src, lds, dst, ldd, M, C, 1);
 }
 
 // rows x cols bf16, cols multiple of 8, strides multiple of 8 elements
 __global__ void copy2d_bf16_kernel(const uint4* __restrict__ src, long long lds8, uint4* __restrict__ dst,
                                    long long ldd8, int rows, int cols8) {
+  grid_dep_wait();
+  grid_dep_launch();
   long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   long long n = (long long)rows * cols8;
   for (; i < n; i += (long long)gridDim.x * blockDim.x) {
@@ -254,12 +262,14 @@ void copy2d_bf16_launch(const bf16* src, long long lds, bf16* dst, long long ldd
   long long n = (long long)rows * (cols / 8);
   int blocks = (int)((n + 255) / 256);
   if (blocks > 8192) blocks = 8192;
-  copy2d_bf16_kernel<<<blocks, 256, 0, s>>>(reinterpret_cast<const uint4*>(src), lds / 8,
-                                            reinterpret_cast<uint4*>(dst), ldd / 8, rows, cols / 8);
+  launch_pdl(copy2d_bf16_kernel, dim3(blocks), dim3(256), 0, s, reinterpret_cast<const uint4*>(src), lds / 8,
+             reinterpret_cast<uint4*>(dst), ldd / 8, rows, cols / 8);
 }
 
 __global__ void select_row_kernel(const float* __restrict__ src, long long stride, const int* __restrict__ idx,
                                   float* __restrict__ dst, long long n) {
+  grid_dep_wait();
+  grid_dep_launch();
   const float* s = src + (long long)(*idx) * stride;
   long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   const long long n4 = n / 4;
@@ -273,7 +283,7 @@ void select_row_launch(const float* src, long long stride, const int* idx_dev, f
   int blocks = (int)((n / 4 + 255) / 256);
   if (blocks < 1) blocks = 1;
   if (blocks > 2048) blocks = 2048;
-  select_row_kernel<<<blocks, 256, 0, s>>>(src, stride, idx_dev, dst, n);
+  launch_pdl(select_row_kernel, dim3(blocks), dim3(256), 0, s, src, stride, idx_dev, dst, n);
 }
 
 // ------------------------------------------------------------------ SYNTH-1 (see include/tsv.h)

@@ -305,6 +305,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  grid_dep_wait();  // A (and the fp32 stream) come from the previous kernel
 
   if (warp == 0) {
     if (lane == 0) {
@@ -387,6 +388,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       mbar_arrive(&tempty[acc]);
     }
   }
+  grid_dep_launch();
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -452,6 +454,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
   cluster_sync();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  grid_dep_wait();  // A (and the fp32 stream) come from the previous kernel
 
   if (warp == 0) {
     if (lane == 0) {
@@ -530,6 +533,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
       mbar_arrive_remote(&tempty[acc], 0);
     }
   }
+  grid_dep_launch();
   tc_fence_before();
   cluster_sync();
   tc_fence_after();
@@ -675,9 +679,9 @@ static void launch_bn(const GemmPlan& p, cudaStream_t s) {
       cudaFuncSetAttribute(gemm_tc2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, Gemm2Cfg::SMEM_BYTES);
       attr2 |= 1ull << dev;
     }
-    gemm_tc2_kernel<<<p.grid, GEMM_THREADS, Gemm2Cfg::SMEM_BYTES, s>>>(maps, a);
+    launch_pdl(gemm_tc2_kernel, dim3(p.grid), dim3(GEMM_THREADS), Gemm2Cfg::SMEM_BYTES, s, maps, a);
   } else {
-    gemm_tc_kernel<BN><<<p.grid, GEMM_THREADS, C::SMEM_BYTES, s>>>(maps, a);
+    launch_pdl(gemm_tc_kernel<BN>, dim3(p.grid), dim3(GEMM_THREADS), C::SMEM_BYTES, s, maps, a);
   }
 }
 

@@ -11,6 +11,25 @@ namespace tsv {
 
 using bf16 = __nv_bfloat16;
 
+// Launch with programmatic stream serialisation (PDL): inside a captured step graph the next
+// kernel's prologue overlaps this kernel's tail; kernels call grid_dep_wait() before reading
+// their inputs (ptx.cuh).
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                              Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+
 // ------------------------------------------------------------------ GEMM  y = A W^T (+ bias) -> epilogue
 enum EpiMode : int {
   EPI_STORE_BF16 = 0,   // out0[m,n] = bf16(acc + b)

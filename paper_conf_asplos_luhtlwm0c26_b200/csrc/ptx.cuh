@@ -131,6 +131,14 @@ TSV_DEV void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
 }
 TSV_DEV void tmem_ld_wait() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 
+// ------------------------------------------------------------------ programmatic dependent launch
+// Kernels of the step are launched with programmatic stream serialisation: the next kernel's CTAs
+// may start (prologue: barrier init, TMEM alloc, descriptor prefetch) once every CTA of the
+// current kernel executed launch_dependents; grid_dep_wait() blocks until the previous kernel has
+// completed and its memory is visible.  Without the launch attribute both are no-ops.
+TSV_DEV void grid_dep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+TSV_DEV void grid_dep_launch() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 // ------------------------------------------------------------------ clusters / CTA pairs (cta_group::2)
 TSV_DEV uint32_t cluster_ctarank() {
   uint32_t r;
