@@ -37,6 +37,10 @@ class ModelDesc(C.Structure):
                 ("guidance_embed", C.c_int)]
 
 
+class SchedRequest(C.Structure):
+    _fields_ = [("deadline", C.c_double), ("remaining_steps", C.c_int), ("table_row", C.c_int)]
+
+
 _i32, _i64, _u64, _p, _f32 = C.c_int, C.c_int64, C.c_uint64, C.c_void_p, C.c_float
 _P = C.POINTER
 
@@ -78,6 +82,11 @@ _SIGS = {
     "tsv_op_qk_norm_rope": (_i32, [_p, _i64, _i32, _i32, _i32, _i32, _p, _p, _p, _p, _p, _p, _p, _i32, _p]),
     "tsv_op_attention": (_i32, [_p, _i64, _p, _i64, _p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p]),
     "tsv_op_synth": (_i32, [_p, _u64, C.c_uint32, _u64, _i64, _i32, _f32, _p]),
+    "tsv_sched_allocate": (_i32, [_P(C.c_double), _i32, _P(_i32), _i32, _P(SchedRequest), C.c_double, _i32, _P(_i32),
+                                  _P(_i32)]),
+    "tsv_sched_round": (_i32, [_P(C.c_double), _i32, _P(_i32), _i32, _P(SchedRequest), _i32, C.c_double, C.c_double,
+                               _i32, _P(_i32), _P(_i32), _P(_i32)]),
+    "tsv_sched_last_error": (C.c_char_p, []),
 }
 
 EXPORTED = sorted(_SIGS)
@@ -95,3 +104,8 @@ def last_error() -> str:
 def check(status: int) -> None:
     if status != TSV_OK:
         raise TsvError(status, last_error())
+
+
+def check_sched(status: int) -> None:
+    if status != TSV_OK:
+        raise TsvError(status, lib.tsv_sched_last_error().decode(errors="replace"))

@@ -11,7 +11,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 BUILD = os.path.join(ROOT, "build", "tsv")
 LIB = os.path.join(PKG, "libtsv.so")
-SOURCES = ["gemm.cu", "attention.cu", "attention_tc.cu", "elementwise.cu", "engine.cu", "model.cpp"]
+SOURCES = ["gemm.cu", "attention.cu", "attention_tc.cu", "elementwise.cu", "engine.cu", "model.cpp", "sched.cpp"]
 HEADERS = ["ptx.cuh", "kernels.h", "model.h"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
@@ -34,7 +34,8 @@ def build(verbose: bool = False, force: bool = False) -> str:
     nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
     inc, lib = nccl_dirs()
     os.makedirs(BUILD, exist_ok=True)
-    hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [os.path.join(ROOT, "include", f) for f in ("tsv.h", "tsv_ops.h")]
+    hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [os.path.join(ROOT, "include", f)
+                                                       for f in ("tsv.h", "tsv_ops.h", "tsv_sched.h")]
     flags = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + inc, "-I" + os.path.join(ROOT, "include"),
                     "--expt-relaxed-constexpr", "-Xptxas", "-v" if verbose else "-O3"]
 

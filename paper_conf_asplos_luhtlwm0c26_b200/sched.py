@@ -1,0 +1,47 @@
+"""Binding of libtsv.so's round-based scheduler (include/tsv_sched.h): argument marshalling only."""
+from __future__ import annotations
+
+import ctypes as C
+
+import numpy as np
+
+from ._lib import SchedRequest, check_sched, lib
+
+
+def _table(T, ks):
+    T = np.ascontiguousarray(T, dtype=np.float64)
+    ks = list(ks)
+    return T, (C.c_int * len(ks))(*ks), T.shape[0], len(ks)
+
+
+def _reqs(requests):
+    arr = (SchedRequest * max(len(requests), 1))()
+    for i, (deadline, steps, row) in enumerate(requests):
+        arr[i].deadline = deadline
+        arr[i].remaining_steps = steps
+        arr[i].table_row = row
+    return arr
+
+
+def allocate(T, ks, deadline: float, steps: int, row: int, now: float, N: int):
+    """-> (steps per degree (list aligned with ks), late flag)."""
+    T, kk, n_res, n_k = _table(T, ks)
+    r = _reqs([(deadline, steps, row)])
+    out = (C.c_int * n_k)()
+    late = C.c_int()
+    check_sched(lib.tsv_sched_allocate(T.ctypes.data_as(C.POINTER(C.c_double)), n_res, kk, n_k, r, now, N, out,
+                                       C.byref(late)))
+    return list(out), bool(late.value)
+
+
+def schedule_round(T, ks, requests, now: float, tau: float, N: int):
+    """requests: [(deadline, remaining_steps, table_row)] -> (survivors, [(gpus, steps)])."""
+    T, kk, n_res, n_k = _table(T, ks)
+    R = len(requests)
+    arr = _reqs(requests)
+    g = (C.c_int * max(R, 1))()
+    s = (C.c_int * max(R, 1))()
+    sv = C.c_int()
+    check_sched(lib.tsv_sched_round(T.ctypes.data_as(C.POINTER(C.c_double)), n_res, kk, n_k, arr, R, now, tau, N, g, s,
+                                    C.byref(sv)))
+    return sv.value, [(g[i], s[i]) for i in range(R)]

@@ -13,7 +13,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def _declared():
     names = set()
-    for h in ("tsv.h", "tsv_ops.h"):
+    for h in ("tsv.h", "tsv_ops.h", "tsv_sched.h"):
         src = open(os.path.join(ROOT, "include", h)).read()
         names |= set(re.findall(r"\b(tsv_[a-z_0-9]+)\s*\(", src))
     return names

@@ -1,0 +1,134 @@
+"""NEXT #1 — round-based scheduler (CPU): the C++ implementation against the plain oracle
+(oracle/sched.py) and the oracle's DP against exhaustive search (App. B)."""
+import itertools
+import math
+
+import numpy as np
+import pytest
+
+from oracle import sched as OS
+
+KS = [1, 2, 4, 8]
+
+
+def random_table(rng, n_res=4):
+    # T(res, k) shaped like a DiT step: sublinear scaling in k (Insight 2)
+    base = np.array([0.02, 0.05, 0.2, 1.0])[:n_res] * rng.uniform(0.8, 1.2, n_res)
+    eff = np.array([1.0, 0.9, 0.75, 0.55]) * rng.uniform(0.9, 1.0, 4)
+    T = base[:, None] / (np.array(KS)[None, :] * eff[None, :])
+    return T
+
+
+@pytest.fixture(scope="module")
+def sched():
+    import __graft_entry__
+    __graft_entry__.build()
+    from paper_conf_asplos_luhtlwm0c26_b200 import sched as S
+    return S
+
+
+def test_allocate_matches_oracle(sched):
+    rng = np.random.default_rng(0)
+    for _ in range(200):
+        T = random_table(rng)
+        row = int(rng.integers(0, 4))
+        steps = int(rng.integers(1, 21))
+        N = int(rng.choice([1, 2, 4, 8]))
+        budget = float(rng.uniform(0.2, 1.2)) * steps * T[row, 0]
+        spk, late = sched.allocate(T, KS, budget, steps, row, 0.0, N)
+        ref = OS.allocate(T[row], KS, steps, budget, N)
+        if ref is None:
+            assert late
+            assert sum(spk) == steps
+        else:
+            assert not late
+            got = sorted((s, k) for s, k in zip(spk, KS) if s)
+            assert got == sorted(ref)
+
+
+def test_allocation_optimality_brute_force():
+    """The oracle's allocation is the exact optimum of eq. (checked on small S against an
+    independent enumeration over per-step degree sequences)."""
+    rng = np.random.default_rng(1)
+    for _ in range(50):
+        T = random_table(rng)[0]
+        steps = int(rng.integers(1, 6))
+        budget = float(rng.uniform(0.3, 1.1)) * steps * T[0]
+        best = None
+        for seq in itertools.product(range(4), repeat=steps):
+            time = sum(T[j] for j in seq)
+            if time <= budget + 1e-12:
+                cost = sum(KS[j] * T[j] for j in seq)
+                best = cost if best is None else min(best, cost)
+        ref = OS.allocate(T, KS, steps, budget, 8)
+        if best is None:
+            assert ref is None
+        else:
+            assert math.isclose(sum(s * k * T[KS.index(k)] for s, k in ref), best, rel_tol=1e-9)
+
+
+def _instance(rng, R, N):
+    T = random_table(rng)
+    reqs = []
+    for _ in range(R):
+        row = int(rng.integers(0, 4))
+        steps = int(rng.integers(1, 21))
+        deadline = float(rng.uniform(0.1, 1.5)) * steps * T[row, 0]
+        reqs.append((deadline, steps, row))
+    return T, reqs
+
+
+def test_dp_equals_exhaustive():
+    """Alg. 1's group-knapsack DP attains the optimum of the per-round problem (exhaustive search,
+    App. B) on small instances (R <= 6, N <= 8)."""
+    rng = np.random.default_rng(2)
+    for _ in range(300):
+        R, N = int(rng.integers(1, 7)), int(rng.choice([1, 2, 4, 8]))
+        T, raw = _instance(rng, R, N)
+        tau = float(rng.uniform(0.05, 0.5))
+        reqs = []
+        for d, s, row in raw:
+            t_of = {k: t for k, t in zip(KS, T[row]) if k <= N}
+            alloc = OS.allocate(T[row], KS, s, d, N) or [(s, 1)]
+            reqs.append(dict(alloc=alloc, T=lambda A, t_of=t_of: t_of[A], T_min=min(t_of.values()), deadline=d))
+        v, plan = OS.dp_round(reqs, tau, 0.0, N)
+        assert v == OS.exhaustive_round(reqs, tau, 0.0, N)
+        assert sum(w for _, _, w in plan) <= N
+
+
+def test_round_matches_oracle(sched):
+    rng = np.random.default_rng(3)
+    for _ in range(300):
+        R, N = int(rng.integers(0, 9)), int(rng.choice([1, 2, 4, 8]))
+        T, reqs = _instance(rng, R, N)
+        tau = float(rng.uniform(0.05, 0.5))
+        now = float(rng.uniform(0, 0.05))
+        got = sched.schedule_round(T, KS, reqs, now, tau, N)
+        ref = OS.schedule_round(T, KS, reqs, now, tau, N)
+        assert got[0] == ref[0]
+        assert got[1] == [tuple(x) for x in ref[1]]
+        assert sum(g for g, _ in got[1]) <= N
+
+
+def test_round_semantics(sched):
+    T = np.array([[1.0, 0.6, 0.35, 0.2]])
+    # a single request that can only meet its deadline at k = 8 gets 8 GPUs
+    sv, plan = sched.schedule_round(T, KS, [(0.2 * 5 + 1e-9, 5, 0)], 0.0, 1.0, 8)
+    assert plan == [(8, 5)] and sv == 1
+    # with only 4 GPUs it is late: best effort on one GPU
+    sv, plan = sched.schedule_round(T, KS, [(1.0, 5, 0)], 0.0, 1.0, 4)
+    assert plan == [(1, 1)] and sv == 0
+    # bad arguments
+    with pytest.raises(Exception):
+        sched.schedule_round(T, KS, [(1.0, 5, 3)], 0.0, 1.0, 4)
+
+
+def test_scheduler_latency(sched):
+    """Decision time stays far below the paper's < 10 ms for 64 requests on 8 GPUs."""
+    import time
+    rng = np.random.default_rng(4)
+    T, reqs = _instance(rng, 64, 8)
+    t0 = time.perf_counter()
+    for _ in range(10):
+        sched.schedule_round(T, KS, reqs, 0.0, 0.25, 8)
+    assert (time.perf_counter() - t0) / 10 < 0.010
