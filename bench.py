@@ -30,6 +30,29 @@ sys.path.insert(0, ROOT)
 METRIC = "DiT step latency (ms) per resolution at SP=1/2/4/8; attn+GEMM TFLOP/s vs peak"
 
 
+def gemm_traffic(res: int):
+    """Mean DRAM bytes (read + write) per GEMM launch from the newest committed ncu launch list of
+    one step at this resolution (profiles/rNN/launches_<res>.csv), or None."""
+    import csv
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*", f"launches_{res}.csv")))
+    if not files:
+        return None
+    rows = list(csv.reader(open(files[-1])))
+    hi = [i for i, r in enumerate(rows) if "Kernel Name" in r][0]
+    h = rows[hi]
+    ii, ki, mi, vi, ui = (h.index(c) for c in ("ID", "Kernel Name", "Metric Name", "Metric Value", "Metric Unit"))
+    scale = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+    per = {}
+    for r in rows[hi + 1:]:
+        if len(r) > vi and "gemm" in r[ki] and r[mi].startswith("dram__bytes"):
+            per[r[ii]] = per.get(r[ii], 0.0) + float(r[vi].replace(",", "")) * scale.get(r[ui], 1.0)
+    if not per:
+        return None
+    return {"bytes_per_launch": round(sum(per.values()) / len(per)), "launches": len(per),
+            "source": os.path.relpath(files[-1], ROOT) + " (ncu, cold cache)"}
+
+
 def peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -250,6 +273,7 @@ def run_ours(args):
         e2e_ms = float(t.item())
 
     pk = peaks()
+    traffic = gemm_traffic(res) if world == 1 else None
     gemm_fl, attn_fl = flux_flops(res, world)
     g_ms = prof["gemm"]["ms"] / prof["gemm"]["launches"] if prof["gemm"]["launches"] else 0
     g_fl = prof["gemm"]["flops"] / max(prof["gemm"]["launches"], 1)
@@ -268,10 +292,15 @@ def run_ours(args):
                        "sp": world, "resolution": res, "global_batch": 1, "seq_len": Li + 512,
                        "parallelism": f"ulysses-sp{world}",
                        "l2": "inputs larger than L2 (23.7 GB of weights streamed per step); no flush"},
-            "roofline": {"bound": "tensor", "kernel": "gemm_tc_kernel (tcgen05 GEMM, all GEMM launches)",
+            "roofline": {"bound": "tensor",
+                         "kernel": "gemm_tc2_kernel / gemm_tc_kernel (tcgen05 GEMM, all GEMM launches of the step)",
                          "achieved": round(achieved, 2) if achieved else None, "peak": pk["tflops"],
                          "unit": "TFLOP/s", "frac": round(achieved / pk["tflops"], 4) if achieved else None,
-                         "traffic": None, "peak_source": pk["source"] + " bf16_tflops_sustained"},
+                         "traffic": traffic["bytes_per_launch"] if traffic else None,
+                         "traffic_detail": traffic,
+                         "algorithmic_bytes_per_launch": round(prof["gemm"]["bytes"] / max(prof["gemm"]["launches"], 1)),
+                         "algorithmic_flops_per_launch": round(g_fl),
+                         "peak_source": pk["source"] + " bf16_tflops_sustained"},
             "step_tflops": round(step_tf, 2), "attention_tflops": round(attn_tf, 2) if attn_tf else None,
             "time_share": shares,
             "e2e": {"value": round(e2e_ms, 4), "unit": "ms", "h2d_bytes_per_step": int(host.nbytes),
