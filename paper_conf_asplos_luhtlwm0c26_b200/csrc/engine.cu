@@ -137,6 +137,13 @@ struct Slot {
 };
 
 // per (request, slot): state that depends only on the request
+// one profiled launch: CUDA events around it on its stream (recorded again on every graph replay)
+struct ProfRec {
+  int cls;
+  int device;
+  cudaEvent_t a, b;
+};
+
 struct ReqDev {
   DevBuf mod;       // fp32 [S, n_mod]
   DevBuf dt;        // fp32 [S]
@@ -147,6 +154,10 @@ struct ReqDev {
   cudaGraphExec_t gexec = nullptr;
   uint64_t gkey = 0;
   int64_t gkernels = 0;
+  // profiled graphs: the event pairs captured in the graph and the per-class algorithmic counters
+  std::vector<ProfRec> gprof;
+  double gflops[8] = {0}, gbytes[8] = {0};
+  int64_t glaunch[8] = {0};
 };
 // per (request, slot, shard): state that depends on the group position
 struct ReqShard {
@@ -205,7 +216,6 @@ struct tsv_engine {
   // per-kernel-class profiling (tsv_engine_profile)
   bool prof = false;
   bool graphs = true;  // replay each step as a CUDA graph when a group has one local rank
-  struct ProfRec { int cls; int device; cudaEvent_t a, b; };
   std::vector<ProfRec> prof_recs;
   std::map<int, std::vector<cudaEvent_t>> ev_pool;  // by device
   double prof_flops[8] = {0}, prof_bytes[8] = {0};
@@ -926,7 +936,7 @@ static tsv_status do_step(tsv_engine* e, Request& R, int step, int gi, tsv_event
     int st = step;
     CK(cudaMemcpyAsync(c.rd->step.p, &st, sizeof(int), cudaMemcpyHostToDevice, c.s->stream));
   }
-  if (e->graphs && E.rc.size() == 1 && !e->prof) {
+  if (e->graphs && E.rc.size() == 1) {
     // one local rank: replay (or capture once) the whole step as a CUDA graph
     RankCtx& c = E.rc[0];
     ReqDev& rd = *c.rd;
@@ -938,14 +948,28 @@ static tsv_status do_step(tsv_engine* e, Request& R, int step, int gi, tsv_event
     for (const void* p : ptrs) mix(reinterpret_cast<uintptr_t>(p));
     mix((uint64_t)gi);
     mix((uint64_t)c.rows);
+    mix((uint64_t)e->prof);   // a profiled graph carries event-record nodes around every launch
     if (!rd.gexec || rd.gkey != key) {
       if (rd.gexec) { cudaGraphExecDestroy(rd.gexec); rd.gexec = nullptr; }
       CK(cudaSetDevice(c.s->device));
       const int64_t k0 = e->kernel_count;
+      const size_t r0 = e->prof_recs.size();
+      double f0[8], b0[8];
+      int64_t l0[8];
+      for (int i = 0; i < 8; ++i) { f0[i] = e->prof_flops[i]; b0[i] = e->prof_bytes[i]; l0[i] = e->prof_launch[i]; }
       CK(cudaStreamBeginCapture(c.s->stream, cudaStreamCaptureModeThreadLocal));
       tsv_status st = run_step(E);
       cudaGraph_t graph = nullptr;
       cudaError_t ce = cudaStreamEndCapture(c.s->stream, &graph);
+      // what ProfScope recorded during capture belongs to the graph: re-added at every replay
+      rd.gprof.assign(e->prof_recs.begin() + r0, e->prof_recs.end());
+      e->prof_recs.resize(r0);
+      for (int i = 0; i < 8; ++i) {
+        rd.gflops[i] = e->prof_flops[i] - f0[i];
+        rd.gbytes[i] = e->prof_bytes[i] - b0[i];
+        rd.glaunch[i] = e->prof_launch[i] - l0[i];
+        e->prof_flops[i] = f0[i]; e->prof_bytes[i] = b0[i]; e->prof_launch[i] = l0[i];
+      }
       if (st != TSV_OK) { if (graph) cudaGraphDestroy(graph); return st; }
       if (ce != cudaSuccess) return fail(TSV_E_CUDA, "step capture: %s", cudaGetErrorString(ce));
       ce = cudaGraphInstantiate(&rd.gexec, graph, 0);
@@ -957,6 +981,15 @@ static tsv_status do_step(tsv_engine* e, Request& R, int step, int gi, tsv_event
     }
     CK(cudaGraphLaunch(rd.gexec, c.s->stream));
     e->kernel_count += rd.gkernels;
+    if (e->prof) {
+      // the graph's event pairs now hold this replay's timestamps
+      e->prof_recs.insert(e->prof_recs.end(), rd.gprof.begin(), rd.gprof.end());
+      for (int i = 0; i < 8; ++i) {
+        e->prof_flops[i] += rd.gflops[i];
+        e->prof_bytes[i] += rd.gbytes[i];
+        e->prof_launch[i] += rd.glaunch[i];
+      }
+    }
   } else {
     TRY(run_step(E));
   }
@@ -1475,10 +1508,7 @@ tsv_status tsv_engine_set_graphs(tsv_engine* e, int enable) {
 
 tsv_status tsv_engine_profile(tsv_engine* e, int enable) {
   if (!e) return fail(TSV_E_INVAL, "null engine");
-  for (auto& r : e->prof_recs) {
-    e->ev_pool[r.device].push_back(r.a);
-    e->ev_pool[r.device].push_back(r.b);
-  }
+  // events are not recycled: profiled step graphs keep re-recording theirs
   e->prof_recs.clear();
   for (int i = 0; i < 8; ++i) { e->prof_flops[i] = 0; e->prof_bytes[i] = 0; e->prof_launch[i] = 0; }
   e->prof = enable != 0;
