@@ -163,3 +163,49 @@ def flux_step_sp(cfg: ModelCfg, W: Weights, x_lat, T, y, t: float, t_next: float
     v = [F.final_layer(W, img[r], vec) for r in range(k)]
     xs = shard(x_lat, k)
     return gather(v), gather([xs[r] + (t_next - t) * v[r] for r in range(k)])
+
+
+def sd3_step_sp(cfg: ModelCfg, W: Weights, x_lat, T_c, y_c, T_u, y_u, t: float, t_next: float,
+                height: int, width: int, k: int):
+    """sd3.sd3_step computed by k simulated Ulysses ranks (both CFG branches).  Rows after
+    the first all-to-all follow diffusers' joint order [img_0..img_{k-1}; txt_0..txt_{k-1}]."""
+    from . import sd3 as S3
+    H, D = cfg.heads, cfg.head_dim
+    if H % k:
+        raise ValueError("k must divide the head count (S24)")
+    L_i = x_lat.shape[0]
+    pe = shard(S3.pos_embed(cfg, height // 16, width // 16), k)
+
+    def branch(T, y):
+        L_t = T.shape[0]
+        vec = S3.conditioning_vec(cfg, W, t, y)
+        img = [F.linear(p, W["img_in.w"], W["img_in.b"]) + pe[r] for r, p in enumerate(shard(x_lat, k))]
+        txt = [F.linear(p, W["txt_in.w"], W["txt_in.b"]) for p in shard(T, k)]
+        for j in range(cfg.n_double):
+            last = j == cfg.n_double - 1
+            pi, pt = f"joint{j}.img.", f"joint{j}.txt."
+            mi = F.modulation(W, pi, vec, 6)
+            mt = F.modulation(W, pt, vec, 2 if last else 6)
+            t_sh, t_sc = (mt[1], mt[0]) if last else (mt[0], mt[1])
+            qi = [F.split_qkv(F.linear(F.ln_modulate(x, mi[0], mi[1]), W[pi + "qkv.w"], W[pi + "qkv.b"]), H, D)
+                  for x in img]
+            qt = [F.split_qkv(F.linear(F.ln_modulate(x, t_sh, t_sc), W[pt + "qkv.w"], W[pt + "qkv.b"]), H, D)
+                  for x in txt]
+            Q, K, V = (_a2a_seq_to_head([a[c] for a in qi], [a[c] for a in qt], k, H) for c in range(3))
+            O = [F.attention(Q[d], K[d], V[d]) for d in range(k)]
+            o_i, o_t = _a2a_head_to_seq(O, k, H, D, L_i, L_t)      # (first stream, second stream)
+            for r in range(k):
+                x = img[r] + mi[2] * F.linear(o_i[r], W[pi + "proj.w"], W[pi + "proj.b"])
+                hdn = F.gelu_tanh(F.linear(F.ln_modulate(x, mi[3], mi[4]), W[pi + "fc1.w"], W[pi + "fc1.b"]))
+                img[r] = x + mi[5] * F.linear(hdn, W[pi + "fc2.w"], W[pi + "fc2.b"])
+                if not last:
+                    x = txt[r] + mt[2] * F.linear(o_t[r], W[pt + "proj.w"], W[pt + "proj.b"])
+                    hdn = F.gelu_tanh(F.linear(F.ln_modulate(x, mt[3], mt[4]), W[pt + "fc1.w"], W[pt + "fc1.b"]))
+                    txt[r] = x + mt[5] * F.linear(hdn, W[pt + "fc2.w"], W[pt + "fc2.b"])
+        return [S3.final_layer(W, img[r], vec) for r in range(k)]
+
+    v_u = branch(T_u, y_u)
+    v_c = branch(T_c, y_c)
+    v = [v_u[r] + cfg.cfg_scale * (v_c[r] - v_u[r]) for r in range(k)]
+    xs = shard(x_lat, k)
+    return gather(v), gather([xs[r] + (t_next - t) * v[r] for r in range(k)])

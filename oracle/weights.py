@@ -42,3 +42,11 @@ def request_inputs(cfg: ModelCfg, height: int, width: int, seed: int):
     T = synth.gen_tensor(seed, 2, (cfg.text_tokens, cfg.ctx_dim), "x")
     y = synth.gen_tensor(seed, 3, (cfg.vec_dim,), "x")
     return x, T, y
+
+
+def sd3_request_inputs(cfg: ModelCfg, height: int, width: int, seed: int):
+    """SD3 CFG pair: x_T, (T_c, y_c) conditional, (T_u, y_u) unconditional (tensor ids 1-5)."""
+    x, T_c, y_c = request_inputs(cfg, height, width, seed)
+    T_u = synth.gen_tensor(seed, 4, (cfg.text_tokens, cfg.ctx_dim), "x")
+    y_u = synth.gen_tensor(seed, 5, (cfg.vec_dim,), "x")
+    return x, T_c, y_c, T_u, y_u

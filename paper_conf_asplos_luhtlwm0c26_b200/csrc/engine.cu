@@ -258,12 +258,14 @@ struct ProfScope {
     e->prof_bytes[cls] += bytes;
     e->prof_launch[cls] += 1;
     a = pool_event(e, s->device);
-    cudaEventRecord(a, s->stream);
+    // External: inside a step-graph capture this becomes an event-record node replayed with
+    // the graph (a plain record would only add an intra-graph dependency).
+    cudaEventRecordWithFlags(a, s->stream, cudaEventRecordExternal);
   }
   ~ProfScope() {
     if (!a) return;
     cudaEvent_t b = pool_event(e, s->device);
-    cudaEventRecord(b, s->stream);
+    cudaEventRecordWithFlags(b, s->stream, cudaEventRecordExternal);
     e->prof_recs.push_back({cls, s->device, a, b});
   }
 };
