@@ -1,13 +1,16 @@
 """Benchmark: one FLUX.1-dev-shaped denoising step (the whole hot path, S:§8(a) a1-a12) under
 step-level Ulysses SP, through libtsv.so's C-ABI.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--res 512] [--impl ours|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--res 512] [--model flux|sd3] [--impl ours|reference]
 
 N = 1: BASELINE.json config 2 (FLUX 512x512 = 1024 image + 512 text tokens, SP=1).
 N > 1 (torchrun, one process per GPU): the same request at SP = N on ranks [0..N) over NCCL
 (strong scaling: the step's work is fixed).  Metric: step latency (ms, lower is better), timed
 with CUDA events on the engine's stream, max over ranks.  Inputs are larger than L2 (23.7 GB of
 weights streamed per step), so no L2 flush is needed between timed steps.
+
+--model sd3: the SD3-medium-shaped CFG step of config 5 (24 joint blocks, L_t = 333, batch-2 CFG
+pair) instead of FLUX (a secondary line; the default N = 1 run is config 2).
 
 --impl reference: the float64 CPU oracle on the box's host cores (the tier's reference arm),
 timed on a bounded sample of the same step (one double + one single block at full width,
@@ -74,6 +77,27 @@ def flux_flops(res: int, k: int = 1, Lt: int = 512, h=3072, F=12288, H=24, D=128
     gemm += 2 * li * h * inch
     attn = (nd + ns) * 4 * L * L * D * (H // k)
     return gemm, attn
+
+
+def sd3_flops(res: int, k: int = 1, Lt: int = 333, h=1536, F=6144, H=24, D=64, nd=24, inch=64, ctx=4096, B=2):
+    """SD3 CFG step per rank: B = 2 evaluations; the last block's txt stream stops at its QKV."""
+    Li = (res // 16) ** 2
+    lt, li = -(-Lt // k), -(-Li // k)
+    L = Lt + Li
+    gemm = 2 * li * inch * h + B * 2 * lt * ctx * h
+    per_stream = h * (3 * h + h + 2 * F)
+    gemm += B * (nd * 2 * li * per_stream + (nd - 1) * 2 * lt * per_stream + 2 * lt * h * 3 * h)
+    gemm += B * 2 * li * h * inch
+    attn = B * nd * 4 * L * L * D * (H // k)
+    return gemm, attn
+
+
+MODELS = {
+    "flux": dict(Lt=512, flops=flux_flops, desc="FLUX.1-dev-shaped denoising step", shapes="FLUX.1-dev shapes",
+                 weights_gb=23.7),
+    "sd3": dict(Lt=333, flops=sd3_flops, desc="SD3-medium-shaped CFG denoising step (batch-2 CFG pair)",
+                shapes="SD3-medium shapes", weights_gb=4.2),
+}
 
 
 # --------------------------------------------------------------------------- clocks sampler
@@ -160,17 +184,48 @@ def oracle_sample(res: int, n_samples: int = 1):
                f"weights pre-generated (untimed); BLAS threads = {cores}")
 
 
+def oracle_sample_sd3(res: int):
+    """SD3: embed + joint block 0 + final of one CFG branch at full width, extrapolated to 24
+    joint blocks x 2 branches (weights pre-generated, not timed)."""
+    import numpy as np
+    from oracle import flux as F
+    from oracle import sd3 as S3
+    from oracle.config import SD3
+    from oracle.weights import Weights, sd3_request_inputs
+    cfg = SD3
+    W = Weights(cfg, cache_bytes=8 << 30)
+    x, Tc, yc, _, _ = sd3_request_inputs(cfg, res, res, 1000)
+    Li, Lt = x.shape[0], Tc.shape[0]
+    for n in W.table:
+        if n.startswith(("joint0.", "img_in", "txt_in", "final", "time_in", "vector_in")):
+            W[n]
+    vec = S3.conditioning_vec(cfg, W, 0.5, yc)
+    t0 = time.perf_counter()
+    img = F.linear(x, W["img_in.w"], W["img_in.b"]) + S3.pos_embed(cfg, res // 16, res // 16)
+    txt = F.linear(Tc, W["txt_in.w"], W["txt_in.b"])
+    t1 = time.perf_counter()
+    S3.joint_block(cfg, W, 0, img, txt, vec)
+    t2 = time.perf_counter()
+    S3.final_layer(W, img, vec)
+    t3 = time.perf_counter()
+    ms = 2 * ((t1 - t0) + cfg.n_double * (t2 - t1) + (t3 - t2)) * 1e3
+    cores = len(os.sched_getaffinity(0))
+    return ms, dict(kind="oracle", cores=cores,
+                    sample=f"float64 numpy oracle: embed + joint block 0 + final of one CFG branch of SD3 "
+                           f"{res}x{res} (L={Li + Lt}) at full width, extrapolated to 24 blocks x 2 branches; "
+                           f"weights pre-generated (untimed); BLAS threads = {cores}")
+
+
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
     res = args.res
-    for _ in range(min(args.warmup, 1)):
-        pass
+    mdl = MODELS[args.model]
     ms_list = []
     steps = max(1, min(args.steps, 3))
     for _ in range(steps):
-        ms, detail = oracle_sample(res)
+        ms, detail = (oracle_sample_sd3 if args.model == "sd3" else oracle_sample)(res)
         ms_list.append(ms)
     ms = statistics.median(ms_list)
     detail["value"] = ms
@@ -178,7 +233,7 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC, "value": ms, "unit": "ms", "n_gpus": args.gpus,
             "steps": steps, "warmup": 0, "ms_per_step": ms, "higher_is_better": False, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic (SYNTH-1 seeded weights and inputs)",
-            "config": {"workload": f"FLUX.1-dev-shaped step {res}x{res} ({(res // 16) ** 2} image + 512 text tokens)",
+            "config": {"workload": f"{mdl['desc']} {res}x{res} ({(res // 16) ** 2} image + {mdl['Lt']} text tokens)",
                        "sp": 1, "resolution": res},
             "cpu_baseline": detail,
             "e2e": {"value": ms, "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -201,7 +256,8 @@ def run_ours(args):
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    eng = tsv.Engine("flux", devices=[local], rank_base=rank, world_size=world)
+    mdl = MODELS[args.model]
+    eng = tsv.Engine(args.model, devices=[local], rank_base=rank, world_size=world)
     if world > 1:
         obj = [tsv.nccl_unique_id() if rank == 0 else None, tsv.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
@@ -273,8 +329,8 @@ def run_ours(args):
         e2e_ms = float(t.item())
 
     pk = peaks()
-    traffic = gemm_traffic(res) if world == 1 else None
-    gemm_fl, attn_fl = flux_flops(res, world)
+    traffic = gemm_traffic(res) if world == 1 and args.model == "flux" else None
+    gemm_fl, attn_fl = mdl["flops"](res, world)
     g_ms = prof["gemm"]["ms"] / prof["gemm"]["launches"] if prof["gemm"]["launches"] else 0
     g_fl = prof["gemm"]["flops"] / max(prof["gemm"]["launches"], 1)
     achieved = (g_fl / (g_ms * 1e-3)) / 1e12 if g_ms else None
@@ -287,11 +343,11 @@ def run_ours(args):
         line = {
             "metric": METRIC, "value": round(ms, 4), "unit": "ms", "n_gpus": world, "steps": K, "warmup": Wm,
             "ms_per_step": round(ms, 4), "higher_is_better": False, "scaling": "strong", "vs_baseline": None,
-            "dtype": "bf16", "data": "synthetic (SYNTH-1 seeded weights and inputs, FLUX.1-dev shapes)",
-            "config": {"workload": f"FLUX.1-dev-shaped denoising step {res}x{res} ({Li} image + 512 text tokens)",
-                       "sp": world, "resolution": res, "global_batch": 1, "seq_len": Li + 512,
+            "dtype": "bf16", "data": f"synthetic (SYNTH-1 seeded weights and inputs, {mdl['shapes']})",
+            "config": {"workload": f"{mdl['desc']} {res}x{res} ({Li} image + {mdl['Lt']} text tokens)",
+                       "sp": world, "resolution": res, "global_batch": 1, "seq_len": Li + mdl["Lt"],
                        "parallelism": f"ulysses-sp{world}",
-                       "l2": "inputs larger than L2 (23.7 GB of weights streamed per step); no flush"},
+                       "l2": f"inputs larger than L2 ({mdl['weights_gb']} GB of weights streamed per step); no flush"},
             "roofline": {"bound": "tensor",
                          "kernel": "gemm_tc2_kernel / gemm_tc_kernel (tcgen05 GEMM, all GEMM launches of the step)",
                          "achieved": round(achieved, 2) if achieved else None, "peak": pk["tflops"],
@@ -309,7 +365,7 @@ def run_ours(args):
             "clocks": clk.summary(),
         }
         if world == 1 and not args.no_cpu_baseline:
-            ms_cpu, detail = oracle_sample(res)
+            ms_cpu, detail = (oracle_sample_sd3 if args.model == "sd3" else oracle_sample)(res)
             detail["value"] = round(ms_cpu, 1)
             detail["unit"] = "ms"
             line["cpu_baseline"] = detail
@@ -326,6 +382,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--res", type=int, default=512)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--model", default="flux", choices=sorted(MODELS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":

@@ -54,6 +54,14 @@
  *            +0 mod.w [3h,h] +1 mod.b [3h] +2 lin1.w [3h+F,h] +3 lin1.b [3h+F] +4 q_norm.g [D]
  *            +5 k_norm.g [D] +6 lin2.w [h,h+F] +7 lin2.b [h]
  *   request inputs: 1 x_T [L_i,in] (fp32)  2 T [L_t,ctx] (bf16)  3 y [vec] (bf16)
+ *
+ * SD3 family (family = TSV_FAMILY_SD3): the same ids where the tensor exists.  Globals 0-7 and
+ * 12-19 (no guidance embedder; img_in = the 2x2 patch-embed conv flattened in (c, ph, pw) order;
+ * final.mod rows are (scale, shift)).  Joint block j, stream s: the double-block ids without the
+ * QK-norm gains (+4, +5); qkv.w stacks to_q; to_k; to_v (img) or add_q; add_k; add_v (txt).  The
+ * txt stream of the last block is context_pre_only: +0 mod.w [2h,h] (scale, shift), +1 mod.b
+ * [2h], +2 qkv.w, +3 qkv.b only.  Request inputs: 1 x_T, 2 T_c, 3 y_c (conditional branch),
+ * 4 T_u [L_t,ctx], 5 y_u [vec] (unconditional branch of the CFG pair).
  */
 #ifndef TSV_H_
 #define TSV_H_
@@ -94,10 +102,23 @@ typedef struct {
   int axes_dim[3];   /* RoPE axes split of D: (16, 56, 56) */
   float theta;       /* RoPE base: 10000 */
   int guidance_embed;/* 1: FLUX-dev guidance embedder present */
+  int family;        /* TSV_FAMILY_FLUX (double + single blocks, QK-RMSNorm, 3-axis RoPE) or
+                        TSV_FAMILY_SD3 (SD3-medium MMDiT: joint blocks only, no QK-norm, no RoPE,
+                        2-D sin-cos position embedding, context_pre_only last block, CFG pair;
+                        DESIGN.md O-SD3).  axes_dim / theta / guidance_embed are ignored for SD3. */
+  float cfg_scale;   /* SD3: classifier-free guidance scale s (7.0): v = v_u + s (v_c - v_u) */
+  float shift;       /* SD3: flow-matching schedule shift (3.0): t_j = s u / (1 + (s - 1) u), u = 1 - j/S */
+  int pe_max;        /* SD3: pos_embed_max_size (192) */
+  int pe_base;       /* SD3: base_size (64); patch (r, c) sits at ((r + top) pe_base / pe_max, ...) */
 } tsv_model_desc;
 
+#define TSV_FAMILY_FLUX 0
+#define TSV_FAMILY_SD3 1
+
 /* Named presets: "flux" (FLUX.1-dev shapes), "tiny" (config 1: h=256, H=4, D=64, F=1024,
- * 1 double block, L_t=64), "tiny_s" (tiny + 1 single block), "tiny2" (2 double + 2 single). */
+ * 1 double block, L_t=64), "tiny_s" (tiny + 1 single block), "tiny2" (2 double + 2 single),
+ * "sd3" (SD3-medium shapes, config 5: h=1536, H=24, D=64, F=6144, 24 joint blocks, L_t=333,
+ * ctx 4096, pooled 2048, CFG 7, shift 3) and "tiny_sd3" (h=256, H=4, 2 joint blocks, L_t=77). */
 tsv_status tsv_model_preset(const char* name, tsv_model_desc* out);
 
 /* Create an engine hosting global ranks [rank_base, rank_base + n_local) on devices[0..n_local).
@@ -122,20 +143,23 @@ tsv_status tsv_engine_init_world(tsv_engine* eng, const uint8_t nccl_id[128]);
 tsv_status tsv_group_create(tsv_engine* eng, const int* ranks, int k, const uint8_t* nccl_id, tsv_group* out);
 
 /* Create a request: height/width in pixels (multiples of 16, L_i = (H/16)(W/16)),
- * num_steps S >= 1, guidance g.  Inputs x_T, T, y are SYNTH-1 from `seed` (tensor ids 1-3) and
- * held in host memory until the first step lands on a group.  Errors: TSV_E_INVAL. */
+ * num_steps S >= 1, guidance g (FLUX guidance embedding; ignored for SD3, whose guidance is the
+ * model's cfg_scale).  Inputs x_T, T, y are SYNTH-1 from `seed` (tensor ids 1-3; SD3 also 4-5)
+ * and held in host memory until the first step lands on a group.  Errors: TSV_E_INVAL. */
 tsv_status tsv_request_create(tsv_engine* eng, int height_px, int width_px, int num_steps, uint64_t seed,
                               float guidance, tsv_request* out);
 
 /* Replace the request's inputs before its first step: x [L_i*in] fp32 row-major, T [L_t*ctx]
- * bf16 bits, y [vec] bf16 bits.  Any pointer may be NULL (keeps the current value).
+ * bf16 bits, y [vec] bf16 bits.  SD3: T is [2][L_t*ctx] = (T_c, T_u) and y is [2][vec] =
+ * (y_c, y_u).  Any pointer may be NULL (keeps the current value).
  * Errors: TSV_E_STATE if a step already ran. */
 tsv_status tsv_request_set_inputs(tsv_engine* eng, tsv_request req, const float* x, const uint16_t* T,
                                   const uint16_t* y);
 
 /* Run denoising step `step` of `req` on `group`:  v = DiT(x_s, t_s, T, y, g),
  * x_{s+1} = x_s + (t_{s+1} - t_s) v  (flow-matching Euler; schedule t_j = sigma(1 - j/S),
- * DESIGN.md).  `step` must equal the request's next step else TSV_E_STATE; if the
+ * DESIGN.md).  SD3: v = v_u + s (v_c - v_u) over the CFG pair, both branches in the same
+ * launches (batch 2, S23).  `step` must equal the request's next step else TSV_E_STATE; if the
  * group differs from the request's current group, the latent is resharded first (timed
  * separately).  Asynchronous: `done` (may be NULL) completes when every rank of the group
  * finished.  Multi-process: every process hosting a rank of the group makes the call; processes

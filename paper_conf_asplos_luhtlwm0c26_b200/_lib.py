@@ -34,7 +34,11 @@ class ModelDesc(C.Structure):
     _fields_ = [("hidden", C.c_int), ("heads", C.c_int), ("head_dim", C.c_int), ("mlp_hidden", C.c_int),
                 ("n_double", C.c_int), ("n_single", C.c_int), ("in_ch", C.c_int), ("ctx_dim", C.c_int),
                 ("vec_dim", C.c_int), ("text_tokens", C.c_int), ("axes_dim", C.c_int * 3), ("theta", C.c_float),
-                ("guidance_embed", C.c_int)]
+                ("guidance_embed", C.c_int), ("family", C.c_int), ("cfg_scale", C.c_float), ("shift", C.c_float),
+                ("pe_max", C.c_int), ("pe_base", C.c_int)]
+
+
+FAMILY_FLUX, FAMILY_SD3 = 0, 1
 
 
 class SchedRequest(C.Structure):

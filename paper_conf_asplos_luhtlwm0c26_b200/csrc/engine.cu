@@ -164,6 +164,10 @@ struct ReqShard {
   int rank_in_group = 0, k = 1;
   int64_t t0 = 0, nt = 0, i0 = 0, ni = 0;  // txt rows [t0, t0+nt), img rows [i0, i0+ni)
   DevBuf lat, vel, T, cosb, sinb;
+  DevBuf pe;  // SD3: fp32 [ni, h] sin-cos position embedding of this shard's image rows
+  void release() {
+    lat.release(); vel.release(); T.release(); cosb.release(); sinb.release(); pe.release();
+  }
 };
 
 struct Group {
@@ -184,8 +188,8 @@ struct Request {
   int next_step = 0;
   int group = -1;
   std::vector<float> x_host;      // [Li, in] until the first landing
-  std::vector<uint16_t> T_host;   // [Lt, ctx] bf16 bits
-  std::vector<uint16_t> y_host;   // [vec] bf16 bits
+  std::vector<uint16_t> T_host;   // [B][Lt, ctx] bf16 bits (SD3: branch 0 = T_c, 1 = T_u)
+  std::vector<uint16_t> y_host;   // [B][vec] bf16 bits
   std::vector<double> ts;         // t_0..t_S
   std::map<int, ReqDev> dev;      // by slot
   std::map<int, ReqShard> shard;  // by slot (current group)
@@ -277,16 +281,18 @@ static tsv_status gemm(tsv_engine* e, Slot& s, const bf16* A, long long lda, con
   const char* err = nullptr;
   if (gemm_plan(&p, A, lda, Wt, ldw, M, N, K, epi, s.ds->num_sms, &err))
     return fail(TSV_E_INVAL, "%s (M=%d N=%d K=%d)", err, M, N, K);
-  const double out_b = (epi.mode <= EPI_SPLIT_GELU) ? 2.0 : (epi.mode == EPI_STORE_F32 ? 4.0 : 8.0);
+  const double out_b = (epi.mode <= EPI_SPLIT_GELU) ? 2.0
+                       : (epi.mode == EPI_STORE_F32 ? 4.0 : (epi.mode == EPI_CFG_EULER ? 16.0 : 8.0));
   ProfScope ps(e, s, KC_GEMM, 2.0 * M * N * (double)K,
                2.0 * ((double)M * K + (double)N * K) + out_b * (double)M * N);
   gemm_launch(p, s.stream);
   return TSV_OK;
 }
-// Up to two problems with the same N, K in one persistent launch (the img and txt streams of a
-// double block): better wave quantization than two launches of half the tiles each.
+// Up to four problems with the same N, K in one persistent launch (the img and txt streams of a
+// double block; x2 for SD3's CFG pair): better wave quantization than one launch per problem.
 static tsv_status gemm_multi(tsv_engine* e, Slot& s, const GemmProblem* probs, int np, int N, int K) {
-  GemmProblem nz[2];
+  if (np > GEMM_MAX_PROBLEMS) return fail(TSV_E_INVAL, "gemm_multi: %d problems", np);
+  GemmProblem nz[GEMM_MAX_PROBLEMS];
   int n = 0;
   for (int i = 0; i < np; ++i)
     if (probs[i].M > 0) nz[n++] = probs[i];
@@ -297,7 +303,8 @@ static tsv_status gemm_multi(tsv_engine* e, Slot& s, const GemmProblem* probs, i
     return fail(TSV_E_INVAL, "%s (N=%d K=%d)", err, N, K);
   double fl = 0, by = 2.0 * N * K * n;
   for (int i = 0; i < n; ++i) {
-    const double out_b = (nz[i].epi.mode <= EPI_SPLIT_GELU) ? 2.0 : (nz[i].epi.mode == EPI_STORE_F32 ? 4.0 : 8.0);
+    const double out_b = (nz[i].epi.mode <= EPI_SPLIT_GELU) ? 2.0
+                         : (nz[i].epi.mode == EPI_STORE_F32 ? 4.0 : (nz[i].epi.mode == EPI_CFG_EULER ? 16.0 : 8.0));
     fl += 2.0 * nz[i].M * N * (double)K;
     by += 2.0 * nz[i].M * K + out_b * nz[i].M * N;
   }
@@ -345,14 +352,15 @@ static tsv_status ensure_reqdev(tsv_engine* e, Request& R, int si) {
   if (rd.ready) return TSV_OK;
   Slot& s = e->slots[si];
   const Model& m = e->model;
-  const int h = m.h, S = R.S;
+  const int h = m.h, S = R.S, B = m.B;
   CK(cudaSetDevice(s.device));
-  TRY(dev_alloc(rd.mod, s.device, (size_t)S * m.n_mod * 4));
+  TRY(dev_alloc(rd.mod, s.device, (size_t)S * B * m.n_mod * 4));
   TRY(dev_alloc(rd.dt, s.device, (size_t)S * 4));
-  TRY(dev_alloc(rd.cur, s.device, ((size_t)m.n_mod + 4) * 4));
+  TRY(dev_alloc(rd.cur, s.device, ((size_t)B * m.n_mod + 4) * 4));
   TRY(dev_alloc(rd.step, s.device, 16));
-  // host-side: sinusoidal embeddings e(t_s), e(g) (fp64 -> bf16), y (bf16), dt
-  const int Sp = S;
+  // host-side: sinusoidal embeddings e(t_s), e(g) (fp64 -> bf16), y (bf16), dt.  Row i*B + b is
+  // step i of CFG branch b (SD3: b = 0 conditional, 1 unconditional).
+  const int Sp = S * B;
   std::vector<uint16_t> et((size_t)Sp * 256), eg((size_t)Sp * 256), ey((size_t)Sp * m.vec);
   auto emb = [](double t, uint16_t* out) {
     for (int j = 0; j < 128; ++j) {
@@ -364,17 +372,19 @@ static tsv_status ensure_reqdev(tsv_engine* e, Request& R, int si) {
   };
   std::vector<float> dt(S);
   for (int i = 0; i < S; ++i) {
-    emb(R.ts[i], &et[(size_t)i * 256]);
-    emb((double)R.guidance, &eg[(size_t)i * 256]);
-    memcpy(&ey[(size_t)i * m.vec], R.y_host.data(), m.vec * 2);
+    for (int b = 0; b < B; ++b) {
+      emb(R.ts[i], &et[(size_t)(i * B + b) * 256]);
+      emb((double)R.guidance, &eg[(size_t)(i * B + b) * 256]);
+      memcpy(&ey[(size_t)(i * B + b) * m.vec], R.y_host.data() + (size_t)b * m.vec, m.vec * 2);
+    }
     dt[i] = (float)(R.ts[i + 1] - R.ts[i]);
   }
-  // scratch: et, eg, ey (bf16 [S,256],[S,256],[S,vec]); hid bf16 [S,h]; vec f32 [S,h]; asilu bf16 [S,h]
-  const size_t o_et = 0, o_eg = o_et + (size_t)S * 256 * 2, o_ey = o_eg + (size_t)S * 256 * 2;
-  const size_t o_hid = (o_ey + (size_t)S * m.vec * 2 + 255) & ~size_t(255);
-  const size_t o_vec = (o_hid + (size_t)S * h * 2 + 255) & ~size_t(255);
-  const size_t o_as = (o_vec + (size_t)S * h * 4 + 255) & ~size_t(255);
-  const size_t total = o_as + (size_t)S * h * 2;
+  // scratch: et, eg, ey (bf16 [Sp,256],[Sp,256],[Sp,vec]); hid bf16 [Sp,h]; vec f32 [Sp,h]; asilu bf16 [Sp,h]
+  const size_t o_et = 0, o_eg = o_et + (size_t)Sp * 256 * 2, o_ey = o_eg + (size_t)Sp * 256 * 2;
+  const size_t o_hid = (o_ey + (size_t)Sp * m.vec * 2 + 255) & ~size_t(255);
+  const size_t o_vec = (o_hid + (size_t)Sp * h * 2 + 255) & ~size_t(255);
+  const size_t o_as = (o_vec + (size_t)Sp * h * 4 + 255) & ~size_t(255);
+  const size_t total = o_as + (size_t)Sp * h * 2;
   TRY(dev_alloc(s.scratch, s.device, total));
   uint8_t* sc = reinterpret_cast<uint8_t*>(s.scratch.p);
   CK(cudaMemcpyAsync(sc + o_et, et.data(), et.size() * 2, cudaMemcpyHostToDevice, s.stream));
@@ -391,19 +401,19 @@ static tsv_status ensure_reqdev(tsv_engine* e, Request& R, int si) {
   bool first = true;
   for (auto& ml : mlps) {
     if (!ml.on) continue;
-    TRY(gemm(e, s, reinterpret_cast<bf16*>(sc + ml.off), ml.K, e->W(s, ml.w1), ml.K, S, h, ml.K,
+    TRY(gemm(e, s, reinterpret_cast<bf16*>(sc + ml.off), ml.K, e->W(s, ml.w1), ml.K, Sp, h, ml.K,
              epi_of(EPI_SILU_BF16, hid, h, e->W(s, ml.b1))));
-    TRY(gemm(e, s, hid, h, e->W(s, ml.w2), h, S, h, h,
+    TRY(gemm(e, s, hid, h, e->W(s, ml.w2), h, Sp, h, h,
              epi_of(first ? EPI_STORE_F32 : EPI_ACCUM_F32, vec, h, e->W(s, ml.b2))));
     first = false;
   }
   {
-    ProfScope ps(e, s, KC_OTHER, 0.0, (double)S * h * 6.0);
-    silu_bf16_launch(vec, h, as, h, S, h, s.stream);
+    ProfScope ps(e, s, KC_OTHER, 0.0, (double)Sp * h * 6.0);
+    silu_bf16_launch(vec, h, as, h, Sp, h, s.stream);
   }
-  // modulation table for all steps: [S, n_mod] = SiLU(vec) W_mod^T + b   (TT:layers.py:142)
+  // modulation table for all steps: [S*B, n_mod] = SiLU(vec) W_mod^T + b   (TT:layers.py:142)
   const bf16* wb = reinterpret_cast<const bf16*>(s.ds->weights.p);
-  TRY(gemm(e, s, as, h, wb + m.modw_off, h, S, (int)m.n_mod, h,
+  TRY(gemm(e, s, as, h, wb + m.modw_off, h, Sp, (int)m.n_mod, h,
            epi_of(EPI_STORE_F32, rd.mod.p, m.n_mod, wb + m.modb_off)));
   CK(cudaGetLastError());
   rd.ready = true;
@@ -433,6 +443,31 @@ static void rope_rows(const Model& m, const Request& R, int64_t t0, int64_t nt, 
   }
 }
 
+// SD3 2-D sin-cos position embedding of image rows [i0, i0 + ni) (fp64 -> fp32; DESIGN.md O-SD3,
+// S13): patch (r, c) of the n_r x n_c grid sits at ((r + top) / q, (c + left) / q), q = pe_max /
+// pe_base, top = floor((pe_max - n_r) / 2); channels [sin(c' w), cos(c' w), sin(r' w), cos(r' w)]
+// with w_j = 10000^(-j / (h/4)).
+static void pos_embed_rows(const Model& m, const Request& R, int64_t i0, int64_t ni, std::vector<float>& pe) {
+  const int64_t n_r = R.height / 16, n_c = R.width / 16;
+  const int quarter = m.h / 4;
+  auto floordiv2 = [](int64_t a) { return a >= 0 ? a / 2 : -((-a + 1) / 2); };
+  const int64_t top = floordiv2(m.d.pe_max - n_r), left = floordiv2(m.d.pe_max - n_c);
+  const double q = (double)m.d.pe_max / m.d.pe_base;
+  pe.assign((size_t)ni * m.h, 0.f);
+  for (int64_t r = 0; r < ni; ++r) {
+    const int64_t p = i0 + r;
+    const double pr = (double)(p / n_c + top) / q, pc = (double)(p % n_c + left) / q;
+    float* o = &pe[(size_t)r * m.h];
+    for (int j = 0; j < quarter; ++j) {
+      const double w = 1.0 / std::pow(10000.0, (double)j / quarter);
+      o[j] = (float)std::sin(pc * w);
+      o[quarter + j] = (float)std::cos(pc * w);
+      o[2 * quarter + j] = (float)std::sin(pr * w);
+      o[3 * quarter + j] = (float)std::cos(pr * w);
+    }
+  }
+}
+
 static tsv_status setup_shard(tsv_engine* e, Request& R, int si, int rank_in_group, int k, ReqShard& sh) {
   Slot& s = e->slots[si];
   const Model& m = e->model;
@@ -445,12 +480,25 @@ static tsv_status setup_shard(tsv_engine* e, Request& R, int si, int rank_in_gro
   CK(cudaSetDevice(s.device));
   TRY(dev_alloc(sh.lat, s.device, std::max<size_t>(1, sh.ni) * m.in * 4));
   TRY(dev_alloc(sh.vel, s.device, std::max<size_t>(1, sh.ni) * m.in * 4));
-  TRY(dev_alloc(sh.T, s.device, std::max<size_t>(1, sh.nt) * m.ctx * 2));
+  TRY(dev_alloc(sh.T, s.device, std::max<size_t>(1, sh.nt) * m.B * m.ctx * 2));
   const size_t rows = sh.nt + sh.ni;
+  if (sh.nt)
+    for (int b = 0; b < m.B; ++b)
+      CK(cudaMemcpyAsync(reinterpret_cast<uint16_t*>(sh.T.p) + (size_t)b * sh.nt * m.ctx,
+                         R.T_host.data() + ((size_t)b * R.Lt + sh.t0) * m.ctx, sh.nt * m.ctx * 2,
+                         cudaMemcpyHostToDevice, s.stream));
+  if (m.sd3) {
+    std::vector<float> pe;
+    pos_embed_rows(m, R, sh.i0, sh.ni, pe);
+    TRY(dev_alloc(sh.pe, s.device, std::max<size_t>(1, sh.ni) * m.h * 4));
+    if (sh.ni) {
+      CK(cudaMemcpyAsync(sh.pe.p, pe.data(), pe.size() * 4, cudaMemcpyHostToDevice, s.stream));
+      CK(cudaStreamSynchronize(s.stream));
+    }
+    return TSV_OK;
+  }
   TRY(dev_alloc(sh.cosb, s.device, std::max<size_t>(1, rows) * (m.D / 2) * 4));
   TRY(dev_alloc(sh.sinb, s.device, std::max<size_t>(1, rows) * (m.D / 2) * 4));
-  if (sh.nt)
-    CK(cudaMemcpyAsync(sh.T.p, R.T_host.data() + sh.t0 * m.ctx, sh.nt * m.ctx * 2, cudaMemcpyHostToDevice, s.stream));
   std::vector<float> c, sn;
   rope_rows(m, R, sh.t0, sh.nt, sh.i0, sh.ni, c, sn);
   if (rows) {
@@ -465,17 +513,18 @@ static tsv_status ensure_workspace(tsv_engine* e, Slot& s, int64_t rows, int64_t
   const Model& m = e->model;
   const int64_t h = m.h, F = m.F;
   Workspace& w = s.ws;
-  const int64_t r = std::max<int64_t>(rows, 1);
+  const int64_t r1 = std::max<int64_t>(rows, 1);
+  const int64_t r = r1 * m.B;  // every activation buffer holds the B evaluations back to back
   TRY(dev_alloc(w.x, s.device, r * h * 4));
   TRY(dev_alloc(w.u, s.device, r * h * 2));
   TRY(dev_alloc(w.qkv, s.device, r * 3 * h * 2));
   TRY(dev_alloc(w.cat, s.device, r * (h + F) * 2));
   TRY(dev_alloc(w.hbuf, s.device, r * F * 2));
-  TRY(dev_alloc(w.latb, s.device, r * m.in * 2));
+  TRY(dev_alloc(w.latb, s.device, r1 * m.in * 2));
   if (k > 1) {
     TRY(dev_alloc(w.pack, s.device, r * 3 * h * 2));
-    TRY(dev_alloc(w.recv, s.device, L * 3 * (h / k) * 2));
-    TRY(dev_alloc(w.obuf, s.device, L * (h / k) * 2));
+    TRY(dev_alloc(w.recv, s.device, m.B * L * 3 * (h / k) * 2));
+    TRY(dev_alloc(w.obuf, s.device, m.B * L * (h / k) * 2));
     TRY(dev_alloc(w.orecv, s.device, r * h * 2));
   }
   return TSV_OK;
@@ -544,20 +593,29 @@ static tsv_status a2a_exec(StepEnv& E, int which) {
   Group& g = *E.g;
   const int k = g.k;
   const int64_t w = (which == 1 ? 3 : 1) * (int64_t)m.h / k;  // bf16 per row
-  auto sendbuf = [&](RankCtx& c) { return which == 1 ? c.pack : c.obuf; };
-  auto recvbuf = [&](RankCtx& c) { return which == 1 ? c.recv : c.orecv; };
+  const int64_t L = E.R->Lt + E.R->Li;
+  // B evaluations (SD3's CFG pair) exchange back to back: the [k][rows_r] buffer of branch b
+  // starts at b * k * rows_r * w, the [L] buffer at b * L * w.
+  const int B = m.B;
+  auto sendbuf = [&](RankCtx& c, int b) {
+    return which == 1 ? c.pack + b * k * c.rows * w : c.obuf + b * L * w;
+  };
+  auto recvbuf = [&](RankCtx& c, int b) {
+    return which == 1 ? c.recv + b * L * w : c.orecv + b * k * c.rows * w;
+  };
   std::vector<A2AOp> ops;
   if (g.comm) {
     RankCtx& c = E.rc[0];
     const int r = g.local_positions[0];
     CK(cudaSetDevice(c.s->device));
-    ProfScope ps(e, *c.s, KC_A2A, 0.0, 2.0 * c.rows * w * (k - 1));
+    ProfScope ps(e, *c.s, KC_A2A, 0.0, 2.0 * B * c.rows * w * (k - 1));
     a2a_plan(which, E.R->Lt, E.R->Li, k, r, ops);
     NK(ncclGroupStart());
-    for (const A2AOp& o : ops) {
-      if (o.send) NK(ncclSend(sendbuf(c) + o.row0 * w, o.rows * w, ncclBfloat16, o.peer, g.comm, c.s->stream));
-      else NK(ncclRecv(recvbuf(c) + o.row0 * w, o.rows * w, ncclBfloat16, o.peer, g.comm, c.s->stream));
-    }
+    for (int b = 0; b < B; ++b)
+      for (const A2AOp& o : ops) {
+        if (o.send) NK(ncclSend(sendbuf(c, b) + o.row0 * w, o.rows * w, ncclBfloat16, o.peer, g.comm, c.s->stream));
+        else NK(ncclRecv(recvbuf(c, b) + o.row0 * w, o.rows * w, ncclBfloat16, o.peer, g.comm, c.s->stream));
+      }
     NK(ncclGroupEnd());
     return TSV_OK;
   }
@@ -568,7 +626,7 @@ static tsv_status a2a_exec(StepEnv& E, int which) {
   for (int d = 0; d < k; ++d) {
     RankCtx& dst = E.rc[d];
     CK(cudaSetDevice(dst.s->device));
-    ProfScope ps(e, *dst.s, KC_A2A, 0.0, 2.0 * dst.rows * w * (k - 1), 0);
+    ProfScope ps(e, *dst.s, KC_A2A, 0.0, 2.0 * B * dst.rows * w * (k - 1), 0);
     for (int r = 0; r < k; ++r) CK(cudaStreamWaitEvent(dst.s->stream, g.ev_a[r], 0));
     std::vector<int> nth_recv(k, 0);
     for (const A2AOp& o : plans[d]) {
@@ -580,8 +638,9 @@ static tsv_status a2a_exec(StepEnv& E, int which) {
         if (so.send && so.peer == d && seen++ == idx) { match = &so; break; }
       if (!match || match->rows != o.rows) return fail(TSV_E_STATE, "all-to-all plan mismatch");
       RankCtx& src = E.rc[p];
-      CK(cudaMemcpyPeerAsync(recvbuf(dst) + o.row0 * w, dst.s->device, sendbuf(src) + match->row0 * w, src.s->device,
-                             o.rows * w * 2, dst.s->stream));
+      for (int b = 0; b < B; ++b)
+        CK(cudaMemcpyPeerAsync(recvbuf(dst, b) + o.row0 * w, dst.s->device, sendbuf(src, b) + match->row0 * w,
+                               src.s->device, o.rows * w * 2, dst.s->stream));
     }
     CK(cudaEventRecord(g.ev_b[d], dst.s->stream));
   }
@@ -601,11 +660,12 @@ static tsv_status a2a_o(StepEnv& E) {
   TRY(a2a_exec(E, 2));
   for (auto& c : E.rc) {
     CK(cudaSetDevice(c.s->device));
-    for (int d = 0; d < k; ++d) {
-      ProfScope ps(e, *c.s, KC_OTHER, 0.0, 4.0 * c.rows * w);
-      copy2d_bf16_launch(c.orecv + (int64_t)d * c.rows * w, w, c.cat + d * w, m.h + m.F, (int)c.rows, (int)w,
-                         c.s->stream);
-    }
+    for (int b = 0; b < m.B; ++b)
+      for (int d = 0; d < k; ++d) {
+        ProfScope ps(e, *c.s, KC_OTHER, 0.0, 4.0 * c.rows * w);
+        copy2d_bf16_launch(c.orecv + ((int64_t)b * k + d) * c.rows * w, w, c.cat + b * c.rows * (m.h + m.F) + d * w,
+                           m.h + m.F, (int)c.rows, (int)w, c.s->stream);
+      }
   }
   return TSV_OK;
 }
@@ -619,17 +679,21 @@ static tsv_status attention_all(StepEnv& E) {
   for (auto& c : E.rc) {
     CK(cudaSetDevice(c.s->device));
     const double Lq = k == 1 ? (double)c.rows : (double)L;
-    ProfScope ps(e, *c.s, KC_ATTN, 4.0 * Lq * Lq * m.D * (m.H / k), 8.0 * Lq * m.D * (m.H / k));
-    int rc;
-    if (k == 1) {
-      rc = attention_launch(c.qkv, 3 * m.h, c.qkv + m.h, 3 * m.h, c.qkv + 2 * m.h, 3 * m.h, c.cat, m.h + m.F,
-                            (int)c.rows, m.H, m.D, c.s->stream);
-    } else {
-      const int64_t w = 3 * (int64_t)m.h / k;
-      rc = attention_launch(c.recv, w, c.recv + m.h / k, w, c.recv + 2 * m.h / k, w, c.obuf, m.h / k, (int)L,
-                            m.H / k, m.D, c.s->stream);
+    for (int b = 0; b < m.B; ++b) {  // one launch per evaluation (SD3: CFG branch)
+      ProfScope ps(e, *c.s, KC_ATTN, 4.0 * Lq * Lq * m.D * (m.H / k), 8.0 * Lq * m.D * (m.H / k));
+      int rc;
+      if (k == 1) {
+        const bf16* q = c.qkv + b * c.rows * 3 * m.h;
+        rc = attention_launch(q, 3 * m.h, q + m.h, 3 * m.h, q + 2 * m.h, 3 * m.h, c.cat + b * c.rows * (m.h + m.F),
+                              m.h + m.F, (int)c.rows, m.H, m.D, c.s->stream);
+      } else {
+        const int64_t w = 3 * (int64_t)m.h / k;
+        const bf16* q = c.recv + b * L * w;
+        rc = attention_launch(q, w, q + m.h / k, w, q + 2 * m.h / k, w, c.obuf + b * L * (m.h / k), m.h / k, (int)L,
+                              m.H / k, m.D, c.s->stream);
+      }
+      if (rc) return fail(TSV_E_CUDA, "attention: tensor map creation failed");
     }
-    if (rc) return fail(TSV_E_CUDA, "attention: tensor map creation failed");
   }
   return TSV_OK;
 }
@@ -663,6 +727,8 @@ static void lnmod2(StepEnv& E, RankCtx& c, int64_t mod_txt, int64_t mod_img, int
   ln_mod2_launch(c.x, h, c.u, h, mt, mt + h, mi, mi + h, (int)c.nt, (int)c.rows, h, c.s->stream);
 }
 
+static tsv_status run_step_sd3(StepEnv& E);
+
 static tsv_status run_step(StepEnv& E) {
   tsv_engine* e = E.e;
   const Model& m = e->model;
@@ -673,12 +739,14 @@ static tsv_status run_step(StepEnv& E) {
   for (auto& c : E.rc) {
     Slot& s = *c.s;
     CK(cudaSetDevice(s.device));
-    ProfScope ps(e, s, KC_OTHER, 0.0, 8.0 * m.n_mod, 2);
+    const int64_t nm = m.B * m.n_mod;
+    ProfScope ps(e, s, KC_OTHER, 0.0, 8.0 * nm, 2);
     const int* step_dev = reinterpret_cast<const int*>(c.rd->step.p);
     float* cur = reinterpret_cast<float*>(c.rd->cur.p);
-    select_row_launch(reinterpret_cast<const float*>(c.rd->mod.p), m.n_mod, step_dev, cur, m.n_mod, s.stream);
-    select_row_launch(reinterpret_cast<const float*>(c.rd->dt.p), 1, step_dev, cur + m.n_mod, 1, s.stream);
+    select_row_launch(reinterpret_cast<const float*>(c.rd->mod.p), nm, step_dev, cur, nm, s.stream);
+    select_row_launch(reinterpret_cast<const float*>(c.rd->dt.p), 1, step_dev, cur + nm, 1, s.stream);
   }
+  if (m.sd3) return run_step_sd3(E);
   // a1: embeddings
   for (auto& c : E.rc) {
     Slot& s = *c.s;
@@ -776,6 +844,139 @@ static tsv_status run_step(StepEnv& E) {
   return TSV_OK;
 }
 
+// SD3-medium step (DESIGN.md O-SD3).  B = 2 evaluations (b = 0 conditional, b = 1 unconditional
+// branch of the CFG pair, S23) share every launch: evaluation b owns rows [b*rows, (b+1)*rows) of
+// each activation buffer, laid out [txt_r ; img_r] like FLUX.  Joint blocks are double blocks
+// without QK-norm and RoPE, so the QKV epilogue is a plain store (k = 1) or a pure Ulysses pack
+// (k > 1); joint attention over [txt; img] equals diffusers' [img; txt] (no position-dependent
+// term, the softmax is permutation-equivariant).  The last block's txt stream is context_pre_only
+// (AdaLayerNormContinuous (scale, shift), QKV only).  The CFG combine is fused into the Euler
+// epilogue of the final linear.
+static tsv_status run_step_sd3(StepEnv& E) {
+  tsv_engine* e = E.e;
+  const Model& m = e->model;
+  const int h = m.h, F = m.F, B = m.B;
+  const int64_t ldc = h + F, nm = m.n_mod;
+  const int k = E.g->k;
+  const int nd = m.d.n_double;
+  // a1: img = x W^T + b + PE (identical for both evaluations), txt_b = T_b W^T + b
+  for (auto& c : E.rc) {
+    Slot& s = *c.s;
+    CK(cudaSetDevice(s.device));
+    const int64_t R = c.rows;
+    if (c.ni) {
+      float* xi0 = c.x + c.nt * h;
+      {
+        ProfScope ps(e, s, KC_OTHER, 0.0, 6.0 * c.ni * m.in);
+        f32_to_bf16_launch(reinterpret_cast<float*>(c.sh->lat.p), m.in, c.latb, m.in, (int)c.ni, m.in, s.stream);
+      }
+      CK(cudaMemcpyAsync(xi0, c.sh->pe.p, c.ni * h * 4, cudaMemcpyDeviceToDevice, s.stream));
+      TRY(gemm(e, s, c.latb, m.in, e->W(s, 0), m.in, (int)c.ni, h, m.in, epi_of(EPI_ACCUM_F32, xi0, h, e->W(s, 1))));
+      for (int b = 1; b < B; ++b)
+        CK(cudaMemcpyAsync(xi0 + b * R * h, xi0, c.ni * h * 4, cudaMemcpyDeviceToDevice, s.stream));
+    }
+    if (c.nt) {
+      GemmProblem pt[2];
+      for (int b = 0; b < B; ++b)
+        pt[b] = {reinterpret_cast<bf16*>(c.sh->T.p) + b * c.nt * m.ctx, m.ctx, e->W(s, 2), m.ctx, (int)c.nt,
+                 epi_of(EPI_STORE_F32, c.x + b * R * h, h, e->W(s, 3))};
+      TRY(gemm_multi(e, s, pt, B, h, m.ctx));
+    }
+  }
+  for (int j = 0; j < nd; ++j) {
+    const bool last = j == nd - 1;  // context_pre_only
+    for (auto& c : E.rc) {
+      Slot& s = *c.s;
+      CK(cudaSetDevice(s.device));
+      const int64_t R = c.rows;
+      if (!R) continue;
+      // a2: LN-modulate both streams of both evaluations
+      for (int b = 0; b < B; ++b) {
+        const float* mi = c.mod + b * nm + m.mod_double(j, 0);
+        const float* mt = c.mod + b * nm + m.mod_double(j, 1);
+        ProfScope ps(e, s, KC_LNMOD, 0.0, (double)R * h * 6.0 + 16.0 * h);
+        ln_mod2_launch(c.x + b * R * h, h, c.u + b * R * h, h, last ? mt + h : mt, last ? mt : mt + h, mi, mi + h,
+                       (int)c.nt, (int)R, h, s.stream);
+      }
+      // a3 (+ Ulysses pack for k > 1): 2 streams x 2 evaluations in one launch
+      GemmProblem pq[GEMM_MAX_PROBLEMS];
+      int n = 0;
+      for (int b = 0; b < B; ++b)
+        for (int st = 0; st < 2; ++st) {
+          const int base = double_base(j, st);
+          const int64_t r0 = st == 0 ? c.nt : 0, nr = st == 0 ? c.ni : c.nt;
+          GemmEpi ep = epi_of(EPI_STORE_BF16, c.qkv + (b * R + r0) * 3 * h, 3 * h, e->W(s, base + 3));
+          if (k > 1) {
+            ep.qk_h = h; ep.qk_D = m.D; ep.k_sp = k;
+            ep.pack = c.pack + b * R * 3 * h; ep.pack_rows = (int)R; ep.pack_row0 = (int)r0;
+          }
+          pq[n++] = {c.u + (b * R + r0) * h, h, e->W(s, base + 2), h, (int)nr, ep};
+        }
+      TRY(gemm_multi(e, s, pq, n, 3 * h, h));
+    }
+    if (k > 1) TRY(a2a_qkv(E));
+    TRY(attention_all(E));
+    if (k > 1) TRY(a2a_o(E));
+    for (auto& c : E.rc) {
+      Slot& s = *c.s;
+      CK(cudaSetDevice(s.device));
+      const int64_t R = c.rows;
+      if (!R) continue;
+      GemmProblem pp[GEMM_MAX_PROBLEMS], p1[GEMM_MAX_PROBLEMS], p2[GEMM_MAX_PROBLEMS];
+      int n = 0;
+      for (int b = 0; b < B; ++b)
+        for (int st = 0; st < 2; ++st) {
+          if (last && st == 1) continue;  // the context_pre_only txt stream ends at its QKV
+          const int base = double_base(j, st);
+          const int64_t r0 = st == 0 ? c.nt : 0, nr = st == 0 ? c.ni : c.nt;
+          const float* md = c.mod + b * nm + m.mod_double(j, st);
+          float* x = c.x + (b * R + r0) * h;
+          pp[n] = {c.cat + (b * R + r0) * ldc, ldc, e->W(s, base + 6), h, (int)nr,
+                   epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 7), md + 2 * h)};
+          p1[n] = {c.u + (b * R + r0) * h, h, e->W(s, base + 8), h, (int)nr,
+                   epi_of(EPI_GELU_BF16, c.hbuf + (b * R + r0) * F, F, e->W(s, base + 9))};
+          p2[n] = {c.hbuf + (b * R + r0) * F, F, e->W(s, base + 10), F, (int)nr,
+                   epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 11), md + 5 * h)};
+          ++n;
+        }
+      TRY(gemm_multi(e, s, pp, n, h, h));  // a8: out-proj + gated residual
+      for (int b = 0; b < B; ++b) {         // a9: LN-modulate
+        const float* mi = c.mod + b * nm + m.mod_double(j, 0);
+        const float* mt = c.mod + b * nm + m.mod_double(j, 1);
+        if (last) {
+          lnmod(e, s, c.x + (b * R + c.nt) * h, c.u + (b * R + c.nt) * h, mi + 3 * h, mi + 4 * h, (int)c.ni);
+        } else {
+          ProfScope ps(e, s, KC_LNMOD, 0.0, (double)R * h * 6.0 + 16.0 * h);
+          ln_mod2_launch(c.x + b * R * h, h, c.u + b * R * h, h, mt + 3 * h, mt + 4 * h, mi + 3 * h, mi + 4 * h,
+                         (int)c.nt, (int)R, h, s.stream);
+        }
+      }
+      TRY(gemm_multi(e, s, p1, n, F, h));  // fc1 + GELU
+      TRY(gemm_multi(e, s, p2, n, h, F));  // fc2 + gated residual
+    }
+  }
+  // final: AdaLayerNormContinuous (scale, shift) per evaluation, linear; v_u stored, then the
+  // conditional GEMM's epilogue forms v = v_u + s (v_c - v_u) and x += dt v
+  for (auto& c : E.rc) {
+    Slot& s = *c.s;
+    CK(cudaSetDevice(s.device));
+    if (!c.ni) continue;
+    const int64_t R = c.rows;
+    for (int b = 0; b < B; ++b) {
+      const float* md = c.mod + b * nm + m.mod_final();
+      lnmod(e, s, c.x + (b * R + c.nt) * h, c.u + b * R * h, md + h, md, (int)c.ni);
+    }
+    const float* dt = reinterpret_cast<const float*>(c.rd->cur.p) + B * nm;
+    TRY(gemm(e, s, c.u + R * h, h, e->W(s, 18), h, (int)c.ni, m.in, h,
+             epi_of(EPI_STORE_F32, c.sh->vel.p, m.in, e->W(s, 19))));
+    GemmEpi ep = epi_of(EPI_CFG_EULER, c.sh->lat.p, m.in, e->W(s, 19), nullptr, c.sh->vel.p, m.in, 0, dt);
+    ep.alpha = m.d.cfg_scale;
+    TRY(gemm(e, s, c.u, h, e->W(s, 18), h, (int)c.ni, m.in, h, ep));
+  }
+  for (auto& c : E.rc) CK(cudaGetLastError());
+  return TSV_OK;
+}
+
 // ------------------------------------------------------------------ landing / reshard
 static tsv_status record_last(tsv_engine* e, Request& R, int si) {
   Slot& s = e->slots[si];
@@ -861,10 +1062,7 @@ static tsv_status move_request(tsv_engine* e, Request& R, int gi) {
     // old buffers: wait until every copy finished before freeing
     for (auto& kv : next) TRY(record_last(e, R, kv.first));
     for (auto& kv : next) CK(cudaEventSynchronize(R.last[kv.first]));
-    for (auto& kv : R.shard) {
-      kv.second.lat.release(); kv.second.vel.release(); kv.second.T.release();
-      kv.second.cosb.release(); kv.second.sinb.release();
-    }
+    for (auto& kv : R.shard) kv.second.release();
   }
   R.shard.swap(next);
   R.group = gi;
@@ -945,8 +1143,8 @@ static tsv_status do_step(tsv_engine* e, Request& R, int step, int gi, tsv_event
     uint64_t key = 1469598103934665603ull;
     auto mix = [&](uint64_t v) { key = (key ^ v) * 1099511628211ull; };
     const void* ptrs[] = {c.x, c.u, c.qkv, c.cat, c.hbuf, c.latb, c.pack, c.recv, c.obuf, c.orecv,
-                          c.sh->lat.p, c.sh->vel.p, c.sh->T.p, c.sh->cosb.p, c.sh->sinb.p, rd.mod.p, rd.cur.p,
-                          rd.step.p};
+                          c.sh->lat.p, c.sh->vel.p, c.sh->T.p, c.sh->cosb.p, c.sh->sinb.p, c.sh->pe.p, rd.mod.p,
+                          rd.cur.p, rd.step.p};
     for (const void* p : ptrs) mix(reinterpret_cast<uintptr_t>(p));
     mix((uint64_t)gi);
     mix((uint64_t)c.rows);
@@ -1028,6 +1226,13 @@ tsv_status tsv_model_preset(const char* name, tsv_model_desc* out) {
     d = {256, 4, 64, 1024, 1, 0, 64, 512, 256, 64, {8, 28, 28}, 10000.f, 1};
     if (n == "tiny_s") d.n_single = 1;
     if (n == "tiny2") { d.n_double = 2; d.n_single = 2; }
+  } else if (n == "sd3" || n == "tiny_sd3") {
+    // SD3-medium (config 5): h 1536, 24 heads of 64, F 6144, 24 joint blocks, L_t = 333 (77 CLIP +
+    // 256 T5), ctx 4096, pooled 2048; "tiny_sd3": h 256, 4 heads, 2 joint blocks, L_t = 77
+    d = {1536, 24, 64, 6144, 24, 0, 64, 4096, 2048, 333, {0, 0, 0}, 10000.f, 0};
+    if (n == "tiny_sd3") { d.hidden = 256; d.heads = 4; d.mlp_hidden = 1024; d.n_double = 2; d.ctx_dim = 512;
+                           d.vec_dim = 256; d.text_tokens = 77; }
+    d.family = TSV_FAMILY_SD3; d.cfg_scale = 7.0f; d.shift = 3.0f; d.pe_max = 192; d.pe_base = 64;
   } else {
     return fail(TSV_E_INVAL, "unknown preset '%s'", name);
   }
@@ -1093,10 +1298,7 @@ void tsv_engine_destroy(tsv_engine* e) {
   }
   for (auto& kv : e->requests) {
     for (auto& d : kv.second.dev) release_reqdev(d.second);
-    for (auto& sh : kv.second.shard) {
-      sh.second.lat.release(); sh.second.vel.release(); sh.second.T.release();
-      sh.second.cosb.release(); sh.second.sinb.release();
-    }
+    for (auto& sh : kv.second.shard) sh.second.release();
     for (auto& l : kv.second.last) cudaEventDestroy(l.second);
   }
   for (auto& g : e->groups) {
@@ -1214,19 +1416,33 @@ tsv_status tsv_request_create(tsv_engine* e, int height, int width, int num_step
   R.Lt = m.Lt;
   R.x_host.resize((size_t)R.Li * m.in);
   for (size_t i = 0; i < R.x_host.size(); ++i) R.x_host[i] = synth_r(seed, 1, i) * synth_scale(1.0);
-  R.T_host.resize((size_t)R.Lt * m.ctx);
+  // T, y of evaluation b: SYNTH-1 ids (2, 3) for b = 0 and (4, 5) for SD3's unconditional b = 1
+  const size_t nT = (size_t)R.Lt * m.ctx;
   const float c1 = synth_scale(1.0);
-  for (size_t i = 0; i < R.T_host.size(); ++i) R.T_host[i] = f32_to_bf16_bits(synth_r(seed, 2, i) * c1);
-  R.y_host.resize(m.vec);
-  for (size_t i = 0; i < R.y_host.size(); ++i) R.y_host[i] = f32_to_bf16_bits(synth_r(seed, 3, i) * c1);
-  // schedule t_j = sigma(1 - j/S), sigma(u) = e^mu / (e^mu + (1/u - 1)), mu linear in L_i
-  const double mu = 0.5 + (1.15 - 0.5) / (4096.0 - 256.0) * ((double)R.Li - 256.0);
+  R.T_host.resize(nT * m.B);
+  R.y_host.resize((size_t)m.vec * m.B);
+  for (int b = 0; b < m.B; ++b) {
+    for (size_t i = 0; i < nT; ++i) R.T_host[b * nT + i] = f32_to_bf16_bits(synth_r(seed, 2 + 2 * b, i) * c1);
+    for (int i = 0; i < m.vec; ++i) R.y_host[(size_t)b * m.vec + i] = f32_to_bf16_bits(synth_r(seed, 3 + 2 * b, i) * c1);
+  }
   R.ts.resize(num_steps + 1);
-  for (int j = 0; j <= num_steps; ++j) {
-    const double u = 1.0 - (double)j / num_steps;
-    R.ts[j] = u > 0 ? std::exp(mu) / (std::exp(mu) + (1.0 / u - 1.0)) : 0.0;
+  if (m.sd3) {
+    // SD3: t_j = s u / (1 + (s - 1) u), u = 1 - j/S (shift s = 3; S20)
+    const double sh = m.d.shift;
+    for (int j = 0; j <= num_steps; ++j) {
+      const double u = 1.0 - (double)j / num_steps;
+      R.ts[j] = sh * u / (1.0 + (sh - 1.0) * u);
+    }
+  } else {
+    // schedule t_j = sigma(1 - j/S), sigma(u) = e^mu / (e^mu + (1/u - 1)), mu linear in L_i
+    const double mu = 0.5 + (1.15 - 0.5) / (4096.0 - 256.0) * ((double)R.Li - 256.0);
+    for (int j = 0; j <= num_steps; ++j) {
+      const double u = 1.0 - (double)j / num_steps;
+      R.ts[j] = u > 0 ? std::exp(mu) / (std::exp(mu) + (1.0 / u - 1.0)) : 0.0;
+    }
   }
   R.ts[0] = 1.0;
+  R.ts[num_steps] = 0.0;
   const int64_t id = e->next_req++;
   e->requests.emplace(id, std::move(R));
   *out = id;
@@ -1380,10 +1596,7 @@ tsv_status tsv_request_destroy(tsv_engine* e, tsv_request r) {
   Request& R = it->second;
   for (auto& l : R.last) { cudaEventSynchronize(l.second); cudaEventDestroy(l.second); }
   for (auto& d : R.dev) release_reqdev(d.second);
-  for (auto& sh : R.shard) {
-    sh.second.lat.release(); sh.second.vel.release(); sh.second.T.release();
-    sh.second.cosb.release(); sh.second.sinb.release();
-  }
+  for (auto& sh : R.shard) sh.second.release();
   e->requests.erase(it);
   return TSV_OK;
 }

@@ -33,16 +33,17 @@ struct GemmCfg {
   static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ + 4 * 32 * 36 * 4;
 };
 
-// Up to two problems with the same N and K (e.g. the img and txt streams of a double block)
-// share one persistent launch: tiles [0, tile0[1]) belong to problem 0, the rest to problem 1.
+// Up to GEMM_MAX_PROBLEMS problems with the same N and K (e.g. the img and txt streams of a double
+// block, times the two CFG branches for SD3) share one persistent launch: tiles
+// [tile0[q], tile0[q+1]) belong to problem q.
 struct GemmArgs {
   int N, K, num_n, num_tiles, nprob;
-  int M[2], num_m[2], tile0[2];
-  GemmEpi epi[2];
+  int M[GEMM_MAX_PROBLEMS], num_m[GEMM_MAX_PROBLEMS], tile0[GEMM_MAX_PROBLEMS];
+  GemmEpi epi[GEMM_MAX_PROBLEMS];
 };
 struct GemmMaps {
-  CUtensorMap A[2];
-  CUtensorMap B[2];
+  CUtensorMap A[GEMM_MAX_PROBLEMS];
+  CUtensorMap B[GEMM_MAX_PROBLEMS];
 };
 
 // Rasterisation: groups of GROUP_N weight-column tiles; inside a group the n index varies fastest,
@@ -51,7 +52,10 @@ struct GemmMaps {
 // num_n / GROUP_N times instead of num_n times (measured: 2.8 GB -> algorithmic for 2048^2 fc1).
 constexpr int GROUP_N = 8;
 __device__ __forceinline__ void decode_tile(const GemmArgs& a, int t, int& p, int& m_blk, int& n_blk) {
-  p = (a.nprob > 1 && t >= a.tile0[1]) ? 1 : 0;
+  p = 0;
+#pragma unroll
+  for (int q = 1; q < GEMM_MAX_PROBLEMS; ++q)
+    if (q < a.nprob && t >= a.tile0[q]) p = q;
   const int lt = t - a.tile0[p];
   const int nm = a.num_m[p];
   const int group = lt / (GROUP_N * nm);
@@ -125,7 +129,7 @@ __device__ __forceinline__ void epilogue_qk_head(const GemmEpi& e, int M, int ro
                                                  float* stg, int lane) {
   const int D = e.qk_D;
   const int row = row0 + lane;
-  const bool norm = col0 < 2 * e.qk_h;
+  const bool norm = col0 < 2 * e.qk_h && e.gq != nullptr;
   float rn = 1.f;
   if (norm) {
     float ss = 0.f;
@@ -247,7 +251,17 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpi& e, int M, int row0
                                : make_float4(0.f, 0.f, 0.f, 0.f);
   float4 g = make_float4(1.f, 1.f, 1.f, 1.f);
   if (mode == EPI_RESID_GATE) g = __ldg(reinterpret_cast<const float4*>(e.gate + col));
-  if (mode == EPI_EULER) {
+  if (mode == EPI_CFG_EULER) {  // a = v_c; out1 holds v_u: a <- v_u + alpha (v_c - v_u)
+    const float* vu = reinterpret_cast<const float*>(e.out1) + col;
+#pragma unroll
+    for (int it = 0; it < 8; ++it) {
+      if (rbase + it * 4 >= M) continue;
+      const float4 u = *reinterpret_cast<const float4*>(vu + (long long)(rbase + it * 4) * e.ld1);
+      a[it] = make_float4(u.x + e.alpha * (a[it].x - u.x), u.y + e.alpha * (a[it].y - u.y),
+                          u.z + e.alpha * (a[it].z - u.z), u.w + e.alpha * (a[it].w - u.w));
+    }
+  }
+  if (mode == EPI_EULER || mode == EPI_CFG_EULER) {
     const float dt = *e.scalar;
     g = make_float4(dt, dt, dt, dt);
     if (e.out1) {
@@ -568,21 +582,23 @@ static int make_tmap_2d(CUtensorMap* m, const void* base, uint64_t inner, uint64
 }
 
 static const char* check_epi(const GemmEpi& epi, int bn) {
+  if (epi.mode == EPI_CFG_EULER && (!epi.out1 || !epi.scalar)) return "gemm: CFG Euler needs v_u (out1) and dt";
   if (!epi.qk_h) return nullptr;
   if (epi.qk_D != 64 && epi.qk_D != 128) return "gemm: fused QK-norm needs D in {64, 128}";
   if (bn % epi.qk_D || epi.qk_h % epi.qk_D || (epi.qk_h / epi.qk_D) % epi.k_sp)
     return "gemm: fused QK-norm needs D | BN, D | h and k_sp | heads";
   if (epi.mode != EPI_STORE_BF16 && epi.mode != EPI_SPLIT_GELU) return "gemm: fused QK-norm needs a bf16 store";
   if (epi.mode == EPI_SPLIT_GELU && epi.n_split != 3 * epi.qk_h) return "gemm: split must be at 3h";
-  if (!epi.gq || !epi.gk || !epi.cosb || !epi.sinb || (epi.k_sp > 1 && !epi.pack))
-    return "gemm: fused QK-norm needs gains, RoPE tables (and the pack buffer)";
+  if (epi.gq && (!epi.gk || !epi.cosb || !epi.sinb)) return "gemm: fused QK-norm needs both gains and RoPE tables";
+  if (!epi.gq && epi.k_sp <= 1) return "gemm: a QKV epilogue without norm needs k_sp > 1 (else a plain store)";
+  if (epi.k_sp > 1 && !epi.pack) return "gemm: the Ulysses pack needs the pack buffer";
   return nullptr;
 }
 
 int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int K, int num_sms, const char** err,
                     int force_bn, int force_pair) {
   *err = nullptr;
-  if (nprob < 1 || nprob > 2) { *err = "gemm: 1 or 2 problems per launch"; return -1; }
+  if (nprob < 1 || nprob > GEMM_MAX_PROBLEMS) { *err = "gemm: 1 to 4 problems per launch"; return -1; }
   if (N <= 0 || K <= 0) { *err = "gemm: empty shape"; return -1; }
   if (K % BK) { *err = "gemm: K must be a multiple of 64"; return -1; }
   if (N % 64) { *err = "gemm: N must be a multiple of 64"; return -1; }
@@ -664,7 +680,7 @@ static void launch_bn(const GemmPlan& p, cudaStream_t s) {
   GemmMaps maps;
   const int bm = p.pair ? 256 : BM;
   a.N = p.N; a.K = p.K; a.num_n = p.N / BN; a.num_tiles = p.tiles; a.nprob = p.nprob;
-  for (int q = 0; q < 2; ++q) {
+  for (int q = 0; q < GEMM_MAX_PROBLEMS; ++q) {
     const int qq = q < p.nprob ? q : 0;
     a.M[q] = p.Mq[qq];
     a.num_m[q] = (p.Mq[qq] + bm - 1) / bm;

@@ -40,7 +40,10 @@ enum EpiMode : int {
   EPI_STORE_F32 = 5,    // out0 (fp32) [m,n] = acc + b
   EPI_ACCUM_F32 = 6,    // out0 (fp32) [m,n] += acc + b
   EPI_EULER = 7,        // v = acc + b; out1 (fp32, optional) [m,n] = v; out0 (fp32) [m,n] += (*scalar) * v
+  EPI_CFG_EULER = 8,    // v_c = acc + b; v = out1 + alpha (v_c - out1) (out1 holds v_u on entry);
+                        // out1 (fp32) [m,n] = v; out0 (fp32) [m,n] += (*scalar) * v   (SD3 CFG, S23)
 };
+constexpr int GEMM_MAX_PROBLEMS = 4;
 
 struct GemmEpi {
   int mode = EPI_STORE_BF16;
@@ -52,9 +55,11 @@ struct GemmEpi {
   const bf16* bias = nullptr;   // [N]
   const float* gate = nullptr;  // [N]
   const float* scalar = nullptr;
+  float alpha = 0.f;            // EPI_CFG_EULER guidance scale
   // Fused a4 (QK-RMSNorm + RoPE, Ulysses pack) for a QKV-producing GEMM (modes STORE_BF16 /
   // SPLIT_GELU): columns [0, 3*qk_h) are "(K H D)" q|k|v; q and k heads get
-  // RoPE(RMSNorm(y) * g), v passes through.  qk_h = 0 disables.
+  // RoPE(RMSNorm(y) * g), v passes through.  qk_h = 0 disables; gq = gk = null keeps the
+  // Ulysses pack but skips norm and RoPE (SD3: no QK-norm, no RoPE).
   int qk_h = 0;
   int qk_D = 0;
   const bf16* gq = nullptr;
@@ -79,9 +84,9 @@ struct GemmProblem {
 
 struct GemmPlan {
   int nprob = 1;
-  CUtensorMap tmAq[2], tmBq[2];
-  int Mq[2] = {0, 0}, tile0[2] = {0, 0};
-  GemmEpi epiq[2];
+  CUtensorMap tmAq[GEMM_MAX_PROBLEMS], tmBq[GEMM_MAX_PROBLEMS];
+  int Mq[GEMM_MAX_PROBLEMS] = {0, 0, 0, 0}, tile0[GEMM_MAX_PROBLEMS] = {0, 0, 0, 0};
+  GemmEpi epiq[GEMM_MAX_PROBLEMS];
   int M = 0, N = 0, K = 0;
   int BN = 256;
   int tiles = 0, grid = 0;
@@ -93,7 +98,8 @@ struct GemmPlan {
 // Returns 0 on success, nonzero (and sets *err) on invalid arguments.
 int gemm_plan(GemmPlan* p, const bf16* A, long long lda, const bf16* W, long long ldw, int M, int N, int K,
               const GemmEpi& epi, int num_sms, const char** err, int force_bn = 0, int force_pair = -1);
-// One launch for up to two problems sharing N and K (persistent tile loop over both).
+// One launch for up to GEMM_MAX_PROBLEMS problems sharing N and K (persistent tile loop over all;
+// each problem has its own A, W and epilogue).
 int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int K, int num_sms, const char** err,
                     int force_bn = 0, int force_pair = -1);
 void gemm_launch(const GemmPlan& p, cudaStream_t s);

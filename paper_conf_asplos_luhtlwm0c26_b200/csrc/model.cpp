@@ -2,6 +2,8 @@
 // include/tsv.h "Tensor ids").
 #include "model.h"
 
+#include <algorithm>
+
 namespace tsv {
 
 namespace {
@@ -20,7 +22,14 @@ bool build_model(const tsv_model_desc& d, Model* m, std::string* err) {
     return false;
   }
   if (d.head_dim != 64 && d.head_dim != 128) { *err = "model: head_dim must be 64 or 128"; return false; }
-  if (d.axes_dim[0] + d.axes_dim[1] + d.axes_dim[2] != d.head_dim || (d.axes_dim[0] | d.axes_dim[1] | d.axes_dim[2]) & 1) {
+  if (d.family != TSV_FAMILY_FLUX && d.family != TSV_FAMILY_SD3) { *err = "model: unknown family"; return false; }
+  const bool sd3 = d.family == TSV_FAMILY_SD3;
+  if (sd3 && (d.n_single != 0 || d.n_double < 1 || d.pe_max <= 0 || d.pe_base <= 0 || d.hidden % 4)) {
+    *err = "model: SD3 needs joint blocks only (n_single = 0, n_double >= 1) and pe_max, pe_base > 0";
+    return false;
+  }
+  if (!sd3 && (d.axes_dim[0] + d.axes_dim[1] + d.axes_dim[2] != d.head_dim ||
+               (d.axes_dim[0] | d.axes_dim[1] | d.axes_dim[2]) & 1)) {
     *err = "model: axes_dim must be even and sum to head_dim";
     return false;
   }
@@ -33,7 +42,10 @@ bool build_model(const tsv_model_desc& d, Model* m, std::string* err) {
   m->h = d.hidden; m->H = d.heads; m->D = d.head_dim; m->F = d.mlp_hidden; m->in = d.in_ch;
   m->ctx = d.ctx_dim; m->vec = d.vec_dim; m->Lt = d.text_tokens;
   const int64_t h = m->h, F = m->F, D = m->D, in = m->in;
-  m->n_mod = (12 * (int64_t)d.n_double + 3 * (int64_t)d.n_single + 2) * h;
+  m->sd3 = sd3;
+  m->B = sd3 ? 2 : 1;
+  m->n_mod = (12 * (int64_t)d.n_double + 3 * (int64_t)d.n_single + 2 - (sd3 ? 4 : 0)) * h;
+  m->mod_final_off = m->n_mod - 2 * h;
 
   std::vector<Spec> specs = {
       {0, "img_in.w", h, in, 'w', in}, {1, "img_in.b", h, 1, 'b', 0},
@@ -47,16 +59,29 @@ bool build_model(const tsv_model_desc& d, Model* m, std::string* err) {
       {16, "final.mod.w", 2 * h, h, 'w', h}, {17, "final.mod.b", 2 * h, 1, 'b', 0},
       {18, "final.lin.w", in, h, 'w', h}, {19, "final.lin.b", in, 1, 'b', 0},
   };
+  if (sd3) {  // no guidance embedder
+    specs.erase(std::remove_if(specs.begin(), specs.end(), [](const Spec& x) { return x.id >= 8 && x.id <= 11; }),
+                specs.end());
+  }
   for (int j = 0; j < d.n_double; ++j)
     for (int s = 0; s < 2; ++s) {
       const int b = double_base(j, s);
-      const std::string p = "double" + std::to_string(j) + (s ? ".txt." : ".img.");
+      const std::string p = (sd3 ? "joint" : "double") + std::to_string(j) + (s ? ".txt." : ".img.");
+      if (sd3 && s == 1 && j == d.n_double - 1) {  // context_pre_only: AdaLayerNormContinuous + QKV only
+        specs.push_back({b + 0, p + "mod.w", 2 * h, h, 'w', h});
+        specs.push_back({b + 1, p + "mod.b", 2 * h, 1, 'b', 0});
+        specs.push_back({b + 2, p + "qkv.w", 3 * h, h, 'w', h});
+        specs.push_back({b + 3, p + "qkv.b", 3 * h, 1, 'b', 0});
+        continue;
+      }
       specs.push_back({b + 0, p + "mod.w", 6 * h, h, 'w', h});
       specs.push_back({b + 1, p + "mod.b", 6 * h, 1, 'b', 0});
       specs.push_back({b + 2, p + "qkv.w", 3 * h, h, 'w', h});
       specs.push_back({b + 3, p + "qkv.b", 3 * h, 1, 'b', 0});
-      specs.push_back({b + 4, p + "q_norm.g", D, 1, 'g', 0});
-      specs.push_back({b + 5, p + "k_norm.g", D, 1, 'g', 0});
+      if (!sd3) {
+        specs.push_back({b + 4, p + "q_norm.g", D, 1, 'g', 0});
+        specs.push_back({b + 5, p + "k_norm.g", D, 1, 'g', 0});
+      }
       specs.push_back({b + 6, p + "proj.w", h, h, 'w', h});
       specs.push_back({b + 7, p + "proj.b", h, 1, 'b', 0});
       specs.push_back({b + 8, p + "fc1.w", F, h, 'w', h});

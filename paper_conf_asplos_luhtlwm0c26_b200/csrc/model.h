@@ -26,7 +26,11 @@ inline float synth_scale(double sigma) { return (float)(std::sqrt(3.0) * sigma);
 struct Model {
   tsv_model_desc d{};
   int h = 0, H = 0, D = 0, F = 0, in = 0, ctx = 0, vec = 0, Lt = 0;
-  int64_t n_mod = 0;          // modulation-table width per step: (12 n_double + 3 n_single + 2) h
+  bool sd3 = false;           // TSV_FAMILY_SD3
+  int B = 1;                  // transformer evaluations per step: 1, or 2 for SD3's CFG pair
+  int64_t n_mod = 0;          // modulation-table width per evaluation: (12 n_double + 3 n_single + 2) h
+                              // (SD3: (12 n_double - 4 + 2) h, the last txt stream has 2 chunks)
+  int64_t mod_final_off = 0;
   size_t modw_off = 0;        // concatenated modulation weights [n_mod, h]
   size_t modb_off = 0;        // concatenated modulation biases [n_mod]
   size_t total = 0;           // blob elements (bf16)
@@ -39,7 +43,7 @@ struct Model {
   // offsets (columns) into one step's modulation row
   int64_t mod_double(int j, int s) const { return (int64_t)j * 12 * h + (int64_t)s * 6 * h; }
   int64_t mod_single(int j) const { return (int64_t)d.n_double * 12 * h + (int64_t)j * 3 * h; }
-  int64_t mod_final() const { return (int64_t)d.n_double * 12 * h + (int64_t)d.n_single * 3 * h; }
+  int64_t mod_final() const { return mod_final_off; }
 };
 
 static inline int double_base(int j, int s) { return 64 + 32 * j + 16 * s; }

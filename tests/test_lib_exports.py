@@ -61,3 +61,13 @@ def test_presets_and_errors(tsv):
         tsv.shard_range(10, 0, 0)
     with pytest.raises(tsv.TsvError):
         tsv.shard_range(10, 2, 2)
+
+
+def test_sd3_presets(tsv):
+    d = tsv.model_preset("sd3")
+    assert (d.hidden, d.heads, d.head_dim, d.mlp_hidden, d.n_double, d.n_single, d.text_tokens, d.vec_dim) == \
+        (1536, 24, 64, 6144, 24, 0, 333, 2048)
+    assert d.family == 1 and d.cfg_scale == 7.0 and d.shift == 3.0 and (d.pe_max, d.pe_base) == (192, 64)
+    t = tsv.model_preset("tiny_sd3")
+    assert (t.hidden, t.heads, t.n_double, t.text_tokens, t.family) == (256, 4, 2, 77, 1)
+    assert tsv.model_preset("flux").family == 0

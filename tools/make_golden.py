@@ -3,6 +3,11 @@
 flux512_seed1000_S1.npz: FLUX.1-dev-shaped step at 512x512, request seed 1000, guidance 3.5,
 S = 1 (t_0 = 1 -> t_1 = 0), weights SYNTH-1 seed 0x7E7125E7.  Keys: v, x_next (float64).
 Runtime: several minutes on 8 cores (12 B synthetic parameters + ~21 TFLOP of fp64).
+
+sd3_512_seed1000_S20.npz: SD3-medium-shaped CFG step 0 of S = 20 at 512x512 (t_0 = 1 ->
+t_1 = shift(0.95)), request seed 1000 (inputs ids 1-5), same weight seed.  Keys: v, x_next.
+
+Usage: python tools/make_golden.py [flux|sd3 ...]   (default: both)
 """
 import os
 import sys
@@ -14,11 +19,22 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 from oracle import flux as F  # noqa: E402
-from oracle.config import FLUX  # noqa: E402
-from oracle.weights import Weights, request_inputs  # noqa: E402
+from oracle import sd3 as S3  # noqa: E402
+from oracle.config import FLUX, SD3  # noqa: E402
+from oracle.weights import Weights, request_inputs, sd3_request_inputs  # noqa: E402
 
 
-def main():
+def sd3():
+    t0 = time.time()
+    x, Tc, yc, Tu, yu = sd3_request_inputs(SD3, 512, 512, 1000)
+    W = Weights(SD3, cache_bytes=20 << 30)     # 2 B parameters: keep them for the second branch
+    v, xn = S3.request_step(SD3, W, x, Tc, yc, Tu, yu, 0, 20, 512, 512)
+    out = os.path.join(ROOT, "tests", "golden", "sd3_512_seed1000_S20.npz")
+    np.savez_compressed(out, v=v, x_next=xn)
+    print(f"wrote {out} in {time.time() - t0:.1f} s; |v|max={np.abs(v).max():.4f}")
+
+
+def flux():
     t0 = time.time()
     x, T, y = request_inputs(FLUX, 512, 512, 1000)
     W = Weights(FLUX, cache_bytes=0)
@@ -26,6 +42,12 @@ def main():
     out = os.path.join(ROOT, "tests", "golden", "flux512_seed1000_S1.npz")
     np.savez_compressed(out, v=v, x_next=xn)
     print(f"wrote {out} in {time.time() - t0:.1f} s; |v|max={np.abs(v).max():.4f}")
+
+
+def main():
+    which = sys.argv[1:] or ["flux", "sd3"]
+    for w in which:
+        {"flux": flux, "sd3": sd3}[w]()
 
 
 if __name__ == "__main__":
