@@ -129,3 +129,20 @@ def test_sd3_latency_table(tsv, sd3_engine):
     ms, cv = sd3_engine.latency_table([512, 1024], [1, 2], warmup=1, iters=3)
     assert ms.shape == (2, 2) and np.all(ms > 0)
     assert ms[1, 0] > ms[0, 0]
+
+
+def test_mixed_round_tool(tsv, tmp_path):
+    """Config 5 machinery end to end at tiny shapes: latency table -> deadlines -> DP packer rounds
+    -> disjoint-group placement with reshards -> every request completes all its steps."""
+    import json
+    import subprocess
+    import sys
+    out = tmp_path / "round.json"
+    subprocess.run([sys.executable, os.path.join(ROOT, "tools", "mixed_round.py"), "--model", "tiny_sd3",
+                    "--gpus", "4", "--res", "128", "256", "512", "--steps", "6", "--table-iters", "2",
+                    "--out", str(out)], check=True, timeout=600)
+    r = json.load(open(out))
+    assert len(r["completion"]) == 3 and all(c["finish_s"] > 0 for c in r["completion"])
+    assert sum(e["steps"] for rd in r["rounds"] for e in rd["requests"]) == 3 * 6
+    for rd in r["rounds"]:
+        assert sum(e["gpus"] for e in rd["requests"]) <= 4
