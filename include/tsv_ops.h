@@ -64,7 +64,9 @@ tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int
 /* a6: O = softmax(q k^T / sqrt(D)) v, non-causal, per head h < H; q(l, h) at q + l*ldq + h*D
  * (bf16, same for k, v, o).  D in {64, 128}.  Operands and row strides 16-byte aligned.
  * impl 0: the tcgen05/TMEM kernel the step uses; impl 1: the mma.sync (FA2-style) baseline,
- * kept only for comparison. */
+ * kept only for comparison; impl 2: the one-query-tile tcgen05 kernel (P in shared memory);
+ * impl 11..15: the step's kernel with 1..5 of every 8 exp2 pairs evaluated by polynomial on the
+ * FMA pipe instead of MUFU (tuning sweeps).  Other values: TSV_E_INVAL. */
 tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
                             void* o, int64_t ldo, int L, int H, int D, int impl, void* stream);
 

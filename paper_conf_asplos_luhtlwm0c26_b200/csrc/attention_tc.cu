@@ -351,7 +351,8 @@ struct FaCfg {
 };
 constexpr int FA_THREADS = 384;
 
-template <int D>
+// NPOLY of every 8 exp2 pairs are evaluated on the FMA/ALU pipes (poly_exp2_x2), the rest on MUFU.
+template <int D, int NPOLY>
 __global__ void __launch_bounds__(FA_THREADS, 1)
     attention_fa_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
@@ -504,7 +505,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       if (kbase + AT_BN <= L) {
         // Per tile each softmax warpgroup must finish inside the ~1024-cycle window in which the
         // tensor core works on the other query tile.  MUFU.EX2 alone needs 1024 cycles per tile
-        // (16/clk/SM), so 3 pairs in 8 are evaluated on the FMA/ALU pipes (Cody-Waite split +
+        // (16/clk/SM), so NPOLY pairs in 8 are evaluated on the FMA/ALU pipes (Cody-Waite split +
         // cubic, rel. error < 1e-3 << bf16 ulp of P), and the arithmetic uses paired FP32 ops.
         const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(neg_m, neg_m);
         float2 lsum[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f),
@@ -516,7 +517,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
             const float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2,
                                         nm2);
             float2 p;
-            if (((i >> 1) & 7) >= 5) p = poly_exp2_x2(x);
+            if (((i >> 1) & 7) >= 8 - NPOLY) p = poly_exp2_x2(x);
             else p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
             lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], p);     // 8 independent partial sums
             sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);  // packed P overwrites consumed S
@@ -613,6 +614,24 @@ static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L
   return r == CUDA_SUCCESS ? 0 : -2;
 }
 
+// default share of exp2 evaluated by polynomial, per head dim (tools/microbench.py sweep)
+template <int D>
+constexpr int default_npoly() { return 2; }   // measured best for D = 64 and 128 (profiles/README.md)
+
+template <int D, int NP>
+static void launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
+                      int L, int H, float scale_log2, cudaStream_t s) {
+  static unsigned long long done = 0;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!(done >> dev & 1ull)) {
+    cudaFuncSetAttribute(attention_fa_kernel<D, NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, FaCfg<D>::SMEM);
+    done |= 1ull << dev;
+  }
+  dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H);
+  launch_pdl(attention_fa_kernel<D, NP>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo, L, scale_log2);
+}
+
 template <int D>
 static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv, bf16* o,
                      long long ldo, int L, int H, int version, cudaStream_t s) {
@@ -625,7 +644,6 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
   cudaGetDevice(&dev);
   if (!(done >> dev & 1ull)) {
     cudaFuncSetAttribute(attention_tc_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, AttnCfg<D>::SMEM);
-    cudaFuncSetAttribute(attention_fa_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, FaCfg<D>::SMEM);
     done |= 1ull << dev;
   }
   const float scale_log2 = (1.0f / sqrtf((float)D)) * 1.4426950408889634f;
@@ -633,8 +651,16 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     dim3 grid((L + AT_BM - 1) / AT_BM, H);
     attention_tc_kernel<D><<<grid, AT_THREADS, AttnCfg<D>::SMEM, s>>>(tq, tk, tv, o, ldo, L, scale_log2);
   } else {
-    dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H);
-    launch_pdl(attention_fa_kernel<D>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo, L, scale_log2);
+    // version 3: the default poly share; 10 + n: n of 8 exp2 pairs by polynomial (tuning sweeps)
+    const int np = version >= 10 ? version - 10 : default_npoly<D>();
+    switch (np) {
+      case 1: launch_fa<D, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, s); break;
+      case 2: launch_fa<D, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, s); break;
+      case 3: launch_fa<D, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, s); break;
+      case 4: launch_fa<D, 4>(tq, tk, tv, o, ldo, L, H, scale_log2, s); break;
+      case 5: launch_fa<D, 5>(tq, tk, tv, o, ldo, L, H, scale_log2, s); break;
+      default: return -3;
+    }
   }
   return 0;
 }

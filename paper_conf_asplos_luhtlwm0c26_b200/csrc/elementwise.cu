@@ -28,15 +28,18 @@ template <int T, int NV>
 __global__ void __launch_bounds__(T) ln_mod_kernel(const float* __restrict__ x, long long ldx, bf16* __restrict__ u,
                                                    long long ldu, const float* __restrict__ shift0,
                                                    const float* __restrict__ scale0, const float* __restrict__ shift1,
-                                                   const float* __restrict__ scale1, int n_first) {
+                                                   const float* __restrict__ scale1, int n_first, int rows_b,
+                                                   long long mstride) {
   __shared__ float red[T / 32];
   const int row = blockIdx.x;
   const int t = threadIdx.x;
   grid_dep_wait();
-  // rows [0, n_first) take (shift0, scale0), the others (shift1, scale1): both streams of a
-  // double block in one launch
-  const float* shift = row < n_first ? shift0 : shift1;
-  const float* scale = row < n_first ? scale0 : scale1;
+  // rows are B blocks of rows_b (SD3's CFG pair; B = 1 for FLUX); block b's modulation vectors sit
+  // b * mstride floats further.  Inside a block rows [0, n_first) take (shift0, scale0), the others
+  // (shift1, scale1): both streams of a double block in one launch
+  const int b = row / rows_b, r = row - b * rows_b;
+  const float* shift = (r < n_first ? shift0 : shift1) + b * mstride;
+  const float* scale = (r < n_first ? scale0 : scale1) + b * mstride;
   constexpr int h = 4 * T * NV;
   const float4* xr = reinterpret_cast<const float4*>(x + (long long)row * ldx);
   float4 v[NV], shv[NV], scv[NV];
@@ -77,14 +80,16 @@ __global__ void __launch_bounds__(256) ln_mod_generic(const float* __restrict__ 
                                                       long long ldu, const float* __restrict__ shift0,
                                                       const float* __restrict__ scale0,
                                                       const float* __restrict__ shift1,
-                                                      const float* __restrict__ scale1, int n_first, int M, int h) {
+                                                      const float* __restrict__ scale1, int n_first, int M, int h,
+                                                      int rows_b, long long mstride) {
   const int row = blockIdx.x * 8 + (threadIdx.x >> 5);
   const int lane = threadIdx.x & 31;
   grid_dep_wait();
   grid_dep_launch();
   if (row >= M) return;
-  const float* shift = row < n_first ? shift0 : shift1;
-  const float* scale = row < n_first ? scale0 : scale1;
+  const int b = row / rows_b, r = row - b * rows_b;
+  const float* shift = (r < n_first ? shift0 : shift1) + b * mstride;
+  const float* scale = (r < n_first ? scale0 : scale1) + b * mstride;
   const float* xr = x + (long long)row * ldx;
   float s = 0.f;
   for (int c = lane; c < h; c += 32) s += xr[c];
@@ -98,25 +103,35 @@ __global__ void __launch_bounds__(256) ln_mod_generic(const float* __restrict__ 
     u[(long long)row * ldu + c] = __float2bfloat16_rn((xr[c] - mean) * rstd * (1.f + scale[c]) + shift[c]);
 }
 
-void ln_mod2_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift0,
-                    const float* scale0, const float* shift1, const float* scale1, int n_first, int M, int h,
-                    cudaStream_t s) {
+void ln_mod2b_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift0,
+                     const float* scale0, const float* shift1, const float* scale1, int n_first, int rows_b, int B,
+                     long long mstride, int h, cudaStream_t s) {
+  const int M = rows_b * B;
   if (M <= 0) return;
   switch (h) {
     case 3072:
-      launch_pdl(ln_mod_kernel<256, 3>, dim3(M), dim3(256), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
+      launch_pdl(ln_mod_kernel<256, 3>, dim3(M), dim3(256), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first,
+                 rows_b, mstride);
       break;
     case 1536:
-      launch_pdl(ln_mod_kernel<128, 3>, dim3(M), dim3(128), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
+      launch_pdl(ln_mod_kernel<128, 3>, dim3(M), dim3(128), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first,
+                 rows_b, mstride);
       break;
     case 256:
-      launch_pdl(ln_mod_kernel<32, 2>, dim3(M), dim3(32), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first);
+      launch_pdl(ln_mod_kernel<32, 2>, dim3(M), dim3(32), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first,
+                 rows_b, mstride);
       break;
     default:
       launch_pdl(ln_mod_generic, dim3((M + 7) / 8), dim3(256), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1,
-                 n_first, M, h);
+                 n_first, M, h, rows_b, mstride);
       break;
   }
+}
+
+void ln_mod2_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift0,
+                    const float* scale0, const float* shift1, const float* scale1, int n_first, int M, int h,
+                    cudaStream_t s) {
+  ln_mod2b_launch(x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first, M, 1, 0, h, s);
 }
 
 void ln_mod_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift, const float* scale,

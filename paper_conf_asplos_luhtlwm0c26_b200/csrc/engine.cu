@@ -890,13 +890,13 @@ static tsv_status run_step_sd3(StepEnv& E) {
       CK(cudaSetDevice(s.device));
       const int64_t R = c.rows;
       if (!R) continue;
-      // a2: LN-modulate both streams of both evaluations
-      for (int b = 0; b < B; ++b) {
-        const float* mi = c.mod + b * nm + m.mod_double(j, 0);
-        const float* mt = c.mod + b * nm + m.mod_double(j, 1);
-        ProfScope ps(e, s, KC_LNMOD, 0.0, (double)R * h * 6.0 + 16.0 * h);
-        ln_mod2_launch(c.x + b * R * h, h, c.u + b * R * h, h, last ? mt + h : mt, last ? mt : mt + h, mi, mi + h,
-                       (int)c.nt, (int)R, h, s.stream);
+      // a2: LN-modulate both streams of both evaluations in one launch
+      {
+        const float* mi = c.mod + m.mod_double(j, 0);
+        const float* mt = c.mod + m.mod_double(j, 1);
+        ProfScope ps(e, s, KC_LNMOD, 0.0, (double)B * R * h * 6.0 + 16.0 * B * h);
+        ln_mod2b_launch(c.x, h, c.u, h, last ? mt + h : mt, last ? mt : mt + h, mi, mi + h, (int)c.nt, (int)R, B, nm,
+                        h, s.stream);
       }
       // a3 (+ Ulysses pack for k > 1): 2 streams x 2 evaluations in one launch
       GemmProblem pq[GEMM_MAX_PROBLEMS];
@@ -940,16 +940,14 @@ static tsv_status run_step_sd3(StepEnv& E) {
           ++n;
         }
       TRY(gemm_multi(e, s, pp, n, h, h));  // a8: out-proj + gated residual
-      for (int b = 0; b < B; ++b) {         // a9: LN-modulate
-        const float* mi = c.mod + b * nm + m.mod_double(j, 0);
-        const float* mt = c.mod + b * nm + m.mod_double(j, 1);
-        if (last) {
-          lnmod(e, s, c.x + (b * R + c.nt) * h, c.u + (b * R + c.nt) * h, mi + 3 * h, mi + 4 * h, (int)c.ni);
-        } else {
-          ProfScope ps(e, s, KC_LNMOD, 0.0, (double)R * h * 6.0 + 16.0 * h);
-          ln_mod2_launch(c.x + b * R * h, h, c.u + b * R * h, h, mt + 3 * h, mt + 4 * h, mi + 3 * h, mi + 4 * h,
-                         (int)c.nt, (int)R, h, s.stream);
-        }
+      {                                     // a9: LN-modulate (both evaluations, one launch)
+        const float* mi = c.mod + m.mod_double(j, 0);
+        // context_pre_only: the txt rows are dead after the attention; they are normalised with
+        // the img vectors (in bounds, result unused) so both evaluations stay one launch
+        const float* mt = last ? mi : c.mod + m.mod_double(j, 1);
+        ProfScope ps(e, s, KC_LNMOD, 0.0, (double)B * R * h * 6.0 + 16.0 * B * h);
+        ln_mod2b_launch(c.x, h, c.u, h, mt + 3 * h, mt + 4 * h, mi + 3 * h, mi + 4 * h, (int)c.nt, (int)R, B, nm, h,
+                        s.stream);
       }
       TRY(gemm_multi(e, s, p1, n, F, h));  // fc1 + GELU
       TRY(gemm_multi(e, s, p2, n, h, F));  // fc2 + gated residual
@@ -962,16 +960,18 @@ static tsv_status run_step_sd3(StepEnv& E) {
     CK(cudaSetDevice(s.device));
     if (!c.ni) continue;
     const int64_t R = c.rows;
-    for (int b = 0; b < B; ++b) {
-      const float* md = c.mod + b * nm + m.mod_final();
-      lnmod(e, s, c.x + (b * R + c.nt) * h, c.u + b * R * h, md + h, md, (int)c.ni);
+    {
+      // both evaluations' img rows (txt rows normalised too, unused): u_b rows [nt, R)
+      const float* md = c.mod + m.mod_final();
+      ProfScope ps(e, s, KC_LNMOD, 0.0, (double)B * R * h * 6.0 + 16.0 * B * h);
+      ln_mod2b_launch(c.x, h, c.u, h, md + h, md, md + h, md, (int)c.nt, (int)R, B, nm, h, s.stream);
     }
     const float* dt = reinterpret_cast<const float*>(c.rd->cur.p) + B * nm;
-    TRY(gemm(e, s, c.u + R * h, h, e->W(s, 18), h, (int)c.ni, m.in, h,
+    TRY(gemm(e, s, c.u + (R + c.nt) * h, h, e->W(s, 18), h, (int)c.ni, m.in, h,
              epi_of(EPI_STORE_F32, c.sh->vel.p, m.in, e->W(s, 19))));
     GemmEpi ep = epi_of(EPI_CFG_EULER, c.sh->lat.p, m.in, e->W(s, 19), nullptr, c.sh->vel.p, m.in, 0, dt);
     ep.alpha = m.d.cfg_scale;
-    TRY(gemm(e, s, c.u, h, e->W(s, 18), h, (int)c.ni, m.in, h, ep));
+    TRY(gemm(e, s, c.u + c.nt * h, h, e->W(s, 18), h, (int)c.ni, m.in, h, ep));
   }
   for (auto& c : E.rc) CK(cudaGetLastError());
   return TSV_OK;
@@ -1829,13 +1829,14 @@ tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int
 tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
                             void* o, int64_t ldo, int L, int H, int D, int impl, void* stream) {
   if (D != 64 && D != 128) return fail(TSV_E_INVAL, "D must be 64 or 128");
+  if (impl < 0 || (impl > 2 && (impl < 11 || impl > 15))) return fail(TSV_E_INVAL, "bad attention impl %d", impl);
   if (impl == 1) {
     attention_mma_launch(reinterpret_cast<const bf16*>(q), ldq, reinterpret_cast<const bf16*>(k), ldk,
                          reinterpret_cast<const bf16*>(v), ldv, reinterpret_cast<bf16*>(o), ldo, L, H, D,
                          reinterpret_cast<cudaStream_t>(stream));
   } else if (attention_launch(reinterpret_cast<const bf16*>(q), ldq, reinterpret_cast<const bf16*>(k), ldk,
                               reinterpret_cast<const bf16*>(v), ldv, reinterpret_cast<bf16*>(o), ldo, L, H, D,
-                              reinterpret_cast<cudaStream_t>(stream), impl == 2 ? 2 : 3)) {
+                              reinterpret_cast<cudaStream_t>(stream), impl == 0 ? 3 : impl)) {
     return fail(TSV_E_INVAL, "attention: operands must be 16-byte aligned with 16-byte row strides");
   }
   CK(cudaGetLastError());

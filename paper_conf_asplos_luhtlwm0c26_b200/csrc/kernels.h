@@ -113,6 +113,12 @@ void ln_mod2_launch(const float* x, long long ldx, bf16* u, long long ldu, const
                     const float* scale0, const float* shift1, const float* scale1, int n_first, int M, int h,
                     cudaStream_t s);
 
+// B blocks of rows_b rows (block b = rows [b*rows_b, (b+1)*rows_b)); inside a block rows [0, n_first)
+// use (shift0, scale0), the rest (shift1, scale1); block b's vectors are offset by b * mstride floats.
+void ln_mod2b_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift0,
+                     const float* scale0, const float* shift1, const float* scale1, int n_first, int rows_b, int B,
+                     long long mstride, int h, cudaStream_t s);
+
 // In-place on a qkv buffer [rows, 3*H*D] (row stride ld): q,k <- RoPE(RMSNorm(.) * g).
 // Rows [0, n_first) use gains (gq0, gk0), rows [n_first, rows) use (gq1, gk1).
 // cos/sin tables: [rows, D/2] fp32.

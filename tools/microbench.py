@@ -48,15 +48,19 @@ def gemm_cases():
 
 
 def attn_cases():
-    for L, H, D in ((1536, 24, 128), (4608, 24, 128), (16896, 24, 128), (16896, 3, 128), (4608, 24, 64)):
+    sweep = os.environ.get("ATTN_SWEEP")     # "1": also time the poly-share variants (impl 12..15)
+    for L, H, D in ((1536, 24, 128), (4608, 24, 128), (16896, 24, 128), (16896, 3, 128), (1357, 24, 64),
+                    (4429, 24, 64), (16717, 24, 64)):
         qkv = torch.randn(L, 3 * H * D, device="cuda").to(torch.bfloat16)
         o = torch.empty(L, H * D, dtype=torch.bfloat16, device="cuda")
         ld = 3 * H * D
-        for impl in (0, 1):
+        impls = (0, 1) + ((11, 12, 13, 14) if sweep else ())
+        for impl in impls:
             f = lambda: tsv.op_attention(qkv, qkv[:, H * D:], qkv[:, 2 * H * D:], o, L, H, D, ldq=ld, ldk=ld,
                                          ldv=ld, impl=impl)
             ms = timeit(f, iters=5 if L > 8000 else 20)
-            print(json.dumps({"op": "attention", "impl": ["tcgen05", "mma.sync"][impl], "L": L, "H": H, "D": D,
+            name = {0: "tcgen05", 1: "mma.sync"}.get(impl, f"tcgen05-poly{impl - 10}")
+            print(json.dumps({"op": "attention", "impl": name, "L": L, "H": H, "D": D,
                               "ms": round(ms, 4), "tflops": round(4 * L * L * D * H / ms / 1e9, 1)}), flush=True)
 
 

@@ -12,7 +12,8 @@ GPUs of one box with per-step SP degrees chosen from the measured latency table 
 3. Rounds of length tau = tau_steps * T(largest res, N): each round the C++ DP packer
    (tsv_sched_round, Alg. 1) chooses (GPUs, steps) per request; requests are placed on disjoint,
    aligned GPU groups (buddy placement of power-of-two blocks) and run concurrently; the latent is
-   resharded whenever a request's group changes.
+   resharded whenever a request's group changes.  GPUs the packer leaves idle go to
+   requests it did not schedule (one GPU each; a work-conserving tool policy outside Alg. 1).
 4. Report per round: the plan, makespan, each request's in-round step latency vs the table
    (interference), GPU-busy fraction; and each request's completion time vs its deadline.
 
@@ -104,6 +105,15 @@ def main():
         live = [q for q in reqs if q["done"] < args.steps]
         sv, plan = sched.schedule_round(T, ks, [(deadline[q["res"]], args.steps - q["done"], q["row"]) for q in live],
                                         clock, tau, N)
+        plan = list(plan)
+        # work-conserving fill (tool policy, outside Alg. 1): GPUs the packer leaves idle go to
+        # requests it did not schedule this round (doomed or late), one GPU each
+        used = sum(g for g, _ in plan)
+        for j, q in enumerate(live):
+            if plan[j][0] == 0 and used < N:
+                n = max(1, min(args.steps - q["done"], int(tau // T[q["row"], 0])))
+                plan[j] = (1, n)
+                used += 1
         place = buddy_place(plan, N)
         evs = []
         for j, q in enumerate(live):
@@ -138,19 +148,19 @@ def main():
         for q, *_ in evs:
             if q["done"] >= args.steps and q["finish"] is None:
                 q["finish"] = clock
-        rounds.append(dict(survivors=sv, makespan_s=round(span, 5),
+        rounds.append(dict(survivors=int(sv), makespan_s=round(span, 5),
                            gpu_busy=round(busy / (N * span), 4) if span else None, requests=entries))
         if not evs:
             raise RuntimeError("scheduler returned an empty plan")
 
-    out = dict(model=args.model, gpus=N, devices=ndev, virtual_ranks=virtual,
+    out = dict(model=args.model, gpus=N, devices=ndev, virtual_ranks=bool(virtual),
                note=("ranks are virtual (several per device): device time is serialised, timings are not "
                      "representative of N GPUs") if virtual else "one rank per GPU",
                steps=args.steps, ks=ks, res=res, table_ms=np.round(ms, 3).tolist(), table_cv=np.round(cv, 4).tolist(),
                table_build_s=round(table_s, 1), tau_s=round(tau, 5),
                deadlines_s={str(r): round(d, 4) for r, d in deadline.items()}, rounds=rounds,
                completion=[dict(res=q["res"], finish_s=round(q["finish"], 4), deadline_s=round(deadline[q["res"]], 4),
-                                met=q["finish"] <= deadline[q["res"]] + 1e-9) for q in reqs],
+                                met=bool(q["finish"] <= deadline[q["res"]] + 1e-9)) for q in reqs],
                total_s=round(clock, 4))
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     json.dump(out, open(args.out, "w"), indent=1)
