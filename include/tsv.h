@@ -225,8 +225,22 @@ tsv_status tsv_engine_profile(tsv_engine* eng, int enable);
 /* When a group has exactly one rank in this process, each step is captured once as a CUDA graph
  * (per request, group and buffer set) and replayed for later steps; the step index is read from
  * device memory, so one graph serves every step.  enable = 0 launches kernels directly.  Default
- * on; profiling (tsv_engine_profile) always launches directly. */
+ * on; with profiling on, the profiled graph carries an event pair around every launch. */
 tsv_status tsv_engine_set_graphs(tsv_engine* eng, int enable);
+
+/* Ulysses transport of groups whose ranks all live in this process (S:§8(f) NEXT #2):
+ *   TSV_TRANSPORT_FUSED (default): the all-to-alls are fused into the producers' epilogues —
+ *     the QKV GEMM stores each head block's q|k|v straight into the owning rank's attention input
+ *     ([L][3][H/k][D], global row order) and the attention kernel stores each output row straight
+ *     into the owning rank's [txt_r; img_r] activation rows; a stream barrier (events) per exchange
+ *     point is all that is left of the collective.  Stores go to peer memory over NVLink when the
+ *     ranks are on different GPUs (peer access is enabled at engine creation).
+ *   TSV_TRANSPORT_EXCHANGE: pack buffer + explicit exchange (peer copies in-process; NCCL
+ *     send/recv across processes) + unpack — the baseline, bit-identical results.
+ * Groups spanning processes always use NCCL (exchange).  Errors: TSV_E_INVAL. */
+#define TSV_TRANSPORT_EXCHANGE 0
+#define TSV_TRANSPORT_FUSED 1
+tsv_status tsv_engine_set_transport(tsv_engine* eng, int mode);
 tsv_status tsv_engine_profile_read(tsv_engine* eng, double* ms, int64_t* launches, double* flops, double* bytes);
 /* Number of kernels this engine launched so far (all slots). */
 tsv_status tsv_engine_kernel_count(tsv_engine* eng, int64_t* count);

@@ -183,6 +183,11 @@ class Engine:
 
     PROF_CLASSES = ("gemm", "attention", "ln_mod", "qk_norm_rope", "a2a", "other")
 
+    def set_transport(self, fused: bool = True):
+        """Ulysses all-to-alls of in-process groups: fused into the epilogues (default) or the
+        pack / exchange / unpack baseline."""
+        check(lib.tsv_engine_set_transport(self.h, 1 if fused else 0))
+
     def set_graphs(self, enable: bool = True):
         check(lib.tsv_engine_set_graphs(self.h, int(enable)))
 

@@ -77,6 +77,7 @@ _SIGS = {
     "tsv_engine_kernel_count": (_i32, [_p, _P(_i64)]),
     "tsv_engine_profile": (_i32, [_p, _i32]),
     "tsv_engine_set_graphs": (_i32, [_p, _i32]),
+    "tsv_engine_set_transport": (_i32, [_p, _i32]),
     "tsv_engine_profile_read": (_i32, [_p, _P(C.c_double), _P(_i64), _P(C.c_double), _P(C.c_double)]),
     "tsv_op_gemm": (_i32, [_p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p, _i64, _p, _i64, _i32, _p, _p, _p, _i32, _i32,
                             _p]),

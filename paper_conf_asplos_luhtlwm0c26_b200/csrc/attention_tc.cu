@@ -356,7 +356,7 @@ template <int D, int NPOLY>
 __global__ void __launch_bounds__(FA_THREADS, 1)
     attention_fa_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
-                        float scale_log2) {
+                        float scale_log2, const __grid_constant__ AttnScatter sc) {
   using C = FaCfg<D>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -561,13 +561,27 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     tc_fence_after();
     const float inv = 1.f / l_sum;
     const int grow = q0 + t * AT_BM + row;
+    // output row: local (plain) or, fused a7, the owning rank's row of its stream-concatenated input
+    bf16* orow = o + (long long)grow * ldo + head * D;
+    if (sc.k > 0 && grow < L) {
+      int p = 0, lr;
+      if (grow < sc.Lt) {
+        while (p + 1 < sc.k && grow >= sc.t_off[p + 1]) ++p;
+        lr = grow - sc.t_off[p];
+      } else {
+        const int gi = grow - sc.Lt;
+        while (p + 1 < sc.k && gi >= sc.i_off[p + 1]) ++p;
+        lr = sc.nt[p] + gi - sc.i_off[p];
+      }
+      orow = sc.dst[p] + (long long)lr * sc.ld + sc.col0 + head * D;
+    }
 #pragma unroll
     for (int c = 0; c < D / 32; ++c) {
       uint32_t ov[32];
       tmem_ld32(o_col + c * 32, ov);
       tmem_ld_wait();
       if (grow < L) {
-        uint4* dst = reinterpret_cast<uint4*>(o + (long long)grow * ldo + head * D + c * 32);
+        uint4* dst = reinterpret_cast<uint4*>(orow + c * 32);
 #pragma unroll
         for (int qd = 0; qd < 4; ++qd) {
           uint4 v;
@@ -620,7 +634,7 @@ constexpr int default_npoly() { return 2; }   // measured best for D = 64 and 12
 
 template <int D, int NP>
 static void launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
-                      int L, int H, float scale_log2, cudaStream_t s) {
+                      int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s) {
   static unsigned long long done = 0;
   int dev = 0;
   cudaGetDevice(&dev);
@@ -629,12 +643,13 @@ static void launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtens
     done |= 1ull << dev;
   }
   dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H);
-  launch_pdl(attention_fa_kernel<D, NP>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo, L, scale_log2);
+  launch_pdl(attention_fa_kernel<D, NP>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo, L, scale_log2,
+             sc);
 }
 
 template <int D>
 static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv, bf16* o,
-                     long long ldo, int L, int H, int version, cudaStream_t s) {
+                     long long ldo, int L, int H, int version, const AttnScatter& sc, cudaStream_t s) {
   CUtensorMap tq, tk, tv;
   if (make_tmap_heads(&tq, q, D, H, L, ldq) || make_tmap_heads(&tk, k, D, H, L, ldk) ||
       make_tmap_heads(&tv, v, D, H, L, ldv))
@@ -654,11 +669,11 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     // version 3: the default poly share; 10 + n: n of 8 exp2 pairs by polynomial (tuning sweeps)
     const int np = version >= 10 ? version - 10 : default_npoly<D>();
     switch (np) {
-      case 1: launch_fa<D, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, s); break;
-      case 2: launch_fa<D, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, s); break;
-      case 3: launch_fa<D, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, s); break;
-      case 4: launch_fa<D, 4>(tq, tk, tv, o, ldo, L, H, scale_log2, s); break;
-      case 5: launch_fa<D, 5>(tq, tk, tv, o, ldo, L, H, scale_log2, s); break;
+      case 1: launch_fa<D, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 2: launch_fa<D, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 3: launch_fa<D, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 4: launch_fa<D, 4>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 5: launch_fa<D, 5>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
       default: return -3;
     }
   }
@@ -669,13 +684,19 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
 // version 3: two query tiles per CTA, P in TMEM (the step's kernel); version 2: one query tile,
 // P in shared memory (kept for comparison).
 int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
-                     bf16* o, long long ldo, int L, int H, int D, cudaStream_t s, int version) {
+                     bf16* o, long long ldo, int L, int H, int D, cudaStream_t s, int version,
+                     const AttnScatter* scatter) {
   if (L <= 0 || H <= 0) return 0;
+  AttnScatter sc;
+  if (scatter) {
+    sc = *scatter;
+    if (sc.k < 1 || sc.k > 8 || version == 2) return -4;
+  }
   if (((ldq | ldk | ldv) * 2) % 16 || ((reinterpret_cast<uintptr_t>(q) | reinterpret_cast<uintptr_t>(k) |
                                         reinterpret_cast<uintptr_t>(v)) & 15))
     return -1;
-  if (D == 128) return launch_tc<128>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, s);
-  if (D == 64) return launch_tc<64>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, s);
+  if (D == 128) return launch_tc<128>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, sc, s);
+  if (D == 64) return launch_tc<64>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, sc, s);
   return -1;
 }
 

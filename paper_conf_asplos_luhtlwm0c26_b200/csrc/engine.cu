@@ -220,6 +220,7 @@ struct tsv_engine {
   // per-kernel-class profiling (tsv_engine_profile)
   bool prof = false;
   bool graphs = true;  // replay each step as a CUDA graph when a group has one local rank
+  int transport = TSV_TRANSPORT_FUSED;  // in-process groups: all-to-alls as epilogue peer stores
   std::vector<ProfRec> prof_recs;
   std::map<int, std::vector<cudaEvent_t>> ev_pool;  // by device
   double prof_flops[8] = {0}, prof_bytes[8] = {0};
@@ -547,6 +548,7 @@ struct StepEnv {
   Request* R;
   Group* g;
   int step;
+  bool fused = false;     // all-to-alls fused into the QKV-GEMM / attention epilogues (peer stores)
   std::vector<RankCtx> rc;
   // global layout for the all-to-alls
   std::vector<int64_t> t_off, t_cnt, i_off, i_cnt;  // per group rank
@@ -649,10 +651,44 @@ static tsv_status a2a_exec(StepEnv& E, int which) {
   return TSV_OK;
 }
 
-static tsv_status a2a_qkv(StepEnv& E) { return a2a_exec(E, 1); }
+// In-process group barrier: every member's stream waits for every member's work so far.  With the
+// fused transport this is the whole all-to-all: the data already moved in the producers' epilogues.
+static tsv_status group_sync(StepEnv& E) {
+  Group& g = *E.g;
+  const int k = g.k;
+  ProfScope ps(E.e, *E.rc[0].s, KC_A2A, 0.0, 0.0, 0);
+  for (int r = 0; r < k; ++r) {
+    CK(cudaSetDevice(E.rc[r].s->device));
+    CK(cudaEventRecord(g.ev_a[r], E.rc[r].s->stream));
+  }
+  for (int r = 0; r < k; ++r) {
+    CK(cudaSetDevice(E.rc[r].s->device));
+    for (int d = 0; d < k; ++d)
+      if (d != r) CK(cudaStreamWaitEvent(E.rc[r].s->stream, g.ev_a[d], 0));
+  }
+  return TSV_OK;
+}
+
+static tsv_status a2a_qkv(StepEnv& E) { return E.fused ? group_sync(E) : a2a_exec(E, 1); }
+
+// Fused a5 destinations for one QKV-GEMM problem of rank c, evaluation b: kind 0 = its txt rows,
+// 1 = its img rows, 2 = its [txt_r; img_r] rows (single blocks).
+static void peer_epi(StepEnv& E, RankCtx& c, GemmEpi& epi, int b, int kind) {
+  const Model& m = E.e->model;
+  const int k = E.g->k;
+  const int64_t L = E.R->Lt + E.R->Li, w = 3 * (int64_t)m.h / k;
+  const int r = c.sh->rank_in_group;
+  for (int d = 0; d < k; ++d) epi.peer[d] = E.rc[d].recv + b * L * w;
+  const int tg = (int)E.t_off[r], ig = (int)(E.R->Lt + E.i_off[r]);
+  epi.peer_nt = 1 << 30;
+  if (kind == 0) epi.peer_row0 = tg;
+  else if (kind == 1) epi.peer_row0 = ig;
+  else { epi.peer_row0 = tg; epi.peer_nt = (int)c.nt; epi.peer_row1 = ig; }
+}
 
 // all-to-all #2 then unpack: cat[i, d*h/k + c] = orecv[d][i][c]
 static tsv_status a2a_o(StepEnv& E) {
+  if (E.fused) return group_sync(E);   // the attention epilogues stored into every owner's cat
   tsv_engine* e = E.e;
   const Model& m = e->model;
   const int k = E.g->k;
@@ -686,6 +722,25 @@ static tsv_status attention_all(StepEnv& E) {
         const bf16* q = c.qkv + b * c.rows * 3 * m.h;
         rc = attention_launch(q, 3 * m.h, q + m.h, 3 * m.h, q + 2 * m.h, 3 * m.h, c.cat + b * c.rows * (m.h + m.F),
                               m.h + m.F, (int)c.rows, m.H, m.D, c.s->stream);
+      } else if (E.fused) {
+        // fused a7: each output row goes straight to its owner's cat[:, r*h/k + ...]
+        const int64_t w = 3 * (int64_t)m.h / k;
+        const bf16* q = c.recv + b * L * w;
+        AttnScatter sc;
+        sc.k = k;
+        sc.Lt = (int)E.R->Lt;
+        sc.col0 = c.sh->rank_in_group * (m.h / k);
+        sc.ld = m.h + m.F;
+        for (int p = 0; p < k; ++p) {
+          sc.dst[p] = E.rc[p].cat + b * E.rc[p].rows * (m.h + m.F);
+          sc.t_off[p] = (int)E.t_off[p];
+          sc.i_off[p] = (int)E.i_off[p];
+          sc.nt[p] = (int)E.rc[p].nt;
+        }
+        sc.t_off[k] = (int)E.R->Lt;
+        sc.i_off[k] = (int)E.R->Li;
+        rc = attention_launch(q, w, q + m.h / k, w, q + 2 * m.h / k, w, nullptr, 0, (int)L, m.H / k, m.D, c.s->stream,
+                              3, &sc);
       } else {
         const int64_t w = 3 * (int64_t)m.h / k;
         const bf16* q = c.recv + b * L * w;
@@ -700,7 +755,7 @@ static tsv_status attention_all(StepEnv& E) {
 
 // a4 fused into the QKV GEMM epilogue: QK-RMSNorm + RoPE on rows [r0, r0 + n) of this rank, written
 // in place (k = 1) or straight into the Ulysses send buffer (k > 1).
-static GemmEpi qk_fused(StepEnv& E, RankCtx& c, GemmEpi epi, int64_t r0, const bf16* gq, const bf16* gk) {
+static GemmEpi qk_fused(StepEnv& E, RankCtx& c, GemmEpi epi, int64_t r0, const bf16* gq, const bf16* gk, int kind) {
   const Model& m = E.e->model;
   epi.qk_h = m.h;
   epi.qk_D = m.D;
@@ -712,6 +767,7 @@ static GemmEpi qk_fused(StepEnv& E, RankCtx& c, GemmEpi epi, int64_t r0, const b
   epi.pack = E.g->k > 1 ? c.pack : nullptr;
   epi.pack_rows = (int)c.rows;
   epi.pack_row0 = (int)r0;
+  if (E.fused) peer_epi(E, c, epi, 0, kind);
   return epi;
 }
 
@@ -775,7 +831,7 @@ static tsv_status run_step(StepEnv& E) {
         const int64_t r0 = st == 0 ? c.nt : 0, n = st == 0 ? c.ni : c.nt;
         pq[st] = {c.u + r0 * h, h, e->W(s, base + 2), h, (int)n,
                   qk_fused(E, c, epi_of(EPI_STORE_BF16, c.qkv + r0 * 3 * h, 3 * h, e->W(s, base + 3)), r0,
-                           e->W(s, base + 4), e->W(s, base + 5))};
+                           e->W(s, base + 4), e->W(s, base + 5), st == 0 ? 1 : 0)};
       }
       TRY(gemm_multi(e, s, pq, 2, 3 * h, h));   // a3 + a4 for both streams in one launch
     }
@@ -815,7 +871,7 @@ static tsv_status run_step(StepEnv& E) {
       lnmod(e, s, c.x, c.u, md, md + h, (int)c.rows);
       TRY(gemm(e, s, c.u, h, e->W(s, base + 2), h, (int)c.rows, 3 * h + F, h,
                qk_fused(E, c, epi_of(EPI_SPLIT_GELU, c.qkv, 3 * h, e->W(s, base + 3), nullptr, c.cat + h, ldc, 3 * h),
-                        0, e->W(s, base + 4), e->W(s, base + 5))));
+                        0, e->W(s, base + 4), e->W(s, base + 5), 2)));
     }
     if (E.g->k > 1) TRY(a2a_qkv(E));
     TRY(attention_all(E));
@@ -909,6 +965,7 @@ static tsv_status run_step_sd3(StepEnv& E) {
           if (k > 1) {
             ep.qk_h = h; ep.qk_D = m.D; ep.k_sp = k;
             ep.pack = c.pack + b * R * 3 * h; ep.pack_rows = (int)R; ep.pack_row0 = (int)r0;
+            if (E.fused) peer_epi(E, c, ep, b, st == 0 ? 1 : 0);
           }
           pq[n++] = {c.u + (b * R + r0) * h, h, e->W(s, base + 2), h, (int)nr, ep};
         }
@@ -1097,6 +1154,7 @@ static tsv_status do_step(tsv_engine* e, Request& R, int step, int gi, tsv_event
   const Model& m = e->model;
   StepEnv E;
   E.e = e; E.R = &R; E.g = &g; E.step = step;
+  E.fused = e->transport == TSV_TRANSPORT_FUSED && g.all_local && g.k > 1;
   const int k = g.k;
   E.t_off.resize(k); E.t_cnt.resize(k); E.i_off.resize(k); E.i_cnt.resize(k);
   for (int r = 0; r < k; ++r) {
@@ -1712,6 +1770,13 @@ tsv_status tsv_debug_read_weight(tsv_engine* e, int id, uint16_t* host, size_t n
   Slot& s = e->slots[0];
   CK(cudaSetDevice(s.device));
   CK(cudaMemcpy(host, reinterpret_cast<const bf16*>(s.ds->weights.p) + t->offset, n * 2, cudaMemcpyDeviceToHost));
+  return TSV_OK;
+}
+
+tsv_status tsv_engine_set_transport(tsv_engine* e, int mode) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  if (mode != TSV_TRANSPORT_EXCHANGE && mode != TSV_TRANSPORT_FUSED) return fail(TSV_E_INVAL, "bad transport %d", mode);
+  e->transport = mode;
   return TSV_OK;
 }
 

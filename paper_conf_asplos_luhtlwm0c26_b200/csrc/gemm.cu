@@ -97,6 +97,10 @@ __device__ __forceinline__ bf16* qkv_dst(const GemmEpi& e, int row, int n) {
   const int part = n / h, hd = (n - part * h) / D, d = n % D;
   const int hk = h / D / e.k_sp;
   const int dst = hd / hk, hl = hd - dst * hk;
+  if (e.peer[0]) {
+    const long long g = row < e.peer_nt ? (long long)e.peer_row0 + row : (long long)e.peer_row1 + (row - e.peer_nt);
+    return e.peer[dst] + ((g * 3 + part) * hk + hl) * D + d;
+  }
   return e.pack + ((((long long)dst * e.pack_rows + e.pack_row0 + row) * 3 + part) * hk + hl) * D + d;
 }
 
@@ -591,7 +595,12 @@ static const char* check_epi(const GemmEpi& epi, int bn) {
   if (epi.mode == EPI_SPLIT_GELU && epi.n_split != 3 * epi.qk_h) return "gemm: split must be at 3h";
   if (epi.gq && (!epi.gk || !epi.cosb || !epi.sinb)) return "gemm: fused QK-norm needs both gains and RoPE tables";
   if (!epi.gq && epi.k_sp <= 1) return "gemm: a QKV epilogue without norm needs k_sp > 1 (else a plain store)";
-  if (epi.k_sp > 1 && !epi.pack) return "gemm: the Ulysses pack needs the pack buffer";
+  if (epi.k_sp > 1 && !epi.pack && !epi.peer[0]) return "gemm: the Ulysses pack needs the pack buffer or peer buffers";
+  if (epi.peer[0]) {
+    if (epi.k_sp > 8) return "gemm: at most 8 peers";
+    for (int d = 0; d < epi.k_sp; ++d)
+      if (!epi.peer[d]) return "gemm: missing peer buffer";
+  }
   return nullptr;
 }
 

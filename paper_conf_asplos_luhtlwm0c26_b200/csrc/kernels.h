@@ -71,6 +71,27 @@ struct GemmEpi {
   bf16* pack = nullptr;
   int pack_rows = 0;
   int pack_row0 = 0;
+  // Fused a5 (k_sp > 1 and peer[0] != null): the q|k|v columns of head block dst go straight into
+  // rank dst's attention input peer[dst] = [L][3][H/k_sp][D] at the row's global position (the
+  // all-to-all #1 becomes the epilogue's stores: local, or peer memory over NVLink).  A problem
+  // covers at most two contiguous global ranges (a single block's [txt_r; img_r] rows).
+  bf16* peer[8] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+  int peer_row0 = 0;   // GEMM rows [0, peer_nt) -> global rows peer_row0 + m
+  int peer_nt = 1 << 30;
+  int peer_row1 = 0;   // GEMM rows [peer_nt, M) -> global rows peer_row1 + m - peer_nt
+};
+
+// Fused a7 for the attention epilogue: output row g (global order [txt_0..txt_{k-1};
+// img_0..img_{k-1}], Lt text rows) of local head hl goes to the rank p owning g, at its local row
+// (txt: g - t_off[p]; img: nt[p] + g - Lt - i_off[p]) and column col0 + hl*D of dst[p] (row stride
+// ld).  k = 0: plain output o[g*ldo + hl*D].
+struct AttnScatter {
+  int k = 0;
+  int Lt = 0;
+  int col0 = 0;
+  long long ld = 0;
+  bf16* dst[8];
+  int t_off[9], i_off[9], nt[8];
 };
 
 struct GemmProblem {
@@ -133,7 +154,8 @@ void qk_norm_rope_launch(bf16* qkv, long long ld, int rows, int n_first, int H, 
 // attention_mma_launch: the mma.sync (FA2-style) baseline kept for comparison.
 // q(l, h) at q + l*ldq + h*D (same for k, v, o). L rows.
 int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
-                     bf16* o, long long ldo, int L, int H, int D, cudaStream_t s, int version = 3);
+                     bf16* o, long long ldo, int L, int H, int D, cudaStream_t s, int version = 3,
+                     const AttnScatter* scatter = nullptr);
 void attention_mma_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
                           bf16* o, long long ldo, int L, int H, int D, cudaStream_t s);
 

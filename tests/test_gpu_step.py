@@ -196,3 +196,22 @@ def test_flux_512_step_vs_golden(tsv):
         rel, cos = _metrics(got, ref)
         assert rel <= TOL_REL and cos >= TOL_COS, (rel, cos)
     eng.close()
+
+
+@pytest.mark.parametrize("model,res", [("tiny2", (208, 240)), ("tiny_sd3", (208, 240))])
+@pytest.mark.parametrize("k", [2, 4])
+def test_fused_transport_bitwise_equals_exchange(tsv, model, res, k):
+    """NEXT #2: the all-to-alls fused into the QKV-GEMM / attention epilogues (peer stores) give
+    bit-identical results to the pack / exchange / unpack baseline (same arithmetic, different
+    destinations)."""
+    out = []
+    for fused in (True, False):
+        eng = tsv.Engine(model, devices=[0] * 4)
+        eng.set_transport(fused)
+        g = eng.group_create(list(range(k))[::-1])
+        req = eng.request_create(*res, num_steps=3, seed=1010)
+        for s in range(2):
+            eng.request_step(req, s, g)
+        out.append((eng.read_latent(req), eng.read_velocity(req)))
+        eng.close()
+    assert np.array_equal(out[0][0], out[1][0]) and np.array_equal(out[0][1], out[1][1])
