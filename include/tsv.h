@@ -167,6 +167,16 @@ tsv_status tsv_request_set_inputs(tsv_engine* eng, tsv_request req, const float*
  * TSV_E_STATE, TSV_E_CUDA, TSV_E_NCCL. */
 tsv_status tsv_request_step(tsv_engine* eng, tsv_request req, int step, tsv_group group, tsv_event* done);
 
+/* Selective batching (S:§8(f) NEXT #3): run the NEXT step of each of the n requests
+ * (each at its own step index, schedule and inputs) as ONE batched step on `group` — every GEMM,
+ * LN and all-to-all launch covers all of them (per-request modulation, latents and Euler), attention
+ * runs per request.  The requests must share the resolution; they are moved (resharded) onto the
+ * group first if needed.  n <= 8 for FLUX, <= 4 for SD3 (whose requests are CFG pairs).  Results
+ * equal n separate tsv_request_step calls (same arithmetic per row).  Errors: TSV_E_INVAL (unknown
+ * or repeated request, mixed resolutions, n out of range), TSV_E_STATE (a request has no step left),
+ * TSV_E_CUDA, TSV_E_NCCL. */
+tsv_status tsv_request_step_batch(tsv_engine* eng, const tsv_request* reqs, int n, tsv_group group, tsv_event* done);
+
 /* Move the latent of `req` to `group` without running a step: bit-exact row moves given by the
  * reshard map (tsv_reshard_plan).  Asynchronous, ordered after the request's last step. */
 tsv_status tsv_request_reshard(tsv_engine* eng, tsv_request req, tsv_group group, tsv_event* done);

@@ -119,6 +119,13 @@ class Engine:
         check(lib.tsv_request_step(self.h, req, step, group, C.byref(ev)))
         return ev.value
 
+    def request_step_batch(self, reqs, group: int) -> int:
+        """The next step of every request in `reqs` (same resolution) as one batched step."""
+        arr = (C.c_int64 * len(reqs))(*reqs)
+        ev = C.c_int64(-1)
+        check(lib.tsv_request_step_batch(self.h, arr, len(reqs), group, C.byref(ev)))
+        return ev.value
+
     def request_reshard(self, req: int, group: int) -> int:
         ev = C.c_int64(-1)
         check(lib.tsv_request_reshard(self.h, req, group, C.byref(ev)))

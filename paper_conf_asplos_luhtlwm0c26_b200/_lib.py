@@ -59,6 +59,7 @@ _SIGS = {
     "tsv_request_create": (_i32, [_p, _i32, _i32, _i32, _u64, _f32, _P(_i64)]),
     "tsv_request_set_inputs": (_i32, [_p, _i64, _P(_f32), _P(C.c_uint16), _P(C.c_uint16)]),
     "tsv_request_step": (_i32, [_p, _i64, _i32, C.c_int32, _P(_i64)]),
+    "tsv_request_step_batch": (_i32, [_p, _P(_i64), _i32, C.c_int32, _P(_i64)]),
     "tsv_request_reshard": (_i32, [_p, _i64, C.c_int32, _P(_i64)]),
     "tsv_event_wait": (_i32, [_p, _i64]),
     "tsv_event_query": (_i32, [_p, _i64, _P(_i32)]),

@@ -125,6 +125,23 @@ struct DeviceState {
 
 struct Workspace {
   DevBuf x, u, qkv, cat, hbuf, latb, pack, recv, obuf, orecv;
+  DevBuf bmod;  // fp32 [B][n_mod] this step's modulation rows of every evaluation, then B dt values
+};
+
+// A captured step graph (per slot; keyed by every buffer pointer, group, batch and profiling flag)
+struct ProfRec {
+  int cls;
+  int device;
+  cudaEvent_t a, b;
+};
+struct StepGraph {
+  cudaGraphExec_t exec = nullptr;
+  int64_t kernels = 0;
+  std::vector<int64_t> reqs;          // requests whose buffers the graph references
+  std::vector<ProfRec> prof;          // profiled graphs: the event pairs recorded at every replay
+  double flops[8] = {0}, bytes[8] = {0};
+  int64_t launch[8] = {0};
+  uint64_t last_use = 0;
 };
 
 struct Slot {
@@ -134,30 +151,15 @@ struct Slot {
   cudaStream_t stream = nullptr;
   Workspace ws;
   DevBuf scratch;  // conditioning temporaries
+  std::map<uint64_t, StepGraph> graphs;
 };
 
 // per (request, slot): state that depends only on the request
-// one profiled launch: CUDA events around it on its stream (recorded again on every graph replay)
-struct ProfRec {
-  int cls;
-  int device;
-  cudaEvent_t a, b;
-};
-
 struct ReqDev {
-  DevBuf mod;       // fp32 [S, n_mod]
+  DevBuf mod;       // fp32 [S * B_model, n_mod]
   DevBuf dt;        // fp32 [S]
-  DevBuf cur;       // fp32 [n_mod + 1]: this step's modulation row and dt (selected on device)
   DevBuf step;      // int: the step index the next launch runs
   bool ready = false;
-  // CUDA graph of the whole step for this (request, slot, group, buffers); replayed every step
-  cudaGraphExec_t gexec = nullptr;
-  uint64_t gkey = 0;
-  int64_t gkernels = 0;
-  // profiled graphs: the event pairs captured in the graph and the per-class algorithmic counters
-  std::vector<ProfRec> gprof;
-  double gflops[8] = {0}, gbytes[8] = {0};
-  int64_t glaunch[8] = {0};
 };
 // per (request, slot, shard): state that depends on the group position
 struct ReqShard {
@@ -181,6 +183,7 @@ struct Group {
 };
 
 struct Request {
+  int64_t id = 0;
   int height = 0, width = 0, S = 0;
   uint64_t seed = 0;
   float guidance = 3.5f;
@@ -221,6 +224,7 @@ struct tsv_engine {
   bool prof = false;
   bool graphs = true;  // replay each step as a CUDA graph when a group has one local rank
   int transport = TSV_TRANSPORT_FUSED;  // in-process groups: all-to-alls as epilogue peer stores
+  uint64_t graph_clock = 0;
   std::vector<ProfRec> prof_recs;
   std::map<int, std::vector<cudaEvent_t>> ev_pool;  // by device
   double prof_flops[8] = {0}, prof_bytes[8] = {0};
@@ -313,15 +317,7 @@ static tsv_status gemm_multi(tsv_engine* e, Slot& s, const GemmProblem* probs, i
   gemm_launch(p, s.stream);
   return TSV_OK;
 }
-static void lnmod(tsv_engine* e, Slot& s, const float* x, bf16* u, const float* shift, const float* scale, int n) {
-  const int h = e->model.h;
-  ProfScope ps(e, s, KC_LNMOD, 0.0, (double)n * h * 6.0 + 8.0 * h);
-  ln_mod_launch(x, h, u, h, shift, scale, n, h, s.stream);
-}
 
-struct StepEnv;
-struct RankCtx;
-static void lnmod2(StepEnv& E, RankCtx& c, int64_t mod_txt, int64_t mod_img, int chunk);
 
 static GemmEpi epi_of(int mode, void* out0, long long ld0, const bf16* bias, const float* gate = nullptr,
                       void* out1 = nullptr, long long ld1 = 0, int n_split = 0, const float* scalar = nullptr) {
@@ -357,7 +353,6 @@ static tsv_status ensure_reqdev(tsv_engine* e, Request& R, int si) {
   CK(cudaSetDevice(s.device));
   TRY(dev_alloc(rd.mod, s.device, (size_t)S * B * m.n_mod * 4));
   TRY(dev_alloc(rd.dt, s.device, (size_t)S * 4));
-  TRY(dev_alloc(rd.cur, s.device, ((size_t)B * m.n_mod + 4) * 4));
   TRY(dev_alloc(rd.step, s.device, 16));
   // host-side: sinusoidal embeddings e(t_s), e(g) (fp64 -> bf16), y (bf16), dt.  Row i*B + b is
   // step i of CFG branch b (SD3: b = 0 conditional, 1 unconditional).
@@ -510,22 +505,24 @@ static tsv_status setup_shard(tsv_engine* e, Request& R, int si, int rank_in_gro
   return TSV_OK;
 }
 
-static tsv_status ensure_workspace(tsv_engine* e, Slot& s, int64_t rows, int64_t L, int k) {
+// B = evaluations per step (requests in the batch x CFG branches)
+static tsv_status ensure_workspace(tsv_engine* e, Slot& s, int64_t rows, int64_t L, int k, int B) {
   const Model& m = e->model;
   const int64_t h = m.h, F = m.F;
   Workspace& w = s.ws;
   const int64_t r1 = std::max<int64_t>(rows, 1);
-  const int64_t r = r1 * m.B;  // every activation buffer holds the B evaluations back to back
+  const int64_t r = r1 * B;  // every activation buffer holds the B evaluations back to back
   TRY(dev_alloc(w.x, s.device, r * h * 4));
   TRY(dev_alloc(w.u, s.device, r * h * 2));
   TRY(dev_alloc(w.qkv, s.device, r * 3 * h * 2));
   TRY(dev_alloc(w.cat, s.device, r * (h + F) * 2));
   TRY(dev_alloc(w.hbuf, s.device, r * F * 2));
-  TRY(dev_alloc(w.latb, s.device, r1 * m.in * 2));
+  TRY(dev_alloc(w.latb, s.device, r * m.in * 2));
+  TRY(dev_alloc(w.bmod, s.device, ((size_t)B * m.n_mod + 64) * 4));
   if (k > 1) {
     TRY(dev_alloc(w.pack, s.device, r * 3 * h * 2));
-    TRY(dev_alloc(w.recv, s.device, m.B * L * 3 * (h / k) * 2));
-    TRY(dev_alloc(w.obuf, s.device, m.B * L * (h / k) * 2));
+    TRY(dev_alloc(w.recv, s.device, B * L * 3 * (h / k) * 2));
+    TRY(dev_alloc(w.obuf, s.device, B * L * (h / k) * 2));
     TRY(dev_alloc(w.orecv, s.device, r * h * 2));
   }
   return TSV_OK;
@@ -535,19 +532,22 @@ static tsv_status ensure_workspace(tsv_engine* e, Slot& s, int64_t rows, int64_t
 struct RankCtx {
   int si;                 // slot index
   Slot* s;
-  ReqShard* sh;
-  ReqDev* rd;
-  int64_t nt, ni, rows;   // local rows: [txt (nt) ; img (ni)]
+  ReqShard* sh;           // request 0's shard (the batch shares resolution and group: same rows)
+  std::vector<ReqShard*> shq;  // per request of the batch
+  std::vector<ReqDev*> rdq;
+  int64_t nt, ni, rows;   // local rows per evaluation: [txt (nt) ; img (ni)]
   float* x;
   bf16 *u, *qkv, *cat, *hbuf, *latb, *pack, *recv, *obuf, *orecv;
-  const float* mod;       // this step's modulation row
+  float* mod;             // this step's modulation rows: evaluation b at mod + b * n_mod; dt of
+                          // request q at mod + B * n_mod + q
 };
 
 struct StepEnv {
   tsv_engine* e;
-  Request* R;
+  Request* R;             // request 0 of the batch (shared L_t, L_i)
+  std::vector<Request*> Rq;
+  int B = 1;              // evaluations: requests x CFG branches; evaluation b = q * B_model + branch
   Group* g;
-  int step;
   bool fused = false;     // all-to-alls fused into the QKV-GEMM / attention epilogues (peer stores)
   std::vector<RankCtx> rc;
   // global layout for the all-to-alls
@@ -598,7 +598,7 @@ static tsv_status a2a_exec(StepEnv& E, int which) {
   const int64_t L = E.R->Lt + E.R->Li;
   // B evaluations (SD3's CFG pair) exchange back to back: the [k][rows_r] buffer of branch b
   // starts at b * k * rows_r * w, the [L] buffer at b * L * w.
-  const int B = m.B;
+  const int B = E.B;
   auto sendbuf = [&](RankCtx& c, int b) {
     return which == 1 ? c.pack + b * k * c.rows * w : c.obuf + b * L * w;
   };
@@ -696,7 +696,7 @@ static tsv_status a2a_o(StepEnv& E) {
   TRY(a2a_exec(E, 2));
   for (auto& c : E.rc) {
     CK(cudaSetDevice(c.s->device));
-    for (int b = 0; b < m.B; ++b)
+    for (int b = 0; b < E.B; ++b)
       for (int d = 0; d < k; ++d) {
         ProfScope ps(e, *c.s, KC_OTHER, 0.0, 4.0 * c.rows * w);
         copy2d_bf16_launch(c.orecv + ((int64_t)b * k + d) * c.rows * w, w, c.cat + b * c.rows * (m.h + m.F) + d * w,
@@ -715,7 +715,7 @@ static tsv_status attention_all(StepEnv& E) {
   for (auto& c : E.rc) {
     CK(cudaSetDevice(c.s->device));
     const double Lq = k == 1 ? (double)c.rows : (double)L;
-    for (int b = 0; b < m.B; ++b) {  // one launch per evaluation (SD3: CFG branch)
+    for (int b = 0; b < E.B; ++b) {  // one launch per evaluation (request x CFG branch)
       ProfScope ps(e, *c.s, KC_ATTN, 4.0 * Lq * Lq * m.D * (m.H / k), 8.0 * Lq * m.D * (m.H / k));
       int rc;
       if (k == 1) {
@@ -755,7 +755,8 @@ static tsv_status attention_all(StepEnv& E) {
 
 // a4 fused into the QKV GEMM epilogue: QK-RMSNorm + RoPE on rows [r0, r0 + n) of this rank, written
 // in place (k = 1) or straight into the Ulysses send buffer (k > 1).
-static GemmEpi qk_fused(StepEnv& E, RankCtx& c, GemmEpi epi, int64_t r0, const bf16* gq, const bf16* gk, int kind) {
+static GemmEpi qk_fused(StepEnv& E, RankCtx& c, GemmEpi epi, int64_t r0, const bf16* gq, const bf16* gk, int kind,
+                        int b) {
   const Model& m = E.e->model;
   epi.qk_h = m.h;
   epi.qk_D = m.D;
@@ -764,76 +765,86 @@ static GemmEpi qk_fused(StepEnv& E, RankCtx& c, GemmEpi epi, int64_t r0, const b
   epi.cosb = reinterpret_cast<const float*>(c.sh->cosb.p) + r0 * (m.D / 2);
   epi.sinb = reinterpret_cast<const float*>(c.sh->sinb.p) + r0 * (m.D / 2);
   epi.k_sp = E.g->k;
-  epi.pack = E.g->k > 1 ? c.pack : nullptr;
+  epi.pack = E.g->k > 1 ? c.pack + b * c.rows * 3 * m.h : nullptr;
   epi.pack_rows = (int)c.rows;
   epi.pack_row0 = (int)r0;
-  if (E.fused) peer_epi(E, c, epi, 0, kind);
+  if (E.fused) peer_epi(E, c, epi, b, kind);
   return epi;
 }
 
-// a2 / a9 of a double block for both streams in one launch: rows [0, nt) use the txt stream's
-// (shift, scale) = modulation chunks (chunk, chunk + 1), rows [nt, rows) the img stream's.
-static void lnmod2(StepEnv& E, RankCtx& c, int64_t mod_txt, int64_t mod_img, int chunk) {
-  tsv_engine* e = E.e;
-  const int h = e->model.h;
-  if (!c.rows) return;
-  const float* mt = c.mod + mod_txt + (int64_t)chunk * h;
-  const float* mi = c.mod + mod_img + (int64_t)chunk * h;
-  ProfScope ps(e, *c.s, KC_LNMOD, 0.0, (double)c.rows * h * 6.0 + 16.0 * h);
-  ln_mod2_launch(c.x, h, c.u, h, mt, mt + h, mi, mi + h, (int)c.nt, (int)c.rows, h, c.s->stream);
-}
 
 static tsv_status run_step_sd3(StepEnv& E);
+
+// this step's modulation rows and dt of every request of the batch, selected on the device from
+// each request's step index (so one captured graph serves every step)
+static void select_rows(StepEnv& E, RankCtx& c) {
+  tsv_engine* e = E.e;
+  const Model& m = e->model;
+  Slot& s = *c.s;
+  const int64_t nm = m.B * m.n_mod;
+  for (size_t q = 0; q < E.Rq.size(); ++q) {
+    ProfScope ps(e, s, KC_OTHER, 0.0, 8.0 * nm, 2);
+    const int* step_dev = reinterpret_cast<const int*>(c.rdq[q]->step.p);
+    select_row_launch(reinterpret_cast<const float*>(c.rdq[q]->mod.p), nm, step_dev, c.mod + q * nm, nm, s.stream);
+    select_row_launch(reinterpret_cast<const float*>(c.rdq[q]->dt.p), 1, step_dev, c.mod + E.B * m.n_mod + q, 1,
+                      s.stream);
+  }
+}
 
 static tsv_status run_step(StepEnv& E) {
   tsv_engine* e = E.e;
   const Model& m = e->model;
-  const int h = m.h, F = m.F;
-  const int64_t ldc = h + F;
-  // this step's modulation row and dt, selected on the device from the step index (so one
-  // captured graph serves every step of the request)
+  const int h = m.h, F = m.F, B = E.B;
+  const int64_t ldc = h + F, nm = m.n_mod;
   for (auto& c : E.rc) {
-    Slot& s = *c.s;
-    CK(cudaSetDevice(s.device));
-    const int64_t nm = m.B * m.n_mod;
-    ProfScope ps(e, s, KC_OTHER, 0.0, 8.0 * nm, 2);
-    const int* step_dev = reinterpret_cast<const int*>(c.rd->step.p);
-    float* cur = reinterpret_cast<float*>(c.rd->cur.p);
-    select_row_launch(reinterpret_cast<const float*>(c.rd->mod.p), nm, step_dev, cur, nm, s.stream);
-    select_row_launch(reinterpret_cast<const float*>(c.rd->dt.p), 1, step_dev, cur + nm, 1, s.stream);
+    CK(cudaSetDevice(c.s->device));
+    select_rows(E, c);
   }
   if (m.sd3) return run_step_sd3(E);
+  // FLUX: evaluation b = request b of the batch; its rows are [b*R, (b+1)*R) of every buffer.
   // a1: embeddings
   for (auto& c : E.rc) {
     Slot& s = *c.s;
     CK(cudaSetDevice(s.device));
-    if (c.ni) {
-      {
+    const int64_t R = c.rows;
+    GemmProblem pi[GEMM_MAX_PROBLEMS], pt[GEMM_MAX_PROBLEMS];
+    for (int b = 0; b < B; ++b) {
+      if (c.ni) {
         ProfScope ps(e, s, KC_OTHER, 0.0, 6.0 * c.ni * m.in);
-        f32_to_bf16_launch(reinterpret_cast<float*>(c.sh->lat.p), m.in, c.latb, m.in, (int)c.ni, m.in, s.stream);
+        f32_to_bf16_launch(reinterpret_cast<float*>(c.shq[b]->lat.p), m.in, c.latb + b * c.ni * m.in, m.in, (int)c.ni,
+                           m.in, s.stream);
       }
-      TRY(gemm(e, s, c.latb, m.in, e->W(s, 0), m.in, (int)c.ni, h, m.in,
-               epi_of(EPI_STORE_F32, c.x + c.nt * h, h, e->W(s, 1))));
+      pi[b] = {c.latb + b * c.ni * m.in, m.in, e->W(s, 0), m.in, (int)c.ni,
+               epi_of(EPI_STORE_F32, c.x + (b * R + c.nt) * h, h, e->W(s, 1))};
+      pt[b] = {reinterpret_cast<bf16*>(c.shq[b]->T.p), m.ctx, e->W(s, 2), m.ctx, (int)c.nt,
+               epi_of(EPI_STORE_F32, c.x + b * R * h, h, e->W(s, 3))};
     }
-    if (c.nt)
-      TRY(gemm(e, s, reinterpret_cast<bf16*>(c.sh->T.p), m.ctx, e->W(s, 2), m.ctx, (int)c.nt, h, m.ctx,
-               epi_of(EPI_STORE_F32, c.x, h, e->W(s, 3))));
+    TRY(gemm_multi(e, s, pi, B, h, m.in));
+    TRY(gemm_multi(e, s, pt, B, h, m.ctx));
   }
   // double-stream blocks
   for (int j = 0; j < m.d.n_double; ++j) {
     for (auto& c : E.rc) {
       Slot& s = *c.s;
       CK(cudaSetDevice(s.device));
-      GemmProblem pq[2];
-      lnmod2(E, c, m.mod_double(j, 1), m.mod_double(j, 0), 0);   // a2 for both streams: rows [txt; img]
-      for (int st = 0; st < 2; ++st) {  // 0 = img, 1 = txt
-        const int base = double_base(j, st);
-        const int64_t r0 = st == 0 ? c.nt : 0, n = st == 0 ? c.ni : c.nt;
-        pq[st] = {c.u + r0 * h, h, e->W(s, base + 2), h, (int)n,
-                  qk_fused(E, c, epi_of(EPI_STORE_BF16, c.qkv + r0 * 3 * h, 3 * h, e->W(s, base + 3)), r0,
-                           e->W(s, base + 4), e->W(s, base + 5), st == 0 ? 1 : 0)};
+      const int64_t R = c.rows;
+      {  // a2 for both streams of every evaluation: rows [txt; img] per evaluation
+        const float* mt = c.mod + m.mod_double(j, 1);
+        const float* mi = c.mod + m.mod_double(j, 0);
+        ProfScope ps(e, s, KC_LNMOD, 0.0, (double)B * R * h * 6.0 + 16.0 * B * h);
+        ln_mod2b_launch(c.x, h, c.u, h, mt, mt + h, mi, mi + h, (int)c.nt, (int)R, B, nm, h, s.stream);
       }
-      TRY(gemm_multi(e, s, pq, 2, 3 * h, h));   // a3 + a4 for both streams in one launch
+      GemmProblem pq[GEMM_MAX_PROBLEMS];
+      int n = 0;
+      for (int b = 0; b < B; ++b)
+        for (int st = 0; st < 2; ++st) {  // 0 = img, 1 = txt
+          const int base = double_base(j, st);
+          const int64_t r0 = st == 0 ? c.nt : 0, nr = st == 0 ? c.ni : c.nt;
+          pq[n++] = {c.u + (b * R + r0) * h, h, e->W(s, base + 2), h, (int)nr,
+                     qk_fused(E, c, epi_of(EPI_STORE_BF16, c.qkv + (b * R + r0) * 3 * h, 3 * h, e->W(s, base + 3)), r0,
+                              e->W(s, base + 4), e->W(s, base + 5), st == 0 ? 1 : 0, b)};
+        }
+      TRY(gemm_multi(e, s, pq, n, 3 * h, h));   // a3 + a4 for both streams in one launch
     }
     if (E.g->k > 1) TRY(a2a_qkv(E));
     TRY(attention_all(E));
@@ -841,23 +852,33 @@ static tsv_status run_step(StepEnv& E) {
     for (auto& c : E.rc) {
       Slot& s = *c.s;
       CK(cudaSetDevice(s.device));
-      GemmProblem pp[2], p1[2], p2[2];
-      for (int st = 0; st < 2; ++st) {
-        const int base = double_base(j, st);
-        const int64_t r0 = st == 0 ? c.nt : 0, n = st == 0 ? c.ni : c.nt;
-        const float* md = c.mod + m.mod_double(j, st);
-        float* x = c.x + r0 * h;
-        pp[st] = {c.cat + r0 * ldc, ldc, e->W(s, base + 6), h, (int)n,
-                  epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 7), md + 2 * h)};
-        p1[st] = {c.u + r0 * h, h, e->W(s, base + 8), h, (int)n,
-                  epi_of(EPI_GELU_BF16, c.hbuf + r0 * F, F, e->W(s, base + 9))};
-        p2[st] = {c.hbuf + r0 * F, F, e->W(s, base + 10), F, (int)n,
-                  epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 11), md + 5 * h)};
+      const int64_t R = c.rows;
+      GemmProblem pp[GEMM_MAX_PROBLEMS], p1[GEMM_MAX_PROBLEMS], p2[GEMM_MAX_PROBLEMS];
+      int n = 0;
+      for (int b = 0; b < B; ++b)
+        for (int st = 0; st < 2; ++st) {
+          const int base = double_base(j, st);
+          const int64_t r0 = st == 0 ? c.nt : 0, nr = st == 0 ? c.ni : c.nt;
+          const float* md = c.mod + b * nm + m.mod_double(j, st);
+          float* x = c.x + (b * R + r0) * h;
+          pp[n] = {c.cat + (b * R + r0) * ldc, ldc, e->W(s, base + 6), h, (int)nr,
+                   epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 7), md + 2 * h)};
+          p1[n] = {c.u + (b * R + r0) * h, h, e->W(s, base + 8), h, (int)nr,
+                   epi_of(EPI_GELU_BF16, c.hbuf + (b * R + r0) * F, F, e->W(s, base + 9))};
+          p2[n] = {c.hbuf + (b * R + r0) * F, F, e->W(s, base + 10), F, (int)nr,
+                   epi_of(EPI_RESID_GATE, x, h, e->W(s, base + 11), md + 5 * h)};
+          ++n;
+        }
+      TRY(gemm_multi(e, s, pp, n, h, h));        // a8: out-proj + gated residual, both streams
+      {                                          // a9: LN-modulate both streams
+        const float* mt = c.mod + m.mod_double(j, 1);
+        const float* mi = c.mod + m.mod_double(j, 0);
+        ProfScope ps(e, s, KC_LNMOD, 0.0, (double)B * R * h * 6.0 + 16.0 * B * h);
+        ln_mod2b_launch(c.x, h, c.u, h, mt + 3 * h, mt + 4 * h, mi + 3 * h, mi + 4 * h, (int)c.nt, (int)R, B, nm, h,
+                        s.stream);
       }
-      TRY(gemm_multi(e, s, pp, 2, h, h));        // a8: out-proj + gated residual, both streams
-      lnmod2(E, c, m.mod_double(j, 1), m.mod_double(j, 0), 3);   // a9: LN-modulate both streams
-      TRY(gemm_multi(e, s, p1, 2, F, h));        // fc1 + GELU
-      TRY(gemm_multi(e, s, p2, 2, h, F));        // fc2 + gated residual
+      TRY(gemm_multi(e, s, p1, n, F, h));        // fc1 + GELU
+      TRY(gemm_multi(e, s, p2, n, h, F));        // fc2 + gated residual
     }
   }
   // single-stream blocks on x = [txt; img] (zero-copy join, a10)
@@ -866,12 +887,20 @@ static tsv_status run_step(StepEnv& E) {
     for (auto& c : E.rc) {
       Slot& s = *c.s;
       CK(cudaSetDevice(s.device));
-      if (!c.rows) continue;
-      const float* md = c.mod + m.mod_single(j);
-      lnmod(e, s, c.x, c.u, md, md + h, (int)c.rows);
-      TRY(gemm(e, s, c.u, h, e->W(s, base + 2), h, (int)c.rows, 3 * h + F, h,
-               qk_fused(E, c, epi_of(EPI_SPLIT_GELU, c.qkv, 3 * h, e->W(s, base + 3), nullptr, c.cat + h, ldc, 3 * h),
-                        0, e->W(s, base + 4), e->W(s, base + 5), 2)));
+      const int64_t R = c.rows;
+      if (!R) continue;
+      {
+        const float* md = c.mod + m.mod_single(j);
+        ProfScope ps(e, s, KC_LNMOD, 0.0, (double)B * R * h * 6.0 + 16.0 * B * h);
+        ln_mod2b_launch(c.x, h, c.u, h, md, md + h, md, md + h, (int)R, (int)R, B, nm, h, s.stream);
+      }
+      GemmProblem p1[GEMM_MAX_PROBLEMS];
+      for (int b = 0; b < B; ++b)
+        p1[b] = {c.u + b * R * h, h, e->W(s, base + 2), h, (int)R,
+                 qk_fused(E, c, epi_of(EPI_SPLIT_GELU, c.qkv + b * R * 3 * h, 3 * h, e->W(s, base + 3), nullptr,
+                                       c.cat + b * R * ldc + h, ldc, 3 * h),
+                          0, e->W(s, base + 4), e->W(s, base + 5), 2, b)};
+      TRY(gemm_multi(e, s, p1, B, 3 * h + F, h));
     }
     if (E.g->k > 1) TRY(a2a_qkv(E));
     TRY(attention_all(E));
@@ -879,63 +908,82 @@ static tsv_status run_step(StepEnv& E) {
     for (auto& c : E.rc) {
       Slot& s = *c.s;
       CK(cudaSetDevice(s.device));
-      if (!c.rows) continue;
-      const float* md = c.mod + m.mod_single(j);
-      TRY(gemm(e, s, c.cat, ldc, e->W(s, base + 6), ldc, (int)c.rows, h, h + F,
-               epi_of(EPI_RESID_GATE, c.x, h, e->W(s, base + 7), md + 2 * h)));
+      const int64_t R = c.rows;
+      if (!R) continue;
+      GemmProblem p2[GEMM_MAX_PROBLEMS];
+      for (int b = 0; b < B; ++b) {
+        const float* md = c.mod + b * nm + m.mod_single(j);
+        p2[b] = {c.cat + b * R * ldc, ldc, e->W(s, base + 6), ldc, (int)R,
+                 epi_of(EPI_RESID_GATE, c.x + b * R * h, h, e->W(s, base + 7), md + 2 * h)};
+      }
+      TRY(gemm_multi(e, s, p2, B, h, h + F));
     }
   }
-  // final layer + Euler (a11, a12)
+  // final layer + Euler (a11, a12), every request of the batch in one launch
   for (auto& c : E.rc) {
     Slot& s = *c.s;
     CK(cudaSetDevice(s.device));
     if (!c.ni) continue;
-    const float* md = c.mod + m.mod_final();
-    lnmod(e, s, c.x + c.nt * h, c.u, md, md + h, (int)c.ni);
-    TRY(gemm(e, s, c.u, h, e->W(s, 18), h, (int)c.ni, m.in, h,
-             epi_of(EPI_EULER, c.sh->lat.p, m.in, e->W(s, 19), nullptr, c.sh->vel.p, m.in, 0,
-                    reinterpret_cast<const float*>(c.rd->cur.p) + m.n_mod)));
+    const int64_t R = c.rows;
+    {
+      const float* md = c.mod + m.mod_final();
+      ProfScope ps(e, s, KC_LNMOD, 0.0, (double)B * R * h * 6.0 + 16.0 * B * h);
+      ln_mod2b_launch(c.x, h, c.u, h, md, md + h, md, md + h, (int)c.nt, (int)R, B, nm, h, s.stream);
+    }
+    GemmProblem pf[GEMM_MAX_PROBLEMS];
+    for (int b = 0; b < B; ++b)
+      pf[b] = {c.u + (b * R + c.nt) * h, h, e->W(s, 18), h, (int)c.ni,
+               epi_of(EPI_EULER, c.shq[b]->lat.p, m.in, e->W(s, 19), nullptr, c.shq[b]->vel.p, m.in, 0,
+                      c.mod + B * nm + b)};
+    TRY(gemm_multi(e, s, pf, B, m.in, h));
   }
   for (auto& c : E.rc) CK(cudaGetLastError());
   return TSV_OK;
 }
 
-// SD3-medium step (DESIGN.md O-SD3).  B = 2 evaluations (b = 0 conditional, b = 1 unconditional
-// branch of the CFG pair, S23) share every launch: evaluation b owns rows [b*rows, (b+1)*rows) of
-// each activation buffer, laid out [txt_r ; img_r] like FLUX.  Joint blocks are double blocks
-// without QK-norm and RoPE, so the QKV epilogue is a plain store (k = 1) or a pure Ulysses pack
-// (k > 1); joint attention over [txt; img] equals diffusers' [img; txt] (no position-dependent
-// term, the softmax is permutation-equivariant).  The last block's txt stream is context_pre_only
-// (AdaLayerNormContinuous (scale, shift), QKV only).  The CFG combine is fused into the Euler
-// epilogue of the final linear.
+// SD3-medium step (DESIGN.md O-SD3).  Every request contributes B_model = 2 evaluations (branch 0
+// conditional, 1 unconditional, S23); evaluation b = q*2 + branch owns rows [b*rows, (b+1)*rows) of
+// each activation buffer, laid out [txt_r ; img_r] like FLUX, and all evaluations share every
+// launch.  Joint blocks are double blocks without QK-norm and RoPE, so the QKV epilogue is a plain
+// store (k = 1) or a pure Ulysses pack / peer store (k > 1); joint attention over [txt; img] equals
+// diffusers' [img; txt] (no position-dependent term, the softmax is permutation-equivariant).  The
+// last block's txt stream is context_pre_only (AdaLayerNormContinuous (scale, shift), QKV only).
+// The CFG combine is fused into the Euler epilogue of the final linear.
 static tsv_status run_step_sd3(StepEnv& E) {
   tsv_engine* e = E.e;
   const Model& m = e->model;
-  const int h = m.h, F = m.F, B = m.B;
+  const int h = m.h, F = m.F, B = E.B, nq = (int)E.Rq.size();
   const int64_t ldc = h + F, nm = m.n_mod;
   const int k = E.g->k;
   const int nd = m.d.n_double;
-  // a1: img = x W^T + b + PE (identical for both evaluations), txt_b = T_b W^T + b
+  // a1: img = x W^T + b + PE (identical for both branches of a request), txt_b = T_b W^T + b
   for (auto& c : E.rc) {
     Slot& s = *c.s;
     CK(cudaSetDevice(s.device));
     const int64_t R = c.rows;
     if (c.ni) {
-      float* xi0 = c.x + c.nt * h;
-      {
-        ProfScope ps(e, s, KC_OTHER, 0.0, 6.0 * c.ni * m.in);
-        f32_to_bf16_launch(reinterpret_cast<float*>(c.sh->lat.p), m.in, c.latb, m.in, (int)c.ni, m.in, s.stream);
+      GemmProblem pi[GEMM_MAX_PROBLEMS];
+      for (int q = 0; q < nq; ++q) {
+        float* xi = c.x + (2 * q * R + c.nt) * h;
+        {
+          ProfScope ps(e, s, KC_OTHER, 0.0, 6.0 * c.ni * m.in);
+          f32_to_bf16_launch(reinterpret_cast<float*>(c.shq[q]->lat.p), m.in, c.latb + q * c.ni * m.in, m.in,
+                             (int)c.ni, m.in, s.stream);
+        }
+        CK(cudaMemcpyAsync(xi, c.shq[q]->pe.p, c.ni * h * 4, cudaMemcpyDeviceToDevice, s.stream));
+        pi[q] = {c.latb + q * c.ni * m.in, m.in, e->W(s, 0), m.in, (int)c.ni, epi_of(EPI_ACCUM_F32, xi, h, e->W(s, 1))};
       }
-      CK(cudaMemcpyAsync(xi0, c.sh->pe.p, c.ni * h * 4, cudaMemcpyDeviceToDevice, s.stream));
-      TRY(gemm(e, s, c.latb, m.in, e->W(s, 0), m.in, (int)c.ni, h, m.in, epi_of(EPI_ACCUM_F32, xi0, h, e->W(s, 1))));
-      for (int b = 1; b < B; ++b)
-        CK(cudaMemcpyAsync(xi0 + b * R * h, xi0, c.ni * h * 4, cudaMemcpyDeviceToDevice, s.stream));
+      TRY(gemm_multi(e, s, pi, nq, h, m.in));
+      for (int q = 0; q < nq; ++q) {
+        float* xi = c.x + (2 * q * R + c.nt) * h;
+        CK(cudaMemcpyAsync(xi + R * h, xi, c.ni * h * 4, cudaMemcpyDeviceToDevice, s.stream));
+      }
     }
     if (c.nt) {
-      GemmProblem pt[2];
+      GemmProblem pt[GEMM_MAX_PROBLEMS];
       for (int b = 0; b < B; ++b)
-        pt[b] = {reinterpret_cast<bf16*>(c.sh->T.p) + b * c.nt * m.ctx, m.ctx, e->W(s, 2), m.ctx, (int)c.nt,
-                 epi_of(EPI_STORE_F32, c.x + b * R * h, h, e->W(s, 3))};
+        pt[b] = {reinterpret_cast<bf16*>(c.shq[b / 2]->T.p) + (b % 2) * c.nt * m.ctx, m.ctx, e->W(s, 2), m.ctx,
+                 (int)c.nt, epi_of(EPI_STORE_F32, c.x + b * R * h, h, e->W(s, 3))};
       TRY(gemm_multi(e, s, pt, B, h, m.ctx));
     }
   }
@@ -946,7 +994,7 @@ static tsv_status run_step_sd3(StepEnv& E) {
       CK(cudaSetDevice(s.device));
       const int64_t R = c.rows;
       if (!R) continue;
-      // a2: LN-modulate both streams of both evaluations in one launch
+      // a2: LN-modulate both streams of every evaluation in one launch
       {
         const float* mi = c.mod + m.mod_double(j, 0);
         const float* mt = c.mod + m.mod_double(j, 1);
@@ -954,7 +1002,7 @@ static tsv_status run_step_sd3(StepEnv& E) {
         ln_mod2b_launch(c.x, h, c.u, h, last ? mt + h : mt, last ? mt : mt + h, mi, mi + h, (int)c.nt, (int)R, B, nm,
                         h, s.stream);
       }
-      // a3 (+ Ulysses pack for k > 1): 2 streams x 2 evaluations in one launch
+      // a3 (+ Ulysses pack / peer stores for k > 1): 2 streams x B evaluations in one launch
       GemmProblem pq[GEMM_MAX_PROBLEMS];
       int n = 0;
       for (int b = 0; b < B; ++b)
@@ -997,10 +1045,10 @@ static tsv_status run_step_sd3(StepEnv& E) {
           ++n;
         }
       TRY(gemm_multi(e, s, pp, n, h, h));  // a8: out-proj + gated residual
-      {                                     // a9: LN-modulate (both evaluations, one launch)
+      {                                     // a9: LN-modulate (every evaluation, one launch)
         const float* mi = c.mod + m.mod_double(j, 0);
         // context_pre_only: the txt rows are dead after the attention; they are normalised with
-        // the img vectors (in bounds, result unused) so both evaluations stay one launch
+        // the img vectors (in bounds, result unused) so all evaluations stay one launch
         const float* mt = last ? mi : c.mod + m.mod_double(j, 1);
         ProfScope ps(e, s, KC_LNMOD, 0.0, (double)B * R * h * 6.0 + 16.0 * B * h);
         ln_mod2b_launch(c.x, h, c.u, h, mt + 3 * h, mt + 4 * h, mi + 3 * h, mi + 4 * h, (int)c.nt, (int)R, B, nm, h,
@@ -1018,17 +1066,21 @@ static tsv_status run_step_sd3(StepEnv& E) {
     if (!c.ni) continue;
     const int64_t R = c.rows;
     {
-      // both evaluations' img rows (txt rows normalised too, unused): u_b rows [nt, R)
       const float* md = c.mod + m.mod_final();
       ProfScope ps(e, s, KC_LNMOD, 0.0, (double)B * R * h * 6.0 + 16.0 * B * h);
       ln_mod2b_launch(c.x, h, c.u, h, md + h, md, md + h, md, (int)c.nt, (int)R, B, nm, h, s.stream);
     }
-    const float* dt = reinterpret_cast<const float*>(c.rd->cur.p) + B * nm;
-    TRY(gemm(e, s, c.u + (R + c.nt) * h, h, e->W(s, 18), h, (int)c.ni, m.in, h,
-             epi_of(EPI_STORE_F32, c.sh->vel.p, m.in, e->W(s, 19))));
-    GemmEpi ep = epi_of(EPI_CFG_EULER, c.sh->lat.p, m.in, e->W(s, 19), nullptr, c.sh->vel.p, m.in, 0, dt);
-    ep.alpha = m.d.cfg_scale;
-    TRY(gemm(e, s, c.u + c.nt * h, h, e->W(s, 18), h, (int)c.ni, m.in, h, ep));
+    GemmProblem pu[GEMM_MAX_PROBLEMS], pc[GEMM_MAX_PROBLEMS];
+    for (int q = 0; q < nq; ++q) {
+      pu[q] = {c.u + ((2 * q + 1) * R + c.nt) * h, h, e->W(s, 18), h, (int)c.ni,
+               epi_of(EPI_STORE_F32, c.shq[q]->vel.p, m.in, e->W(s, 19))};
+      GemmEpi ep = epi_of(EPI_CFG_EULER, c.shq[q]->lat.p, m.in, e->W(s, 19), nullptr, c.shq[q]->vel.p, m.in, 0,
+                          c.mod + B * nm + q);
+      ep.alpha = m.d.cfg_scale;
+      pc[q] = {c.u + (2 * q * R + c.nt) * h, h, e->W(s, 18), h, (int)c.ni, ep};
+    }
+    TRY(gemm_multi(e, s, pu, nq, m.in, h));
+    TRY(gemm_multi(e, s, pc, nq, m.in, h));
   }
   for (auto& c : E.rc) CK(cudaGetLastError());
   return TSV_OK;
@@ -1143,34 +1195,45 @@ static tsv_status new_event(tsv_engine* e, const std::vector<int>& slots_, tsv_e
   return TSV_OK;
 }
 
-static tsv_status do_step(tsv_engine* e, Request& R, int step, int gi, tsv_event* done) {
+static void drop_graph(StepGraph& gr) {
+  if (gr.exec) cudaGraphExecDestroy(gr.exec);
+  gr.exec = nullptr;
+}
+
+// One step of every request in Rs (each at its own next step) as one batched step on group gi.
+// The requests share the resolution (checked by the caller); their shards land on the group first.
+static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi, tsv_event* done) {
   Group& g = e->groups[gi];
   if (g.local_slots.empty()) {
     if (done) *done = -1;
-    R.next_step = step + 1;
+    for (Request* R : Rs) R->next_step++;
     return TSV_OK;
   }
-  if (R.group != gi) TRY(move_request(e, R, gi));
+  for (Request* R : Rs)
+    if (R->group != gi) TRY(move_request(e, *R, gi));
   const Model& m = e->model;
+  Request& R0 = *Rs[0];
   StepEnv E;
-  E.e = e; E.R = &R; E.g = &g; E.step = step;
+  E.e = e; E.R = &R0; E.Rq = Rs; E.g = &g;
+  E.B = (int)Rs.size() * m.B;
   E.fused = e->transport == TSV_TRANSPORT_FUSED && g.all_local && g.k > 1;
   const int k = g.k;
   E.t_off.resize(k); E.t_cnt.resize(k); E.i_off.resize(k); E.i_cnt.resize(k);
   for (int r = 0; r < k; ++r) {
-    E.t_off[r] = shard_begin(R.Lt, k, r);
-    E.t_cnt[r] = shard_begin(R.Lt, k, r + 1) - E.t_off[r];
-    E.i_off[r] = shard_begin(R.Li, k, r);
-    E.i_cnt[r] = shard_begin(R.Li, k, r + 1) - E.i_off[r];
+    E.t_off[r] = shard_begin(R0.Lt, k, r);
+    E.t_cnt[r] = shard_begin(R0.Lt, k, r + 1) - E.t_off[r];
+    E.i_off[r] = shard_begin(R0.Li, k, r);
+    E.i_cnt[r] = shard_begin(R0.Li, k, r + 1) - E.i_off[r];
   }
-  const int64_t L = R.Lt + R.Li;
+  const int64_t L = R0.Lt + R0.Li;
   for (size_t q = 0; q < g.local_slots.size(); ++q) {
     const int si = g.local_slots[q];
     Slot& s = e->slots[si];
-    ReqShard& sh = R.shard[si];
-    TRY(ensure_workspace(e, s, sh.nt + sh.ni, L, k));
+    ReqShard& sh = R0.shard[si];
+    TRY(ensure_workspace(e, s, sh.nt + sh.ni, L, k, E.B));
     RankCtx c;
-    c.si = si; c.s = &s; c.sh = &sh; c.rd = &R.dev[si];
+    c.si = si; c.s = &s; c.sh = &sh;
+    for (Request* R : Rs) { c.shq.push_back(&R->shard[si]); c.rdq.push_back(&R->dev[si]); }
     c.nt = sh.nt; c.ni = sh.ni; c.rows = sh.nt + sh.ni;
     c.x = reinterpret_cast<float*>(s.ws.x.p);
     c.u = reinterpret_cast<bf16*>(s.ws.u.p);
@@ -1182,89 +1245,124 @@ static tsv_status do_step(tsv_engine* e, Request& R, int step, int gi, tsv_event
     c.recv = reinterpret_cast<bf16*>(s.ws.recv.p);
     c.obuf = reinterpret_cast<bf16*>(s.ws.obuf.p);
     c.orecv = reinterpret_cast<bf16*>(s.ws.orecv.p);
-    c.mod = reinterpret_cast<const float*>(c.rd->cur.p);
+    c.mod = reinterpret_cast<float*>(s.ws.bmod.p);
     E.rc.push_back(c);
   }
-  // each slot's stream must follow the request's previous work on that slot; then publish the
-  // step index (pageable source: staged at call time, so the host value can change right after)
+  // each slot's stream must follow every request's previous work on that slot; then publish the
+  // step indices (pageable source: staged at call time, so the host value can change right after)
   for (auto& c : E.rc) {
     CK(cudaSetDevice(c.s->device));
-    auto it = R.last.find(c.si);
-    if (it != R.last.end()) CK(cudaStreamWaitEvent(c.s->stream, it->second, 0));
-    int st = step;
-    CK(cudaMemcpyAsync(c.rd->step.p, &st, sizeof(int), cudaMemcpyHostToDevice, c.s->stream));
+    for (size_t q = 0; q < Rs.size(); ++q) {
+      auto it = Rs[q]->last.find(c.si);
+      if (it != Rs[q]->last.end()) CK(cudaStreamWaitEvent(c.s->stream, it->second, 0));
+      int st = Rs[q]->next_step;
+      CK(cudaMemcpyAsync(c.rdq[q]->step.p, &st, sizeof(int), cudaMemcpyHostToDevice, c.s->stream));
+    }
   }
   if (e->graphs && E.rc.size() == 1) {
-    // one local rank: replay (or capture once) the whole step as a CUDA graph
+    // one local rank: replay (or capture once) the whole step as a CUDA graph, cached per slot by
+    // every buffer it references
     RankCtx& c = E.rc[0];
-    ReqDev& rd = *c.rd;
+    Slot& slot = *c.s;
     uint64_t key = 1469598103934665603ull;
     auto mix = [&](uint64_t v) { key = (key ^ v) * 1099511628211ull; };
-    const void* ptrs[] = {c.x, c.u, c.qkv, c.cat, c.hbuf, c.latb, c.pack, c.recv, c.obuf, c.orecv,
-                          c.sh->lat.p, c.sh->vel.p, c.sh->T.p, c.sh->cosb.p, c.sh->sinb.p, c.sh->pe.p, rd.mod.p,
-                          rd.cur.p, rd.step.p};
+    const void* ptrs[] = {c.x, c.u, c.qkv, c.cat, c.hbuf, c.latb, c.pack, c.recv, c.obuf, c.orecv, c.mod};
     for (const void* p : ptrs) mix(reinterpret_cast<uintptr_t>(p));
+    for (size_t q = 0; q < Rs.size(); ++q) {
+      const ReqShard* sh = c.shq[q];
+      const ReqDev* rd = c.rdq[q];
+      const void* rp[] = {sh->lat.p, sh->vel.p, sh->T.p, sh->cosb.p, sh->sinb.p, sh->pe.p, rd->mod.p, rd->dt.p,
+                          rd->step.p};
+      for (const void* p : rp) mix(reinterpret_cast<uintptr_t>(p));
+      mix((uint64_t)Rs[q]->id);
+    }
     mix((uint64_t)gi);
     mix((uint64_t)c.rows);
+    mix((uint64_t)Rs.size());
     mix((uint64_t)e->prof);   // a profiled graph carries event-record nodes around every launch
-    if (!rd.gexec || rd.gkey != key) {
-      if (rd.gexec) { cudaGraphExecDestroy(rd.gexec); rd.gexec = nullptr; }
-      CK(cudaSetDevice(c.s->device));
+    auto it = slot.graphs.find(key);
+    if (it == slot.graphs.end()) {
+      // bounded cache: evict the least recently used graph
+      if (slot.graphs.size() >= 64) {
+        auto lru = slot.graphs.begin();
+        for (auto jt = slot.graphs.begin(); jt != slot.graphs.end(); ++jt)
+          if (jt->second.last_use < lru->second.last_use) lru = jt;
+        drop_graph(lru->second);
+        slot.graphs.erase(lru);
+      }
+      CK(cudaSetDevice(slot.device));
+      StepGraph gr;
+      for (Request* R : Rs) gr.reqs.push_back(R->id);
       const int64_t k0 = e->kernel_count;
       const size_t r0 = e->prof_recs.size();
       double f0[8], b0[8];
       int64_t l0[8];
       for (int i = 0; i < 8; ++i) { f0[i] = e->prof_flops[i]; b0[i] = e->prof_bytes[i]; l0[i] = e->prof_launch[i]; }
-      CK(cudaStreamBeginCapture(c.s->stream, cudaStreamCaptureModeThreadLocal));
+      CK(cudaStreamBeginCapture(slot.stream, cudaStreamCaptureModeThreadLocal));
       tsv_status st = run_step(E);
       cudaGraph_t graph = nullptr;
-      cudaError_t ce = cudaStreamEndCapture(c.s->stream, &graph);
+      cudaError_t ce = cudaStreamEndCapture(slot.stream, &graph);
       // what ProfScope recorded during capture belongs to the graph: re-added at every replay
-      rd.gprof.assign(e->prof_recs.begin() + r0, e->prof_recs.end());
+      gr.prof.assign(e->prof_recs.begin() + r0, e->prof_recs.end());
       e->prof_recs.resize(r0);
       for (int i = 0; i < 8; ++i) {
-        rd.gflops[i] = e->prof_flops[i] - f0[i];
-        rd.gbytes[i] = e->prof_bytes[i] - b0[i];
-        rd.glaunch[i] = e->prof_launch[i] - l0[i];
+        gr.flops[i] = e->prof_flops[i] - f0[i];
+        gr.bytes[i] = e->prof_bytes[i] - b0[i];
+        gr.launch[i] = e->prof_launch[i] - l0[i];
         e->prof_flops[i] = f0[i]; e->prof_bytes[i] = b0[i]; e->prof_launch[i] = l0[i];
       }
       if (st != TSV_OK) { if (graph) cudaGraphDestroy(graph); return st; }
       if (ce != cudaSuccess) return fail(TSV_E_CUDA, "step capture: %s", cudaGetErrorString(ce));
-      ce = cudaGraphInstantiate(&rd.gexec, graph, 0);
+      ce = cudaGraphInstantiate(&gr.exec, graph, 0);
       cudaGraphDestroy(graph);
-      if (ce != cudaSuccess) { rd.gexec = nullptr; return fail(TSV_E_CUDA, "graph instantiate: %s", cudaGetErrorString(ce)); }
-      rd.gkey = key;
-      rd.gkernels = e->kernel_count - k0;
+      if (ce != cudaSuccess) return fail(TSV_E_CUDA, "graph instantiate: %s", cudaGetErrorString(ce));
+      gr.kernels = e->kernel_count - k0;
       e->kernel_count = k0;
+      it = slot.graphs.emplace(key, std::move(gr)).first;
     }
-    CK(cudaGraphLaunch(rd.gexec, c.s->stream));
-    e->kernel_count += rd.gkernels;
+    StepGraph& gr = it->second;
+    gr.last_use = ++e->graph_clock;
+    CK(cudaGraphLaunch(gr.exec, slot.stream));
+    e->kernel_count += gr.kernels;
     if (e->prof) {
       // the graph's event pairs now hold this replay's timestamps
-      e->prof_recs.insert(e->prof_recs.end(), rd.gprof.begin(), rd.gprof.end());
+      e->prof_recs.insert(e->prof_recs.end(), gr.prof.begin(), gr.prof.end());
       for (int i = 0; i < 8; ++i) {
-        e->prof_flops[i] += rd.gflops[i];
-        e->prof_bytes[i] += rd.gbytes[i];
-        e->prof_launch[i] += rd.glaunch[i];
+        e->prof_flops[i] += gr.flops[i];
+        e->prof_bytes[i] += gr.bytes[i];
+        e->prof_launch[i] += gr.launch[i];
       }
     }
   } else {
     TRY(run_step(E));
   }
-  for (auto& c : E.rc) TRY(record_last(e, R, c.si));
-  R.next_step = step + 1;
-  R.has_velocity = true;
+  for (Request* R : Rs) {
+    for (auto& c : E.rc) TRY(record_last(e, *R, c.si));
+    R->next_step++;
+    R->has_velocity = true;
+  }
   if (done) TRY(new_event(e, g.local_slots, done));
   return TSV_OK;
 }
 
 static void release_reqdev(ReqDev& d) {
-  if (d.gexec) cudaGraphExecDestroy(d.gexec);
-  d.gexec = nullptr;
   d.mod.release();
   d.dt.release();
-  d.cur.release();
   d.step.release();
+}
+
+// drop every cached step graph that references request `id` (its buffers are about to be freed)
+static void drop_request_graphs(tsv_engine* e, int64_t id) {
+  for (auto& s : e->slots)
+    for (auto it = s.graphs.begin(); it != s.graphs.end();) {
+      const auto& r = it->second.reqs;
+      if (std::find(r.begin(), r.end(), id) != r.end()) {
+        drop_graph(it->second);
+        it = s.graphs.erase(it);
+      } else {
+        ++it;
+      }
+    }
 }
 
 }  // namespace tsv
@@ -1354,6 +1452,8 @@ void tsv_engine_destroy(tsv_engine* e) {
     cudaSetDevice(s.device);
     cudaStreamSynchronize(s.stream);
   }
+  for (auto& s : e->slots)
+    for (auto& kv : s.graphs) drop_graph(kv.second);
   for (auto& kv : e->requests) {
     for (auto& d : kv.second.dev) release_reqdev(d.second);
     for (auto& sh : kv.second.shard) sh.second.release();
@@ -1369,7 +1469,8 @@ void tsv_engine_destroy(tsv_engine* e) {
     for (auto& p : rec.evs) cudaEventDestroy(p.second);
   for (auto& s : e->slots) {
     Workspace& w = s.ws;
-    for (DevBuf* b : {&w.x, &w.u, &w.qkv, &w.cat, &w.hbuf, &w.latb, &w.pack, &w.recv, &w.obuf, &w.orecv, &s.scratch})
+    for (DevBuf* b : {&w.x, &w.u, &w.qkv, &w.cat, &w.hbuf, &w.latb, &w.pack, &w.recv, &w.obuf, &w.orecv, &w.bmod,
+                      &s.scratch})
       b->release();
     cudaSetDevice(s.device);
     cudaStreamDestroy(s.stream);
@@ -1502,6 +1603,7 @@ tsv_status tsv_request_create(tsv_engine* e, int height, int width, int num_step
   R.ts[0] = 1.0;
   R.ts[num_steps] = 0.0;
   const int64_t id = e->next_req++;
+  R.id = id;
   e->requests.emplace(id, std::move(R));
   *out = id;
   return TSV_OK;
@@ -1532,7 +1634,26 @@ tsv_status tsv_request_step(tsv_engine* e, tsv_request r, int step, tsv_group gi
     return fail(TSV_E_STATE, "step %d requested but the next step is %d (step dependency, P:235-239)", step,
                 R->next_step);
   if (step >= R->S) return fail(TSV_E_STATE, "request has only %d steps", R->S);
-  return do_step(e, *R, step, gi, done);
+  return do_step(e, std::vector<Request*>{R}, gi, done);
+}
+
+tsv_status tsv_request_step_batch(tsv_engine* e, const tsv_request* reqs, int n, tsv_group gi, tsv_event* done) {
+  if (!e || !reqs) return fail(TSV_E_INVAL, "null argument");
+  if (gi < 0 || gi >= (int)e->groups.size()) return fail(TSV_E_INVAL, "unknown group %d", gi);
+  const int max_req = GEMM_MAX_PROBLEMS / (2 * e->model.B);
+  if (n < 1 || n > max_req) return fail(TSV_E_INVAL, "batch of %d requests (1..%d for this model)", n, max_req);
+  std::vector<Request*> Rs;
+  for (int i = 0; i < n; ++i) {
+    Request* R = get_req(e, reqs[i]);
+    if (!R) return fail(TSV_E_INVAL, "unknown request %lld", (long long)reqs[i]);
+    for (Request* o : Rs)
+      if (o == R) return fail(TSV_E_INVAL, "request %lld appears twice", (long long)reqs[i]);
+    if (R->next_step >= R->S) return fail(TSV_E_STATE, "request %lld has no step left", (long long)reqs[i]);
+    if (!Rs.empty() && (R->height != Rs[0]->height || R->width != Rs[0]->width))
+      return fail(TSV_E_INVAL, "a batch needs one resolution (P:411)");
+    Rs.push_back(R);
+  }
+  return do_step(e, Rs, gi, done);
 }
 
 tsv_status tsv_request_reshard(tsv_engine* e, tsv_request r, tsv_group gi, tsv_event* done) {
@@ -1653,6 +1774,7 @@ tsv_status tsv_request_destroy(tsv_engine* e, tsv_request r) {
   if (it == e->requests.end()) return fail(TSV_E_INVAL, "unknown request %lld", (long long)r);
   Request& R = it->second;
   for (auto& l : R.last) { cudaEventSynchronize(l.second); cudaEventDestroy(l.second); }
+  drop_request_graphs(e, r);
   for (auto& d : R.dev) release_reqdev(d.second);
   for (auto& sh : R.shard) sh.second.release();
   e->requests.erase(it);

@@ -45,6 +45,8 @@ struct GemmMaps {
   CUtensorMap A[GEMM_MAX_PROBLEMS];
   CUtensorMap B[GEMM_MAX_PROBLEMS];
 };
+// > 4 KB of kernel parameters (CUDA 12.1+, up to 32 764 bytes)
+static_assert(sizeof(GemmArgs) + sizeof(GemmMaps) <= 32764, "GEMM kernel parameters too large");
 
 // Rasterisation: groups of GROUP_N weight-column tiles; inside a group the n index varies fastest,
 // then m.  A wave of 148 concurrent tiles therefore touches <= GROUP_N weight tiles and
@@ -607,7 +609,7 @@ static const char* check_epi(const GemmEpi& epi, int bn) {
 int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int K, int num_sms, const char** err,
                     int force_bn, int force_pair) {
   *err = nullptr;
-  if (nprob < 1 || nprob > GEMM_MAX_PROBLEMS) { *err = "gemm: 1 to 4 problems per launch"; return -1; }
+  if (nprob < 1 || nprob > GEMM_MAX_PROBLEMS) { *err = "gemm: 1 to 16 problems per launch"; return -1; }
   if (N <= 0 || K <= 0) { *err = "gemm: empty shape"; return -1; }
   if (K % BK) { *err = "gemm: K must be a multiple of 64"; return -1; }
   if (N % 64) { *err = "gemm: N must be a multiple of 64"; return -1; }

@@ -43,7 +43,7 @@ enum EpiMode : int {
   EPI_CFG_EULER = 8,    // v_c = acc + b; v = out1 + alpha (v_c - out1) (out1 holds v_u on entry);
                         // out1 (fp32) [m,n] = v; out0 (fp32) [m,n] += (*scalar) * v   (SD3 CFG, S23)
 };
-constexpr int GEMM_MAX_PROBLEMS = 4;
+constexpr int GEMM_MAX_PROBLEMS = 16;  // 2 streams x up to 8 evaluations (requests x CFG branches)
 
 struct GemmEpi {
   int mode = EPI_STORE_BF16;
@@ -106,7 +106,7 @@ struct GemmProblem {
 struct GemmPlan {
   int nprob = 1;
   CUtensorMap tmAq[GEMM_MAX_PROBLEMS], tmBq[GEMM_MAX_PROBLEMS];
-  int Mq[GEMM_MAX_PROBLEMS] = {0, 0, 0, 0}, tile0[GEMM_MAX_PROBLEMS] = {0, 0, 0, 0};
+  int Mq[GEMM_MAX_PROBLEMS] = {}, tile0[GEMM_MAX_PROBLEMS] = {};
   GemmEpi epiq[GEMM_MAX_PROBLEMS];
   int M = 0, N = 0, K = 0;
   int BN = 256;
