@@ -38,6 +38,19 @@ tsv_status tsv_sched_allocate(const double* T, int n_res, const int* ks, int n_k
 tsv_status tsv_sched_round(const double* T, int n_res, const int* ks, int n_k, const tsv_sched_request* reqs, int R,
                            double now, double tau, int N, int* gpus_out, int* steps_out, int* survivors);
 
+/* GPU placement with preservation and elastic scale-up (S:§8(f) NEXT #4).  gpus[i] =
+ * GPUs granted to request i this round (0 or a power of two, e.g. tsv_sched_round's gpus_out),
+ * rows[i] its table row, prev_mask[i] the bitmask of the GPUs it held in the previous round (0 =
+ * none).  N <= 64.  Placement: requests in decreasing size (ties: lower index) each take the free
+ * aligned block (start % size == 0) with the largest overlap with prev_mask[i] (ties: lowest
+ * start), so a request whose size is unchanged and whose block is free keeps its GPUs (no
+ * reshard).  Elastic scale-up (scale_up != 0, work-conserving): while some placed request of size
+ * g has its buddy block (the other half of its aligned 2g block) entirely idle and T(row, 2g) <
+ * T(row, g), the one with the largest T(g) / T(2g) (ties: lower index) doubles in place.  Output:
+ * mask_out[i] (popcount = the final size).  Errors: TSV_E_INVAL (sizes, total > N, no fit). */
+tsv_status tsv_sched_place(const double* T, int n_res, const int* ks, int n_k, const int* rows, const int* gpus,
+                           const uint64_t* prev_mask, int R, int N, int scale_up, uint64_t* mask_out);
+
 const char* tsv_sched_last_error(void);
 
 #ifdef __cplusplus

@@ -45,3 +45,16 @@ def schedule_round(T, ks, requests, now: float, tau: float, N: int):
     check_sched(lib.tsv_sched_round(T.ctypes.data_as(C.POINTER(C.c_double)), n_res, kk, n_k, arr, R, now, tau, N, g, s,
                                     C.byref(sv)))
     return sv.value, [(g[i], s[i]) for i in range(R)]
+
+
+def place(T, ks, rows, gpus, prev, N: int, scale_up: bool = True):
+    """-> [set of GPU ids] per request.  prev: [set of GPU ids held last round] per request."""
+    T, kk, n_res, n_k = _table(T, ks)
+    R = len(gpus)
+    rr = (C.c_int * max(R, 1))(*rows)
+    gg = (C.c_int * max(R, 1))(*gpus)
+    pm = (C.c_uint64 * max(R, 1))(*[sum(1 << g for g in p) for p in prev])
+    out = (C.c_uint64 * max(R, 1))()
+    check_sched(lib.tsv_sched_place(T.ctypes.data_as(C.POINTER(C.c_double)), n_res, kk, n_k, rr, gg, pm, R, N,
+                                    1 if scale_up else 0, out))
+    return [{b for b in range(N) if out[i] >> b & 1} for i in range(R)]

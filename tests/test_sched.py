@@ -132,3 +132,57 @@ def test_scheduler_latency(sched):
     for _ in range(10):
         sched.schedule_round(T, KS, reqs, 0.0, 0.25, 8)
     assert (time.perf_counter() - t0) / 10 < 0.010
+
+
+# ----------------------------------------------------------------------------- placement (NEXT #4)
+def _rand_plan(rng, N):
+    sizes = []
+    left = N
+    while left > 0 and rng.random() < 0.8:
+        g = int(rng.choice([k for k in KS if k <= left]))
+        sizes.append(g)
+        left -= g
+    sizes += [0] * int(rng.integers(0, 3))
+    rng.shuffle(sizes)
+    return sizes
+
+
+def test_place_matches_oracle(sched):
+    rng = np.random.default_rng(5)
+    for _ in range(500):
+        N = int(rng.choice([2, 4, 8, 16]))
+        T = random_table(rng)
+        gpus = _rand_plan(rng, N)
+        R = len(gpus)
+        rows = [int(rng.integers(0, 4)) for _ in range(R)]
+        prev = [set(int(x) for x in rng.choice(N, size=int(rng.integers(0, N + 1)), replace=False)) for _ in range(R)]
+        for up in (False, True):
+            got = sched.place(T, KS, rows, gpus, prev, N, up)
+            ref = OS.place(T, KS, rows, gpus, prev, N, up)
+            assert got == ref
+            used = set()
+            for i, b in enumerate(got):
+                assert not (b & used)                       # disjoint
+                used |= b
+                if b:
+                    g, s = len(b), min(b)
+                    assert b == set(range(s, s + g)) and s % g == 0   # aligned power-of-two block
+                    assert g >= gpus[i] if up else g == gpus[i]
+                else:
+                    assert gpus[i] == 0
+
+
+def test_place_preserves_previous_blocks(sched):
+    T = np.array([[1.0, 0.6, 0.35, 0.2]])
+    # same sizes as last round and those blocks are free: every request keeps its GPUs
+    prev = [{4, 5, 6, 7}, {2, 3}, {1}]
+    got = sched.place(T, KS, [0, 0, 0], [4, 2, 1], prev, 8, False)
+    assert got == prev
+    # elastic scale-up: the idle GPU 0 doubles the 1-GPU request in place (buddy of {1})
+    got = sched.place(T, KS, [0, 0, 0], [4, 2, 1], prev, 8, True)
+    assert got == [{4, 5, 6, 7}, {2, 3}, {0, 1}]
+    # no gain from a larger degree: no scale-up
+    Tflat = np.array([[1.0, 1.0, 1.0, 1.0]])
+    assert sched.place(Tflat, KS, [0], [1], [set()], 8, True) == [{0}]
+    with pytest.raises(Exception):
+        sched.place(T, KS, [0, 0], [8, 1], [set(), set()], 8, False)   # over capacity
