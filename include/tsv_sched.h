@@ -44,7 +44,9 @@ tsv_status tsv_sched_round(const double* T, int n_res, const int* ks, int n_k, c
  * none).  N <= 64.  Placement: requests in decreasing size (ties: lower index) each take the free
  * aligned block (start % size == 0) with the largest overlap with prev_mask[i] (ties: lowest
  * start), so a request whose size is unchanged and whose block is free keeps its GPUs (no
- * reshard).  Elastic scale-up (scale_up != 0, work-conserving): while some placed request of size
+ * reshard).  Elastic scale-up (scale_up != 0, work-conserving, "no GPU remains unused"):
+ * first every request left without GPUs takes one idle GPU (one it held before if free, else the
+ * lowest), in index order; then while some placed request of size
  * g has its buddy block (the other half of its aligned 2g block) entirely idle and T(row, 2g) <
  * T(row, g), the one with the largest T(g) / T(2g) (ties: lower index) doubles in place.  Output:
  * mask_out[i] (popcount = the final size).  Errors: TSV_E_INVAL (sizes, total > N, no fit). */

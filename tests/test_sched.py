@@ -170,6 +170,8 @@ def test_place_matches_oracle(sched):
                     assert g >= gpus[i] if up else g == gpus[i]
                 else:
                     assert gpus[i] == 0
+            if up:   # work-conserving: GPUs stay idle only if every request already has some
+                assert len(used) == N or all(got)
 
 
 def test_place_preserves_previous_blocks(sched):

@@ -1,0 +1,66 @@
+"""Step-latency table T(res, k) for the serving simulator (tools/serve_sim.py) from ONE GPU.
+
+k = 1: measured (tsv_latency_table, CUDA events, median).  k > 1: the per-rank compute measured
+with k virtual ranks on the one device (fused transport: the all-to-alls are epilogue stores plus
+an event barrier, so the measured time is the ranks' compute) divided by k, plus a modeled NVLink 5
+all-to-all per attention: bytes_r (k - 1) / k / 900 GB/s + 10 us, two per block.  This is a model
+for k > 1 (virtual ranks share one GPU's SMs), stated as such in the output; an 8-GPU measurement
+replaces it.
+
+  python tools/latency_table_model.py [--model flux] [--out profiles/r01/latency_table_model.json]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+RES = [256, 512, 1024, 2048]
+KS = [1, 2, 4, 8]
+
+
+def main():
+    import paper_conf_asplos_luhtlwm0c26_b200 as tsv
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--model", default="flux")
+    ap.add_argument("--iters", type=int, default=5)
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r01", "latency_table_model.json"))
+    args = ap.parse_args()
+    d = tsv.model_preset(args.model)
+    h, Lt = d.hidden, d.text_tokens
+    blocks = d.n_double + d.n_single
+    B = 2 if d.family == 1 else 1
+    eng = tsv.Engine(args.model, devices=[0] * 8)
+    ms, cv = eng.latency_table(RES, KS, warmup=2, iters=args.iters)
+    eng.close()
+    table = []
+    comm = []
+    for i, r in enumerate(RES):
+        Li = (r // 16) ** 2
+        row, crow = [], []
+        for j, k in enumerate(KS):
+            if k == 1:
+                row.append(float(ms[i, j]))
+                crow.append(0.0)
+                continue
+            rows_r = -(-(Li + Lt) // k)
+            bytes_r = B * rows_r * (3 * h + h) * 2 * (k - 1) / k       # a2a #1 (q|k|v) + #2 (o)
+            c_ms = blocks * (bytes_r / 900e9 + 2 * 10e-6) * 1e3
+            row.append(float(ms[i, j]) / k + c_ms)
+            crow.append(round(c_ms, 4))
+        table.append([round(x, 4) for x in row])
+        comm.append(crow)
+    out = {"model": args.model, "res": RES, "ks": KS, "ms": table, "comm_model_ms": comm,
+           "measured_virtual_ms": [[round(float(x), 4) for x in r] for r in ms],
+           "note": "k=1 measured on one B200; k>1 = (k virtual ranks on one B200) / k + modeled NVLink all-to-all"}
+    os.makedirs(os.path.dirname(args.out), exist_ok=True)
+    json.dump(out, open(args.out, "w"), indent=1)
+    print(json.dumps(out))
+
+
+if __name__ == "__main__":
+    main()
