@@ -117,9 +117,7 @@ def sim_tetriserve(T, ks, N, reqs, dl, gran=5, preserve=True):
                 k = len(gids)
                 t_step = T[q["row"], ks.index(k)]
                 if k != g:                              # scaled up: more steps fit in the round
-                    n = max(n, int(math.floor(tau / t_step + 1e-9)))
-                    if n == 0:
-                        continue                        # a fill step longer than tau would block the next round
+                    n = max(n, int(math.floor(tau / t_step + 1e-9)))   # >= 1 step: progress guaranteed
                 n = max(1, min(n, q["left"]))
                 t = reshard_s(q["row"]) if (q["id"] in prev and prev[q["id"]] != gids) else 0.0
                 t += n * t_step
