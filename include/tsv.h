@@ -247,10 +247,30 @@ tsv_status tsv_engine_set_graphs(tsv_engine* eng, int enable);
  *     ranks are on different GPUs (peer access is enabled at engine creation).
  *   TSV_TRANSPORT_EXCHANGE: pack buffer + explicit exchange (peer copies in-process; NCCL
  *     send/recv across processes) + unpack — the baseline, bit-identical results.
- * Groups spanning processes always use NCCL (exchange).  Errors: TSV_E_INVAL. */
+ * Groups spanning processes use NCCL (exchange) unless their members exchanged CUDA-IPC windows
+ * (tsv_group_ipc_export / _import below), then the fused stores go straight into the other
+ * processes' windows and a device-side flag barrier replaces each all-to-all.  Errors: TSV_E_INVAL. */
 #define TSV_TRANSPORT_EXCHANGE 0
 #define TSV_TRANSPORT_FUSED 1
 tsv_status tsv_engine_set_transport(tsv_engine* eng, int mode);
+
+/* Fused transport across processes (one rank per process; S:§8(f) NEXT #2).  Collective over the
+ * group's members, in this order:
+ *   1. every member calls tsv_group_ipc_export: allocates its windows — the attention input
+ *      [max_evals][max_tokens][3][H/k][D] bf16, the activation rows [max_evals][max_tokens/k + 2]
+ *      [h + F] bf16 and 256 barrier flags — and writes an opaque blob (out = NULL: *len = blob
+ *      size); max_tokens >= L_t + L_i of every request the group will run, max_evals >= requests
+ *      per batch x CFG branches (<= 8);
+ *   2. the caller all-gathers the k blobs (e.g. torch.distributed), concatenated in group-rank order;
+ *   3. every member calls tsv_group_ipc_import, which maps the peers' windows (cudaIpcOpenMemHandle).
+ * Afterwards steps on the group (with TSV_TRANSPORT_FUSED) need no NCCL communicator: the QKV and
+ * attention epilogues store into the owners' windows and a device barrier orders the members (a
+ * stalled peer makes the barrier give up after ~10 s instead of hanging).  Groups may then be
+ * created without nccl_id or a world communicator.  Errors: TSV_E_INVAL (sizes, foreign blob),
+ * TSV_E_STATE (import before export), TSV_E_UNSUPPORTED (group not spanning processes), TSV_E_CUDA. */
+tsv_status tsv_group_ipc_export(tsv_engine* eng, tsv_group group, int64_t max_tokens, int max_evals, uint8_t* out,
+                                size_t* len);
+tsv_status tsv_group_ipc_import(tsv_engine* eng, tsv_group group, const uint8_t* blobs, size_t blob_len);
 tsv_status tsv_engine_profile_read(tsv_engine* eng, double* ms, int64_t* launches, double* flops, double* bytes);
 /* Number of kernels this engine launched so far (all slots). */
 tsv_status tsv_engine_kernel_count(tsv_engine* eng, int64_t* count);

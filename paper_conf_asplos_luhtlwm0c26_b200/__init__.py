@@ -102,6 +102,20 @@ class Engine:
         self._groups[ranks] = g.value
         return g.value
 
+    def group_ipc_export(self, group: int, max_tokens: int, max_evals: int = 2) -> bytes:
+        """Step 1 of the cross-process fused transport: this rank's window handles (a blob)."""
+        n = C.c_size_t(0)
+        check(lib.tsv_group_ipc_export(self.h, group, max_tokens, max_evals, None, C.byref(n)))
+        buf = (C.c_uint8 * n.value)()
+        check(lib.tsv_group_ipc_export(self.h, group, max_tokens, max_evals, buf, C.byref(n)))
+        return bytes(buf)
+
+    def group_ipc_import(self, group: int, blobs) -> None:
+        """Step 3: every member's blob, in group-rank order."""
+        joined = b"".join(blobs)
+        arr = (C.c_uint8 * len(joined)).from_buffer_copy(joined)
+        check(lib.tsv_group_ipc_import(self.h, group, arr, len(blobs[0])))
+
     # --------------------------------------------------------------- requests
     def request_create(self, height: int, width: int, num_steps: int = 20, seed: int = 1000,
                        guidance: float = 3.5) -> int:

@@ -56,6 +56,8 @@ _SIGS = {
     "tsv_nccl_unique_id": (_i32, [_P(C.c_uint8)]),
     "tsv_engine_init_world": (_i32, [_p, _P(C.c_uint8)]),
     "tsv_group_create": (_i32, [_p, _P(_i32), _i32, _P(C.c_uint8), _P(C.c_int32)]),
+    "tsv_group_ipc_export": (_i32, [_p, C.c_int32, _i64, _i32, _P(C.c_uint8), _P(C.c_size_t)]),
+    "tsv_group_ipc_import": (_i32, [_p, C.c_int32, _P(C.c_uint8), C.c_size_t]),
     "tsv_request_create": (_i32, [_p, _i32, _i32, _i32, _u64, _f32, _P(_i64)]),
     "tsv_request_set_inputs": (_i32, [_p, _i64, _P(_f32), _P(C.c_uint16), _P(C.c_uint16)]),
     "tsv_request_step": (_i32, [_p, _i64, _i32, C.c_int32, _P(_i64)]),

@@ -331,4 +331,32 @@ void synth_launch(void* dst, uint64_t seed, uint32_t tensor_id, uint64_t idx0, l
   synth_kernel<<<(unsigned)blocks, 256, 0, s>>>(dst, seed, tensor_id, idx0, n, kind, c);
 }
 
+// ------------------------------------------------------------------ cross-process barrier
+__global__ void ipc_barrier_kernel(const __grid_constant__ IpcBarrier b) {
+  grid_dep_wait();
+  int* own = b.flags[b.rank];
+  const int epoch = own[63] + 1;   // this member's barrier count (every member calls the same sequence)
+  own[63] = epoch;
+  __threadfence_system();          // this GPU's earlier peer stores are visible before the flag
+  for (int p = 0; p < b.k; ++p)
+    if (p != b.rank) asm volatile("st.release.sys.global.s32 [%0], %1;" ::"l"(b.flags[p] + b.rank), "r"(epoch) : "memory");
+  for (int p = 0; p < b.k; ++p) {
+    if (p == b.rank) continue;
+    long long spins = 0;
+    for (;;) {
+      int v;
+      asm volatile("ld.acquire.sys.global.s32 %0, [%1];" : "=r"(v) : "l"(own + p) : "memory");
+      if (v >= epoch) break;
+      __nanosleep(200);
+      if (++spins > (1ll << 25)) { own[62] = 1; break; }   // ~10 s: give up rather than hang
+    }
+  }
+  __threadfence_system();
+  grid_dep_launch();
+}
+
+void ipc_barrier_launch(const IpcBarrier& b, cudaStream_t s) {
+  launch_pdl(ipc_barrier_kernel, dim3(1), dim3(1), 0, s, b);
+}
+
 }  // namespace tsv

@@ -180,6 +180,14 @@ struct Group {
   std::vector<int> local_positions;  // group rank of each local member
   ncclComm_t comm = nullptr;         // multi-process transport (one local rank)
   std::vector<cudaEvent_t> ev_a, ev_b;  // per local member, for in-process all-to-all ordering
+  // cross-process fused transport (CUDA IPC windows; tsv_group_ipc_export / _import): this rank's
+  // attention-input and activation windows, mapped into every member, and barrier flags
+  bool ipc = false;
+  int64_t win_tokens = 0;
+  int win_evals = 0;
+  DevBuf win_recv, win_cat, win_flags;
+  std::vector<void*> peer_recv, peer_cat, peer_flags;  // by group rank (own entry = own window)
+  std::vector<void*> opened;                           // IPC mappings to close
 };
 
 struct Request {
@@ -552,6 +560,9 @@ struct StepEnv {
   std::vector<RankCtx> rc;
   // global layout for the all-to-alls
   std::vector<int64_t> t_off, t_cnt, i_off, i_cnt;  // per group rank
+  // fused transport: every member's attention input and activation buffer, by group rank
+  std::vector<bf16*> recv_of, cat_of;
+  bool ipc = false;       // members in other processes (CUDA IPC windows, device barrier)
 };
 
 // ------------------------------------------------------------------ Ulysses all-to-alls (a5, a7)
@@ -656,6 +667,16 @@ static tsv_status a2a_exec(StepEnv& E, int which) {
 static tsv_status group_sync(StepEnv& E) {
   Group& g = *E.g;
   const int k = g.k;
+  if (E.ipc) {
+    // members in other processes: a device-side barrier over the IPC flag windows
+    ProfScope ps(E.e, *E.rc[0].s, KC_A2A, 0.0, 0.0, 1);
+    IpcBarrier b;
+    b.k = k;
+    b.rank = g.local_positions[0];
+    for (int d = 0; d < k; ++d) b.flags[d] = reinterpret_cast<int*>(g.peer_flags[d]);
+    ipc_barrier_launch(b, E.rc[0].s->stream);
+    return TSV_OK;
+  }
   ProfScope ps(E.e, *E.rc[0].s, KC_A2A, 0.0, 0.0, 0);
   for (int r = 0; r < k; ++r) {
     CK(cudaSetDevice(E.rc[r].s->device));
@@ -678,7 +699,7 @@ static void peer_epi(StepEnv& E, RankCtx& c, GemmEpi& epi, int b, int kind) {
   const int k = E.g->k;
   const int64_t L = E.R->Lt + E.R->Li, w = 3 * (int64_t)m.h / k;
   const int r = c.sh->rank_in_group;
-  for (int d = 0; d < k; ++d) epi.peer[d] = E.rc[d].recv + b * L * w;
+  for (int d = 0; d < k; ++d) epi.peer[d] = E.recv_of[d] + b * L * w;
   const int tg = (int)E.t_off[r], ig = (int)(E.R->Lt + E.i_off[r]);
   epi.peer_nt = 1 << 30;
   if (kind == 0) epi.peer_row0 = tg;
@@ -732,10 +753,10 @@ static tsv_status attention_all(StepEnv& E) {
         sc.col0 = c.sh->rank_in_group * (m.h / k);
         sc.ld = m.h + m.F;
         for (int p = 0; p < k; ++p) {
-          sc.dst[p] = E.rc[p].cat + b * E.rc[p].rows * (m.h + m.F);
+          sc.dst[p] = E.cat_of[p] + b * (E.t_cnt[p] + E.i_cnt[p]) * (m.h + m.F);
           sc.t_off[p] = (int)E.t_off[p];
           sc.i_off[p] = (int)E.i_off[p];
-          sc.nt[p] = (int)E.rc[p].nt;
+          sc.nt[p] = (int)E.t_cnt[p];
         }
         sc.t_off[k] = (int)E.R->Lt;
         sc.i_off[k] = (int)E.R->Li;
@@ -1216,7 +1237,13 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
   StepEnv E;
   E.e = e; E.R = &R0; E.Rq = Rs; E.g = &g;
   E.B = (int)Rs.size() * m.B;
-  E.fused = e->transport == TSV_TRANSPORT_FUSED && g.all_local && g.k > 1;
+  E.fused = e->transport == TSV_TRANSPORT_FUSED && (g.all_local || g.ipc) && g.k > 1;
+  E.ipc = E.fused && !g.all_local;
+  if (!g.all_local && !g.comm && !E.ipc)
+    return fail(TSV_E_STATE, "group spans processes without NCCL: exchange IPC windows first (tsv_group_ipc_export/import)");
+  if (E.ipc && (R0.Lt + R0.Li > g.win_tokens || E.B > g.win_evals))
+    return fail(TSV_E_INVAL, "step (L = %lld, %d evaluations) exceeds the group's IPC windows (%lld, %d)",
+                (long long)(R0.Lt + R0.Li), E.B, (long long)g.win_tokens, g.win_evals);
   const int k = g.k;
   E.t_off.resize(k); E.t_cnt.resize(k); E.i_off.resize(k); E.i_cnt.resize(k);
   for (int r = 0; r < k; ++r) {
@@ -1246,7 +1273,17 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
     c.obuf = reinterpret_cast<bf16*>(s.ws.obuf.p);
     c.orecv = reinterpret_cast<bf16*>(s.ws.orecv.p);
     c.mod = reinterpret_cast<float*>(s.ws.bmod.p);
+    if (E.ipc) {  // the attention input and activation rows live in the group's shared windows
+      c.recv = reinterpret_cast<bf16*>(g.win_recv.p);
+      c.cat = reinterpret_cast<bf16*>(g.win_cat.p);
+    }
     E.rc.push_back(c);
+  }
+  if (E.fused) {
+    for (int d = 0; d < k; ++d) {
+      E.recv_of.push_back(E.ipc ? reinterpret_cast<bf16*>(g.peer_recv[d]) : E.rc[d].recv);
+      E.cat_of.push_back(E.ipc ? reinterpret_cast<bf16*>(g.peer_cat[d]) : E.rc[d].cat);
+    }
   }
   // each slot's stream must follow every request's previous work on that slot; then publish the
   // step indices (pageable source: staged at call time, so the host value can change right after)
@@ -1460,6 +1497,8 @@ void tsv_engine_destroy(tsv_engine* e) {
     for (auto& l : kv.second.last) cudaEventDestroy(l.second);
   }
   for (auto& g : e->groups) {
+    for (void* p : g.opened) cudaIpcCloseMemHandle(p);
+    g.win_recv.release(); g.win_cat.release(); g.win_flags.release();
     if (g.comm) ncclCommDestroy(g.comm);
     for (auto ev : g.ev_a) cudaEventDestroy(ev);
     for (auto ev : g.ev_b) cudaEventDestroy(ev);
@@ -1526,10 +1565,12 @@ tsv_status tsv_group_create(tsv_engine* e, const int* ranks, int k, const uint8_
       ncclUniqueId id;
       memcpy(&id, nccl_id, 128);
       NK(ncclCommInitRank(&g.comm, k, id, g.local_positions[0]));
-    } else {
-      if (!e->world_comm) return fail(TSV_E_STATE, "group across processes needs nccl_id or init_world");
+    } else if (e->world_comm) {
       NK(ncclCommSplit(e->world_comm, 1, g.local_positions[0], &g.comm, nullptr));
     }
+  }
+  if (!g.all_local && g.comm) {
+    Slot& s = e->slots[g.local_slots[0]];
     // warm the communicator once
     DevBuf tmp;
     TRY(dev_alloc(tmp, s.device, 256 * k));
@@ -1559,6 +1600,90 @@ tsv_status tsv_group_create(tsv_engine* e, const int* ranks, int k, const uint8_
   }
   e->groups.push_back(std::move(g));
   *out = (tsv_group)e->groups.size() - 1;
+  return TSV_OK;
+}
+
+// ------------------------------------------------------------------ cross-process fused transport
+namespace {
+struct IpcBlob {
+  uint32_t magic;
+  int32_t rank;
+  int64_t tokens;
+  int32_t evals;
+  int32_t pad;
+  cudaIpcMemHandle_t recv, cat, flags;
+};
+}  // namespace
+
+tsv_status tsv_group_ipc_export(tsv_engine* e, tsv_group gi, int64_t max_tokens, int max_evals, uint8_t* out,
+                                size_t* len) {
+  if (!e || !len) return fail(TSV_E_INVAL, "null argument");
+  if (gi < 0 || gi >= (int)e->groups.size()) return fail(TSV_E_INVAL, "unknown group %d", gi);
+  Group& g = e->groups[gi];
+  if (g.all_local || g.local_slots.size() != 1) return fail(TSV_E_UNSUPPORTED, "IPC windows are for groups spanning processes with one local rank");
+  if (max_tokens <= 0 || max_evals < 1 || max_evals > GEMM_MAX_PROBLEMS / 2) return fail(TSV_E_INVAL, "bad window size");
+  if (!out) { *len = sizeof(IpcBlob); return TSV_OK; }
+  if (*len < sizeof(IpcBlob)) return fail(TSV_E_INVAL, "blob buffer too small (%zu bytes)", sizeof(IpcBlob));
+  const Model& m = e->model;
+  const int k = g.k;
+  Slot& s = e->slots[g.local_slots[0]];
+  const int64_t rows_max = max_tokens / k + 2;
+  TRY(dev_alloc(g.win_recv, s.device, (size_t)max_evals * max_tokens * 3 * (m.h / k) * 2));
+  TRY(dev_alloc(g.win_cat, s.device, (size_t)max_evals * rows_max * (m.h + m.F) * 2));
+  TRY(dev_alloc(g.win_flags, s.device, 256 * sizeof(int)));
+  CK(cudaSetDevice(s.device));
+  CK(cudaMemset(g.win_flags.p, 0, 256 * sizeof(int)));
+  CK(cudaDeviceSynchronize());
+  IpcBlob b{};
+  b.magic = 0x7E7151C0u;
+  b.rank = g.local_positions[0];
+  b.tokens = max_tokens;
+  b.evals = max_evals;
+  CK(cudaIpcGetMemHandle(&b.recv, g.win_recv.p));
+  CK(cudaIpcGetMemHandle(&b.cat, g.win_cat.p));
+  CK(cudaIpcGetMemHandle(&b.flags, g.win_flags.p));
+  memcpy(out, &b, sizeof b);
+  *len = sizeof b;
+  g.win_tokens = max_tokens;
+  g.win_evals = max_evals;
+  return TSV_OK;
+}
+
+tsv_status tsv_group_ipc_import(tsv_engine* e, tsv_group gi, const uint8_t* blobs, size_t blob_len) {
+  if (!e || !blobs) return fail(TSV_E_INVAL, "null argument");
+  if (gi < 0 || gi >= (int)e->groups.size()) return fail(TSV_E_INVAL, "unknown group %d", gi);
+  Group& g = e->groups[gi];
+  if (!g.win_recv.p) return fail(TSV_E_STATE, "export this rank's windows first");
+  if (blob_len != sizeof(IpcBlob)) return fail(TSV_E_INVAL, "blob length %zu, expected %zu", blob_len, sizeof(IpcBlob));
+  const int k = g.k, me = g.local_positions[0];
+  Slot& s = e->slots[g.local_slots[0]];
+  CK(cudaSetDevice(s.device));
+  g.peer_recv.assign(k, nullptr);
+  g.peer_cat.assign(k, nullptr);
+  g.peer_flags.assign(k, nullptr);
+  for (int d = 0; d < k; ++d) {
+    IpcBlob b;
+    memcpy(&b, blobs + (size_t)d * sizeof(IpcBlob), sizeof b);
+    if (b.magic != 0x7E7151C0u || b.rank != d) return fail(TSV_E_INVAL, "blob %d is not group rank %d's", d, d);
+    if (b.tokens != g.win_tokens || b.evals != g.win_evals) return fail(TSV_E_INVAL, "members exported different window sizes");
+    if (d == me) {
+      g.peer_recv[d] = g.win_recv.p;
+      g.peer_cat[d] = g.win_cat.p;
+      g.peer_flags[d] = g.win_flags.p;
+      continue;
+    }
+    void* pr = nullptr;
+    void* pc = nullptr;
+    void* pf = nullptr;
+    CK(cudaIpcOpenMemHandle(&pr, b.recv, cudaIpcMemLazyEnablePeerAccess));
+    CK(cudaIpcOpenMemHandle(&pc, b.cat, cudaIpcMemLazyEnablePeerAccess));
+    CK(cudaIpcOpenMemHandle(&pf, b.flags, cudaIpcMemLazyEnablePeerAccess));
+    g.opened.insert(g.opened.end(), {pr, pc, pf});
+    g.peer_recv[d] = pr;
+    g.peer_cat[d] = pc;
+    g.peer_flags[d] = pf;
+  }
+  g.ipc = true;
   return TSV_OK;
 }
 

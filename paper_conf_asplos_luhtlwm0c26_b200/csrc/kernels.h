@@ -169,6 +169,17 @@ void copy2d_bf16_launch(const bf16* src, long long lds, bf16* dst, long long ldd
 void select_row_launch(const float* src, long long stride, const int* idx_dev, float* dst, long long n,
                        cudaStream_t s);
 
+// Cross-process group barrier over CUDA-IPC flag windows (fused transport, one rank per process):
+// member r bumps its epoch, stores it into every peer's flags[r] (release, system scope) and waits
+// until every peer's epoch has arrived in its own flags (acquire).  Bounded wait: after ~10 s it
+// records an error flag (flags[rank][62]) and returns instead of hanging.
+struct IpcBarrier {
+  int* flags[8];
+  int k = 0;
+  int rank = 0;
+};
+void ipc_barrier_launch(const IpcBarrier& b, cudaStream_t s);
+
 // ------------------------------------------------------------------ SYNTH-1 generator
 // kind: 0 'w'/'b'/'x' (bf16 = rne(r*c)), 1 'g' (bf16 = rne(1 + r*c)), 2 'f' (fp32 = r*c)
 void synth_launch(void* dst, uint64_t seed, uint32_t tensor_id, uint64_t idx0, long long n, int kind, float c,

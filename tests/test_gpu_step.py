@@ -215,3 +215,44 @@ def test_fused_transport_bitwise_equals_exchange(tsv, model, res, k):
         out.append((eng.read_latent(req), eng.read_velocity(req)))
         eng.close()
     assert np.array_equal(out[0][0], out[1][0]) and np.array_equal(out[0][1], out[1][1])
+
+
+def test_config3_flux1024_sp_degrees_agree(tsv):
+    """BASELINE config 3 at full FLUX size: one 1024^2 step at SP = 1, 2, 4, 8 (virtual ranks on one
+    GPU, fused transport) — the SP invariance property (S:§8(c) P9) at the bench's shapes."""
+    eng = tsv.Engine("flux", devices=[0] * 8)
+    outs = {}
+    for k in (1, 2, 4, 8):
+        g = eng.group_create(list(range(k)))
+        r = eng.request_create(1024, 1024, num_steps=20, seed=1400)
+        eng.event_wait(eng.request_step(r, 0, g))
+        outs[k] = (eng.read_latent(r).astype(np.float64), eng.read_velocity(r).astype(np.float64))
+        eng.request_destroy(r)
+    for k in (2, 4, 8):
+        for a, b in zip(outs[k], outs[1]):
+            rel, cos = _metrics(a, b)
+            assert rel <= 1e-2 and cos >= 0.9999, (k, rel, cos)
+    eng.close()
+
+
+def test_config4_flux2048_step_level_sp_schedule(tsv):
+    """BASELINE config 4 at full FLUX size: a 2048^2 request running steps 0-4 at k = 2 on [0,1],
+    5-9 at k = 8, 10-14 at k = 4 on [4..7], 15-19 at k = 2 on [2,3]; every reshard is a bit-exact
+    move and the 20-step trajectory matches an all-k=1 run of the same seed."""
+    eng = tsv.Engine("flux", devices=[0] * 8)
+    plan = [[0, 1], list(range(8)), [4, 5, 6, 7], [2, 3]]
+    groups = [eng.group_create(p) for p in plan]
+    g1 = eng.group_create([0])
+    ra = eng.request_create(2048, 2048, num_steps=20, seed=1500)
+    rb = eng.request_create(2048, 2048, num_steps=20, seed=1500)
+    for s in range(20):
+        g = groups[s // 5]
+        if s % 5 == 0 and s > 0:
+            before = eng.read_latent(ra)
+            eng.event_wait(eng.request_reshard(ra, g))
+            assert np.array_equal(before, eng.read_latent(ra))
+        eng.request_step(ra, s, g)
+        eng.request_step(rb, s, g1)
+    rel, cos = _metrics(eng.read_latent(ra).astype(np.float64), eng.read_latent(rb).astype(np.float64))
+    assert rel <= 1e-2 and cos >= 0.9999, (rel, cos)
+    eng.close()
