@@ -48,9 +48,12 @@ tsv_status tsv_op_gemm_qkv(const void* A, int64_t lda, const void* W, int64_t ld
                            const void* gq, const void* gk, const float* cosb, const float* sinb, int k_sp,
                            void* pack, int pack_rows, int pack_row0, void* stream);
 
-/* a2: u[m, :] = bf16(LN(x[m, :]) * (1 + scale) + shift); x fp32, LN without affine, eps 1e-6. */
+/* a2: u[m, :] = bf16(LN(x[m, :]) * (1 + scale) + shift); x fp32, LN without affine, eps 1e-6.
+ * impl 0: one CTA per row (block reductions); impl 1: one warp per row (h in {1536, 3072}; other h
+ * fall back to impl 0).  The engine uses the one tsv_engine's default selects (impl 0 unless
+ * measured otherwise).  Errors: TSV_E_INVAL (h % 128, impl). */
 tsv_status tsv_op_ln_mod(const float* x, int64_t ldx, void* u, int64_t ldu, const float* shift,
-                         const float* scale, int M, int h, void* stream);
+                         const float* scale, int M, int h, int impl, void* stream);
 
 /* a4: on qkv bf16 [rows, 3*H*D] (columns "(K H D)"), q and k of every head become
  * RoPE(RMSNorm(x) * g) (eps 1e-6; pair (2j, 2j+1) rotated by the per-row table angle j).

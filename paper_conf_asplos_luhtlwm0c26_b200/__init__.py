@@ -266,9 +266,9 @@ def op_gemm_qkv(A, W, out0, h, D, gq, gk, cosb, sinb, bias=None, mode="STORE_BF1
                               pack_rows, pack_row0, _stream(stream)))
 
 
-def op_ln_mod(x, u, shift, scale, stream=None):
+def op_ln_mod(x, u, shift, scale, impl=0, stream=None):
     M, h = x.shape
-    check(lib.tsv_op_ln_mod(_ptr(x), x.stride(0), _ptr(u), u.stride(0), _ptr(shift), _ptr(scale), M, h,
+    check(lib.tsv_op_ln_mod(_ptr(x), x.stride(0), _ptr(u), u.stride(0), _ptr(shift), _ptr(scale), M, h, impl,
                             _stream(stream)))
 
 

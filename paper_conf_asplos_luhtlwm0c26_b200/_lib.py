@@ -86,7 +86,7 @@ _SIGS = {
                             _p]),
     "tsv_op_gemm_qkv": (_i32, [_p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p, _i64, _p, _i64, _p, _i32, _i32,
                                _p, _p, _p, _p, _i32, _p, _i32, _i32, _p]),
-    "tsv_op_ln_mod":(_i32, [_p, _i64, _p, _i64, _p, _p, _i32, _i32, _p]),
+    "tsv_op_ln_mod": (_i32, [_p, _i64, _p, _i64, _p, _p, _i32, _i32, _i32, _p]),
     "tsv_op_qk_norm_rope": (_i32, [_p, _i64, _i32, _i32, _i32, _i32, _p, _p, _p, _p, _p, _p, _p, _i32, _p]),
     "tsv_op_attention": (_i32, [_p, _i64, _p, _i64, _p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p]),
     "tsv_op_synth": (_i32, [_p, _u64, C.c_uint32, _u64, _i64, _i32, _f32, _p]),

@@ -75,6 +75,60 @@ __global__ void __launch_bounds__(T) ln_mod_kernel(const float* __restrict__ x, 
   }
 }
 
+// Warp per row (8 rows per 256-thread CTA): the row stays in registers (NV float4 per lane), both
+// reductions are warp shuffles (no block barriers), the modulation vectors come through L1 (shared
+// by every row of a stream).  Rows [0, n_first) of each block of rows_b take (shift0, scale0).
+template <int NV>
+__global__ void __launch_bounds__(256) ln_mod_warp_kernel(const float* __restrict__ x, long long ldx,
+                                                          bf16* __restrict__ u, long long ldu,
+                                                          const float* __restrict__ shift0,
+                                                          const float* __restrict__ scale0,
+                                                          const float* __restrict__ shift1,
+                                                          const float* __restrict__ scale1, int n_first, int rows_b,
+                                                          long long mstride, int M) {
+  const int row = blockIdx.x * 8 + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  grid_dep_wait();
+  if (row >= M) return;
+  const int b = row / rows_b, r = row - b * rows_b;
+  const float* shift = (r < n_first ? shift0 : shift1) + b * mstride;
+  const float* scale = (r < n_first ? scale0 : scale1) + b * mstride;
+  constexpr int h = 128 * NV;
+  const float4* xr = reinterpret_cast<const float4*>(x + (long long)row * ldx);
+  float4 v[NV];
+#pragma unroll
+  for (int i = 0; i < NV; ++i) v[i] = xr[i * 32 + lane];
+  float sm = 0.f;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) sm += (v[i].x + v[i].y) + (v[i].z + v[i].w);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) sm += __shfl_xor_sync(0xffffffffu, sm, o);
+  const float mean = sm * (1.0f / h);
+  float q = 0.f;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const float a = v[i].x - mean, bb = v[i].y - mean, c = v[i].z - mean, d = v[i].w - mean;
+    q += (a * a + bb * bb) + (c * c + d * d);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
+  const float rstd = rsqrtf(q * (1.0f / h) + 1e-6f);
+  uint2* ur = reinterpret_cast<uint2*>(u + (long long)row * ldu);
+  const float4* shp = reinterpret_cast<const float4*>(shift);
+  const float4* scp = reinterpret_cast<const float4*>(scale);
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const int c = i * 32 + lane;
+    const float4 sh = __ldg(shp + c), sc = __ldg(scp + c);
+    const float a = (v[i].x - mean) * rstd * (1.f + sc.x) + sh.x;
+    const float bb = (v[i].y - mean) * rstd * (1.f + sc.y) + sh.y;
+    const float cc = (v[i].z - mean) * rstd * (1.f + sc.z) + sh.z;
+    const float d = (v[i].w - mean) * rstd * (1.f + sc.w) + sh.w;
+    ur[c] = make_uint2(pack_bf16x2(a, bb), pack_bf16x2(cc, d));
+  }
+  grid_dep_launch();
+}
+
 // generic fallback (h multiple of 128): two passes over global memory
 __global__ void __launch_bounds__(256) ln_mod_generic(const float* __restrict__ x, long long ldx, bf16* __restrict__ u,
                                                       long long ldu, const float* __restrict__ shift0,
@@ -103,11 +157,23 @@ __global__ void __launch_bounds__(256) ln_mod_generic(const float* __restrict__ 
     u[(long long)row * ldu + c] = __float2bfloat16_rn((xr[c] - mean) * rstd * (1.f + scale[c]) + shift[c]);
 }
 
+int g_ln_impl = 0;   // 0: CTA per row, 1: warp per row (tsv_op_ln_mod impl; microbench sweeps)
+
 void ln_mod2b_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift0,
                      const float* scale0, const float* shift1, const float* scale1, int n_first, int rows_b, int B,
                      long long mstride, int h, cudaStream_t s) {
   const int M = rows_b * B;
   if (M <= 0) return;
+  if (g_ln_impl == 1 && (h == 3072 || h == 1536)) {
+    const dim3 grid((M + 7) / 8);
+    if (h == 3072)
+      launch_pdl(ln_mod_warp_kernel<24>, grid, dim3(256), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first,
+                 rows_b, mstride, M);
+    else
+      launch_pdl(ln_mod_warp_kernel<12>, grid, dim3(256), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first,
+                 rows_b, mstride, M);
+    return;
+  }
   switch (h) {
     case 3072:
       launch_pdl(ln_mod_kernel<256, 3>, dim3(M), dim3(256), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first,

@@ -2118,9 +2118,13 @@ tsv_status tsv_op_gemm_qkv(const void* A, int64_t lda, const void* Wt, int64_t l
 }
 
 tsv_status tsv_op_ln_mod(const float* x, int64_t ldx, void* u, int64_t ldu, const float* shift, const float* scale,
-                         int M, int h, void* stream) {
+                         int M, int h, int impl, void* stream) {
   if (h % 128) return fail(TSV_E_INVAL, "h must be a multiple of 128");
+  if (impl < 0 || impl > 1) return fail(TSV_E_INVAL, "bad impl %d", impl);
+  const int keep = g_ln_impl;
+  g_ln_impl = impl;
   ln_mod_launch(x, ldx, reinterpret_cast<bf16*>(u), ldu, shift, scale, M, h, reinterpret_cast<cudaStream_t>(stream));
+  g_ln_impl = keep;
   CK(cudaGetLastError());
   return TSV_OK;
 }

@@ -134,6 +134,7 @@ void ln_mod2_launch(const float* x, long long ldx, bf16* u, long long ldu, const
                     const float* scale0, const float* shift1, const float* scale1, int n_first, int M, int h,
                     cudaStream_t s);
 
+extern int g_ln_impl;  // LN-modulate kernel choice: 0 CTA per row, 1 warp per row
 // B blocks of rows_b rows (block b = rows [b*rows_b, (b+1)*rows_b)); inside a block rows [0, n_first)
 // use (shift0, scale0), the rest (shift1, scale1); block b's vectors are offset by b * mstride floats.
 void ln_mod2b_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift0,

@@ -155,14 +155,15 @@ def test_gemm_rejects_bad_shapes(tsv):
 
 
 # ----------------------------------------------------------------------------- LN-modulate
-@pytest.mark.parametrize("M,h", [(1, 256), (333, 256), (1536, 3072), (77, 1536), (5, 640)])
-def test_ln_mod(tsv, M, h):
+@pytest.mark.parametrize("impl", [0, 1])
+@pytest.mark.parametrize("M,h", [(1, 256), (333, 256), (1536, 3072), (77, 1536), (5, 640), (13, 3072)])
+def test_ln_mod(tsv, M, h, impl):
     rng = np.random.default_rng(M + h)
     x = (rng.standard_normal((M, h)) * 3 + 0.5).astype(np.float32)
     sh = rng.standard_normal(h).astype(np.float32)
     sc = rng.standard_normal(h).astype(np.float32)
     u = torch.zeros(M, h, dtype=torch.bfloat16, device="cuda")
-    tsv.op_ln_mod(_f32(x), u, _f32(sh), _f32(sc))
+    tsv.op_ln_mod(_f32(x), u, _f32(sh), _f32(sc), impl=impl)
     torch.cuda.synchronize()
     ref = F.ln_modulate(x.astype(np.float64), sh, sc)
     err = np.abs(_np(u) - ref)

@@ -65,13 +65,14 @@ def attn_cases():
 
 
 def ln_cases():
-    for M, h in ((1024, 3072), (1536, 3072), (16896, 3072)):
+    for M, h in ((1024, 3072), (1536, 3072), (16896, 3072), (2714, 1536), (8858, 1536)):
         x = torch.randn(M, h, device="cuda")
         u = torch.empty(M, h, dtype=torch.bfloat16, device="cuda")
         sh, sc = torch.randn(h, device="cuda"), torch.randn(h, device="cuda")
-        ms = timeit(lambda: tsv.op_ln_mod(x, u, sh, sc))
-        print(json.dumps({"op": "ln_mod", "M": M, "h": h, "ms": round(ms, 4),
-                          "GBps": round(M * h * 6 / ms / 1e6, 1)}), flush=True)
+        for impl in (0, 1):
+            ms = timeit(lambda: tsv.op_ln_mod(x, u, sh, sc, impl=impl))
+            print(json.dumps({"op": "ln_mod", "impl": ["cta_per_row", "warp_per_row"][impl], "M": M, "h": h,
+                              "ms": round(ms, 4), "GBps": round(M * h * 6 / ms / 1e6, 1)}), flush=True)
 
 
 def qk_cases():
