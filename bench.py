@@ -263,8 +263,25 @@ def run_ours(args):
         dist.broadcast_object_list(obj, src=0)
         eng.init_world(obj[0])
         g = eng.group_create(list(range(world)), nccl_id=obj[1])
+        transport = "nccl-exchange"
+        if args.transport == "fused":
+            # the product path: all-to-alls fused into the epilogues as stores into the other
+            # processes' CUDA-IPC windows (tsv_group_ipc_export / _import); NCCL stays the fallback
+            try:
+                blob = eng.group_ipc_export(g, max_tokens=(args.res // 16) ** 2 + mdl["Lt"], max_evals=2)
+                blobs = [None] * world
+                dist.all_gather_object(blobs, blob)
+                eng.group_ipc_import(g, blobs)
+                eng.set_transport(True)
+                transport = "fused-ipc"
+            except tsv.TsvError as ex:
+                print(f"[bench] fused IPC transport unavailable ({ex}); using NCCL", file=sys.stderr)
+                eng.set_transport(False)
+        else:
+            eng.set_transport(False)
     else:
         g = eng.group_create([0])
+        transport = "none"
     res = args.res
     K, Wm = args.steps, args.warmup
     total_steps = Wm + K + Wm + K + 2 + 2   # timed + profiled + e2e passes
@@ -346,7 +363,7 @@ def run_ours(args):
             "dtype": "bf16", "data": f"synthetic (SYNTH-1 seeded weights and inputs, {mdl['shapes']})",
             "config": {"workload": f"{mdl['desc']} {res}x{res} ({Li} image + {mdl['Lt']} text tokens)",
                        "sp": world, "resolution": res, "global_batch": 1, "seq_len": Li + mdl["Lt"],
-                       "parallelism": f"ulysses-sp{world}",
+                       "parallelism": f"ulysses-sp{world}", "transport": transport,
                        "l2": f"inputs larger than L2 ({mdl['weights_gb']} GB of weights streamed per step); no flush"},
             "roofline": {"bound": "tensor",
                          "kernel": "gemm_tc2_kernel / gemm_tc_kernel (tcgen05 GEMM, all GEMM launches of the step)",
@@ -383,6 +400,9 @@ def main():
     ap.add_argument("--res", type=int, default=512)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--model", default="flux", choices=sorted(MODELS))
+    ap.add_argument("--transport", default="fused", choices=["fused", "nccl"],
+                    help="N > 1: Ulysses all-to-alls fused into the epilogues over CUDA-IPC peer memory (default) "
+                         "or NCCL send/recv")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":

@@ -92,18 +92,39 @@ __device__ __forceinline__ void store_bf16x32(bf16* ob, const float (&v)[32]) {
   }
 }
 
-// destination of qkv column n (in [0, 3h)) of GEMM row `row` (plain [M, ld0] or Ulysses pack)
-__device__ __forceinline__ bf16* qkv_dst(const GemmEpi& e, int row, int n) {
-  if (e.k_sp <= 1) return reinterpret_cast<bf16*>(e.out0) + (long long)row * e.ld0 + n;
+// Destination of one head block (columns [col0, col0 + D), head-aligned) of the QKV output:
+// element (row, d) goes to base + rowmap(row) * stride + d.  Plain [M, ld0]; Ulysses pack
+// [k][pack_rows][3][H/k][D]; or (fused a5) the owner's [L][3][H/k][D] at the row's global position.
+// Computed once per head so the store loop has no integer divisions.
+struct QkvDst {
+  bf16* base;
+  long long stride;
+  int nt;             // rows < nt map to r0 + row, the rest to r1 + row - nt
+  long long r0, r1;
+  __device__ __forceinline__ bf16* at(int row) const {
+    return base + (row < nt ? r0 + row : r1 + (row - nt)) * stride;
+  }
+};
+__device__ __forceinline__ QkvDst qkv_head_dst(const GemmEpi& e, int col0) {
+  QkvDst q;
+  if (e.k_sp <= 1) {
+    q.base = reinterpret_cast<bf16*>(e.out0) + col0;
+    q.stride = e.ld0; q.nt = 1 << 30; q.r0 = 0; q.r1 = 0;
+    return q;
+  }
   const int h = e.qk_h, D = e.qk_D;
-  const int part = n / h, hd = (n - part * h) / D, d = n % D;
+  const int part = col0 / h, hd = (col0 - part * h) / D;
   const int hk = h / D / e.k_sp;
   const int dst = hd / hk, hl = hd - dst * hk;
+  q.stride = 3LL * hk * D;
   if (e.peer[0]) {
-    const long long g = row < e.peer_nt ? (long long)e.peer_row0 + row : (long long)e.peer_row1 + (row - e.peer_nt);
-    return e.peer[dst] + ((g * 3 + part) * hk + hl) * D + d;
+    q.base = e.peer[dst] + ((long long)part * hk + hl) * D;
+    q.nt = e.peer_nt; q.r0 = e.peer_row0; q.r1 = e.peer_row1;
+  } else {
+    q.base = e.pack + ((long long)dst * e.pack_rows + e.pack_row0) * q.stride + ((long long)part * hk + hl) * D;
+    q.nt = 1 << 30; q.r0 = 0; q.r1 = 0;
   }
-  return e.pack + ((((long long)dst * e.pack_rows + e.pack_row0 + row) * 3 + part) * hk + hl) * D + d;
+  return q;
 }
 
 // ------------------------------------------------------------------ epilogue (coalesced via smem)
@@ -153,6 +174,7 @@ __device__ __forceinline__ void epilogue_qk_head(const GemmEpi& e, int M, int ro
     rn = rsqrtf(ss / (float)D + 1e-6f);
   }
   const bf16* g = col0 < e.qk_h ? e.gq : e.gk;
+  const QkvDst qd = qkv_head_dst(e, col0);
   for (int c = 0; c < D / 32; ++c) {
     uint32_t r[32];
     tmem_ld32(tcol + c * 32, r);
@@ -188,7 +210,7 @@ __device__ __forceinline__ void epilogue_qk_head(const GemmEpi& e, int M, int ro
     for (int it = 0; it < 8; ++it) {
       const int rr = it * 4 + (lane >> 3);
       if (row0 + rr < M)
-        *reinterpret_cast<uint2*>(qkv_dst(e, row0 + rr, col0 + c * 32 + c4 * 4)) = pack4_bf16(stage_read(stg, rr, c4));
+        *reinterpret_cast<uint2*>(qd.at(row0 + rr) + c * 32 + c4 * 4) = pack4_bf16(stage_read(stg, rr, c4));
     }
     __syncwarp();
   }

@@ -47,6 +47,23 @@ def gemm_cases():
                           "tflops": round(2 * M * N * K / ref / 1e9, 1)}), flush=True)
 
 
+def qkv_epilogue_cases():
+    """QKV GEMM: plain bf16 store vs the fused QK-RMSNorm + RoPE epilogue (a4) at FLUX shapes."""
+    for M in (1536, 16896):
+        N, K, h, D = 9216, 3072, 3072, 128
+        A = torch.randn(M, K, device="cuda").to(torch.bfloat16)
+        W = (torch.randn(N, K, device="cuda") / math.sqrt(K)).to(torch.bfloat16)
+        o = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
+        g = torch.ones(D, dtype=torch.bfloat16, device="cuda")
+        cs = torch.ones(M, D // 2, device="cuda")
+        sn = torch.zeros(M, D // 2, device="cuda")
+        plain = timeit(lambda: tsv.op_gemm(A, W, "STORE_BF16", o))
+        fused = timeit(lambda: tsv.op_gemm_qkv(A, W, o, h, D, g, g, cs, sn))
+        print(json.dumps({"op": "qkv_gemm", "M": M, "plain_ms": round(plain, 4), "fused_ms": round(fused, 4),
+                          "plain_tflops": round(2 * M * N * K / plain / 1e9, 1),
+                          "fused_tflops": round(2 * M * N * K / fused / 1e9, 1)}), flush=True)
+
+
 def attn_cases():
     sweep = os.environ.get("ATTN_SWEEP")     # "1": also time the poly-share variants (impl 12..15)
     for L, H, D in ((1536, 24, 128), (4608, 24, 128), (16896, 24, 128), (16896, 3, 128), (1357, 24, 64),
@@ -88,4 +105,4 @@ def qk_cases():
 if __name__ == "__main__":
     which = sys.argv[1:] or ["gemm", "attn", "ln", "qk"]
     for w in which:
-        {"gemm": gemm_cases, "attn": attn_cases, "ln": ln_cases, "qk": qk_cases}[w]()
+        {"gemm": gemm_cases, "attn": attn_cases, "ln": ln_cases, "qk": qk_cases, "qkv": qkv_epilogue_cases}[w]()
