@@ -443,19 +443,21 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
 // tcgen05.mma.cta_group::2 (M = 256, N = 256), which reads A and B from both CTAs' shared memory
 // at the same offsets and leaves CTA r's 128 output rows in CTA r's TMEM.  Per SM this halves the
 // operand bytes read from shared memory per MMA compared with the 1-CTA 128 x 256 tile.
+template <int BN_>
 struct Gemm2Cfg {
-  static constexpr int BN = 256;
+  static constexpr int BN = BN_;
   static constexpr int A_BYTES = 128 * BK * 2;
   static constexpr int B_BYTES = (BN / 2) * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES = 6;
+  static constexpr int STAGES = BN == 256 ? 6 : 8;
   static constexpr int TMEM_COLS = 2 * BN;
   static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + 4 * 32 * 36 * 4;
 };
 
+template <int BN_>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
     gemm_tc2_kernel(const __grid_constant__ GemmMaps maps, const __grid_constant__ GemmArgs args) {
-  using C = Gemm2Cfg;
+  using C = Gemm2Cfg<BN_>;
   constexpr int BN = C::BN;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -665,7 +667,7 @@ int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int
   long long pair_tiles = 0;
   for (int q = 0; q < nprob; ++q) pair_tiles += (long long)((probs[q].M + 255) / 256) * (N / 256);
   const bool pair_auto = bn == 256 && maxM > 128 && (K >= 8192 || pair_tiles * 2 >= (long long)num_sms * 9 / 10);
-  const bool pair = force_pair >= 0 ? (force_pair > 0 && bn == 256) : pair_auto;
+  const bool pair = force_pair >= 0 ? (force_pair > 0 && bn >= 128) : pair_auto;
   const int bm = pair ? 256 : BM;
   p->nprob = nprob; p->N = N; p->K = K; p->BN = bn; p->pair = pair;
   int tiles = 0;
@@ -722,13 +724,15 @@ static void launch_bn(const GemmPlan& p, cudaStream_t s) {
     maps.A[q] = p.tmAq[qq];
     maps.B[q] = p.tmBq[qq];
   }
-  if (p.pair) {
+  if constexpr (BN < 128) {
+    // no CTA-pair variant for 64-wide tiles (gemm_plan never selects it)
+  } else if (p.pair) {
     static unsigned long long attr2 = 0;
     if (!(attr2 >> dev & 1ull)) {
-      cudaFuncSetAttribute(gemm_tc2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, Gemm2Cfg::SMEM_BYTES);
+      cudaFuncSetAttribute(gemm_tc2_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Gemm2Cfg<BN>::SMEM_BYTES);
       attr2 |= 1ull << dev;
     }
-    launch_pdl(gemm_tc2_kernel, dim3(p.grid), dim3(GEMM_THREADS), Gemm2Cfg::SMEM_BYTES, s, maps, a);
+    launch_pdl(gemm_tc2_kernel<BN>, dim3(p.grid), dim3(GEMM_THREADS), Gemm2Cfg<BN>::SMEM_BYTES, s, maps, a);
   } else {
     launch_pdl(gemm_tc_kernel<BN>, dim3(p.grid), dim3(GEMM_THREADS), C::SMEM_BYTES, s, maps, a);
   }

@@ -31,12 +31,15 @@ def timeit(fn, iters=20, warm=3):
 def gemm_cases():
     # FLUX 512^2 (M = 1024 img / 512 txt / 1536 joint) and 2048^2 k=8 shapes
     shapes = [(1024, 9216, 3072), (512, 9216, 3072), (1024, 3072, 3072), (1024, 12288, 3072), (1024, 3072, 12288),
-              (1536, 21504, 3072), (1536, 3072, 15360), (4096, 12288, 3072), (8192, 3072, 12288)]
+              (1536, 21504, 3072), (1536, 3072, 15360), (4096, 12288, 3072), (8192, 3072, 12288),
+              (1536, 3072, 3072), (1536, 3072, 12288), (2714, 1536, 1536), (2714, 1536, 6144)]
+    if os.environ.get("GEMM_SHAPES") == "small":
+        shapes = shapes[-4:]
     for M, N, K in shapes:
         A = torch.randn(M, K, device="cuda").to(torch.bfloat16)
         W = (torch.randn(N, K, device="cuda") / math.sqrt(K)).to(torch.bfloat16)
         o = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
-        for bn, pair in ((0, -1), (128, 0), (256, 0), (256, 1)):
+        for bn, pair in ((0, -1), (128, 0), (256, 0), (256, 1), (128, 1)):
             if N % (bn or 64):
                 continue
             ms = timeit(lambda: tsv.op_gemm(A, W, "STORE_BF16", o, force_bn=bn, force_pair=pair))
