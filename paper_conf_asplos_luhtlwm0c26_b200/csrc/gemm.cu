@@ -724,18 +724,20 @@ static void launch_bn(const GemmPlan& p, cudaStream_t s) {
     maps.A[q] = p.tmAq[qq];
     maps.B[q] = p.tmBq[qq];
   }
-  if constexpr (BN < 128) {
-    // no CTA-pair variant for 64-wide tiles (gemm_plan never selects it)
-  } else if (p.pair) {
-    static unsigned long long attr2 = 0;
-    if (!(attr2 >> dev & 1ull)) {
-      cudaFuncSetAttribute(gemm_tc2_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Gemm2Cfg<BN>::SMEM_BYTES);
-      attr2 |= 1ull << dev;
+  if constexpr (BN >= 128) {
+    if (p.pair) {
+      static unsigned long long attr2 = 0;
+      if (!(attr2 >> dev & 1ull)) {
+        cudaFuncSetAttribute(gemm_tc2_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             Gemm2Cfg<BN>::SMEM_BYTES);
+        attr2 |= 1ull << dev;
+      }
+      launch_pdl(gemm_tc2_kernel<BN>, dim3(p.grid), dim3(GEMM_THREADS), Gemm2Cfg<BN>::SMEM_BYTES, s, maps, a);
+      return;
     }
-    launch_pdl(gemm_tc2_kernel<BN>, dim3(p.grid), dim3(GEMM_THREADS), Gemm2Cfg<BN>::SMEM_BYTES, s, maps, a);
-  } else {
-    launch_pdl(gemm_tc_kernel<BN>, dim3(p.grid), dim3(GEMM_THREADS), C::SMEM_BYTES, s, maps, a);
   }
+  // 1-CTA tiles (the only variant for 64-wide tiles: gemm_plan never pairs them)
+  launch_pdl(gemm_tc_kernel<BN>, dim3(p.grid), dim3(GEMM_THREADS), C::SMEM_BYTES, s, maps, a);
 }
 
 void gemm_launch(const GemmPlan& p, cudaStream_t s) {

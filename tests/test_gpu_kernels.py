@@ -72,7 +72,7 @@ GEMM_SHAPES = [(1, 64, 64), (100, 256, 128), (128, 768, 256), (300, 1024, 256), 
 
 
 @pytest.mark.parametrize("M,N,K", GEMM_SHAPES)
-@pytest.mark.parametrize("bn,pair", [(0, -1), (64, 0), (128, 0), (256, 0), (256, 1)])
+@pytest.mark.parametrize("bn,pair", [(0, -1), (64, 0), (128, 0), (128, 1), (256, 0), (256, 1)])
 def test_gemm_integer_exact(tsv, M, N, K, bn, pair):
     if bn and N % bn:
         pytest.skip("N not a multiple of the tile")
