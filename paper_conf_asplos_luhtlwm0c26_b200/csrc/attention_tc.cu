@@ -352,7 +352,10 @@ struct FaCfg {
 constexpr int FA_THREADS = 384;
 
 // NPOLY of every 8 exp2 pairs are evaluated on the FMA/ALU pipes (poly_exp2_x2), the rest on MUFU.
-template <int D, int NPOLY>
+// SPLIT: P_t{j} is handed to the MMA thread in two halves (keys 0-63, then 64-127), each with its
+// own barrier, so PV over the first 64 keys runs on the tensor core while the softmax warps still
+// evaluate the second half's exponentials.
+template <int D, int NPOLY, bool SPLIT>
 __global__ void __launch_bounds__(FA_THREADS, 1)
     attention_fa_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
@@ -365,9 +368,10 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   uint64_t* kv_full = bars + 1;    // [2 stages]
   uint64_t* kv_empty = bars + 3;   // [2 stages]
   uint64_t* s_full = bars + 5;     // [2 q-tiles]
-  uint64_t* p_full = bars + 7;     // [2 q-tiles]
+  uint64_t* p_full = bars + 7;     // [2 q-tiles]  (SPLIT: first half of P)
   uint64_t* o_done = bars + 9;     // [2 q-tiles]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 12);
+  uint64_t* p_full2 = bars + 14;   // [2 q-tiles]  SPLIT: second half of P
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int head = blockIdx.y;
@@ -384,6 +388,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       mbar_init(&kv_empty[i], 1);
       mbar_init(&s_full[i], 1);
       mbar_init(&p_full[i], 128);
+      mbar_init(&p_full2[i], 128);
       mbar_init(&o_done[i], 1);
     }
     fence_mbar_init();
@@ -393,8 +398,12 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  // registers: the producer / MMA warpgroup needs few, the softmax warpgroups hold a 128-score row
+  // each (64 * 128 + 216 * 256 <= 168 * 384, the launch allocation: inc blocks until the pool has them)
   grid_dep_wait();
-  if (warp == 0) {
+  if (warp < 4) {
+   regs_dec<64>();
+   if (warp == 0) {
     if (lane == 0) {
       // ---------------------------------------------------------------- producer
       mbar_arrive_expect_tx(q_full, 2 * C::Q_TILE);
@@ -414,7 +423,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         }
       }
     }
-  } else if (warp == 1) {
+   } else if (warp == 1) {
     if (lane == 0) {
       // ---------------------------------------------------------------- MMA issuer
       constexpr uint32_t idesc_s = make_idesc_bf16(AT_BM, AT_BN);
@@ -431,13 +440,18 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         umma_commit(&s_full[t]);
       };
       auto issue_pv = [&](int t, int j) {
+        const uint32_t sV = smem_u32(sm + C::OFF_V + (j & 1) * C::KV_TILE);
         mbar_wait(&p_full[t], j & 1);
         tc_fence_after();
-        const uint32_t sV = smem_u32(sm + C::OFF_V + (j & 1) * C::KV_TILE);
 #pragma unroll
-        for (int kk = 0; kk < AT_BN / 16; ++kk)
+        for (int kk = 0; kk < AT_BN / 16; ++kk) {
+          if (SPLIT && kk == AT_BN / 32) {
+            mbar_wait(&p_full2[t], j & 1);
+            tc_fence_after();
+          }
           umma_bf16_ts(tmem + C::O_COL + t * D, tmem + t * 128 + kk * 8,
                        make_sw128_mn_desc(sV + kk * 2048, AT_BN * 128), idesc_o, (j | kk) != 0);
+        }
       };
       for (int j = 0; j < n_tiles; ++j) {
         mbar_wait(&kv_full[j & 1], (j >> 1) & 1);
@@ -455,7 +469,9 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         umma_commit(&o_done[t]);
       }
     }
-  } else if (warp >= 4) {
+   }
+  } else {
+    regs_inc<216>();
     // ---------------------------------------------------------------- softmax WG t (thread = query row)
     const int t = (warp - 4) >> 2;
     const int wq = (warp - 4) & 3;
@@ -472,11 +488,12 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
       tmem_ld_wait();
       const int kbase = j * AT_BN;
+      const bool full = kbase + AT_BN <= L;
       // row max with 8 independent accumulators (a single chain would be 128 dependent FMNMX)
       float mx[8];
 #pragma unroll
       for (int q = 0; q < 8; ++q) mx[q] = -FLT_MAX;
-      if (kbase + AT_BN > L) {
+      if (!full) {
 #pragma unroll
         for (int c = 0; c < 4; ++c)
 #pragma unroll
@@ -499,62 +516,69 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         m_ref = mt;
       }
       l_sum *= alpha;
-      // P = 2^(s * scale_log2 - m_ref) as packed bf16 pairs, in place of S (columns 0..63 of S_t)
-      float ls0 = 0.f, ls1 = 0.f;
+      // P = 2^(s * scale_log2 - m_ref) as packed bf16 pairs, in place of S (columns 0..63 of S_t):
+      // keys [64h, 64h + 64) land in sr[h] and TMEM columns [32h, 32h + 32)
       const float neg_m = -m_ref;
-      if (kbase + AT_BN <= L) {
-        // Per tile each softmax warpgroup must finish inside the ~1024-cycle window in which the
-        // tensor core works on the other query tile.  MUFU.EX2 alone needs 1024 cycles per tile
-        // (16/clk/SM), so NPOLY pairs in 8 are evaluated on the FMA/ALU pipes (Cody-Waite split +
-        // cubic, rel. error < 1e-3 << bf16 ulp of P), and the arithmetic uses paired FP32 ops.
-        const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(neg_m, neg_m);
-        float2 lsum[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f),
-                          make_float2(0.f, 0.f)};
+      float2 lsum[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
 #pragma unroll
-        for (int c = 0; c < 4; ++c)
+      for (int h = 0; h < 2; ++h) {
+        if (full) {
+          // Per tile each softmax warpgroup must finish inside the ~1024-cycle window in which the
+          // tensor core works on the other query tile.  MUFU.EX2 alone needs 1024 cycles per tile
+          // (16/clk/SM), so NPOLY pairs in 8 are evaluated on the FMA/ALU pipes (Cody-Waite split +
+          // cubic, rel. error < 1e-3 << bf16 ulp of P), and the arithmetic uses paired FP32 ops.
+          const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(neg_m, neg_m);
 #pragma unroll
-          for (int i = 0; i < 32; i += 2) {
-            const float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2,
-                                        nm2);
-            float2 p;
-            if (((i >> 1) & 7) >= 8 - NPOLY) p = poly_exp2_x2(x);
-            else p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
-            lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], p);     // 8 independent partial sums
-            sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);  // packed P overwrites consumed S
+          for (int c = 2 * h; c < 2 * h + 2; ++c)
+#pragma unroll
+            for (int i = 0; i < 32; i += 2) {
+              const float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])),
+                                          sc2, nm2);
+              float2 p;
+              if (((i >> 1) & 7) >= 8 - NPOLY) p = poly_exp2_x2(x);
+              else p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
+              lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], p);     // 8 independent partial sums
+              sr[h][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);        // packed P overwrites consumed S
+            }
+        } else {
+#pragma unroll
+          for (int c = 2 * h; c < 2 * h + 2; ++c)
+#pragma unroll
+            for (int i = 0; i < 32; i += 2) {
+              const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
+              const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
+              lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], make_float2(p0, p1));
+              sr[h][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);
+            }
+        }
+        if (h == 0 && __any_sync(0xffffffffu, rescale)) {
+          // S_t{j} complete => PV_t{j-1} complete (in-order pipe): O_t can be rescaled now, before any
+          // part of P_t{j} is handed over (here S columns 64-127 are consumed: registers are free)
+#pragma unroll
+          for (int c = 0; c < D / 32; ++c) {
+            uint32_t ov[32];
+            tmem_ld32(o_col + c * 32, ov);
+            tmem_ld_wait();
+#pragma unroll
+            for (int i = 0; i < 32; ++i) ov[i] = __float_as_uint(__uint_as_float(ov[i]) * alpha);
+            tmem_st32(o_col + c * 32, ov);
           }
-        const float2 l01 = __fadd2_rn(lsum[0], lsum[1]), l23 = __fadd2_rn(lsum[2], lsum[3]);
-        const float2 l4 = __fadd2_rn(l01, l23);
-        ls0 = l4.x + l4.y;
-      } else {
-#pragma unroll
-        for (int c = 0; c < 4; ++c)
-#pragma unroll
-          for (int i = 0; i < 32; i += 2) {
-            const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
-            const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
-            ls0 += p0;
-            ls1 += p1;
-            sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);
+        }
+        if (SPLIT || h == 1) {
+          if (SPLIT) {
+            tmem_st32(s_col + 32 * h, sr[h]);
+          } else {
+            tmem_st32(s_col, sr[0]);
+            tmem_st32(s_col + 32, sr[1]);
           }
-      }
-      l_sum += ls0 + ls1;
-      // S_t{j} complete => PV_t{j-1} complete (in-order pipe): O_t can be rescaled right away
-      if (__any_sync(0xffffffffu, rescale)) {
-#pragma unroll
-        for (int c = 0; c < D / 32; ++c) {
-          uint32_t ov[32];
-          tmem_ld32(o_col + c * 32, ov);
-          tmem_ld_wait();
-#pragma unroll
-          for (int i = 0; i < 32; ++i) ov[i] = __float_as_uint(__uint_as_float(ov[i]) * alpha);
-          tmem_st32(o_col + c * 32, ov);
+          tmem_st_wait();
+          tc_fence_before();
+          mbar_arrive(h == 0 ? &p_full[t] : (SPLIT ? &p_full2[t] : &p_full[t]));
         }
       }
-      tmem_st32(s_col, sr[0]);
-      tmem_st32(s_col + 32, sr[1]);
-      tmem_st_wait();
-      tc_fence_before();
-      mbar_arrive(&p_full[t]);
+      const float2 l01 = __fadd2_rn(lsum[0], lsum[1]), l23 = __fadd2_rn(lsum[2], lsum[3]);
+      const float2 l4 = __fadd2_rn(l01, l23);
+      l_sum += l4.x + l4.y;
     }
     // epilogue: O_t / l -> bf16
     mbar_wait(&o_done[t], 0);
@@ -632,18 +656,19 @@ static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L
 template <int D>
 constexpr int default_npoly() { return 2; }   // measured best for D = 64 and 128 (profiles/README.md)
 
-template <int D, int NP>
+template <int D, int NP, bool SPLIT = false>
 static void launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
                       int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s) {
   static unsigned long long done = 0;
   int dev = 0;
   cudaGetDevice(&dev);
   if (!(done >> dev & 1ull)) {
-    cudaFuncSetAttribute(attention_fa_kernel<D, NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, FaCfg<D>::SMEM);
+    cudaFuncSetAttribute(attention_fa_kernel<D, NP, SPLIT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         FaCfg<D>::SMEM);
     done |= 1ull << dev;
   }
   dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H);
-  launch_pdl(attention_fa_kernel<D, NP>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo, L, scale_log2,
+  launch_pdl(attention_fa_kernel<D, NP, SPLIT>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo, L, scale_log2,
              sc);
 }
 
@@ -666,8 +691,19 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     dim3 grid((L + AT_BM - 1) / AT_BM, H);
     attention_tc_kernel<D><<<grid, AT_THREADS, AttnCfg<D>::SMEM, s>>>(tq, tk, tv, o, ldo, L, scale_log2);
   } else {
-    // version 3: the default poly share; 10 + n: n of 8 exp2 pairs by polynomial (tuning sweeps)
-    const int np = version >= 10 ? version - 10 : default_npoly<D>();
+    // version 3: the default poly share; 10 + n: n of 8 exp2 pairs by polynomial (tuning sweeps);
+    // 20 + n: the same with P handed over in two halves (SPLIT)
+    const int np = version >= 10 ? version % 10 : default_npoly<D>();
+    if (version >= 20) {
+      switch (np) {
+        case 1: launch_fa<D, 1, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+        case 2: launch_fa<D, 2, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+        case 3: launch_fa<D, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+        case 4: launch_fa<D, 4, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+        default: return -3;
+      }
+      return 0;
+    }
     switch (np) {
       case 1: launch_fa<D, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
       case 2: launch_fa<D, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;

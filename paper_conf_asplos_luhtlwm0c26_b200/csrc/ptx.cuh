@@ -136,6 +136,11 @@ TSV_DEV void tmem_ld_wait() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: 
 // may start (prologue: barrier init, TMEM alloc, descriptor prefetch) once every CTA of the
 // current kernel executed launch_dependents; grid_dep_wait() blocks until the previous kernel has
 // completed and its memory is visible.  Without the launch attribute both are no-ops.
+// warpgroup register reallocation (all 4 warps of a warpgroup execute it)
+template <int N>
+TSV_DEV void regs_dec() { asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(N)); }
+template <int N>
+TSV_DEV void regs_inc() { asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(N)); }
 TSV_DEV void grid_dep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 TSV_DEV void grid_dep_launch() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 

@@ -208,7 +208,7 @@ def test_qk_norm_rope(tsv, H, D, rows, n_first):
 
 
 # ----------------------------------------------------------------------------- attention
-@pytest.mark.parametrize("impl", [0, 1])
+@pytest.mark.parametrize("impl", [0, 1, 22])
 @pytest.mark.parametrize("L,H,D", [(1, 2, 64), (63, 4, 64), (320, 4, 64), (1000, 3, 128), (1536, 2, 128),
                                    (4700, 1, 128)])
 def test_attention(tsv, L, H, D, impl):
@@ -243,7 +243,8 @@ def test_attention_special_cases(tsv):
     assert np.max(np.abs(_np(o).reshape(L, H, D) - ref)) < 2e-2
 
 
-def test_attention_rescale_path(tsv):
+@pytest.mark.parametrize("impl", [0, 22])
+def test_attention_rescale_path(tsv, impl):
     """Scores growing along the key axis force the conditional O rescale (max grows by > 2^8)."""
     L, H, D = 700, 1, 128
     rng = np.random.default_rng(9)
@@ -252,7 +253,8 @@ def test_attention_rescale_path(tsv):
     v = rng.standard_normal((L, H, D))
     ref = F.attention(q, k, v)
     o = torch.zeros(L, H * D, dtype=torch.bfloat16, device="cuda")
-    tsv.op_attention(_bf16(q.reshape(L, -1)), _bf16(k.reshape(L, -1)), _bf16(v.reshape(L, -1)), o, L, H, D)
+    tsv.op_attention(_bf16(q.reshape(L, -1)), _bf16(k.reshape(L, -1)), _bf16(v.reshape(L, -1)), o, L, H, D,
+                     impl=impl)
     torch.cuda.synchronize()
     # compare against the oracle on the bf16-rounded inputs
     qb, kb, vb = (synth.bf16_bits_to_f32(synth.bf16_rne_bits(a.astype(np.float32))).astype(np.float64)

@@ -75,11 +75,14 @@ def attn_cases():
         o = torch.empty(L, H * D, dtype=torch.bfloat16, device="cuda")
         ld = 3 * H * D
         impls = (0, 1) + ((11, 12, 13, 14) if sweep else ())
+        if os.environ.get("ATTN_IMPLS"):
+            impls = tuple(int(x) for x in os.environ["ATTN_IMPLS"].split(","))
         for impl in impls:
             f = lambda: tsv.op_attention(qkv, qkv[:, H * D:], qkv[:, 2 * H * D:], o, L, H, D, ldq=ld, ldk=ld,
                                          ldv=ld, impl=impl)
             ms = timeit(f, iters=5 if L > 8000 else 20)
-            name = {0: "tcgen05", 1: "mma.sync"}.get(impl, f"tcgen05-poly{impl - 10}")
+            name = {0: "tcgen05", 1: "mma.sync"}.get(
+                impl, f"tcgen05-poly{impl % 10}" + ("-splitP" if impl >= 20 else ""))
             print(json.dumps({"op": "attention", "impl": name, "L": L, "H": H, "D": D,
                               "ms": round(ms, 4), "tflops": round(4 * L * L * D * H / ms / 1e9, 1)}), flush=True)
 
