@@ -654,7 +654,7 @@ static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L
 
 // default share of exp2 evaluated by polynomial, per head dim (tools/microbench.py sweep)
 template <int D>
-constexpr int default_npoly() { return 2; }   // measured best for D = 64 and 128 (profiles/README.md)
+constexpr int default_npoly() { return 1; }   // measured best for D = 64 and 128 (profiles/README.md)
 
 template <int D, int NP, bool SPLIT = false>
 static void launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
