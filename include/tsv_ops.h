@@ -33,7 +33,10 @@ enum {
 /* A [M, K] bf16 (row stride lda elements), W [N, K] bf16 (nn.Linear layout, row stride ldw),
  * bias [N] bf16 or NULL, gate [N] fp32, scalar: device fp32.  K % 64 == 0, N % 64 == 0, 16-byte
  * aligned operands and row strides.  force_bn in {0 (auto), 64, 128, 256}; force_pair: -1 auto,
- * 0 single-CTA tiles, 1 CTA-pair (cta_group::2) 256 x 256 tiles (needs BN = 256). */
+ * 0 single-CTA tiles, 1 CTA-pair (cta_group::2) 256 x 256 tiles (needs BN = 256).
+ * Launched with programmatic dependent launch: W is treated as a constant (its first tiles are
+ * requested before the wait on the previous kernel), so W must not be written by the kernel
+ * launched immediately before on the same stream if that kernel is one of this library's. */
 tsv_status tsv_op_gemm(const void* A, int64_t lda, const void* W, int64_t ldw, int M, int N, int K, int mode,
                        void* out0, int64_t ld0, void* out1, int64_t ld1, int n_split, const void* bias,
                        const float* gate, const float* scalar, int force_bn, int force_pair, void* stream);

@@ -9,7 +9,7 @@ import ctypes as C
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libtsv.so")
+LIB_PATH = os.environ.get("TSV_LIB") or os.path.join(_HERE, "libtsv.so")   # TSV_LIB: A/B builds (tools/ab_bench.sh)
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libtsv.so not built ({LIB_PATH}); run `python -c 'import __graft_entry__ as g; g.build()'`")

@@ -73,6 +73,7 @@ __global__ void __launch_bounds__(T) ln_mod_kernel(const float* __restrict__ x, 
     float d = (v[i].w - mean) * rstd * (1.f + sc.w) + sh.w;
     ur[c] = make_uint2(pack_bf16x2(a, b), pack_bf16x2(cc, d));
   }
+  grid_dep_launch();   // the next kernel (a GEMM) may start its prologue / weight prefetch
 }
 
 // Warp per row (8 rows per 256-thread CTA): the row stays in registers (NV float4 per lane), both

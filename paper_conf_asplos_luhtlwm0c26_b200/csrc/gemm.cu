@@ -347,7 +347,20 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
-  grid_dep_wait();  // A (and the fp32 stream) come from the previous kernel
+  // The weights (B) do not depend on the previous kernel: the first stages of the first tile are
+  // requested before the programmatic-dependency wait, so their HBM latency overlaps the previous
+  // kernel's tail.  A (and the fp32 stream) come from the previous kernel: after the wait.
+  int npre = 0;
+  if (warp == 0 && lane == 0 && (int)blockIdx.x < args.num_tiles) {
+    int pr, m_blk, n_blk;
+    decode_tile(args, blockIdx.x, pr, m_blk, n_blk);
+    npre = num_k < C::STAGES ? num_k : C::STAGES;
+    for (int kb = 0; kb < npre; ++kb) {
+      mbar_arrive_expect_tx(&full[kb], C::STAGE_BYTES);
+      tma_load_2d(&maps.B[pr], &full[kb], sB + kb * C::B_BYTES, kb * BK, n_blk * BN);
+    }
+  }
+  grid_dep_wait();
 
   if (warp == 0) {
     if (lane == 0) {
@@ -361,9 +374,10 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
         const CUtensorMap* tB = &maps.B[pr];
         for (int kb = 0; kb < num_k; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
+          const bool pre = t == (int)blockIdx.x && kb < npre;   // B already requested
+          if (!pre) mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
           tma_load_2d(tA, &full[stage], sA + stage * C::A_BYTES, kb * BK, m_blk * BM);
-          tma_load_2d(tB, &full[stage], sB + stage * C::B_BYTES, kb * BK, n_blk * BN);
+          if (!pre) tma_load_2d(tB, &full[stage], sB + stage * C::B_BYTES, kb * BK, n_blk * BN);
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
       }
@@ -498,6 +512,17 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
   cluster_sync();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  // weights of the first stages before the programmatic-dependency wait (see gemm_tc_kernel)
+  int npre = 0;
+  if (warp == 0 && lane == 0 && cid < args.num_tiles) {
+    int pr, m_blk, n_blk;
+    decode_tile(args, cid, pr, m_blk, n_blk);
+    npre = num_k < C::STAGES ? num_k : C::STAGES;
+    for (int kb = 0; kb < npre; ++kb) {
+      if (leader) mbar_arrive_expect_tx(&full[kb], 2 * C::STAGE_BYTES);
+      tma_load_2d_pair(&maps.B[pr], &full[kb], sB + kb * C::B_BYTES, kb * BK, n_blk * BN + (int)rank * (BN / 2));
+    }
+  }
   grid_dep_wait();  // A (and the fp32 stream) come from the previous kernel
 
   if (warp == 0) {
@@ -511,9 +536,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
         const CUtensorMap* tB = &maps.B[pr];
         for (int kb = 0; kb < num_k; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          if (leader) mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
+          const bool pre = t == cid && kb < npre;   // B already requested
+          if (leader && !pre) mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
           tma_load_2d_pair(tA, &full[stage], sA + stage * C::A_BYTES, kb * BK, m_blk * 256 + (int)rank * 128);
-          tma_load_2d_pair(tB, &full[stage], sB + stage * C::B_BYTES, kb * BK, n_blk * BN + (int)rank * (BN / 2));
+          if (!pre)
+            tma_load_2d_pair(tB, &full[stage], sB + stage * C::B_BYTES, kb * BK, n_blk * BN + (int)rank * (BN / 2));
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
       }
