@@ -399,10 +399,10 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
   // registers: the producer / MMA warpgroup needs few, the softmax warpgroups hold a 128-score row
-  // each (64 * 128 + 216 * 256 <= 168 * 384, the launch allocation: inc blocks until the pool has them)
+  // each (80 * 128 + 208 * 256 <= 168 * 384, the launch allocation: inc blocks until the pool has them)
   grid_dep_wait();
   if (warp < 4) {
-   regs_dec<64>();
+   regs_dec<80>();
    if (warp == 0) {
     if (lane == 0) {
       // ---------------------------------------------------------------- producer
@@ -424,54 +424,63 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       }
     }
    } else if (warp == 1) {
-    if (lane == 0) {
-      // ---------------------------------------------------------------- MMA issuer
-      constexpr uint32_t idesc_s = make_idesc_bf16(AT_BM, AT_BN);
-      constexpr uint32_t idesc_o = make_idesc_bf16_bmn(AT_BM, D);
-      mbar_wait(q_full, 0);
-      auto issue_s = [&](int t, int j) {
-        const uint32_t sQ = smem_u32(sm + C::OFF_Q + t * C::Q_TILE);
-        const uint32_t sK = smem_u32(sm + C::OFF_K + (j & 1) * C::KV_TILE);
+    // ---------------------------------------------------------------- MMA issuer
+    // The whole warp runs the loop (warp-uniform control flow keeps descriptors in uniform
+    // registers); one elected lane issues each batch of MMAs back to back.  Descriptors are bases +
+    // compile-time offsets (the 14-bit address field cannot carry: smem < 256 KB).
+    constexpr uint32_t idesc_s = make_idesc_bf16(AT_BM, AT_BN);
+    constexpr uint32_t idesc_o = make_idesc_bf16_bmn(AT_BM, D);
+    const uint64_t dq0 = make_sw128_desc(smem_u32(sm + C::OFF_Q));
+    const uint64_t dk0 = make_sw128_desc(smem_u32(sm + C::OFF_K));
+    const uint64_t dv0 = make_sw128_mn_desc(smem_u32(sm + C::OFF_V), AT_BN * 128);
+    mbar_wait(q_full, 0);
+    auto issue_s = [&](int t, int j) {
+      const uint64_t dq = dq0 + (uint64_t)((t * C::Q_TILE) >> 4);
+      const uint64_t dk = dk0 + (uint64_t)(((j & 1) * C::KV_TILE) >> 4);
+      if (elect_one()) {
 #pragma unroll
         for (int kk = 0; kk < D / 16; ++kk) {
-          const uint32_t off = (kk >> 2) * (AT_BM * 128) + (kk & 3) * 32;
-          umma_bf16_ss(tmem + t * 128, make_sw128_desc(sQ + off), make_sw128_desc(sK + off), idesc_s, kk > 0);
+          const uint32_t off = ((kk >> 2) * (AT_BM * 128) + (kk & 3) * 32) >> 4;
+          umma_bf16_ss(tmem + t * 128, dq + off, dk + off, idesc_s, kk > 0);
         }
         umma_commit(&s_full[t]);
-      };
-      auto issue_pv = [&](int t, int j) {
-        const uint32_t sV = smem_u32(sm + C::OFF_V + (j & 1) * C::KV_TILE);
-        mbar_wait(&p_full[t], j & 1);
-        tc_fence_after();
+      }
+      __syncwarp();
+    };
+    auto issue_pv = [&](int t, int j, bool release) {
+      const uint64_t dv = dv0 + (uint64_t)(((j & 1) * C::KV_TILE) >> 4);
+      mbar_wait(&p_full[t], j & 1);
+      tc_fence_after();
+      if (elect_one()) {
 #pragma unroll
         for (int kk = 0; kk < AT_BN / 16; ++kk) {
           if (SPLIT && kk == AT_BN / 32) {
             mbar_wait(&p_full2[t], j & 1);
             tc_fence_after();
           }
-          umma_bf16_ts(tmem + C::O_COL + t * D, tmem + t * 128 + kk * 8,
-                       make_sw128_mn_desc(sV + kk * 2048, AT_BN * 128), idesc_o, (j | kk) != 0);
+          umma_bf16_ts(tmem + C::O_COL + t * D, tmem + t * 128 + kk * 8, dv + (uint64_t)(kk * (2048 >> 4)), idesc_o,
+                       (j | kk) != 0);
         }
-      };
-      for (int j = 0; j < n_tiles; ++j) {
-        mbar_wait(&kv_full[j & 1], (j >> 1) & 1);
-        tc_fence_after();
-        for (int t = 0; t < 2; ++t) {
-          if (j > 0) {
-            issue_pv(t, j - 1);
-            if (t == 1) umma_commit(&kv_empty[(j - 1) & 1]);
-          }
-          issue_s(t, j);
-        }
+        if (release) umma_commit(&kv_empty[j & 1]);
       }
+      __syncwarp();
+    };
+    for (int j = 0; j < n_tiles; ++j) {
+      mbar_wait(&kv_full[j & 1], (j >> 1) & 1);
+      tc_fence_after();
       for (int t = 0; t < 2; ++t) {
-        issue_pv(t, n_tiles - 1);
-        umma_commit(&o_done[t]);
+        if (j > 0) issue_pv(t, j - 1, t == 1);
+        issue_s(t, j);
       }
+    }
+    for (int t = 0; t < 2; ++t) {
+      issue_pv(t, n_tiles - 1, false);
+      if (elect_one()) umma_commit(&o_done[t]);
+      __syncwarp();
     }
    }
   } else {
-    regs_inc<216>();
+    regs_inc<208>();
     // ---------------------------------------------------------------- softmax WG t (thread = query row)
     const int t = (warp - 4) >> 2;
     const int wq = (warp - 4) & 3;
@@ -625,6 +634,298 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   if (warp == 2) tmem_dealloc<512>(tmem);
 }
 
+// ------------------------------------------------------------------ v5: 64-key tiles, S double-buffered
+// v3's chain S_t(j) -> softmax -> PV_t(j) -> S_t(j+1) serialises the softmax with the tensor core
+// (P_t(j) aliases the only S_t buffer).  v5 uses 64-key K/V tiles so that each query tile owns two
+// 64-column S buffers (TMEM: S_t,b at 128 t + 64 b, O_t at 256 + D t; 512 columns for D = 128):
+// the MMA thread issues S_t(j+1) into the other buffer BEFORE PV_t(j), so the tensor core computes
+// the next scores while the softmax warps exponentiate the current ones.  Per iteration the MMA
+// thread issues PV_0(j), S_0(j+2), PV_1(j), S_1(j+2): S_t(j+2) reuses buffer j & 1 right behind
+// PV_t(j) in the same in-order tcgen05 pipe, so each softmax warpgroup has two tiles of look-ahead.  Because S_t(j) no longer implies "PV_t(j-1) complete", a rare
+// O rescale first waits on pv_done[t] (committed after every PV_t).
+template <int D>
+struct Fa5Cfg {
+  static constexpr int BN = 64;                          // keys per K/V tile
+  static constexpr int NSUB = D / 64;
+  static constexpr int Q_TILE = AT_BM * D * 2;
+  static constexpr int KV_TILE = BN * D * 2;             // one K (or V) tile
+  static constexpr int NST = D == 128 ? 4 : 6;           // K/V stages
+  static constexpr int OFF_Q = 0;                        // 2 tiles
+  static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;
+  static constexpr int OFF_V = OFF_K + NST * KV_TILE;
+  static constexpr int OFF_BAR = OFF_V + NST * KV_TILE;
+  static constexpr int SMEM = OFF_BAR + 256 + 1024;
+  static constexpr int O_COL = 256;
+};
+
+template <int D, int NPOLY>
+__global__ void __launch_bounds__(FA_THREADS, 1)
+    attention_fa5_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
+                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
+                         float scale_log2, const __grid_constant__ AttnScatter sc) {
+  using C = Fa5Cfg<D>;
+  constexpr int BN = C::BN, NST = C::NST;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
+  uint64_t* q_full = bars + 0;
+  uint64_t* kv_full = bars + 1;            // [NST]
+  uint64_t* kv_empty = bars + 1 + NST;     // [NST]
+  uint64_t* s_full = bars + 1 + 2 * NST;   // [2 t][2 buffers]
+  uint64_t* p_full = bars + 5 + 2 * NST;   // [2 t][2 buffers]
+  uint64_t* pv_done = bars + 9 + 2 * NST;  // [2 t], every PV_t
+  uint64_t* o_done = bars + 11 + 2 * NST;  // [2 t], the last PV_t
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 14 + 2 * NST);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int head = blockIdx.y;
+  const int q0 = blockIdx.x * 2 * AT_BM;
+  const int n_tiles = (L + BN - 1) / BN;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmQ);
+    tma_prefetch_desc(&tmK);
+    tma_prefetch_desc(&tmV);
+    mbar_init(q_full, 1);
+    for (int i = 0; i < NST; ++i) {
+      mbar_init(&kv_full[i], 1);
+      mbar_init(&kv_empty[i], 1);
+    }
+    for (int i = 0; i < 4; ++i) {
+      mbar_init(&s_full[i], 1);
+      mbar_init(&p_full[i], 128);
+    }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&pv_done[i], 1);
+      mbar_init(&o_done[i], 1);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 2) tmem_alloc<512>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  grid_dep_wait();
+  if (warp < 4) {
+    regs_dec<80>();
+    if (warp == 0) {
+      if (lane == 0) {
+        // -------------------------------------------------------------- producer
+        mbar_arrive_expect_tx(q_full, 2 * C::Q_TILE);
+        for (int t = 0; t < 2; ++t)
+          for (int s = 0; s < C::NSUB; ++s)
+            tma_load_3d(&tmQ, q_full, sm + C::OFF_Q + t * C::Q_TILE + s * (AT_BM * 128), s * 64, head,
+                        q0 + t * AT_BM);
+        for (int j = 0; j < n_tiles; ++j) {
+          const int st = j % NST;
+          if (j >= NST) mbar_wait(&kv_empty[st], ((j / NST) - 1) & 1);
+          mbar_arrive_expect_tx(&kv_full[st], 2 * C::KV_TILE);
+          for (int s = 0; s < C::NSUB; ++s) {
+            tma_load_3d(&tmK, &kv_full[st], sm + C::OFF_K + st * C::KV_TILE + s * (BN * 128), s * 64, head, j * BN);
+            tma_load_3d(&tmV, &kv_full[st], sm + C::OFF_V + st * C::KV_TILE + s * (BN * 128), s * 64, head, j * BN);
+          }
+        }
+      }
+    } else if (warp == 1) {
+      // -------------------------------------------------------------- MMA issuer (whole warp,
+      // one elected lane per MMA batch; descriptors = bases + compile-time offsets, see v3)
+      constexpr uint32_t idesc_s = make_idesc_bf16(AT_BM, BN);
+      constexpr uint32_t idesc_o = make_idesc_bf16_bmn(AT_BM, D);
+      const uint64_t dq0 = make_sw128_desc(smem_u32(sm + C::OFF_Q));
+      const uint64_t dk0 = make_sw128_desc(smem_u32(sm + C::OFF_K));
+      const uint64_t dv0 = make_sw128_mn_desc(smem_u32(sm + C::OFF_V), BN * 128);
+      mbar_wait(q_full, 0);
+      auto issue_s = [&](int t, int j) {   // S_t(j) into buffer j & 1 (K tile already resident)
+        const uint64_t dq = dq0 + (uint64_t)((t * C::Q_TILE) >> 4);
+        const uint64_t dk = dk0 + (uint64_t)(((j % NST) * C::KV_TILE) >> 4);
+        if (elect_one()) {
+#pragma unroll
+          for (int kk = 0; kk < D / 16; ++kk) {
+            const uint32_t offq = ((kk >> 2) * (AT_BM * 128) + (kk & 3) * 32) >> 4;
+            const uint32_t offk = ((kk >> 2) * (BN * 128) + (kk & 3) * 32) >> 4;
+            umma_bf16_ss(tmem + t * 128 + (j & 1) * 64, dq + offq, dk + offk, idesc_s, kk > 0);
+          }
+          umma_commit(&s_full[t * 2 + (j & 1)]);
+        }
+        __syncwarp();
+      };
+      auto issue_pv = [&](int t, int j) {  // O_t += P_t(j) V(j); P_t(j) in TMEM buffer j & 1
+        const uint64_t dv = dv0 + (uint64_t)(((j % NST) * C::KV_TILE) >> 4);
+        mbar_wait(&p_full[t * 2 + (j & 1)], (j >> 1) & 1);
+        tc_fence_after();
+        if (elect_one()) {
+#pragma unroll
+          for (int kk = 0; kk < BN / 16; ++kk)
+            umma_bf16_ts(tmem + C::O_COL + t * D, tmem + t * 128 + (j & 1) * 64 + kk * 8,
+                         dv + (uint64_t)(kk * (2048 >> 4)), idesc_o, (j | kk) != 0);
+          umma_commit(&pv_done[t]);
+          if (j == n_tiles - 1) umma_commit(&o_done[t]);
+        }
+        __syncwarp();
+      };
+      // two tiles of look-ahead per query tile: S_t(j+2) (into buffer j & 1) right behind PV_t(j)
+      for (int j = 0; j < 2 && j < n_tiles; ++j) {
+        mbar_wait(&kv_full[j], 0);
+        tc_fence_after();
+        issue_s(0, j);
+        issue_s(1, j);
+      }
+      for (int j = 0; j < n_tiles; ++j) {
+        const bool ahead = j + 2 < n_tiles;
+        for (int t = 0; t < 2; ++t) {
+          issue_pv(t, j);
+          if (ahead) {
+            if (t == 0) {
+              mbar_wait(&kv_full[(j + 2) % NST], ((j + 2) / NST) & 1);
+              tc_fence_after();
+            }
+            issue_s(t, j + 2);
+          }
+        }
+        if (elect_one()) umma_commit(&kv_empty[j % NST]);
+        __syncwarp();
+      }
+    }
+  } else {
+    regs_inc<208>();
+    // ---------------------------------------------------------------- softmax WG t (thread = query row)
+    const int t = (warp - 4) >> 2;
+    const int wq = (warp - 4) & 3;
+    const int row = wq * 32 + lane;
+    const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
+    const uint32_t o_col = tmem + lane_base + C::O_COL + t * D;
+    float m_ref = -FLT_MAX, l_sum = 0.f;
+    for (int j = 0; j < n_tiles; ++j) {
+      const uint32_t s_col = tmem + lane_base + t * 128 + (j & 1) * 64;
+      mbar_wait(&s_full[t * 2 + (j & 1)], (j >> 1) & 1);
+      tc_fence_after();
+      uint32_t sr[2][32];
+      tmem_ld32(s_col, sr[0]);
+      tmem_ld32(s_col + 32, sr[1]);
+      tmem_ld_wait();
+      const int kbase = j * BN;
+      const bool full = kbase + BN <= L;
+      if (!full) {
+#pragma unroll
+        for (int c = 0; c < 2; ++c)
+#pragma unroll
+          for (int i = 0; i < 32; ++i)
+            if (kbase + c * 32 + i >= L) sr[c][i] = __float_as_uint(-INFINITY);
+      }
+      float mx[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) mx[q] = -FLT_MAX;
+#pragma unroll
+      for (int c = 0; c < 2; ++c)
+#pragma unroll
+        for (int i = 0; i < 32; ++i) mx[i & 7] = fmaxf(mx[i & 7], __uint_as_float(sr[c][i]));
+      const float mt = fmaxf(fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3])),
+                             fmaxf(fmaxf(mx[4], mx[5]), fmaxf(mx[6], mx[7]))) * scale_log2;
+      bool rescale = false;
+      float alpha = 1.f;
+      if (j == 0) {
+        m_ref = mt;
+      } else if (mt > m_ref + RESCALE_THRESHOLD) {
+        rescale = true;
+        alpha = exp2f(m_ref - mt);
+        m_ref = mt;
+      }
+      l_sum *= alpha;
+      const float neg_m = -m_ref;
+      float2 lsum[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+      if (full) {
+        const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(neg_m, neg_m);
+#pragma unroll
+        for (int c = 0; c < 2; ++c)
+#pragma unroll
+          for (int i = 0; i < 32; i += 2) {
+            const float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2,
+                                        nm2);
+            float2 p;
+            if (((i >> 1) & 7) >= 8 - NPOLY) p = poly_exp2_x2(x);
+            else p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
+            lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], p);
+            sr[0][c * 16 + i / 2] = pack_bf16x2(p.x, p.y);      // packed P overwrites consumed S
+          }
+      } else {
+#pragma unroll
+        for (int c = 0; c < 2; ++c)
+#pragma unroll
+          for (int i = 0; i < 32; i += 2) {
+            const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
+            const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
+            lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], make_float2(p0, p1));
+            sr[0][c * 16 + i / 2] = pack_bf16x2(p0, p1);
+          }
+      }
+      if (__any_sync(0xffffffffu, rescale)) {
+        // O_t must hold exactly tiles < j: wait for PV_t(j-1) (S_t(j) was issued before it)
+        mbar_wait(&pv_done[t], (j - 1) & 1);
+        tc_fence_after();
+#pragma unroll
+        for (int c = 0; c < D / 32; ++c) {
+          uint32_t ov[32];
+          tmem_ld32(o_col + c * 32, ov);
+          tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 32; ++i) ov[i] = __float_as_uint(__uint_as_float(ov[i]) * alpha);
+          tmem_st32(o_col + c * 32, ov);
+        }
+      }
+      tmem_st32(s_col, sr[0]);
+      tmem_st_wait();
+      tc_fence_before();
+      mbar_arrive(&p_full[t * 2 + (j & 1)]);
+      const float2 l01 = __fadd2_rn(lsum[0], lsum[1]), l23 = __fadd2_rn(lsum[2], lsum[3]);
+      const float2 l4 = __fadd2_rn(l01, l23);
+      l_sum += l4.x + l4.y;
+    }
+    // epilogue: O_t / l -> bf16 once the last PV_t is complete (pv_done may be two phases behind
+    // here: S_t(n-1) complete only implies PV_t(n-3) complete)
+    mbar_wait(&o_done[t], 0);
+    tc_fence_after();
+    const float inv = 1.f / l_sum;
+    const int grow = q0 + t * AT_BM + row;
+    bf16* orow = o + (long long)grow * ldo + head * D;
+    if (sc.k > 0 && grow < L) {
+      int p = 0, lr;
+      if (grow < sc.Lt) {
+        while (p + 1 < sc.k && grow >= sc.t_off[p + 1]) ++p;
+        lr = grow - sc.t_off[p];
+      } else {
+        const int gi = grow - sc.Lt;
+        while (p + 1 < sc.k && gi >= sc.i_off[p + 1]) ++p;
+        lr = sc.nt[p] + gi - sc.i_off[p];
+      }
+      orow = sc.dst[p] + (long long)lr * sc.ld + sc.col0 + head * D;
+    }
+#pragma unroll
+    for (int c = 0; c < D / 32; ++c) {
+      uint32_t ov[32];
+      tmem_ld32(o_col + c * 32, ov);
+      tmem_ld_wait();
+      if (grow < L) {
+        uint4* dst = reinterpret_cast<uint4*>(orow + c * 32);
+#pragma unroll
+        for (int qd = 0; qd < 4; ++qd) {
+          uint4 v;
+          v.x = pack_bf16x2(__uint_as_float(ov[qd * 8 + 0]) * inv, __uint_as_float(ov[qd * 8 + 1]) * inv);
+          v.y = pack_bf16x2(__uint_as_float(ov[qd * 8 + 2]) * inv, __uint_as_float(ov[qd * 8 + 3]) * inv);
+          v.z = pack_bf16x2(__uint_as_float(ov[qd * 8 + 4]) * inv, __uint_as_float(ov[qd * 8 + 5]) * inv);
+          v.w = pack_bf16x2(__uint_as_float(ov[qd * 8 + 6]) * inv, __uint_as_float(ov[qd * 8 + 7]) * inv);
+          dst[qd] = v;
+        }
+      }
+    }
+  }
+  grid_dep_launch();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 2) tmem_dealloc<512>(tmem);
+}
+
 // ------------------------------------------------------------------ host
 static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -639,12 +940,12 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 }
 
 // [rows][heads][D] view of a strided activation: element (r, h, d) at base + r*ld + h*D + d
-static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L, long long ld) {
+static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L, long long ld, int box_rows = 128) {
   auto enc = encode_fn();
   if (!enc) return -1;
   cuuint64_t dims[3] = {(cuuint64_t)D, (cuuint64_t)H, (cuuint64_t)L};
   cuuint64_t strides[2] = {(cuuint64_t)D * 2, (cuuint64_t)ld * 2};
-  cuuint32_t box[3] = {64, 1, 128};
+  cuuint32_t box[3] = {64, 1, (cuuint32_t)box_rows};
   cuuint32_t es[3] = {1, 1, 1};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(base), dims, strides, box, es,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -654,7 +955,7 @@ static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L
 
 // default share of exp2 evaluated by polynomial, per head dim (tools/microbench.py sweep)
 template <int D>
-constexpr int default_npoly() { return 1; }   // measured best for D = 64 and 128 (profiles/README.md)
+constexpr int default_npoly() { return D == 64 ? 2 : 1; }   // measured (profiles/README.md)
 
 template <int D, int NP, bool SPLIT = false>
 static void launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
@@ -672,6 +973,21 @@ static void launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtens
              sc);
 }
 
+template <int D, int NP>
+static void launch_fa5(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
+                       int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s) {
+  static unsigned long long done = 0;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!(done >> dev & 1ull)) {
+    cudaFuncSetAttribute(attention_fa5_kernel<D, NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, Fa5Cfg<D>::SMEM);
+    done |= 1ull << dev;
+  }
+  dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H);
+  launch_pdl(attention_fa5_kernel<D, NP>, grid, dim3(FA_THREADS), Fa5Cfg<D>::SMEM, s, tq, tk, tv, o, ldo, L,
+             scale_log2, sc);
+}
+
 template <int D>
 static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv, bf16* o,
                      long long ldo, int L, int H, int version, const AttnScatter& sc, cudaStream_t s) {
@@ -687,6 +1003,19 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     done |= 1ull << dev;
   }
   const float scale_log2 = (1.0f / sqrtf((float)D)) * 1.4426950408889634f;
+  if (version >= 40) {   // v5: 64-key K/V tiles, double-buffered S; 40 + n: n of 8 exp2 pairs by polynomial
+    CUtensorMap tk64, tv64;
+    if (make_tmap_heads(&tk64, k, D, H, L, ldk, 64) || make_tmap_heads(&tv64, v, D, H, L, ldv, 64)) return -1;
+    switch (version - 40) {
+      case 0: launch_fa5<D, 0>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
+      case 1: launch_fa5<D, 1>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
+      case 2: launch_fa5<D, 2>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
+      case 3: launch_fa5<D, 3>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
+      case 4: launch_fa5<D, 4>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
+      default: return -3;
+    }
+    return 0;
+  }
   if (version == 2) {
     dim3 grid((L + AT_BM - 1) / AT_BM, H);
     attention_tc_kernel<D><<<grid, AT_THREADS, AttnCfg<D>::SMEM, s>>>(tq, tk, tv, o, ldo, L, scale_log2);

@@ -208,7 +208,7 @@ def test_qk_norm_rope(tsv, H, D, rows, n_first):
 
 
 # ----------------------------------------------------------------------------- attention
-@pytest.mark.parametrize("impl", [0, 1, 22])
+@pytest.mark.parametrize("impl", [0, 1, 22, 42])
 @pytest.mark.parametrize("L,H,D", [(1, 2, 64), (63, 4, 64), (320, 4, 64), (1000, 3, 128), (1536, 2, 128),
                                    (4700, 1, 128)])
 def test_attention(tsv, L, H, D, impl):
@@ -243,7 +243,7 @@ def test_attention_special_cases(tsv):
     assert np.max(np.abs(_np(o).reshape(L, H, D) - ref)) < 2e-2
 
 
-@pytest.mark.parametrize("impl", [0, 22])
+@pytest.mark.parametrize("impl", [0, 22, 42])
 def test_attention_rescale_path(tsv, impl):
     """Scores growing along the key axis force the conditional O rescale (max grows by > 2^8)."""
     L, H, D = 700, 1, 128

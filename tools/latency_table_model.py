@@ -29,17 +29,26 @@ def main():
     ap.add_argument("--model", default="flux")
     ap.add_argument("--iters", type=int, default=5)
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r01", "latency_table_model.json"))
+    ap.add_argument("--res", default=",".join(str(r) for r in RES))
     args = ap.parse_args()
+    res_list = [int(r) for r in args.res.split(",")]
     d = tsv.model_preset(args.model)
     h, Lt = d.hidden, d.text_tokens
     blocks = d.n_double + d.n_single
     B = 2 if d.family == 1 else 1
     eng = tsv.Engine(args.model, devices=[0] * 8)
-    ms, cv = eng.latency_table(RES, KS, warmup=2, iters=args.iters)
+    ms, cv = eng.latency_table(res_list, KS, warmup=2, iters=args.iters)
     eng.close()
+    import importlib.util
+    spec = importlib.util.spec_from_file_location("_bench", os.path.join(ROOT, "bench.py"))
+    bench = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(bench)
+    flops = bench.MODELS[args.model]["flops"]
+    peak = bench.peaks()["tflops"] * 1e12
     table = []
     comm = []
-    for i, r in enumerate(RES):
+    roof = []
+    for i, r in enumerate(res_list):
         Li = (r // 16) ** 2
         row, crow = [], []
         for j, k in enumerate(KS):
@@ -54,7 +63,17 @@ def main():
             crow.append(round(c_ms, 4))
         table.append([round(x, 4) for x in row])
         comm.append(crow)
-    out = {"model": args.model, "res": RES, "ks": KS, "ms": table, "comm_model_ms": comm,
+        # roofline: per-rank algorithmic GEMM + attention FLOPs at the sustained bf16 peak, plus the
+        # modeled all-to-all (the elementwise passes and weight streaming are below 3 % here)
+        rrow = []
+        for j, k in enumerate(KS):
+            g, a = flops(r, k)
+            t_roof = (g + a) / peak * 1e3 + crow[j]
+            rrow.append(round(t_roof / row[j], 4))
+        roof.append(rrow)
+    out = {"model": args.model, "res": res_list, "ks": KS, "ms": table, "comm_model_ms": comm,
+           "roofline_frac": roof, "roofline_peak_tflops": peak / 1e12,
+           "efficiency_vs_k1": [[round(row[0] / (k * row[j]), 4) for j, k in enumerate(KS)] for row in table],
            "measured_virtual_ms": [[round(float(x), 4) for x in r] for r in ms],
            "note": "k=1 measured on one B200; k>1 = (k virtual ranks on one B200) / k + modeled NVLink all-to-all"}
     os.makedirs(os.path.dirname(args.out), exist_ok=True)

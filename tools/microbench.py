@@ -82,7 +82,7 @@ def attn_cases():
                                          ldv=ld, impl=impl)
             ms = timeit(f, iters=5 if L > 8000 else 20)
             name = {0: "tcgen05", 1: "mma.sync"}.get(
-                impl, f"tcgen05-poly{impl % 10}" + ("-splitP" if impl >= 20 else ""))
+                impl, f"tcgen05-poly{impl % 10}" + ("-v5" if impl >= 40 else "-splitP" if impl >= 20 else ""))
             print(json.dumps({"op": "attention", "impl": name, "L": L, "H": H, "D": D,
                               "ms": round(ms, 4), "tflops": round(4 * L * L * D * H / ms / 1e9, 1)}), flush=True)
 
