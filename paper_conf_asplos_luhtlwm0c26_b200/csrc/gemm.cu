@@ -698,7 +698,24 @@ int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int
   long long pair_tiles = 0;
   for (int q = 0; q < nprob; ++q) pair_tiles += (long long)((probs[q].M + 255) / 256) * (N / 256);
   const bool pair_auto = bn == 256 && maxM > 128 && (K >= 8192 || pair_tiles * 2 >= (long long)num_sms * 9 / 10);
-  const bool pair = force_pair >= 0 ? (force_pair > 0 && bn >= 128) : pair_auto;
+  bool pair = force_pair >= 0 ? (force_pair > 0 && bn >= 128) : pair_auto;
+  if (force_pair < 0 && !force_bn && bn == 256 && maxM > 128 && qk_D <= 128) {
+    // 256 x 128 pair tiles vs the choice above.  Per-SM time ~ waves * K * BN * e + E (one epilogue
+    // and pipeline fill not overlapped), fitted to tools/microbench.py after the warp-wide MMA
+    // issue: e = 1 (256-wide tiles) / 1.2 (128-wide), E = 420k / 210k.  E.g. 1536x3072x3072
+    // 836 vs 745 TFLOP/s and 576x3072x3072 644 vs 453 (128 wins: two tiles per pair overlap the
+    // epilogue), 1536x3072x15360 1537 vs 1399 (256 wins: one full wave, long K).
+    long long single_tiles = 0;
+    for (int q = 0; q < nprob; ++q) single_tiles += (long long)((probs[q].M + BM - 1) / BM) * (N / 256);
+    const long long pairs = num_sms / 2;
+    const double c_pair256 = (double)((pair_tiles + pairs - 1) / pairs) * K * 256.0 + 420e3;
+    const double c_single = (double)((single_tiles + num_sms - 1) / num_sms) * K * 256.0 + 420e3;
+    const double c_pair128 = (double)((2 * pair_tiles + pairs - 1) / pairs) * K * 128.0 * 1.2 + 210e3;
+    if (c_pair128 < (pair ? c_pair256 : c_single)) {
+      bn = 128;
+      pair = true;
+    }
+  }
   const int bm = pair ? 256 : BM;
   p->nprob = nprob; p->N = N; p->K = K; p->BN = bn; p->pair = pair;
   int tiles = 0;

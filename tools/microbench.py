@@ -32,9 +32,11 @@ def gemm_cases():
     # FLUX 512^2 (M = 1024 img / 512 txt / 1536 joint) and 2048^2 k=8 shapes
     shapes = [(1024, 9216, 3072), (512, 9216, 3072), (1024, 3072, 3072), (1024, 12288, 3072), (1024, 3072, 12288),
               (1536, 21504, 3072), (1536, 3072, 15360), (4096, 12288, 3072), (8192, 3072, 12288),
-              (1536, 3072, 3072), (1536, 3072, 12288), (2714, 1536, 1536), (2714, 1536, 6144)]
+              (1536, 3072, 3072), (1536, 3072, 12288), (2714, 1536, 1536), (2714, 1536, 6144),
+              (2714, 4608, 1536), (2714, 6144, 1536), (8858, 1536, 1536), (8858, 4608, 1536), (8858, 1536, 6144),
+              (576, 3072, 3072), (576, 9216, 3072), (2112, 3072, 12288)]
     if os.environ.get("GEMM_SHAPES") == "small":
-        shapes = shapes[-4:]
+        shapes = shapes[-10:]
     for M, N, K in shapes:
         A = torch.randn(M, K, device="cuda").to(torch.bfloat16)
         W = (torch.randn(N, K, device="cuda") / math.sqrt(K)).to(torch.bfloat16)
