@@ -13,6 +13,7 @@
 //               by more than 2^8, so P stays <= 256 and rescales are rare), final 1/l and store.
 // TMEM: S0 | S1 | O  (128 + 128 + D fp32 columns).
 #include <cfloat>
+#include <cstdlib>
 #include <cudaTypedefs.h>
 
 #include "kernels.h"
@@ -355,7 +356,14 @@ constexpr int FA_THREADS = 384;
 // SPLIT: P_t{j} is handed to the MMA thread in two halves (keys 0-63, then 64-127), each with its
 // own barrier, so PV over the first 64 keys runs on the tensor core while the softmax warps still
 // evaluate the second half's exponentials.
-template <int D, int NPOLY, bool SPLIT>
+// LAZY: the row max is not recomputed per tile.  P = 2^(s*scale - m_ref) is evaluated with the
+// running reference directly; the tile's row sum bounds every p in it (p <= sum), so a row whose
+// sum stays <= 2^LAZY_LOG2 has no p > 2^LAZY_LOG2 and needs no rescale (m_ref is only a
+// stabiliser: softmax is exact for any reference that keeps p finite).  Otherwise (the max grew
+// a lot: early tiles) the warp reloads S from TMEM and takes the exact path (row max, rescale).
+// Saves the 128 FMNMX per row per tile and the max-before-exp dependency on the softmax chain.
+constexpr float LAZY_LIMIT = 65536.0f;   // 2^16
+template <int D, int NPOLY, bool SPLIT, bool LAZY = false>
 __global__ void __launch_bounds__(FA_THREADS, 1)
     attention_fa_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
@@ -493,11 +501,59 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       mbar_wait(&s_full[t], j & 1);
       tc_fence_after();
       uint32_t sr[4][32];
-#pragma unroll
-      for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
-      tmem_ld_wait();
       const int kbase = j * AT_BN;
       const bool full = kbase + AT_BN <= L;
+      const bool lazy = LAZY && !SPLIT && j > 0 && full;
+      if (!lazy) {
+#pragma unroll
+        for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
+        tmem_ld_wait();
+      }
+      if (lazy) {
+        const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(-m_ref, -m_ref);
+        float2 lz[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+        // no max before the exponentials: the TMEM loads are pipelined with the arithmetic (chunk
+        // c + 1 is in flight while chunk c is exponentiated)
+        tmem_ld32(s_col, sr[0]);
+        tmem_ld_wait_dep(sr[0]);
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          if (c < 3) tmem_ld32(s_col + (c + 1) * 32, sr[c + 1]);
+#pragma unroll
+          for (int i = 0; i < 32; i += 2) {
+            float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2, nm2);
+            float2 p;
+            if (((i >> 1) & 7) >= 8 - NPOLY) {
+              // the polynomial path wraps the exponent field outside [-126, 127]: clamp both sides
+              // (a clamped x > 64 still makes the sum exceed the limit)
+              x.x = fminf(x.x, 64.f);
+              x.y = fminf(x.y, 64.f);
+              p = poly_exp2_x2(x);
+            } else {
+              p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
+            }
+            lz[(i >> 1) & 3] = __fadd2_rn(lz[(i >> 1) & 3], p);
+            sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);
+          }
+          if (c < 3) tmem_ld_wait_dep(sr[c + 1]);
+        }
+        const float2 l01 = __fadd2_rn(lz[0], lz[1]), l23 = __fadd2_rn(lz[2], lz[3]);
+        const float2 l4 = __fadd2_rn(l01, l23);
+        const float ts = l4.x + l4.y;
+        if (!__any_sync(0xffffffffu, !(ts <= LAZY_LIMIT))) {   // also catches inf / NaN
+          l_sum += ts;
+          tmem_st32(s_col, sr[0]);
+          tmem_st32(s_col + 32, sr[1]);
+          tmem_st_wait();
+          tc_fence_before();
+          mbar_arrive(&p_full[t]);
+          continue;
+        }
+        // rare: reload the untouched S columns and take the exact path below
+#pragma unroll
+        for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
+        tmem_ld_wait();
+      }
       // row max with 8 independent accumulators (a single chain would be 128 dependent FMNMX)
       float mx[8];
 #pragma unroll
@@ -926,6 +982,311 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   if (warp == 2) tmem_dealloc<512>(tmem);
 }
 
+// ------------------------------------------------------------------ v6: CTA pair (cta_group::2)
+// A cluster of 2 CTAs computes 512 queries of one head as two pair tiles t = 0, 1 of 256 queries:
+// CTA r holds rows [256 t + 128 r, +128) of pair tile t (its Q tiles, its S/P/O rows in its TMEM).
+// The even CTA issues tcgen05.mma.cta_group::2 with M = 256: S_t = Q_t K^T (N = 128 keys, each CTA
+// holds 64 of the keys) and O_t += P_t V (N = D, each CTA holds D/2 columns of V).  Per SM the
+// S MMA reads 96 B/clk of shared memory instead of 128 (the 1-CTA kernel's S MMA sits at the
+// shared-memory port limit, like a 128x128 GEMM tile) and K/V tiles cost half the TMA bytes.
+// Softmax: v3's lazy-max body per CTA; P hand-over is one arrive per softmax warp on the even
+// CTA's barrier (8 warps per pair tile).
+template <int D>
+struct Fa2Cfg {
+  static constexpr int NSUB = D / 64;
+  static constexpr int Q_TILE = AT_BM * D * 2;          // 128 rows
+  static constexpr int K_HALF = (AT_BN / 2) * D * 2;    // 64 keys x D
+  static constexpr int V_HALF = AT_BN * (D / 2) * 2;    // 128 keys x D/2 (one 128-byte swizzle column)
+  static constexpr int STAGE = K_HALF + V_HALF;
+  static constexpr int NST = 4;
+  static constexpr int OFF_Q = 0;                        // 2 tiles
+  static constexpr int OFF_KV = OFF_Q + 2 * Q_TILE;      // NST stages of [K half | V half]
+  static constexpr int OFF_BAR = OFF_KV + NST * STAGE;
+  static constexpr int SMEM = OFF_BAR + 256 + 1024;
+  static constexpr int O_COL = 256;
+};
+static_assert(Fa2Cfg<128>::SMEM <= 227 * 1024, "pair attention smem");
+
+template <int D, int NPOLY>
+__global__ void __launch_bounds__(FA_THREADS, 1)
+    attention_fa2_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
+                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
+                         float scale_log2, const __grid_constant__ AttnScatter sc) {
+  static_assert(D == 128, "pair kernel: D = 128 (V halves are one 64-column swizzle block)");
+  using C = Fa2Cfg<D>;
+  constexpr int NST = C::NST;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
+  uint64_t* q_full = bars + 0;             // even CTA: both CTAs' Q bytes
+  uint64_t* kv_full = bars + 1;            // [NST] even CTA: both halves
+  uint64_t* kv_empty = bars + 1 + NST;     // [NST] both CTAs (multicast commit)
+  uint64_t* s_full = bars + 1 + 2 * NST;   // [2 t] both CTAs (multicast commit)
+  uint64_t* p_full = bars + 3 + 2 * NST;   // [2 t] even CTA: 8 softmax warps
+  uint64_t* o_done = bars + 5 + 2 * NST;   // [2 t] both CTAs
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 8 + 2 * NST);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_ctarank();
+  const bool leader = rank == 0;
+  const int head = blockIdx.y;
+  const int qc = (blockIdx.x >> 1) * 4 * AT_BM;   // the pair's first query
+  const int n_tiles = (L + AT_BN - 1) / AT_BN;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmQ);
+    tma_prefetch_desc(&tmK);
+    tma_prefetch_desc(&tmV);
+    mbar_init(q_full, 1);
+    for (int i = 0; i < NST; ++i) {
+      mbar_init(&kv_full[i], 1);
+      mbar_init(&kv_empty[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&s_full[i], 1);
+      mbar_init(&p_full[i], 8);
+      mbar_init(&o_done[i], 1);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 2) tmem_alloc_pair<512>(tmem_slot);
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  grid_dep_wait();
+  if (warp < 4) {
+    regs_dec<80>();
+    if (warp == 0) {
+      if (lane == 0) {
+        // -------------------------------------------------------------- producer (both CTAs)
+        if (leader) mbar_arrive_expect_tx(q_full, 2 * 2 * C::Q_TILE);
+        for (int t = 0; t < 2; ++t)
+          for (int s = 0; s < C::NSUB; ++s)
+            tma_load_3d_pair(&tmQ, q_full, sm + C::OFF_Q + t * C::Q_TILE + s * (AT_BM * 128), s * 64, head,
+                             qc + t * 2 * AT_BM + (int)rank * AT_BM);
+        for (int j = 0; j < n_tiles; ++j) {
+          const int st = j % NST;
+          if (j >= NST) mbar_wait(&kv_empty[st], ((j / NST) - 1) & 1);
+          if (leader) mbar_arrive_expect_tx(&kv_full[st], 2 * C::STAGE);
+          uint8_t* sk = sm + C::OFF_KV + st * C::STAGE;
+          for (int s = 0; s < C::NSUB; ++s)   // keys [128 j + 64 r, +64), all D
+            tma_load_3d_pair(&tmK, &kv_full[st], sk + s * ((AT_BN / 2) * 128), s * 64, head,
+                             j * AT_BN + (int)rank * (AT_BN / 2));
+          // keys [128 j, +128), columns [64 r, +64)
+          tma_load_3d_pair(&tmV, &kv_full[st], sk + C::K_HALF, (int)rank * 64, head, j * AT_BN);
+        }
+      }
+    } else if (warp == 1 && leader) {
+      // -------------------------------------------------------------- MMA issuer (even CTA, whole warp)
+      constexpr uint32_t idesc_s = make_idesc_bf16(2 * AT_BM, AT_BN);
+      constexpr uint32_t idesc_o = make_idesc_bf16_bmn(2 * AT_BM, D);
+      const uint64_t dq0 = make_sw128_desc(smem_u32(sm + C::OFF_Q));
+      const uint64_t dk0 = make_sw128_desc(smem_u32(sm + C::OFF_KV));
+      const uint64_t dv0 = make_sw128_mn_desc(smem_u32(sm + C::OFF_KV + C::K_HALF), AT_BN * 128);
+      mbar_wait(q_full, 0);
+      auto issue_s = [&](int t, int j) {
+        const uint64_t dq = dq0 + (uint64_t)((t * C::Q_TILE) >> 4);
+        const uint64_t dk = dk0 + (uint64_t)(((j % NST) * C::STAGE) >> 4);
+        if (elect_one()) {
+#pragma unroll
+          for (int kk = 0; kk < D / 16; ++kk) {
+            const uint32_t offq = ((kk >> 2) * (AT_BM * 128) + (kk & 3) * 32) >> 4;
+            const uint32_t offk = ((kk >> 2) * ((AT_BN / 2) * 128) + (kk & 3) * 32) >> 4;
+            umma_bf16_ss_pair(tmem + t * 128, dq + offq, dk + offk, idesc_s, kk > 0);
+          }
+          umma_commit_pair(&s_full[t]);
+        }
+        __syncwarp();
+      };
+      auto issue_pv = [&](int t, int j, bool release) {
+        const uint64_t dv = dv0 + (uint64_t)(((j % NST) * C::STAGE) >> 4);
+        mbar_wait(&p_full[t], j & 1);
+        tc_fence_after();
+        if (elect_one()) {
+#pragma unroll
+          for (int kk = 0; kk < AT_BN / 16; ++kk)
+            umma_bf16_ts_pair(tmem + C::O_COL + t * D, tmem + t * 128 + kk * 8, dv + (uint64_t)(kk * (2048 >> 4)),
+                              idesc_o, (j | kk) != 0);
+          if (release) umma_commit_pair(&kv_empty[j % NST]);
+        }
+        __syncwarp();
+      };
+      for (int j = 0; j < n_tiles; ++j) {
+        mbar_wait(&kv_full[j % NST], (j / NST) & 1);
+        tc_fence_after();
+        for (int t = 0; t < 2; ++t) {
+          if (j > 0) issue_pv(t, j - 1, t == 1);
+          issue_s(t, j);
+        }
+      }
+      for (int t = 0; t < 2; ++t) {
+        issue_pv(t, n_tiles - 1, false);
+        if (elect_one()) umma_commit_pair(&o_done[t]);
+        __syncwarp();
+      }
+    }
+  } else {
+    regs_inc<208>();
+    // ---------------------------------------------------------------- softmax WG t (thread = query row)
+    const int t = (warp - 4) >> 2;
+    const int wq = (warp - 4) & 3;
+    const int row = wq * 32 + lane;
+    const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
+    const uint32_t s_col = tmem + lane_base + t * 128;
+    const uint32_t o_col = tmem + lane_base + C::O_COL + t * D;
+    float m_ref = -FLT_MAX, l_sum = 0.f;
+    auto hand_over = [&]() {   // P_t(j) stored: one arrive per warp on the even CTA's barrier
+      tmem_st_wait();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive_remote(&p_full[t], 0);
+    };
+    for (int j = 0; j < n_tiles; ++j) {
+      mbar_wait(&s_full[t], j & 1);
+      tc_fence_after();
+      uint32_t sr[4][32];
+#pragma unroll
+      for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
+      tmem_ld_wait();
+      const int kbase = j * AT_BN;
+      const bool full = kbase + AT_BN <= L;
+      if (j > 0 && full) {
+        // lazy max (see attention_fa_kernel): P with the running reference, exact path if any row's
+        // tile sum exceeds the bound
+        const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(-m_ref, -m_ref);
+        float2 lz[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+#pragma unroll
+          for (int i = 0; i < 32; i += 2) {
+            float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2, nm2);
+            float2 p;
+            if (((i >> 1) & 7) >= 8 - NPOLY) {
+              x.x = fminf(x.x, 64.f);
+              x.y = fminf(x.y, 64.f);
+              p = poly_exp2_x2(x);
+            } else {
+              p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
+            }
+            lz[(i >> 1) & 3] = __fadd2_rn(lz[(i >> 1) & 3], p);
+            sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);
+          }
+        const float2 l01 = __fadd2_rn(lz[0], lz[1]), l23 = __fadd2_rn(lz[2], lz[3]);
+        const float2 l4 = __fadd2_rn(l01, l23);
+        const float ts = l4.x + l4.y;
+        if (!__any_sync(0xffffffffu, !(ts <= LAZY_LIMIT))) {
+          l_sum += ts;
+          tmem_st32(s_col, sr[0]);
+          tmem_st32(s_col + 32, sr[1]);
+          hand_over();
+          continue;
+        }
+#pragma unroll
+        for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
+        tmem_ld_wait();
+      }
+      // exact path: first tile, the masked last tile, and lazy overflows
+      float mx[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) mx[q] = -FLT_MAX;
+      if (!full) {
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+#pragma unroll
+          for (int i = 0; i < 32; ++i)
+            if (kbase + c * 32 + i >= L) sr[c][i] = __float_as_uint(-INFINITY);
+      }
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int i = 0; i < 32; ++i) mx[i & 7] = fmaxf(mx[i & 7], __uint_as_float(sr[c][i]));
+      const float mt = fmaxf(fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3])),
+                             fmaxf(fmaxf(mx[4], mx[5]), fmaxf(mx[6], mx[7]))) * scale_log2;
+      bool rescale = false;
+      float alpha = 1.f;
+      if (j == 0) {
+        m_ref = mt;
+      } else if (mt > m_ref + RESCALE_THRESHOLD) {
+        rescale = true;
+        alpha = exp2f(m_ref - mt);
+        m_ref = mt;
+      }
+      l_sum *= alpha;
+      const float neg_m = -m_ref;
+      float2 lsum[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int i = 0; i < 32; i += 2) {
+          const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
+          const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
+          lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], make_float2(p0, p1));
+          sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);
+        }
+      if (__any_sync(0xffffffffu, rescale)) {
+        // S_t(j) complete => PV_t(j-1) complete (in-order pipe of the pair): O_t holds tiles < j
+#pragma unroll
+        for (int c = 0; c < D / 32; ++c) {
+          uint32_t ov[32];
+          tmem_ld32(o_col + c * 32, ov);
+          tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 32; ++i) ov[i] = __float_as_uint(__uint_as_float(ov[i]) * alpha);
+          tmem_st32(o_col + c * 32, ov);
+        }
+      }
+      tmem_st32(s_col, sr[0]);
+      tmem_st32(s_col + 32, sr[1]);
+      hand_over();
+      const float2 l01 = __fadd2_rn(lsum[0], lsum[1]), l23 = __fadd2_rn(lsum[2], lsum[3]);
+      const float2 l4 = __fadd2_rn(l01, l23);
+      l_sum += l4.x + l4.y;
+    }
+    // epilogue: O_t / l -> bf16
+    mbar_wait(&o_done[t], 0);
+    tc_fence_after();
+    const float inv = 1.f / l_sum;
+    const int grow = qc + t * 2 * AT_BM + (int)rank * AT_BM + row;
+    bf16* orow = o + (long long)grow * ldo + head * D;
+    if (sc.k > 0 && grow < L) {
+      int p = 0, lr;
+      if (grow < sc.Lt) {
+        while (p + 1 < sc.k && grow >= sc.t_off[p + 1]) ++p;
+        lr = grow - sc.t_off[p];
+      } else {
+        const int gi = grow - sc.Lt;
+        while (p + 1 < sc.k && gi >= sc.i_off[p + 1]) ++p;
+        lr = sc.nt[p] + gi - sc.i_off[p];
+      }
+      orow = sc.dst[p] + (long long)lr * sc.ld + sc.col0 + head * D;
+    }
+#pragma unroll
+    for (int c = 0; c < D / 32; ++c) {
+      uint32_t ov[32];
+      tmem_ld32(o_col + c * 32, ov);
+      tmem_ld_wait();
+      if (grow < L) {
+        uint4* dst = reinterpret_cast<uint4*>(orow + c * 32);
+#pragma unroll
+        for (int qd = 0; qd < 4; ++qd) {
+          uint4 v;
+          v.x = pack_bf16x2(__uint_as_float(ov[qd * 8 + 0]) * inv, __uint_as_float(ov[qd * 8 + 1]) * inv);
+          v.y = pack_bf16x2(__uint_as_float(ov[qd * 8 + 2]) * inv, __uint_as_float(ov[qd * 8 + 3]) * inv);
+          v.z = pack_bf16x2(__uint_as_float(ov[qd * 8 + 4]) * inv, __uint_as_float(ov[qd * 8 + 5]) * inv);
+          v.w = pack_bf16x2(__uint_as_float(ov[qd * 8 + 6]) * inv, __uint_as_float(ov[qd * 8 + 7]) * inv);
+          dst[qd] = v;
+        }
+      }
+    }
+  }
+  grid_dep_launch();
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  if (warp == 2) tmem_dealloc_pair<512>(tmem);
+}
+
 // ------------------------------------------------------------------ host
 static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -957,19 +1318,19 @@ static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L
 template <int D>
 constexpr int default_npoly() { return D == 64 ? 2 : 1; }   // measured (profiles/README.md)
 
-template <int D, int NP, bool SPLIT = false>
+template <int D, int NP, bool SPLIT = false, bool LAZY = false>
 static void launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
                       int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s) {
   static unsigned long long done = 0;
   int dev = 0;
   cudaGetDevice(&dev);
   if (!(done >> dev & 1ull)) {
-    cudaFuncSetAttribute(attention_fa_kernel<D, NP, SPLIT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaFuncSetAttribute(attention_fa_kernel<D, NP, SPLIT, LAZY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          FaCfg<D>::SMEM);
     done |= 1ull << dev;
   }
   dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H);
-  launch_pdl(attention_fa_kernel<D, NP, SPLIT>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo, L, scale_log2,
+  launch_pdl(attention_fa_kernel<D, NP, SPLIT, LAZY>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo, L, scale_log2,
              sc);
 }
 
@@ -988,6 +1349,34 @@ static void launch_fa5(const CUtensorMap& tq, const CUtensorMap& tk, const CUten
              scale_log2, sc);
 }
 
+template <int NP>
+static void launch_fa2(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
+                       int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s) {
+  static unsigned long long done = 0;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!(done >> dev & 1ull)) {
+    cudaFuncSetAttribute(attention_fa2_kernel<128, NP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         Fa2Cfg<128>::SMEM);
+    done |= 1ull << dev;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(2 * ((L + 4 * AT_BM - 1) / (4 * AT_BM)), H);
+  cfg.blockDim = dim3(FA_THREADS);
+  cfg.dynamicSmemBytes = Fa2Cfg<128>::SMEM;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  attr[1].id = cudaLaunchAttributeClusterDimension;
+  attr[1].val.clusterDim.x = 2;
+  attr[1].val.clusterDim.y = 1;
+  attr[1].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 2;
+  cudaLaunchKernelEx(&cfg, attention_fa2_kernel<128, NP>, tq, tk, tv, o, ldo, L, scale_log2, sc);
+}
+
 template <int D>
 static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv, bf16* o,
                      long long ldo, int L, int H, int version, const AttnScatter& sc, cudaStream_t s) {
@@ -1003,7 +1392,7 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     done |= 1ull << dev;
   }
   const float scale_log2 = (1.0f / sqrtf((float)D)) * 1.4426950408889634f;
-  if (version >= 40) {   // v5: 64-key K/V tiles, double-buffered S; 40 + n: n of 8 exp2 pairs by polynomial
+  if (version >= 40 && version < 50) {   // v5: 64-key K/V tiles, double-buffered S; 40 + n: n of 8 exp2 pairs by polynomial
     CUtensorMap tk64, tv64;
     if (make_tmap_heads(&tk64, k, D, H, L, ldk, 64) || make_tmap_heads(&tv64, v, D, H, L, ldv, 64)) return -1;
     switch (version - 40) {
@@ -1012,6 +1401,30 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
       case 2: launch_fa5<D, 2>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
       case 3: launch_fa5<D, 3>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
       case 4: launch_fa5<D, 4>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
+      default: return -3;
+    }
+    return 0;
+  }
+  if (version >= 60) {   // 60 + n: CTA-pair kernel (D = 128 only), lazy max, n of 8 exp2 pairs by polynomial
+    if (D != 128) return -3;
+    CUtensorMap tk64, tv64;   // K halves: 64-key boxes; V halves: 128 keys x 64 columns (the default box)
+    if (make_tmap_heads(&tk64, k, D, H, L, ldk, 64)) return -1;
+    switch (version - 60) {
+      case 0: launch_fa2<0>(tq, tk64, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 1: launch_fa2<1>(tq, tk64, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 2: launch_fa2<2>(tq, tk64, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 3: launch_fa2<3>(tq, tk64, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      default: return -3;
+    }
+    return 0;
+  }
+  if (version >= 50) {   // 50 + n: lazy row max (see attention_fa_kernel), n of 8 exp2 pairs by polynomial
+    switch (version - 50) {
+      case 0: launch_fa<D, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 1: launch_fa<D, 1, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 2: launch_fa<D, 2, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 3: launch_fa<D, 3, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 4: launch_fa<D, 4, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
       default: return -3;
     }
     return 0;
@@ -1045,6 +1458,19 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
   return 0;
 }
 
+// The step's variant per head dim (profiles/README.md, attention table); TSV_ATTN_D128 / TSV_ATTN_D64
+// override it with any tsv_op_attention impl number >= 3 (same-box A/B of whole steps).
+static int default_version(int D) {
+  static int v[2] = {-1, -1};
+  int& r = v[D == 128];
+  if (r < 0) {
+    const char* e = getenv(D == 128 ? "TSV_ATTN_D128" : "TSV_ATTN_D64");
+    r = e ? atoi(e) : (D == 128 ? 52 : 53);   // lazy max; 2 (D = 128) / 3 (D = 64) of 8 exp2 pairs by polynomial
+    if (r < 3) r = 3;
+  }
+  return r;
+}
+
 // returns 0 if the tensor-core path was launched, nonzero if the layout is unsupported by TMA.
 // version 3: two query tiles per CTA, P in TMEM (the step's kernel); version 2: one query tile,
 // P in shared memory (kept for comparison).
@@ -1060,6 +1486,7 @@ int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk,
   if (((ldq | ldk | ldv) * 2) % 16 || ((reinterpret_cast<uintptr_t>(q) | reinterpret_cast<uintptr_t>(k) |
                                         reinterpret_cast<uintptr_t>(v)) & 15))
     return -1;
+  if (version == 3) version = default_version(D);
   if (D == 128) return launch_tc<128>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, sc, s);
   if (D == 64) return launch_tc<64>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, sc, s);
   return -1;

@@ -208,10 +208,12 @@ def test_qk_norm_rope(tsv, H, D, rows, n_first):
 
 
 # ----------------------------------------------------------------------------- attention
-@pytest.mark.parametrize("impl", [0, 1, 22, 42])
+@pytest.mark.parametrize("impl", [0, 1, 22, 42, 51, 52, 61, 62])
 @pytest.mark.parametrize("L,H,D", [(1, 2, 64), (63, 4, 64), (320, 4, 64), (1000, 3, 128), (1536, 2, 128),
                                    (4700, 1, 128)])
 def test_attention(tsv, L, H, D, impl):
+    if impl >= 60 and D != 128:
+        pytest.skip("CTA-pair kernel is D = 128 only")
     rng = np.random.default_rng(L + H + D)
     qkv = rng.standard_normal((L, 3, H, D)).astype(np.float32) * np.float32(1.5)
     qkv = synth.bf16_bits_to_f32(synth.bf16_rne_bits(qkv)).astype(np.float64)
@@ -243,7 +245,7 @@ def test_attention_special_cases(tsv):
     assert np.max(np.abs(_np(o).reshape(L, H, D) - ref)) < 2e-2
 
 
-@pytest.mark.parametrize("impl", [0, 22, 42])
+@pytest.mark.parametrize("impl", [0, 22, 42, 51, 52, 61, 62])
 def test_attention_rescale_path(tsv, impl):
     """Scores growing along the key axis force the conditional O rescale (max grows by > 2^8)."""
     L, H, D = 700, 1, 128
@@ -261,3 +263,27 @@ def test_attention_rescale_path(tsv, impl):
                   for a in (q, k, v))
     ref = F.attention(qb, kb, vb)
     assert _rel(_np(o).reshape(L, H, D), ref) < 2e-2
+
+
+@pytest.mark.parametrize("D,impl", [(64, 0), (64, 51), (64, 52), (128, 0), (128, 52), (128, 61), (128, 62)])
+@pytest.mark.parametrize("jump", [3.0, 12.0, 200.0])
+def test_attention_score_jump(tsv, D, impl, jump):
+    """A later key tile whose scores exceed the running maximum by `jump` (log2 units): small jumps
+    stay on the lazy path (p up to 2^jump), large ones overflow the lazy sum bound (or exp2 itself)
+    and must take the exact path with an O rescale."""
+    L, H = 900, 2
+    rng = np.random.default_rng(int(jump))
+    q = np.ones((L, H, D)) / np.sqrt(D)
+    k = rng.standard_normal((L, H, D)) * 0.3
+    k[500:] += jump / np.log2(np.e)           # score(s) = q.k / sqrt(D) -> + jump*ln2 for keys >= 500
+    v = rng.standard_normal((L, H, D))
+    qb, kb, vb = (synth.bf16_bits_to_f32(synth.bf16_rne_bits(a.astype(np.float32))).astype(np.float64)
+                  for a in (q, k, v))
+    o = torch.zeros(L, H * D, dtype=torch.bfloat16, device="cuda")
+    tsv.op_attention(_bf16(qb.reshape(L, -1)), _bf16(kb.reshape(L, -1)), _bf16(vb.reshape(L, -1)), o, L, H, D,
+                     impl=impl)
+    torch.cuda.synchronize()
+    ref = F.attention(qb, kb, vb)
+    got = _np(o).reshape(L, H, D)
+    assert np.all(np.isfinite(got))
+    assert _rel(got, ref) < 2e-2

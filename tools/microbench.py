@@ -79,14 +79,21 @@ def attn_cases():
         impls = (0, 1) + ((11, 12, 13, 14) if sweep else ())
         if os.environ.get("ATTN_IMPLS"):
             impls = tuple(int(x) for x in os.environ["ATTN_IMPLS"].split(","))
+        fns = {impl: (lambda impl=impl: tsv.op_attention(qkv, qkv[:, H * D:], qkv[:, 2 * H * D:], o, L, H, D,
+                                                         ldq=ld, ldk=ld, ldv=ld, impl=impl)) for impl in impls}
+        # interleaved rounds (the box is power-capped: clocks drift over a run), median per impl
+        times = {impl: [] for impl in impls}
+        for _ in range(int(os.environ.get("ATTN_ROUNDS", "3"))):
+            for impl in impls:
+                times[impl].append(timeit(fns[impl], iters=5 if L > 8000 else 20))
         for impl in impls:
-            f = lambda: tsv.op_attention(qkv, qkv[:, H * D:], qkv[:, 2 * H * D:], o, L, H, D, ldq=ld, ldk=ld,
-                                         ldv=ld, impl=impl)
-            ms = timeit(f, iters=5 if L > 8000 else 20)
+            ms = sorted(times[impl])[len(times[impl]) // 2]
             name = {0: "tcgen05", 1: "mma.sync"}.get(
-                impl, f"tcgen05-poly{impl % 10}" + ("-v5" if impl >= 40 else "-splitP" if impl >= 20 else ""))
+                impl, f"tcgen05-poly{impl % 10}" + ("-lazymax" if impl >= 50 else "-v5" if impl >= 40
+                                                    else "-splitP" if impl >= 20 else ""))
             print(json.dumps({"op": "attention", "impl": name, "L": L, "H": H, "D": D,
-                              "ms": round(ms, 4), "tflops": round(4 * L * L * D * H / ms / 1e9, 1)}), flush=True)
+                              "ms": round(ms, 4), "tflops": round(4 * L * L * D * H / ms / 1e9, 1),
+                              "all_ms": [round(t, 4) for t in times[impl]]}), flush=True)
 
 
 def ln_cases():
