@@ -41,6 +41,18 @@ tsv_status tsv_op_gemm(const void* A, int64_t lda, const void* W, int64_t ldw, i
                        void* out0, int64_t ld0, void* out1, int64_t ld1, int n_split, const void* bias,
                        const float* gate, const float* scalar, int force_bn, int force_pair, void* stream);
 
+/* The same GEMM with split-K (a8 / a9 on small row counts): K is cut into `splits` ranges
+ * (0: the engine's automatic choice, which may be 1); each range's fp32 partial goes to ws and the
+ * last range to finish an output tile sums the partials in range order 0..splits-1 and applies the
+ * epilogue once (mode TSV_EPI_RESID_GATE: out0 += gate * (A W^T + bias), or TSV_EPI_ACCUM_F32:
+ * out0 += A W^T + bias), so the result is deterministic.  sem: device int buffer of
+ * sem_ints >= 4 * output tiles entries, zero on entry and left zero; ws: device buffer of ws_bytes
+ * (splits * tiles * 128 * tile width * 4 bytes are used; the split factor is capped to fit).  One
+ * (sem, ws) pair per concurrently running launch.  TSV_E_INVAL if the mode is not accumulating. */
+tsv_status tsv_op_gemm_split(const void* A, int64_t lda, const void* W, int64_t ldw, int M, int N, int K, int mode,
+                             void* out0, int64_t ld0, const void* bias, const float* gate, int splits, int* sem,
+                             int sem_ints, float* ws, int64_t ws_bytes, void* stream);
+
 /* a3 + a4 fused (the step's QKV / linear1 GEMM): y = A W^T + bias with columns "(K H D)" =
  * [q | k | v] over [0, 3h) (+ GELU columns >= 3h into out1 when mode = TSV_EPI_SPLIT_GELU,
  * n_split = 3h).  q and k heads become RoPE(RMSNorm(y) * g) (eps 1e-6; gq/gk bf16 [D]; cos/sin fp32

@@ -256,6 +256,17 @@ def op_gemm(A, W, mode, out0, out1=None, bias=None, gate=None, scalar=None, n_sp
                           _stream(stream)))
 
 
+def op_gemm_split(A, W, mode, out0, sem, ws, splits=0, bias=None, gate=None, stream=None):
+    """Split-K GEMM into the fp32 stream (mode RESID_GATE / ACCUM_F32); sem: zeroed int32 device
+    buffer; ws: fp32 device workspace for the partials."""
+    M, K = A.shape
+    N = W.shape[0]
+    check(lib.tsv_op_gemm_split(_ptr(A), A.stride(0), _ptr(W), W.stride(0), M, N, K,
+                                EPI[mode] if isinstance(mode, str) else mode, _ptr(out0), out0.stride(0), _ptr(bias),
+                                _ptr(gate), splits, _ptr(sem), sem.numel(), _ptr(ws), ws.numel() * 4,
+                                _stream(stream)))
+
+
 def op_gemm_qkv(A, W, out0, h, D, gq, gk, cosb, sinb, bias=None, mode="STORE_BF16", out1=None, ld1=None,
                 k_sp=1, pack=None, pack_rows=0, pack_row0=0, stream=None):
     M, K = A.shape

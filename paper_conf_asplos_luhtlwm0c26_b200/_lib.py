@@ -84,6 +84,8 @@ _SIGS = {
     "tsv_engine_profile_read": (_i32, [_p, _P(C.c_double), _P(_i64), _P(C.c_double), _P(C.c_double)]),
     "tsv_op_gemm": (_i32, [_p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p, _i64, _p, _i64, _i32, _p, _p, _p, _i32, _i32,
                             _p]),
+    "tsv_op_gemm_split": (_i32, [_p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p, _i64, _p, _p, _i32, _p, _i32, _p,
+                                  _i64, _p]),
     "tsv_op_gemm_qkv": (_i32, [_p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p, _i64, _p, _i64, _p, _i32, _i32,
                                _p, _p, _p, _p, _i32, _p, _i32, _i32, _p]),
     "tsv_op_ln_mod": (_i32, [_p, _i64, _p, _i64, _p, _p, _i32, _i32, _i32, _p]),

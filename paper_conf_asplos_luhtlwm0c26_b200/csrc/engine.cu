@@ -151,8 +151,29 @@ struct Slot {
   cudaStream_t stream = nullptr;
   Workspace ws;
   DevBuf scratch;  // conditioning temporaries
+  DevBuf sem;      // split-K arrival counters of this slot's GEMM launches (zero between launches)
+  DevBuf splitws;  // split-K partials
+  GemmSplitWs sws() const {
+    GemmSplitWs w;
+    w.sem = reinterpret_cast<int*>(sem.p);
+    w.sem_ints = (int)(sem.bytes / sizeof(int));
+    w.ws = reinterpret_cast<float*>(splitws.p);
+    w.ws_bytes = (long long)splitws.bytes;
+    return w;
+  }
   std::map<uint64_t, StepGraph> graphs;
 };
+constexpr int SEM_INTS = 4096;
+constexpr size_t SPLIT_WS_BYTES = 32u << 20;
+// TSV_SPLITK=0 disables split-K for small GEMM launches (A/B measurements)
+static bool splitk_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("TSV_SPLITK");
+    v = e ? atoi(e) != 0 : 1;
+  }
+  return v != 0;
+}
 
 // per (request, slot): state that depends only on the request
 struct ReqDev {
@@ -292,7 +313,8 @@ static tsv_status gemm(tsv_engine* e, Slot& s, const bf16* A, long long lda, con
   if (M <= 0) return TSV_OK;
   GemmPlan p;
   const char* err = nullptr;
-  if (gemm_plan(&p, A, lda, Wt, ldw, M, N, K, epi, s.ds->num_sms, &err))
+  const GemmSplitWs w = s.sws();
+  if (gemm_plan(&p, A, lda, Wt, ldw, M, N, K, epi, s.ds->num_sms, &err, 0, -1, splitk_enabled() ? &w : nullptr))
     return fail(TSV_E_INVAL, "%s (M=%d N=%d K=%d)", err, M, N, K);
   const double out_b = (epi.mode <= EPI_SPLIT_GELU) ? 2.0
                        : (epi.mode == EPI_STORE_F32 ? 4.0 : (epi.mode == EPI_CFG_EULER ? 16.0 : 8.0));
@@ -312,7 +334,8 @@ static tsv_status gemm_multi(tsv_engine* e, Slot& s, const GemmProblem* probs, i
   if (!n) return TSV_OK;
   GemmPlan p;
   const char* err = nullptr;
-  if (gemm_plan_multi(&p, nz, n, N, K, s.ds->num_sms, &err))
+  const GemmSplitWs w = s.sws();
+  if (gemm_plan_multi(&p, nz, n, N, K, s.ds->num_sms, &err, 0, -1, splitk_enabled() ? &w : nullptr))
     return fail(TSV_E_INVAL, "%s (N=%d K=%d)", err, N, K);
   double fl = 0, by = 2.0 * N * K * n;
   for (int i = 0; i < n; ++i) {
@@ -1464,7 +1487,18 @@ tsv_status tsv_engine_create(const tsv_model_desc* model, const int* devices, in
     }
     s.ds = it->second.get();
     CK(cudaSetDevice(s.device));
-    CK(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+    // TSV_VIRTUAL_SERIAL=1: virtual ranks on one device share one stream, so every kernel runs alone
+    // on the GPU as it would on a rank's own GPU (per-rank timing of k > 1 on one device); default:
+    // one stream per rank (the ranks' kernels overlap)
+    const char* vs = getenv("TSV_VIRTUAL_SERIAL");
+    Slot* first = nullptr;
+    for (int j = 0; j < i; ++j)
+      if (e->slots[j].device == s.device) { first = &e->slots[j]; break; }
+    if (vs && atoi(vs) && first) s.stream = first->stream;
+    else CK(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+    TRY(dev_alloc(s.sem, s.device, SEM_INTS * sizeof(int)));
+    CK(cudaMemset(s.sem.p, 0, SEM_INTS * sizeof(int)));
+    TRY(dev_alloc(s.splitws, s.device, SPLIT_WS_BYTES));
   }
   // peer access between distinct local devices (in-process all-to-all and reshard)
   for (auto& a : e->devs)
@@ -2081,6 +2115,30 @@ tsv_status tsv_op_gemm(const void* A, int64_t lda, const void* Wt, int64_t ldw, 
   GemmEpi epi = epi_of(mode, out0, ld0, reinterpret_cast<const bf16*>(bias), gate, out1, ld1, n_split, scalar);
   if (gemm_plan(&p, reinterpret_cast<const bf16*>(A), lda, reinterpret_cast<const bf16*>(Wt), ldw, M, N, K, epi, sms,
                 &err, force_bn, force_pair))
+    return fail(TSV_E_INVAL, "%s", err);
+  gemm_launch(p, reinterpret_cast<cudaStream_t>(stream));
+  CK(cudaGetLastError());
+  return TSV_OK;
+}
+
+tsv_status tsv_op_gemm_split(const void* A, int64_t lda, const void* Wt, int64_t ldw, int M, int N, int K, int mode,
+                             void* out0, int64_t ld0, const void* bias, const float* gate, int splits, int* sem,
+                             int sem_ints, float* ws, int64_t ws_bytes, void* stream) {
+  if (mode != EPI_RESID_GATE && mode != EPI_ACCUM_F32) return fail(TSV_E_INVAL, "split-K needs RESID_GATE or ACCUM_F32");
+  if (!sem || !ws || splits < 0) return fail(TSV_E_INVAL, "split-K needs counters, a workspace and splits >= 0");
+  GemmSplitWs w;
+  w.sem = sem;
+  w.sem_ints = sem_ints;
+  w.ws = ws;
+  w.ws_bytes = ws_bytes;
+  int dev = 0, sms = 148;
+  CK(cudaGetDevice(&dev));
+  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  GemmPlan p;
+  const char* err = nullptr;
+  GemmEpi epi = epi_of(mode, out0, ld0, reinterpret_cast<const bf16*>(bias), gate, nullptr, 0, 0, nullptr);
+  if (gemm_plan(&p, reinterpret_cast<const bf16*>(A), lda, reinterpret_cast<const bf16*>(Wt), ldw, M, N, K, epi, sms,
+                &err, 0, -1, &w, splits))
     return fail(TSV_E_INVAL, "%s", err);
   gemm_launch(p, reinterpret_cast<cudaStream_t>(stream));
   CK(cudaGetLastError());

@@ -38,6 +38,13 @@ struct GemmCfg {
 // [tile0[q], tile0[q+1]) belong to problem q.
 struct GemmArgs {
   int N, K, num_n, num_tiles, nprob;
+  // split-K (1-CTA tiles only): tile t = split s * tiles_per_split + t0 covers k-blocks
+  // [s * kps, min(num_k, (s + 1) * kps)).  Each split stores its fp32 partial (per epilogue warp:
+  // 32 rows x BN) into ws and counts itself in sem[4 t0 + warp]; the last to arrive sums the
+  // partials in split order 0..splits-1 (deterministic whoever arrives last) and runs the epilogue.
+  int splits, kps, tiles_per_split;
+  int* sem;
+  float* ws;
   int M[GEMM_MAX_PROBLEMS], num_m[GEMM_MAX_PROBLEMS], tile0[GEMM_MAX_PROBLEMS];
   GemmEpi epi[GEMM_MAX_PROBLEMS];
 };
@@ -216,13 +223,21 @@ __device__ __forceinline__ void epilogue_qk_head(const GemmEpi& e, int M, int ro
   }
 }
 
-__device__ __forceinline__ void epilogue_chunk(const GemmEpi& e, int M, int row0, int n0, const uint32_t (&r)[32],
-                                               float* stg, int lane) {
+// TMEM chunk (thread = row, 32 columns) -> row-coalesced layout through the warp's staging tile:
+// a[it] = columns [4 c4, 4 c4 + 4) of row it * 4 + (lane >> 3), c4 = lane & 7.
+__device__ __forceinline__ void stage_chunk(const uint32_t (&r)[32], float* stg, int lane, float4 (&a)[8]) {
   float v[32];
 #pragma unroll
   for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
   stage_write(stg, lane, v);
   __syncwarp();
+#pragma unroll
+  for (int it = 0; it < 8; ++it) a[it] = stage_read(stg, it * 4 + (lane >> 3), lane & 7);
+  __syncwarp();  // the staging tile may be overwritten by the next chunk from here on
+}
+
+// epilogue of one 32 x 32 chunk in the staged layout (bias, activation / fp32-stream update, stores)
+__device__ __forceinline__ void finish_chunk(const GemmEpi& e, int M, int row0, int n0, float4 (&a)[8], int lane) {
   const int c4 = lane & 7;
   const int col = n0 + c4 * 4;  // this lane's 4 columns for all 8 row groups
   float4 b = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -230,6 +245,10 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpi& e, int M, int row0
     const uint2 bu = __ldg(reinterpret_cast<const uint2*>(e.bias + col));
     const float2 b0 = unpack_bf16x2(bu.x), b1 = unpack_bf16x2(bu.y);
     b = make_float4(b0.x, b0.y, b1.x, b1.y);
+  }
+#pragma unroll
+  for (int it = 0; it < 8; ++it) {
+    a[it].x += b.x; a[it].y += b.y; a[it].z += b.z; a[it].w += b.w;
   }
   int mode = e.mode;
   bf16* ob = nullptr;
@@ -246,13 +265,6 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpi& e, int M, int row0
   } else if (mode <= EPI_SILU_BF16) {
     ob = reinterpret_cast<bf16*>(e.out0) + col;
   }
-  float4 a[8];
-#pragma unroll
-  for (int it = 0; it < 8; ++it) {
-    a[it] = stage_read(stg, it * 4 + (lane >> 3), c4);
-    a[it].x += b.x; a[it].y += b.y; a[it].z += b.z; a[it].w += b.w;
-  }
-  __syncwarp();  // the staging tile may be overwritten by the next chunk from here on
   const int rbase = row0 + (lane >> 3);
   if (mode <= EPI_SILU_BF16) {
 #pragma unroll
@@ -275,8 +287,8 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpi& e, int M, int row0
   float4 x[8];
 #pragma unroll
   for (int it = 0; it < 8; ++it)
-    x[it] = rbase + it * 4 < M ? *reinterpret_cast<const float4*>(out + (long long)(rbase + it * 4) * e.ld0)
-                               : make_float4(0.f, 0.f, 0.f, 0.f);
+    x[it] = rbase + it * 4 < M ? __ldcg(reinterpret_cast<const float4*>(out + (long long)(rbase + it * 4) * e.ld0))
+                               : make_float4(0.f, 0.f, 0.f, 0.f);   // L2: split-K partners write from other SMs
   float4 g = make_float4(1.f, 1.f, 1.f, 1.f);
   if (mode == EPI_RESID_GATE) g = __ldg(reinterpret_cast<const float4*>(e.gate + col));
   if (mode == EPI_CFG_EULER) {  // a = v_c; out1 holds v_u: a <- v_u + alpha (v_c - v_u)
@@ -305,6 +317,71 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpi& e, int M, int row0
                                  x[it].w + g.w * a[it].w);
     if (rbase + it * 4 < M) *reinterpret_cast<float4*>(out + (long long)(rbase + it * 4) * e.ld0) = y;
   }
+}
+
+__device__ __forceinline__ void epilogue_chunk(const GemmEpi& e, int M, int row0, int n0, const uint32_t (&r)[32],
+                                               float* stg, int lane) {
+  float4 a[8];
+  stage_chunk(r, stg, lane, a);
+  finish_chunk(e, M, row0, n0, a, lane);
+}
+
+// split-K epilogue of one epilogue warp (32 rows x BN of one output tile): store the fp32 partial
+// (row-coalesced) into its workspace slot; the last of the args.splits partials to arrive (counter
+// per slot) sums them in split order 0..splits-1 and runs the tile's epilogue.  `slot` indexes the
+// warp's rows inside the tile (nslot per tile); the counter is re-armed to 0 for the next launch.
+template <int BN>
+__device__ __forceinline__ void split_epilogue(const GemmArgs& args, const GemmEpi& epi, int Mp, int row0, int n_blk,
+                                               uint32_t tbase, float* stg, int lane, int t0, int sp, int slot,
+                                               int nslot) {
+  const size_t part = (size_t)32 * BN;
+  auto ws_at = [&](int s) { return args.ws + ((size_t)(s * args.tiles_per_split + t0) * nslot + slot) * part; };
+  const int c4 = lane & 7;
+  float* mine = ws_at(sp) + (size_t)(lane >> 3) * BN + c4 * 4;
+#pragma unroll 1
+  for (int c = 0; c < BN / 32; ++c) {
+    uint32_t r[32];
+    tmem_ld32(tbase + c * 32, r);
+    tmem_ld_wait();
+    float4 a[8];
+    stage_chunk(r, stg, lane, a);
+#pragma unroll
+    for (int it = 0; it < 8; ++it) __stcg(reinterpret_cast<float4*>(mine + (size_t)it * 4 * BN + c * 32), a[it]);
+  }
+  __threadfence();
+  __syncwarp();
+  int* cnt = args.sem + t0 * nslot + slot;
+  int done = 0;
+  if (lane == 0) done = atomicAdd(cnt, 1);
+  done = __shfl_sync(0xffffffffu, done, 0);
+  if (done != args.splits - 1) return;
+  __threadfence();
+#pragma unroll 1
+  for (int c = 0; c < BN / 32; c += 2) {   // two chunks per round: 16 independent L2 loads in flight
+    float4 a[2][8];
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+      for (int it = 0; it < 8; ++it) a[h][it] = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll 1
+    for (int s2 = 0; s2 < args.splits; ++s2) {   // fixed order: deterministic whoever arrives last
+      const float* src = ws_at(s2) + (size_t)(lane >> 3) * BN + c4 * 4 + c * 32;
+      float4 u[2][8];
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int it = 0; it < 8; ++it) u[h][it] = __ldcg(reinterpret_cast<const float4*>(src + (size_t)it * 4 * BN + h * 32));
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int it = 0; it < 8; ++it) {
+          a[h][it].x += u[h][it].x; a[h][it].y += u[h][it].y; a[h][it].z += u[h][it].z; a[h][it].w += u[h][it].w;
+        }
+    }
+    finish_chunk(epi, Mp, row0, n_blk * BN + c * 32, a[0], lane);
+    finish_chunk(epi, Mp, row0, n_blk * BN + (c + 1) * 32, a[1], lane);
+  }
+  if (lane == 0) *cnt = 0;   // re-armed for the next launch (the kernel boundary orders it)
 }
 
 template <int BN>
@@ -350,14 +427,22 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   // The weights (B) do not depend on the previous kernel: the first stages of the first tile are
   // requested before the programmatic-dependency wait, so their HBM latency overlaps the previous
   // kernel's tail.  A (and the fp32 stream) come from the previous kernel: after the wait.
+  // split-K range of tile t
+  auto krange = [&](int t, int& t0, int& s, int& kb0, int& kb1) {
+    s = t / args.tiles_per_split;
+    t0 = t - s * args.tiles_per_split;
+    kb0 = s * args.kps;
+    kb1 = min(num_k, kb0 + args.kps);
+  };
   int npre = 0;
   if (warp == 0 && lane == 0 && (int)blockIdx.x < args.num_tiles) {
-    int pr, m_blk, n_blk;
-    decode_tile(args, blockIdx.x, pr, m_blk, n_blk);
-    npre = num_k < C::STAGES ? num_k : C::STAGES;
-    for (int kb = 0; kb < npre; ++kb) {
-      mbar_arrive_expect_tx(&full[kb], C::STAGE_BYTES);
-      tma_load_2d(&maps.B[pr], &full[kb], sB + kb * C::B_BYTES, kb * BK, n_blk * BN);
+    int pr, m_blk, n_blk, t0, sp, kb0, kb1;
+    krange(blockIdx.x, t0, sp, kb0, kb1);
+    decode_tile(args, t0, pr, m_blk, n_blk);
+    npre = kb1 - kb0 < C::STAGES ? kb1 - kb0 : C::STAGES;
+    for (int i = 0; i < npre; ++i) {
+      mbar_arrive_expect_tx(&full[i], C::STAGE_BYTES);
+      tma_load_2d(&maps.B[pr], &full[i], sB + i * C::B_BYTES, (kb0 + i) * BK, n_blk * BN);
     }
   }
   grid_dep_wait();
@@ -368,13 +453,14 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       int stage = 0;
       uint32_t phase = 0;
       for (int t = blockIdx.x; t < args.num_tiles; t += gridDim.x) {
-        int pr, m_blk, n_blk;
-        decode_tile(args, t, pr, m_blk, n_blk);
+        int pr, m_blk, n_blk, t0, sp, kb0, kb1;
+        krange(t, t0, sp, kb0, kb1);
+        decode_tile(args, t0, pr, m_blk, n_blk);
         const CUtensorMap* tA = &maps.A[pr];
         const CUtensorMap* tB = &maps.B[pr];
-        for (int kb = 0; kb < num_k; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          const bool pre = t == (int)blockIdx.x && kb < npre;   // B already requested
+          const bool pre = t == (int)blockIdx.x && kb - kb0 < npre;   // B already requested
           if (!pre) mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
           tma_load_2d(tA, &full[stage], sA + stage * C::A_BYTES, kb * BK, m_blk * BM);
           if (!pre) tma_load_2d(tB, &full[stage], sB + stage * C::B_BYTES, kb * BK, n_blk * BN);
@@ -391,21 +477,24 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
     uint32_t phase = 0;
     int it = 0;
     for (int t = blockIdx.x; t < args.num_tiles; t += gridDim.x, ++it) {
+      int t0, sp, kb0, kb1;
+      krange(t, t0, sp, kb0, kb1);
       const int acc = it & 1;
       const uint32_t acc_phase = (it >> 1) & 1;
       mbar_wait(&tempty[acc], acc_phase ^ 1);
       tc_fence_after();
       const uint32_t d_tmem = tmem_base + acc * BN;
-      for (int kb = 0; kb < num_k; ++kb) {
+      for (int kb = kb0; kb < kb1; ++kb) {
         mbar_wait(&full[stage], phase);
         tc_fence_after();
         const uint64_t da = da0 + (uint64_t)((stage * C::A_BYTES) >> 4);
         const uint64_t db = db0 + (uint64_t)((stage * C::B_BYTES) >> 4);
         if (elect_one()) {
 #pragma unroll
-          for (int k = 0; k < BK / 16; ++k) umma_bf16_ss(d_tmem, da + 2 * k, db + 2 * k, idesc, (kb | k) != 0);
+          for (int k = 0; k < BK / 16; ++k)
+            umma_bf16_ss(d_tmem, da + 2 * k, db + 2 * k, idesc, (kb != kb0 || k != 0) ? 1u : 0u);
           umma_commit(&empty[stage]);
-          if (kb == num_k - 1) umma_commit(&tfull[acc]);
+          if (kb == kb1 - 1) umma_commit(&tfull[acc]);
         }
         __syncwarp();
         if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
@@ -417,8 +506,9 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
     float* stg = stg_all + wq * STG_FLOATS;
     int it = 0;
     for (int t = blockIdx.x; t < args.num_tiles; t += gridDim.x, ++it) {
-      int pr, m_blk, n_blk;
-      decode_tile(args, t, pr, m_blk, n_blk);
+      int pr, m_blk, n_blk, t0, sp, kb0, kb1;
+      krange(t, t0, sp, kb0, kb1);
+      decode_tile(args, t0, pr, m_blk, n_blk);
       const GemmEpi& epi = args.epi[pr];
       const int Mp = args.M[pr];
       const int acc = it & 1;
@@ -427,7 +517,9 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       tc_fence_after();
       const int row0 = m_blk * BM + wq * 32;
       const uint32_t tbase = tmem_base + ((uint32_t)(wq * 32) << 16) + acc * BN;
-      if (epi.qk_h > 0 && n_blk * BN < 3 * epi.qk_h) {
+      if (args.splits > 1) {
+        split_epilogue<BN>(args, epi, Mp, row0, n_blk, tbase, stg, lane, t0, sp, wq, 4);
+      } else if (epi.qk_h > 0 && n_blk * BN < 3 * epi.qk_h) {
 #pragma unroll 1
         for (int hd = 0; hd < BN / epi.qk_D; ++hd)
           epilogue_qk_head(epi, Mp, row0, n_blk * BN + hd * epi.qk_D, tbase + hd * epi.qk_D, stg, lane);
@@ -513,14 +605,21 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
   // weights of the first stages before the programmatic-dependency wait (see gemm_tc_kernel)
+  auto krange = [&](int t, int& t0, int& s, int& kb0, int& kb1) {   // split-K range (see GemmArgs)
+    s = t / args.tiles_per_split;
+    t0 = t - s * args.tiles_per_split;
+    kb0 = s * args.kps;
+    kb1 = min(num_k, kb0 + args.kps);
+  };
   int npre = 0;
   if (warp == 0 && lane == 0 && cid < args.num_tiles) {
-    int pr, m_blk, n_blk;
-    decode_tile(args, cid, pr, m_blk, n_blk);
-    npre = num_k < C::STAGES ? num_k : C::STAGES;
-    for (int kb = 0; kb < npre; ++kb) {
-      if (leader) mbar_arrive_expect_tx(&full[kb], 2 * C::STAGE_BYTES);
-      tma_load_2d_pair(&maps.B[pr], &full[kb], sB + kb * C::B_BYTES, kb * BK, n_blk * BN + (int)rank * (BN / 2));
+    int pr, m_blk, n_blk, t0, sp, kb0, kb1;
+    krange(cid, t0, sp, kb0, kb1);
+    decode_tile(args, t0, pr, m_blk, n_blk);
+    npre = kb1 - kb0 < C::STAGES ? kb1 - kb0 : C::STAGES;
+    for (int i = 0; i < npre; ++i) {
+      if (leader) mbar_arrive_expect_tx(&full[i], 2 * C::STAGE_BYTES);
+      tma_load_2d_pair(&maps.B[pr], &full[i], sB + i * C::B_BYTES, (kb0 + i) * BK, n_blk * BN + (int)rank * (BN / 2));
     }
   }
   grid_dep_wait();  // A (and the fp32 stream) come from the previous kernel
@@ -530,13 +629,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
       int stage = 0;
       uint32_t phase = 0;
       for (int t = cid; t < args.num_tiles; t += ncl) {
-        int pr, m_blk, n_blk;
-        decode_tile(args, t, pr, m_blk, n_blk);
+        int pr, m_blk, n_blk, t0, sp, kb0, kb1;
+        krange(t, t0, sp, kb0, kb1);
+        decode_tile(args, t0, pr, m_blk, n_blk);
         const CUtensorMap* tA = &maps.A[pr];
         const CUtensorMap* tB = &maps.B[pr];
-        for (int kb = 0; kb < num_k; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          const bool pre = t == cid && kb < npre;   // B already requested
+          const bool pre = t == cid && kb - kb0 < npre;   // B already requested
           if (leader && !pre) mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
           tma_load_2d_pair(tA, &full[stage], sA + stage * C::A_BYTES, kb * BK, m_blk * 256 + (int)rank * 128);
           if (!pre)
@@ -554,12 +654,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
       uint32_t phase = 0;
       int it = 0;
       for (int t = cid; t < args.num_tiles; t += ncl, ++it) {
+        int t0, sp, kb0, kb1;
+        krange(t, t0, sp, kb0, kb1);
         const int acc = it & 1;
         const uint32_t acc_phase = (it >> 1) & 1;
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + acc * BN;
-        for (int kb = 0; kb < num_k; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&full[stage], phase);
           tc_fence_after();
           const uint64_t da = da0 + (uint64_t)((stage * C::A_BYTES) >> 4);
@@ -567,9 +669,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
           if (elect_one()) {
 #pragma unroll
             for (int k = 0; k < BK / 16; ++k)
-              umma_bf16_ss_pair(d_tmem, da + 2 * k, db + 2 * k, idesc, (kb | k) != 0);
+              umma_bf16_ss_pair(d_tmem, da + 2 * k, db + 2 * k, idesc, (kb != kb0 || k != 0) ? 1u : 0u);
             umma_commit_pair(&empty[stage]);
-            if (kb == num_k - 1) umma_commit_pair(&tfull[acc]);
+            if (kb == kb1 - 1) umma_commit_pair(&tfull[acc]);
           }
           __syncwarp();
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
@@ -581,8 +683,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
     float* stg = stg_all + wq * STG_FLOATS;
     int it = 0;
     for (int t = cid; t < args.num_tiles; t += ncl, ++it) {
-      int pr, m_blk, n_blk;
-      decode_tile(args, t, pr, m_blk, n_blk);
+      int pr, m_blk, n_blk, t0, sp, kb0, kb1;
+      krange(t, t0, sp, kb0, kb1);
+      decode_tile(args, t0, pr, m_blk, n_blk);
       const GemmEpi& epi = args.epi[pr];
       const int Mp = args.M[pr];
       const int acc = it & 1;
@@ -591,7 +694,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
       tc_fence_after();
       const int row0 = m_blk * 256 + (int)rank * 128 + wq * 32;
       const uint32_t tbase = tmem_base + ((uint32_t)(wq * 32) << 16) + acc * BN;
-      if (epi.qk_h > 0 && n_blk * BN < 3 * epi.qk_h) {
+      if (args.splits > 1) {
+        split_epilogue<BN>(args, epi, Mp, row0, n_blk, tbase, stg, lane, t0, sp, (int)rank * 4 + wq, 8);
+      } else if (epi.qk_h > 0 && n_blk * BN < 3 * epi.qk_h) {
 #pragma unroll 1
         for (int hd = 0; hd < BN / epi.qk_D; ++hd)
           epilogue_qk_head(epi, Mp, row0, n_blk * BN + hd * epi.qk_D, tbase + hd * epi.qk_D, stg, lane);
@@ -662,9 +767,16 @@ static const char* check_epi(const GemmEpi& epi, int bn) {
 }
 
 int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int K, int num_sms, const char** err,
-                    int force_bn, int force_pair) {
+                    int force_bn, int force_pair, const GemmSplitWs* sws, int force_splits) {
   *err = nullptr;
-  if (nprob < 1 || nprob > GEMM_MAX_PROBLEMS) { *err = "gemm: 1 to 16 problems per launch"; return -1; }
+  p->splits = 1; p->kps = K / BK; p->sem = nullptr; p->ws = nullptr;
+  // Split-K for launches too small to fill the GPU (small M: the text stream, SP = 4/8 shards,
+  // 256^2 / 512^2 at k >= 2), for the fp32-accumulating epilogues only (x += g (acc + b) is linear
+  // in acc).  Few tiles otherwise leave most SMs idle while the weights stream through a handful of
+  // them (each SM pulls ~64 B/clk from L2: a weight-streaming GEMM needs most of the 148 SMs).
+  bool split_ok = sws != nullptr && sws->sem && sws->ws;
+  for (int q = 0; q < nprob && split_ok; ++q)
+    split_ok = (probs[q].epi.mode == EPI_RESID_GATE || probs[q].epi.mode == EPI_ACCUM_F32) && !probs[q].epi.qk_h;
   if (N <= 0 || K <= 0) { *err = "gemm: empty shape"; return -1; }
   if (K % BK) { *err = "gemm: K must be a multiple of 64"; return -1; }
   if (N % 64) { *err = "gemm: N must be a multiple of 64"; return -1; }
@@ -740,13 +852,50 @@ int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int
   }
   p->M = probs[0].M;
   p->epi = probs[0].epi;
+  int want_splits = 1;
+  if (split_ok) {
+    const int num_k = K / BK;
+    const long long units = pair ? num_sms / 2 : num_sms;   // clusters or CTAs
+    if (force_splits > 0) {
+      want_splits = force_splits;
+    } else if (tiles * 2 <= units) {
+      want_splits = (int)(units / tiles);
+      if (want_splits > num_k / 4) want_splits = num_k / 4;   // >= 256 of K per split
+      if (want_splits > 4) want_splits = 4;   // measured: the in-order reduction makes S > 4 lose
+    }
+    const long long per_split = (long long)tiles * bm * bn * 4;   // fp32 partials
+    if (want_splits * per_split > sws->ws_bytes) want_splits = (int)(sws->ws_bytes / per_split);
+    if ((long long)tiles * (pair ? 8 : 4) > sws->sem_ints) want_splits = 1;
+  }
+  if (want_splits > 1) {
+    const int num_k = K / BK;
+    int kps = (num_k + want_splits - 1) / want_splits;
+    if (kps < 1) kps = 1;
+    p->splits = (num_k + kps - 1) / kps;
+    p->kps = kps;
+    if (p->splits > 1) {
+      p->sem = sws->sem;
+      p->ws = sws->ws;
+      p->tiles = tiles * p->splits;
+      if (pair) {
+        const int clusters = p->tiles < num_sms / 2 ? p->tiles : num_sms / 2;
+        p->grid = 2 * clusters;
+      } else {
+        p->grid = p->tiles < num_sms ? p->tiles : num_sms;
+      }
+    } else {
+      p->splits = 1;
+      p->kps = num_k;
+    }
+  }
   return 0;
 }
 
 int gemm_plan(GemmPlan* p, const bf16* A, long long lda, const bf16* W, long long ldw, int M, int N, int K,
-              const GemmEpi& epi, int num_sms, const char** err, int force_bn, int force_pair) {
+              const GemmEpi& epi, int num_sms, const char** err, int force_bn, int force_pair, const GemmSplitWs* sws,
+              int force_splits) {
   GemmProblem g{A, lda, W, ldw, M, epi};
-  return gemm_plan_multi(p, &g, 1, N, K, num_sms, err, force_bn, force_pair);
+  return gemm_plan_multi(p, &g, 1, N, K, num_sms, err, force_bn, force_pair, sws, force_splits);
 }
 
 template <int BN>
@@ -763,6 +912,7 @@ static void launch_bn(const GemmPlan& p, cudaStream_t s) {
   GemmMaps maps;
   const int bm = p.pair ? 256 : BM;
   a.N = p.N; a.K = p.K; a.num_n = p.N / BN; a.num_tiles = p.tiles; a.nprob = p.nprob;
+  a.splits = p.splits; a.kps = p.kps; a.tiles_per_split = p.tiles / p.splits; a.sem = p.sem; a.ws = p.ws;
   for (int q = 0; q < GEMM_MAX_PROBLEMS; ++q) {
     const int qq = q < p.nprob ? q : 0;
     a.M[q] = p.Mq[qq];

@@ -112,17 +112,33 @@ struct GemmPlan {
   int BN = 256;
   int tiles = 0, grid = 0;
   bool pair = false;  // CTA-pair (cta_group::2) 256 x 256 tiles
+  int splits = 1;     // split-K factor (1-CTA tiles, fp32-accumulating epilogues only)
+  int kps = 0;        // k-blocks (of 64) per split
+  int* sem = nullptr; // split-K arrival counters, 4 per output tile, zero between launches
+  float* ws = nullptr; // split-K partials
   GemmEpi epi;
+};
+// split-K workspace of one stream: counters (zeroed once, left zero by every launch) + partials
+struct GemmSplitWs {
+  int* sem = nullptr;
+  int sem_ints = 0;
+  float* ws = nullptr;
+  long long ws_bytes = 0;
 };
 
 // A: [M, K] bf16 row stride lda (elements); W: [N, K] bf16 row stride ldw. K % 64 == 0, N % 64 == 0.
 // Returns 0 on success, nonzero (and sets *err) on invalid arguments.
+// sws: a split-K workspace (per stream: concurrent launches need their own) enables split-K for
+// small launches with fp32-accumulating epilogues; force_splits > 0 requests that factor (tests).
+// Null: no split-K.
 int gemm_plan(GemmPlan* p, const bf16* A, long long lda, const bf16* W, long long ldw, int M, int N, int K,
-              const GemmEpi& epi, int num_sms, const char** err, int force_bn = 0, int force_pair = -1);
+              const GemmEpi& epi, int num_sms, const char** err, int force_bn = 0, int force_pair = -1,
+              const GemmSplitWs* sws = nullptr, int force_splits = 0);
 // One launch for up to GEMM_MAX_PROBLEMS problems sharing N and K (persistent tile loop over all;
 // each problem has its own A, W and epilogue).
 int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int K, int num_sms, const char** err,
-                    int force_bn = 0, int force_pair = -1);
+                    int force_bn = 0, int force_pair = -1, const GemmSplitWs* sws = nullptr,
+                    int force_splits = 0);
 void gemm_launch(const GemmPlan& p, cudaStream_t s);
 
 // ------------------------------------------------------------------ elementwise / norm kernels

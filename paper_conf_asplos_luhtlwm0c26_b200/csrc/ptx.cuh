@@ -225,6 +225,16 @@ TSV_DEV void umma_commit_pair(uint64_t* bar) {
       : "memory");
 }
 
+// ------------------------------------------------------------------ gpu-scope flags
+TSV_DEV int ld_acquire_gpu(const int* p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+TSV_DEV void st_release_gpu(int* p, int v) {
+  asm volatile("st.release.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
 // ------------------------------------------------------------------ numerics
 TSV_DEV float gelu_tanh(float x) {
   // 0.5 x (1 + tanh(sqrt(2/pi) (x + 0.044715 x^3)))

@@ -92,6 +92,50 @@ def test_gemm_integer_exact(tsv, M, N, K, bn, pair):
     assert torch.equal(outb.cpu(), ref_b)
 
 
+@pytest.mark.parametrize("M,N,K", [(1, 3072, 3072), (192, 3072, 12288), (300, 1536, 6144), (576, 3072, 15360),
+                                   (1024, 3072, 3072), (70, 128, 1024)])
+@pytest.mark.parametrize("splits", [0, 2, 5, 16])
+def test_gemm_split_k_integer_exact(tsv, M, N, K, splits):
+    """Split-K into the fp32 stream: integer operands make every partial sum exact, so any split
+    factor (incl. more tiles than SMs: persistent CTAs) must reproduce x0 + A W^T + b bit for bit,
+    and the semaphores must be left re-armed (all zero)."""
+    rng = np.random.default_rng(M + N + K + splits)
+    A = rng.integers(-2, 3, (M, K)).astype(np.float32)
+    W = rng.integers(-2, 3, (N, K)).astype(np.float32)
+    b = rng.integers(-4, 5, N).astype(np.float32)
+    x0 = rng.integers(-100, 101, (M, N)).astype(np.float32)
+    exact = x0.astype(np.float64) + A.astype(np.float64) @ W.astype(np.float64).T + b   # |.| < 2^24
+    x = _f32(x0)
+    sem = torch.zeros(4096, dtype=torch.int32, device="cuda")
+    ws = torch.empty(64 << 18, dtype=torch.float32, device="cuda")
+    tsv.op_gemm_split(_bf16(A), _bf16(W), "ACCUM_F32", x, sem, ws, splits=splits, bias=_bf16(b))
+    torch.cuda.synchronize()
+    assert np.array_equal(x.cpu().numpy().astype(np.float64), exact)
+    assert torch.count_nonzero(sem) == 0
+
+
+def test_gemm_split_k_resid_gate_deterministic(tsv):
+    rng = np.random.default_rng(21)
+    M, N, K = 192, 3072, 12288
+    A = synth.bf16_bits_to_f32(synth.bf16_rne_bits(rng.standard_normal((M, K)).astype(np.float32)))
+    W = synth.bf16_bits_to_f32(synth.bf16_rne_bits((rng.standard_normal((N, K)) / math.sqrt(K)).astype(np.float32)))
+    b = synth.bf16_bits_to_f32(synth.bf16_rne_bits((0.1 * rng.standard_normal(N)).astype(np.float32)))
+    x0 = rng.standard_normal((M, N)).astype(np.float32)
+    gate = rng.standard_normal(N).astype(np.float32)
+    y = A.astype(np.float64) @ W.astype(np.float64).T + b
+    sem = torch.zeros(4096, dtype=torch.int32, device="cuda")
+    ws = torch.empty(64 << 18, dtype=torch.float32, device="cuda")
+    outs = []
+    for splits in (6, 6, 0):
+        x = _f32(x0)
+        tsv.op_gemm_split(_bf16(A), _bf16(W), "RESID_GATE", x, sem, ws, splits=splits, bias=_bf16(b), gate=_f32(gate))
+        torch.cuda.synchronize()
+        assert _rel(_np(x), x0 + gate * y) < 1e-5
+        outs.append(x.cpu())
+    assert torch.equal(outs[0], outs[1])      # fixed split order: run-to-run bitwise
+    assert torch.count_nonzero(sem) == 0
+
+
 def test_gemm_epilogues_vs_oracle(tsv):
     rng = np.random.default_rng(11)
     M, N, K = 200, 768, 512

@@ -30,7 +30,12 @@ def main():
     ap.add_argument("--iters", type=int, default=5)
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r01", "latency_table_model.json"))
     ap.add_argument("--res", default=",".join(str(r) for r in RES))
+    ap.add_argument("--serial", action="store_true",
+                    help="virtual ranks share one stream (TSV_VIRTUAL_SERIAL=1): each rank's kernels run alone "
+                         "on the GPU, so time / k is the per-rank time of a real k-GPU group (minus NVLink)")
     args = ap.parse_args()
+    if args.serial:
+        os.environ["TSV_VIRTUAL_SERIAL"] = "1"
     res_list = [int(r) for r in args.res.split(",")]
     d = tsv.model_preset(args.model)
     h, Lt = d.hidden, d.text_tokens
@@ -75,7 +80,11 @@ def main():
            "roofline_frac": roof, "roofline_peak_tflops": peak / 1e12,
            "efficiency_vs_k1": [[round(row[0] / (k * row[j]), 4) for j, k in enumerate(KS)] for row in table],
            "measured_virtual_ms": [[round(float(x), 4) for x in r] for r in ms],
-           "note": "k=1 measured on one B200; k>1 = (k virtual ranks on one B200) / k + modeled NVLink all-to-all"}
+           "note": "k=1 measured on one B200; k>1 = (k virtual ranks on one B200) / k + modeled NVLink all-to-all"
+                   + ("; virtual ranks serialised on one stream (each kernel alone on the GPU, as on a rank's own "
+                      "GPU)" if args.serial else "; virtual ranks on concurrent streams (overlap: optimistic for "
+                      "small per-rank launches)"),
+           "splitk": os.environ.get("TSV_SPLITK", "1") != "0"}
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     json.dump(out, open(args.out, "w"), indent=1)
     print(json.dumps(out))

@@ -69,6 +69,32 @@ def qkv_epilogue_cases():
                           "fused_tflops": round(2 * M * N * K / fused / 1e9, 1)}), flush=True)
 
 
+def split_cases():
+    # small-M fp32-stream GEMMs (text stream, SP = 4/8 shards): split-K vs one K range
+    sem = torch.zeros(4096, dtype=torch.int32, device="cuda")
+    ws = torch.empty(64 << 18, dtype=torch.float32, device="cuda")
+    for M, N, K in ((64, 3072, 12288), (192, 3072, 12288), (192, 3072, 15360), (576, 3072, 15360),
+                    (576, 3072, 3072), (288, 3072, 12288), (333, 1536, 6144), (1024, 3072, 3072)):
+        A = torch.randn(M, K, device="cuda").to(torch.bfloat16)
+        W = (torch.randn(N, K, device="cuda") / math.sqrt(K)).to(torch.bfloat16)
+        x = torch.zeros(M, N, device="cuda")
+        g = torch.ones(N, device="cuda")
+        res = {}
+        for splits in (1, 0):
+            res[splits] = timeit(lambda: tsv.op_gemm_split(A, W, "RESID_GATE", x, sem, ws, splits=splits, gate=g))
+        if os.environ.get("SPLIT_SWEEP"):
+            sw = {s_: round(timeit(lambda: tsv.op_gemm_split(A, W, "RESID_GATE", x, sem, ws, splits=s_, gate=g)), 4)
+                  for s_ in (2, 3, 4, 6, 8)}
+            one = round(timeit(lambda: tsv.op_gemm(A, W, "RESID_GATE", x, gate=g, force_bn=256, force_pair=0)), 4)
+            print(json.dumps({"op": "gemm_split_sweep", "M": M, "N": N, "K": K, "ms_by_splits": sw,
+                              "ms_1cta_nosplit": one}), flush=True)
+        wbytes = N * K * 2
+        print(json.dumps({"op": "gemm_split", "M": M, "N": N, "K": K, "ms_nosplit": round(res[1], 4),
+                          "ms_auto": round(res[0], 4), "speedup": round(res[1] / res[0], 2),
+                          "tflops_auto": round(2 * M * N * K / res[0] / 1e9, 1),
+                          "weight_GBps_auto": round(wbytes / res[0] / 1e6, 1)}), flush=True)
+
+
 def attn_cases():
     sweep = os.environ.get("ATTN_SWEEP")     # "1": also time the poly-share variants (impl 12..15)
     for L, H, D in ((1536, 24, 128), (4608, 24, 128), (16896, 24, 128), (16896, 3, 128), (1357, 24, 64),
@@ -120,4 +146,4 @@ def qk_cases():
 if __name__ == "__main__":
     which = sys.argv[1:] or ["gemm", "attn", "ln", "qk"]
     for w in which:
-        {"gemm": gemm_cases, "attn": attn_cases, "ln": ln_cases, "qk": qk_cases, "qkv": qkv_epilogue_cases}[w]()
+        {"gemm": gemm_cases, "split": split_cases, "attn": attn_cases, "ln": ln_cases, "qk": qk_cases, "qkv": qkv_epilogue_cases}[w]()
