@@ -149,6 +149,7 @@ struct Slot {
   int device = -1;
   DeviceState* ds = nullptr;
   cudaStream_t stream = nullptr;
+  bool own_stream = true;  // false: shares another slot's stream (TSV_VIRTUAL_SERIAL)
   Workspace ws;
   DevBuf scratch;  // conditioning temporaries
   DevBuf sem;      // split-K arrival counters of this slot's GEMM launches (zero between launches)
@@ -165,14 +166,10 @@ struct Slot {
 };
 constexpr int SEM_INTS = 4096;
 constexpr size_t SPLIT_WS_BYTES = 32u << 20;
-// TSV_SPLITK=0 disables split-K for small GEMM launches (A/B measurements)
-static bool splitk_enabled() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("TSV_SPLITK");
-    v = e ? atoi(e) != 0 : 1;
-  }
-  return v != 0;
+// TSV_SPLITK=0 (read at engine creation) disables split-K for small GEMM launches (A/B measurements)
+static bool splitk_env() {
+  const char* v = getenv("TSV_SPLITK");
+  return v ? atoi(v) != 0 : true;
 }
 
 // per (request, slot): state that depends only on the request
@@ -240,6 +237,7 @@ using namespace tsv;
 struct tsv_engine {
   Model model;
   uint64_t weight_seed = 0;
+  bool splitk = true;      // split-K for small fp32-stream GEMM launches (TSV_SPLITK at creation)
   int rank_base = 0, n_local = 0, world = 0;
   std::vector<Slot> slots;
   std::map<int, std::unique_ptr<DeviceState>> devs;
@@ -314,7 +312,7 @@ static tsv_status gemm(tsv_engine* e, Slot& s, const bf16* A, long long lda, con
   GemmPlan p;
   const char* err = nullptr;
   const GemmSplitWs w = s.sws();
-  if (gemm_plan(&p, A, lda, Wt, ldw, M, N, K, epi, s.ds->num_sms, &err, 0, -1, splitk_enabled() ? &w : nullptr))
+  if (gemm_plan(&p, A, lda, Wt, ldw, M, N, K, epi, s.ds->num_sms, &err, 0, -1, e->splitk ? &w : nullptr))
     return fail(TSV_E_INVAL, "%s (M=%d N=%d K=%d)", err, M, N, K);
   const double out_b = (epi.mode <= EPI_SPLIT_GELU) ? 2.0
                        : (epi.mode == EPI_STORE_F32 ? 4.0 : (epi.mode == EPI_CFG_EULER ? 16.0 : 8.0));
@@ -335,7 +333,7 @@ static tsv_status gemm_multi(tsv_engine* e, Slot& s, const GemmProblem* probs, i
   GemmPlan p;
   const char* err = nullptr;
   const GemmSplitWs w = s.sws();
-  if (gemm_plan_multi(&p, nz, n, N, K, s.ds->num_sms, &err, 0, -1, splitk_enabled() ? &w : nullptr))
+  if (gemm_plan_multi(&p, nz, n, N, K, s.ds->num_sms, &err, 0, -1, e->splitk ? &w : nullptr))
     return fail(TSV_E_INVAL, "%s (N=%d K=%d)", err, N, K);
   double fl = 0, by = 2.0 * N * K * n;
   for (int i = 0; i < n; ++i) {
@@ -1468,6 +1466,7 @@ tsv_status tsv_engine_create(const tsv_model_desc* model, const int* devices, in
   std::string err;
   if (!build_model(*model, &e->model, &err)) return fail(TSV_E_INVAL, "%s", err.c_str());
   e->weight_seed = weight_seed;
+  e->splitk = splitk_env();
   e->rank_base = rank_base;
   e->n_local = n_local;
   e->world = world_size;
@@ -1494,8 +1493,12 @@ tsv_status tsv_engine_create(const tsv_model_desc* model, const int* devices, in
     Slot* first = nullptr;
     for (int j = 0; j < i; ++j)
       if (e->slots[j].device == s.device) { first = &e->slots[j]; break; }
-    if (vs && atoi(vs) && first) s.stream = first->stream;
-    else CK(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+    if (vs && atoi(vs) && first) {
+      s.stream = first->stream;
+      s.own_stream = false;
+    } else {
+      CK(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+    }
     TRY(dev_alloc(s.sem, s.device, SEM_INTS * sizeof(int)));
     CK(cudaMemset(s.sem.p, 0, SEM_INTS * sizeof(int)));
     TRY(dev_alloc(s.splitws, s.device, SPLIT_WS_BYTES));
@@ -1543,10 +1546,10 @@ void tsv_engine_destroy(tsv_engine* e) {
   for (auto& s : e->slots) {
     Workspace& w = s.ws;
     for (DevBuf* b : {&w.x, &w.u, &w.qkv, &w.cat, &w.hbuf, &w.latb, &w.pack, &w.recv, &w.obuf, &w.orecv, &w.bmod,
-                      &s.scratch})
+                      &s.scratch, &s.sem, &s.splitws})
       b->release();
     cudaSetDevice(s.device);
-    cudaStreamDestroy(s.stream);
+    if (s.own_stream) cudaStreamDestroy(s.stream);
   }
   for (auto& d : e->devs) d.second->weights.release();
   delete e;
