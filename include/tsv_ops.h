@@ -93,6 +93,17 @@ tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int
 tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
                             void* o, int64_t ldo, int L, int H, int D, int impl, void* stream);
 
+/* a6 with the key range split (flash-decoding style) for launches with too few CTAs (SP = 4/8 head
+ * shards, small images): nsplit key ranges (0: the engine's automatic choice, possibly 1; capped at
+ * 8 and by the workspace), each range's unnormalised O, reference and sum go to ws and the last
+ * range to finish a query tile merges them in range order (deterministic).  The step's attention
+ * kernel (impl 0).  cnt: zeroed device ints (>= 8 per 256-query block and head), left zero;
+ * ws: fp32 device workspace (nsplit x 2 x 128 x (D + 2) floats per 256-query block and head).
+ * Same operand rules as tsv_op_attention. */
+tsv_status tsv_op_attention_split(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
+                                  void* o, int64_t ldo, int L, int H, int D, int nsplit, int* cnt, int cnt_ints,
+                                  float* ws, int64_t ws_bytes, void* stream);
+
 /* SYNTH-1 on device: n values of (seed, tensor_id) starting at element idx0.
  * kind 0: bf16 rne(r*c); 1: bf16 rne(1 + r*c); 2: fp32 r*c. */
 tsv_status tsv_op_synth(void* dst, uint64_t seed, uint32_t tensor_id, uint64_t idx0, int64_t n, int kind, float c,

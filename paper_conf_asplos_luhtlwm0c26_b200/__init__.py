@@ -289,6 +289,14 @@ def op_qk_norm_rope(qkv, n_first, H, D, gq0, gk0, gq1, gk1, cosb, sinb, pack=Non
                                   _ptr(gk1), _ptr(cosb), _ptr(sinb), _ptr(pack), k_sp, _stream(stream)))
 
 
+def op_attention_split(q, k, v, o, L, H, D, cnt, ws, nsplit=0, ldq=None, ldk=None, ldv=None, ldo=None, stream=None):
+    """The step's attention with the key range split nsplit ways (0: automatic); cnt: zeroed int32
+    device buffer, ws: fp32 device workspace."""
+    check(lib.tsv_op_attention_split(_ptr(q), ldq or q.stride(0), _ptr(k), ldk or k.stride(0), _ptr(v),
+                                     ldv or v.stride(0), _ptr(o), ldo or o.stride(0), L, H, D, nsplit, _ptr(cnt),
+                                     cnt.numel(), _ptr(ws), ws.numel() * 4, _stream(stream)))
+
+
 def op_attention(q, k, v, o, L, H, D, ldq=None, ldk=None, ldv=None, ldo=None, impl=0, stream=None):
     """impl 0: tcgen05 kernel (the step's); impl 1: mma.sync baseline (comparison only)."""
     check(lib.tsv_op_attention(_ptr(q), ldq or q.stride(0), _ptr(k), ldk or k.stride(0), _ptr(v), ldv or v.stride(0),

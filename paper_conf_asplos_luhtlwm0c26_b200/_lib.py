@@ -86,6 +86,8 @@ _SIGS = {
                             _p]),
     "tsv_op_gemm_split": (_i32, [_p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p, _i64, _p, _p, _i32, _p, _i32, _p,
                                   _i64, _p]),
+    "tsv_op_attention_split": (_i32, [_p, _i64, _p, _i64, _p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p, _i32, _p,
+                                       _i64, _p]),
     "tsv_op_gemm_qkv": (_i32, [_p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p, _i64, _p, _i64, _p, _i32, _i32,
                                _p, _p, _p, _p, _i32, _p, _i32, _i32, _p]),
     "tsv_op_ln_mod": (_i32, [_p, _i64, _p, _i64, _p, _p, _i32, _i32, _i32, _p]),

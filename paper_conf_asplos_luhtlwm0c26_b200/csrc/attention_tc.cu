@@ -363,11 +363,19 @@ constexpr int FA_THREADS = 384;
 // a lot: early tiles) the warp reloads S from TMEM and takes the exact path (row max, rescale).
 // Saves the 128 FMNMX per row per tile and the max-before-exp dependency on the softmax chain.
 constexpr float LAZY_LIMIT = 65536.0f;   // 2^16
+// KV split (blockIdx.z = split): see AttnSplitWs.  nsplit = 1: the whole key range, no workspace.
+struct AttnSplitArgs {
+  int nsplit = 1, tps = 0;   // splits, key tiles per split
+  int* cnt = nullptr;
+  float* ws = nullptr;
+};
+
 template <int D, int NPOLY, bool SPLIT, bool LAZY = false>
 __global__ void __launch_bounds__(FA_THREADS, 1)
     attention_fa_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
-                        float scale_log2, const __grid_constant__ AttnScatter sc) {
+                        float scale_log2, const __grid_constant__ AttnScatter sc,
+                        const __grid_constant__ AttnSplitArgs sa) {
   using C = FaCfg<D>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -384,7 +392,10 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int head = blockIdx.y;
   const int q0 = blockIdx.x * 2 * AT_BM;
-  const int n_tiles = (L + AT_BN - 1) / AT_BN;
+  // this CTA's key tiles: [j0, j0 + n_tiles) (all of them unless the launch splits the keys)
+  const int n_all = (L + AT_BN - 1) / AT_BN;
+  const int j0 = sa.nsplit > 1 ? (int)blockIdx.z * sa.tps : 0;
+  const int n_tiles = sa.nsplit > 1 ? min(n_all - j0, sa.tps) : n_all;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tmQ);
@@ -425,9 +436,9 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         mbar_arrive_expect_tx(&kv_full[st], 2 * C::KV_TILE);
         for (int s = 0; s < C::NSUB; ++s) {
           tma_load_3d(&tmK, &kv_full[st], sm + C::OFF_K + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
-                      j * AT_BN);
+                      (j0 + j) * AT_BN);
           tma_load_3d(&tmV, &kv_full[st], sm + C::OFF_V + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
-                      j * AT_BN);
+                      (j0 + j) * AT_BN);
         }
       }
     }
@@ -501,7 +512,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       mbar_wait(&s_full[t], j & 1);
       tc_fence_after();
       uint32_t sr[4][32];
-      const int kbase = j * AT_BN;
+      const int kbase = (j0 + j) * AT_BN;
       const bool full = kbase + AT_BN <= L;
       const bool lazy = LAZY && !SPLIT && j > 0 && full;
       if (!lazy) {
@@ -648,7 +659,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     // epilogue: O_t / l -> bf16
     mbar_wait(&o_done[t], 0);
     tc_fence_after();
-    const float inv = 1.f / l_sum;
+    float inv = 1.f / l_sum;
     const int grow = q0 + t * AT_BM + row;
     // output row: local (plain) or, fused a7, the owning rank's row of its stream-concatenated input
     bf16* orow = o + (long long)grow * ldo + head * D;
@@ -664,6 +675,76 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       }
       orow = sc.dst[p] + (long long)lr * sc.ld + sc.col0 + head * D;
     }
+    if (sa.nsplit > 1) {
+      // KV split: unnormalised O_t (layout [D][128]: coalesced across the warp's rows), reference m
+      // and sum l of this split -> ws; the last split of these 32 rows merges in split order:
+      // O = sum_s 2^(m_s - M) O_s / sum_s 2^(m_s - M) l_s, M = max_s m_s
+      const size_t slab = (size_t)AT_BM * (D + 2);
+      const int nqb = gridDim.x;
+      const size_t qt = ((size_t)head * nqb + blockIdx.x) * 2 + t;   // query tile
+      auto ws_at = [&](int s2) { return sa.ws + (qt * sa.nsplit + s2) * slab; };
+      float* mine = ws_at(blockIdx.z);
+#pragma unroll
+      for (int c = 0; c < D / 32; ++c) {
+        uint32_t ov[32];
+        tmem_ld32(o_col + c * 32, ov);
+        tmem_ld_wait();
+#pragma unroll
+        for (int i = 0; i < 32; ++i) __stcg(mine + (size_t)(c * 32 + i) * AT_BM + row, __uint_as_float(ov[i]));
+      }
+      __stcg(mine + (size_t)D * AT_BM + row, m_ref);
+      __stcg(mine + (size_t)(D + 1) * AT_BM + row, l_sum);
+      __threadfence();
+      __syncwarp();
+      int* cnt = sa.cnt + qt * 4 + wq;
+      int done = 0;
+      if (lane == 0) done = atomicAdd(cnt, 1);
+      done = __shfl_sync(0xffffffffu, done, 0);
+      if (done == sa.nsplit - 1) {
+        __threadfence();
+        float mmax = -FLT_MAX;
+        float ms[8], wsum = 0.f;
+#pragma unroll
+        for (int s2 = 0; s2 < 8; ++s2)
+          if (s2 < sa.nsplit) {
+            ms[s2] = __ldcg(ws_at(s2) + (size_t)D * AT_BM + row);
+            mmax = fmaxf(mmax, ms[s2]);
+          }
+#pragma unroll
+        for (int s2 = 0; s2 < 8; ++s2)
+          if (s2 < sa.nsplit) {
+            ms[s2] = exp2f(ms[s2] - mmax);   // now the merge weight of split s2
+            wsum += ms[s2] * __ldcg(ws_at(s2) + (size_t)(D + 1) * AT_BM + row);
+          }
+        inv = 1.f / wsum;
+#pragma unroll
+        for (int c = 0; c < D / 32; ++c) {
+          float acc[32];
+#pragma unroll
+          for (int i = 0; i < 32; ++i) acc[i] = 0.f;
+#pragma unroll
+          for (int s2 = 0; s2 < 8; ++s2)
+            if (s2 < sa.nsplit) {
+              const float* src = ws_at(s2) + (size_t)(c * 32) * AT_BM + row;
+#pragma unroll
+              for (int i = 0; i < 32; ++i) acc[i] = fmaf(ms[s2], __ldcg(src + (size_t)i * AT_BM), acc[i]);
+            }
+          if (grow < L) {
+            uint4* dst = reinterpret_cast<uint4*>(orow + c * 32);
+#pragma unroll
+            for (int qd = 0; qd < 4; ++qd) {
+              uint4 v;
+              v.x = pack_bf16x2(acc[qd * 8 + 0] * inv, acc[qd * 8 + 1] * inv);
+              v.y = pack_bf16x2(acc[qd * 8 + 2] * inv, acc[qd * 8 + 3] * inv);
+              v.z = pack_bf16x2(acc[qd * 8 + 4] * inv, acc[qd * 8 + 5] * inv);
+              v.w = pack_bf16x2(acc[qd * 8 + 6] * inv, acc[qd * 8 + 7] * inv);
+              dst[qd] = v;
+            }
+          }
+        }
+        if (lane == 0) *cnt = 0;   // re-armed for the next launch
+      }
+    } else
 #pragma unroll
     for (int c = 0; c < D / 32; ++c) {
       uint32_t ov[32];
@@ -1320,7 +1401,8 @@ constexpr int default_npoly() { return D == 64 ? 2 : 1; }   // measured (profile
 
 template <int D, int NP, bool SPLIT = false, bool LAZY = false>
 static void launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
-                      int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s) {
+                      int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s,
+                      const AttnSplitArgs& sa = AttnSplitArgs()) {
   static unsigned long long done = 0;
   int dev = 0;
   cudaGetDevice(&dev);
@@ -1329,9 +1411,9 @@ static void launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtens
                          FaCfg<D>::SMEM);
     done |= 1ull << dev;
   }
-  dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H);
+  dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H, sa.nsplit);
   launch_pdl(attention_fa_kernel<D, NP, SPLIT, LAZY>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo, L, scale_log2,
-             sc);
+             sc, sa);
 }
 
 template <int D, int NP>
@@ -1377,9 +1459,48 @@ static void launch_fa2(const CUtensorMap& tq, const CUtensorMap& tk, const CUten
   cudaLaunchKernelEx(&cfg, attention_fa2_kernel<128, NP>, tq, tk, tv, o, ldo, L, scale_log2, sc);
 }
 
+// KV-split factor for a launch of C = ceil(L/256) x H CTAs: the S in 1..8 minimising the estimated
+// makespan (below), each split >= 4 key tiles.
+static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
+  AttnSplitArgs a;
+  if (!w || !w->cnt || !w->ws) return a;
+  static int sms_of[64] = {0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!sms_of[dev & 63]) cudaDeviceGetAttribute(&sms_of[dev & 63], cudaDevAttrMultiProcessorCount, dev);
+  const int sms = sms_of[dev & 63] ? sms_of[dev & 63] : 148;
+  const int n_all = (L + AT_BN - 1) / AT_BN;
+  const long long C = (long long)((L + 2 * AT_BM - 1) / (2 * AT_BM)) * H;
+  int best = 1;
+  if (w->force > 0) {
+    best = w->force < n_all ? w->force : n_all;
+  } else {
+    // makespan in key-tile units: waves x (tiles per split + fixed cost), the fixed cost (prologue,
+    // pipeline fill, epilogue; + the merge when split) fitted to tools/microbench.py attnsplit
+    double bestc = (double)((C + sms - 1) / sms) * (n_all + 2);
+    for (int S = 2; S <= 8; ++S) {
+      const int tps = (n_all + S - 1) / S;
+      if (tps < 4) break;
+      const double cost = (double)((C * S + sms - 1) / sms) * (tps + 6);
+      if (cost < bestc * 0.95) { bestc = cost; best = S; }
+    }
+  }
+  if (best < 2) return a;
+  const int tps = (n_all + best - 1) / best;
+  best = (n_all + tps - 1) / tps;   // no empty split
+  if (best < 2 || best > 8) return a;
+  if ((long long)C * 2 * best * AT_BM * (D + 2) * 4 > w->ws_bytes || C * 2 * 4 > w->cnt_ints) return a;
+  a.nsplit = best;
+  a.tps = tps;
+  a.cnt = w->cnt;
+  a.ws = w->ws;
+  return a;
+}
+
 template <int D>
 static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv, bf16* o,
-                     long long ldo, int L, int H, int version, const AttnScatter& sc, cudaStream_t s) {
+                     long long ldo, int L, int H, int version, const AttnScatter& sc, cudaStream_t s,
+                     const AttnSplitWs* spw) {
   CUtensorMap tq, tk, tv;
   if (make_tmap_heads(&tq, q, D, H, L, ldq) || make_tmap_heads(&tk, k, D, H, L, ldk) ||
       make_tmap_heads(&tv, v, D, H, L, ldv))
@@ -1419,12 +1540,13 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     return 0;
   }
   if (version >= 50) {   // 50 + n: lazy row max (see attention_fa_kernel), n of 8 exp2 pairs by polynomial
+    const AttnSplitArgs sa = plan_kv_split(L, H, D, spw);
     switch (version - 50) {
-      case 0: launch_fa<D, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      case 1: launch_fa<D, 1, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      case 2: launch_fa<D, 2, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      case 3: launch_fa<D, 3, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      case 4: launch_fa<D, 4, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
+      case 0: launch_fa<D, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+      case 1: launch_fa<D, 1, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+      case 2: launch_fa<D, 2, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+      case 3: launch_fa<D, 3, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+      case 4: launch_fa<D, 4, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
       default: return -3;
     }
     return 0;
@@ -1476,7 +1598,7 @@ static int default_version(int D) {
 // P in shared memory (kept for comparison).
 int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
                      bf16* o, long long ldo, int L, int H, int D, cudaStream_t s, int version,
-                     const AttnScatter* scatter) {
+                     const AttnScatter* scatter, const AttnSplitWs* split) {
   if (L <= 0 || H <= 0) return 0;
   AttnScatter sc;
   if (scatter) {
@@ -1487,8 +1609,8 @@ int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk,
                                         reinterpret_cast<uintptr_t>(v)) & 15))
     return -1;
   if (version == 3) version = default_version(D);
-  if (D == 128) return launch_tc<128>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, sc, s);
-  if (D == 64) return launch_tc<64>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, sc, s);
+  if (D == 128) return launch_tc<128>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, sc, s, split);
+  if (D == 64) return launch_tc<64>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, sc, s, split);
   return -1;
 }
 

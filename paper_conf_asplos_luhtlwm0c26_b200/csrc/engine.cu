@@ -154,6 +154,14 @@ struct Slot {
   DevBuf scratch;  // conditioning temporaries
   DevBuf sem;      // split-K arrival counters of this slot's GEMM launches (zero between launches)
   DevBuf splitws;  // split-K partials
+  AttnSplitWs aws() const {   // the attention's KV split reuses the GEMM split-K buffers (same stream)
+    AttnSplitWs w;
+    w.cnt = reinterpret_cast<int*>(sem.p);
+    w.cnt_ints = (int)(sem.bytes / sizeof(int));
+    w.ws = reinterpret_cast<float*>(splitws.p);
+    w.ws_bytes = (long long)splitws.bytes;
+    return w;
+  }
   GemmSplitWs sws() const {
     GemmSplitWs w;
     w.sem = reinterpret_cast<int*>(sem.p);
@@ -165,7 +173,7 @@ struct Slot {
   std::map<uint64_t, StepGraph> graphs;
 };
 constexpr int SEM_INTS = 4096;
-constexpr size_t SPLIT_WS_BYTES = 32u << 20;
+constexpr size_t SPLIT_WS_BYTES = 128u << 20;
 // TSV_SPLITK=0 (read at engine creation) disables split-K for small GEMM launches (A/B measurements)
 static bool splitk_env() {
   const char* v = getenv("TSV_SPLITK");
@@ -759,11 +767,13 @@ static tsv_status attention_all(StepEnv& E) {
     const double Lq = k == 1 ? (double)c.rows : (double)L;
     for (int b = 0; b < E.B; ++b) {  // one launch per evaluation (request x CFG branch)
       ProfScope ps(e, *c.s, KC_ATTN, 4.0 * Lq * Lq * m.D * (m.H / k), 8.0 * Lq * m.D * (m.H / k));
+      const AttnSplitWs kvw = c.s->aws();
+      const AttnSplitWs* kvs = e->splitk ? &kvw : nullptr;
       int rc;
       if (k == 1) {
         const bf16* q = c.qkv + b * c.rows * 3 * m.h;
         rc = attention_launch(q, 3 * m.h, q + m.h, 3 * m.h, q + 2 * m.h, 3 * m.h, c.cat + b * c.rows * (m.h + m.F),
-                              m.h + m.F, (int)c.rows, m.H, m.D, c.s->stream);
+                              m.h + m.F, (int)c.rows, m.H, m.D, c.s->stream, 3, nullptr, kvs);
       } else if (E.fused) {
         // fused a7: each output row goes straight to its owner's cat[:, r*h/k + ...]
         const int64_t w = 3 * (int64_t)m.h / k;
@@ -782,12 +792,12 @@ static tsv_status attention_all(StepEnv& E) {
         sc.t_off[k] = (int)E.R->Lt;
         sc.i_off[k] = (int)E.R->Li;
         rc = attention_launch(q, w, q + m.h / k, w, q + 2 * m.h / k, w, nullptr, 0, (int)L, m.H / k, m.D, c.s->stream,
-                              3, &sc);
+                              3, &sc, kvs);
       } else {
         const int64_t w = 3 * (int64_t)m.h / k;
         const bf16* q = c.recv + b * L * w;
         rc = attention_launch(q, w, q + m.h / k, w, q + 2 * m.h / k, w, c.obuf + b * L * (m.h / k), m.h / k, (int)L,
-                              m.H / k, m.D, c.s->stream);
+                              m.H / k, m.D, c.s->stream, 3, nullptr, kvs);
       }
       if (rc) return fail(TSV_E_CUDA, "attention: tensor map creation failed");
     }
@@ -2216,6 +2226,25 @@ tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t l
                               reinterpret_cast<cudaStream_t>(stream), impl == 0 ? 3 : impl)) {
     return fail(TSV_E_INVAL, "attention: operands must be 16-byte aligned with 16-byte row strides");
   }
+  CK(cudaGetLastError());
+  return TSV_OK;
+}
+
+tsv_status tsv_op_attention_split(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
+                                  void* o, int64_t ldo, int L, int H, int D, int nsplit, int* cnt, int cnt_ints,
+                                  float* ws, int64_t ws_bytes, void* stream) {
+  if (D != 64 && D != 128) return fail(TSV_E_INVAL, "D must be 64 or 128");
+  if (!cnt || !ws || nsplit < 0) return fail(TSV_E_INVAL, "KV split needs counters, a workspace and nsplit >= 0");
+  AttnSplitWs w;
+  w.cnt = cnt;
+  w.cnt_ints = cnt_ints;
+  w.ws = ws;
+  w.ws_bytes = ws_bytes;
+  w.force = nsplit;
+  if (attention_launch(reinterpret_cast<const bf16*>(q), ldq, reinterpret_cast<const bf16*>(k), ldk,
+                       reinterpret_cast<const bf16*>(v), ldv, reinterpret_cast<bf16*>(o), ldo, L, H, D,
+                       reinterpret_cast<cudaStream_t>(stream), 3, nullptr, &w))
+    return fail(TSV_E_INVAL, "attention: operands must be 16-byte aligned with 16-byte row strides");
   CK(cudaGetLastError());
   return TSV_OK;
 }

@@ -170,9 +170,20 @@ void qk_norm_rope_launch(bf16* qkv, long long ld, int rows, int n_first, int H, 
 // attention_launch: tcgen05/TMEM kernel (returns nonzero if the layout is not TMA-compatible).
 // attention_mma_launch: the mma.sync (FA2-style) baseline kept for comparison.
 // q(l, h) at q + l*ldq + h*D (same for k, v, o). L rows.
+// KV-split (flash-decoding style) for launches with too few CTAs to fill the GPU (SP = 4/8 head
+// shards, small images): split s of a (query block, head) covers key tiles [s tps, (s+1) tps);
+// each split stores its unnormalised O (fp32, [D][128] per query tile), reference m and sum l to ws
+// and the last split of a query-tile warp (counter in cnt) merges them in split order.
+struct AttnSplitWs {
+  int* cnt = nullptr;   // zero on entry, left zero
+  int cnt_ints = 0;
+  float* ws = nullptr;
+  long long ws_bytes = 0;
+  int force = 0;        // > 0: this split factor (tests); 0: automatic
+};
 int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
                      bf16* o, long long ldo, int L, int H, int D, cudaStream_t s, int version = 3,
-                     const AttnScatter* scatter = nullptr);
+                     const AttnScatter* scatter = nullptr, const AttnSplitWs* split = nullptr);
 void attention_mma_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
                           bf16* o, long long ldo, int L, int H, int D, cudaStream_t s);
 

@@ -274,6 +274,36 @@ def test_attention(tsv, L, H, D, impl):
     assert torch.count_nonzero(o[:, H * D:]) == 0
 
 
+@pytest.mark.parametrize("L,H,D", [(1000, 3, 128), (1536, 3, 128), (4700, 1, 128), (1357, 2, 64), (4429, 3, 64),
+                                   (600, 1, 64)])
+@pytest.mark.parametrize("nsplit", [0, 2, 3, 8])
+def test_attention_kv_split(tsv, L, H, D, nsplit):
+    """KV split: each key range's partial (O, m, l) merged in range order equals softmax attention
+    (oracle), is deterministic run to run, and leaves the counters re-armed."""
+    rng = np.random.default_rng(L * 3 + H + D + nsplit)
+    qkv = rng.standard_normal((L, 3, H, D)).astype(np.float32) * np.float32(1.5)
+    qkv = synth.bf16_bits_to_f32(synth.bf16_rne_bits(qkv)).astype(np.float64)
+    qkv[L // 2:, 1] += 0.8          # later keys score higher: the ranges' references differ
+    qkv = synth.bf16_bits_to_f32(synth.bf16_rne_bits(qkv.astype(np.float32))).astype(np.float64)
+    ref = F.attention(qkv[:, 0], qkv[:, 1], qkv[:, 2])
+    t = _bf16(qkv.reshape(L, 3 * H * D))
+    ld = 3 * H * D
+    cnt = torch.zeros(4096, dtype=torch.int32, device="cuda")
+    ws = torch.empty(16 << 20, dtype=torch.float32, device="cuda")
+    outs = []
+    for _ in range(2):
+        o = torch.zeros(L, H * D, dtype=torch.bfloat16, device="cuda")
+        tsv.op_attention_split(t, t[:, H * D:], t[:, 2 * H * D:], o, L, H, D, cnt, ws, nsplit=nsplit, ldq=ld, ldk=ld,
+                               ldv=ld)
+        torch.cuda.synchronize()
+        outs.append(o.cpu())
+        got = _np(o).reshape(L, H, D)
+        assert _rel(got, ref) < 1.5e-2
+        assert np.sum(got * ref) / np.linalg.norm(got) / np.linalg.norm(ref) > 0.9999
+    assert torch.equal(outs[0], outs[1])
+    assert torch.count_nonzero(cnt) == 0
+
+
 def test_attention_special_cases(tsv):
     # identical keys -> mean(V) (S:§8(c) P3)
     L, H, D = 300, 2, 128

@@ -95,6 +95,27 @@ def split_cases():
                           "weight_GBps_auto": round(wbytes / res[0] / 1e6, 1)}), flush=True)
 
 
+def attn_split_cases():
+    # SP = 4/8 head shards (few CTAs): KV split (auto) vs one key range
+    cnt = torch.zeros(4096, dtype=torch.int32, device="cuda")
+    ws = torch.empty(32 << 20, dtype=torch.float32, device="cuda")
+    for L, H, D in ((16896, 3, 128), (16896, 6, 128), (4608, 3, 128), (4608, 6, 128), (1536, 3, 128),
+                    (1536, 6, 128), (16717, 3, 64), (4429, 3, 64), (1357, 3, 64)):
+        qkv = torch.randn(L, 3 * H * D, device="cuda").to(torch.bfloat16)
+        o = torch.empty(L, H * D, dtype=torch.bfloat16, device="cuda")
+        ld = 3 * H * D
+        res = {}
+        for ns in (1, 0):
+            f = lambda: tsv.op_attention_split(qkv, qkv[:, H * D:], qkv[:, 2 * H * D:], o, L, H, D, cnt, ws,
+                                               nsplit=ns, ldq=ld, ldk=ld, ldv=ld)
+            res[ns] = timeit(f, iters=10 if L > 8000 else 30)
+        fl = 4 * L * L * D * H
+        print(json.dumps({"op": "attention_kv_split", "L": L, "H": H, "D": D, "ms_one": round(res[1], 4),
+                          "ms_auto": round(res[0], 4), "speedup": round(res[1] / res[0], 2),
+                          "tflops_one": round(fl / res[1] / 1e9, 1), "tflops_auto": round(fl / res[0] / 1e9, 1)}),
+              flush=True)
+
+
 def attn_cases():
     sweep = os.environ.get("ATTN_SWEEP")     # "1": also time the poly-share variants (impl 12..15)
     for L, H, D in ((1536, 24, 128), (4608, 24, 128), (16896, 24, 128), (16896, 3, 128), (1357, 24, 64),
@@ -146,4 +167,4 @@ def qk_cases():
 if __name__ == "__main__":
     which = sys.argv[1:] or ["gemm", "attn", "ln", "qk"]
     for w in which:
-        {"gemm": gemm_cases, "split": split_cases, "attn": attn_cases, "ln": ln_cases, "qk": qk_cases, "qkv": qkv_epilogue_cases}[w]()
+        {"gemm": gemm_cases, "split": split_cases, "attnsplit": attn_split_cases, "attn": attn_cases, "ln": ln_cases, "qk": qk_cases, "qkv": qkv_epilogue_cases}[w]()
