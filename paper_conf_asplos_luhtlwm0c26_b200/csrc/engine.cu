@@ -303,15 +303,20 @@ struct ProfScope {
     e->prof_launch[cls] += 1;
     a = pool_event(e, s->device);
     // External: inside a step-graph capture this becomes an event-record node replayed with
-    // the graph (a plain record would only add an intra-graph dependency).
-    cudaEventRecordWithFlags(a, s->stream, cudaEventRecordExternal);
+    // the graph (a plain record would only add an intra-graph dependency).  Outside a capture
+    // (direct launches: k > 1 with several local ranks) the flag is invalid: plain record.
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    cudaStreamIsCapturing(s->stream, &cs);
+    flags = cs == cudaStreamCaptureStatusActive ? cudaEventRecordExternal : cudaEventRecordDefault;
+    cudaEventRecordWithFlags(a, s->stream, flags);
   }
   ~ProfScope() {
     if (!a) return;
     cudaEvent_t b = pool_event(e, s->device);
-    cudaEventRecordWithFlags(b, s->stream, cudaEventRecordExternal);
+    cudaEventRecordWithFlags(b, s->stream, flags);
     e->prof_recs.push_back({cls, s->device, a, b});
   }
+  unsigned flags = cudaEventRecordDefault;
 };
 
 static tsv_status gemm(tsv_engine* e, Slot& s, const bf16* A, long long lda, const bf16* Wt, long long ldw, int M,
