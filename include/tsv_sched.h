@@ -38,6 +38,14 @@ tsv_status tsv_sched_allocate(const double* T, int n_res, const int* ks, int n_k
 tsv_status tsv_sched_round(const double* T, int n_res, const int* ks, int n_k, const tsv_sched_request* reqs, int R,
                            double now, double tau, int N, int* gpus_out, int* steps_out, int* survivors);
 
+/* tsv_sched_round with the tie at Alg. 1 line 21 (several capacities c attaining the optimum)
+ * selectable: work_conserving = 0 takes the smallest c (= tsv_sched_round, reading S31: requests
+ * with slack are deferred), != 0 the largest (reading S31b: every request that can make progress
+ * now runs at its minimal allocation; the survivor count is the same optimum). */
+tsv_status tsv_sched_round_ex(const double* T, int n_res, const int* ks, int n_k, const tsv_sched_request* reqs,
+                              int R, double now, double tau, int N, int work_conserving, int* gpus_out,
+                              int* steps_out, int* survivors);
+
 /* GPU placement with preservation and elastic scale-up (S:§8(f) NEXT #4).  gpus[i] =
  * GPUs granted to request i this round (0 or a power of two, e.g. tsv_sched_round's gpus_out),
  * rows[i] its table row, prev_mask[i] the bitmask of the GPUs it held in the previous round (0 =

@@ -98,6 +98,8 @@ _SIGS = {
                                   _P(_i32)]),
     "tsv_sched_round": (_i32, [_P(C.c_double), _i32, _P(_i32), _i32, _P(SchedRequest), _i32, C.c_double, C.c_double,
                                _i32, _P(_i32), _P(_i32), _P(_i32)]),
+    "tsv_sched_round_ex": (_i32, [_P(C.c_double), _i32, _P(_i32), _i32, _P(SchedRequest), _i32, C.c_double,
+                                  C.c_double, _i32, _i32, _P(_i32), _P(_i32), _P(_i32)]),
     "tsv_sched_place": (_i32, [_P(C.c_double), _i32, _P(_i32), _i32, _P(_i32), _P(_i32), _P(C.c_uint64), _i32, _i32,
                                _i32, _P(C.c_uint64)]),
     "tsv_sched_last_error": (C.c_char_p, []),

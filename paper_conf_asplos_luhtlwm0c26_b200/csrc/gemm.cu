@@ -384,7 +384,8 @@ __device__ __forceinline__ void split_epilogue(const GemmArgs& args, const GemmE
   if (lane == 0) *cnt = 0;   // re-armed for the next launch (the kernel boundary orders it)
 }
 
-template <int BN>
+// SPLITK: the split-K instantiation (args.splits > 1); the plain one compiles without any of it
+template <int BN, bool SPLITK = false>
 __global__ void __launch_bounds__(GEMM_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ GemmMaps maps, const __grid_constant__ GemmArgs args) {
   using C = GemmCfg<BN>;
@@ -429,10 +430,14 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   // kernel's tail.  A (and the fp32 stream) come from the previous kernel: after the wait.
   // split-K range of tile t
   auto krange = [&](int t, int& t0, int& s, int& kb0, int& kb1) {
-    s = t / args.tiles_per_split;
-    t0 = t - s * args.tiles_per_split;
-    kb0 = s * args.kps;
-    kb1 = min(num_k, kb0 + args.kps);
+    if (SPLITK) {
+      s = t / args.tiles_per_split;
+      t0 = t - s * args.tiles_per_split;
+      kb0 = s * args.kps;
+      kb1 = min(num_k, kb0 + args.kps);
+    } else {
+      s = 0; t0 = t; kb0 = 0; kb1 = num_k;
+    }
   };
   int npre = 0;
   if (warp == 0 && lane == 0 && (int)blockIdx.x < args.num_tiles) {
@@ -517,7 +522,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       tc_fence_after();
       const int row0 = m_blk * BM + wq * 32;
       const uint32_t tbase = tmem_base + ((uint32_t)(wq * 32) << 16) + acc * BN;
-      if (args.splits > 1) {
+      if (SPLITK) {
         split_epilogue<BN>(args, epi, Mp, row0, n_blk, tbase, stg, lane, t0, sp, wq, 4);
       } else if (epi.qk_h > 0 && n_blk * BN < 3 * epi.qk_h) {
 #pragma unroll 1
@@ -560,7 +565,7 @@ struct Gemm2Cfg {
   static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + 4 * 32 * 36 * 4;
 };
 
-template <int BN_>
+template <int BN_, bool SPLITK = false>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
     gemm_tc2_kernel(const __grid_constant__ GemmMaps maps, const __grid_constant__ GemmArgs args) {
   using C = Gemm2Cfg<BN_>;
@@ -606,10 +611,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
   const uint32_t tmem_base = *tmem_slot;
   // weights of the first stages before the programmatic-dependency wait (see gemm_tc_kernel)
   auto krange = [&](int t, int& t0, int& s, int& kb0, int& kb1) {   // split-K range (see GemmArgs)
-    s = t / args.tiles_per_split;
-    t0 = t - s * args.tiles_per_split;
-    kb0 = s * args.kps;
-    kb1 = min(num_k, kb0 + args.kps);
+    if (SPLITK) {
+      s = t / args.tiles_per_split;
+      t0 = t - s * args.tiles_per_split;
+      kb0 = s * args.kps;
+      kb1 = min(num_k, kb0 + args.kps);
+    } else {
+      s = 0; t0 = t; kb0 = 0; kb1 = num_k;
+    }
   };
   int npre = 0;
   if (warp == 0 && lane == 0 && cid < args.num_tiles) {
@@ -694,7 +703,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
       tc_fence_after();
       const int row0 = m_blk * 256 + (int)rank * 128 + wq * 32;
       const uint32_t tbase = tmem_base + ((uint32_t)(wq * 32) << 16) + acc * BN;
-      if (args.splits > 1) {
+      if (SPLITK) {
         split_epilogue<BN>(args, epi, Mp, row0, n_blk, tbase, stg, lane, t0, sp, (int)rank * 4 + wq, 8);
       } else if (epi.qk_h > 0 && n_blk * BN < 3 * epi.qk_h) {
 #pragma unroll 1
@@ -905,9 +914,11 @@ static void launch_bn(const GemmPlan& p, cudaStream_t s) {
   int dev = 0;
   cudaGetDevice(&dev);
   if (!(attr_done >> dev & 1ull)) {
-    cudaFuncSetAttribute(gemm_tc_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
+    cudaFuncSetAttribute(gemm_tc_kernel<BN, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
+    cudaFuncSetAttribute(gemm_tc_kernel<BN, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
     attr_done |= 1ull << dev;
   }
+  const bool sk = p.splits > 1;
   GemmArgs a;
   GemmMaps maps;
   const int bm = p.pair ? 256 : BM;
@@ -926,16 +937,20 @@ static void launch_bn(const GemmPlan& p, cudaStream_t s) {
     if (p.pair) {
       static unsigned long long attr2 = 0;
       if (!(attr2 >> dev & 1ull)) {
-        cudaFuncSetAttribute(gemm_tc2_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaFuncSetAttribute(gemm_tc2_kernel<BN, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             Gemm2Cfg<BN>::SMEM_BYTES);
+        cudaFuncSetAttribute(gemm_tc2_kernel<BN, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              Gemm2Cfg<BN>::SMEM_BYTES);
         attr2 |= 1ull << dev;
       }
-      launch_pdl(gemm_tc2_kernel<BN>, dim3(p.grid), dim3(GEMM_THREADS), Gemm2Cfg<BN>::SMEM_BYTES, s, maps, a);
+      if (sk) launch_pdl(gemm_tc2_kernel<BN, true>, dim3(p.grid), dim3(GEMM_THREADS), Gemm2Cfg<BN>::SMEM_BYTES, s, maps, a);
+      else launch_pdl(gemm_tc2_kernel<BN, false>, dim3(p.grid), dim3(GEMM_THREADS), Gemm2Cfg<BN>::SMEM_BYTES, s, maps, a);
       return;
     }
   }
   // 1-CTA tiles (the only variant for 64-wide tiles: gemm_plan never pairs them)
-  launch_pdl(gemm_tc_kernel<BN>, dim3(p.grid), dim3(GEMM_THREADS), C::SMEM_BYTES, s, maps, a);
+  if (sk) launch_pdl(gemm_tc_kernel<BN, true>, dim3(p.grid), dim3(GEMM_THREADS), C::SMEM_BYTES, s, maps, a);
+  else launch_pdl(gemm_tc_kernel<BN, false>, dim3(p.grid), dim3(GEMM_THREADS), C::SMEM_BYTES, s, maps, a);
 }
 
 void gemm_launch(const GemmPlan& p, cudaStream_t s) {

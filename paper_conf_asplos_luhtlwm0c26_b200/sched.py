@@ -34,16 +34,17 @@ def allocate(T, ks, deadline: float, steps: int, row: int, now: float, N: int):
     return list(out), bool(late.value)
 
 
-def schedule_round(T, ks, requests, now: float, tau: float, N: int):
-    """requests: [(deadline, remaining_steps, table_row)] -> (survivors, [(gpus, steps)])."""
+def schedule_round(T, ks, requests, now: float, tau: float, N: int, work_conserving: bool = False):
+    """requests: [(deadline, remaining_steps, table_row)] -> (survivors, [(gpus, steps)]).
+    work_conserving: Alg. 1's argmax tie goes to the largest capacity (S31b) instead of the smallest."""
     T, kk, n_res, n_k = _table(T, ks)
     R = len(requests)
     arr = _reqs(requests)
     g = (C.c_int * max(R, 1))()
     s = (C.c_int * max(R, 1))()
     sv = C.c_int()
-    check_sched(lib.tsv_sched_round(T.ctypes.data_as(C.POINTER(C.c_double)), n_res, kk, n_k, arr, R, now, tau, N, g, s,
-                                    C.byref(sv)))
+    check_sched(lib.tsv_sched_round_ex(T.ctypes.data_as(C.POINTER(C.c_double)), n_res, kk, n_k, arr, R, now, tau, N,
+                                       1 if work_conserving else 0, g, s, C.byref(sv)))
     return sv.value, [(g[i], s[i]) for i in range(R)]
 
 

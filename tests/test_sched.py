@@ -103,11 +103,24 @@ def test_round_matches_oracle(sched):
         T, reqs = _instance(rng, R, N)
         tau = float(rng.uniform(0.05, 0.5))
         now = float(rng.uniform(0, 0.05))
-        got = sched.schedule_round(T, KS, reqs, now, tau, N)
-        ref = OS.schedule_round(T, KS, reqs, now, tau, N)
-        assert got[0] == ref[0]
-        assert got[1] == [tuple(x) for x in ref[1]]
-        assert sum(g for g, _ in got[1]) <= N
+        for wc in (False, True):
+            got = sched.schedule_round(T, KS, reqs, now, tau, N, work_conserving=wc)
+            ref = OS.schedule_round(T, KS, reqs, now, tau, N, work_conserving=wc)
+            assert got[0] == ref[0]
+            assert got[1] == [tuple(x) for x in ref[1]]
+            assert sum(g for g, _ in got[1]) <= N
+
+
+def test_round_work_conserving_tie(sched):
+    """Alg. 1 line 21 tie: a request with ample slack survives with or without running, so the
+    smallest-capacity optimum (S31) defers it while the largest-capacity one (S31b) runs it now at
+    its minimal allocation; the survivor count is the same."""
+    T = np.array([[1.0, 0.6, 0.35, 0.2]])
+    reqs = [(100.0, 5, 0)]
+    sv0, plan0 = sched.schedule_round(T, KS, reqs, 0.0, 1.0, 8)
+    sv1, plan1 = sched.schedule_round(T, KS, reqs, 0.0, 1.0, 8, work_conserving=True)
+    assert sv0 == sv1 == 1
+    assert plan0 == [(0, 0)] and plan1 == [(1, 1)]
 
 
 def test_round_semantics(sched):

@@ -17,6 +17,9 @@ Policies:
                  on their GPUs and scales idle GPUs up; a request whose GPUs change pays
                  a reshard (latent bytes over NVLink).
   tetriserve-np  the same without placement preservation and scale-up (Table 5 ablation analogue).
+  tetriserve-wc  the same as tetriserve with Alg. 1's argmax tie taken at the largest capacity
+                 (reading S31b: every request that can make progress runs now at its minimal
+                 allocation) instead of the smallest (S31: requests with slack are deferred).
   fixed-k        every request runs all its steps at SP degree k on k GPUs, FCFS (xDiT-style).
 
 The simulator itself is plain Python; only the scheduling decisions come from the C-ABI.
@@ -69,7 +72,7 @@ def reshard_s(row):
     return Li * 64 * 4 / NVLINK_BPS + 20e-6
 
 
-def sim_tetriserve(T, ks, N, reqs, dl, gran=5, preserve=True):
+def sim_tetriserve(T, ks, N, reqs, dl, gran=5, preserve=True, wc=False):
     """Rounds every tau.  GPUs still busy from earlier work (a best-effort step longer than tau)
     are excluded from the round; the packer and the placement work on the free GPUs (NVSwitch:
     any subset can form a group, S14), mapped to their ids in ascending order."""
@@ -101,7 +104,8 @@ def sim_tetriserve(T, ks, N, reqs, dl, gran=5, preserve=True):
             # the packer needs power-of-two degrees <= the free capacity
             ks_r = [k for k in ks if k <= nf]
             Tr = T[:, [ks.index(k) for k in ks_r]]
-            sv, plan = sched.schedule_round(Tr, ks_r, [(q["deadline"], q["left"], q["row"]) for q in cand], now, tau, nf)
+            sv, plan = sched.schedule_round(Tr, ks_r, [(q["deadline"], q["left"], q["row"]) for q in cand], now, tau, nf,
+                                            work_conserving=wc)
             idx = {g: j for j, g in enumerate(free)}
             prv = [{idx[g] for g in prev.get(q["id"], set()) if g in idx} if preserve else set() for q in cand]
             nf2 = 1 << (nf.bit_length() - 1)          # placement works on an aligned pool
@@ -174,6 +178,8 @@ def run(T, ks, N=8, n=300, rate=12.0, mix="uniform", scales=(1.0, 1.25, 1.5), se
         row["tetriserve"] = round(sar(d, reqs, dl), 4)
         d, b = sim_tetriserve(T, ks, N, reqs, dl, gran=gran, preserve=False)
         row["tetriserve-np"] = round(sar(d, reqs, dl), 4)
+        d, b = sim_tetriserve(T, ks, N, reqs, dl, gran=gran, preserve=True, wc=True)
+        row["tetriserve-wc"] = round(sar(d, reqs, dl), 4)
         for k in ks:
             d, b = sim_fixed(T, ks, N, reqs, k)
             row[f"fixed-{k}"] = round(sar(d, reqs, dl), 4)
