@@ -202,8 +202,8 @@ def main():
     ap.add_argument("--gran", type=int, default=5, help="round = gran steps of the largest resolution at k = N (P:562)")
     args = ap.parse_args()
     tab = json.load(open(args.table))
-    assert tab["res"] == RES, "table rows must be 256, 512, 1024, 2048"
-    T = np.array(tab["ms"], dtype=float) / 1e3
+    assert all(r in tab["res"] for r in RES), "the table needs rows 256, 512, 1024, 2048"
+    T = np.array([tab["ms"][tab["res"].index(r)] for r in RES], dtype=float) / 1e3
     for mix in (["uniform", "skewed"] if args.mix == "both" else [args.mix]):
         rate = args.rate
         if args.load is not None:
