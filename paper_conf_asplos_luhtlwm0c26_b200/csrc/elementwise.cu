@@ -76,6 +76,78 @@ __global__ void __launch_bounds__(T) ln_mod_kernel(const float* __restrict__ x, 
   grid_dep_launch();   // the next kernel (a GEMM) may start its prologue / weight prefetch
 }
 
+// Persistent-row variant: CTA b handles rows b, b + grid, ... (grid ~ 4 CTAs per SM), keeps the
+// modulation vectors in registers while consecutive rows share them (one reload at the txt/img
+// boundary), and prefetches the next row's x while the current row is reduced and written.
+template <int T, int NV>
+__global__ void __launch_bounds__(T) ln_mod_rows_kernel(const float* __restrict__ x, long long ldx,
+                                                        bf16* __restrict__ u, long long ldu,
+                                                        const float* __restrict__ shift0,
+                                                        const float* __restrict__ scale0,
+                                                        const float* __restrict__ shift1,
+                                                        const float* __restrict__ scale1, int n_first, int rows_b,
+                                                        long long mstride, int M) {
+  __shared__ float red[T / 32];
+  const int t = threadIdx.x;
+  constexpr int h = 4 * T * NV;
+  grid_dep_wait();
+  int row = blockIdx.x;
+  float4 v[NV], shv[NV], scv[NV];
+  const float* cur = nullptr;
+  if (row < M) {
+    const float4* xr = reinterpret_cast<const float4*>(x + (long long)row * ldx);
+#pragma unroll
+    for (int i = 0; i < NV; ++i) v[i] = __ldcs(xr + i * T + t);
+  }
+  for (; row < M; row += gridDim.x) {
+    const int b = row / rows_b, r = row - b * rows_b;
+    const float* shift = (r < n_first ? shift0 : shift1) + b * mstride;
+    if (shift != cur) {   // uniform across the CTA
+      const float* scale = (r < n_first ? scale0 : scale1) + b * mstride;
+#pragma unroll
+      for (int i = 0; i < NV; ++i) {
+        shv[i] = __ldg(reinterpret_cast<const float4*>(shift) + i * T + t);
+        scv[i] = __ldg(reinterpret_cast<const float4*>(scale) + i * T + t);
+      }
+      cur = shift;
+    }
+    const int nrow = row + gridDim.x;
+    float4 vn[NV];
+    if (nrow < M) {   // prefetch the next row under this row's reductions
+      const float4* xn = reinterpret_cast<const float4*>(x + (long long)nrow * ldx);
+#pragma unroll
+      for (int i = 0; i < NV; ++i) vn[i] = __ldcs(xn + i * T + t);
+    }
+    float sm = 0.f;
+#pragma unroll
+    for (int i = 0; i < NV; ++i) sm += (v[i].x + v[i].y) + (v[i].z + v[i].w);
+    const float mean = block_sum<T>(sm, red) * (1.0f / h);
+    float q = 0.f;
+#pragma unroll
+    for (int i = 0; i < NV; ++i) {
+      float a = v[i].x - mean, bb = v[i].y - mean, c = v[i].z - mean, d = v[i].w - mean;
+      q += (a * a + bb * bb) + (c * c + d * d);
+    }
+    const float rstd = rsqrtf(block_sum<T>(q, red) * (1.0f / h) + 1e-6f);
+    uint2* ur = reinterpret_cast<uint2*>(u + (long long)row * ldu);
+#pragma unroll
+    for (int i = 0; i < NV; ++i) {
+      const int c = i * T + t;
+      const float4 sh = shv[i], sc = scv[i];
+      const float a = (v[i].x - mean) * rstd * (1.f + sc.x) + sh.x;
+      const float bb = (v[i].y - mean) * rstd * (1.f + sc.y) + sh.y;
+      const float cc = (v[i].z - mean) * rstd * (1.f + sc.z) + sh.z;
+      const float d = (v[i].w - mean) * rstd * (1.f + sc.w) + sh.w;
+      ur[c] = make_uint2(pack_bf16x2(a, bb), pack_bf16x2(cc, d));
+    }
+    if (nrow < M) {
+#pragma unroll
+      for (int i = 0; i < NV; ++i) v[i] = vn[i];
+    }
+  }
+  grid_dep_launch();
+}
+
 // Warp per row (8 rows per 256-thread CTA): the row stays in registers (NV float4 per lane), both
 // reductions are warp shuffles (no block barriers), the modulation vectors come through L1 (shared
 // by every row of a stream).  Rows [0, n_first) of each block of rows_b take (shift0, scale0).
@@ -158,7 +230,9 @@ __global__ void __launch_bounds__(256) ln_mod_generic(const float* __restrict__ 
     u[(long long)row * ldu + c] = __float2bfloat16_rn((xr[c] - mean) * rstd * (1.f + scale[c]) + shift[c]);
 }
 
-int g_ln_impl = 0;   // 0: CTA per row, 1: warp per row (tsv_op_ln_mod impl; microbench sweeps)
+// LN-modulate kernel choice (tsv_op_ln_mod impl; TSV_LN_IMPL): 0 CTA per row, 1 warp per row,
+// 2 persistent rows (the default: same-box FLUX 512^2 step A/B -0.5 %)
+int g_ln_impl = 2;
 
 void ln_mod2b_launch(const float* x, long long ldx, bf16* u, long long ldu, const float* shift0,
                      const float* scale0, const float* shift1, const float* scale1, int n_first, int rows_b, int B,
@@ -173,6 +247,25 @@ void ln_mod2b_launch(const float* x, long long ldx, bf16* u, long long ldu, cons
     else
       launch_pdl(ln_mod_warp_kernel<12>, grid, dim3(256), 0, s, x, ldx, u, ldu, shift0, scale0, shift1, scale1, n_first,
                  rows_b, mstride, M);
+    return;
+  }
+  if (g_ln_impl == 2 && (h == 3072 || h == 1536 || h == 256)) {
+    static int sms = 0;
+    if (!sms) {
+      int dev = 0;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    }
+    const int grid = M < 4 * sms ? M : 4 * sms;
+    if (h == 3072)
+      launch_pdl(ln_mod_rows_kernel<256, 3>, dim3(grid), dim3(256), 0, s, x, ldx, u, ldu, shift0, scale0, shift1,
+                 scale1, n_first, rows_b, mstride, M);
+    else if (h == 1536)
+      launch_pdl(ln_mod_rows_kernel<128, 3>, dim3(grid), dim3(128), 0, s, x, ldx, u, ldu, shift0, scale0, shift1,
+                 scale1, n_first, rows_b, mstride, M);
+    else
+      launch_pdl(ln_mod_rows_kernel<32, 2>, dim3(grid), dim3(32), 0, s, x, ldx, u, ldu, shift0, scale0, shift1,
+                 scale1, n_first, rows_b, mstride, M);
     return;
   }
   switch (h) {

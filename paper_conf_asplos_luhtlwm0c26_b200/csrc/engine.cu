@@ -1482,6 +1482,7 @@ tsv_status tsv_engine_create(const tsv_model_desc* model, const int* devices, in
   if (!build_model(*model, &e->model, &err)) return fail(TSV_E_INVAL, "%s", err.c_str());
   e->weight_seed = weight_seed;
   e->splitk = splitk_env();
+  if (const char* li = getenv("TSV_LN_IMPL")) g_ln_impl = atoi(li);   // LN-modulate variant (A/B)
   e->rank_base = rank_base;
   e->n_local = n_local;
   e->world = world_size;
@@ -2196,7 +2197,7 @@ tsv_status tsv_op_gemm_qkv(const void* A, int64_t lda, const void* Wt, int64_t l
 tsv_status tsv_op_ln_mod(const float* x, int64_t ldx, void* u, int64_t ldu, const float* shift, const float* scale,
                          int M, int h, int impl, void* stream) {
   if (h % 128) return fail(TSV_E_INVAL, "h must be a multiple of 128");
-  if (impl < 0 || impl > 1) return fail(TSV_E_INVAL, "bad impl %d", impl);
+  if (impl < 0 || impl > 2) return fail(TSV_E_INVAL, "bad impl %d", impl);
   const int keep = g_ln_impl;
   g_ln_impl = impl;
   ln_mod_launch(x, ldx, reinterpret_cast<bf16*>(u), ldu, shift, scale, M, h, reinterpret_cast<cudaStream_t>(stream));

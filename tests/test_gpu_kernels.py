@@ -199,7 +199,7 @@ def test_gemm_rejects_bad_shapes(tsv):
 
 
 # ----------------------------------------------------------------------------- LN-modulate
-@pytest.mark.parametrize("impl", [0, 1])
+@pytest.mark.parametrize("impl", [0, 1, 2])
 @pytest.mark.parametrize("M,h", [(1, 256), (333, 256), (1536, 3072), (77, 1536), (5, 640), (13, 3072)])
 def test_ln_mod(tsv, M, h, impl):
     rng = np.random.default_rng(M + h)

@@ -292,3 +292,22 @@ def test_split_k_step_matches_unsplit(tsv, monkeypatch):
     for a, b in zip(out[0], out[1]):
         rel, cos = _metrics(b.astype(np.float64), a.astype(np.float64))
         assert rel <= 1e-2 and cos >= 0.9999
+
+
+@pytest.mark.parametrize("model", ["tiny2", "tiny_sd3"])
+def test_ln_impls_bitwise(tsv, model, monkeypatch):
+    """The LN-modulate variants (TSV_LN_IMPL 0: CTA per row, 2: persistent rows) run the same
+    per-row arithmetic: bit-identical steps."""
+    out = []
+    for impl in ("0", "2"):
+        monkeypatch.setenv("TSV_LN_IMPL", impl)
+        eng = tsv.Engine(model, devices=[0, 0])
+        g = eng.group_create([0, 1])
+        req = eng.request_create(208, 240, num_steps=3, seed=1013)
+        for s in range(2):
+            eng.request_step(req, s, g)
+        out.append((eng.read_latent(req), eng.read_velocity(req)))
+        eng.close()
+    monkeypatch.setenv("TSV_LN_IMPL", "0")
+    tsv.Engine(model, devices=[0]).close()   # restore the process-wide default
+    assert np.array_equal(out[0][0], out[1][0]) and np.array_equal(out[0][1], out[1][1])

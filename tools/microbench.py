@@ -148,9 +148,9 @@ def ln_cases():
         x = torch.randn(M, h, device="cuda")
         u = torch.empty(M, h, dtype=torch.bfloat16, device="cuda")
         sh, sc = torch.randn(h, device="cuda"), torch.randn(h, device="cuda")
-        for impl in (0, 1):
+        for impl in (0, 1, 2):
             ms = timeit(lambda: tsv.op_ln_mod(x, u, sh, sc, impl=impl))
-            print(json.dumps({"op": "ln_mod", "impl": ["cta_per_row", "warp_per_row"][impl], "M": M, "h": h,
+            print(json.dumps({"op": "ln_mod", "impl": ["cta_per_row", "warp_per_row", "persistent_rows"][impl], "M": M, "h": h,
                               "ms": round(ms, 4), "GBps": round(M * h * 6 / ms / 1e6, 1)}), flush=True)
 
 
