@@ -308,6 +308,6 @@ def test_ln_impls_bitwise(tsv, model, monkeypatch):
             eng.request_step(req, s, g)
         out.append((eng.read_latent(req), eng.read_velocity(req)))
         eng.close()
-    monkeypatch.setenv("TSV_LN_IMPL", "0")
-    tsv.Engine(model, devices=[0]).close()   # restore the process-wide default
+    monkeypatch.setenv("TSV_LN_IMPL", "2")
+    tsv.Engine(model, devices=[0]).close()   # restore the process-wide default (impl 2)
     assert np.array_equal(out[0][0], out[1][0]) and np.array_equal(out[0][1], out[1][1])
