@@ -304,6 +304,38 @@ def test_attention_kv_split(tsv, L, H, D, nsplit):
     assert torch.count_nonzero(cnt) == 0
 
 
+@pytest.mark.parametrize("L,H,D,split", [(16896, 24, 128, False), (16896, 3, 128, True), (16717, 24, 64, False),
+                                         (4429, 3, 64, True)])
+def test_attention_sampled_full_size(tsv, L, H, D, split):
+    """BASELINE sizes (FLUX 2048^2 joint L = 16 896, SD3 2048^2 / 1024^2 L = 16 717 / 4429; H = 3 is an
+    SP = 8 head shard, run with the KV split): sampled query rows of sampled heads against the
+    float64 definition over all L keys, in the launch configuration the step uses."""
+    g = torch.Generator(device="cuda").manual_seed(L + H + D)
+    qkv = (torch.randn(L, 3 * H * D, device="cuda", generator=g) * 1.5).to(torch.bfloat16)
+    o = torch.zeros(L, H * D, dtype=torch.bfloat16, device="cuda")
+    ld = 3 * H * D
+    if split:
+        cnt = torch.zeros(4096, dtype=torch.int32, device="cuda")
+        ws = torch.empty(32 << 20, dtype=torch.float32, device="cuda")
+        tsv.op_attention_split(qkv, qkv[:, H * D:], qkv[:, 2 * H * D:], o, L, H, D, cnt, ws, nsplit=0, ldq=ld, ldk=ld,
+                               ldv=ld)
+    else:
+        tsv.op_attention(qkv, qkv[:, H * D:], qkv[:, 2 * H * D:], o, L, H, D, ldq=ld, ldk=ld, ldv=ld)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(L)
+    rows = np.concatenate([[0, L - 1], rng.choice(L, 14, replace=False)])
+    heads = sorted(set([0, H - 1] + list(rng.choice(H, min(H, 2), replace=False))))
+    t = qkv.view(L, 3, H, D)
+    for hh in heads:
+        k = t[:, 1, hh].double().cpu().numpy()
+        v = t[:, 2, hh].double().cpu().numpy()
+        q = t[rows, 0, hh].double().cpu().numpy()
+        ref = F.attention(q[:, None, :], k[:, None, :], v[:, None, :])[:, 0]   # oracle: queries x all keys
+        got = o.view(L, H, D)[rows, hh].double().cpu().numpy()
+        assert _rel(got, ref) < 1.5e-2, hh
+        assert np.sum(got * ref) / np.linalg.norm(got) / np.linalg.norm(ref) > 0.9999
+
+
 def test_attention_special_cases(tsv):
     # identical keys -> mean(V) (S:§8(c) P3)
     L, H, D = 300, 2, 128
