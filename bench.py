@@ -223,15 +223,21 @@ def run_reference(args):
     res = args.res
     mdl = MODELS[args.model]
     ms_list = []
-    steps = max(1, min(args.steps, 3))
+    sample = oracle_sample_sd3 if args.model == "sd3" else oracle_sample
+    # each step is a bounded sample (~1-2 min of host BLAS at 512^2): at most 1 warm-up and 2 timed
+    # samples keep the whole reference run within a few minutes
+    warm = min(args.warmup, 1)
+    steps = max(1, min(args.steps, 2))
+    for _ in range(warm):
+        sample(res)
     for _ in range(steps):
-        ms, detail = (oracle_sample_sd3 if args.model == "sd3" else oracle_sample)(res)
+        ms, detail = sample(res)
         ms_list.append(ms)
     ms = statistics.median(ms_list)
     detail["value"] = ms
     detail["unit"] = "ms"
     line = {"impl": "reference", "metric": METRIC, "value": ms, "unit": "ms", "n_gpus": args.gpus,
-            "steps": steps, "warmup": 0, "ms_per_step": ms, "higher_is_better": False, "scaling": "strong",
+            "steps": steps, "warmup": warm, "ms_per_step": ms, "higher_is_better": False, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic (SYNTH-1 seeded weights and inputs)",
             "config": {"workload": f"{mdl['desc']} {res}x{res} ({(res // 16) ** 2} image + {mdl['Lt']} text tokens)",
                        "sp": 1, "resolution": res},
