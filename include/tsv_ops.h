@@ -66,8 +66,9 @@ tsv_status tsv_op_gemm_qkv(const void* A, int64_t lda, const void* W, int64_t ld
 /* a2: u[m, :] = bf16(LN(x[m, :]) * (1 + scale) + shift); x fp32, LN without affine, eps 1e-6.
  * impl 0: one CTA per row (block reductions); impl 1: one warp per row; impl 2: persistent CTAs
  * (~4 per SM) looping over rows with the modulation vectors kept in registers and the next row
- * prefetched (impl 1: h in {1536, 3072}; impl 2: h in {256, 1536, 3072}; other h fall back to
- * impl 0).  The engine's step uses impl 2 (TSV_LN_IMPL at engine creation selects another).
+ * prefetched, used for launches of <= 16 rows per SM (else impl 0).  impl 1: h in {1536, 3072};
+ * impl 2: h in {256, 1536, 3072}; other h fall back to impl 0.  The engine's step uses impl 2
+ * (TSV_LN_IMPL at engine creation selects another).
  * Errors: TSV_E_INVAL (h % 128, impl). */
 tsv_status tsv_op_ln_mod(const float* x, int64_t ldx, void* u, int64_t ldu, const float* shift,
                          const float* scale, int M, int h, int impl, void* stream);

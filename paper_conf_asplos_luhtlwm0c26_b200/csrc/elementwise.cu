@@ -249,13 +249,15 @@ void ln_mod2b_launch(const float* x, long long ldx, bf16* u, long long ldu, cons
                  rows_b, mstride, M);
     return;
   }
-  if (g_ln_impl == 2 && (h == 3072 || h == 1536 || h == 256)) {
-    static int sms = 0;
-    if (!sms) {
-      int dev = 0;
-      cudaGetDevice(&dev);
-      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    }
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  }
+  // persistent rows only pay off while the launch is about one wave of row-CTAs (512^2: -0.5 % step);
+  // at 2048^2 (16 896 rows) the CTA-per-row kernel streams faster (measured, profiles/README.md)
+  if (g_ln_impl == 2 && (h == 3072 || h == 1536 || h == 256) && M <= 16 * sms) {
     const int grid = M < 4 * sms ? M : 4 * sms;
     if (h == 3072)
       launch_pdl(ln_mod_rows_kernel<256, 3>, dim3(grid), dim3(256), 0, s, x, ldx, u, ldu, shift0, scale0, shift1,
