@@ -21,6 +21,7 @@ Policies:
                  (reading S31b: every request that can make progress runs now at its minimal
                  allocation) instead of the smallest (S31: requests with slack are deferred).
   fixed-k        every request runs all its steps at SP degree k on k GPUs, FCFS (xDiT-style).
+  rssp           resolution-specific SP: 1 / 1 / 2 / 8 GPUs for 256^2 / 512^2 / 1024^2 / 2048^2, FCFS.
 
 The simulator itself is plain Python; only the scheduling decisions come from the C-ABI.
 Timing comes from the table (device-measured per-rank step latencies, see latency_table_model).
@@ -162,6 +163,24 @@ def sim_fixed(T, ks, N, reqs, k):
     return done, busy
 
 
+def sim_rssp(T, ks, N, reqs, degrees):
+    """Resolution-specific SP: each resolution has its own fixed degree (profiled offline:
+    1 / 1 / 2 / 8 for 256^2 / 512^2 / 1024^2 / 2048^2 in the paper); FCFS, a request starts when its
+    degree's worth of GPUs is free (any subset: NVSwitch, S14) and holds them for all its steps."""
+    free_at = [0.0] * N
+    done, busy = {}, 0.0
+    for q in sorted(reqs, key=lambda r: r["arrival"]):
+        k = degrees[q["row"]]
+        order = sorted(range(N), key=lambda g: free_at[g])[:k]
+        t0 = max(q["arrival"], max(free_at[g] for g in order))
+        t = q["steps"] * T[q["row"], ks.index(k)]
+        for g in order:
+            free_at[g] = t0 + t
+        done[q["id"]] = t0 + t
+        busy += k * t
+    return done, busy
+
+
 def sar(done, reqs, dl):
     ok = sum(1 for q in reqs if done[q["id"]] <= q["arrival"] + dl[RES[q["row"]]] + 1e-9)
     return ok / len(reqs)
@@ -183,6 +202,8 @@ def run(T, ks, N=8, n=300, rate=12.0, mix="uniform", scales=(1.0, 1.25, 1.5), se
         for k in ks:
             d, b = sim_fixed(T, ks, N, reqs, k)
             row[f"fixed-{k}"] = round(sar(d, reqs, dl), 4)
+        d, b = sim_rssp(T, ks, N, reqs, [1, 1, 2, 8] if N >= 8 else [1, 1, 2, N])
+        row["rssp"] = round(sar(d, reqs, dl), 4)
         out.append(row)
     return out
 
