@@ -44,11 +44,12 @@ tsv_status tsv_op_gemm(const void* A, int64_t lda, const void* W, int64_t ldw, i
 /* The same GEMM with split-K (a8 / a9 on small row counts): K is cut into `splits` ranges
  * (0: the engine's automatic choice, which may be 1); each range's fp32 partial goes to ws and the
  * last range to finish an output tile sums the partials in range order 0..splits-1 and applies the
- * epilogue once (mode TSV_EPI_RESID_GATE: out0 += gate * (A W^T + bias), or TSV_EPI_ACCUM_F32:
- * out0 += A W^T + bias), so the result is deterministic.  sem: device int buffer of
+ * epilogue once, so the result is deterministic.  Modes: TSV_EPI_STORE_BF16 / GELU_BF16 /
+ * SILU_BF16 / STORE_F32 (out0 = f(A W^T + bias)), TSV_EPI_RESID_GATE (out0 += gate * (A W^T +
+ * bias)), TSV_EPI_ACCUM_F32 (out0 += A W^T + bias).  sem: device int buffer of
  * sem_ints >= 4 * output tiles entries, zero on entry and left zero; ws: device buffer of ws_bytes
  * (splits * tiles * 128 * tile width * 4 bytes are used; the split factor is capped to fit).  One
- * (sem, ws) pair per concurrently running launch.  TSV_E_INVAL if the mode is not accumulating. */
+ * (sem, ws) pair per concurrently running launch.  TSV_E_INVAL for other modes. */
 tsv_status tsv_op_gemm_split(const void* A, int64_t lda, const void* W, int64_t ldw, int M, int N, int K, int mode,
                              void* out0, int64_t ld0, const void* bias, const float* gate, int splits, int* sem,
                              int sem_ints, float* ws, int64_t ws_bytes, void* stream);

@@ -2143,7 +2143,9 @@ tsv_status tsv_op_gemm(const void* A, int64_t lda, const void* Wt, int64_t ldw, 
 tsv_status tsv_op_gemm_split(const void* A, int64_t lda, const void* Wt, int64_t ldw, int M, int N, int K, int mode,
                              void* out0, int64_t ld0, const void* bias, const float* gate, int splits, int* sem,
                              int sem_ints, float* ws, int64_t ws_bytes, void* stream) {
-  if (mode != EPI_RESID_GATE && mode != EPI_ACCUM_F32) return fail(TSV_E_INVAL, "split-K needs RESID_GATE or ACCUM_F32");
+  if (mode != EPI_RESID_GATE && mode != EPI_ACCUM_F32 && mode != EPI_STORE_F32 && mode != EPI_STORE_BF16 &&
+      mode != EPI_GELU_BF16 && mode != EPI_SILU_BF16)
+    return fail(TSV_E_INVAL, "split-K op: mode must be STORE_BF16, GELU_BF16, SILU_BF16, STORE_F32, RESID_GATE or ACCUM_F32");
   if (!sem || !ws || splits < 0) return fail(TSV_E_INVAL, "split-K needs counters, a workspace and splits >= 0");
   GemmSplitWs w;
   w.sem = sem;

@@ -780,12 +780,14 @@ int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int
   *err = nullptr;
   p->splits = 1; p->kps = K / BK; p->sem = nullptr; p->ws = nullptr;
   // Split-K for launches too small to fill the GPU (small M: the text stream, SP = 4/8 shards,
-  // 256^2 / 512^2 at k >= 2), for the fp32-accumulating epilogues only (x += g (acc + b) is linear
-  // in acc).  Few tiles otherwise leave most SMs idle while the weights stream through a handful of
-  // them (each SM pulls ~64 B/clk from L2: a weight-streaming GEMM needs most of the 148 SMs).
+  // 256^2 / 512^2 at k >= 2): the splits' fp32 partials are summed by the last split, which then
+  // runs the ordinary epilogue, so any epilogue but the fused QK-norm / RoPE / pack one qualifies.
+  // Few tiles otherwise leave most SMs idle while the weights stream through a handful of them
+  // (each SM pulls ~64 B/clk from L2: a weight-streaming GEMM needs most of the 148 SMs).
   bool split_ok = sws != nullptr && sws->sem && sws->ws;
   for (int q = 0; q < nprob && split_ok; ++q)
-    split_ok = (probs[q].epi.mode == EPI_RESID_GATE || probs[q].epi.mode == EPI_ACCUM_F32) && !probs[q].epi.qk_h;
+    split_ok = !probs[q].epi.qk_h;   // the last split runs the tile's ordinary epilogue (any mode but the
+                                     // fused QK-norm / RoPE / pack one) on the summed partials
   if (N <= 0 || K <= 0) { *err = "gemm: empty shape"; return -1; }
   if (K % BK) { *err = "gemm: K must be a multiple of 64"; return -1; }
   if (N % 64) { *err = "gemm: N must be a multiple of 64"; return -1; }
@@ -868,9 +870,12 @@ int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int
     if (force_splits > 0) {
       want_splits = force_splits;
     } else if (tiles * 2 <= units) {
-      want_splits = (int)(units / tiles);
+      // measured (tools/microbench.py split, SPLIT_SWEEP): CTA pairs are best filling the SM pairs
+      // once (S = 3 for 24 pair tiles), 1-CTA tiles at about half the SMs (S = 6 for 12 tiles):
+      // beyond that the partial-sum traffic and the in-order reduction cost more than they give
+      want_splits = (int)(pair ? units / tiles : units / (2 * tiles));
       if (want_splits > num_k / 4) want_splits = num_k / 4;   // >= 256 of K per split
-      if (want_splits > 4) want_splits = 4;   // measured: the in-order reduction makes S > 4 lose
+      if (want_splits > 6) want_splits = 6;
     }
     const long long per_split = (long long)tiles * bm * bn * 4;   // fp32 partials
     if (want_splits * per_split > sws->ws_bytes) want_splits = (int)(sws->ws_bytes / per_split);

@@ -114,6 +114,36 @@ def test_gemm_split_k_integer_exact(tsv, M, N, K, splits):
     assert torch.count_nonzero(sem) == 0
 
 
+@pytest.mark.parametrize("M,N,K", [(64, 3072, 4096), (192, 12288, 3072), (100, 1536, 1536)])
+def test_gemm_split_k_store_modes(tsv, M, N, K):
+    """Split-K with the non-accumulating epilogues (the last split applies them to the summed
+    partials): fp32 store bit-exact on integer operands, bf16 / GELU equal to the unsplit launch
+    after rounding (same fp32 sum up to order) within one bf16 ulp."""
+    rng = np.random.default_rng(M + N + K)
+    A = rng.integers(-2, 3, (M, K)).astype(np.float32)
+    W = rng.integers(-2, 3, (N, K)).astype(np.float32)
+    b = rng.integers(-4, 5, N).astype(np.float32)
+    exact = A.astype(np.float64) @ W.astype(np.float64).T + b
+    sem = torch.zeros(4096, dtype=torch.int32, device="cuda")
+    ws = torch.empty(64 << 18, dtype=torch.float32, device="cuda")
+    o = torch.zeros(M, N, device="cuda")
+    tsv.op_gemm_split(_bf16(A), _bf16(W), "STORE_F32", o, sem, ws, splits=3, bias=_bf16(b))
+    torch.cuda.synchronize()
+    assert np.array_equal(o.cpu().numpy().astype(np.float64), exact)
+    Af = synth.bf16_bits_to_f32(synth.bf16_rne_bits(rng.standard_normal((M, K)).astype(np.float32)))
+    Wf = synth.bf16_bits_to_f32(synth.bf16_rne_bits((rng.standard_normal((N, K)) / math.sqrt(K)).astype(np.float32)))
+    y = Af.astype(np.float64) @ Wf.astype(np.float64).T + b
+    for mode, fn in (("STORE_BF16", lambda v: v), ("GELU_BF16", F.gelu_tanh)):
+        o1 = torch.zeros(M, N, dtype=torch.bfloat16, device="cuda")
+        o2 = torch.zeros(M, N, dtype=torch.bfloat16, device="cuda")
+        tsv.op_gemm_split(_bf16(Af), _bf16(Wf), mode, o1, sem, ws, splits=4, bias=_bf16(b))
+        tsv.op_gemm(_bf16(Af), _bf16(Wf), mode, o2, bias=_bf16(b))
+        torch.cuda.synchronize()
+        assert _rel(_np(o1), fn(y)) < 1e-2
+        assert _rel(_np(o1), _np(o2)) < 1e-2
+    assert torch.count_nonzero(sem) == 0
+
+
 def test_gemm_split_k_resid_gate_deterministic(tsv):
     rng = np.random.default_rng(21)
     M, N, K = 192, 3072, 12288

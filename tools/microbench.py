@@ -84,7 +84,7 @@ def split_cases():
             res[splits] = timeit(lambda: tsv.op_gemm_split(A, W, "RESID_GATE", x, sem, ws, splits=splits, gate=g))
         if os.environ.get("SPLIT_SWEEP"):
             sw = {s_: round(timeit(lambda: tsv.op_gemm_split(A, W, "RESID_GATE", x, sem, ws, splits=s_, gate=g)), 4)
-                  for s_ in (2, 3, 4, 6, 8)}
+                  for s_ in (2, 3, 4, 6, 8, 12)}
             one = round(timeit(lambda: tsv.op_gemm(A, W, "RESID_GATE", x, gate=g, force_bn=256, force_pair=0)), 4)
             print(json.dumps({"op": "gemm_split_sweep", "M": M, "N": N, "K": K, "ms_by_splits": sw,
                               "ms_1cta_nosplit": one}), flush=True)
