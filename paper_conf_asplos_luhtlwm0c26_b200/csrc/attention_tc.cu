@@ -717,27 +717,31 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
             wsum += ms[s2] * __ldcg(ws_at(s2) + (size_t)(D + 1) * AT_BM + row);
           }
         inv = 1.f / wsum;
+        // the whole row (D values) accumulates in registers, one split at a time: each split's D
+        // loads are independent, so the merge costs nsplit L2 round trips (not nsplit x D/32)
+        float acc[D];
 #pragma unroll
-        for (int c = 0; c < D / 32; ++c) {
-          float acc[32];
+        for (int i = 0; i < D; ++i) acc[i] = 0.f;
 #pragma unroll
-          for (int i = 0; i < 32; ++i) acc[i] = 0.f;
+        for (int s2 = 0; s2 < 8; ++s2)
+          if (s2 < sa.nsplit) {
+            const float* src = ws_at(s2) + row;
+            const float w = ms[s2];
 #pragma unroll
-          for (int s2 = 0; s2 < 8; ++s2)
-            if (s2 < sa.nsplit) {
-              const float* src = ws_at(s2) + (size_t)(c * 32) * AT_BM + row;
+            for (int i = 0; i < D; ++i) acc[i] = fmaf(w, __ldcg(src + (size_t)i * AT_BM), acc[i]);
+          }
+        if (grow < L) {
 #pragma unroll
-              for (int i = 0; i < 32; ++i) acc[i] = fmaf(ms[s2], __ldcg(src + (size_t)i * AT_BM), acc[i]);
-            }
-          if (grow < L) {
+          for (int c = 0; c < D / 32; ++c) {
             uint4* dst = reinterpret_cast<uint4*>(orow + c * 32);
 #pragma unroll
             for (int qd = 0; qd < 4; ++qd) {
+              const float* a8 = acc + c * 32 + qd * 8;
               uint4 v;
-              v.x = pack_bf16x2(acc[qd * 8 + 0] * inv, acc[qd * 8 + 1] * inv);
-              v.y = pack_bf16x2(acc[qd * 8 + 2] * inv, acc[qd * 8 + 3] * inv);
-              v.z = pack_bf16x2(acc[qd * 8 + 4] * inv, acc[qd * 8 + 5] * inv);
-              v.w = pack_bf16x2(acc[qd * 8 + 6] * inv, acc[qd * 8 + 7] * inv);
+              v.x = pack_bf16x2(a8[0] * inv, a8[1] * inv);
+              v.y = pack_bf16x2(a8[2] * inv, a8[3] * inv);
+              v.z = pack_bf16x2(a8[4] * inv, a8[5] * inv);
+              v.w = pack_bf16x2(a8[6] * inv, a8[7] * inv);
               dst[qd] = v;
             }
           }

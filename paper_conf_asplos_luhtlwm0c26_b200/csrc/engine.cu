@@ -1332,25 +1332,31 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
       CK(cudaMemcpyAsync(c.rdq[q]->step.p, &st, sizeof(int), cudaMemcpyHostToDevice, c.s->stream));
     }
   }
-  if (e->graphs && E.rc.size() == 1) {
-    // one local rank: replay (or capture once) the whole step as a CUDA graph, cached per slot by
-    // every buffer it references
-    RankCtx& c = E.rc[0];
-    Slot& slot = *c.s;
+  // one local rank, or several virtual ranks sharing one stream (TSV_VIRTUAL_SERIAL): replay (or
+  // capture once) the whole step as a CUDA graph on that stream
+  bool one_stream = true;
+  for (auto& c : E.rc) one_stream = one_stream && c.s->stream == E.rc[0].s->stream;
+  if (e->graphs && one_stream) {
+    // cached per (first) slot by every buffer the step references
+    Slot& slot = *E.rc[0].s;
     uint64_t key = 1469598103934665603ull;
     auto mix = [&](uint64_t v) { key = (key ^ v) * 1099511628211ull; };
-    const void* ptrs[] = {c.x, c.u, c.qkv, c.cat, c.hbuf, c.latb, c.pack, c.recv, c.obuf, c.orecv, c.mod};
-    for (const void* p : ptrs) mix(reinterpret_cast<uintptr_t>(p));
-    for (size_t q = 0; q < Rs.size(); ++q) {
-      const ReqShard* sh = c.shq[q];
-      const ReqDev* rd = c.rdq[q];
-      const void* rp[] = {sh->lat.p, sh->vel.p, sh->T.p, sh->cosb.p, sh->sinb.p, sh->pe.p, rd->mod.p, rd->dt.p,
-                          rd->step.p};
-      for (const void* p : rp) mix(reinterpret_cast<uintptr_t>(p));
-      mix((uint64_t)Rs[q]->id);
+    for (const RankCtx& c : E.rc) {
+      const void* ptrs[] = {c.x, c.u, c.qkv, c.cat, c.hbuf, c.latb, c.pack, c.recv, c.obuf, c.orecv, c.mod};
+      for (const void* p : ptrs) mix(reinterpret_cast<uintptr_t>(p));
+      for (size_t q = 0; q < Rs.size(); ++q) {
+        const ReqShard* sh = c.shq[q];
+        const ReqDev* rd = c.rdq[q];
+        const void* rp[] = {sh->lat.p, sh->vel.p, sh->T.p, sh->cosb.p, sh->sinb.p, sh->pe.p, rd->mod.p, rd->dt.p,
+                            rd->step.p};
+        for (const void* p : rp) mix(reinterpret_cast<uintptr_t>(p));
+        mix((uint64_t)Rs[q]->id);
+      }
+      mix((uint64_t)c.rows);
+      mix((uint64_t)c.si);
     }
+    mix((uint64_t)E.rc.size());
     mix((uint64_t)gi);
-    mix((uint64_t)c.rows);
     mix((uint64_t)Rs.size());
     mix((uint64_t)e->prof);   // a profiled graph carries event-record nodes around every launch
     auto it = slot.graphs.find(key);
