@@ -1465,7 +1465,14 @@ static void launch_fa2(const CUtensorMap& tq, const CUtensorMap& tk, const CUten
 
 // KV-split factor for a launch of C = ceil(L/256) x H CTAs: the S in 1..8 minimising the estimated
 // makespan (below), each split >= 4 key tiles.
+static int KV_MIN_TILES = 4, KV_SPLIT_COST = 6;   // TSV_KV_MIN / TSV_KV_COST override (tuning)
 static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
+  static bool env_read = false;
+  if (!env_read) {
+    if (const char* v = getenv("TSV_KV_MIN")) KV_MIN_TILES = atoi(v);
+    if (const char* v = getenv("TSV_KV_COST")) KV_SPLIT_COST = atoi(v);
+    env_read = true;
+  }
   AttnSplitArgs a;
   if (!w || !w->cnt || !w->ws) return a;
   static int sms_of[64] = {0};
@@ -1484,8 +1491,8 @@ static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
     double bestc = (double)((C + sms - 1) / sms) * (n_all + 2);
     for (int S = 2; S <= 8; ++S) {
       const int tps = (n_all + S - 1) / S;
-      if (tps < 4) break;
-      const double cost = (double)((C * S + sms - 1) / sms) * (tps + 6);
+      if (tps < KV_MIN_TILES) break;
+      const double cost = (double)((C * S + sms - 1) / sms) * (tps + KV_SPLIT_COST);
       if (cost < bestc * 0.95) { bestc = cost; best = S; }
     }
   }
