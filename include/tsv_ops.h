@@ -85,7 +85,7 @@ tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int
 
 /* a6: O = softmax(q k^T / sqrt(D)) v, non-causal, per head h < H; q(l, h) at q + l*ldq + h*D
  * (bf16, same for k, v, o).  D in {64, 128}.  Operands and row strides 16-byte aligned.
- * impl 0: the tcgen05/TMEM kernel the step uses (= impl 52 for D = 128, 53 for D = 64; the
+ * impl 0: the tcgen05/TMEM kernel the step uses (= impl 51 for D = 128, 52 for D = 64; the
  * environment variables TSV_ATTN_D128 / TSV_ATTN_D64 select another impl >= 3 for the step);
  * impl 1: the mma.sync (FA2-style) baseline, kept only for comparison; impl 2: the one-query-tile
  * tcgen05 kernel (P in shared memory); variants of the two-query-tile kernel (tuning sweeps):

@@ -1598,7 +1598,7 @@ static int default_version(int D) {
   int& r = v[D == 128];
   if (r < 0) {
     const char* e = getenv(D == 128 ? "TSV_ATTN_D128" : "TSV_ATTN_D64");
-    r = e ? atoi(e) : (D == 128 ? 52 : 53);   // lazy max; 2 (D = 128) / 3 (D = 64) of 8 exp2 pairs by polynomial
+    r = e ? atoi(e) : (D == 128 ? 51 : 52);   // lazy max; 1 (D = 128) / 2 (D = 64) of 8 exp2 pairs by polynomial (in-step A/B)
     if (r < 3) r = 3;
   }
   return r;
