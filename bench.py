@@ -259,12 +259,29 @@ def run_ours(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    # TSV_BENCH_ONE_GPU=1 (tests only): every rank on device 0, gloo for the host-side collectives and
+    # the fused CUDA-IPC transport for the step (NCCL refuses two ranks on one GPU) -- exercises the
+    # N > 1 code path of this script on a one-GPU box; the numbers are not a scaling measurement
+    one_gpu = os.environ.get("TSV_BENCH_ONE_GPU") == "1" and world > 1
+    local = 0 if one_gpu else local
+    red_dev = "cpu" if one_gpu else "cuda"
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if one_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     mdl = MODELS[args.model]
     eng = tsv.Engine(args.model, devices=[local], rank_base=rank, world_size=world)
-    if world > 1:
+    if one_gpu:
+        g = eng.group_create(list(range(world)))
+        blob = eng.group_ipc_export(g, max_tokens=(args.res // 16) ** 2 + mdl["Lt"], max_evals=2)
+        blobs = [None] * world
+        dist.all_gather_object(blobs, blob)
+        eng.group_ipc_import(g, blobs)
+        eng.set_transport(True)
+        transport = "fused-ipc (one GPU, test mode)"
+    elif world > 1:
         obj = [tsv.nccl_unique_id() if rank == 0 else None, tsv.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         eng.init_world(obj[0])
@@ -316,7 +333,7 @@ def run_ours(args):
     launches = eng.kernel_count() - kc0
     ms = total_ms / K
     if world > 1:
-        t = torch.tensor([ms], device="cuda")
+        t = torch.tensor([ms], device=red_dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
 
@@ -347,7 +364,7 @@ def run_ours(args):
             e2e_times.append((time.perf_counter() - t0) * 1e3)
     e2e_ms = statistics.median(e2e_times)
     if world > 1:
-        t = torch.tensor([e2e_ms], device="cuda")
+        t = torch.tensor([e2e_ms], device=red_dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_ms = float(t.item())
 

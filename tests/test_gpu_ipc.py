@@ -46,3 +46,25 @@ def test_two_process_ipc_fused_equals_in_process(model, tmp_path):
     x, v = eng.read_latent(req), eng.read_velocity(req)
     eng.close()
     assert np.array_equal(got["x"], x) and np.array_equal(got["v"], v)
+
+
+def test_bench_two_ranks_one_gpu():
+    """bench.py's N > 1 code path (torchrun, two ranks, max-over-ranks timing, e2e, JSON line) on a
+    one-GPU box: TSV_BENCH_ONE_GPU=1 puts both ranks on device 0 with the fused CUDA-IPC transport
+    (NCCL refuses two ranks on one GPU).  Not a scaling measurement."""
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import json
+    port = _port()
+    env = dict(os.environ, TSV_BENCH_ONE_GPU="1")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr",
+           "127.0.0.1", "--master-port", str(port), os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "3",
+           "--warmup", "3", "--res", "256", "--no-cpu-baseline"]
+    r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=600, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["config"]["sp"] == 2 and "fused-ipc" in d["config"]["transport"]
+    assert d["value"] > 0 and d["e2e"]["value"] > 0 and d["gpu_launches"] > 0
+    assert d["warmup"] == 3 and d["steps"] == 3
