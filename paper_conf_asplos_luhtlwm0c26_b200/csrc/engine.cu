@@ -174,6 +174,12 @@ struct Slot {
 };
 constexpr int SEM_INTS = 4096;
 constexpr size_t SPLIT_WS_BYTES = 128u << 20;
+// TSV_GEMM_BN / TSV_GEMM_PAIR (read at engine creation): force the step GEMMs' tile width / CTA
+// pairing (planner A/B measurements only; 0 / -1 = the planner's choice)
+static int gemm_force_env(const char* name, int dflt) {
+  const char* v = getenv(name);
+  return v ? atoi(v) : dflt;
+}
 // TSV_SPLITK=0 (read at engine creation) disables split-K for small GEMM launches (A/B measurements)
 static bool splitk_env() {
   const char* v = getenv("TSV_SPLITK");
@@ -246,6 +252,7 @@ struct tsv_engine {
   Model model;
   uint64_t weight_seed = 0;
   bool splitk = true;      // split-K for small fp32-stream GEMM launches (TSV_SPLITK at creation)
+  int force_bn = 0, force_pair = -1;   // TSV_GEMM_BN / TSV_GEMM_PAIR (A/B only)
   int rank_base = 0, n_local = 0, world = 0;
   std::vector<Slot> slots;
   std::map<int, std::unique_ptr<DeviceState>> devs;
@@ -325,7 +332,10 @@ static tsv_status gemm(tsv_engine* e, Slot& s, const bf16* A, long long lda, con
   GemmPlan p;
   const char* err = nullptr;
   const GemmSplitWs w = s.sws();
-  if (gemm_plan(&p, A, lda, Wt, ldw, M, N, K, epi, s.ds->num_sms, &err, 0, -1, e->splitk ? &w : nullptr))
+  int fbn = e->force_bn;
+  if (fbn && (N % fbn || (epi.qk_h && fbn < epi.qk_D))) fbn = 0;   // keep the planner's where illegal
+  if (gemm_plan(&p, A, lda, Wt, ldw, M, N, K, epi, s.ds->num_sms, &err, fbn, fbn ? e->force_pair : -1,
+                e->splitk ? &w : nullptr))
     return fail(TSV_E_INVAL, "%s (M=%d N=%d K=%d)", err, M, N, K);
   const double out_b = (epi.mode <= EPI_SPLIT_GELU) ? 2.0
                        : (epi.mode == EPI_STORE_F32 ? 4.0 : (epi.mode == EPI_CFG_EULER ? 16.0 : 8.0));
@@ -346,7 +356,9 @@ static tsv_status gemm_multi(tsv_engine* e, Slot& s, const GemmProblem* probs, i
   GemmPlan p;
   const char* err = nullptr;
   const GemmSplitWs w = s.sws();
-  if (gemm_plan_multi(&p, nz, n, N, K, s.ds->num_sms, &err, 0, -1, e->splitk ? &w : nullptr))
+  int fbn = e->force_bn;
+  if (fbn && (N % fbn || (nz[0].epi.qk_h && fbn < nz[0].epi.qk_D))) fbn = 0;   // keep the planner's where illegal
+  if (gemm_plan_multi(&p, nz, n, N, K, s.ds->num_sms, &err, fbn, fbn ? e->force_pair : -1, e->splitk ? &w : nullptr))
     return fail(TSV_E_INVAL, "%s (N=%d K=%d)", err, N, K);
   double fl = 0, by = 2.0 * N * K * n;
   for (int i = 0; i < n; ++i) {
@@ -1488,6 +1500,8 @@ tsv_status tsv_engine_create(const tsv_model_desc* model, const int* devices, in
   if (!build_model(*model, &e->model, &err)) return fail(TSV_E_INVAL, "%s", err.c_str());
   e->weight_seed = weight_seed;
   e->splitk = splitk_env();
+  e->force_bn = gemm_force_env("TSV_GEMM_BN", 0);
+  e->force_pair = gemm_force_env("TSV_GEMM_PAIR", -1);
   if (const char* li = getenv("TSV_LN_IMPL")) g_ln_impl = atoi(li);   // LN-modulate variant (A/B)
   e->rank_base = rank_base;
   e->n_local = n_local;
