@@ -199,8 +199,11 @@ struct ReqShard {
   int64_t t0 = 0, nt = 0, i0 = 0, ni = 0;  // txt rows [t0, t0+nt), img rows [i0, i0+ni)
   DevBuf lat, vel, T, cosb, sinb;
   DevBuf pe;  // SD3: fp32 [ni, h] sin-cos position embedding of this shard's image rows
+  DevBuf txt;         // fp32 [branches][nt, h]: a1 text embedding T W^T + b (constant per request)
+  bool txt_ok = false;  // txt computed (enqueued) on this shard's stream
   void release() {
-    lat.release(); vel.release(); T.release(); cosb.release(); sinb.release(); pe.release();
+    lat.release(); vel.release(); T.release(); cosb.release(); sinb.release(); pe.release(); txt.release();
+    txt_ok = false;
   }
 };
 
@@ -531,6 +534,8 @@ static tsv_status setup_shard(tsv_engine* e, Request& R, int si, int rank_in_gro
   TRY(dev_alloc(sh.lat, s.device, std::max<size_t>(1, sh.ni) * m.in * 4));
   TRY(dev_alloc(sh.vel, s.device, std::max<size_t>(1, sh.ni) * m.in * 4));
   TRY(dev_alloc(sh.T, s.device, std::max<size_t>(1, sh.nt) * m.B * m.ctx * 2));
+  TRY(dev_alloc(sh.txt, s.device, std::max<size_t>(1, sh.nt) * m.B * m.h * 4));
+  sh.txt_ok = false;
   const size_t rows = sh.nt + sh.ni;
   if (sh.nt)
     for (int b = 0; b < m.B; ++b)
@@ -860,6 +865,35 @@ static void select_rows(StepEnv& E, RankCtx& c) {
   }
 }
 
+
+// a1 text embedding txt = T W_txt^T + b: constant per (request, shard), so it is computed on the
+// shard's first step into sh.txt and copied into the residual stream rows [b R, b R + nt) on every
+// step (a 4 x ctx/h smaller copy instead of an M = nt, K = 4096 weight-streaming GEMM).  per_req =
+// evaluations per request (1 FLUX, 2 SD3 CFG branches; branch br uses T rows br * nt).
+static tsv_status txt_embed(tsv_engine* e, Slot& s, const std::vector<ReqShard*>& shq, float* x, int64_t R, int64_t nt,
+                            int B, int per_req) {
+  if (!nt) return TSV_OK;
+  const Model& m = e->model;
+  const int h = m.h;
+  GemmProblem pt[GEMM_MAX_PROBLEMS];
+  int n = 0;
+  for (int b = 0; b < B; ++b) {
+    ReqShard* sh = shq[b / per_req];
+    const int br = b % per_req;
+    if (!sh->txt_ok)
+      pt[n++] = {reinterpret_cast<bf16*>(sh->T.p) + br * nt * m.ctx, m.ctx, e->W(s, 2), m.ctx, (int)nt,
+                 epi_of(EPI_STORE_F32, reinterpret_cast<float*>(sh->txt.p) + br * nt * h, h, e->W(s, 3))};
+  }
+  if (n) TRY(gemm_multi(e, s, pt, n, h, m.ctx));
+  for (int b = 0; b < B; ++b) {
+    ReqShard* sh = shq[b / per_req];
+    sh->txt_ok = true;
+    CK(cudaMemcpyAsync(x + b * R * h, reinterpret_cast<float*>(sh->txt.p) + (b % per_req) * nt * h,
+                       nt * h * sizeof(float), cudaMemcpyDeviceToDevice, s.stream));
+  }
+  return TSV_OK;
+}
+
 static tsv_status run_step(StepEnv& E) {
   tsv_engine* e = E.e;
   const Model& m = e->model;
@@ -876,7 +910,7 @@ static tsv_status run_step(StepEnv& E) {
     Slot& s = *c.s;
     CK(cudaSetDevice(s.device));
     const int64_t R = c.rows;
-    GemmProblem pi[GEMM_MAX_PROBLEMS], pt[GEMM_MAX_PROBLEMS];
+    GemmProblem pi[GEMM_MAX_PROBLEMS];
     for (int b = 0; b < B; ++b) {
       if (c.ni) {
         ProfScope ps(e, s, KC_OTHER, 0.0, 6.0 * c.ni * m.in);
@@ -885,11 +919,9 @@ static tsv_status run_step(StepEnv& E) {
       }
       pi[b] = {c.latb + b * c.ni * m.in, m.in, e->W(s, 0), m.in, (int)c.ni,
                epi_of(EPI_STORE_F32, c.x + (b * R + c.nt) * h, h, e->W(s, 1))};
-      pt[b] = {reinterpret_cast<bf16*>(c.shq[b]->T.p), m.ctx, e->W(s, 2), m.ctx, (int)c.nt,
-               epi_of(EPI_STORE_F32, c.x + b * R * h, h, e->W(s, 3))};
     }
     TRY(gemm_multi(e, s, pi, B, h, m.in));
-    TRY(gemm_multi(e, s, pt, B, h, m.ctx));
+    TRY(txt_embed(e, s, c.shq, c.x, R, c.nt, B, 1));
   }
   // double-stream blocks
   for (int j = 0; j < m.d.n_double; ++j) {
@@ -1048,13 +1080,7 @@ static tsv_status run_step_sd3(StepEnv& E) {
         CK(cudaMemcpyAsync(xi + R * h, xi, c.ni * h * 4, cudaMemcpyDeviceToDevice, s.stream));
       }
     }
-    if (c.nt) {
-      GemmProblem pt[GEMM_MAX_PROBLEMS];
-      for (int b = 0; b < B; ++b)
-        pt[b] = {reinterpret_cast<bf16*>(c.shq[b / 2]->T.p) + (b % 2) * c.nt * m.ctx, m.ctx, e->W(s, 2), m.ctx,
-                 (int)c.nt, epi_of(EPI_STORE_F32, c.x + b * R * h, h, e->W(s, 3))};
-      TRY(gemm_multi(e, s, pt, B, h, m.ctx));
-    }
+    TRY(txt_embed(e, s, c.shq, c.x, R, c.nt, B, 2));
   }
   for (int j = 0; j < nd; ++j) {
     const bool last = j == nd - 1;  // context_pre_only
@@ -1363,6 +1389,7 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
                             rd->step.p};
         for (const void* p : rp) mix(reinterpret_cast<uintptr_t>(p));
         mix((uint64_t)Rs[q]->id);
+        mix((uint64_t)sh->txt_ok);   // the first step on a shard also computes the text embedding
       }
       mix((uint64_t)c.rows);
       mix((uint64_t)c.si);
