@@ -338,15 +338,20 @@ __global__ void __launch_bounds__(AT_THREADS, 1)
 // in-order tcgen05 pipe makes "S_t{j} complete" imply "O_t holds tiles < j", so a rare rescale
 // of O (running max grew by > 2^8) needs no extra wait.
 // TMEM: S0 | S1 | O0 | O1 (128 + 128 + D + D fp32 columns).  Smem: Q0, Q1, 2 K/V stages.
+#ifndef TSV_FA_NST64
+#define TSV_FA_NST64 4
+#endif
 template <int D>
 struct FaCfg {
   static constexpr int NSUB = D / 64;
   static constexpr int Q_TILE = AT_BM * D * 2;
   static constexpr int KV_TILE = AT_BN * D * 2;
+  // K/V ring depth: D = 128 fills shared memory with 2 stages; D = 64 has room for 4
+  static constexpr int NST = TSV_FA_NST64 > 0 && D == 64 ? TSV_FA_NST64 : 2;
   static constexpr int OFF_Q = 0;                        // 2 tiles
-  static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // 2 stages
-  static constexpr int OFF_V = OFF_K + 2 * KV_TILE;      // 2 stages
-  static constexpr int OFF_BAR = OFF_V + 2 * KV_TILE;
+  static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // NST stages
+  static constexpr int OFF_V = OFF_K + NST * KV_TILE;    // NST stages
+  static constexpr int OFF_BAR = OFF_V + NST * KV_TILE;
   static constexpr int SMEM = OFF_BAR + 256 + 1024;
   static constexpr int O_COL = 256;
 };
@@ -380,14 +385,15 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
+  constexpr int NST = C::NST;
   uint64_t* q_full = bars + 0;
-  uint64_t* kv_full = bars + 1;    // [2 stages]
-  uint64_t* kv_empty = bars + 3;   // [2 stages]
-  uint64_t* s_full = bars + 5;     // [2 q-tiles]
-  uint64_t* p_full = bars + 7;     // [2 q-tiles]  (SPLIT: first half of P)
-  uint64_t* o_done = bars + 9;     // [2 q-tiles]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 12);
-  uint64_t* p_full2 = bars + 14;   // [2 q-tiles]  SPLIT: second half of P
+  uint64_t* kv_full = bars + 1;              // [NST stages]
+  uint64_t* kv_empty = bars + 1 + NST;       // [NST stages]
+  uint64_t* s_full = bars + 1 + 2 * NST;     // [2 q-tiles]
+  uint64_t* p_full = bars + 3 + 2 * NST;     // [2 q-tiles]  (SPLIT: first half of P)
+  uint64_t* o_done = bars + 5 + 2 * NST;     // [2 q-tiles]
+  uint64_t* p_full2 = bars + 7 + 2 * NST;    // [2 q-tiles]  SPLIT: second half of P
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 10 + 2 * NST);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int head = blockIdx.y;
@@ -402,9 +408,11 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     tma_prefetch_desc(&tmK);
     tma_prefetch_desc(&tmV);
     mbar_init(q_full, 1);
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < NST; ++i) {
       mbar_init(&kv_full[i], 1);
       mbar_init(&kv_empty[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
       mbar_init(&s_full[i], 1);
       mbar_init(&p_full[i], 128);
       mbar_init(&p_full2[i], 128);
@@ -431,8 +439,8 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
           tma_load_3d(&tmQ, q_full, sm + C::OFF_Q + t * C::Q_TILE + s * (AT_BM * 128), s * 64, head,
                       q0 + t * AT_BM);
       for (int j = 0; j < n_tiles; ++j) {
-        const int st = j & 1;
-        if (j >= 2) mbar_wait(&kv_empty[st], ((j - 2) >> 1) & 1);
+        const int st = j % NST;
+        if (j >= NST) mbar_wait(&kv_empty[st], ((j / NST) - 1) & 1);
         mbar_arrive_expect_tx(&kv_full[st], 2 * C::KV_TILE);
         for (int s = 0; s < C::NSUB; ++s) {
           tma_load_3d(&tmK, &kv_full[st], sm + C::OFF_K + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
@@ -455,7 +463,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     mbar_wait(q_full, 0);
     auto issue_s = [&](int t, int j) {
       const uint64_t dq = dq0 + (uint64_t)((t * C::Q_TILE) >> 4);
-      const uint64_t dk = dk0 + (uint64_t)(((j & 1) * C::KV_TILE) >> 4);
+      const uint64_t dk = dk0 + (uint64_t)(((j % NST) * C::KV_TILE) >> 4);
       if (elect_one()) {
 #pragma unroll
         for (int kk = 0; kk < D / 16; ++kk) {
@@ -467,7 +475,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       __syncwarp();
     };
     auto issue_pv = [&](int t, int j, bool release) {
-      const uint64_t dv = dv0 + (uint64_t)(((j & 1) * C::KV_TILE) >> 4);
+      const uint64_t dv = dv0 + (uint64_t)(((j % NST) * C::KV_TILE) >> 4);
       mbar_wait(&p_full[t], j & 1);
       tc_fence_after();
       if (elect_one()) {
@@ -480,12 +488,12 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
           umma_bf16_ts(tmem + C::O_COL + t * D, tmem + t * 128 + kk * 8, dv + (uint64_t)(kk * (2048 >> 4)), idesc_o,
                        (j | kk) != 0);
         }
-        if (release) umma_commit(&kv_empty[j & 1]);
+        if (release) umma_commit(&kv_empty[j % NST]);
       }
       __syncwarp();
     };
     for (int j = 0; j < n_tiles; ++j) {
-      mbar_wait(&kv_full[j & 1], (j >> 1) & 1);
+      mbar_wait(&kv_full[j % NST], (j / NST) & 1);
       tc_fence_after();
       for (int t = 0; t < 2; ++t) {
         if (j > 0) issue_pv(t, j - 1, t == 1);
