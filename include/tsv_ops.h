@@ -85,15 +85,10 @@ tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int
 
 /* a6: O = softmax(q k^T / sqrt(D)) v, non-causal, per head h < H; q(l, h) at q + l*ldq + h*D
  * (bf16, same for k, v, o).  D in {64, 128}.  Operands and row strides 16-byte aligned.
- * impl 0: the tcgen05/TMEM kernel the step uses (= impl 51 for D = 128, 52 for D = 64; the
- * environment variables TSV_ATTN_D128 / TSV_ATTN_D64 select another impl >= 3 for the step);
- * impl 1: the mma.sync (FA2-style) baseline, kept only for comparison; impl 2: the one-query-tile
- * tcgen05 kernel (P in shared memory); variants of the two-query-tile kernel (tuning sweeps):
- * 11..15: 1..5 of every 8 exp2 pairs evaluated by polynomial on the FMA pipe instead of MUFU;
- * 21..24: the same with P handed over in two halves; 40..44: 64-key K/V tiles with double-buffered
- * S; 50..54: lazy row max (no per-tile max unless a row's tile sum exceeds 2^16);
- * 60..63: CTA-pair (cta_group::2, M = 256) kernel with lazy max, D = 128 only.
- * Other values: TSV_E_INVAL. */
+ * impl 0: the tcgen05/TMEM kernel the step uses (= impl 51 for D = 128, 53 for D = 64; the
+ * environment variables TSV_ATTN_D128 / TSV_ATTN_D64 select another impl for the step);
+ * 50..54: the same kernel with 0..4 of every 8 exp2 pairs evaluated by polynomial on the FMA pipe
+ * instead of MUFU.EX2 (tuning sweeps).  Other values: TSV_E_INVAL. */
 tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
                             void* o, int64_t ldo, int L, int H, int D, int impl, void* stream);
 

@@ -11,7 +11,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 BUILD = os.path.join(ROOT, "build", "tsv")
 LIB = os.path.join(PKG, "libtsv.so")
-SOURCES = ["gemm.cu", "attention.cu", "attention_tc.cu", "elementwise.cu", "engine.cu", "model.cpp", "sched.cpp"]
+SOURCES = ["gemm.cu", "attention_tc.cu", "elementwise.cu", "engine.cu", "model.cpp", "sched.cpp"]
 HEADERS = ["ptx.cuh", "kernels.h", "model.h"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

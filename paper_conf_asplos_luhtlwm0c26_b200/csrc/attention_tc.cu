@@ -1,17 +1,36 @@
 // Joint text+image attention on the 5th-gen tensor cores (S:§8(a) a6):
-//   O = softmax(q k^T / sqrt(D)) v, non-causal, per head, fp32 online softmax, bf16 operands.
+//   O = softmax(q k^T / sqrt(D)) v, non-causal, per head, fp32 softmax, bf16 operands.
 //
-// One CTA = one (head, 128-query tile).  Warp roles:
-//   warp 0      TMA producer: Q once, then K/V tiles of 128 keys into a 2-stage ring
+// One CTA = one head x 256 queries as two 128-query tiles t = 0, 1 that share every K/V tile
+// (half the K/V traffic per query).  Warp roles:
+//   warp 0      TMA producer: Q0, Q1 once, then K/V tiles of 128 keys into an NST-stage ring
 //               (3-D tensor maps [rows][heads][D] -> one map serves every head and layout);
-//   warp 1      single-thread tcgen05.mma issuer:  S_j = Q K_j^T into one of two TMEM S buffers
-//               (issued one tile ahead), then O += P_j V_j (V consumed MN-major straight from the
-//               TMA tile, no transpose);
-//   warps 4-7   softmax: thread i owns query row i (TMEM lane i): tcgen05.ld of its 128 scores,
-//               row max / exp2 / row sum in registers, P_j as bf16 into a 128B-swizzled K-major
-//               smem tile (double-buffered), conditional O rescale (only when the running max grows
-//               by more than 2^8, so P stays <= 256 and rescales are rare), final 1/l and store.
-// TMEM: S0 | S1 | O  (128 + 128 + D fp32 columns).
+//   warp 1      tcgen05.mma issuer (the whole warp runs the loop, one elected lane issues):
+//               S_t(j) = Q_t K_j^T into TMEM, O_t += P_t(j) V_j with P read from TMEM and V
+//               consumed MN-major straight from the TMA tile (no transpose, no smem P);
+//   warps 4-11  two softmax warpgroups (4-7: tile 0, 8-11: tile 1), thread = query row = TMEM lane.
+// The two warpgroups ping-pong with the tensor core: while WG0 turns S_0(j) into P_0(j), the MMA
+// warp runs PV_1(j-1) and S_1(j), and vice versa.  P_t(j) is written back into the S_t columns as
+// bf16 (tcgen05.st), so S_t(j+1) must follow PV_t(j): the MMA warp issues PV_t(j) before S_t(j+1),
+// and the in-order tcgen05 pipe makes "S_t(j) complete" imply "O_t holds tiles < j" (a rare O
+// rescale needs no extra wait).
+// TMEM: S0 | S1 | O0 | O1 (128 + 128 + D + D fp32 columns).  Smem: Q0, Q1, NST K/V stages.
+//
+// Softmax (lazy row max): P = 2^(s * scale_log2 - m_ref) is evaluated with the running reference
+// m_ref directly, without a per-tile max: the tile's row sum bounds every p in it (p <= sum), so a
+// row whose sum stays <= 2^16 needs no rescale (m_ref only stabilises: softmax is exact for any
+// reference that keeps p finite).  Otherwise (the max grew a lot: early tiles) the warp reloads S
+// from TMEM and takes the exact path (row max, conditional O rescale when the max grows by > 2^8).
+// Without the max the four TMEM loads of S are pipelined under the exponentials.  NPOLY of every 8
+// exp2 pairs are evaluated on the FMA pipe (Cody-Waite split + cubic) to relieve MUFU.EX2.
+//
+// KV split (blockIdx.z): for launches with too few CTAs (SP = 4/8 head shards), each split covers
+// a key range and the last split of a 32-row warp merges the (O, m, l) partials in range order.
+//
+// Measured dead ends (profiles/README.md): one query tile per CTA with P in shared
+// memory; 64-key tiles with double-buffered S (the N = 64 S MMA re-reads Q from shared memory at
+// 192 B/clk); P handed over in two halves; CTA-pair (cta_group::2) tiles (-17 %: the pair couples
+// both CTAs' softmax chains); two softmax warps per row; packed ex2 (two MUFU ops per instruction).
 #include <cfloat>
 #include <cstdlib>
 #include <cudaTypedefs.h>
@@ -23,26 +42,10 @@ namespace tsv {
 
 namespace {
 
-constexpr int AT_BM = 128;     // queries per CTA
+constexpr int AT_BM = 128;     // queries per tile
 constexpr int AT_BN = 128;     // keys per tile
-constexpr int AT_THREADS = 256;
 constexpr float RESCALE_THRESHOLD = 8.0f;  // log2 domain
-
-template <int D>
-struct AttnCfg {
-  static constexpr int NSUB = D / 64;                  // 64-wide sub-tiles of the head dim
-  static constexpr int Q_BYTES = AT_BM * D * 2;
-  static constexpr int KV_TILE = AT_BN * D * 2;         // one K (or V) tile
-  static constexpr int P_BYTES = AT_BM * AT_BN * 2;     // 2 sub-tiles of 64 keys
-  static constexpr int OFF_Q = 0;
-  static constexpr int OFF_K = OFF_Q + Q_BYTES;              // 2 stages
-  static constexpr int OFF_V = OFF_K + 2 * KV_TILE;          // 2 stages
-  static constexpr int OFF_P = OFF_V + 2 * KV_TILE;          // 2 buffers
-  static constexpr int OFF_BAR = OFF_P + 2 * P_BYTES;
-  static constexpr int SMEM = OFF_BAR + 256 + 1024;
-  static constexpr int TMEM_COLS = 512;
-  static constexpr int O_COL = 256;
-};
+constexpr float LAZY_LIMIT = 65536.0f;     // 2^16
 
 __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&r)[32]) {
   asm volatile(
@@ -59,24 +62,14 @@ __device__ __forceinline__ float fast_exp2(float x) {  // MUFU.EX2; ex2(-inf) = 
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
   return y;
 }
-// 2^x without the MUFU: x = n + f (n = round(x), |f| <= 1/2), 2^f by a cubic (Taylor of e^(f ln2),
-// rel. error <= 7e-4 on |f| <= 1/2), 2^n added to the exponent field.  x is clamped at -126 so the
-// exponent add cannot wrap (the true value is < 2^-126 there).  Finite x only.
-__device__ __forceinline__ float poly_exp2(float x) {
-  x = fmaxf(x, -126.0f);
-  const float t = x + 12582912.0f;          // 1.5 * 2^23: round(x) lands in the low mantissa bits
-  const float n = t - 12582912.0f;
-  const float f = x - n;
-  float p = fmaf(0.0555041086648216f, f, 0.2402265069591007f);
-  p = fmaf(p, f, 0.6931471805599453f);
-  p = fmaf(p, f, 1.0f);
-  return __int_as_float(__float_as_int(p) + (__float_as_int(t) << 23));
-}
-// The same on a pair, with the sm_100 paired FP32 ops (FADD2 / FFMA2: two lanes per instruction).
+// 2^x without the MUFU on a pair, with the sm_100 paired FP32 ops (FADD2 / FFMA2): x = n + f
+// (n = round(x), |f| <= 1/2), 2^f by a cubic (Taylor of e^(f ln2), rel. error <= 7e-4 on
+// |f| <= 1/2, below the bf16 rounding P gets anyway), 2^n added to the exponent field.  x is
+// clamped at -126 so the exponent add cannot wrap (the true value is < 2^-126 there).
 __device__ __forceinline__ float2 poly_exp2_x2(float2 x) {
   x.x = fmaxf(x.x, -126.0f);
   x.y = fmaxf(x.y, -126.0f);
-  const float2 magic = make_float2(12582912.0f, 12582912.0f);
+  const float2 magic = make_float2(12582912.0f, 12582912.0f);   // 1.5 * 2^23: round(x) in the low bits
   const float2 t = __fadd2_rn(x, magic);
   const float2 n = __fadd2_rn(t, make_float2(-12582912.0f, -12582912.0f));
   const float2 f = __ffma2_rn(n, make_float2(-1.0f, -1.0f), x);
@@ -104,270 +97,22 @@ __host__ __device__ constexpr uint32_t make_idesc_bf16_bmn(int M, int N) {
 }  // namespace
 
 template <int D>
-__global__ void __launch_bounds__(AT_THREADS, 1)
-    attention_tc_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
-                        const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
-                        float scale_log2) {
-  using C = AttnCfg<D>;
-  extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
-  uint64_t* q_full = bars + 0;
-  uint64_t* kv_full = bars + 1;    // [2]
-  uint64_t* kv_empty = bars + 3;   // [2]
-  uint64_t* s_full = bars + 5;     // [2]
-  uint64_t* s_free = bars + 7;     // [2]
-  uint64_t* p_full = bars + 9;     // [2]
-  uint64_t* pv_done = bars + 11;   // [2]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 14);
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int head = blockIdx.y;
-  const int q0 = blockIdx.x * AT_BM;
-  const int n_tiles = (L + AT_BN - 1) / AT_BN;
-
-  if (warp == 0 && lane == 0) {
-    tma_prefetch_desc(&tmQ);
-    tma_prefetch_desc(&tmK);
-    tma_prefetch_desc(&tmV);
-    mbar_init(q_full, 1);
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(&kv_full[i], 1);
-      mbar_init(&kv_empty[i], 1);
-      mbar_init(&s_full[i], 1);
-      mbar_init(&s_free[i], 128);
-      mbar_init(&p_full[i], 128);
-      mbar_init(&pv_done[i], 1);
-    }
-    fence_mbar_init();
-  }
-  if (warp == 2) tmem_alloc<C::TMEM_COLS>(tmem_slot);
-  tc_fence_before();
-  __syncthreads();
-  tc_fence_after();
-  const uint32_t tmem = *tmem_slot;
-  grid_dep_wait();
-
-  if (warp == 0) {
-    if (lane == 0) {
-      // ---------------------------------------------------------------- producer
-      mbar_arrive_expect_tx(q_full, C::Q_BYTES);
-      for (int s = 0; s < C::NSUB; ++s)
-        tma_load_3d(&tmQ, q_full, sm + C::OFF_Q + s * (AT_BM * 128), s * 64, head, q0);
-      for (int j = 0; j < n_tiles; ++j) {
-        const int st = j & 1;
-        if (j >= 2) mbar_wait(&kv_empty[st], ((j - 2) >> 1) & 1);
-        mbar_arrive_expect_tx(&kv_full[st], 2 * C::KV_TILE);
-        for (int s = 0; s < C::NSUB; ++s) {
-          tma_load_3d(&tmK, &kv_full[st], sm + C::OFF_K + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
-                      j * AT_BN);
-          tma_load_3d(&tmV, &kv_full[st], sm + C::OFF_V + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
-                      j * AT_BN);
-        }
-      }
-    }
-  } else if (warp == 1) {
-    if (lane == 0) {
-      // ---------------------------------------------------------------- MMA issuer
-      constexpr uint32_t idesc_s = make_idesc_bf16(AT_BM, AT_BN);
-      constexpr uint32_t idesc_o = make_idesc_bf16_bmn(AT_BM, D);
-      const uint32_t sQ = smem_u32(sm + C::OFF_Q);
-      mbar_wait(q_full, 0);
-      auto issue_s = [&](int j) {
-        const int st = j & 1;
-        mbar_wait(&kv_full[st], (j >> 1) & 1);
-        if (j >= 2) mbar_wait(&s_free[st], ((j - 2) >> 1) & 1);
-        tc_fence_after();
-        const uint32_t sK = smem_u32(sm + C::OFF_K + st * C::KV_TILE);
-#pragma unroll
-        for (int kk = 0; kk < D / 16; ++kk) {
-          const uint32_t off = (kk >> 2) * (AT_BM * 128) + (kk & 3) * 32;
-          const uint32_t offk = (kk >> 2) * (AT_BN * 128) + (kk & 3) * 32;
-          umma_bf16_ss(tmem + st * 128, make_sw128_desc(sQ + off), make_sw128_desc(sK + offk), idesc_s, kk > 0);
-        }
-        umma_commit(&s_full[st]);
-      };
-      issue_s(0);
-      for (int j = 0; j < n_tiles; ++j) {
-        if (j + 1 < n_tiles) issue_s(j + 1);
-        const int st = j & 1;
-        mbar_wait(&p_full[st], (j >> 1) & 1);
-        tc_fence_after();
-        const uint32_t sP = smem_u32(sm + C::OFF_P + st * C::P_BYTES);
-        const uint32_t sV = smem_u32(sm + C::OFF_V + st * C::KV_TILE);
-#pragma unroll
-        for (int kk = 0; kk < AT_BN / 16; ++kk) {
-          const uint32_t offp = (kk >> 2) * (AT_BM * 128) + (kk & 3) * 32;
-          umma_bf16_ss(tmem + C::O_COL, make_sw128_desc(sP + offp),
-                       make_sw128_mn_desc(sV + kk * 2048, AT_BN * 128), idesc_o, (j | kk) != 0);
-        }
-        umma_commit(&pv_done[st]);
-        umma_commit(&kv_empty[st]);
-      }
-    }
-  } else if (warp >= 4) {
-    // ---------------------------------------------------------------- softmax (thread = query row)
-    const int wq = warp - 4;
-    const int row = wq * 32 + lane;
-    const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
-    float m_ref = -FLT_MAX, l_sum = 0.f;
-    for (int j = 0; j < n_tiles; ++j) {
-      const int st = j & 1;
-      mbar_wait(&s_full[st], (j >> 1) & 1);
-      tc_fence_after();
-      uint32_t sr[4][32];
-#pragma unroll
-      for (int c = 0; c < 4; ++c) tmem_ld32(tmem + lane_base + st * 128 + c * 32, sr[c]);
-      tmem_ld_wait();
-      tc_fence_before();
-      mbar_arrive(&s_free[st]);
-      const int kbase = j * AT_BN;
-      // row max on the raw scores (scale > 0); keys >= L only exist in the last tile
-      // row max with 8 independent accumulators (a single chain would be 128 dependent FMNMX)
-      float mx[8];
-#pragma unroll
-      for (int q = 0; q < 8; ++q) mx[q] = -FLT_MAX;
-      if (kbase + AT_BN > L) {
-#pragma unroll
-        for (int c = 0; c < 4; ++c)
-#pragma unroll
-          for (int i = 0; i < 32; ++i)
-            if (kbase + c * 32 + i >= L) sr[c][i] = __float_as_uint(-INFINITY);
-      }
-#pragma unroll
-      for (int c = 0; c < 4; ++c)
-#pragma unroll
-        for (int i = 0; i < 32; ++i) mx[i & 7] = fmaxf(mx[i & 7], __uint_as_float(sr[c][i]));
-      const float mt = fmaxf(fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3])),
-                             fmaxf(fmaxf(mx[4], mx[5]), fmaxf(mx[6], mx[7]))) * scale_log2;
-      bool rescale = false;
-      float alpha = 1.f;
-      if (j == 0) {
-        m_ref = mt;
-      } else if (mt > m_ref + RESCALE_THRESHOLD) {
-        rescale = true;
-        alpha = exp2f(m_ref - mt);
-        m_ref = mt;
-      }
-      l_sum *= alpha;
-      // P = exp2(x - m_ref) -> bf16, packed in pairs
-      // P = 2^(s * scale_log2 - m_ref): one FFMA + one MUFU.EX2 per score
-      uint32_t pk[64];
-      float ls0 = 0.f, ls1 = 0.f;
-      const float neg_m = -m_ref;
-#pragma unroll
-      for (int c = 0; c < 4; ++c)
-#pragma unroll
-        for (int i = 0; i < 32; i += 2) {
-          const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
-          const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
-          ls0 += p0;
-          ls1 += p1;
-          pk[c * 16 + i / 2] = pack_bf16x2(p0, p1);
-        }
-      l_sum += ls0 + ls1;
-      if (j >= 2) mbar_wait(&pv_done[st], ((j - 2) >> 1) & 1);  // P buffer st free
-      // tcgen05.ld/st are warp-collective (.sync.aligned): rescale the whole warp's rows together
-      // (alpha = 1 for rows that did not need it).
-      if (__any_sync(0xffffffffu, rescale)) {
-        mbar_wait(&pv_done[st ^ 1], ((j - 1) >> 1) & 1);         // O holds tiles < j
-        tc_fence_after();
-#pragma unroll
-        for (int c = 0; c < D / 32; ++c) {
-          uint32_t ov[32];
-          tmem_ld32(tmem + lane_base + C::O_COL + c * 32, ov);
-          tmem_ld_wait();
-#pragma unroll
-          for (int i = 0; i < 32; ++i) ov[i] = __float_as_uint(__uint_as_float(ov[i]) * alpha);
-          tmem_st32(tmem + lane_base + C::O_COL + c * 32, ov);
-        }
-        tmem_st_wait();
-      }
-      // write P row into the K-major SW128 tile: sub-tile t (keys 64t..), atom row/8, chunk ^ (row & 7)
-      uint8_t* pbase = sm + C::OFF_P + st * C::P_BYTES + (row >> 3) * 1024 + (row & 7) * 128;
-#pragma unroll
-      for (int t = 0; t < 2; ++t)
-#pragma unroll
-        for (int ch = 0; ch < 8; ++ch) {
-          const int q = t * 32 + ch * 4;  // index into pk (pairs)
-          uint4 v = make_uint4(pk[q], pk[q + 1], pk[q + 2], pk[q + 3]);
-          *reinterpret_cast<uint4*>(pbase + t * (AT_BM * 128) + ((ch ^ (row & 7)) << 4)) = v;
-        }
-      fence_proxy_async();
-      tc_fence_before();
-      mbar_arrive(&p_full[st]);
-    }
-    // epilogue: O / l -> bf16
-    const int jl = n_tiles - 1;
-    mbar_wait(&pv_done[jl & 1], (jl >> 1) & 1);
-    tc_fence_after();
-    const float inv = 1.f / l_sum;
-    const int grow = q0 + row;
-#pragma unroll
-    for (int c = 0; c < D / 32; ++c) {
-      uint32_t ov[32];
-      tmem_ld32(tmem + lane_base + C::O_COL + c * 32, ov);
-      tmem_ld_wait();
-      if (grow < L) {
-        uint4* dst = reinterpret_cast<uint4*>(o + (long long)grow * ldo + head * D + c * 32);
-#pragma unroll
-        for (int qd = 0; qd < 4; ++qd) {
-          uint4 v;
-          v.x = pack_bf16x2(__uint_as_float(ov[qd * 8 + 0]) * inv, __uint_as_float(ov[qd * 8 + 1]) * inv);
-          v.y = pack_bf16x2(__uint_as_float(ov[qd * 8 + 2]) * inv, __uint_as_float(ov[qd * 8 + 3]) * inv);
-          v.z = pack_bf16x2(__uint_as_float(ov[qd * 8 + 4]) * inv, __uint_as_float(ov[qd * 8 + 5]) * inv);
-          v.w = pack_bf16x2(__uint_as_float(ov[qd * 8 + 6]) * inv, __uint_as_float(ov[qd * 8 + 7]) * inv);
-          dst[qd] = v;
-        }
-      }
-    }
-  }
-  tc_fence_before();
-  __syncthreads();
-  tc_fence_after();
-  if (warp == 2) tmem_dealloc<C::TMEM_COLS>(tmem);
-}
-
-// ------------------------------------------------------------------ v3: two query tiles per CTA
-// One CTA = one head x 256 queries as two 128-query tiles t = 0, 1 that share every K/V tile
-// (half the K/V traffic per query).  Two softmax warpgroups (warps 4-7: tile 0, 8-11: tile 1)
-// ping-pong with the tensor core: while WG0 turns S0_j into P0_j, the single MMA thread runs
-// PV1_{j-1} and S1_j, and vice versa.  P_j is written back into the S_t TMEM columns as bf16
-// (tcgen05.st) and consumed from TMEM by the PV MMA (A operand in TMEM), so no shared-memory P.
-// Because S_t{j+1} overwrites P_t{j} in TMEM, the MMA thread issues PV_t{j} before S_t{j+1}; the
-// in-order tcgen05 pipe makes "S_t{j} complete" imply "O_t holds tiles < j", so a rare rescale
-// of O (running max grew by > 2^8) needs no extra wait.
-// TMEM: S0 | S1 | O0 | O1 (128 + 128 + D + D fp32 columns).  Smem: Q0, Q1, 2 K/V stages.
-#ifndef TSV_FA_NST64
-#define TSV_FA_NST64 4
-#endif
-template <int D>
 struct FaCfg {
   static constexpr int NSUB = D / 64;
   static constexpr int Q_TILE = AT_BM * D * 2;
   static constexpr int KV_TILE = AT_BN * D * 2;
   // K/V ring depth: D = 128 fills shared memory with 2 stages; D = 64 has room for 4
-  static constexpr int NST = TSV_FA_NST64 > 0 && D == 64 ? TSV_FA_NST64 : 2;
+  static constexpr int NST = D == 64 ? 4 : 2;
   static constexpr int OFF_Q = 0;                        // 2 tiles
   static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // NST stages
   static constexpr int OFF_V = OFF_K + NST * KV_TILE;    // NST stages
   static constexpr int OFF_BAR = OFF_V + NST * KV_TILE;
-  static constexpr int SMEM = OFF_BAR + 256 + 1024;
+  static constexpr int SMEM = OFF_BAR + 256 + 1024;      // barriers + 1 KB alignment slack
   static constexpr int O_COL = 256;
 };
+static_assert(FaCfg<128>::SMEM <= 232448 && FaCfg<64>::SMEM <= 232448, "attention shared memory > 227 KB");
 constexpr int FA_THREADS = 384;
 
-// NPOLY of every 8 exp2 pairs are evaluated on the FMA/ALU pipes (poly_exp2_x2), the rest on MUFU.
-// SPLIT: P_t{j} is handed to the MMA thread in two halves (keys 0-63, then 64-127), each with its
-// own barrier, so PV over the first 64 keys runs on the tensor core while the softmax warps still
-// evaluate the second half's exponentials.
-// LAZY: the row max is not recomputed per tile.  P = 2^(s*scale - m_ref) is evaluated with the
-// running reference directly; the tile's row sum bounds every p in it (p <= sum), so a row whose
-// sum stays <= 2^LAZY_LOG2 has no p > 2^LAZY_LOG2 and needs no rescale (m_ref is only a
-// stabiliser: softmax is exact for any reference that keeps p finite).  Otherwise (the max grew
-// a lot: early tiles) the warp reloads S from TMEM and takes the exact path (row max, rescale).
-// Saves the 128 FMNMX per row per tile and the max-before-exp dependency on the softmax chain.
-constexpr float LAZY_LIMIT = 65536.0f;   // 2^16
 // KV split (blockIdx.z = split): see AttnSplitWs.  nsplit = 1: the whole key range, no workspace.
 struct AttnSplitArgs {
   int nsplit = 1, tps = 0;   // splits, key tiles per split
@@ -375,7 +120,7 @@ struct AttnSplitArgs {
   float* ws = nullptr;
 };
 
-template <int D, int NPOLY, bool SPLIT, bool LAZY = false>
+template <int D, int NPOLY>
 __global__ void __launch_bounds__(FA_THREADS, 1)
     attention_fa_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
@@ -390,10 +135,9 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   uint64_t* kv_full = bars + 1;              // [NST stages]
   uint64_t* kv_empty = bars + 1 + NST;       // [NST stages]
   uint64_t* s_full = bars + 1 + 2 * NST;     // [2 q-tiles]
-  uint64_t* p_full = bars + 3 + 2 * NST;     // [2 q-tiles]  (SPLIT: first half of P)
+  uint64_t* p_full = bars + 3 + 2 * NST;     // [2 q-tiles]
   uint64_t* o_done = bars + 5 + 2 * NST;     // [2 q-tiles]
-  uint64_t* p_full2 = bars + 7 + 2 * NST;    // [2 q-tiles]  SPLIT: second half of P
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 10 + 2 * NST);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 8 + 2 * NST);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int head = blockIdx.y;
@@ -415,7 +159,6 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     for (int i = 0; i < 2; ++i) {
       mbar_init(&s_full[i], 1);
       mbar_init(&p_full[i], 128);
-      mbar_init(&p_full2[i], 128);
       mbar_init(&o_done[i], 1);
     }
     fence_mbar_init();
@@ -480,14 +223,9 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       tc_fence_after();
       if (elect_one()) {
 #pragma unroll
-        for (int kk = 0; kk < AT_BN / 16; ++kk) {
-          if (SPLIT && kk == AT_BN / 32) {
-            mbar_wait(&p_full2[t], j & 1);
-            tc_fence_after();
-          }
+        for (int kk = 0; kk < AT_BN / 16; ++kk)
           umma_bf16_ts(tmem + C::O_COL + t * D, tmem + t * 128 + kk * 8, dv + (uint64_t)(kk * (2048 >> 4)), idesc_o,
                        (j | kk) != 0);
-        }
         if (release) umma_commit(&kv_empty[j % NST]);
       }
       __syncwarp();
@@ -516,23 +254,22 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     const uint32_t s_col = tmem + lane_base + t * 128;
     const uint32_t o_col = tmem + lane_base + C::O_COL + t * D;
     float m_ref = -FLT_MAX, l_sum = 0.f;
+    auto hand_over = [&]() {   // P_t(j) is in TMEM: release it to the MMA warp
+      tmem_st_wait();
+      tc_fence_before();
+      mbar_arrive(&p_full[t]);   // (one arrival per warp after __syncwarp measured no faster)
+    };
     for (int j = 0; j < n_tiles; ++j) {
       mbar_wait(&s_full[t], j & 1);
       tc_fence_after();
       uint32_t sr[4][32];
       const int kbase = (j0 + j) * AT_BN;
       const bool full = kbase + AT_BN <= L;
-      const bool lazy = LAZY && !SPLIT && j > 0 && full;
-      if (!lazy) {
-#pragma unroll
-        for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
-        tmem_ld_wait();
-      }
-      if (lazy) {
+      if (j > 0 && full) {
+        // lazy path: no max before the exponentials, so the TMEM loads are pipelined with the
+        // arithmetic (chunk c + 1 is in flight while chunk c is exponentiated)
         const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(-m_ref, -m_ref);
         float2 lz[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
-        // no max before the exponentials: the TMEM loads are pipelined with the arithmetic (chunk
-        // c + 1 is in flight while chunk c is exponentiated)
         tmem_ld32(s_col, sr[0]);
         tmem_ld_wait_dep(sr[0]);
 #pragma unroll
@@ -552,6 +289,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
               p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
             }
             lz[(i >> 1) & 3] = __fadd2_rn(lz[(i >> 1) & 3], p);
+            // packed P overwrites consumed S: keys [64h, 64h + 64) land in sr[h]
             sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);
           }
           if (c < 3) tmem_ld_wait_dep(sr[c + 1]);
@@ -563,17 +301,15 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
           l_sum += ts;
           tmem_st32(s_col, sr[0]);
           tmem_st32(s_col + 32, sr[1]);
-          tmem_st_wait();
-          tc_fence_before();
-          mbar_arrive(&p_full[t]);
+          hand_over();
           continue;
         }
-        // rare: reload the untouched S columns and take the exact path below
-#pragma unroll
-        for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
-        tmem_ld_wait();
       }
-      // row max with 8 independent accumulators (a single chain would be 128 dependent FMNMX)
+      // exact path (first tile, the ragged last tile, or a lazy tile whose sum overflowed): reload
+      // S, row max with 8 independent accumulators (one chain would be 128 dependent FMNMX)
+#pragma unroll
+      for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
+      tmem_ld_wait();
       float mx[8];
 #pragma unroll
       for (int q = 0; q < 8; ++q) mx[q] = -FLT_MAX;
@@ -600,66 +336,34 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         m_ref = mt;
       }
       l_sum *= alpha;
-      // P = 2^(s * scale_log2 - m_ref) as packed bf16 pairs, in place of S (columns 0..63 of S_t):
-      // keys [64h, 64h + 64) land in sr[h] and TMEM columns [32h, 32h + 32)
       const float neg_m = -m_ref;
       float2 lsum[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        if (full) {
-          // Per tile each softmax warpgroup must finish inside the ~1024-cycle window in which the
-          // tensor core works on the other query tile.  MUFU.EX2 alone needs 1024 cycles per tile
-          // (16/clk/SM), so NPOLY pairs in 8 are evaluated on the FMA/ALU pipes (Cody-Waite split +
-          // cubic, rel. error < 1e-3 << bf16 ulp of P), and the arithmetic uses paired FP32 ops.
-          const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(neg_m, neg_m);
+      for (int c = 0; c < 4; ++c)
 #pragma unroll
-          for (int c = 2 * h; c < 2 * h + 2; ++c)
-#pragma unroll
-            for (int i = 0; i < 32; i += 2) {
-              const float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])),
-                                          sc2, nm2);
-              float2 p;
-              if (((i >> 1) & 7) >= 8 - NPOLY) p = poly_exp2_x2(x);
-              else p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
-              lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], p);     // 8 independent partial sums
-              sr[h][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);        // packed P overwrites consumed S
-            }
-        } else {
-#pragma unroll
-          for (int c = 2 * h; c < 2 * h + 2; ++c)
-#pragma unroll
-            for (int i = 0; i < 32; i += 2) {
-              const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
-              const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
-              lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], make_float2(p0, p1));
-              sr[h][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);
-            }
+        for (int i = 0; i < 32; i += 2) {   // all MUFU here (masked keys give ex2(-inf) = 0)
+          const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
+          const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
+          lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], make_float2(p0, p1));
+          sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);
         }
-        if (h == 0 && __any_sync(0xffffffffu, rescale)) {
-          // S_t{j} complete => PV_t{j-1} complete (in-order pipe): O_t can be rescaled now, before any
-          // part of P_t{j} is handed over (here S columns 64-127 are consumed: registers are free)
+      if (__any_sync(0xffffffffu, rescale)) {
+        // S_t(j) complete => PV_t(j-1) complete (in-order pipe): O_t can be rescaled now, before
+        // P_t(j) is handed over.  tcgen05.ld/st are warp-collective: the whole warp's rows are
+        // rescaled together (alpha = 1 for rows that did not need it).
 #pragma unroll
-          for (int c = 0; c < D / 32; ++c) {
-            uint32_t ov[32];
-            tmem_ld32(o_col + c * 32, ov);
-            tmem_ld_wait();
+        for (int c = 0; c < D / 32; ++c) {
+          uint32_t ov[32];
+          tmem_ld32(o_col + c * 32, ov);
+          tmem_ld_wait();
 #pragma unroll
-            for (int i = 0; i < 32; ++i) ov[i] = __float_as_uint(__uint_as_float(ov[i]) * alpha);
-            tmem_st32(o_col + c * 32, ov);
-          }
-        }
-        if (SPLIT || h == 1) {
-          if (SPLIT) {
-            tmem_st32(s_col + 32 * h, sr[h]);
-          } else {
-            tmem_st32(s_col, sr[0]);
-            tmem_st32(s_col + 32, sr[1]);
-          }
-          tmem_st_wait();
-          tc_fence_before();
-          mbar_arrive(h == 0 ? &p_full[t] : (SPLIT ? &p_full2[t] : &p_full[t]));
+          for (int i = 0; i < 32; ++i) ov[i] = __float_as_uint(__uint_as_float(ov[i]) * alpha);
+          tmem_st32(o_col + c * 32, ov);
         }
       }
+      tmem_st32(s_col, sr[0]);
+      tmem_st32(s_col + 32, sr[1]);
+      hand_over();
       const float2 l01 = __fadd2_rn(lsum[0], lsum[1]), l23 = __fadd2_rn(lsum[2], lsum[3]);
       const float2 l4 = __fadd2_rn(l01, l23);
       l_sum += l4.x + l4.y;
@@ -783,603 +487,6 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   if (warp == 2) tmem_dealloc<512>(tmem);
 }
 
-// ------------------------------------------------------------------ v5: 64-key tiles, S double-buffered
-// v3's chain S_t(j) -> softmax -> PV_t(j) -> S_t(j+1) serialises the softmax with the tensor core
-// (P_t(j) aliases the only S_t buffer).  v5 uses 64-key K/V tiles so that each query tile owns two
-// 64-column S buffers (TMEM: S_t,b at 128 t + 64 b, O_t at 256 + D t; 512 columns for D = 128):
-// the MMA thread issues S_t(j+1) into the other buffer BEFORE PV_t(j), so the tensor core computes
-// the next scores while the softmax warps exponentiate the current ones.  Per iteration the MMA
-// thread issues PV_0(j), S_0(j+2), PV_1(j), S_1(j+2): S_t(j+2) reuses buffer j & 1 right behind
-// PV_t(j) in the same in-order tcgen05 pipe, so each softmax warpgroup has two tiles of look-ahead.  Because S_t(j) no longer implies "PV_t(j-1) complete", a rare
-// O rescale first waits on pv_done[t] (committed after every PV_t).
-template <int D>
-struct Fa5Cfg {
-  static constexpr int BN = 64;                          // keys per K/V tile
-  static constexpr int NSUB = D / 64;
-  static constexpr int Q_TILE = AT_BM * D * 2;
-  static constexpr int KV_TILE = BN * D * 2;             // one K (or V) tile
-  static constexpr int NST = D == 128 ? 4 : 6;           // K/V stages
-  static constexpr int OFF_Q = 0;                        // 2 tiles
-  static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;
-  static constexpr int OFF_V = OFF_K + NST * KV_TILE;
-  static constexpr int OFF_BAR = OFF_V + NST * KV_TILE;
-  static constexpr int SMEM = OFF_BAR + 256 + 1024;
-  static constexpr int O_COL = 256;
-};
-
-template <int D, int NPOLY>
-__global__ void __launch_bounds__(FA_THREADS, 1)
-    attention_fa5_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
-                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
-                         float scale_log2, const __grid_constant__ AttnScatter sc) {
-  using C = Fa5Cfg<D>;
-  constexpr int BN = C::BN, NST = C::NST;
-  extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
-  uint64_t* q_full = bars + 0;
-  uint64_t* kv_full = bars + 1;            // [NST]
-  uint64_t* kv_empty = bars + 1 + NST;     // [NST]
-  uint64_t* s_full = bars + 1 + 2 * NST;   // [2 t][2 buffers]
-  uint64_t* p_full = bars + 5 + 2 * NST;   // [2 t][2 buffers]
-  uint64_t* pv_done = bars + 9 + 2 * NST;  // [2 t], every PV_t
-  uint64_t* o_done = bars + 11 + 2 * NST;  // [2 t], the last PV_t
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 14 + 2 * NST);
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int head = blockIdx.y;
-  const int q0 = blockIdx.x * 2 * AT_BM;
-  const int n_tiles = (L + BN - 1) / BN;
-
-  if (warp == 0 && lane == 0) {
-    tma_prefetch_desc(&tmQ);
-    tma_prefetch_desc(&tmK);
-    tma_prefetch_desc(&tmV);
-    mbar_init(q_full, 1);
-    for (int i = 0; i < NST; ++i) {
-      mbar_init(&kv_full[i], 1);
-      mbar_init(&kv_empty[i], 1);
-    }
-    for (int i = 0; i < 4; ++i) {
-      mbar_init(&s_full[i], 1);
-      mbar_init(&p_full[i], 128);
-    }
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(&pv_done[i], 1);
-      mbar_init(&o_done[i], 1);
-    }
-    fence_mbar_init();
-  }
-  if (warp == 2) tmem_alloc<512>(tmem_slot);
-  tc_fence_before();
-  __syncthreads();
-  tc_fence_after();
-  const uint32_t tmem = *tmem_slot;
-  grid_dep_wait();
-  if (warp < 4) {
-    regs_dec<80>();
-    if (warp == 0) {
-      if (lane == 0) {
-        // -------------------------------------------------------------- producer
-        mbar_arrive_expect_tx(q_full, 2 * C::Q_TILE);
-        for (int t = 0; t < 2; ++t)
-          for (int s = 0; s < C::NSUB; ++s)
-            tma_load_3d(&tmQ, q_full, sm + C::OFF_Q + t * C::Q_TILE + s * (AT_BM * 128), s * 64, head,
-                        q0 + t * AT_BM);
-        for (int j = 0; j < n_tiles; ++j) {
-          const int st = j % NST;
-          if (j >= NST) mbar_wait(&kv_empty[st], ((j / NST) - 1) & 1);
-          mbar_arrive_expect_tx(&kv_full[st], 2 * C::KV_TILE);
-          for (int s = 0; s < C::NSUB; ++s) {
-            tma_load_3d(&tmK, &kv_full[st], sm + C::OFF_K + st * C::KV_TILE + s * (BN * 128), s * 64, head, j * BN);
-            tma_load_3d(&tmV, &kv_full[st], sm + C::OFF_V + st * C::KV_TILE + s * (BN * 128), s * 64, head, j * BN);
-          }
-        }
-      }
-    } else if (warp == 1) {
-      // -------------------------------------------------------------- MMA issuer (whole warp,
-      // one elected lane per MMA batch; descriptors = bases + compile-time offsets, see v3)
-      constexpr uint32_t idesc_s = make_idesc_bf16(AT_BM, BN);
-      constexpr uint32_t idesc_o = make_idesc_bf16_bmn(AT_BM, D);
-      const uint64_t dq0 = make_sw128_desc(smem_u32(sm + C::OFF_Q));
-      const uint64_t dk0 = make_sw128_desc(smem_u32(sm + C::OFF_K));
-      const uint64_t dv0 = make_sw128_mn_desc(smem_u32(sm + C::OFF_V), BN * 128);
-      mbar_wait(q_full, 0);
-      auto issue_s = [&](int t, int j) {   // S_t(j) into buffer j & 1 (K tile already resident)
-        const uint64_t dq = dq0 + (uint64_t)((t * C::Q_TILE) >> 4);
-        const uint64_t dk = dk0 + (uint64_t)(((j % NST) * C::KV_TILE) >> 4);
-        if (elect_one()) {
-#pragma unroll
-          for (int kk = 0; kk < D / 16; ++kk) {
-            const uint32_t offq = ((kk >> 2) * (AT_BM * 128) + (kk & 3) * 32) >> 4;
-            const uint32_t offk = ((kk >> 2) * (BN * 128) + (kk & 3) * 32) >> 4;
-            umma_bf16_ss(tmem + t * 128 + (j & 1) * 64, dq + offq, dk + offk, idesc_s, kk > 0);
-          }
-          umma_commit(&s_full[t * 2 + (j & 1)]);
-        }
-        __syncwarp();
-      };
-      auto issue_pv = [&](int t, int j) {  // O_t += P_t(j) V(j); P_t(j) in TMEM buffer j & 1
-        const uint64_t dv = dv0 + (uint64_t)(((j % NST) * C::KV_TILE) >> 4);
-        mbar_wait(&p_full[t * 2 + (j & 1)], (j >> 1) & 1);
-        tc_fence_after();
-        if (elect_one()) {
-#pragma unroll
-          for (int kk = 0; kk < BN / 16; ++kk)
-            umma_bf16_ts(tmem + C::O_COL + t * D, tmem + t * 128 + (j & 1) * 64 + kk * 8,
-                         dv + (uint64_t)(kk * (2048 >> 4)), idesc_o, (j | kk) != 0);
-          umma_commit(&pv_done[t]);
-          if (j == n_tiles - 1) umma_commit(&o_done[t]);
-        }
-        __syncwarp();
-      };
-      // two tiles of look-ahead per query tile: S_t(j+2) (into buffer j & 1) right behind PV_t(j)
-      for (int j = 0; j < 2 && j < n_tiles; ++j) {
-        mbar_wait(&kv_full[j], 0);
-        tc_fence_after();
-        issue_s(0, j);
-        issue_s(1, j);
-      }
-      for (int j = 0; j < n_tiles; ++j) {
-        const bool ahead = j + 2 < n_tiles;
-        for (int t = 0; t < 2; ++t) {
-          issue_pv(t, j);
-          if (ahead) {
-            if (t == 0) {
-              mbar_wait(&kv_full[(j + 2) % NST], ((j + 2) / NST) & 1);
-              tc_fence_after();
-            }
-            issue_s(t, j + 2);
-          }
-        }
-        if (elect_one()) umma_commit(&kv_empty[j % NST]);
-        __syncwarp();
-      }
-    }
-  } else {
-    regs_inc<208>();
-    // ---------------------------------------------------------------- softmax WG t (thread = query row)
-    const int t = (warp - 4) >> 2;
-    const int wq = (warp - 4) & 3;
-    const int row = wq * 32 + lane;
-    const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
-    const uint32_t o_col = tmem + lane_base + C::O_COL + t * D;
-    float m_ref = -FLT_MAX, l_sum = 0.f;
-    for (int j = 0; j < n_tiles; ++j) {
-      const uint32_t s_col = tmem + lane_base + t * 128 + (j & 1) * 64;
-      mbar_wait(&s_full[t * 2 + (j & 1)], (j >> 1) & 1);
-      tc_fence_after();
-      uint32_t sr[2][32];
-      tmem_ld32(s_col, sr[0]);
-      tmem_ld32(s_col + 32, sr[1]);
-      tmem_ld_wait();
-      const int kbase = j * BN;
-      const bool full = kbase + BN <= L;
-      if (!full) {
-#pragma unroll
-        for (int c = 0; c < 2; ++c)
-#pragma unroll
-          for (int i = 0; i < 32; ++i)
-            if (kbase + c * 32 + i >= L) sr[c][i] = __float_as_uint(-INFINITY);
-      }
-      float mx[8];
-#pragma unroll
-      for (int q = 0; q < 8; ++q) mx[q] = -FLT_MAX;
-#pragma unroll
-      for (int c = 0; c < 2; ++c)
-#pragma unroll
-        for (int i = 0; i < 32; ++i) mx[i & 7] = fmaxf(mx[i & 7], __uint_as_float(sr[c][i]));
-      const float mt = fmaxf(fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3])),
-                             fmaxf(fmaxf(mx[4], mx[5]), fmaxf(mx[6], mx[7]))) * scale_log2;
-      bool rescale = false;
-      float alpha = 1.f;
-      if (j == 0) {
-        m_ref = mt;
-      } else if (mt > m_ref + RESCALE_THRESHOLD) {
-        rescale = true;
-        alpha = exp2f(m_ref - mt);
-        m_ref = mt;
-      }
-      l_sum *= alpha;
-      const float neg_m = -m_ref;
-      float2 lsum[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
-      if (full) {
-        const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(neg_m, neg_m);
-#pragma unroll
-        for (int c = 0; c < 2; ++c)
-#pragma unroll
-          for (int i = 0; i < 32; i += 2) {
-            const float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2,
-                                        nm2);
-            float2 p;
-            if (((i >> 1) & 7) >= 8 - NPOLY) p = poly_exp2_x2(x);
-            else p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
-            lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], p);
-            sr[0][c * 16 + i / 2] = pack_bf16x2(p.x, p.y);      // packed P overwrites consumed S
-          }
-      } else {
-#pragma unroll
-        for (int c = 0; c < 2; ++c)
-#pragma unroll
-          for (int i = 0; i < 32; i += 2) {
-            const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
-            const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
-            lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], make_float2(p0, p1));
-            sr[0][c * 16 + i / 2] = pack_bf16x2(p0, p1);
-          }
-      }
-      if (__any_sync(0xffffffffu, rescale)) {
-        // O_t must hold exactly tiles < j: wait for PV_t(j-1) (S_t(j) was issued before it)
-        mbar_wait(&pv_done[t], (j - 1) & 1);
-        tc_fence_after();
-#pragma unroll
-        for (int c = 0; c < D / 32; ++c) {
-          uint32_t ov[32];
-          tmem_ld32(o_col + c * 32, ov);
-          tmem_ld_wait();
-#pragma unroll
-          for (int i = 0; i < 32; ++i) ov[i] = __float_as_uint(__uint_as_float(ov[i]) * alpha);
-          tmem_st32(o_col + c * 32, ov);
-        }
-      }
-      tmem_st32(s_col, sr[0]);
-      tmem_st_wait();
-      tc_fence_before();
-      mbar_arrive(&p_full[t * 2 + (j & 1)]);
-      const float2 l01 = __fadd2_rn(lsum[0], lsum[1]), l23 = __fadd2_rn(lsum[2], lsum[3]);
-      const float2 l4 = __fadd2_rn(l01, l23);
-      l_sum += l4.x + l4.y;
-    }
-    // epilogue: O_t / l -> bf16 once the last PV_t is complete (pv_done may be two phases behind
-    // here: S_t(n-1) complete only implies PV_t(n-3) complete)
-    mbar_wait(&o_done[t], 0);
-    tc_fence_after();
-    const float inv = 1.f / l_sum;
-    const int grow = q0 + t * AT_BM + row;
-    bf16* orow = o + (long long)grow * ldo + head * D;
-    if (sc.k > 0 && grow < L) {
-      int p = 0, lr;
-      if (grow < sc.Lt) {
-        while (p + 1 < sc.k && grow >= sc.t_off[p + 1]) ++p;
-        lr = grow - sc.t_off[p];
-      } else {
-        const int gi = grow - sc.Lt;
-        while (p + 1 < sc.k && gi >= sc.i_off[p + 1]) ++p;
-        lr = sc.nt[p] + gi - sc.i_off[p];
-      }
-      orow = sc.dst[p] + (long long)lr * sc.ld + sc.col0 + head * D;
-    }
-#pragma unroll
-    for (int c = 0; c < D / 32; ++c) {
-      uint32_t ov[32];
-      tmem_ld32(o_col + c * 32, ov);
-      tmem_ld_wait();
-      if (grow < L) {
-        uint4* dst = reinterpret_cast<uint4*>(orow + c * 32);
-#pragma unroll
-        for (int qd = 0; qd < 4; ++qd) {
-          uint4 v;
-          v.x = pack_bf16x2(__uint_as_float(ov[qd * 8 + 0]) * inv, __uint_as_float(ov[qd * 8 + 1]) * inv);
-          v.y = pack_bf16x2(__uint_as_float(ov[qd * 8 + 2]) * inv, __uint_as_float(ov[qd * 8 + 3]) * inv);
-          v.z = pack_bf16x2(__uint_as_float(ov[qd * 8 + 4]) * inv, __uint_as_float(ov[qd * 8 + 5]) * inv);
-          v.w = pack_bf16x2(__uint_as_float(ov[qd * 8 + 6]) * inv, __uint_as_float(ov[qd * 8 + 7]) * inv);
-          dst[qd] = v;
-        }
-      }
-    }
-  }
-  grid_dep_launch();
-  tc_fence_before();
-  __syncthreads();
-  tc_fence_after();
-  if (warp == 2) tmem_dealloc<512>(tmem);
-}
-
-// ------------------------------------------------------------------ v6: CTA pair (cta_group::2)
-// A cluster of 2 CTAs computes 512 queries of one head as two pair tiles t = 0, 1 of 256 queries:
-// CTA r holds rows [256 t + 128 r, +128) of pair tile t (its Q tiles, its S/P/O rows in its TMEM).
-// The even CTA issues tcgen05.mma.cta_group::2 with M = 256: S_t = Q_t K^T (N = 128 keys, each CTA
-// holds 64 of the keys) and O_t += P_t V (N = D, each CTA holds D/2 columns of V).  Per SM the
-// S MMA reads 96 B/clk of shared memory instead of 128 (the 1-CTA kernel's S MMA sits at the
-// shared-memory port limit, like a 128x128 GEMM tile) and K/V tiles cost half the TMA bytes.
-// Softmax: v3's lazy-max body per CTA; P hand-over is one arrive per softmax warp on the even
-// CTA's barrier (8 warps per pair tile).
-template <int D>
-struct Fa2Cfg {
-  static constexpr int NSUB = D / 64;
-  static constexpr int Q_TILE = AT_BM * D * 2;          // 128 rows
-  static constexpr int K_HALF = (AT_BN / 2) * D * 2;    // 64 keys x D
-  static constexpr int V_HALF = AT_BN * (D / 2) * 2;    // 128 keys x D/2 (one 128-byte swizzle column)
-  static constexpr int STAGE = K_HALF + V_HALF;
-  static constexpr int NST = 4;
-  static constexpr int OFF_Q = 0;                        // 2 tiles
-  static constexpr int OFF_KV = OFF_Q + 2 * Q_TILE;      // NST stages of [K half | V half]
-  static constexpr int OFF_BAR = OFF_KV + NST * STAGE;
-  static constexpr int SMEM = OFF_BAR + 256 + 1024;
-  static constexpr int O_COL = 256;
-};
-static_assert(Fa2Cfg<128>::SMEM <= 227 * 1024, "pair attention smem");
-
-template <int D, int NPOLY>
-__global__ void __launch_bounds__(FA_THREADS, 1)
-    attention_fa2_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
-                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
-                         float scale_log2, const __grid_constant__ AttnScatter sc) {
-  static_assert(D == 128, "pair kernel: D = 128 (V halves are one 64-column swizzle block)");
-  using C = Fa2Cfg<D>;
-  constexpr int NST = C::NST;
-  extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
-  uint64_t* q_full = bars + 0;             // even CTA: both CTAs' Q bytes
-  uint64_t* kv_full = bars + 1;            // [NST] even CTA: both halves
-  uint64_t* kv_empty = bars + 1 + NST;     // [NST] both CTAs (multicast commit)
-  uint64_t* s_full = bars + 1 + 2 * NST;   // [2 t] both CTAs (multicast commit)
-  uint64_t* p_full = bars + 3 + 2 * NST;   // [2 t] even CTA: 8 softmax warps
-  uint64_t* o_done = bars + 5 + 2 * NST;   // [2 t] both CTAs
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 8 + 2 * NST);
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const uint32_t rank = cluster_ctarank();
-  const bool leader = rank == 0;
-  const int head = blockIdx.y;
-  const int qc = (blockIdx.x >> 1) * 4 * AT_BM;   // the pair's first query
-  const int n_tiles = (L + AT_BN - 1) / AT_BN;
-
-  if (warp == 0 && lane == 0) {
-    tma_prefetch_desc(&tmQ);
-    tma_prefetch_desc(&tmK);
-    tma_prefetch_desc(&tmV);
-    mbar_init(q_full, 1);
-    for (int i = 0; i < NST; ++i) {
-      mbar_init(&kv_full[i], 1);
-      mbar_init(&kv_empty[i], 1);
-    }
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(&s_full[i], 1);
-      mbar_init(&p_full[i], 8);
-      mbar_init(&o_done[i], 1);
-    }
-    fence_mbar_init();
-  }
-  if (warp == 2) tmem_alloc_pair<512>(tmem_slot);
-  tc_fence_before();
-  cluster_sync();
-  tc_fence_after();
-  const uint32_t tmem = *tmem_slot;
-  grid_dep_wait();
-  if (warp < 4) {
-    regs_dec<80>();
-    if (warp == 0) {
-      if (lane == 0) {
-        // -------------------------------------------------------------- producer (both CTAs)
-        if (leader) mbar_arrive_expect_tx(q_full, 2 * 2 * C::Q_TILE);
-        for (int t = 0; t < 2; ++t)
-          for (int s = 0; s < C::NSUB; ++s)
-            tma_load_3d_pair(&tmQ, q_full, sm + C::OFF_Q + t * C::Q_TILE + s * (AT_BM * 128), s * 64, head,
-                             qc + t * 2 * AT_BM + (int)rank * AT_BM);
-        for (int j = 0; j < n_tiles; ++j) {
-          const int st = j % NST;
-          if (j >= NST) mbar_wait(&kv_empty[st], ((j / NST) - 1) & 1);
-          if (leader) mbar_arrive_expect_tx(&kv_full[st], 2 * C::STAGE);
-          uint8_t* sk = sm + C::OFF_KV + st * C::STAGE;
-          for (int s = 0; s < C::NSUB; ++s)   // keys [128 j + 64 r, +64), all D
-            tma_load_3d_pair(&tmK, &kv_full[st], sk + s * ((AT_BN / 2) * 128), s * 64, head,
-                             j * AT_BN + (int)rank * (AT_BN / 2));
-          // keys [128 j, +128), columns [64 r, +64)
-          tma_load_3d_pair(&tmV, &kv_full[st], sk + C::K_HALF, (int)rank * 64, head, j * AT_BN);
-        }
-      }
-    } else if (warp == 1 && leader) {
-      // -------------------------------------------------------------- MMA issuer (even CTA, whole warp)
-      constexpr uint32_t idesc_s = make_idesc_bf16(2 * AT_BM, AT_BN);
-      constexpr uint32_t idesc_o = make_idesc_bf16_bmn(2 * AT_BM, D);
-      const uint64_t dq0 = make_sw128_desc(smem_u32(sm + C::OFF_Q));
-      const uint64_t dk0 = make_sw128_desc(smem_u32(sm + C::OFF_KV));
-      const uint64_t dv0 = make_sw128_mn_desc(smem_u32(sm + C::OFF_KV + C::K_HALF), AT_BN * 128);
-      mbar_wait(q_full, 0);
-      auto issue_s = [&](int t, int j) {
-        const uint64_t dq = dq0 + (uint64_t)((t * C::Q_TILE) >> 4);
-        const uint64_t dk = dk0 + (uint64_t)(((j % NST) * C::STAGE) >> 4);
-        if (elect_one()) {
-#pragma unroll
-          for (int kk = 0; kk < D / 16; ++kk) {
-            const uint32_t offq = ((kk >> 2) * (AT_BM * 128) + (kk & 3) * 32) >> 4;
-            const uint32_t offk = ((kk >> 2) * ((AT_BN / 2) * 128) + (kk & 3) * 32) >> 4;
-            umma_bf16_ss_pair(tmem + t * 128, dq + offq, dk + offk, idesc_s, kk > 0);
-          }
-          umma_commit_pair(&s_full[t]);
-        }
-        __syncwarp();
-      };
-      auto issue_pv = [&](int t, int j, bool release) {
-        const uint64_t dv = dv0 + (uint64_t)(((j % NST) * C::STAGE) >> 4);
-        mbar_wait(&p_full[t], j & 1);
-        tc_fence_after();
-        if (elect_one()) {
-#pragma unroll
-          for (int kk = 0; kk < AT_BN / 16; ++kk)
-            umma_bf16_ts_pair(tmem + C::O_COL + t * D, tmem + t * 128 + kk * 8, dv + (uint64_t)(kk * (2048 >> 4)),
-                              idesc_o, (j | kk) != 0);
-          if (release) umma_commit_pair(&kv_empty[j % NST]);
-        }
-        __syncwarp();
-      };
-      for (int j = 0; j < n_tiles; ++j) {
-        mbar_wait(&kv_full[j % NST], (j / NST) & 1);
-        tc_fence_after();
-        for (int t = 0; t < 2; ++t) {
-          if (j > 0) issue_pv(t, j - 1, t == 1);
-          issue_s(t, j);
-        }
-      }
-      for (int t = 0; t < 2; ++t) {
-        issue_pv(t, n_tiles - 1, false);
-        if (elect_one()) umma_commit_pair(&o_done[t]);
-        __syncwarp();
-      }
-    }
-  } else {
-    regs_inc<208>();
-    // ---------------------------------------------------------------- softmax WG t (thread = query row)
-    const int t = (warp - 4) >> 2;
-    const int wq = (warp - 4) & 3;
-    const int row = wq * 32 + lane;
-    const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
-    const uint32_t s_col = tmem + lane_base + t * 128;
-    const uint32_t o_col = tmem + lane_base + C::O_COL + t * D;
-    float m_ref = -FLT_MAX, l_sum = 0.f;
-    auto hand_over = [&]() {   // P_t(j) stored: one arrive per warp on the even CTA's barrier
-      tmem_st_wait();
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive_remote(&p_full[t], 0);
-    };
-    for (int j = 0; j < n_tiles; ++j) {
-      mbar_wait(&s_full[t], j & 1);
-      tc_fence_after();
-      uint32_t sr[4][32];
-#pragma unroll
-      for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
-      tmem_ld_wait();
-      const int kbase = j * AT_BN;
-      const bool full = kbase + AT_BN <= L;
-      if (j > 0 && full) {
-        // lazy max (see attention_fa_kernel): P with the running reference, exact path if any row's
-        // tile sum exceeds the bound
-        const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(-m_ref, -m_ref);
-        float2 lz[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
-#pragma unroll
-        for (int c = 0; c < 4; ++c)
-#pragma unroll
-          for (int i = 0; i < 32; i += 2) {
-            float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2, nm2);
-            float2 p;
-            if (((i >> 1) & 7) >= 8 - NPOLY) {
-              x.x = fminf(x.x, 64.f);
-              x.y = fminf(x.y, 64.f);
-              p = poly_exp2_x2(x);
-            } else {
-              p = make_float2(fast_exp2(x.x), fast_exp2(x.y));
-            }
-            lz[(i >> 1) & 3] = __fadd2_rn(lz[(i >> 1) & 3], p);
-            sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);
-          }
-        const float2 l01 = __fadd2_rn(lz[0], lz[1]), l23 = __fadd2_rn(lz[2], lz[3]);
-        const float2 l4 = __fadd2_rn(l01, l23);
-        const float ts = l4.x + l4.y;
-        if (!__any_sync(0xffffffffu, !(ts <= LAZY_LIMIT))) {
-          l_sum += ts;
-          tmem_st32(s_col, sr[0]);
-          tmem_st32(s_col + 32, sr[1]);
-          hand_over();
-          continue;
-        }
-#pragma unroll
-        for (int c = 0; c < 4; ++c) tmem_ld32(s_col + c * 32, sr[c]);
-        tmem_ld_wait();
-      }
-      // exact path: first tile, the masked last tile, and lazy overflows
-      float mx[8];
-#pragma unroll
-      for (int q = 0; q < 8; ++q) mx[q] = -FLT_MAX;
-      if (!full) {
-#pragma unroll
-        for (int c = 0; c < 4; ++c)
-#pragma unroll
-          for (int i = 0; i < 32; ++i)
-            if (kbase + c * 32 + i >= L) sr[c][i] = __float_as_uint(-INFINITY);
-      }
-#pragma unroll
-      for (int c = 0; c < 4; ++c)
-#pragma unroll
-        for (int i = 0; i < 32; ++i) mx[i & 7] = fmaxf(mx[i & 7], __uint_as_float(sr[c][i]));
-      const float mt = fmaxf(fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3])),
-                             fmaxf(fmaxf(mx[4], mx[5]), fmaxf(mx[6], mx[7]))) * scale_log2;
-      bool rescale = false;
-      float alpha = 1.f;
-      if (j == 0) {
-        m_ref = mt;
-      } else if (mt > m_ref + RESCALE_THRESHOLD) {
-        rescale = true;
-        alpha = exp2f(m_ref - mt);
-        m_ref = mt;
-      }
-      l_sum *= alpha;
-      const float neg_m = -m_ref;
-      float2 lsum[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
-#pragma unroll
-      for (int c = 0; c < 4; ++c)
-#pragma unroll
-        for (int i = 0; i < 32; i += 2) {
-          const float p0 = fast_exp2(fmaf(__uint_as_float(sr[c][i]), scale_log2, neg_m));
-          const float p1 = fast_exp2(fmaf(__uint_as_float(sr[c][i + 1]), scale_log2, neg_m));
-          lsum[(i >> 1) & 3] = __fadd2_rn(lsum[(i >> 1) & 3], make_float2(p0, p1));
-          sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p0, p1);
-        }
-      if (__any_sync(0xffffffffu, rescale)) {
-        // S_t(j) complete => PV_t(j-1) complete (in-order pipe of the pair): O_t holds tiles < j
-#pragma unroll
-        for (int c = 0; c < D / 32; ++c) {
-          uint32_t ov[32];
-          tmem_ld32(o_col + c * 32, ov);
-          tmem_ld_wait();
-#pragma unroll
-          for (int i = 0; i < 32; ++i) ov[i] = __float_as_uint(__uint_as_float(ov[i]) * alpha);
-          tmem_st32(o_col + c * 32, ov);
-        }
-      }
-      tmem_st32(s_col, sr[0]);
-      tmem_st32(s_col + 32, sr[1]);
-      hand_over();
-      const float2 l01 = __fadd2_rn(lsum[0], lsum[1]), l23 = __fadd2_rn(lsum[2], lsum[3]);
-      const float2 l4 = __fadd2_rn(l01, l23);
-      l_sum += l4.x + l4.y;
-    }
-    // epilogue: O_t / l -> bf16
-    mbar_wait(&o_done[t], 0);
-    tc_fence_after();
-    const float inv = 1.f / l_sum;
-    const int grow = qc + t * 2 * AT_BM + (int)rank * AT_BM + row;
-    bf16* orow = o + (long long)grow * ldo + head * D;
-    if (sc.k > 0 && grow < L) {
-      int p = 0, lr;
-      if (grow < sc.Lt) {
-        while (p + 1 < sc.k && grow >= sc.t_off[p + 1]) ++p;
-        lr = grow - sc.t_off[p];
-      } else {
-        const int gi = grow - sc.Lt;
-        while (p + 1 < sc.k && gi >= sc.i_off[p + 1]) ++p;
-        lr = sc.nt[p] + gi - sc.i_off[p];
-      }
-      orow = sc.dst[p] + (long long)lr * sc.ld + sc.col0 + head * D;
-    }
-#pragma unroll
-    for (int c = 0; c < D / 32; ++c) {
-      uint32_t ov[32];
-      tmem_ld32(o_col + c * 32, ov);
-      tmem_ld_wait();
-      if (grow < L) {
-        uint4* dst = reinterpret_cast<uint4*>(orow + c * 32);
-#pragma unroll
-        for (int qd = 0; qd < 4; ++qd) {
-          uint4 v;
-          v.x = pack_bf16x2(__uint_as_float(ov[qd * 8 + 0]) * inv, __uint_as_float(ov[qd * 8 + 1]) * inv);
-          v.y = pack_bf16x2(__uint_as_float(ov[qd * 8 + 2]) * inv, __uint_as_float(ov[qd * 8 + 3]) * inv);
-          v.z = pack_bf16x2(__uint_as_float(ov[qd * 8 + 4]) * inv, __uint_as_float(ov[qd * 8 + 5]) * inv);
-          v.w = pack_bf16x2(__uint_as_float(ov[qd * 8 + 6]) * inv, __uint_as_float(ov[qd * 8 + 7]) * inv);
-          dst[qd] = v;
-        }
-      }
-    }
-  }
-  grid_dep_launch();
-  tc_fence_before();
-  cluster_sync();
-  tc_fence_after();
-  if (warp == 2) tmem_dealloc_pair<512>(tmem);
-}
-
 // ------------------------------------------------------------------ host
 static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -1407,68 +514,22 @@ static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L
   return r == CUDA_SUCCESS ? 0 : -2;
 }
 
-// default share of exp2 evaluated by polynomial, per head dim (tools/microbench.py sweep)
-template <int D>
-constexpr int default_npoly() { return D == 64 ? 2 : 1; }   // measured (profiles/README.md)
-
-template <int D, int NP, bool SPLIT = false, bool LAZY = false>
-static void launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
-                      int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s,
-                      const AttnSplitArgs& sa = AttnSplitArgs()) {
+template <int D, int NP>
+static cudaError_t launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o,
+                             long long ldo, int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s,
+                             const AttnSplitArgs& sa) {
   static unsigned long long done = 0;
   int dev = 0;
   cudaGetDevice(&dev);
   if (!(done >> dev & 1ull)) {
-    cudaFuncSetAttribute(attention_fa_kernel<D, NP, SPLIT, LAZY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         FaCfg<D>::SMEM);
+    cudaError_t e = cudaFuncSetAttribute(attention_fa_kernel<D, NP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         FaCfg<D>::SMEM);
+    if (e != cudaSuccess) return e;
     done |= 1ull << dev;
   }
   dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H, sa.nsplit);
-  launch_pdl(attention_fa_kernel<D, NP, SPLIT, LAZY>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo, L, scale_log2,
-             sc, sa);
-}
-
-template <int D, int NP>
-static void launch_fa5(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
-                       int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s) {
-  static unsigned long long done = 0;
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (!(done >> dev & 1ull)) {
-    cudaFuncSetAttribute(attention_fa5_kernel<D, NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, Fa5Cfg<D>::SMEM);
-    done |= 1ull << dev;
-  }
-  dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H);
-  launch_pdl(attention_fa5_kernel<D, NP>, grid, dim3(FA_THREADS), Fa5Cfg<D>::SMEM, s, tq, tk, tv, o, ldo, L,
-             scale_log2, sc);
-}
-
-template <int NP>
-static void launch_fa2(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o, long long ldo,
-                       int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s) {
-  static unsigned long long done = 0;
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (!(done >> dev & 1ull)) {
-    cudaFuncSetAttribute(attention_fa2_kernel<128, NP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         Fa2Cfg<128>::SMEM);
-    done |= 1ull << dev;
-  }
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(2 * ((L + 4 * AT_BM - 1) / (4 * AT_BM)), H);
-  cfg.blockDim = dim3(FA_THREADS);
-  cfg.dynamicSmemBytes = Fa2Cfg<128>::SMEM;
-  cfg.stream = s;
-  cudaLaunchAttribute attr[2];
-  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr[0].val.programmaticStreamSerializationAllowed = 1;
-  attr[1].id = cudaLaunchAttributeClusterDimension;
-  attr[1].val.clusterDim.x = 2;
-  attr[1].val.clusterDim.y = 1;
-  attr[1].val.clusterDim.z = 1;
-  cfg.attrs = attr;
-  cfg.numAttrs = 2;
-  cudaLaunchKernelEx(&cfg, attention_fa2_kernel<128, NP>, tq, tk, tv, o, ldo, L, scale_log2, sc);
+  return launch_pdl(attention_fa_kernel<D, NP>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo,
+                    L, scale_log2, sc, sa);
 }
 
 // KV-split factor for a launch of C = ceil(L/256) x H CTAs: the S in 1..8 minimising the estimated
@@ -1516,6 +577,20 @@ static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
   return a;
 }
 
+// The step's variant per head dim (profiles/README.md, attention table); TSV_ATTN_D128 / TSV_ATTN_D64
+// override it with any tsv_op_attention impl number (same-box A/B of whole steps).
+static int default_version(int D) {
+  static int v[2] = {-1, -1};
+  int& r = v[D == 128];
+  if (r < 0) {
+    const char* e = getenv(D == 128 ? "TSV_ATTN_D128" : "TSV_ATTN_D64");
+    // 1 (D = 128) / 3 (D = 64) of 8 exp2 pairs by polynomial (round-2 sweep, profiles/r02/mb_attn_sweep.jsonl)
+    r = e ? atoi(e) : (D == 128 ? 51 : 53);
+    if (r < 50 || r > 54) r = D == 128 ? 51 : 53;
+  }
+  return r;
+}
+
 template <int D>
 static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv, bf16* o,
                      long long ldo, int L, int H, int version, const AttnScatter& sc, cudaStream_t s,
@@ -1524,97 +599,23 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
   if (make_tmap_heads(&tq, q, D, H, L, ldq) || make_tmap_heads(&tk, k, D, H, L, ldk) ||
       make_tmap_heads(&tv, v, D, H, L, ldv))
     return -1;
-  static unsigned long long done = 0;
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (!(done >> dev & 1ull)) {
-    cudaFuncSetAttribute(attention_tc_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, AttnCfg<D>::SMEM);
-    done |= 1ull << dev;
-  }
   const float scale_log2 = (1.0f / sqrtf((float)D)) * 1.4426950408889634f;
-  if (version >= 40 && version < 50) {   // v5: 64-key K/V tiles, double-buffered S; 40 + n: n of 8 exp2 pairs by polynomial
-    CUtensorMap tk64, tv64;
-    if (make_tmap_heads(&tk64, k, D, H, L, ldk, 64) || make_tmap_heads(&tv64, v, D, H, L, ldv, 64)) return -1;
-    switch (version - 40) {
-      case 0: launch_fa5<D, 0>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
-      case 1: launch_fa5<D, 1>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
-      case 2: launch_fa5<D, 2>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
-      case 3: launch_fa5<D, 3>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
-      case 4: launch_fa5<D, 4>(tq, tk64, tv64, o, ldo, L, H, scale_log2, sc, s); break;
-      default: return -3;
-    }
-    return 0;
+  const AttnSplitArgs sa = plan_kv_split(L, H, D, spw);
+  // version = 50 + n: n of 8 exp2 pairs by polynomial
+  cudaError_t e;
+  switch (version) {
+    case 50: e = launch_fa<D, 0>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 51: e = launch_fa<D, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 52: e = launch_fa<D, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 53: e = launch_fa<D, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 54: e = launch_fa<D, 4>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    default: return -3;
   }
-  if (version >= 60) {   // 60 + n: CTA-pair kernel (D = 128 only), lazy max, n of 8 exp2 pairs by polynomial
-    if (D != 128) return -3;
-    CUtensorMap tk64, tv64;   // K halves: 64-key boxes; V halves: 128 keys x 64 columns (the default box)
-    if (make_tmap_heads(&tk64, k, D, H, L, ldk, 64)) return -1;
-    switch (version - 60) {
-      case 0: launch_fa2<0>(tq, tk64, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      case 1: launch_fa2<1>(tq, tk64, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      case 2: launch_fa2<2>(tq, tk64, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      case 3: launch_fa2<3>(tq, tk64, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      default: return -3;
-    }
-    return 0;
-  }
-  if (version >= 50) {   // 50 + n: lazy row max (see attention_fa_kernel), n of 8 exp2 pairs by polynomial
-    const AttnSplitArgs sa = plan_kv_split(L, H, D, spw);
-    switch (version - 50) {
-      case 0: launch_fa<D, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-      case 1: launch_fa<D, 1, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-      case 2: launch_fa<D, 2, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-      case 3: launch_fa<D, 3, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-      case 4: launch_fa<D, 4, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-      default: return -3;
-    }
-    return 0;
-  }
-  if (version == 2) {
-    dim3 grid((L + AT_BM - 1) / AT_BM, H);
-    attention_tc_kernel<D><<<grid, AT_THREADS, AttnCfg<D>::SMEM, s>>>(tq, tk, tv, o, ldo, L, scale_log2);
-  } else {
-    // version 3: the default poly share; 10 + n: n of 8 exp2 pairs by polynomial (tuning sweeps);
-    // 20 + n: the same with P handed over in two halves (SPLIT)
-    const int np = version >= 10 ? version % 10 : default_npoly<D>();
-    if (version >= 20) {
-      switch (np) {
-        case 1: launch_fa<D, 1, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-        case 2: launch_fa<D, 2, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-        case 3: launch_fa<D, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-        case 4: launch_fa<D, 4, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-        default: return -3;
-      }
-      return 0;
-    }
-    switch (np) {
-      case 1: launch_fa<D, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      case 2: launch_fa<D, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      case 3: launch_fa<D, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      case 4: launch_fa<D, 4>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      case 5: launch_fa<D, 5>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s); break;
-      default: return -3;
-    }
-  }
-  return 0;
+  return e == cudaSuccess ? 0 : -5;
 }
 
-// The step's variant per head dim (profiles/README.md, attention table); TSV_ATTN_D128 / TSV_ATTN_D64
-// override it with any tsv_op_attention impl number >= 3 (same-box A/B of whole steps).
-static int default_version(int D) {
-  static int v[2] = {-1, -1};
-  int& r = v[D == 128];
-  if (r < 0) {
-    const char* e = getenv(D == 128 ? "TSV_ATTN_D128" : "TSV_ATTN_D64");
-    r = e ? atoi(e) : (D == 128 ? 51 : 52);   // lazy max; 1 (D = 128) / 2 (D = 64) of 8 exp2 pairs by polynomial (in-step A/B)
-    if (r < 3) r = 3;
-  }
-  return r;
-}
-
-// returns 0 if the tensor-core path was launched, nonzero if the layout is unsupported by TMA.
-// version 3: two query tiles per CTA, P in TMEM (the step's kernel); version 2: one query tile,
-// P in shared memory (kept for comparison).
+// returns 0 if the kernel was launched; -1: layout unsupported by TMA (alignment), -3: unknown
+// version, -4: bad scatter, -5: launch error (cudaGetLastError has it)
 int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
                      bf16* o, long long ldo, int L, int H, int D, cudaStream_t s, int version,
                      const AttnScatter* scatter, const AttnSplitWs* split) {
@@ -1622,12 +623,12 @@ int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk,
   AttnScatter sc;
   if (scatter) {
     sc = *scatter;
-    if (sc.k < 1 || sc.k > 8 || version == 2) return -4;
+    if (sc.k < 1 || sc.k > 8) return -4;
   }
   if (((ldq | ldk | ldv) * 2) % 16 || ((reinterpret_cast<uintptr_t>(q) | reinterpret_cast<uintptr_t>(k) |
                                         reinterpret_cast<uintptr_t>(v)) & 15))
     return -1;
-  if (version == 3) version = default_version(D);
+  if (version <= 3) version = default_version(D);
   if (D == 128) return launch_tc<128>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, sc, s, split);
   if (D == 64) return launch_tc<64>(q, ldq, k, ldk, v, ldv, o, ldo, L, H, version, sc, s, split);
   return -1;

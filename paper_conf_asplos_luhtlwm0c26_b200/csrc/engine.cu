@@ -821,7 +821,8 @@ static tsv_status attention_all(StepEnv& E) {
         rc = attention_launch(q, w, q + m.h / k, w, q + 2 * m.h / k, w, c.obuf + b * L * (m.h / k), m.h / k, (int)L,
                               m.H / k, m.D, c.s->stream, 3, nullptr, kvs);
       }
-      if (rc) return fail(TSV_E_CUDA, "attention: tensor map creation failed");
+      if (rc == -5) CK(cudaGetLastError());
+      if (rc) return fail(TSV_E_CUDA, "attention launch failed (%d)", rc);
     }
   }
   return TSV_OK;
@@ -2271,16 +2272,13 @@ tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int
 tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
                             void* o, int64_t ldo, int L, int H, int D, int impl, void* stream) {
   if (D != 64 && D != 128) return fail(TSV_E_INVAL, "D must be 64 or 128");
-  if (impl < 0 || (impl > 2 && (impl < 11 || impl > 15) && (impl < 21 || impl > 24) && (impl < 40 || impl > 44) && (impl < 50 || impl > 54) && (impl < 60 || impl > 63))) return fail(TSV_E_INVAL, "bad attention impl %d", impl);
-  if (impl == 1) {
-    attention_mma_launch(reinterpret_cast<const bf16*>(q), ldq, reinterpret_cast<const bf16*>(k), ldk,
-                         reinterpret_cast<const bf16*>(v), ldv, reinterpret_cast<bf16*>(o), ldo, L, H, D,
-                         reinterpret_cast<cudaStream_t>(stream));
-  } else if (attention_launch(reinterpret_cast<const bf16*>(q), ldq, reinterpret_cast<const bf16*>(k), ldk,
-                              reinterpret_cast<const bf16*>(v), ldv, reinterpret_cast<bf16*>(o), ldo, L, H, D,
-                              reinterpret_cast<cudaStream_t>(stream), impl == 0 ? 3 : impl)) {
-    return fail(TSV_E_INVAL, "attention: operands must be 16-byte aligned with 16-byte row strides");
-  }
+  if (impl < 0) return fail(TSV_E_INVAL, "bad attention impl %d", impl);
+  const int rc = attention_launch(reinterpret_cast<const bf16*>(q), ldq, reinterpret_cast<const bf16*>(k), ldk,
+                                  reinterpret_cast<const bf16*>(v), ldv, reinterpret_cast<bf16*>(o), ldo, L, H, D,
+                                  reinterpret_cast<cudaStream_t>(stream), impl == 0 ? 3 : impl);
+  if (rc == -3) return fail(TSV_E_INVAL, "bad attention impl %d", impl);
+  if (rc == -5) CK(cudaGetLastError());
+  if (rc) return fail(TSV_E_INVAL, "attention: operands must be 16-byte aligned with 16-byte row strides");
   CK(cudaGetLastError());
   return TSV_OK;
 }

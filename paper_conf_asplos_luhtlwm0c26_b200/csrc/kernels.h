@@ -167,8 +167,9 @@ void qk_norm_rope_launch(bf16* qkv, long long ld, int rows, int n_first, int H, 
                          bf16* pack_out, int k_sp, cudaStream_t s);
 
 // Joint attention, non-causal: O[l, h*D + d] = softmax(q k^T / sqrt(D)) v for heads h in [0, H).
-// attention_launch: tcgen05/TMEM kernel (returns nonzero if the layout is not TMA-compatible).
-// attention_mma_launch: the mma.sync (FA2-style) baseline kept for comparison.
+// attention_launch: tcgen05/TMEM kernel (returns nonzero if the layout is not TMA-compatible, the
+// version is unknown or the launch failed).  version <= 3: the default per head dim; 50 + n: n of 8
+// exp2 pairs by polynomial (attention_tc.cu).
 // q(l, h) at q + l*ldq + h*D (same for k, v, o). L rows.
 // KV-split (flash-decoding style) for launches with too few CTAs to fill the GPU (SP = 4/8 head
 // shards, small images): split s of a (query block, head) covers key tiles [s tps, (s+1) tps);
@@ -184,8 +185,6 @@ struct AttnSplitWs {
 int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
                      bf16* o, long long ldo, int L, int H, int D, cudaStream_t s, int version = 3,
                      const AttnScatter* scatter = nullptr, const AttnSplitWs* split = nullptr);
-void attention_mma_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
-                          bf16* o, long long ldo, int L, int H, int D, cudaStream_t s);
 
 // dst[m, c] = bf16(src[m, c]) (fp32 -> bf16), row strides in elements
 void f32_to_bf16_launch(const float* src, long long lds, bf16* dst, long long ldd, int M, int C, cudaStream_t s);

@@ -7,7 +7,14 @@ Runtime: several minutes on 8 cores (12 B synthetic parameters + ~21 TFLOP of fp
 sd3_512_seed1000_S20.npz: SD3-medium-shaped CFG step 0 of S = 20 at 512x512 (t_0 = 1 ->
 t_1 = shift(0.95)), request seed 1000 (inputs ids 1-5), same weight seed.  Keys: v, x_next.
 
-Usage: python tools/make_golden.py [flux|sd3 ...]   (default: both)
+flux2048_seed1000_S20_step0.npz: the north-star configuration (BASELINE.json north_star, SURVEY
+§8(d) config 4 "against the oracle at step 0"): FLUX.1-dev-shaped step 0 of S = 20 at 2048x2048
+(L_i = 16 384 image + 512 text tokens), request seed 1000, guidance 3.5, same weight seed.  Keys:
+v, x_next stored as float32 (the oracle computes in float64; float32 storage keeps the file at
+8 MB and its rounding, 2^-24 relative, is far below the 2e-2 tolerance).  Runtime: ~1.5-2 h on
+8 cores (~418 TFLOP of fp64 plus 3.9e11 exponentials).
+
+Usage: python tools/make_golden.py [flux|sd3|flux2048 ...]   (default: flux sd3)
 """
 import os
 import sys
@@ -44,10 +51,20 @@ def flux():
     print(f"wrote {out} in {time.time() - t0:.1f} s; |v|max={np.abs(v).max():.4f}")
 
 
+def flux2048():
+    t0 = time.time()
+    x, T, y = request_inputs(FLUX, 2048, 2048, 1000)
+    W = Weights(FLUX, cache_bytes=0)
+    v, xn = F.request_step(FLUX, W, x, T, y, 0, 20, 3.5, 2048, 2048)
+    out = os.path.join(ROOT, "tests", "golden", "flux2048_seed1000_S20_step0.npz")
+    np.savez_compressed(out, v=v.astype(np.float32), x_next=xn.astype(np.float32))
+    print(f"wrote {out} in {time.time() - t0:.1f} s; |v|max={np.abs(v).max():.4f}")
+
+
 def main():
     which = sys.argv[1:] or ["flux", "sd3"]
     for w in which:
-        {"flux": flux, "sd3": sd3}[w]()
+        {"flux": flux, "sd3": sd3, "flux2048": flux2048}[w]()
 
 
 if __name__ == "__main__":

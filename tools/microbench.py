@@ -123,7 +123,7 @@ def attn_cases():
         qkv = torch.randn(L, 3 * H * D, device="cuda").to(torch.bfloat16)
         o = torch.empty(L, H * D, dtype=torch.bfloat16, device="cuda")
         ld = 3 * H * D
-        impls = (0, 1) + ((11, 12, 13, 14) if sweep else ())
+        impls = (0,) + ((50, 51, 52, 53, 54) if sweep else ())
         if os.environ.get("ATTN_IMPLS"):
             impls = tuple(int(x) for x in os.environ["ATTN_IMPLS"].split(","))
         fns = {impl: (lambda impl=impl: tsv.op_attention(qkv, qkv[:, H * D:], qkv[:, 2 * H * D:], o, L, H, D,
@@ -135,9 +135,7 @@ def attn_cases():
                 times[impl].append(timeit(fns[impl], iters=5 if L > 8000 else 20))
         for impl in impls:
             ms = sorted(times[impl])[len(times[impl]) // 2]
-            name = {0: "tcgen05", 1: "mma.sync"}.get(
-                impl, f"tcgen05-poly{impl % 10}" + ("-lazymax" if impl >= 50 else "-v5" if impl >= 40
-                                                    else "-splitP" if impl >= 20 else ""))
+            name = "tcgen05" if impl == 0 else f"tcgen05-poly{impl % 10}"
             print(json.dumps({"op": "attention", "impl": name, "L": L, "H": H, "D": D,
                               "ms": round(ms, 4), "tflops": round(4 * L * L * D * H / ms / 1e9, 1),
                               "all_ms": [round(t, 4) for t in times[impl]]}), flush=True)
