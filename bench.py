@@ -1,20 +1,23 @@
 """Benchmark: one FLUX.1-dev-shaped denoising step (the whole hot path, S:§8(a) a1-a12) under
 step-level Ulysses SP, through libtsv.so's C-ABI.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--res 512] [--model flux|sd3] [--impl ours|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--res 2048] [--model flux|sd3] [--impl ours|reference]
 
-N = 1: BASELINE.json config 2 (FLUX 512x512 = 1024 image + 512 text tokens, SP=1).
-N > 1 (torchrun, one process per GPU): the same request at SP = N on ranks [0..N) over NCCL
-(strong scaling: the step's work is fixed).  Metric: step latency (ms, lower is better), timed
-with CUDA events on the engine's stream, max over ranks.  Inputs are larger than L2 (23.7 GB of
-weights streamed per step), so no L2 flush is needed between timed steps.
+N = 1: the north-star configuration (BASELINE.json north_star: "a FLUX.1-dev-shaped 2048^2
+denoising step ... at SP=1"; BASELINE config 4's resolution, 16 384 image + 512 text tokens).
+--res 512 gives config 2's line.  N > 1 (torchrun, one process per GPU): the same request at SP = N
+on ranks [0..N) (strong scaling: the step's work is fixed); all-to-alls fused into the epilogues
+over CUDA-IPC peer memory (default) or NCCL send/recv; a second profiled pass on the NCCL exchange
+transport gives the communication share and the all-to-all bus GB/s.  Metric: step latency (ms,
+lower is better), CUDA events on the engine's stream around K graph replays, max over ranks; the
+per-step latencies give the CV.  Inputs are larger than L2 (23.7 GB of weights
+streamed per step), so no L2 flush is needed between timed steps.
 
 --model sd3: the SD3-medium-shaped CFG step of config 5 (24 joint blocks, L_t = 333, batch-2 CFG
-pair) instead of FLUX (a secondary line; the default N = 1 run is config 2).
+pair) instead of FLUX (a secondary line).
 
---impl reference: the float64 CPU oracle on the box's host cores (the tier's reference arm),
-timed on a bounded sample of the same step (one double + one single block at full width,
-extrapolated to 19 + 38 blocks).
+--impl reference: the float64 CPU oracle on the box's host cores (the tier's reference arm), timed
+on a bounded sample of the same step and extrapolated (see oracle_sample).
 """
 from __future__ import annotations
 
@@ -33,12 +36,14 @@ sys.path.insert(0, ROOT)
 METRIC = "DiT step latency (ms) per resolution at SP=1/2/4/8; attn+GEMM TFLOP/s vs peak"
 
 
-def gemm_traffic(res: int):
-    """Mean DRAM bytes (read + write) per GEMM launch from the newest committed ncu launch list of
-    one step at this resolution (profiles/rNN/launches_<res>.csv), or None."""
+def ncu_traffic(res: int, pattern: str, model: str = "flux"):
+    """Mean DRAM bytes (read + write) per launch of kernels whose name contains `pattern`, from the
+    newest committed ncu launch list of one step at this resolution (profiles/rNN/launches_<res>.csv,
+    SD3: launches_sd3<res>.csv), or None."""
     import csv
     import glob
-    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*", f"launches_{res}.csv")))
+    tag = f"sd3{res}" if model == "sd3" else f"{res}"
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*", f"launches_{tag}.csv")))
     if not files:
         return None
     rows = list(csv.reader(open(files[-1])))
@@ -48,7 +53,7 @@ def gemm_traffic(res: int):
     scale = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
     per = {}
     for r in rows[hi + 1:]:
-        if len(r) > vi and "gemm" in r[ki] and r[mi].startswith("dram__bytes"):
+        if len(r) > vi and pattern in r[ki] and r[mi].startswith("dram__bytes"):
             per[r[ii]] = per.get(r[ii], 0.0) + float(r[vi].replace(",", "")) * scale.get(r[ui], 1.0)
     if not per:
         return None
@@ -144,27 +149,40 @@ class Clocks:
 
 
 # --------------------------------------------------------------------------- oracle (reference / cpu_baseline)
-def oracle_sample(res: int, n_samples: int = 1):
-    """Time the float64 oracle on one double + one single FLUX block at full width (weights
-    pre-generated, not timed) and extrapolate to the full 57-block step.  Returns (ms, detail)."""
+SAMPLE_ROWS = 1024   # query / token rows of the bounded oracle sample at L > 4096 (~10-20 s of host work)
+
+
+def oracle_sample(res: int):
+    """The float64 oracle (oracle/flux.py, as it stands) timed on a bounded sample of one FLUX step
+    and extrapolated.  Weights and inputs are generated first (input synthesis, untimed).
+      * L <= 4096 (512^2, 256^2): embed + one double block + one single block + final at full width,
+        x 19 / x 38 for the blocks.
+      * larger L (1024^2 and up): the oracle's per-row work of one double and one single block on
+        n = SAMPLE_ROWS rows -- LN-modulate, the QKV / out / MLP GEMMs, QK-RMSNorm, RoPE, and softmax
+        attention of the n query rows against all L keys -- scaled by L / n, then x 19 / x 38.  Every
+        op is row-local except attention, whose cost is linear in the query rows for fixed keys, so
+        the scaling is exact up to cache effects.
+    Returns (ms, detail)."""
     import numpy as np
     from oracle import flux as F
     from oracle.config import FLUX
     from oracle.weights import Weights, request_inputs
     cfg = FLUX
+    h, H, D = cfg.hidden, cfg.heads, cfg.head_dim
     W = Weights(cfg, cache_bytes=8 << 30)
     x, T, y = request_inputs(cfg, res, res, 1000)
     Li, Lt = x.shape[0], T.shape[0]
-    for n in W.table:  # generate the sampled blocks' weights up front (input synthesis, untimed)
-        if n.startswith(("double0.", "single0.", "img_in", "txt_in", "final", "time_in", "guidance_in", "vector_in")):
-            W[n]
+    L = Li + Lt
+    for nme in W.table:  # generate the sampled blocks' weights up front (input synthesis, untimed)
+        if nme.startswith(("double0.", "single0.", "img_in", "txt_in", "final", "time_in", "guidance_in", "vector_in")):
+            W[nme]
     rng = np.random.default_rng(0)
-    img = rng.standard_normal((Li, cfg.hidden))
-    txt = rng.standard_normal((Lt, cfg.hidden))
     vec = F.conditioning_vec(cfg, W, 0.5, y, 3.5)
-    ang = F.rope_angles(F.position_ids(Lt, res, res), cfg.axes_dim, cfg.theta)
-    times = []
-    for _ in range(n_samples):
+    cores = len(os.sched_getaffinity(0))
+    if L <= 4096:
+        img = rng.standard_normal((Li, h))
+        txt = rng.standard_normal((Lt, h))
+        ang = F.rope_angles(F.position_ids(Lt, res, res), cfg.axes_dim, cfg.theta)
         t0 = time.perf_counter()
         F.linear(x, W["img_in.w"], W["img_in.b"])
         F.linear(T, W["txt_in.w"], W["txt_in.b"])
@@ -175,19 +193,50 @@ def oracle_sample(res: int, n_samples: int = 1):
         t3 = time.perf_counter()
         F.final_layer(W, img, vec)
         t4 = time.perf_counter()
-        times.append(((t1 - t0) + cfg.n_double * (t2 - t1) + cfg.n_single * (t3 - t2) + (t4 - t3)) * 1e3)
-    cores = len(os.sched_getaffinity(0))
-    return statistics.median(times), dict(
-        kind="oracle", cores=cores,
-        sample=f"float64 numpy oracle: embed + 1 double + 1 single block + final of FLUX {res}x{res} "
-               f"(L={Li + Lt}) at full width, extrapolated to 19 double + 38 single blocks; "
-               f"weights pre-generated (untimed); BLAS threads = {cores}")
+        ms = ((t1 - t0) + cfg.n_double * (t2 - t1) + cfg.n_single * (t3 - t2) + (t4 - t3)) * 1e3
+        return ms, dict(kind="oracle", cores=cores, extrapolated=True,
+                        sample=f"float64 numpy oracle: embed + 1 double + 1 single block + final of FLUX {res}x{res} "
+                               f"(L={L}) at full width, x19 / x38 blocks; weights pre-generated (untimed); "
+                               f"BLAS threads = {cores}")
+    n = SAMPLE_ROWS
+    u = rng.standard_normal((n, h))
+    k_all = rng.standard_normal((L, H, D))   # the keys / values every sampled query row attends to
+    v_all = rng.standard_normal((L, H, D))
+    ang = F.rope_angles(F.position_ids(Lt, res, res), cfg.axes_dim, cfg.theta)[:n]
+
+    def qk_rope(qkv, p):
+        q, k, v = F.split_qkv(qkv, H, D)
+        return F.apply_rope(F.rms_norm(q, W[p + "q_norm.g"]), ang), F.apply_rope(F.rms_norm(k, W[p + "k_norm.g"]), ang), v
+
+    t0 = time.perf_counter()   # one double block's per-row work (the img stream's weights for both streams)
+    p = "double0.img."
+    sh1, sc1, g1, sh2, sc2, g2 = F.modulation(W, p, vec, 6)
+    q, _, _ = qk_rope(F.linear(F.ln_modulate(u, sh1, sc1), W[p + "qkv.w"], W[p + "qkv.b"]), p)
+    o = F.attention(q, k_all, v_all)
+    xr = u + g1 * F.linear(o.reshape(n, h), W[p + "proj.w"], W[p + "proj.b"])
+    xr = xr + g2 * F.linear(F.gelu_tanh(F.linear(F.ln_modulate(xr, sh2, sc2), W[p + "fc1.w"], W[p + "fc1.b"])),
+                            W[p + "fc2.w"], W[p + "fc2.b"])
+    t1 = time.perf_counter()   # one single block's per-row work
+    p = "single0."
+    sh, sc, g = F.modulation(W, p, vec, 3)
+    y1 = F.linear(F.ln_modulate(u, sh, sc), W[p + "lin1.w"], W[p + "lin1.b"])
+    q, _, _ = qk_rope(y1[:, :3 * h], p)
+    o = F.attention(q, k_all, v_all).reshape(n, h)
+    xs = u + g * F.linear(np.concatenate([o, F.gelu_tanh(y1[:, 3 * h:])], axis=1), W[p + "lin2.w"], W[p + "lin2.b"])
+    t2 = time.perf_counter()
+    ms = (L / n) * (cfg.n_double * (t1 - t0) + cfg.n_single * (t2 - t1)) * 1e3
+    return ms, dict(kind="oracle", cores=cores, extrapolated=True,
+                    sample=f"float64 numpy oracle (oracle/flux.py ops as they stand): the per-row work of one double "
+                           f"and one single block of FLUX {res}x{res} (L={L}) on {n} token rows -- LN-modulate, "
+                           f"QKV/out/MLP GEMMs, QK-RMSNorm, RoPE, softmax attention of {n} queries over all {L} keys "
+                           f"-- scaled by L/{n} and x19 / x38 blocks (embed/final < 0.1 % omitted); weights "
+                           f"pre-generated (untimed); BLAS threads = {cores}")
 
 
 def oracle_sample_sd3(res: int):
     """SD3: embed + joint block 0 + final of one CFG branch at full width, extrapolated to 24
     joint blocks x 2 branches (weights pre-generated, not timed)."""
-    import numpy as np
+    import numpy as np  # noqa: F401
     from oracle import flux as F
     from oracle import sd3 as S3
     from oracle.config import SD3
@@ -210,7 +259,7 @@ def oracle_sample_sd3(res: int):
     t3 = time.perf_counter()
     ms = 2 * ((t1 - t0) + cfg.n_double * (t2 - t1) + (t3 - t2)) * 1e3
     cores = len(os.sched_getaffinity(0))
-    return ms, dict(kind="oracle", cores=cores,
+    return ms, dict(kind="oracle", cores=cores, extrapolated=True,
                     sample=f"float64 numpy oracle: embed + joint block 0 + final of one CFG branch of SD3 "
                            f"{res}x{res} (L={Li + Lt}) at full width, extrapolated to 24 blocks x 2 branches; "
                            f"weights pre-generated (untimed); BLAS threads = {cores}")
@@ -247,6 +296,31 @@ def run_reference(args):
 
 
 # --------------------------------------------------------------------------- our arm
+NOMINAL_DENSE_BF16 = 2250.0   # TFLOP/s per B200 at the 1965 MHz boost clock (B200_PROFILING.md)
+
+
+def roofline_entry(kind, prof_cls, pk, sm_mhz, traffic, kernel):
+    """Roofline of one kernel class from the profiled pass: achieved = algorithmic FLOPs per launch /
+    mean device time per launch; peak = the measured sustained bf16 peak (MEASURED_PEAKS.json);
+    tensor_util_clock = achieved / (nominal dense peak x in-run SM clock / boost clock), the
+    clock-relative tensor-pipe utilisation the north star names."""
+    n = prof_cls["launches"]
+    if not n or not prof_cls["ms"]:
+        return None
+    t = prof_cls["ms"] / n * 1e-3
+    fl = prof_cls["flops"] / n
+    by = prof_cls["bytes"] / n
+    achieved = fl / t / 1e12
+    at_clock = NOMINAL_DENSE_BF16 * (sm_mhz / 1965.0) if sm_mhz else None
+    return {"bound": "tensor", "kernel": kernel, "achieved": round(achieved, 2), "peak": pk["tflops"],
+            "unit": "TFLOP/s", "frac": round(achieved / pk["tflops"], 4),
+            "traffic": traffic["bytes_per_launch"] if traffic else None, "traffic_detail": traffic,
+            "algorithmic_flops_per_launch": round(fl), "algorithmic_bytes_per_launch": round(by),
+            "launches_per_step": n // 2, "us_per_launch": round(t * 1e6, 2),
+            "tensor_util_clock": round(achieved / at_clock, 4) if at_clock else None,
+            "peak_source": pk["source"] + " bf16_tflops_sustained"}
+
+
 def run_ours(args):
     import numpy as np
     import torch
@@ -272,10 +346,13 @@ def run_ours(args):
         else:
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     mdl = MODELS[args.model]
+    res = args.res
+    Li = (res // 16) ** 2
     eng = tsv.Engine(args.model, devices=[local], rank_base=rank, world_size=world)
+    has_nccl_group = False
     if one_gpu:
         g = eng.group_create(list(range(world)))
-        blob = eng.group_ipc_export(g, max_tokens=(args.res // 16) ** 2 + mdl["Lt"], max_evals=2)
+        blob = eng.group_ipc_export(g, max_tokens=Li + mdl["Lt"], max_evals=2)
         blobs = [None] * world
         dist.all_gather_object(blobs, blob)
         eng.group_ipc_import(g, blobs)
@@ -286,12 +363,13 @@ def run_ours(args):
         dist.broadcast_object_list(obj, src=0)
         eng.init_world(obj[0])
         g = eng.group_create(list(range(world)), nccl_id=obj[1])
+        has_nccl_group = True
         transport = "nccl-exchange"
         if args.transport == "fused":
             # the product path: all-to-alls fused into the epilogues as stores into the other
             # processes' CUDA-IPC windows (tsv_group_ipc_export / _import); NCCL stays the fallback
             try:
-                blob = eng.group_ipc_export(g, max_tokens=(args.res // 16) ** 2 + mdl["Lt"], max_evals=2)
+                blob = eng.group_ipc_export(g, max_tokens=Li + mdl["Lt"], max_evals=2)
                 blobs = [None] * world
                 dist.all_gather_object(blobs, blob)
                 eng.group_ipc_import(g, blobs)
@@ -305,9 +383,8 @@ def run_ours(args):
     else:
         g = eng.group_create([0])
         transport = "none"
-    res = args.res
     K, Wm = args.steps, args.warmup
-    total_steps = Wm + K + Wm + K + 2 + 2   # timed + profiled + e2e passes
+    total_steps = Wm + K + 2 + 2 + K + 1   # warm-up + timed + profiled + NCCL-profiled + e2e passes
     req = eng.request_create(res, res, num_steps=total_steps, seed=1000)
     step = 0
 
@@ -316,6 +393,13 @@ def run_ours(args):
         if world > 1:
             dist.barrier()
 
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=red_dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
     for _ in range(Wm):
         eng.request_step(req, step, g)
         step += 1
@@ -323,30 +407,55 @@ def run_ours(args):
     kc0 = eng.kernel_count()
     with Clocks(local) as clk:
         barrier()
-        ev0 = eng.group_record(g)
+        evs = [eng.group_record(g)]
         for _ in range(K):
             eng.request_step(req, step, g)
             step += 1
-        ev1 = eng.group_record(g)
-        total_ms = eng.event_elapsed_ms(ev0, ev1)
+            evs.append(eng.group_record(g))
+        total_ms = eng.event_elapsed_ms(evs[0], evs[-1])
         barrier()
     launches = eng.kernel_count() - kc0
-    ms = total_ms / K
-    if world > 1:
-        t = torch.tensor([ms], device=red_dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+    per_step = [eng.event_elapsed_ms(evs[i], evs[i + 1]) for i in range(K)]
+    ms = max_over_ranks(total_ms / K)
+    mean = statistics.fmean(per_step)
+    cv = max_over_ranks(statistics.stdev(per_step) / mean if K > 1 else 0.0)
+    median_ms = max_over_ranks(statistics.median(per_step))
+    clocks = clk.summary()
 
     # per-kernel-class device time (a separate profiled pass: events around every launch)
-    eng.profile(True)
-    for _ in range(2):
-        eng.request_step(req, step, g)
-        step += 1
-    prof = eng.profile_read()
-    eng.profile(False)
+    def profiled(n=2):
+        nonlocal step
+        eng.profile(True)
+        for _ in range(n):
+            eng.request_step(req, step, g)
+            step += 1
+        pr = eng.profile_read()
+        eng.profile(False)
+        return pr
+    prof = profiled()
+
+    # N > 1: the same step on the NCCL exchange transport, profiled: the all-to-alls are then separate
+    # NCCL calls whose device time and bytes give the communication share (Fig. 2 analogue)
+    # and the all-to-all bus bandwidth ((k-1)/k of each rank's send buffer / time, nccl-tests busbw)
+    comm = None
+    if world > 1:
+        a2a_fused_ms = prof["a2a"]["ms"] / 2
+        comm = {"transport": transport, "barrier_ms_per_step": round(max_over_ranks(a2a_fused_ms), 4),
+                "barrier_share": round(max_over_ranks(a2a_fused_ms) / ms, 4)}
+        if has_nccl_group and transport.startswith("fused"):
+            eng.set_transport(False)
+            pn = profiled()
+            eng.set_transport(True)
+            a2a_ms = pn["a2a"]["ms"] / 2
+            step_ms = sum(v["ms"] for v in pn.values()) / 2
+            comm["nccl_exchange"] = {
+                "a2a_ms_per_step": round(max_over_ranks(a2a_ms), 4),
+                "a2a_share": round(max_over_ranks(a2a_ms / step_ms), 4),
+                "bus_gbs": round(pn["a2a"]["bytes"] / 2 / (a2a_ms * 1e-3) / 1e9, 1) if a2a_ms else None,
+                "bus_peak_gbs": 900.0,
+                "calls_per_step": pn["a2a"]["launches"] // 2}
 
     # end to end through the public API with host buffers: H2D latent in, step, D2H latent out
-    Li = (res // 16) ** 2
     r0, r1 = tsv.shard_range(Li, world, rank)
     host = np.empty((r1 - r0, 64), np.float32)
     host[:] = eng.read_latent(req, r0, r1 - r0)
@@ -355,29 +464,31 @@ def run_ours(args):
     for i in range(K + 1):
         t0 = time.perf_counter()
         eng.write_latent(req, host, r0)
-        ev = eng.request_step(req, step, g)
+        eng.request_step(req, step, g)
         step += 1
         eng.read_latent(req, r0, r1 - r0, out=host)
         if world > 1:
             dist.barrier()
         if i:
             e2e_times.append((time.perf_counter() - t0) * 1e3)
-    e2e_ms = statistics.median(e2e_times)
-    if world > 1:
-        t = torch.tensor([e2e_ms], device=red_dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_ms = float(t.item())
+    e2e_ms = max_over_ranks(statistics.median(e2e_times))
 
     pk = peaks()
-    traffic = gemm_traffic(res) if world == 1 and args.model == "flux" else None
+    sm = clocks.get("sm_mhz")
     gemm_fl, attn_fl = mdl["flops"](res, world)
-    g_ms = prof["gemm"]["ms"] / prof["gemm"]["launches"] if prof["gemm"]["launches"] else 0
-    g_fl = prof["gemm"]["flops"] / max(prof["gemm"]["launches"], 1)
-    achieved = (g_fl / (g_ms * 1e-3)) / 1e12 if g_ms else None
     step_prof_ms = sum(v["ms"] for v in prof.values()) / 2
     shares = {c: round(v["ms"] / 2 / step_prof_ms, 4) for c, v in prof.items()} if step_prof_ms else {}
-    attn_tf = (prof["attention"]["flops"] / (prof["attention"]["ms"] * 1e-3) / 1e12) if prof["attention"]["ms"] else None
     step_tf = (gemm_fl + attn_fl) / (ms * 1e-3) / 1e12
+    one = world == 1
+    rl = {
+        "gemm": roofline_entry("gemm", prof["gemm"], pk, sm,
+                               ncu_traffic(res, "gemm", args.model) if one else None,
+                               "gemm_tc2_kernel / gemm_tc_kernel (tcgen05 GEMM, all GEMM launches of the step)"),
+        "attention": roofline_entry("attention", prof["attention"], pk, sm,
+                                    ncu_traffic(res, "attention", args.model) if one else None,
+                                    "attention_fa_kernel (tcgen05/TMEM joint attention)"),
+    }
+    dominant = max(("gemm", "attention"), key=lambda c: prof[c]["ms"])
 
     if rank == 0:
         line = {
@@ -388,22 +499,22 @@ def run_ours(args):
                        "sp": world, "resolution": res, "global_batch": 1, "seq_len": Li + mdl["Lt"],
                        "parallelism": f"ulysses-sp{world}", "transport": transport,
                        "l2": f"inputs larger than L2 ({mdl['weights_gb']} GB of weights streamed per step); no flush"},
-            "roofline": {"bound": "tensor",
-                         "kernel": "gemm_tc2_kernel / gemm_tc_kernel (tcgen05 GEMM, all GEMM launches of the step)",
-                         "achieved": round(achieved, 2) if achieved else None, "peak": pk["tflops"],
-                         "unit": "TFLOP/s", "frac": round(achieved / pk["tflops"], 4) if achieved else None,
-                         "traffic": traffic["bytes_per_launch"] if traffic else None,
-                         "traffic_detail": traffic,
-                         "algorithmic_bytes_per_launch": round(prof["gemm"]["bytes"] / max(prof["gemm"]["launches"], 1)),
-                         "algorithmic_flops_per_launch": round(g_fl),
-                         "peak_source": pk["source"] + " bf16_tflops_sustained"},
-            "step_tflops": round(step_tf, 2), "attention_tflops": round(attn_tf, 2) if attn_tf else None,
+            "roofline": dict(rl[dominant], dominant_share=shares.get(dominant)),
+            "roofline_kernels": rl,
+            "step_tflops": round(step_tf, 2),
+            "step_tensor_util": {"vs_sustained_peak": round(step_tf / pk["tflops"], 4),
+                                 "clock_relative": round(step_tf / (NOMINAL_DENSE_BF16 * sm / 1965.0), 4) if sm else None,
+                                 "note": "algorithmic step FLOPs / step time; clock_relative against 2.25 PF x "
+                                         "in-run SM clock / 1965 MHz (ncu tensor-pipe %: profiles/)"},
+            "latency": {"median_ms": round(median_ms, 4), "cv": round(cv, 5), "steps": K},
             "time_share": shares,
             "e2e": {"value": round(e2e_ms, 4), "unit": "ms", "h2d_bytes_per_step": int(host.nbytes),
                     "d2h_bytes_per_step": int(host.nbytes)},
             "gpu_launches": int(launches),
-            "clocks": clk.summary(),
+            "clocks": clocks,
         }
+        if comm:
+            line["comm"] = comm
         if world == 1 and not args.no_cpu_baseline:
             ms_cpu, detail = (oracle_sample_sd3 if args.model == "sd3" else oracle_sample)(res)
             detail["value"] = round(ms_cpu, 1)
@@ -418,9 +529,9 @@ def run_ours(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--res", type=int, default=512)
+    ap.add_argument("--res", type=int, default=2048)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--model", default="flux", choices=sorted(MODELS))
     ap.add_argument("--transport", default="fused", choices=["fused", "nccl"],

@@ -88,6 +88,15 @@ typedef int64_t tsv_request;
 typedef int32_t tsv_group;
 typedef int64_t tsv_event;
 
+/* Caller-supplied device allocator (tsv_engine_set_allocator).  alloc returns `bytes` of device
+ * memory on `device` usable in stream order on `stream` (a cudaStream_t), or NULL on failure;
+ * free returns a pointer obtained from alloc with the same device and stream.  The engine calls
+ * free only once every use of the buffer is ordered before `stream`'s current position (same
+ * contract as cudaFreeAsync / PyTorch's caching allocator).  Both are called from the thread
+ * that makes the engine call. */
+typedef void* (*tsv_alloc_fn)(void* ctx, size_t bytes, int device, void* stream);
+typedef void (*tsv_free_fn)(void* ctx, void* ptr, int device, void* stream);
+
 typedef struct {
   int hidden;        /* h: 3072 for FLUX.1-dev */
   int heads;         /* H: 24 */
@@ -122,11 +131,30 @@ typedef struct {
 tsv_status tsv_model_preset(const char* name, tsv_model_desc* out);
 
 /* Create an engine hosting global ranks [rank_base, rank_base + n_local) on devices[0..n_local).
- * Generates all weights on every distinct device with SYNTH-1 (weight_seed).  Errors:
- * TSV_E_INVAL (bad desc / ranks), TSV_E_OOM, TSV_E_CUDA. */
+ * Device state is set up lazily, on the first call that needs it (tsv_group_create,
+ * tsv_debug_read_weight): streams, then all weights on every distinct device with SYNTH-1
+ * (weight_seed), so that tsv_engine_set_allocator / tsv_engine_set_stream can come first.
+ * Errors: TSV_E_INVAL (bad desc / ranks / device), TSV_E_CUDA. */
 tsv_status tsv_engine_create(const tsv_model_desc* model, const int* devices, int n_local, int rank_base,
                              int world_size, uint64_t weight_seed, tsv_engine** out);
 void tsv_engine_destroy(tsv_engine* eng);
+
+/* Optional PyTorch hooks (north_star: "PyTorch is used only for device memory, streams and process
+ * groups"; S:§8(b) conventions).  Both must be called before the engine's device state exists (before
+ * the first tsv_group_create), else TSV_E_STATE.
+ * tsv_engine_set_allocator: every device buffer of the engine except CUDA-IPC windows (weights,
+ * workspaces, per-request latents / modulation tables / tables) comes from alloc_fn and goes back
+ * through free_fn (see tsv_alloc_fn for the ordering contract); the engine never calls cudaMalloc
+ * for them.  Per-request buffers are allocated on the stream of the rank that uses them and
+ * released stream-ordered on that stream.  Without a caller allocator the engine uses cudaMalloc
+ * for engine-lifetime buffers and cudaMallocAsync / cudaFreeAsync for per-request ones.
+ * Errors: TSV_E_INVAL (NULL function), TSV_E_STATE.
+ * tsv_engine_set_stream: every rank hosted on `device` issues its kernels, copies and collectives
+ * on `cuda_stream` (a cudaStream_t the caller owns and keeps alive while the engine exists),
+ * instead of an engine-created non-blocking stream; virtual ranks on that device then share it
+ * (they run serialised).  Errors: TSV_E_INVAL (device not in the engine), TSV_E_STATE. */
+tsv_status tsv_engine_set_allocator(tsv_engine* eng, void* ctx, tsv_alloc_fn alloc_fn, tsv_free_fn free_fn);
+tsv_status tsv_engine_set_stream(tsv_engine* eng, int device, void* cuda_stream);
 
 /* Multi-process only: NCCL unique id (128 bytes) to be broadcast by the caller (e.g. with
  * torch.distributed) to every member of a group, and the world communicator used by reshard
@@ -178,10 +206,19 @@ tsv_status tsv_request_step(tsv_engine* eng, tsv_request req, int step, tsv_grou
 tsv_status tsv_request_step_batch(tsv_engine* eng, const tsv_request* reqs, int n, tsv_group group, tsv_event* done);
 
 /* Move the latent of `req` to `group` without running a step: bit-exact row moves given by the
- * reshard map (tsv_reshard_plan).  Asynchronous, ordered after the request's last step. */
+ * reshard map (tsv_reshard_plan).  Asynchronous and non-blocking (P:409's "asynchronous,
+ * non-blocking" hand-off): the row copies are ordered after the request's last step on the old
+ * ranks, the new ranks' streams wait for them, and the old shards are released stream-ordered; the
+ * host does not wait for the device.  On a GPU the request never ran on, its per-request state is
+ * set up too: the text rows (pinned host -> device) and their embedding, the RoPE / position
+ * tables (computed on the device), and the modulation table of all steps — copied from another
+ * local rank that already holds it, else computed (one M = S GEMM). */
 tsv_status tsv_request_reshard(tsv_engine* eng, tsv_request req, tsv_group group, tsv_event* done);
 
-/* Events (the latent "future"). */
+/* Events (the latent "future").  For a group using CUDA-IPC windows, wait / query /
+ * elapsed also check the group's device barrier: a member that stalled for ~10 s made the barrier
+ * give up, and the call then returns TSV_E_STATE (the step's results are invalid; the group must
+ * be recreated). */
 tsv_status tsv_event_wait(tsv_engine* eng, tsv_event ev);
 tsv_status tsv_event_query(tsv_engine* eng, tsv_event ev, int* done);
 /* Device time between two events of the same group, max over the group's local ranks (ms). */
@@ -265,7 +302,8 @@ tsv_status tsv_engine_set_transport(tsv_engine* eng, int mode);
  *   3. every member calls tsv_group_ipc_import, which maps the peers' windows (cudaIpcOpenMemHandle).
  * Afterwards steps on the group (with TSV_TRANSPORT_FUSED) need no NCCL communicator: the QKV and
  * attention epilogues store into the owners' windows and a device barrier orders the members (a
- * stalled peer makes the barrier give up after ~10 s instead of hanging).  Groups may then be
+ * stalled peer makes the barrier give up after ~10 s instead of hanging; the next tsv_event_wait /
+ * _query / _elapsed_ms on the group then returns TSV_E_STATE).  Groups may then be
  * created without nccl_id or a world communicator.  Errors: TSV_E_INVAL (sizes, foreign blob),
  * TSV_E_STATE (import before export), TSV_E_UNSUPPORTED (group not spanning processes), TSV_E_CUDA. */
 tsv_status tsv_group_ipc_export(tsv_engine* eng, tsv_group group, int64_t max_tokens, int max_evals, uint8_t* out,

@@ -10,6 +10,7 @@ import ctypes as C
 
 import numpy as np
 
+from . import _lib
 from ._lib import EPI, EXPORTED, LIB_PATH, ModelDesc, TsvError, check, last_error, lib  # noqa: F401
 
 __all__ = ["Engine", "ModelDesc", "TsvError", "model_preset", "shard_range", "reshard_plan", "nccl_unique_id",
@@ -80,6 +81,31 @@ class Engine:
         if self.h:
             lib.tsv_engine_destroy(self.h)
             self.h = None
+
+    # --------------------------------------------------------------- PyTorch hooks (before the first group)
+    def use_torch_allocator(self):
+        """Back every engine buffer (except CUDA-IPC windows) with PyTorch's caching allocator
+        (tsv_engine_set_allocator); the callbacks only forward to torch.cuda.caching_allocator_*."""
+        import torch
+
+        def _alloc(ctx, nbytes, device, stream):
+            try:
+                return torch.cuda.caching_allocator_alloc(int(nbytes), device, stream or 0)
+            except Exception:   # OOM: the engine reports TSV_E_OOM
+                return None
+
+        def _free(ctx, ptr, device, stream):
+            torch.cuda.caching_allocator_delete(ptr)
+
+        self._alloc_cb = _lib.ALLOC_FN(_alloc)   # kept alive as long as the engine
+        self._free_cb = _lib.FREE_FN(_free)
+        check(lib.tsv_engine_set_allocator(self.h, None, self._alloc_cb, self._free_cb))
+
+    def set_stream(self, device: int, stream):
+        """Issue every rank on `device` on `stream` (a torch.cuda.Stream or a raw cudaStream_t)."""
+        handle = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+        self._streams = getattr(self, "_streams", []) + [stream]   # keep the caller's stream alive
+        check(lib.tsv_engine_set_stream(self.h, device, C.c_void_p(handle)))
 
     def __del__(self):
         try:

@@ -48,11 +48,17 @@ class SchedRequest(C.Structure):
 _i32, _i64, _u64, _p, _f32 = C.c_int, C.c_int64, C.c_uint64, C.c_void_p, C.c_float
 _P = C.POINTER
 
+# tsv_alloc_fn / tsv_free_fn (include/tsv.h)
+ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_void_p, C.c_size_t, C.c_int, C.c_void_p)
+FREE_FN = C.CFUNCTYPE(None, C.c_void_p, C.c_void_p, C.c_int, C.c_void_p)
+
 _SIGS = {
     "tsv_last_error": (C.c_char_p, []),
     "tsv_model_preset": (_i32, [C.c_char_p, _P(ModelDesc)]),
     "tsv_engine_create": (_i32, [_P(ModelDesc), _P(_i32), _i32, _i32, _i32, _u64, _P(_p)]),
     "tsv_engine_destroy": (None, [_p]),
+    "tsv_engine_set_allocator": (_i32, [_p, _p, ALLOC_FN, FREE_FN]),
+    "tsv_engine_set_stream": (_i32, [_p, _i32, _p]),
     "tsv_nccl_unique_id": (_i32, [_P(C.c_uint8)]),
     "tsv_engine_init_world": (_i32, [_p, _P(C.c_uint8)]),
     "tsv_group_create": (_i32, [_p, _P(_i32), _i32, _P(C.c_uint8), _P(C.c_int32)]),

@@ -493,6 +493,65 @@ void synth_launch(void* dst, uint64_t seed, uint32_t tensor_id, uint64_t idx0, l
   synth_kernel<<<(unsigned)blocks, 256, 0, s>>>(dst, seed, tensor_id, idx0, n, kind, c);
 }
 
+// ------------------------------------------------------------------ per-shard position tables
+__global__ void rope_table_kernel(float* cosb, float* sinb, int nt, long long i0, int ni, long long wp, int half,
+                                  int d0, int d1, int d2, double theta) {
+  const long long n = (long long)(nt + ni) * half;
+  for (long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x; idx < n;
+       idx += (long long)gridDim.x * blockDim.x) {
+    const long long row = idx / half;
+    const int pair = (int)(idx % half);
+    float c = 1.f, s = 0.f;
+    if (row >= nt) {
+      const long long p = i0 + (row - nt);
+      int a, j, da;
+      if (pair < d0 / 2) { a = 0; j = pair; da = d0; }
+      else if (pair < (d0 + d1) / 2) { a = 1; j = pair - d0 / 2; da = d1; }
+      else { a = 2; j = pair - (d0 + d1) / 2; da = d2; }
+      const double id = a == 0 ? 0.0 : (a == 1 ? (double)(p / wp) : (double)(p % wp));
+      const double ang = id * (1.0 / pow(theta, (2.0 * j) / da));
+      c = (float)cos(ang);
+      s = (float)sin(ang);
+    }
+    cosb[idx] = c;
+    sinb[idx] = s;
+  }
+}
+void rope_table_launch(float* cosb, float* sinb, int nt, long long i0, int ni, long long wp, int D,
+                       const int axes_dim[3], double theta, cudaStream_t s) {
+  const long long n = (long long)(nt + ni) * (D / 2);
+  if (n <= 0) return;
+  const long long blocks = std::min<long long>((n + 255) / 256, 148 * 16);
+  rope_table_kernel<<<(unsigned)blocks, 256, 0, s>>>(cosb, sinb, nt, i0, ni, wp, D / 2, axes_dim[0], axes_dim[1],
+                                                      axes_dim[2], theta);
+}
+
+__global__ void sincos_pe_kernel(float* pe, long long i0, int ni, long long n_c, long long top, long long left,
+                                 double q, int h) {
+  const int quarter = h / 4;
+  const long long n = (long long)ni * quarter;
+  for (long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x; idx < n;
+       idx += (long long)gridDim.x * blockDim.x) {
+    const long long r = idx / quarter;
+    const int j = (int)(idx % quarter);
+    const long long p = i0 + r;
+    const double pr = (double)(p / n_c + top) / q, pc = (double)(p % n_c + left) / q;
+    const double w = 1.0 / pow(10000.0, (double)j / quarter);
+    float* o = pe + r * h;
+    o[j] = (float)sin(pc * w);
+    o[quarter + j] = (float)cos(pc * w);
+    o[2 * quarter + j] = (float)sin(pr * w);
+    o[3 * quarter + j] = (float)cos(pr * w);
+  }
+}
+void sincos_pe_launch(float* pe, long long i0, int ni, long long n_c, long long top, long long left, double q, int h,
+                      cudaStream_t s) {
+  const long long n = (long long)ni * (h / 4);
+  if (n <= 0) return;
+  const long long blocks = std::min<long long>((n + 255) / 256, 148 * 16);
+  sincos_pe_kernel<<<(unsigned)blocks, 256, 0, s>>>(pe, i0, ni, n_c, top, left, q, h);
+}
+
 // ------------------------------------------------------------------ cross-process barrier
 __global__ void ipc_barrier_kernel(const __grid_constant__ IpcBarrier b) {
   grid_dep_wait();

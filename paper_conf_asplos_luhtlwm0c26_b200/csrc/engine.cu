@@ -87,33 +87,63 @@ static inline float bf16_bits_to_f32(uint16_t u) {
 }
 
 // ------------------------------------------------------------------ device buffers
+// Where device memory comes from (tsv_engine_set_allocator): the caller's allocator (e.g. PyTorch's
+// caching allocator), or CUDA.  Buffers are allocated and released *stream-ordered* on the stream
+// that uses them (kind STREAM: cudaMallocAsync / cudaFreeAsync, or the caller's allocator with that
+// stream), so landing and resharding a request never block the host; engine-lifetime buffers
+// (weights, workspaces) are plain allocations (kind STATIC).  IPC windows always use cudaMalloc
+// (kind RAW: cudaIpcGetMemHandle needs an allocation of its own).
+struct Allocator {
+  void* ctx = nullptr;
+  tsv_alloc_fn alloc = nullptr;
+  tsv_free_fn free = nullptr;
+};
+enum AllocKind { AK_STATIC = 0, AK_STREAM = 1, AK_RAW = 2 };
 struct DevBuf {
   void* p = nullptr;
   size_t bytes = 0;
   int device = -1;
+  int kind = AK_STATIC;
+  const Allocator* al = nullptr;   // the caller's allocator (nullptr: CUDA)
+  cudaStream_t stream = nullptr;   // the stream it was allocated on (ordering of the release)
+  // release on the allocation stream; the caller guarantees every use of the buffer is ordered
+  // before the stream's current position (stream-ordered kinds) or has completed (STATIC / RAW)
   void release() {
     if (p) {
       int cur;
       cudaGetDevice(&cur);
       cudaSetDevice(device);
-      cudaFree(p);
+      if (al && kind != AK_RAW) al->free(al->ctx, p, device, stream);
+      else if (kind == AK_STREAM) cudaFreeAsync(p, stream);
+      else cudaFree(p);
       cudaSetDevice(cur);
     }
     p = nullptr;
     bytes = 0;
   }
 };
-static tsv_status dev_alloc(DevBuf& b, int device, size_t bytes) {
+static tsv_status dev_alloc(DevBuf& b, int device, size_t bytes, const Allocator* al = nullptr, int kind = AK_RAW,
+                            cudaStream_t stream = nullptr) {
   if (b.p && b.bytes >= bytes && b.device == device) return TSV_OK;
   b.release();
   if (bytes == 0) return TSV_OK;
   CK(cudaSetDevice(device));
   void* p = nullptr;
-  cudaError_t e = cudaMalloc(&p, bytes);
-  if (e != cudaSuccess) return fail(TSV_E_OOM, "cudaMalloc(%zu) on device %d: %s", bytes, device, cudaGetErrorString(e));
+  if (al && kind != AK_RAW) {
+    p = al->alloc(al->ctx, bytes, device, stream);
+    if (!p) return fail(TSV_E_OOM, "caller allocator returned NULL for %zu bytes on device %d", bytes, device);
+  } else {
+    cudaError_t e = kind == AK_STREAM ? cudaMallocAsync(&p, bytes, stream) : cudaMalloc(&p, bytes);
+    if (e != cudaSuccess)
+      return fail(TSV_E_OOM, "cudaMalloc%s(%zu) on device %d: %s", kind == AK_STREAM ? "Async" : "", bytes, device,
+                  cudaGetErrorString(e));
+  }
   b.p = p;
   b.bytes = bytes;
   b.device = device;
+  b.kind = kind;
+  b.al = al && kind != AK_RAW ? al : nullptr;
+  b.stream = stream;
   return TSV_OK;
 }
 
@@ -187,10 +217,48 @@ static bool splitk_env() {
 }
 
 // per (request, slot): state that depends only on the request
+// Page-locked host memory (inputs and staging of host-computed values): host->device copies from
+// it are truly asynchronous (a pageable source makes cudaMemcpyAsync wait for the stream's prior
+// work before staging).
+template <class T>
+struct Pinned {
+  T* p = nullptr;
+  size_t n = 0;
+  Pinned() = default;
+  Pinned(const Pinned&) = delete;
+  Pinned& operator=(const Pinned&) = delete;
+  Pinned(Pinned&& o) noexcept : p(o.p), n(o.n) { o.p = nullptr; o.n = 0; }
+  Pinned& operator=(Pinned&& o) noexcept {
+    if (this != &o) { reset(); p = o.p; n = o.n; o.p = nullptr; o.n = 0; }
+    return *this;
+  }
+  ~Pinned() { reset(); }
+  void reset() {
+    if (p) cudaFreeHost(p);
+    p = nullptr;
+    n = 0;
+  }
+  tsv_status alloc(size_t count) {
+    reset();
+    if (!count) return TSV_OK;
+    void* q = nullptr;
+    cudaError_t e = cudaHostAlloc(&q, count * sizeof(T), cudaHostAllocPortable);
+    if (e != cudaSuccess) return fail(TSV_E_OOM, "cudaHostAlloc(%zu): %s", count * sizeof(T), cudaGetErrorString(e));
+    p = static_cast<T*>(q);
+    n = count;
+    return TSV_OK;
+  }
+  T* data() { return p; }
+  const T* data() const { return p; }
+  size_t size() const { return n; }
+};
+
 struct ReqDev {
   DevBuf mod;       // fp32 [S * B_model, n_mod]
   DevBuf dt;        // fp32 [S]
   DevBuf step;      // int: the step index the next launch runs
+  Pinned<uint8_t> stage;          // host-computed conditioning inputs until their copies complete
+  cudaEvent_t ready_ev = nullptr; // mod / dt complete (recorded on the slot's stream)
   bool ready = false;
 };
 // per (request, slot, shard): state that depends on the group position
@@ -199,11 +267,10 @@ struct ReqShard {
   int64_t t0 = 0, nt = 0, i0 = 0, ni = 0;  // txt rows [t0, t0+nt), img rows [i0, i0+ni)
   DevBuf lat, vel, T, cosb, sinb;
   DevBuf pe;  // SD3: fp32 [ni, h] sin-cos position embedding of this shard's image rows
-  DevBuf txt;         // fp32 [branches][nt, h]: a1 text embedding T W^T + b (constant per request)
-  bool txt_ok = false;  // txt computed (enqueued) on this shard's stream
+  DevBuf txt;         // fp32 [branches][nt, h]: a1 text embedding T W^T + b (constant per request,
+                      // computed when the shard lands, copied into the residual stream every step)
   void release() {
     lat.release(); vel.release(); T.release(); cosb.release(); sinb.release(); pe.release(); txt.release();
-    txt_ok = false;
   }
 };
 
@@ -221,6 +288,7 @@ struct Group {
   int64_t win_tokens = 0;
   int win_evals = 0;
   DevBuf win_recv, win_cat, win_flags;
+  bool ipc_failed = false;  // the device barrier gave up on a stalled member (check_ipc_barrier)
   std::vector<void*> peer_recv, peer_cat, peer_flags;  // by group rank (own entry = own window)
   std::vector<void*> opened;                           // IPC mappings to close
 };
@@ -233,9 +301,9 @@ struct Request {
   int64_t Li = 0, Lt = 0;
   int next_step = 0;
   int group = -1;
-  std::vector<float> x_host;      // [Li, in] until the first landing
-  std::vector<uint16_t> T_host;   // [B][Lt, ctx] bf16 bits (SD3: branch 0 = T_c, 1 = T_u)
-  std::vector<uint16_t> y_host;   // [B][vec] bf16 bits
+  Pinned<float> x_host;      // [Li, in] until the first landing
+  Pinned<uint16_t> T_host;   // [B][Lt, ctx] bf16 bits (SD3: branch 0 = T_c, 1 = T_u)
+  Pinned<uint16_t> y_host;   // [B][vec] bf16 bits
   std::vector<double> ts;         // t_0..t_S
   std::map<int, ReqDev> dev;      // by slot
   std::map<int, ReqShard> shard;  // by slot (current group)
@@ -245,6 +313,7 @@ struct Request {
 
 struct EventRec {
   std::vector<std::pair<int, cudaEvent_t>> evs;  // (slot, event)
+  int group = -1;                                // the group whose work it marks (-1: none)
 };
 
 }  // namespace tsv
@@ -254,6 +323,11 @@ using namespace tsv;
 struct tsv_engine {
   Model model;
   uint64_t weight_seed = 0;
+  bool inited = false;                       // device state (streams, weights) exists
+  Allocator al;                              // tsv_engine_set_allocator (al.alloc == nullptr: CUDA)
+  std::map<int, cudaStream_t> user_stream;   // tsv_engine_set_stream, by device
+  std::vector<std::pair<cudaGraphExec_t, cudaEvent_t>> dead_graphs;   // dropped, maybe still running
+  const Allocator* alp() const { return al.alloc ? &al : nullptr; }
   bool splitk = true;      // split-K for small fp32-stream GEMM launches (TSV_SPLITK at creation)
   int force_bn = 0, force_pair = -1;   // TSV_GEMM_BN / TSV_GEMM_PAIR (A/B only)
   int rank_base = 0, n_local = 0, world = 0;
@@ -295,6 +369,15 @@ static cudaEvent_t pool_event(tsv_engine* e, int device) {
   cudaEvent_t ev = nullptr;
   cudaEventCreate(&ev);
   return ev;
+}
+
+// Buffers of slot s: engine-lifetime (weights, workspaces) and per-request (stream-ordered on the
+// slot's stream; see DevBuf).
+static tsv_status salloc(tsv_engine* e, DevBuf& b, const Slot& s, size_t bytes) {
+  return dev_alloc(b, s.device, bytes, e->alp(), AK_STATIC, s.stream);
+}
+static tsv_status qalloc(tsv_engine* e, DevBuf& b, const Slot& s, size_t bytes) {
+  return dev_alloc(b, s.device, bytes, e->alp(), AK_STREAM, s.stream);
 }
 
 // Counts one launch of class `cls` (kernels = number of CUDA kernels it launches) and, when
@@ -385,18 +468,18 @@ static GemmEpi epi_of(int mode, void* out0, long long ld0, const bf16* bias, con
 }
 
 // ------------------------------------------------------------------ weights
-static tsv_status init_weights(tsv_engine* e, DeviceState& ds) {
+static tsv_status init_weights(tsv_engine* e, DeviceState& ds, const Slot& s) {
   const Model& m = e->model;
-  TRY(dev_alloc(ds.weights, ds.device, m.total * 2));
+  TRY(salloc(e, ds.weights, s, m.total * 2));
   CK(cudaSetDevice(ds.device));
-  CK(cudaMemset(ds.weights.p, 0, m.total * 2));
+  CK(cudaMemsetAsync(ds.weights.p, 0, m.total * 2, s.stream));
   for (const auto& t : m.tensors) {
     synth_launch(reinterpret_cast<bf16*>(ds.weights.p) + t.offset, e->weight_seed, (uint32_t)t.id, 0, t.numel(),
-                 t.kind, t.c, nullptr);
+                 t.kind, t.c, s.stream);
     e->kernel_count++;  // init-time (not a step kernel)
   }
   CK(cudaGetLastError());
-  CK(cudaDeviceSynchronize());
+  CK(cudaStreamSynchronize(s.stream));
   return TSV_OK;
 }
 
@@ -408,13 +491,34 @@ static tsv_status ensure_reqdev(tsv_engine* e, Request& R, int si) {
   const Model& m = e->model;
   const int h = m.h, S = R.S, B = m.B;
   CK(cudaSetDevice(s.device));
-  TRY(dev_alloc(rd.mod, s.device, (size_t)S * B * m.n_mod * 4));
-  TRY(dev_alloc(rd.dt, s.device, (size_t)S * 4));
-  TRY(dev_alloc(rd.step, s.device, 16));
-  // host-side: sinusoidal embeddings e(t_s), e(g) (fp64 -> bf16), y (bf16), dt.  Row i*B + b is
-  // step i of CFG branch b (SD3: b = 0 conditional, 1 unconditional).
+  const size_t mod_bytes = (size_t)S * B * m.n_mod * 4;
+  TRY(qalloc(e, rd.mod, s, mod_bytes));
+  TRY(qalloc(e, rd.dt, s, (size_t)S * 4));
+  TRY(qalloc(e, rd.step, s, 16));
+  if (!rd.ready_ev) CK(cudaEventCreateWithFlags(&rd.ready_ev, cudaEventDisableTiming));
+  // another rank of this engine already holds the request's table (in-process reshard onto a new
+  // GPU): copy it (85 MB for FLUX at S = 20, a peer copy over NVLink) instead of recomputing it
+  // (which reads the 6.5 GB of modulation weights)
+  for (auto& kv : R.dev) {
+    if (kv.first == si || !kv.second.ready) continue;
+    const Slot& src = e->slots[kv.first];
+    CK(cudaStreamWaitEvent(s.stream, kv.second.ready_ev, 0));
+    CK(cudaMemcpyPeerAsync(rd.mod.p, s.device, kv.second.mod.p, src.device, mod_bytes, s.stream));
+    CK(cudaMemcpyPeerAsync(rd.dt.p, s.device, kv.second.dt.p, src.device, (size_t)S * 4, s.stream));
+    CK(cudaEventRecord(rd.ready_ev, s.stream));
+    rd.ready = true;   // (a ReqDev is only released with its request, after all its copies)
+    return TSV_OK;
+  }
+  // host-side: sinusoidal embeddings e(t_s), e(g) (fp64 -> bf16), y (bf16), dt, staged in pinned
+  // memory owned by rd (the copies stay asynchronous).  Row i*B + b is step i of CFG branch b
+  // (SD3: b = 0 conditional, 1 unconditional).
   const int Sp = S * B;
-  std::vector<uint16_t> et((size_t)Sp * 256), eg((size_t)Sp * 256), ey((size_t)Sp * m.vec);
+  const size_t n_et = (size_t)Sp * 256, n_ey = (size_t)Sp * m.vec;
+  TRY(rd.stage.alloc(2 * (2 * n_et + n_ey) + 4 * (size_t)S));
+  uint16_t* et = reinterpret_cast<uint16_t*>(rd.stage.data());
+  uint16_t* eg = et + n_et;
+  uint16_t* ey = eg + n_et;
+  float* dt = reinterpret_cast<float*>(ey + n_ey);
   auto emb = [](double t, uint16_t* out) {
     for (int j = 0; j < 128; ++j) {
       double f = std::exp(-std::log(10000.0) * j / 128.0);
@@ -423,7 +527,6 @@ static tsv_status ensure_reqdev(tsv_engine* e, Request& R, int si) {
       out[128 + j] = f32_to_bf16_bits((float)std::sin(a));
     }
   };
-  std::vector<float> dt(S);
   for (int i = 0; i < S; ++i) {
     for (int b = 0; b < B; ++b) {
       emb(R.ts[i], &et[(size_t)(i * B + b) * 256]);
@@ -438,12 +541,12 @@ static tsv_status ensure_reqdev(tsv_engine* e, Request& R, int si) {
   const size_t o_vec = (o_hid + (size_t)Sp * h * 2 + 255) & ~size_t(255);
   const size_t o_as = (o_vec + (size_t)Sp * h * 4 + 255) & ~size_t(255);
   const size_t total = o_as + (size_t)Sp * h * 2;
-  TRY(dev_alloc(s.scratch, s.device, total));
+  TRY(salloc(e, s.scratch, s, total));
   uint8_t* sc = reinterpret_cast<uint8_t*>(s.scratch.p);
-  CK(cudaMemcpyAsync(sc + o_et, et.data(), et.size() * 2, cudaMemcpyHostToDevice, s.stream));
-  CK(cudaMemcpyAsync(sc + o_eg, eg.data(), eg.size() * 2, cudaMemcpyHostToDevice, s.stream));
-  CK(cudaMemcpyAsync(sc + o_ey, ey.data(), ey.size() * 2, cudaMemcpyHostToDevice, s.stream));
-  CK(cudaMemcpyAsync(rd.dt.p, dt.data(), S * 4, cudaMemcpyHostToDevice, s.stream));
+  CK(cudaMemcpyAsync(sc + o_et, et, n_et * 2, cudaMemcpyHostToDevice, s.stream));
+  CK(cudaMemcpyAsync(sc + o_eg, eg, n_et * 2, cudaMemcpyHostToDevice, s.stream));
+  CK(cudaMemcpyAsync(sc + o_ey, ey, n_ey * 2, cudaMemcpyHostToDevice, s.stream));
+  CK(cudaMemcpyAsync(rd.dt.p, dt, S * 4, cudaMemcpyHostToDevice, s.stream));
   bf16* hid = reinterpret_cast<bf16*>(sc + o_hid);
   float* vec = reinterpret_cast<float*>(sc + o_vec);
   bf16* as = reinterpret_cast<bf16*>(sc + o_as);
@@ -469,58 +572,16 @@ static tsv_status ensure_reqdev(tsv_engine* e, Request& R, int si) {
   TRY(gemm(e, s, as, h, wb + m.modw_off, h, Sp, (int)m.n_mod, h,
            epi_of(EPI_STORE_F32, rd.mod.p, m.n_mod, wb + m.modb_off)));
   CK(cudaGetLastError());
+  CK(cudaEventRecord(rd.ready_ev, s.stream));
   rd.ready = true;
   return TSV_OK;
 }
 
-// RoPE tables for the rows of one shard (fp64 angles -> fp32 cos/sin, S22)
-static void rope_rows(const Model& m, const Request& R, int64_t t0, int64_t nt, int64_t i0, int64_t ni,
-                      std::vector<float>& c, std::vector<float>& s) {
-  const int half = m.D / 2;
-  c.assign((size_t)(nt + ni) * half, 1.0f);
-  s.assign((size_t)(nt + ni) * half, 0.0f);
-  const int64_t wp = R.width / 16;
-  for (int64_t r = 0; r < ni; ++r) {
-    const int64_t p = i0 + r;
-    const double ids[3] = {0.0, (double)(p / wp), (double)(p % wp)};
-    int pair = 0;
-    for (int a = 0; a < 3; ++a) {
-      const int da = m.d.axes_dim[a];
-      for (int j = 0; j < da / 2; ++j, ++pair) {
-        const double omega = 1.0 / std::pow((double)m.d.theta, (2.0 * j) / da);
-        const double ang = ids[a] * omega;
-        c[(size_t)(nt + r) * half + pair] = (float)std::cos(ang);
-        s[(size_t)(nt + r) * half + pair] = (float)std::sin(ang);
-      }
-    }
-  }
-}
-
-// SD3 2-D sin-cos position embedding of image rows [i0, i0 + ni) (fp64 -> fp32; DESIGN.md O-SD3,
-// S13): patch (r, c) of the n_r x n_c grid sits at ((r + top) / q, (c + left) / q), q = pe_max /
-// pe_base, top = floor((pe_max - n_r) / 2); channels [sin(c' w), cos(c' w), sin(r' w), cos(r' w)]
-// with w_j = 10000^(-j / (h/4)).
-static void pos_embed_rows(const Model& m, const Request& R, int64_t i0, int64_t ni, std::vector<float>& pe) {
-  const int64_t n_r = R.height / 16, n_c = R.width / 16;
-  const int quarter = m.h / 4;
-  auto floordiv2 = [](int64_t a) { return a >= 0 ? a / 2 : -((-a + 1) / 2); };
-  const int64_t top = floordiv2(m.d.pe_max - n_r), left = floordiv2(m.d.pe_max - n_c);
-  const double q = (double)m.d.pe_max / m.d.pe_base;
-  pe.assign((size_t)ni * m.h, 0.f);
-  for (int64_t r = 0; r < ni; ++r) {
-    const int64_t p = i0 + r;
-    const double pr = (double)(p / n_c + top) / q, pc = (double)(p % n_c + left) / q;
-    float* o = &pe[(size_t)r * m.h];
-    for (int j = 0; j < quarter; ++j) {
-      const double w = 1.0 / std::pow(10000.0, (double)j / quarter);
-      o[j] = (float)std::sin(pc * w);
-      o[quarter + j] = (float)std::cos(pc * w);
-      o[2 * quarter + j] = (float)std::sin(pr * w);
-      o[3 * quarter + j] = (float)std::cos(pr * w);
-    }
-  }
-}
-
+// Per-request state of one shard on its slot, all enqueued on the slot's stream (no host wait):
+// buffers (stream-ordered), the text rows T (pinned host -> device), the RoPE cos/sin tables
+// (FLUX; fp64 angles -> fp32, S22) or the SD3 sin-cos position embedding (S13) computed on the
+// device, and the a1 text embedding txt = T W_txt^T + b of the shard's text rows (constant per
+// request: computed here once, copied into the residual stream by every step).
 static tsv_status setup_shard(tsv_engine* e, Request& R, int si, int rank_in_group, int k, ReqShard& sh) {
   Slot& s = e->slots[si];
   const Model& m = e->model;
@@ -531,11 +592,10 @@ static tsv_status setup_shard(tsv_engine* e, Request& R, int si, int rank_in_gro
   sh.i0 = shard_begin(R.Li, k, rank_in_group);
   sh.ni = shard_begin(R.Li, k, rank_in_group + 1) - sh.i0;
   CK(cudaSetDevice(s.device));
-  TRY(dev_alloc(sh.lat, s.device, std::max<size_t>(1, sh.ni) * m.in * 4));
-  TRY(dev_alloc(sh.vel, s.device, std::max<size_t>(1, sh.ni) * m.in * 4));
-  TRY(dev_alloc(sh.T, s.device, std::max<size_t>(1, sh.nt) * m.B * m.ctx * 2));
-  TRY(dev_alloc(sh.txt, s.device, std::max<size_t>(1, sh.nt) * m.B * m.h * 4));
-  sh.txt_ok = false;
+  TRY(qalloc(e, sh.lat, s, std::max<size_t>(1, sh.ni) * m.in * 4));
+  TRY(qalloc(e, sh.vel, s, std::max<size_t>(1, sh.ni) * m.in * 4));
+  TRY(qalloc(e, sh.T, s, std::max<size_t>(1, sh.nt) * m.B * m.ctx * 2));
+  TRY(qalloc(e, sh.txt, s, std::max<size_t>(1, sh.nt) * m.B * m.h * 4));
   const size_t rows = sh.nt + sh.ni;
   if (sh.nt)
     for (int b = 0; b < m.B; ++b)
@@ -543,24 +603,29 @@ static tsv_status setup_shard(tsv_engine* e, Request& R, int si, int rank_in_gro
                          R.T_host.data() + ((size_t)b * R.Lt + sh.t0) * m.ctx, sh.nt * m.ctx * 2,
                          cudaMemcpyHostToDevice, s.stream));
   if (m.sd3) {
-    std::vector<float> pe;
-    pos_embed_rows(m, R, sh.i0, sh.ni, pe);
-    TRY(dev_alloc(sh.pe, s.device, std::max<size_t>(1, sh.ni) * m.h * 4));
-    if (sh.ni) {
-      CK(cudaMemcpyAsync(sh.pe.p, pe.data(), pe.size() * 4, cudaMemcpyHostToDevice, s.stream));
-      CK(cudaStreamSynchronize(s.stream));
-    }
-    return TSV_OK;
+    TRY(qalloc(e, sh.pe, s, std::max<size_t>(1, sh.ni) * m.h * 4));
+    // patch (r, c) of the n_r x n_c grid sits at ((r + top) / q, (c + left) / q), q = pe_max / pe_base,
+    // top = floor((pe_max - n_r) / 2) (floor toward -inf, S13)
+    const int64_t n_r = R.height / 16, n_c = R.width / 16;
+    auto floordiv2 = [](int64_t a) { return a >= 0 ? a / 2 : -((-a + 1) / 2); };
+    ProfScope ps(e, s, KC_OTHER, 0.0, (double)sh.ni * m.h * 4.0);
+    sincos_pe_launch(reinterpret_cast<float*>(sh.pe.p), sh.i0, (int)sh.ni, n_c, floordiv2(m.d.pe_max - n_r),
+                     floordiv2(m.d.pe_max - n_c), (double)m.d.pe_max / m.d.pe_base, m.h, s.stream);
+  } else {
+    TRY(qalloc(e, sh.cosb, s, std::max<size_t>(1, rows) * (m.D / 2) * 4));
+    TRY(qalloc(e, sh.sinb, s, std::max<size_t>(1, rows) * (m.D / 2) * 4));
+    ProfScope ps(e, s, KC_OTHER, 0.0, (double)rows * m.D * 4.0);
+    rope_table_launch(reinterpret_cast<float*>(sh.cosb.p), reinterpret_cast<float*>(sh.sinb.p), (int)sh.nt, sh.i0,
+                      (int)sh.ni, R.width / 16, m.D, m.d.axes_dim, (double)m.d.theta, s.stream);
   }
-  TRY(dev_alloc(sh.cosb, s.device, std::max<size_t>(1, rows) * (m.D / 2) * 4));
-  TRY(dev_alloc(sh.sinb, s.device, std::max<size_t>(1, rows) * (m.D / 2) * 4));
-  std::vector<float> c, sn;
-  rope_rows(m, R, sh.t0, sh.nt, sh.i0, sh.ni, c, sn);
-  if (rows) {
-    CK(cudaMemcpyAsync(sh.cosb.p, c.data(), c.size() * 4, cudaMemcpyHostToDevice, s.stream));
-    CK(cudaMemcpyAsync(sh.sinb.p, sn.data(), sn.size() * 4, cudaMemcpyHostToDevice, s.stream));
-    CK(cudaStreamSynchronize(s.stream));  // host vectors go out of scope
+  if (sh.nt) {
+    GemmProblem pt[GEMM_MAX_PROBLEMS];
+    for (int b = 0; b < m.B; ++b)
+      pt[b] = {reinterpret_cast<bf16*>(sh.T.p) + b * sh.nt * m.ctx, m.ctx, e->W(s, 2), m.ctx, (int)sh.nt,
+               epi_of(EPI_STORE_F32, reinterpret_cast<float*>(sh.txt.p) + b * sh.nt * m.h, m.h, e->W(s, 3))};
+    TRY(gemm_multi(e, s, pt, m.B, m.h, m.ctx));
   }
+  CK(cudaGetLastError());
   return TSV_OK;
 }
 
@@ -571,18 +636,18 @@ static tsv_status ensure_workspace(tsv_engine* e, Slot& s, int64_t rows, int64_t
   Workspace& w = s.ws;
   const int64_t r1 = std::max<int64_t>(rows, 1);
   const int64_t r = r1 * B;  // every activation buffer holds the B evaluations back to back
-  TRY(dev_alloc(w.x, s.device, r * h * 4));
-  TRY(dev_alloc(w.u, s.device, r * h * 2));
-  TRY(dev_alloc(w.qkv, s.device, r * 3 * h * 2));
-  TRY(dev_alloc(w.cat, s.device, r * (h + F) * 2));
-  TRY(dev_alloc(w.hbuf, s.device, r * F * 2));
-  TRY(dev_alloc(w.latb, s.device, r * m.in * 2));
-  TRY(dev_alloc(w.bmod, s.device, ((size_t)B * m.n_mod + 64) * 4));
+  TRY(salloc(e, w.x, s, r * h * 4));
+  TRY(salloc(e, w.u, s, r * h * 2));
+  TRY(salloc(e, w.qkv, s, r * 3 * h * 2));
+  TRY(salloc(e, w.cat, s, r * (h + F) * 2));
+  TRY(salloc(e, w.hbuf, s, r * F * 2));
+  TRY(salloc(e, w.latb, s, r * m.in * 2));
+  TRY(salloc(e, w.bmod, s, ((size_t)B * m.n_mod + 64) * 4));
   if (k > 1) {
-    TRY(dev_alloc(w.pack, s.device, r * 3 * h * 2));
-    TRY(dev_alloc(w.recv, s.device, B * L * 3 * (h / k) * 2));
-    TRY(dev_alloc(w.obuf, s.device, B * L * (h / k) * 2));
-    TRY(dev_alloc(w.orecv, s.device, r * h * 2));
+    TRY(salloc(e, w.pack, s, r * 3 * h * 2));
+    TRY(salloc(e, w.recv, s, B * L * 3 * (h / k) * 2));
+    TRY(salloc(e, w.obuf, s, B * L * (h / k) * 2));
+    TRY(salloc(e, w.orecv, s, r * h * 2));
   }
   return TSV_OK;
 }
@@ -867,28 +932,16 @@ static void select_rows(StepEnv& E, RankCtx& c) {
 }
 
 
-// a1 text embedding txt = T W_txt^T + b: constant per (request, shard), so it is computed on the
-// shard's first step into sh.txt and copied into the residual stream rows [b R, b R + nt) on every
-// step (a 4 x ctx/h smaller copy instead of an M = nt, K = 4096 weight-streaming GEMM).  per_req =
-// evaluations per request (1 FLUX, 2 SD3 CFG branches; branch br uses T rows br * nt).
+// a1 text embedding: the shard's txt = T W_txt^T + b was computed when it landed (setup_shard); every
+// step copies it into the residual stream rows [b R, b R + nt) of evaluation b (a 4 x ctx/h smaller
+// copy instead of an M = nt, K = 4096 weight-streaming GEMM).  per_req = evaluations per request
+// (1 FLUX, 2 SD3 CFG branches; branch br uses txt rows br * nt).
 static tsv_status txt_embed(tsv_engine* e, Slot& s, const std::vector<ReqShard*>& shq, float* x, int64_t R, int64_t nt,
                             int B, int per_req) {
   if (!nt) return TSV_OK;
-  const Model& m = e->model;
-  const int h = m.h;
-  GemmProblem pt[GEMM_MAX_PROBLEMS];
-  int n = 0;
+  const int h = e->model.h;
   for (int b = 0; b < B; ++b) {
     ReqShard* sh = shq[b / per_req];
-    const int br = b % per_req;
-    if (!sh->txt_ok)
-      pt[n++] = {reinterpret_cast<bf16*>(sh->T.p) + br * nt * m.ctx, m.ctx, e->W(s, 2), m.ctx, (int)nt,
-                 epi_of(EPI_STORE_F32, reinterpret_cast<float*>(sh->txt.p) + br * nt * h, h, e->W(s, 3))};
-  }
-  if (n) TRY(gemm_multi(e, s, pt, n, h, m.ctx));
-  for (int b = 0; b < B; ++b) {
-    ReqShard* sh = shq[b / per_req];
-    sh->txt_ok = true;
     CK(cudaMemcpyAsync(x + b * R * h, reinterpret_cast<float*>(sh->txt.p) + (b % per_req) * nt * h,
                        nt * h * sizeof(float), cudaMemcpyDeviceToDevice, s.stream));
   }
@@ -1196,13 +1249,25 @@ static tsv_status record_last(tsv_engine* e, Request& R, int si) {
   return TSV_OK;
 }
 
-// Move the request to group gi.  First landing: latent rows come from the host inputs.
+static void drop_request_graphs(tsv_engine* e, int64_t id);
+
+// Move the request to group gi (a13).  First landing: latent rows come from the pinned
+// host inputs.  Otherwise bit-exact row moves old shard -> new shard by the reshard map, each copy
+// ordered after the request's last work on its source rank.  Nothing here waits on the host: the
+// new shards' state is enqueued on their streams (setup_shard, ensure_reqdev), and the old shards
+// are released stream-ordered on their own streams after every copy that reads them.
 static tsv_status move_request(tsv_engine* e, Request& R, int gi) {
   Group& g = e->groups[gi];
   const Model& m = e->model;
   std::map<int, ReqShard> next;
   for (size_t q = 0; q < g.local_slots.size(); ++q) {
     const int si = g.local_slots[q];
+    Slot& s = e->slots[si];
+    CK(cudaSetDevice(s.device));
+    // the new rank's stream follows the request's previous work there (its shard buffers may reuse
+    // memory the old shard on this slot still reads)
+    auto it = R.last.find(si);
+    if (it != R.last.end()) CK(cudaStreamWaitEvent(s.stream, it->second, 0));
     TRY(setup_shard(e, R, si, g.local_positions[q], g.k, next[si]));
     TRY(ensure_reqdev(e, R, si));
   }
@@ -1214,7 +1279,6 @@ static tsv_status move_request(tsv_engine* e, Request& R, int gi) {
       if (sh.ni)
         CK(cudaMemcpyAsync(sh.lat.p, R.x_host.data() + sh.i0 * m.in, sh.ni * m.in * 4, cudaMemcpyHostToDevice,
                            s.stream));
-      CK(cudaStreamSynchronize(s.stream));
     }
   } else {
     Group& og = e->groups[R.group];
@@ -1264,10 +1328,17 @@ static tsv_status move_request(tsv_engine* e, Request& R, int gi) {
         }
       }
     }
-    // old buffers: wait until every copy finished before freeing
+    // the old shards' buffers: released on their own streams once every new rank's copies (which
+    // read them) are done -- stream-ordered, the host never waits
     for (auto& kv : next) TRY(record_last(e, R, kv.first));
-    for (auto& kv : next) CK(cudaEventSynchronize(R.last[kv.first]));
-    for (auto& kv : R.shard) kv.second.release();
+    for (auto& kv : R.shard) {
+      Slot& os = e->slots[kv.first];
+      CK(cudaSetDevice(os.device));
+      for (auto& nk : next)
+        if (nk.first != kv.first) CK(cudaStreamWaitEvent(os.stream, R.last[nk.first], 0));
+      kv.second.release();
+    }
+    drop_request_graphs(e, R.id);   // cached step graphs reference the old shards' buffers
   }
   R.shard.swap(next);
   R.group = gi;
@@ -1276,8 +1347,9 @@ static tsv_status move_request(tsv_engine* e, Request& R, int gi) {
   return TSV_OK;
 }
 
-static tsv_status new_event(tsv_engine* e, const std::vector<int>& slots_, tsv_event* out) {
+static tsv_status new_event(tsv_engine* e, const std::vector<int>& slots_, tsv_event* out, int gi = -1) {
   EventRec rec;
+  rec.group = gi;
   for (int si : slots_) {
     Slot& s = e->slots[si];
     CK(cudaSetDevice(s.device));
@@ -1291,9 +1363,37 @@ static tsv_status new_event(tsv_engine* e, const std::vector<int>& slots_, tsv_e
   return TSV_OK;
 }
 
-static void drop_graph(StepGraph& gr) {
-  if (gr.exec) cudaGraphExecDestroy(gr.exec);
+// A dropped step graph may still be executing (its last replay is in flight on the slot's stream):
+// it is destroyed once an event recorded behind that replay has completed (sweep_graphs), so that
+// dropping never waits on the device.
+static void drop_graph(tsv_engine* e, Slot& s, StepGraph& gr) {
+  if (!gr.exec) return;
+  cudaEvent_t ev = nullptr;
+  cudaSetDevice(s.device);
+  if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) == cudaSuccess &&
+      cudaEventRecord(ev, s.stream) == cudaSuccess) {
+    e->dead_graphs.push_back({gr.exec, ev});
+  } else {   // cannot defer: wait for the slot's work, then destroy
+    if (ev) cudaEventDestroy(ev);
+    cudaStreamSynchronize(s.stream);
+    cudaGraphExecDestroy(gr.exec);
+  }
   gr.exec = nullptr;
+}
+static void sweep_graphs(tsv_engine* e, bool all) {
+  for (size_t i = 0; i < e->dead_graphs.size();) {
+    auto& d = e->dead_graphs[i];
+    if (all || cudaEventQuery(d.second) == cudaSuccess) {
+      if (all) cudaEventSynchronize(d.second);
+      cudaGraphExecDestroy(d.first);
+      cudaEventDestroy(d.second);
+      d = e->dead_graphs.back();
+      e->dead_graphs.pop_back();
+    } else {
+      cudaGetLastError();   // clear cudaErrorNotReady
+      ++i;
+    }
+  }
 }
 
 // One step of every request in Rs (each at its own next step) as one batched step on group gi.
@@ -1305,6 +1405,7 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
     for (Request* R : Rs) R->next_step++;
     return TSV_OK;
   }
+  sweep_graphs(e, false);
   for (Request* R : Rs)
     if (R->group != gi) TRY(move_request(e, *R, gi));
   const Model& m = e->model;
@@ -1390,7 +1491,6 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
                             rd->step.p};
         for (const void* p : rp) mix(reinterpret_cast<uintptr_t>(p));
         mix((uint64_t)Rs[q]->id);
-        mix((uint64_t)sh->txt_ok);   // the first step on a shard also computes the text embedding
       }
       mix((uint64_t)c.rows);
       mix((uint64_t)c.si);
@@ -1406,7 +1506,7 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
         auto lru = slot.graphs.begin();
         for (auto jt = slot.graphs.begin(); jt != slot.graphs.end(); ++jt)
           if (jt->second.last_use < lru->second.last_use) lru = jt;
-        drop_graph(lru->second);
+        drop_graph(e, slot, lru->second);
         slot.graphs.erase(lru);
       }
       CK(cudaSetDevice(slot.device));
@@ -1460,7 +1560,7 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
     R->next_step++;
     R->has_velocity = true;
   }
-  if (done) TRY(new_event(e, g.local_slots, done));
+  if (done) TRY(new_event(e, g.local_slots, done, gi));
   return TSV_OK;
 }
 
@@ -1468,6 +1568,10 @@ static void release_reqdev(ReqDev& d) {
   d.mod.release();
   d.dt.release();
   d.step.release();
+  if (d.ready_ev) cudaEventDestroy(d.ready_ev);
+  d.ready_ev = nullptr;
+  d.stage.reset();
+  d.ready = false;
 }
 
 // drop every cached step graph that references request `id` (its buffers are about to be freed)
@@ -1476,7 +1580,7 @@ static void drop_request_graphs(tsv_engine* e, int64_t id) {
     for (auto it = s.graphs.begin(); it != s.graphs.end();) {
       const auto& r = it->second.reqs;
       if (std::find(r.begin(), r.end(), id) != r.end()) {
-        drop_graph(it->second);
+        drop_graph(e, s, it->second);
         it = s.graphs.erase(it);
       } else {
         ++it;
@@ -1536,19 +1640,21 @@ tsv_status tsv_engine_create(const tsv_model_desc* model, const int* devices, in
   e->world = world_size;
   e->slots.resize(n_local);
   for (int i = 0; i < n_local; ++i) {
+    e->slots[i].rank = rank_base + i;
+    e->slots[i].device = devices[i];
+  }
+  *out = e.release();
+  return TSV_OK;
+}
+
+// Device state, created on first use (after the optional allocator / stream hooks): per slot a
+// stream (the caller's for its device, else an engine-owned non-blocking one), the device's weights,
+// split-K counters and workspace; peer access (and memory-pool access for the stream-ordered
+// per-request buffers) between the engine's distinct devices.
+static tsv_status ensure_init(tsv_engine* e) {
+  if (e->inited) return TSV_OK;
+  for (int i = 0; i < e->n_local; ++i) {
     Slot& s = e->slots[i];
-    s.rank = rank_base + i;
-    s.device = devices[i];
-    auto it = e->devs.find(s.device);
-    if (it == e->devs.end()) {
-      auto ds = std::make_unique<DeviceState>();
-      ds->device = s.device;
-      CK(cudaSetDevice(s.device));
-      CK(cudaDeviceGetAttribute(&ds->num_sms, cudaDevAttrMultiProcessorCount, s.device));
-      TRY(init_weights(e.get(), *ds));
-      it = e->devs.emplace(s.device, std::move(ds)).first;
-    }
-    s.ds = it->second.get();
     CK(cudaSetDevice(s.device));
     // TSV_VIRTUAL_SERIAL=1: virtual ranks on one device share one stream, so every kernel runs alone
     // on the GPU as it would on a rank's own GPU (per-rank timing of k > 1 on one device); default:
@@ -1557,17 +1663,38 @@ tsv_status tsv_engine_create(const tsv_model_desc* model, const int* devices, in
     Slot* first = nullptr;
     for (int j = 0; j < i; ++j)
       if (e->slots[j].device == s.device) { first = &e->slots[j]; break; }
-    if (vs && atoi(vs) && first) {
+    auto us = e->user_stream.find(s.device);
+    if (us != e->user_stream.end()) {
+      s.stream = us->second;
+      s.own_stream = false;
+    } else if (vs && atoi(vs) && first) {
       s.stream = first->stream;
       s.own_stream = false;
     } else {
       CK(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+      s.own_stream = true;
     }
-    TRY(dev_alloc(s.sem, s.device, SEM_INTS * sizeof(int)));
-    CK(cudaMemset(s.sem.p, 0, SEM_INTS * sizeof(int)));
-    TRY(dev_alloc(s.splitws, s.device, SPLIT_WS_BYTES));
+    auto it = e->devs.find(s.device);
+    if (it == e->devs.end()) {
+      auto ds = std::make_unique<DeviceState>();
+      ds->device = s.device;
+      CK(cudaDeviceGetAttribute(&ds->num_sms, cudaDevAttrMultiProcessorCount, s.device));
+      // stream-ordered pool of the per-request buffers: keep freed memory cached (no release to
+      // the OS at synchronisation points)
+      cudaMemPool_t pool;
+      CK(cudaDeviceGetDefaultMemPool(&pool, s.device));
+      uint64_t keep = UINT64_MAX;
+      CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep));
+      TRY(init_weights(e, *ds, s));
+      it = e->devs.emplace(s.device, std::move(ds)).first;
+    }
+    s.ds = it->second.get();
+    TRY(salloc(e, s.sem, s, SEM_INTS * sizeof(int)));
+    CK(cudaMemsetAsync(s.sem.p, 0, SEM_INTS * sizeof(int), s.stream));
+    TRY(salloc(e, s.splitws, s, SPLIT_WS_BYTES));
   }
-  // peer access between distinct local devices (in-process all-to-all and reshard)
+  // peer access between distinct local devices (in-process all-to-all and reshard), also for the
+  // stream-ordered pools
   for (auto& a : e->devs)
     for (auto& b : e->devs) {
       if (a.first == b.first) continue;
@@ -1578,20 +1705,55 @@ tsv_status tsv_engine_create(const tsv_model_desc* model, const int* devices, in
         cudaError_t r = cudaDeviceEnablePeerAccess(b.first, 0);
         if (r != cudaSuccess && r != cudaErrorPeerAccessAlreadyEnabled) return fail(TSV_E_CUDA, "peer access");
         cudaGetLastError();
+        cudaMemPool_t pool;
+        CK(cudaDeviceGetDefaultMemPool(&pool, b.first));
+        cudaMemAccessDesc d{};
+        d.location.type = cudaMemLocationTypeDevice;
+        d.location.id = a.first;
+        d.flags = cudaMemAccessFlagsProtReadWrite;
+        CK(cudaMemPoolSetAccess(pool, &d, 1));   // device a may access b's pool allocations
       }
     }
-  *out = e.release();
+  for (auto& s : e->slots) {
+    CK(cudaSetDevice(s.device));
+    CK(cudaStreamSynchronize(s.stream));
+  }
+  e->inited = true;
+  return TSV_OK;
+}
+
+tsv_status tsv_engine_set_allocator(tsv_engine* e, void* ctx, tsv_alloc_fn alloc_fn, tsv_free_fn free_fn) {
+  if (!e || !alloc_fn || !free_fn) return fail(TSV_E_INVAL, "null argument");
+  if (e->inited) return fail(TSV_E_STATE, "the allocator must be set before the engine's first group");
+  e->al.ctx = ctx;
+  e->al.alloc = alloc_fn;
+  e->al.free = free_fn;
+  return TSV_OK;
+}
+
+tsv_status tsv_engine_set_stream(tsv_engine* e, int device, void* cuda_stream) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  if (e->inited) return fail(TSV_E_STATE, "streams must be set before the engine's first group");
+  bool found = false;
+  for (auto& s : e->slots) found = found || s.device == device;
+  if (!found) return fail(TSV_E_INVAL, "device %d hosts no rank of this engine", device);
+  e->user_stream[device] = reinterpret_cast<cudaStream_t>(cuda_stream);
   return TSV_OK;
 }
 
 void tsv_engine_destroy(tsv_engine* e) {
   if (!e) return;
+  if (!e->inited) {   // no device state: requests hold only pinned host memory
+    delete e;
+    return;
+  }
   for (auto& s : e->slots) {
     cudaSetDevice(s.device);
     cudaStreamSynchronize(s.stream);
   }
   for (auto& s : e->slots)
-    for (auto& kv : s.graphs) drop_graph(kv.second);
+    for (auto& kv : s.graphs) drop_graph(e, s, kv.second);
+  sweep_graphs(e, true);
   for (auto& kv : e->requests) {
     for (auto& d : kv.second.dev) release_reqdev(d.second);
     for (auto& sh : kv.second.shard) sh.second.release();
@@ -1650,6 +1812,7 @@ tsv_status tsv_group_create(tsv_engine* e, const int* ranks, int k, const uint8_
   }
   if (e->model.H % k) return fail(TSV_E_UNSUPPORTED, "k = %d does not divide the head count %d (S24)", k, e->model.H);
   if ((e->model.h / k) % 64) return fail(TSV_E_UNSUPPORTED, "hidden/k must be a multiple of 64");
+  TRY(ensure_init(e));
   Group g;
   g.ranks.assign(ranks, ranks + k);
   g.k = k;
@@ -1799,16 +1962,17 @@ tsv_status tsv_request_create(tsv_engine* e, int height, int width, int num_step
   R.height = height; R.width = width; R.S = num_steps; R.seed = seed; R.guidance = guidance;
   R.Li = (int64_t)(height / 16) * (width / 16);
   R.Lt = m.Lt;
-  R.x_host.resize((size_t)R.Li * m.in);
-  for (size_t i = 0; i < R.x_host.size(); ++i) R.x_host[i] = synth_r(seed, 1, i) * synth_scale(1.0);
+  // inputs live in pinned host memory: the first landing's copies do not wait on the device
+  TRY(R.x_host.alloc((size_t)R.Li * m.in));
+  for (size_t i = 0; i < R.x_host.size(); ++i) R.x_host.p[i] = synth_r(seed, 1, i) * synth_scale(1.0);
   // T, y of evaluation b: SYNTH-1 ids (2, 3) for b = 0 and (4, 5) for SD3's unconditional b = 1
   const size_t nT = (size_t)R.Lt * m.ctx;
   const float c1 = synth_scale(1.0);
-  R.T_host.resize(nT * m.B);
-  R.y_host.resize((size_t)m.vec * m.B);
+  TRY(R.T_host.alloc(nT * m.B));
+  TRY(R.y_host.alloc((size_t)m.vec * m.B));
   for (int b = 0; b < m.B; ++b) {
-    for (size_t i = 0; i < nT; ++i) R.T_host[b * nT + i] = f32_to_bf16_bits(synth_r(seed, 2 + 2 * b, i) * c1);
-    for (int i = 0; i < m.vec; ++i) R.y_host[(size_t)b * m.vec + i] = f32_to_bf16_bits(synth_r(seed, 3 + 2 * b, i) * c1);
+    for (size_t i = 0; i < nT; ++i) R.T_host.p[b * nT + i] = f32_to_bf16_bits(synth_r(seed, 2 + 2 * b, i) * c1);
+    for (int i = 0; i < m.vec; ++i) R.y_host.p[(size_t)b * m.vec + i] = f32_to_bf16_bits(synth_r(seed, 3 + 2 * b, i) * c1);
   }
   R.ts.resize(num_steps + 1);
   if (m.sd3) {
@@ -1888,14 +2052,32 @@ tsv_status tsv_request_reshard(tsv_engine* e, tsv_request r, tsv_group gi, tsv_e
   if (!R) return fail(TSV_E_INVAL, "unknown request %lld", (long long)r);
   if (gi < 0 || gi >= (int)e->groups.size()) return fail(TSV_E_INVAL, "unknown group %d", gi);
   if (R->group != gi) TRY(move_request(e, *R, gi));
-  if (done) TRY(new_event(e, e->groups[gi].local_slots, done));
+  if (done) TRY(new_event(e, e->groups[gi].local_slots, done, gi));
   return TSV_OK;
 }
 
 tsv_status tsv_group_record(tsv_engine* e, tsv_group gi, tsv_event* out) {
   if (!e || !out) return fail(TSV_E_INVAL, "null argument");
   if (gi < 0 || gi >= (int)e->groups.size()) return fail(TSV_E_INVAL, "unknown group %d", gi);
-  return new_event(e, e->groups[gi].local_slots, out);
+  return new_event(e, e->groups[gi].local_slots, out, gi);
+}
+
+// A group over CUDA-IPC windows: did its device barrier give up on a stalled member (flag 62 of this
+// rank's window, set by ipc_barrier_kernel)?  Called once the event's work completed.
+static tsv_status check_ipc_barrier(tsv_engine* e, int gi) {
+  if (gi < 0 || gi >= (int)e->groups.size()) return TSV_OK;
+  Group& g = e->groups[gi];
+  if (!g.ipc || !g.win_flags.p) return TSV_OK;
+  if (!g.ipc_failed) {
+    int flag = 0;
+    CK(cudaSetDevice(g.win_flags.device));
+    CK(cudaMemcpy(&flag, reinterpret_cast<int*>(g.win_flags.p) + 62, sizeof(int), cudaMemcpyDeviceToHost));
+    g.ipc_failed = flag != 0;
+  }
+  if (g.ipc_failed)
+    return fail(TSV_E_STATE, "group %d: the cross-process barrier timed out waiting for a member (~10 s); the "
+                "step's results are invalid and the group must be recreated", gi);
+  return TSV_OK;
 }
 
 tsv_status tsv_event_wait(tsv_engine* e, tsv_event ev) {
@@ -1903,7 +2085,7 @@ tsv_status tsv_event_wait(tsv_engine* e, tsv_event ev) {
   if (ev == -1) return TSV_OK;
   if (ev < 0 || ev >= (int64_t)e->events.size()) return fail(TSV_E_INVAL, "unknown event");
   for (auto& p : e->events[ev].evs) CK(cudaEventSynchronize(p.second));
-  return TSV_OK;
+  return check_ipc_barrier(e, e->events[ev].group);
 }
 
 tsv_status tsv_event_query(tsv_engine* e, tsv_event ev, int* done) {
@@ -1916,7 +2098,7 @@ tsv_status tsv_event_query(tsv_engine* e, tsv_event ev, int* done) {
     if (q == cudaErrorNotReady) { *done = 0; cudaGetLastError(); }
     else if (q != cudaSuccess) return fail(TSV_E_CUDA, "event query: %s", cudaGetErrorString(q));
   }
-  return TSV_OK;
+  return *done ? check_ipc_barrier(e, e->events[ev].group) : TSV_OK;
 }
 
 tsv_status tsv_event_elapsed_ms(tsv_engine* e, tsv_event a, tsv_event b, float* ms) {
@@ -1935,7 +2117,8 @@ tsv_status tsv_event_elapsed_ms(tsv_engine* e, tsv_event a, tsv_event b, float* 
     mx = std::max(mx, t);
   }
   *ms = mx;
-  return TSV_OK;
+  TRY(check_ipc_barrier(e, e->events[a].group));
+  return check_ipc_barrier(e, e->events[b].group);
 }
 
 static tsv_status latent_io(tsv_engine* e, tsv_request r, int64_t row0, int64_t nrows, float* host, bool write,
@@ -2115,6 +2298,7 @@ tsv_status tsv_debug_read_weight(tsv_engine* e, int id, uint16_t* host, size_t n
   const TensorInfo* t = e->model.find(id);
   if (!t) return fail(TSV_E_INVAL, "unknown tensor id %d", id);
   if (n != (size_t)t->numel()) return fail(TSV_E_INVAL, "tensor %d has %lld elements", id, (long long)t->numel());
+  TRY(ensure_init(e));
   Slot& s = e->slots[0];
   CK(cudaSetDevice(s.device));
   CK(cudaMemcpy(host, reinterpret_cast<const bf16*>(s.ds->weights.p) + t->offset, n * 2, cudaMemcpyDeviceToHost));

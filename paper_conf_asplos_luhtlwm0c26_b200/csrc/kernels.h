@@ -207,6 +207,19 @@ struct IpcBarrier {
 };
 void ipc_barrier_launch(const IpcBarrier& b, cudaStream_t s);
 
+// ------------------------------------------------------------------ per-shard position tables
+// FLUX RoPE tables (S22: angles in fp64, stored fp32) of one shard's rows [txt (nt) ; img (ni)]:
+// cos/sin [nt + ni, D/2]; text rows are position 0 (cos 1, sin 0); image row r is token
+// p = i0 + r at (row p / wp, col p % wp) of the patch grid; pair i belongs to axis a (axes_dim
+// split of D/2 pairs), theta_{p,i} = id_a(p) * theta^(-2j/d_a) with j the pair's index in its axis.
+void rope_table_launch(float* cosb, float* sinb, int nt, long long i0, int ni, long long wp, int D,
+                       const int axes_dim[3], double theta, cudaStream_t s);
+// SD3 2-D sin-cos position embedding (fp64 -> fp32) of image rows [i0, i0 + ni): pe [ni, h], patch
+// p at (pr, pc) = ((p / n_c + top) / q, (p % n_c + left) / q); channels [sin(pc w), cos(pc w),
+// sin(pr w), cos(pr w)], w_j = 10000^(-j / (h/4)).
+void sincos_pe_launch(float* pe, long long i0, int ni, long long n_c, long long top, long long left, double q, int h,
+                      cudaStream_t s);
+
 // ------------------------------------------------------------------ SYNTH-1 generator
 // kind: 0 'w'/'b'/'x' (bf16 = rne(r*c)), 1 'g' (bf16 = rne(1 + r*c)), 2 'f' (fp32 = r*c)
 void synth_launch(void* dst, uint64_t seed, uint32_t tensor_id, uint64_t idx0, long long n, int kind, float c,

@@ -68,3 +68,6 @@ def test_bench_two_ranks_one_gpu():
     assert d["n_gpus"] == 2 and d["config"]["sp"] == 2 and "fused-ipc" in d["config"]["transport"]
     assert d["value"] > 0 and d["e2e"]["value"] > 0 and d["gpu_launches"] > 0
     assert d["warmup"] == 3 and d["steps"] == 3
+    assert d["comm"]["transport"].startswith("fused-ipc") and d["comm"]["barrier_ms_per_step"] >= 0
+    assert d["latency"]["steps"] == 3 and d["latency"]["cv"] >= 0
+    assert d["roofline"]["unit"] == "TFLOP/s" and set(d["roofline_kernels"]) == {"gemm", "attention"}
