@@ -88,7 +88,9 @@ tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int
  * impl 0: the tcgen05/TMEM kernel the step uses (= impl 51 for D = 128, 53 for D = 64; the
  * environment variables TSV_ATTN_D128 / TSV_ATTN_D64 select another impl for the step);
  * 50..54: the same kernel with 0..4 of every 8 exp2 pairs evaluated by polynomial on the FMA pipe
- * instead of MUFU.EX2 (tuning sweeps).  Other values: TSV_E_INVAL. */
+ * instead of MUFU.EX2 (tuning sweeps); 58: all of them by polynomial; 59: DIAGNOSTIC ONLY, wrong
+ * results -- P = the scaled score without any exponential (the pipeline's ceiling without the
+ * softmax arithmetic).  Other values: TSV_E_INVAL. */
 tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
                             void* o, int64_t ldo, int L, int H, int D, int impl, void* stream);
 

@@ -279,7 +279,9 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
           for (int i = 0; i < 32; i += 2) {
             float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2, nm2);
             float2 p;
-            if (((i >> 1) & 7) >= 8 - NPOLY) {
+            if (NPOLY == 9) {
+              p = x;   // diagnostic (impl 59): no exponential -- the pipeline's ceiling without softmax math
+            } else if (((i >> 1) & 7) >= 8 - NPOLY) {
               // the polynomial path wraps the exponent field outside [-126, 127]: clamp both sides
               // (a clamped x > 64 still makes the sum exceed the limit)
               x.x = fminf(x.x, 64.f);
@@ -297,7 +299,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         const float2 l01 = __fadd2_rn(lz[0], lz[1]), l23 = __fadd2_rn(lz[2], lz[3]);
         const float2 l4 = __fadd2_rn(l01, l23);
         const float ts = l4.x + l4.y;
-        if (!__any_sync(0xffffffffu, !(ts <= LAZY_LIMIT))) {   // also catches inf / NaN
+        if (NPOLY == 9 || !__any_sync(0xffffffffu, !(ts <= LAZY_LIMIT))) {   // also catches inf / NaN
           l_sum += ts;
           tmem_st32(s_col, sr[0]);
           tmem_st32(s_col + 32, sr[1]);
@@ -609,6 +611,8 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     case 52: e = launch_fa<D, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 53: e = launch_fa<D, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 54: e = launch_fa<D, 4>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 58: e = launch_fa<D, 8>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // all exp2 by polynomial
+    case 59: e = launch_fa<D, 9>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // diagnostic: no exp2
     default: return -3;
   }
   return e == cudaSuccess ? 0 : -5;

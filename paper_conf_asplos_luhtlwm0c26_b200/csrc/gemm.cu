@@ -11,6 +11,7 @@
 //     tile i+1;  4-8 smem stages depending on BN.
 // Tile order walks M fastest so consecutive CTAs share the same weight tile (weights stream from
 // HBM once per N-column while the activations stay L2-resident).
+#include <cstdlib>
 #include <cstdio>
 #include <cudaTypedefs.h>
 
@@ -45,6 +46,7 @@ struct GemmArgs {
   int splits, kps, tiles_per_split;
   int* sem;
   float* ws;
+  int group_n, serpentine;   // rasterisation (decode_tile)
   int M[GEMM_MAX_PROBLEMS], num_m[GEMM_MAX_PROBLEMS], tile0[GEMM_MAX_PROBLEMS];
   GemmEpi epi[GEMM_MAX_PROBLEMS];
 };
@@ -55,11 +57,12 @@ struct GemmMaps {
 // > 4 KB of kernel parameters (CUDA 12.1+, up to 32 764 bytes)
 static_assert(sizeof(GemmArgs) + sizeof(GemmMaps) <= 32764, "GEMM kernel parameters too large");
 
-// Rasterisation: groups of GROUP_N weight-column tiles; inside a group the n index varies fastest,
-// then m.  A wave of 148 concurrent tiles therefore touches <= GROUP_N weight tiles and
-// ~148/GROUP_N activation row-blocks, both L2-resident, so activations are streamed from HBM about
-// num_n / GROUP_N times instead of num_n times (measured: 2.8 GB -> algorithmic for 2048^2 fc1).
-constexpr int GROUP_N = 8;
+// Rasterisation: groups of group_n weight-column tiles; inside a group the n index varies fastest,
+// then m.  A wave of 148 concurrent tiles therefore touches <= group_n weight tiles and
+// ~148/group_n activation row-blocks, both L2-resident, so activations are streamed from HBM about
+// num_n / group_n times instead of num_n times (measured: 2.8 GB -> algorithmic for 2048^2 fc1).
+// serpentine: odd groups walk m backwards, so a group starts on the activation rows the previous
+// group used last (still in L2) instead of on the evicted first rows.
 __device__ __forceinline__ void decode_tile(const GemmArgs& a, int t, int& p, int& m_blk, int& n_blk) {
   p = 0;
 #pragma unroll
@@ -67,11 +70,13 @@ __device__ __forceinline__ void decode_tile(const GemmArgs& a, int t, int& p, in
     if (q < a.nprob && t >= a.tile0[q]) p = q;
   const int lt = t - a.tile0[p];
   const int nm = a.num_m[p];
-  const int group = lt / (GROUP_N * nm);
-  const int first_n = group * GROUP_N;
-  const int gsize = min(GROUP_N, a.num_n - first_n);
-  const int r = lt - group * GROUP_N * nm;
+  const int G = a.group_n;
+  const int group = lt / (G * nm);
+  const int first_n = group * G;
+  const int gsize = min(G, a.num_n - first_n);
+  const int r = lt - group * G * nm;
   m_blk = r / gsize;
+  if (a.serpentine && (group & 1)) m_blk = nm - 1 - m_blk;
   n_blk = first_n + r % gsize;
 }
 
@@ -841,6 +846,16 @@ int gemm_plan_multi(GemmPlan* p, const GemmProblem* probs, int nprob, int N, int
   }
   const int bm = pair ? 256 : BM;
   p->nprob = nprob; p->N = N; p->K = K; p->BN = bn; p->pair = pair;
+  // TSV_GEMM_GROUP / TSV_GEMM_SERP (read once): rasterisation A/B (tools/ab_*.sh)
+  static int env_group = -1, env_serp = -1;
+  if (env_group < 0) {
+    const char* g = getenv("TSV_GEMM_GROUP");
+    const char* sp = getenv("TSV_GEMM_SERP");
+    env_group = g ? atoi(g) : 0;
+    env_serp = sp ? atoi(sp) : 1;
+  }
+  p->group_n = env_group > 0 ? env_group : 16;   // r02 sweep (profiles/r02): 16 + serpentine, -17 % DRAM bytes at 2048^2
+  p->serpentine = env_serp;
   int tiles = 0;
   for (int q = 0; q < nprob; ++q) {
     const GemmProblem& g = probs[q];
@@ -929,6 +944,7 @@ static void launch_bn(const GemmPlan& p, cudaStream_t s) {
   const int bm = p.pair ? 256 : BM;
   a.N = p.N; a.K = p.K; a.num_n = p.N / BN; a.num_tiles = p.tiles; a.nprob = p.nprob;
   a.splits = p.splits; a.kps = p.kps; a.tiles_per_split = p.tiles / p.splits; a.sem = p.sem; a.ws = p.ws;
+  a.group_n = p.group_n; a.serpentine = p.serpentine;
   for (int q = 0; q < GEMM_MAX_PROBLEMS; ++q) {
     const int qq = q < p.nprob ? q : 0;
     a.M[q] = p.Mq[qq];

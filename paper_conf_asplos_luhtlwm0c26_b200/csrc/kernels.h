@@ -116,6 +116,8 @@ struct GemmPlan {
   int kps = 0;        // k-blocks (of 64) per split
   int* sem = nullptr; // split-K arrival counters, 4 per output tile, zero between launches
   float* ws = nullptr; // split-K partials
+  int group_n = 16;    // rasterisation: weight-column tiles per group
+  int serpentine = 1;  // odd groups walk the row blocks backwards (activation reuse across groups)
   GemmEpi epi;
 };
 // split-K workspace of one stream: counters (zeroed once, left zero by every launch) + partials

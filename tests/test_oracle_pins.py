@@ -245,6 +245,67 @@ def test_double_single_final_vs_torchtitan(tt_layers):
     assert np.allclose(F.final_layer(W, img, vec), rf[0].numpy(), rtol=1e-10, atol=1e-10)
 
 
+def test_flux_step_vs_torchtitan_model(tt_layers):
+    """The whole oracle step (a0 conditioning, a1 img_in AND txt_in embeddings, the [txt; img] join
+    and split, every block, the final layer, a12 Euler) against torchtitan's independent FluxModel
+    forward with the same weights -- the pin of the txt_in leg, which the block-level pins (random
+    txt) and adaLN-Zero (txt irrelevant) leave open.  FluxModel has no guidance embedder (S:§8(c)
+    "Where TT differs" i), so guidance_in is zeroed on the oracle side: MLP_g(e(g)) = 0."""
+    model_mod = pytest.importorskip("torchtitan.experiments.flux.model.model")
+    args_mod = pytest.importorskip("torchtitan.experiments.flux.model.args")
+    cfg = TINY2
+    zero = {n: np.zeros_like(Weights(cfg)[n]) for n in ("guidance_in.in.w", "guidance_in.in.b",
+                                                        "guidance_in.out.w", "guidance_in.out.b")}
+    W = Weights(cfg, overrides=zero)
+    hgt, wid, steps, step = 48, 64, 20, 3
+    x, T, y = request_inputs(cfg, hgt, wid, 1234)
+    v_o, xn_o = F.request_step(cfg, W, x, T, y, step, steps, 3.5, hgt, wid, drop_weights=False)
+
+    a = args_mod.FluxModelArgs(in_channels=cfg.in_ch, out_channels=cfg.in_ch, vec_in_dim=cfg.vec_dim,
+                               context_in_dim=cfg.ctx_dim, hidden_size=cfg.hidden,
+                               mlp_ratio=cfg.mlp_hidden / cfg.hidden, num_heads=cfg.heads, depth=cfg.n_double,
+                               depth_single_blocks=cfg.n_single, axes_dim=tuple(cfg.axes_dim), theta=int(cfg.theta),
+                               qkv_bias=True)
+    m = model_mod.FluxModel(a).double()
+    _load(m.img_in.weight, W, "img_in.w"); _load(m.img_in.bias, W, "img_in.b")
+    _load(m.txt_in.weight, W, "txt_in.w"); _load(m.txt_in.bias, W, "txt_in.b")
+    for nme, mod in (("time_in", m.time_in), ("vector_in", m.vector_in)):
+        _load(mod.in_layer.weight, W, nme + ".in.w"); _load(mod.in_layer.bias, W, nme + ".in.b")
+        _load(mod.out_layer.weight, W, nme + ".out.w"); _load(mod.out_layer.bias, W, nme + ".out.b")
+    for j in range(cfg.n_double):
+        m.double_blocks[j] = _tt_double(tt_layers, cfg, W, j)
+    for j, sb in enumerate(m.single_blocks):
+        p = f"single{j}."
+        _load(sb.modulation.lin.weight, W, p + "mod.w"); _load(sb.modulation.lin.bias, W, p + "mod.b")
+        _load(sb.linear1.weight, W, p + "lin1.w"); _load(sb.linear1.bias, W, p + "lin1.b")
+        _load(sb.linear2.weight, W, p + "lin2.w"); _load(sb.linear2.bias, W, p + "lin2.b")
+        _load(sb.norm.query_norm.weight, W, p + "q_norm.g"); _load(sb.norm.key_norm.weight, W, p + "k_norm.g")
+        sb.norm.query_norm.eps = 1e-6
+        sb.norm.key_norm.eps = 1e-6
+    ll = m.final_layer
+    _load(ll.adaLN_modulation[1].weight, W, "final.mod.w"); _load(ll.adaLN_modulation[1].bias, W, "final.mod.b")
+    _load(ll.linear.weight, W, "final.lin.w"); _load(ll.linear.bias, W, "final.lin.b")
+    ids = F.position_ids(T.shape[0], hgt, wid)
+    ts = F.schedule(steps, x.shape[0])
+    with torch.no_grad():
+        v_t = m(img=torch.from_numpy(x)[None], img_ids=torch.from_numpy(ids[T.shape[0]:])[None],
+                txt=torch.from_numpy(T)[None], txt_ids=torch.from_numpy(ids[:T.shape[0]])[None],
+                timesteps=torch.tensor([ts[step]], dtype=torch.float64), y=torch.from_numpy(y)[None])[0].numpy()
+    # TT rotates q, k in float32 (its RoPE table and apply_rope cast to float, TT:math.py:30-36):
+    # ~1e-7 per rotation, 1e-5 normwise after 2 + 2 blocks; every other op is float64 on both sides
+    vmax = np.abs(v_t).max()
+    assert np.max(np.abs(v_o - v_t)) <= 5e-5 * vmax
+    assert np.max(np.abs(xn_o - (x + (ts[step + 1] - ts[step]) * v_t))) <= 5e-5 * vmax
+    # the pin sees the text embedding: a dropped txt_in bias, or a perturbed txt_in weight, moves v far
+    # outside that bound (perturbations must vary across channels: LayerNorm ignores a constant shift)
+    rng = np.random.default_rng(3)
+    for nme, new in (("txt_in.b", np.zeros_like(W["txt_in.b"])),
+                     ("txt_in.w", W["txt_in.w"] + 0.01 * rng.standard_normal(W["txt_in.w"].shape))):
+        W2 = Weights(cfg, overrides=dict(zero, **{nme: new}))
+        v_2, _ = F.request_step(cfg, W2, x, T, y, step, steps, 3.5, hgt, wid, drop_weights=False)
+        assert np.max(np.abs(v_2 - v_t)) > 2e-3 * vmax, nme
+
+
 def test_conditioning_vec_vs_torchtitan(tt_layers):
     cfg = TINY
     W = Weights(cfg)
