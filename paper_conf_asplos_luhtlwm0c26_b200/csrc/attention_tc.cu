@@ -3,8 +3,9 @@
 //
 // One CTA = one head x 256 queries as two 128-query tiles t = 0, 1 that share every K/V tile
 // (half the K/V traffic per query).  Warp roles:
-//   warp 0      TMA producer: Q0, Q1 once, then K/V tiles of 128 keys into an NST-stage ring
-//               (3-D tensor maps [rows][heads][D] -> one map serves every head and layout);
+//   warps 0, 3  TMA producers: Q0, Q1 once, then K tiles of 128 keys into an NK-stage ring (warp 0)
+//               and V tiles into an NV-stage ring (warp 3) (3-D tensor maps [rows][heads][D] -> one
+//               map serves every head and layout);
 //   warp 1      tcgen05.mma issuer (the whole warp runs the loop, one elected lane issues):
 //               S_t(j) = Q_t K_j^T into TMEM, O_t += P_t(j) V_j with P read from TMEM and V
 //               consumed MN-major straight from the TMA tile (no transpose, no smem P);
@@ -14,7 +15,7 @@
 // bf16 (tcgen05.st), so S_t(j+1) must follow PV_t(j): the MMA warp issues PV_t(j) before S_t(j+1),
 // and the in-order tcgen05 pipe makes "S_t(j) complete" imply "O_t holds tiles < j" (a rare O
 // rescale needs no extra wait).
-// TMEM: S0 | S1 | O0 | O1 (128 + 128 + D + D fp32 columns).  Smem: Q0, Q1, NST K/V stages.
+// TMEM: S0 | S1 | O0 | O1 (128 + 128 + D + D fp32 columns).  Smem: Q0, Q1, NK K and NV V stages.
 //
 // Softmax (lazy row max): P = 2^(s * scale_log2 - m_ref) is evaluated with the running reference
 // m_ref directly, without a per-tile max: the tile's row sum bounds every p in it (p <= sum), so a
@@ -96,21 +97,28 @@ __host__ __device__ constexpr uint32_t make_idesc_bf16_bmn(int M, int N) {
 
 }  // namespace
 
-template <int D>
+// K and V tiles flow through separate rings (NK and NV stages) filled by two producer warps: a K
+// stage is free as soon as both S MMAs of its tile completed, a V stage only after both PV MMAs, so
+// the next K load starts ~one tile of tensor time earlier than with one joint K/V stage (r02: the
+// MMA warp spent most of its stall samples waiting for K/V data with the joint 2-stage ring).
+// KV = 0: NK = NV = 2 (D = 128) / 4 (D = 64); KV = 1: NK = 3, NV = 2; KV = 2: NK = 2, NV = 3 (D = 128
+// fills the 227 KB of shared memory with 3 + 2 stages).
+template <int D, int KV = 0>
 struct FaCfg {
   static constexpr int NSUB = D / 64;
   static constexpr int Q_TILE = AT_BM * D * 2;
   static constexpr int KV_TILE = AT_BN * D * 2;
-  // K/V ring depth: D = 128 fills shared memory with 2 stages; D = 64 has room for 4
-  static constexpr int NST = D == 64 ? 4 : 2;
+  static constexpr int NK = D == 64 ? 4 : (KV == 1 ? 3 : 2);
+  static constexpr int NV = D == 64 ? 4 : (KV == 2 ? 3 : 2);
   static constexpr int OFF_Q = 0;                        // 2 tiles
-  static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // NST stages
-  static constexpr int OFF_V = OFF_K + NST * KV_TILE;    // NST stages
-  static constexpr int OFF_BAR = OFF_V + NST * KV_TILE;
+  static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // NK stages
+  static constexpr int OFF_V = OFF_K + NK * KV_TILE;     // NV stages
+  static constexpr int OFF_BAR = OFF_V + NV * KV_TILE;
   static constexpr int SMEM = OFF_BAR + 256 + 1024;      // barriers + 1 KB alignment slack
   static constexpr int O_COL = 256;
 };
-static_assert(FaCfg<128>::SMEM <= 232448 && FaCfg<64>::SMEM <= 232448, "attention shared memory > 227 KB");
+static_assert(FaCfg<128, 1>::SMEM <= 232448 && FaCfg<128, 2>::SMEM <= 232448 && FaCfg<64>::SMEM <= 232448,
+              "attention shared memory > 227 KB");
 constexpr int FA_THREADS = 384;
 
 // KV split (blockIdx.z = split): see AttnSplitWs.  nsplit = 1: the whole key range, no workspace.
@@ -120,24 +128,26 @@ struct AttnSplitArgs {
   float* ws = nullptr;
 };
 
-template <int D, int NPOLY>
+template <int D, int NPOLY, int KV>
 __global__ void __launch_bounds__(FA_THREADS, 1)
     attention_fa_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
                         float scale_log2, const __grid_constant__ AttnScatter sc,
                         const __grid_constant__ AttnSplitArgs sa) {
-  using C = FaCfg<D>;
+  using C = FaCfg<D, KV>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
-  constexpr int NST = C::NST;
+  constexpr int NK = C::NK, NV = C::NV;
   uint64_t* q_full = bars + 0;
-  uint64_t* kv_full = bars + 1;              // [NST stages]
-  uint64_t* kv_empty = bars + 1 + NST;       // [NST stages]
-  uint64_t* s_full = bars + 1 + 2 * NST;     // [2 q-tiles]
-  uint64_t* p_full = bars + 3 + 2 * NST;     // [2 q-tiles]
-  uint64_t* o_done = bars + 5 + 2 * NST;     // [2 q-tiles]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 8 + 2 * NST);
+  uint64_t* k_full = bars + 1;                    // [NK stages]
+  uint64_t* k_empty = k_full + NK;                // [NK stages]
+  uint64_t* v_full = k_empty + NK;                // [NV stages]
+  uint64_t* v_empty = v_full + NV;                // [NV stages]
+  uint64_t* s_full = v_empty + NV;                // [2 q-tiles]
+  uint64_t* p_full = s_full + 2;                  // [2 q-tiles]
+  uint64_t* o_done = p_full + 2;                  // [2 q-tiles]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(o_done + 3);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int head = blockIdx.y;
@@ -152,9 +162,13 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     tma_prefetch_desc(&tmK);
     tma_prefetch_desc(&tmV);
     mbar_init(q_full, 1);
-    for (int i = 0; i < NST; ++i) {
-      mbar_init(&kv_full[i], 1);
-      mbar_init(&kv_empty[i], 1);
+    for (int i = 0; i < NK; ++i) {
+      mbar_init(&k_full[i], 1);
+      mbar_init(&k_empty[i], 1);
+    }
+    for (int i = 0; i < NV; ++i) {
+      mbar_init(&v_full[i], 1);
+      mbar_init(&v_empty[i], 1);
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(&s_full[i], 1);
@@ -175,22 +189,35 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
    regs_dec<80>();
    if (warp == 0) {
     if (lane == 0) {
-      // ---------------------------------------------------------------- producer
+      // ---------------------------------------------------------------- producer: Q, then the K ring
       mbar_arrive_expect_tx(q_full, 2 * C::Q_TILE);
       for (int t = 0; t < 2; ++t)
         for (int s = 0; s < C::NSUB; ++s)
           tma_load_3d(&tmQ, q_full, sm + C::OFF_Q + t * C::Q_TILE + s * (AT_BM * 128), s * 64, head,
                       q0 + t * AT_BM);
       for (int j = 0; j < n_tiles; ++j) {
-        const int st = j % NST;
-        if (j >= NST) mbar_wait(&kv_empty[st], ((j / NST) - 1) & 1);
-        mbar_arrive_expect_tx(&kv_full[st], 2 * C::KV_TILE);
-        for (int s = 0; s < C::NSUB; ++s) {
-          tma_load_3d(&tmK, &kv_full[st], sm + C::OFF_K + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
+        const int st = j % NK;
+        if (j >= NK) mbar_wait(&k_empty[st], ((j / NK) - 1) & 1);
+        mbar_arrive_expect_tx(&k_full[st], C::KV_TILE);
+        for (int s = 0; s < C::NSUB; ++s)
+          tma_load_3d(&tmK, &k_full[st], sm + C::OFF_K + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
                       (j0 + j) * AT_BN);
-          tma_load_3d(&tmV, &kv_full[st], sm + C::OFF_V + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
+      }
+    }
+   } else if (warp == 3) {
+    if (lane == 0) {
+      // ---------------------------------------------------------------- producer: the V ring
+      // V(0) is needed only after S(0): start once Q has landed (K(0) was issued right behind it), so
+      // the first S MMAs do not share the start-up bandwidth with V traffic (short key loops: small
+      // images, KV splits).  q_full completes exactly once, so this wait cannot miss its phase.
+      mbar_wait(q_full, 0);
+      for (int j = 0; j < n_tiles; ++j) {
+        const int st = j % NV;
+        if (j >= NV) mbar_wait(&v_empty[st], ((j / NV) - 1) & 1);
+        mbar_arrive_expect_tx(&v_full[st], C::KV_TILE);
+        for (int s = 0; s < C::NSUB; ++s)
+          tma_load_3d(&tmV, &v_full[st], sm + C::OFF_V + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
                       (j0 + j) * AT_BN);
-        }
       }
     }
    } else if (warp == 1) {
@@ -204,9 +231,9 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     const uint64_t dk0 = make_sw128_desc(smem_u32(sm + C::OFF_K));
     const uint64_t dv0 = make_sw128_mn_desc(smem_u32(sm + C::OFF_V), AT_BN * 128);
     mbar_wait(q_full, 0);
-    auto issue_s = [&](int t, int j) {
+    auto issue_s = [&](int t, int j) {   // t == 1 releases the K stage (both S MMAs of tile j issued)
       const uint64_t dq = dq0 + (uint64_t)((t * C::Q_TILE) >> 4);
-      const uint64_t dk = dk0 + (uint64_t)(((j % NST) * C::KV_TILE) >> 4);
+      const uint64_t dk = dk0 + (uint64_t)(((j % NK) * C::KV_TILE) >> 4);
       if (elect_one()) {
 #pragma unroll
         for (int kk = 0; kk < D / 16; ++kk) {
@@ -214,11 +241,13 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
           umma_bf16_ss(tmem + t * 128, dq + off, dk + off, idesc_s, kk > 0);
         }
         umma_commit(&s_full[t]);
+        if (t == 1) umma_commit(&k_empty[j % NK]);
       }
       __syncwarp();
     };
-    auto issue_pv = [&](int t, int j, bool release) {
-      const uint64_t dv = dv0 + (uint64_t)(((j % NST) * C::KV_TILE) >> 4);
+    auto issue_pv = [&](int t, int j) {   // t == 0 waits for the V tile, t == 1 releases it
+      const uint64_t dv = dv0 + (uint64_t)(((j % NV) * C::KV_TILE) >> 4);
+      if (t == 0) mbar_wait(&v_full[j % NV], (j / NV) & 1);
       mbar_wait(&p_full[t], j & 1);
       tc_fence_after();
       if (elect_one()) {
@@ -226,20 +255,20 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         for (int kk = 0; kk < AT_BN / 16; ++kk)
           umma_bf16_ts(tmem + C::O_COL + t * D, tmem + t * 128 + kk * 8, dv + (uint64_t)(kk * (2048 >> 4)), idesc_o,
                        (j | kk) != 0);
-        if (release) umma_commit(&kv_empty[j % NST]);
+        if (t == 1) umma_commit(&v_empty[j % NV]);
       }
       __syncwarp();
     };
     for (int j = 0; j < n_tiles; ++j) {
-      mbar_wait(&kv_full[j % NST], (j / NST) & 1);
+      mbar_wait(&k_full[j % NK], (j / NK) & 1);
       tc_fence_after();
       for (int t = 0; t < 2; ++t) {
-        if (j > 0) issue_pv(t, j - 1, t == 1);
+        if (j > 0) issue_pv(t, j - 1);
         issue_s(t, j);
       }
     }
     for (int t = 0; t < 2; ++t) {
-      issue_pv(t, n_tiles - 1, false);
+      issue_pv(t, n_tiles - 1);
       if (elect_one()) umma_commit(&o_done[t]);
       __syncwarp();
     }
@@ -516,7 +545,7 @@ static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L
   return r == CUDA_SUCCESS ? 0 : -2;
 }
 
-template <int D, int NP>
+template <int D, int NP, int KV = 0>
 static cudaError_t launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o,
                              long long ldo, int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s,
                              const AttnSplitArgs& sa) {
@@ -524,14 +553,14 @@ static cudaError_t launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const
   int dev = 0;
   cudaGetDevice(&dev);
   if (!(done >> dev & 1ull)) {
-    cudaError_t e = cudaFuncSetAttribute(attention_fa_kernel<D, NP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         FaCfg<D>::SMEM);
+    cudaError_t e = cudaFuncSetAttribute(attention_fa_kernel<D, NP, KV>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, FaCfg<D, KV>::SMEM);
     if (e != cudaSuccess) return e;
     done |= 1ull << dev;
   }
   dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H, sa.nsplit);
-  return launch_pdl(attention_fa_kernel<D, NP>, grid, dim3(FA_THREADS), FaCfg<D>::SMEM, s, tq, tk, tv, o, ldo,
-                    L, scale_log2, sc, sa);
+  return launch_pdl(attention_fa_kernel<D, NP, KV>, grid, dim3(FA_THREADS), FaCfg<D, KV>::SMEM, s, tq, tk, tv, o,
+                    ldo, L, scale_log2, sc, sa);
 }
 
 // KV-split factor for a launch of C = ceil(L/256) x H CTAs: the S in 1..8 minimising the estimated
@@ -588,7 +617,7 @@ static int default_version(int D) {
     const char* e = getenv(D == 128 ? "TSV_ATTN_D128" : "TSV_ATTN_D64");
     // 1 (D = 128) / 3 (D = 64) of 8 exp2 pairs by polynomial (round-2 sweep, profiles/r02/mb_attn_sweep.jsonl)
     r = e ? atoi(e) : (D == 128 ? 51 : 53);
-    if (r < 50 || r > 54) r = D == 128 ? 51 : 53;
+    if (r < 50 || r > 79) r = D == 128 ? 51 : 53;
   }
   return r;
 }
@@ -613,6 +642,13 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     case 54: e = launch_fa<D, 4>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 58: e = launch_fa<D, 8>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // all exp2 by polynomial
     case 59: e = launch_fa<D, 9>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // diagnostic: no exp2
+    // 60 + n / 70 + n (D = 128): 3 K + 2 V / 2 K + 3 V stages
+    case 61: e = launch_fa<D, 1, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 62: e = launch_fa<D, 2, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 69: e = launch_fa<D, 9, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 71: e = launch_fa<D, 1, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 72: e = launch_fa<D, 2, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 79: e = launch_fa<D, 9, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     default: return -3;
   }
   return e == cudaSuccess ? 0 : -5;

@@ -3,8 +3,12 @@
 This module holds NO arithmetic of the method (no DiT math).  It only turns
 (seed, tensor id, element index) into numbers, following the counter-hash
 specification restated in ``include/tsv.h`` ("SYNTH-1").  The CUDA path has
-its own, independent implementation of the same spec (``csrc/init.cu``); the
-two are checked bit-for-bit against each other in ``tests/test_gpu_init.py``.
+its own, independent implementations of the same spec (``synth_kernel`` in
+``paper_conf_asplos_luhtlwm0c26_b200/csrc/elementwise.cu`` for weights, the
+host generator in ``csrc/engine.cu`` for request inputs); they are checked
+bit-for-bit against this module in ``tests/test_gpu_kernels.py`` (weights via
+``tsv_op_synth`` / ``tsv_debug_read_weight``) and ``tests/test_gpu_step.py``
+(request inputs).
 
 SYNTH-1
   key  = seed XOR (tensor_id << 48) XOR idx                    (uint64)

@@ -135,7 +135,7 @@ def attn_cases():
                 times[impl].append(timeit(fns[impl], iters=5 if L > 8000 else 20))
         for impl in impls:
             ms = sorted(times[impl])[len(times[impl]) // 2]
-            name = "tcgen05" if impl == 0 else f"tcgen05-poly{impl % 10}"
+            name = "tcgen05" if impl == 0 else f"tcgen05-impl{impl}"
             print(json.dumps({"op": "attention", "impl": name, "L": L, "H": H, "D": D,
                               "ms": round(ms, 4), "tflops": round(4 * L * L * D * H / ms / 1e9, 1),
                               "all_ms": [round(t, 4) for t in times[impl]]}), flush=True)
