@@ -102,7 +102,8 @@ __host__ __device__ constexpr uint32_t make_idesc_bf16_bmn(int M, int N) {
 // the next K load starts ~one tile of tensor time earlier than with one joint K/V stage (r02: the
 // MMA warp spent most of its stall samples waiting for K/V data with the joint 2-stage ring).
 // KV = 0: NK = NV = 2 (D = 128) / 4 (D = 64); KV = 1: NK = 3, NV = 2; KV = 2: NK = 2, NV = 3 (D = 128
-// fills the 227 KB of shared memory with 3 + 2 stages).
+// fills the 227 KB of shared memory with 3 + 2 stages); KV = 3: one joint K+V ring (NK = NV stages,
+// one producer, a stage freed after both PV MMAs: round 1's design, kept where it measured better).
 template <int D, int KV = 0>
 struct FaCfg {
   static constexpr int NSUB = D / 64;
@@ -135,6 +136,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
                         float scale_log2, const __grid_constant__ AttnScatter sc,
                         const __grid_constant__ AttnSplitArgs sa) {
   using C = FaCfg<D, KV>;
+  constexpr bool JOINT = KV == 3;   // K and V of a tile share one stage and one barrier pair
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
@@ -198,13 +200,17 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       for (int j = 0; j < n_tiles; ++j) {
         const int st = j % NK;
         if (j >= NK) mbar_wait(&k_empty[st], ((j / NK) - 1) & 1);
-        mbar_arrive_expect_tx(&k_full[st], C::KV_TILE);
-        for (int s = 0; s < C::NSUB; ++s)
+        mbar_arrive_expect_tx(&k_full[st], (JOINT ? 2 : 1) * C::KV_TILE);
+        for (int s = 0; s < C::NSUB; ++s) {
           tma_load_3d(&tmK, &k_full[st], sm + C::OFF_K + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
                       (j0 + j) * AT_BN);
+          if (JOINT)
+            tma_load_3d(&tmV, &k_full[st], sm + C::OFF_V + st * C::KV_TILE + s * (AT_BN * 128), s * 64, head,
+                        (j0 + j) * AT_BN);
+        }
       }
     }
-   } else if (warp == 3) {
+   } else if (warp == 3 && !JOINT) {
     if (lane == 0) {
       // ---------------------------------------------------------------- producer: the V ring
       // V(0) is needed only after S(0): start once Q has landed (K(0) was issued right behind it), so
@@ -241,13 +247,13 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
           umma_bf16_ss(tmem + t * 128, dq + off, dk + off, idesc_s, kk > 0);
         }
         umma_commit(&s_full[t]);
-        if (t == 1) umma_commit(&k_empty[j % NK]);
+        if (t == 1 && !JOINT) umma_commit(&k_empty[j % NK]);
       }
       __syncwarp();
     };
     auto issue_pv = [&](int t, int j) {   // t == 0 waits for the V tile, t == 1 releases it
       const uint64_t dv = dv0 + (uint64_t)(((j % NV) * C::KV_TILE) >> 4);
-      if (t == 0) mbar_wait(&v_full[j % NV], (j / NV) & 1);
+      if (t == 0 && !JOINT) mbar_wait(&v_full[j % NV], (j / NV) & 1);
       mbar_wait(&p_full[t], j & 1);
       tc_fence_after();
       if (elect_one()) {
@@ -255,7 +261,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         for (int kk = 0; kk < AT_BN / 16; ++kk)
           umma_bf16_ts(tmem + C::O_COL + t * D, tmem + t * 128 + kk * 8, dv + (uint64_t)(kk * (2048 >> 4)), idesc_o,
                        (j | kk) != 0);
-        if (t == 1) umma_commit(&v_empty[j % NV]);
+        if (t == 1) umma_commit(JOINT ? &k_empty[j % NK] : &v_empty[j % NV]);
       }
       __syncwarp();
     };
@@ -615,9 +621,10 @@ static int default_version(int D) {
   int& r = v[D == 128];
   if (r < 0) {
     const char* e = getenv(D == 128 ? "TSV_ATTN_D128" : "TSV_ATTN_D64");
-    // 1 (D = 128) / 3 (D = 64) of 8 exp2 pairs by polynomial (round-2 sweep, profiles/r02/mb_attn_sweep.jsonl)
-    r = e ? atoi(e) : (D == 128 ? 51 : 53);
-    if (r < 50 || r > 79) r = D == 128 ? 51 : 53;
+    // D = 128: separate K / V rings, 1 of 8 exp2 pairs by polynomial; D = 64: the joint ring (the split
+    // rings measured -2 % on the SD3 1024^2 step), 3 of 8 (round-2 sweeps, profiles/r02)
+    r = e ? atoi(e) : (D == 128 ? 51 : 83);
+    if (r < 50 || r > 89) r = D == 128 ? 51 : 83;
   }
   return r;
 }
@@ -649,6 +656,10 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     case 71: e = launch_fa<D, 1, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 72: e = launch_fa<D, 2, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 79: e = launch_fa<D, 9, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    // 80 + n: the joint K+V ring (round 1's producer), n of 8 exp2 pairs by polynomial
+    case 81: e = launch_fa<D, 1, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 82: e = launch_fa<D, 2, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 83: e = launch_fa<D, 3, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     default: return -3;
   }
   return e == cudaSuccess ? 0 : -5;

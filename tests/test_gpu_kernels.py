@@ -282,7 +282,7 @@ def test_qk_norm_rope(tsv, H, D, rows, n_first):
 
 
 # ----------------------------------------------------------------------------- attention
-@pytest.mark.parametrize("impl", [0, 50, 51, 52, 53, 54])
+@pytest.mark.parametrize("impl", [0, 50, 51, 52, 53, 54, 61, 71, 81, 83])
 @pytest.mark.parametrize("L,H,D", [(1, 2, 64), (63, 4, 64), (320, 4, 64), (1000, 3, 128), (1536, 2, 128),
                                    (4700, 1, 128)])
 def test_attention(tsv, L, H, D, impl):
@@ -379,7 +379,7 @@ def test_attention_special_cases(tsv):
     assert np.max(np.abs(_np(o).reshape(L, H, D) - ref)) < 2e-2
 
 
-@pytest.mark.parametrize("impl", [0, 51, 52, 53])
+@pytest.mark.parametrize("impl", [0, 51, 52, 53, 61, 81, 83])
 def test_attention_rescale_path(tsv, impl):
     """Scores growing along the key axis force the conditional O rescale (max grows by > 2^8)."""
     L, H, D = 700, 1, 128
@@ -399,7 +399,7 @@ def test_attention_rescale_path(tsv, impl):
     assert _rel(_np(o).reshape(L, H, D), ref) < 2e-2
 
 
-@pytest.mark.parametrize("D,impl", [(64, 0), (64, 51), (64, 52), (128, 0), (128, 52), (128, 53)])
+@pytest.mark.parametrize("D,impl", [(64, 0), (64, 51), (64, 83), (128, 0), (128, 52), (128, 81)])
 @pytest.mark.parametrize("jump", [3.0, 12.0, 200.0])
 def test_attention_score_jump(tsv, D, impl, jump):
     """A later key tile whose scores exceed the running maximum by `jump` (log2 units): small jumps
