@@ -11,11 +11,13 @@
 // Conditioning (a0) runs once per (request, GPU): vec_s for all steps, then the modulation table
 // mod[s] = W_mod SiLU(vec_s) + b as one [S, n_mod] GEMM.
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
 #include <map>
+#include <tuple>
 #include <memory>
 #include <mutex>
 #include <string>
@@ -60,6 +62,15 @@ static tsv_status fail(tsv_status s, const char* fmt, ...) {
     tsv_status s_ = (expr);       \
     if (s_ != TSV_OK) return s_;  \
   } while (0)
+
+// TSV_TRACE=1: host-side timestamps of the landing / reshard phases on stderr (diagnostics)
+static void trace(const char* what) {
+  static const bool on = getenv("TSV_TRACE") && atoi(getenv("TSV_TRACE"));
+  if (!on) return;
+  static auto t0 = std::chrono::steady_clock::now();
+  const auto t = std::chrono::steady_clock::now();
+  fprintf(stderr, "[tsv trace] %10.3f ms  %s\n", std::chrono::duration<double, std::milli>(t - t0).count(), what);
+}
 
 static int64_t shard_begin(int64_t n, int k, int r) { return (int64_t)r * (n / k) + std::min<int64_t>(r, n % k); }
 
@@ -261,16 +272,24 @@ struct ReqDev {
   cudaEvent_t ready_ev = nullptr; // mod / dt complete (recorded on the slot's stream)
   bool ready = false;
 };
-// per (request, slot, shard): state that depends on the group position
+// per (request, slot, shard layout): the constant, position-dependent state of a shard -- kept for
+// the request's lifetime, so a request returning to a rank in the same position (k, rank) reuses it
+// and a reshard then moves only the latent rows (P:409's latent hand-off)
+struct ShardAux {
+  DevBuf T, cosb, sinb;
+  DevBuf pe;   // SD3: fp32 [ni, h] sin-cos position embedding of this shard's image rows
+  DevBuf txt;  // fp32 [branches][nt, h]: a1 text embedding T W^T + b (constant per request,
+               // computed when the layout first lands, copied into the residual stream every step)
+  void release() { T.release(); cosb.release(); sinb.release(); pe.release(); txt.release(); }
+};
+// per (request, slot, shard): the latent state of the current group position
 struct ReqShard {
   int rank_in_group = 0, k = 1;
   int64_t t0 = 0, nt = 0, i0 = 0, ni = 0;  // txt rows [t0, t0+nt), img rows [i0, i0+ni)
-  DevBuf lat, vel, T, cosb, sinb;
-  DevBuf pe;  // SD3: fp32 [ni, h] sin-cos position embedding of this shard's image rows
-  DevBuf txt;         // fp32 [branches][nt, h]: a1 text embedding T W^T + b (constant per request,
-                      // computed when the shard lands, copied into the residual stream every step)
+  DevBuf lat, vel;
+  ShardAux* ax = nullptr;                  // owned by Request::aux
   void release() {
-    lat.release(); vel.release(); T.release(); cosb.release(); sinb.release(); pe.release(); txt.release();
+    lat.release(); vel.release();
   }
 };
 
@@ -307,6 +326,7 @@ struct Request {
   std::vector<double> ts;         // t_0..t_S
   std::map<int, ReqDev> dev;      // by slot
   std::map<int, ReqShard> shard;  // by slot (current group)
+  std::map<std::tuple<int, int, int>, ShardAux> aux;   // by (slot, k, rank in group)
   std::map<int, cudaEvent_t> last;  // by slot: completion of the last submitted work
   bool has_velocity = false;
 };
@@ -594,35 +614,43 @@ static tsv_status setup_shard(tsv_engine* e, Request& R, int si, int rank_in_gro
   CK(cudaSetDevice(s.device));
   TRY(qalloc(e, sh.lat, s, std::max<size_t>(1, sh.ni) * m.in * 4));
   TRY(qalloc(e, sh.vel, s, std::max<size_t>(1, sh.ni) * m.in * 4));
-  TRY(qalloc(e, sh.T, s, std::max<size_t>(1, sh.nt) * m.B * m.ctx * 2));
-  TRY(qalloc(e, sh.txt, s, std::max<size_t>(1, sh.nt) * m.B * m.h * 4));
+  const auto key = std::make_tuple(si, k, rank_in_group);
+  auto found = R.aux.find(key);
+  if (found != R.aux.end()) {   // this layout was set up on this rank before: nothing to recompute
+    sh.ax = &found->second;
+    return TSV_OK;
+  }
+  ShardAux& ax = R.aux[key];
+  sh.ax = &ax;
+  TRY(qalloc(e, ax.T, s, std::max<size_t>(1, sh.nt) * m.B * m.ctx * 2));
+  TRY(qalloc(e, ax.txt, s, std::max<size_t>(1, sh.nt) * m.B * m.h * 4));
   const size_t rows = sh.nt + sh.ni;
   if (sh.nt)
     for (int b = 0; b < m.B; ++b)
-      CK(cudaMemcpyAsync(reinterpret_cast<uint16_t*>(sh.T.p) + (size_t)b * sh.nt * m.ctx,
+      CK(cudaMemcpyAsync(reinterpret_cast<uint16_t*>(ax.T.p) + (size_t)b * sh.nt * m.ctx,
                          R.T_host.data() + ((size_t)b * R.Lt + sh.t0) * m.ctx, sh.nt * m.ctx * 2,
                          cudaMemcpyHostToDevice, s.stream));
   if (m.sd3) {
-    TRY(qalloc(e, sh.pe, s, std::max<size_t>(1, sh.ni) * m.h * 4));
+    TRY(qalloc(e, ax.pe, s, std::max<size_t>(1, sh.ni) * m.h * 4));
     // patch (r, c) of the n_r x n_c grid sits at ((r + top) / q, (c + left) / q), q = pe_max / pe_base,
     // top = floor((pe_max - n_r) / 2) (floor toward -inf, S13)
     const int64_t n_r = R.height / 16, n_c = R.width / 16;
     auto floordiv2 = [](int64_t a) { return a >= 0 ? a / 2 : -((-a + 1) / 2); };
     ProfScope ps(e, s, KC_OTHER, 0.0, (double)sh.ni * m.h * 4.0);
-    sincos_pe_launch(reinterpret_cast<float*>(sh.pe.p), sh.i0, (int)sh.ni, n_c, floordiv2(m.d.pe_max - n_r),
+    sincos_pe_launch(reinterpret_cast<float*>(ax.pe.p), sh.i0, (int)sh.ni, n_c, floordiv2(m.d.pe_max - n_r),
                      floordiv2(m.d.pe_max - n_c), (double)m.d.pe_max / m.d.pe_base, m.h, s.stream);
   } else {
-    TRY(qalloc(e, sh.cosb, s, std::max<size_t>(1, rows) * (m.D / 2) * 4));
-    TRY(qalloc(e, sh.sinb, s, std::max<size_t>(1, rows) * (m.D / 2) * 4));
+    TRY(qalloc(e, ax.cosb, s, std::max<size_t>(1, rows) * (m.D / 2) * 4));
+    TRY(qalloc(e, ax.sinb, s, std::max<size_t>(1, rows) * (m.D / 2) * 4));
     ProfScope ps(e, s, KC_OTHER, 0.0, (double)rows * m.D * 4.0);
-    rope_table_launch(reinterpret_cast<float*>(sh.cosb.p), reinterpret_cast<float*>(sh.sinb.p), (int)sh.nt, sh.i0,
+    rope_table_launch(reinterpret_cast<float*>(ax.cosb.p), reinterpret_cast<float*>(ax.sinb.p), (int)sh.nt, sh.i0,
                       (int)sh.ni, R.width / 16, m.D, m.d.axes_dim, (double)m.d.theta, s.stream);
   }
   if (sh.nt) {
     GemmProblem pt[GEMM_MAX_PROBLEMS];
     for (int b = 0; b < m.B; ++b)
-      pt[b] = {reinterpret_cast<bf16*>(sh.T.p) + b * sh.nt * m.ctx, m.ctx, e->W(s, 2), m.ctx, (int)sh.nt,
-               epi_of(EPI_STORE_F32, reinterpret_cast<float*>(sh.txt.p) + b * sh.nt * m.h, m.h, e->W(s, 3))};
+      pt[b] = {reinterpret_cast<bf16*>(ax.T.p) + b * sh.nt * m.ctx, m.ctx, e->W(s, 2), m.ctx, (int)sh.nt,
+               epi_of(EPI_STORE_F32, reinterpret_cast<float*>(ax.txt.p) + b * sh.nt * m.h, m.h, e->W(s, 3))};
     TRY(gemm_multi(e, s, pt, m.B, m.h, m.ctx));
   }
   CK(cudaGetLastError());
@@ -902,8 +930,8 @@ static GemmEpi qk_fused(StepEnv& E, RankCtx& c, GemmEpi epi, int64_t r0, const b
   epi.qk_D = m.D;
   epi.gq = gq;
   epi.gk = gk;
-  epi.cosb = reinterpret_cast<const float*>(c.sh->cosb.p) + r0 * (m.D / 2);
-  epi.sinb = reinterpret_cast<const float*>(c.sh->sinb.p) + r0 * (m.D / 2);
+  epi.cosb = reinterpret_cast<const float*>(c.sh->ax->cosb.p) + r0 * (m.D / 2);
+  epi.sinb = reinterpret_cast<const float*>(c.sh->ax->sinb.p) + r0 * (m.D / 2);
   epi.k_sp = E.g->k;
   epi.pack = E.g->k > 1 ? c.pack + b * c.rows * 3 * m.h : nullptr;
   epi.pack_rows = (int)c.rows;
@@ -942,7 +970,7 @@ static tsv_status txt_embed(tsv_engine* e, Slot& s, const std::vector<ReqShard*>
   const int h = e->model.h;
   for (int b = 0; b < B; ++b) {
     ReqShard* sh = shq[b / per_req];
-    CK(cudaMemcpyAsync(x + b * R * h, reinterpret_cast<float*>(sh->txt.p) + (b % per_req) * nt * h,
+    CK(cudaMemcpyAsync(x + b * R * h, reinterpret_cast<float*>(sh->ax->txt.p) + (b % per_req) * nt * h,
                        nt * h * sizeof(float), cudaMemcpyDeviceToDevice, s.stream));
   }
   return TSV_OK;
@@ -1125,7 +1153,7 @@ static tsv_status run_step_sd3(StepEnv& E) {
           f32_to_bf16_launch(reinterpret_cast<float*>(c.shq[q]->lat.p), m.in, c.latb + q * c.ni * m.in, m.in,
                              (int)c.ni, m.in, s.stream);
         }
-        CK(cudaMemcpyAsync(xi, c.shq[q]->pe.p, c.ni * h * 4, cudaMemcpyDeviceToDevice, s.stream));
+        CK(cudaMemcpyAsync(xi, c.shq[q]->ax->pe.p, c.ni * h * 4, cudaMemcpyDeviceToDevice, s.stream));
         pi[q] = {c.latb + q * c.ni * m.in, m.in, e->W(s, 0), m.in, (int)c.ni, epi_of(EPI_ACCUM_F32, xi, h, e->W(s, 1))};
       }
       TRY(gemm_multi(e, s, pi, nq, h, m.in));
@@ -1268,8 +1296,11 @@ static tsv_status move_request(tsv_engine* e, Request& R, int gi) {
     // memory the old shard on this slot still reads)
     auto it = R.last.find(si);
     if (it != R.last.end()) CK(cudaStreamWaitEvent(s.stream, it->second, 0));
+    trace("move: setup_shard");
     TRY(setup_shard(e, R, si, g.local_positions[q], g.k, next[si]));
+    trace("move: ensure_reqdev");
     TRY(ensure_reqdev(e, R, si));
+    trace("move: slot done");
   }
   if (R.group < 0) {
     for (auto& kv : next) {
@@ -1328,6 +1359,7 @@ static tsv_status move_request(tsv_engine* e, Request& R, int gi) {
         }
       }
     }
+    trace("move: copies enqueued");
     // the old shards' buffers: released on their own streams once every new rank's copies (which
     // read them) are done -- stream-ordered, the host never waits
     for (auto& kv : next) TRY(record_last(e, R, kv.first));
@@ -1338,7 +1370,9 @@ static tsv_status move_request(tsv_engine* e, Request& R, int gi) {
         if (nk.first != kv.first) CK(cudaStreamWaitEvent(os.stream, R.last[nk.first], 0));
       kv.second.release();
     }
+    trace("move: old shards released");
     drop_request_graphs(e, R.id);   // cached step graphs reference the old shards' buffers
+    trace("move: graphs dropped");
   }
   R.shard.swap(next);
   R.group = gi;
@@ -1487,7 +1521,7 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
       for (size_t q = 0; q < Rs.size(); ++q) {
         const ReqShard* sh = c.shq[q];
         const ReqDev* rd = c.rdq[q];
-        const void* rp[] = {sh->lat.p, sh->vel.p, sh->T.p, sh->cosb.p, sh->sinb.p, sh->pe.p, rd->mod.p, rd->dt.p,
+        const void* rp[] = {sh->lat.p, sh->vel.p, sh->ax->T.p, sh->ax->cosb.p, sh->ax->sinb.p, sh->ax->pe.p, rd->mod.p, rd->dt.p,
                             rd->step.p};
         for (const void* p : rp) mix(reinterpret_cast<uintptr_t>(p));
         mix((uint64_t)Rs[q]->id);
@@ -1686,6 +1720,19 @@ static tsv_status ensure_init(tsv_engine* e) {
       uint64_t keep = UINT64_MAX;
       CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep));
       TRY(init_weights(e, *ds, s));
+      if (!e->alp()) {
+        // pre-grow the pool (TSV_POOL_RESERVE_MB, default 2 GiB: the per-request state of ~18 FLUX
+        // 2048^2 requests on a rank): growing it on a request's first landing maps new memory
+        // (tens of ms of host time) inside what should be an enqueue-only reshard call
+        const char* rv = getenv("TSV_POOL_RESERVE_MB");
+        const size_t mb = rv ? (size_t)atoll(rv) : 2048;
+        if (mb) {
+          void* p = nullptr;
+          CK(cudaMallocAsync(&p, mb << 20, s.stream));
+          CK(cudaFreeAsync(p, s.stream));
+          CK(cudaStreamSynchronize(s.stream));
+        }
+      }
       it = e->devs.emplace(s.device, std::move(ds)).first;
     }
     s.ds = it->second.get();
@@ -1757,6 +1804,7 @@ void tsv_engine_destroy(tsv_engine* e) {
   for (auto& kv : e->requests) {
     for (auto& d : kv.second.dev) release_reqdev(d.second);
     for (auto& sh : kv.second.shard) sh.second.release();
+    for (auto& ax : kv.second.aux) ax.second.release();
     for (auto& l : kv.second.last) cudaEventDestroy(l.second);
   }
   for (auto& g : e->groups) {
@@ -2186,6 +2234,7 @@ tsv_status tsv_request_destroy(tsv_engine* e, tsv_request r) {
   drop_request_graphs(e, r);
   for (auto& d : R.dev) release_reqdev(d.second);
   for (auto& sh : R.shard) sh.second.release();
+  for (auto& ax : R.aux) ax.second.release();
   e->requests.erase(it);
   return TSV_OK;
 }

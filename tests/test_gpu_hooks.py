@@ -76,24 +76,30 @@ def test_hooks_only_before_device_state(tsv):
 
 def test_reshard_does_not_block_the_host(tsv):
     """a13: request_reshard returns while the request's previous step is still running on the old
-    group (the copies are ordered on the device, old shards are released stream-ordered), and the
-    moved latent is bit-identical to the one an unmoved twin request holds."""
+    group (the copies are ordered on the device, old shards are released stream-ordered) -- both on a
+    first landing (per-GPU state set up on the new ranks) and on a return to ranks that already hold
+    the request (a pure latent move) -- and the moved latent is bit-identical to the one an unmoved
+    twin request holds."""
     eng = tsv.Engine("flux", devices=[0] * 4)
     g01, g23 = eng.group_create([0, 1]), eng.group_create([2, 3])
     ra = eng.request_create(2048, 2048, num_steps=20, seed=1600)
     rb = eng.request_create(2048, 2048, num_steps=20, seed=1600)
     for r in (ra, rb):
         eng.event_wait(eng.request_step(r, 0, g01))   # first landing + graph capture
-    ev = eng.request_step(ra, 1, g01)                 # ~0.2-0.4 s of device work
-    t0 = time.perf_counter()
-    eng.request_reshard(ra, g23)
-    host_ms = (time.perf_counter() - t0) * 1e3
-    running = not eng.event_query(ev)
-    eng.event_wait(eng.request_step(rb, 1, g01))
-    assert running, "the step finished before reshard returned: the call waited on the device"
-    assert host_ms < 50.0, host_ms
-    assert np.array_equal(eng.read_latent(ra), eng.read_latent(rb))
-    eng.event_wait(eng.request_step(ra, 2, g23))
-    eng.event_wait(eng.request_step(rb, 2, g01))
+    step = 1
+    for dst, bound_ms in ((g23, 50.0), (g01, 5.0), (g23, 5.0)):   # first landing on 2, 3; then returns
+        src = g01 if dst == g23 else g23
+        ev = eng.request_step(ra, step, src)            # ~0.2-0.4 s of device work
+        t0 = time.perf_counter()
+        eng.request_reshard(ra, dst)
+        host_ms = (time.perf_counter() - t0) * 1e3
+        running = not eng.event_query(ev)
+        eng.event_wait(eng.request_step(rb, step, g01))
+        assert running, "the step finished before reshard returned: the call waited on the device"
+        assert host_ms < bound_ms, (step, host_ms)
+        assert np.array_equal(eng.read_latent(ra), eng.read_latent(rb))
+        step += 1
+    eng.event_wait(eng.request_step(ra, step, g23))
+    eng.event_wait(eng.request_step(rb, step, g01))
     assert np.array_equal(eng.read_latent(ra), eng.read_latent(rb))   # same kernels, same bits
     eng.close()
