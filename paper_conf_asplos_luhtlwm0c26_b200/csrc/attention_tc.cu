@@ -115,9 +115,16 @@ struct FaCfg {
   static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // NK stages
   static constexpr int OFF_V = OFF_K + NK * KV_TILE;     // NV stages
   static constexpr int OFF_BAR = OFF_V + NV * KV_TILE;
+  static constexpr int NBAR = 1 + 2 * NK + 2 * NV + 3 * 2 + 1;   // mbarriers + the TMEM address slot
+  static_assert(NBAR * 8 <= 256, "barrier region");
   static constexpr int SMEM = OFF_BAR + 256 + 1024;      // barriers + 1 KB alignment slack
   static constexpr int O_COL = 256;
 };
+// setmaxnreg: the producer / MMA warpgroup drops to 80 registers, the two softmax warpgroups take
+// 208.  The CTA's pool is what the launch allocated -- 384 threads x the count ptxas fits under
+// __launch_bounds__(384, 1) (64K / 384 rounded down to 8 = 168) -- and an .inc blocks until the pool
+// has the registers, so the split must fit that pool (a 4-tile variant that over-asked hung).
+static_assert(80 * 128 + 208 * 256 <= ((65536 / 384) & ~7) * 384, "setmaxnreg split exceeds the pool");
 static_assert(FaCfg<128, 1>::SMEM <= 232448 && FaCfg<128, 2>::SMEM <= 232448 && FaCfg<64>::SMEM <= 232448,
               "attention shared memory > 227 KB");
 constexpr int FA_THREADS = 384;

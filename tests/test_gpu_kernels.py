@@ -284,7 +284,7 @@ def test_qk_norm_rope(tsv, H, D, rows, n_first):
 # ----------------------------------------------------------------------------- attention
 @pytest.mark.parametrize("impl", [0, 50, 51, 52, 53, 54, 61, 71, 81, 83])
 @pytest.mark.parametrize("L,H,D", [(1, 2, 64), (63, 4, 64), (320, 4, 64), (1000, 3, 128), (1536, 2, 128),
-                                   (4700, 1, 128)])
+                                   (4700, 1, 128), (1357, 3, 64)])
 def test_attention(tsv, L, H, D, impl):
     rng = np.random.default_rng(L + H + D)
     qkv = rng.standard_normal((L, 3, H, D)).astype(np.float32) * np.float32(1.5)
