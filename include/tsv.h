@@ -23,8 +23,8 @@
  *   - The engine owns all device memory (weights, latent shards, workspaces, communicators).
  *     The caller owns every host buffer it passes; host pointers are only read/written during
  *     the call (copies are synchronous with respect to the caller).
- *   - Handles are plain integers.  Requests are destroyed explicitly; groups and events live
- *     as long as the engine.
+ *   - Handles are plain integers.  Requests are destroyed explicitly, events may be released
+ *     (tsv_event_release); groups live as long as the engine.
  *   - Ranks.  An engine hosts "slots" = global SP ranks [rank_base, rank_base + n_local) on the
  *     listed CUDA devices (a device may repeat: virtual ranks on one GPU, used by the
  *     single-GPU SP tests).  world_size is the total number of ranks over all processes.  One
@@ -220,6 +220,9 @@ tsv_status tsv_request_reshard(tsv_engine* eng, tsv_request req, tsv_group group
  * give up, and the call then returns TSV_E_STATE (the step's results are invalid; the group must
  * be recreated). */
 tsv_status tsv_event_wait(tsv_engine* eng, tsv_event ev);
+/* Release an event handle (a serving loop releases each step's event once it is done with it); the
+ * handle may be returned again by a later call.  Waiting on a released handle: TSV_E_INVAL. */
+tsv_status tsv_event_release(tsv_engine* eng, tsv_event ev);
 tsv_status tsv_event_query(tsv_engine* eng, tsv_event ev, int* done);
 /* Device time between two events of the same group, max over the group's local ranks (ms). */
 tsv_status tsv_event_elapsed_ms(tsv_engine* eng, tsv_event start, tsv_event end, float* ms);

@@ -174,6 +174,9 @@ class Engine:
     def event_wait(self, ev: int):
         check(lib.tsv_event_wait(self.h, ev))
 
+    def event_release(self, ev: int):
+        check(lib.tsv_event_release(self.h, ev))
+
     def event_query(self, ev: int) -> bool:
         d = C.c_int()
         check(lib.tsv_event_query(self.h, ev, C.byref(d)))

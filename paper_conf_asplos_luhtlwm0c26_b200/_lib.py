@@ -70,6 +70,7 @@ _SIGS = {
     "tsv_request_step_batch": (_i32, [_p, _P(_i64), _i32, C.c_int32, _P(_i64)]),
     "tsv_request_reshard": (_i32, [_p, _i64, C.c_int32, _P(_i64)]),
     "tsv_event_wait": (_i32, [_p, _i64]),
+    "tsv_event_release": (_i32, [_p, _i64]),
     "tsv_event_query": (_i32, [_p, _i64, _P(_i32)]),
     "tsv_event_elapsed_ms": (_i32, [_p, _i64, _i64, _P(_f32)]),
     "tsv_group_record": (_i32, [_p, C.c_int32, _P(_i64)]),

@@ -357,6 +357,7 @@ struct tsv_engine {
   std::map<int64_t, Request> requests;
   int64_t next_req = 1;
   std::vector<EventRec> events;
+  std::vector<int64_t> free_events;   // released handles (tsv_event_release), reused by new_event
   ncclComm_t world_comm = nullptr;
   int64_t kernel_count = 0;
   // per-kernel-class profiling (tsv_engine_profile)
@@ -1381,6 +1382,8 @@ static tsv_status move_request(tsv_engine* e, Request& R, int gi) {
   return TSV_OK;
 }
 
+// Event handles index e->events; released handles (tsv_event_release) are reused, so a serving
+// loop that releases its step events keeps a bounded set of CUDA events.
 static tsv_status new_event(tsv_engine* e, const std::vector<int>& slots_, tsv_event* out, int gi = -1) {
   EventRec rec;
   rec.group = gi;
@@ -1392,8 +1395,16 @@ static tsv_status new_event(tsv_engine* e, const std::vector<int>& slots_, tsv_e
     CK(cudaEventRecord(ev, s.stream));
     rec.evs.push_back({si, ev});
   }
-  e->events.push_back(std::move(rec));
-  if (out) *out = (tsv_event)e->events.size() - 1;
+  int64_t id;
+  if (!e->free_events.empty()) {
+    id = e->free_events.back();
+    e->free_events.pop_back();
+    e->events[id] = std::move(rec);
+  } else {
+    e->events.push_back(std::move(rec));
+    id = (int64_t)e->events.size() - 1;
+  }
+  if (out) *out = (tsv_event)id;
   return TSV_OK;
 }
 
@@ -1533,6 +1544,7 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
     mix((uint64_t)gi);
     mix((uint64_t)Rs.size());
     mix((uint64_t)e->prof);   // a profiled graph carries event-record nodes around every launch
+    mix((uint64_t)E.fused * 2 + (uint64_t)E.ipc);   // the transport changes the epilogues and exchanges
     auto it = slot.graphs.find(key);
     if (it == slot.graphs.end()) {
       // bounded cache: evict the least recently used graph
@@ -2128,10 +2140,20 @@ static tsv_status check_ipc_barrier(tsv_engine* e, int gi) {
   return TSV_OK;
 }
 
+tsv_status tsv_event_release(tsv_engine* e, tsv_event ev) {
+  if (!e) return fail(TSV_E_INVAL, "null engine");
+  if (ev == -1) return TSV_OK;
+  if (ev < 0 || ev >= (int64_t)e->events.size() || e->events[ev].evs.empty()) return fail(TSV_E_INVAL, "unknown event");
+  for (auto& p : e->events[ev].evs) cudaEventDestroy(p.second);   // legal while pending (released when done)
+  e->events[ev].evs.clear();
+  e->free_events.push_back(ev);
+  return TSV_OK;
+}
+
 tsv_status tsv_event_wait(tsv_engine* e, tsv_event ev) {
   if (!e) return fail(TSV_E_INVAL, "null engine");
   if (ev == -1) return TSV_OK;
-  if (ev < 0 || ev >= (int64_t)e->events.size()) return fail(TSV_E_INVAL, "unknown event");
+  if (ev < 0 || ev >= (int64_t)e->events.size() || e->events[ev].evs.empty()) return fail(TSV_E_INVAL, "unknown event");
   for (auto& p : e->events[ev].evs) CK(cudaEventSynchronize(p.second));
   return check_ipc_barrier(e, e->events[ev].group);
 }
@@ -2139,7 +2161,7 @@ tsv_status tsv_event_wait(tsv_engine* e, tsv_event ev) {
 tsv_status tsv_event_query(tsv_engine* e, tsv_event ev, int* done) {
   if (!e || !done) return fail(TSV_E_INVAL, "null argument");
   if (ev == -1) { *done = 1; return TSV_OK; }
-  if (ev < 0 || ev >= (int64_t)e->events.size()) return fail(TSV_E_INVAL, "unknown event");
+  if (ev < 0 || ev >= (int64_t)e->events.size() || e->events[ev].evs.empty()) return fail(TSV_E_INVAL, "unknown event");
   *done = 1;
   for (auto& p : e->events[ev].evs) {
     cudaError_t q = cudaEventQuery(p.second);
@@ -2151,7 +2173,8 @@ tsv_status tsv_event_query(tsv_engine* e, tsv_event ev, int* done) {
 
 tsv_status tsv_event_elapsed_ms(tsv_engine* e, tsv_event a, tsv_event b, float* ms) {
   if (!e || !ms) return fail(TSV_E_INVAL, "null argument");
-  if (a < 0 || b < 0 || a >= (int64_t)e->events.size() || b >= (int64_t)e->events.size())
+  if (a < 0 || b < 0 || a >= (int64_t)e->events.size() || b >= (int64_t)e->events.size() || e->events[a].evs.empty() ||
+      e->events[b].evs.empty())
     return fail(TSV_E_INVAL, "unknown event");
   auto& ea = e->events[a].evs;
   auto& eb = e->events[b].evs;

@@ -343,3 +343,41 @@ def test_ln_impls_bitwise(tsv, model, monkeypatch):
     monkeypatch.setenv("TSV_LN_IMPL", "2")
     tsv.Engine(model, devices=[0]).close()   # restore the process-wide default (impl 2)
     assert np.array_equal(out[0][0], out[1][0]) and np.array_equal(out[0][1], out[1][1])
+
+
+def test_graph_key_includes_transport(tsv, monkeypatch):
+    """A cached step graph is specific to the Ulysses transport: after switching from the fused
+    epilogue stores to the exchange path the profiled step must run the exchange's all-to-all copies
+    (bytes > 0), not replay the fused graph.  Virtual ranks on one stream (graphs on)."""
+    monkeypatch.setenv("TSV_VIRTUAL_SERIAL", "1")
+    eng = tsv.Engine("tiny2", devices=[0, 0])
+    g = eng.group_create([0, 1])
+    r = eng.request_create(256, 256, num_steps=4, seed=1700)
+    eng.set_transport(True)
+    eng.profile(True)
+    eng.event_wait(eng.request_step(r, 0, g))
+    fused = eng.profile_read()["a2a"]
+    eng.set_transport(False)
+    eng.profile(True)
+    eng.event_wait(eng.request_step(r, 1, g))
+    exch = eng.profile_read()["a2a"]
+    eng.profile(False)
+    assert fused["bytes"] == 0 and exch["bytes"] > 0
+    eng.close()
+
+
+def test_event_release_reuses_handles(tsv):
+    eng = tsv.Engine("tiny", devices=[0])
+    g = eng.group_create([0])
+    r = eng.request_create(256, 256, num_steps=3, seed=1701)
+    e0 = eng.request_step(r, 0, g)
+    eng.event_wait(e0)
+    eng.event_release(e0)
+    with pytest.raises(tsv.TsvError) as e:
+        eng.event_wait(e0)
+    assert e.value.status == -1
+    e1 = eng.request_step(r, 1, g)
+    assert e1 == e0                        # the released handle is reused
+    eng.event_wait(e1)
+    assert eng.event_query(e1)
+    eng.close()
