@@ -796,9 +796,11 @@ static tsv_status a2a_exec(StepEnv& E, int which) {
         if (so.send && so.peer == d && seen++ == idx) { match = &so; break; }
       if (!match || match->rows != o.rows) return fail(TSV_E_STATE, "all-to-all plan mismatch");
       RankCtx& src = E.rc[p];
+      // UVA copy (cudaMemcpyDefault): peer or same-device, and capturable into a step graph
+      // (cudaMemcpyPeerAsync is not)
       for (int b = 0; b < B; ++b)
-        CK(cudaMemcpyPeerAsync(recvbuf(dst, b) + o.row0 * w, dst.s->device, sendbuf(src, b) + match->row0 * w,
-                               src.s->device, o.rows * w * 2, dst.s->stream));
+        CK(cudaMemcpyAsync(recvbuf(dst, b) + o.row0 * w, sendbuf(src, b) + match->row0 * w, o.rows * w * 2,
+                           cudaMemcpyDefault, dst.s->stream));
     }
     CK(cudaEventRecord(g.ev_b[d], dst.s->stream));
   }
