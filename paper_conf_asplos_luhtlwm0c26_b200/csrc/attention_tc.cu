@@ -104,7 +104,12 @@ __host__ __device__ constexpr uint32_t make_idesc_bf16_bmn(int M, int N) {
 // KV = 0: NK = NV = 2 (D = 128) / 4 (D = 64); KV = 1: NK = 3, NV = 2; KV = 2: NK = 2, NV = 3 (D = 128
 // fills the 227 KB of shared memory with 3 + 2 stages); KV = 3: one joint K+V ring (NK = NV stages,
 // one producer, a stage freed after both PV MMAs: round 1's design, kept where it measured better).
-template <int D, int KV = 0>
+// RS (rotating S buffers, D = 64 only): three 128-column S buffers shared by the two query tiles
+// (S index n = 2 j + t lives in buffer n % 3) instead of one per tile, so the MMA warp runs one S
+// ahead -- S_t(j+1) is computed while P_t(j) still waits for its PV MMA -- and a softmax warpgroup
+// finds its next scores ready instead of waiting for PV_t(j) + S_t(j+1) (at D = 64 the tensor work
+// of a tile, 512 cycles, is shorter than its softmax).  TMEM: 3 x 128 (S) + 2 x 64 (O) = 512.
+template <int D, int KV = 0, bool RS = false>
 struct FaCfg {
   static constexpr int NSUB = D / 64;
   static constexpr int Q_TILE = AT_BM * D * 2;
@@ -115,10 +120,12 @@ struct FaCfg {
   static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // NK stages
   static constexpr int OFF_V = OFF_K + NK * KV_TILE;     // NV stages
   static constexpr int OFF_BAR = OFF_V + NV * KV_TILE;
-  static constexpr int NBAR = 1 + 2 * NK + 2 * NV + 3 * 2 + 1;   // mbarriers + the TMEM address slot
+  static constexpr int NBAR = 1 + 2 * NK + 2 * NV + 3 + 2 + 2 + 2 + 1;   // mbarriers + the TMEM address slot
   static_assert(NBAR * 8 <= 256, "barrier region");
   static constexpr int SMEM = OFF_BAR + 256 + 1024;      // barriers + 1 KB alignment slack
-  static constexpr int O_COL = 256;
+  static constexpr int NSB = RS ? 3 : 2;                 // S buffers
+  static constexpr int O_COL = NSB * 128;
+  static_assert(O_COL + 2 * D <= 512, "TMEM columns (RS needs D = 64)");
 };
 // setmaxnreg: the producer / MMA warpgroup drops to 80 registers, the two softmax warpgroups take
 // 208.  The CTA's pool is what the launch allocated -- 384 threads x the count ptxas fits under
@@ -136,13 +143,13 @@ struct AttnSplitArgs {
   float* ws = nullptr;
 };
 
-template <int D, int NPOLY, int KV>
+template <int D, int NPOLY, int KV, bool RS = false>
 __global__ void __launch_bounds__(FA_THREADS, 1)
     attention_fa_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
                         float scale_log2, const __grid_constant__ AttnScatter sc,
                         const __grid_constant__ AttnSplitArgs sa) {
-  using C = FaCfg<D, KV>;
+  using C = FaCfg<D, KV, RS>;
   constexpr bool JOINT = KV == 3;   // K and V of a tile share one stage and one barrier pair
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -153,10 +160,11 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   uint64_t* k_empty = k_full + NK;                // [NK stages]
   uint64_t* v_full = k_empty + NK;                // [NV stages]
   uint64_t* v_empty = v_full + NV;                // [NV stages]
-  uint64_t* s_full = v_empty + NV;                // [2 q-tiles]
-  uint64_t* p_full = s_full + 2;                  // [2 q-tiles]
+  uint64_t* s_full = v_empty + NV;                // [3: per S buffer (RS) / per q-tile]
+  uint64_t* p_full = s_full + 3;                  // [2 q-tiles]
   uint64_t* o_done = p_full + 2;                  // [2 q-tiles]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(o_done + 3);
+  uint64_t* pv_done = o_done + 2;                 // [2 q-tiles] RS: PV_t(j) complete (a rescale's wait)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pv_done + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int head = blockIdx.y;
@@ -179,10 +187,11 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       mbar_init(&v_full[i], 1);
       mbar_init(&v_empty[i], 1);
     }
+    for (int i = 0; i < 3; ++i) mbar_init(&s_full[i], 1);
     for (int i = 0; i < 2; ++i) {
-      mbar_init(&s_full[i], 1);
       mbar_init(&p_full[i], 128);
       mbar_init(&o_done[i], 1);
+      mbar_init(&pv_done[i], 1);
     }
     fence_mbar_init();
   }
@@ -244,16 +253,19 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     const uint64_t dk0 = make_sw128_desc(smem_u32(sm + C::OFF_K));
     const uint64_t dv0 = make_sw128_mn_desc(smem_u32(sm + C::OFF_V), AT_BN * 128);
     mbar_wait(q_full, 0);
+    // S buffer of S index n = 2 j + t: the tile's own (t) or, RS, the rotating n % 3
+    auto sbuf = [](int t, int j) { return RS ? (2 * j + t) % 3 : t; };
     auto issue_s = [&](int t, int j) {   // t == 1 releases the K stage (both S MMAs of tile j issued)
       const uint64_t dq = dq0 + (uint64_t)((t * C::Q_TILE) >> 4);
       const uint64_t dk = dk0 + (uint64_t)(((j % NK) * C::KV_TILE) >> 4);
+      const int b = sbuf(t, j);
       if (elect_one()) {
 #pragma unroll
         for (int kk = 0; kk < D / 16; ++kk) {
           const uint32_t off = ((kk >> 2) * (AT_BM * 128) + (kk & 3) * 32) >> 4;
-          umma_bf16_ss(tmem + t * 128, dq + off, dk + off, idesc_s, kk > 0);
+          umma_bf16_ss(tmem + b * 128, dq + off, dk + off, idesc_s, kk > 0);
         }
-        umma_commit(&s_full[t]);
+        umma_commit(&s_full[b]);
         if (t == 1 && !JOINT) umma_commit(&k_empty[j % NK]);
       }
       __syncwarp();
@@ -265,25 +277,52 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       tc_fence_after();
       if (elect_one()) {
 #pragma unroll
+        const int b = sbuf(t, j);
+#pragma unroll
         for (int kk = 0; kk < AT_BN / 16; ++kk)
-          umma_bf16_ts(tmem + C::O_COL + t * D, tmem + t * 128 + kk * 8, dv + (uint64_t)(kk * (2048 >> 4)), idesc_o,
+          umma_bf16_ts(tmem + C::O_COL + t * D, tmem + b * 128 + kk * 8, dv + (uint64_t)(kk * (2048 >> 4)), idesc_o,
                        (j | kk) != 0);
+        if (RS) umma_commit(&pv_done[t]);
         if (t == 1) umma_commit(JOINT ? &k_empty[j % NK] : &v_empty[j % NV]);
       }
       __syncwarp();
     };
-    for (int j = 0; j < n_tiles; ++j) {
-      mbar_wait(&k_full[j % NK], (j / NK) & 1);
-      tc_fence_after();
-      for (int t = 0; t < 2; ++t) {
-        if (j > 0) issue_pv(t, j - 1);
-        issue_s(t, j);
+    if constexpr (RS) {
+      // S indices 0, 1, 2 up front; then each PV (S index m) is followed by S index m + 3, which
+      // reuses the buffer that PV just read (the in-order tcgen05 pipe orders the two)
+      auto s_at = [&](int m) {
+        const int jj = m >> 1, tt = m & 1;
+        if (jj >= n_tiles) return;
+        if (tt == 0) {
+          mbar_wait(&k_full[jj % NK], (jj / NK) & 1);
+          tc_fence_after();
+        }
+        issue_s(tt, jj);
+      };
+      for (int m = 0; m < 3; ++m) s_at(m);
+      for (int j = 0; j < n_tiles; ++j)
+        for (int t = 0; t < 2; ++t) {
+          issue_pv(t, j);
+          if (j == n_tiles - 1) {
+            if (elect_one()) umma_commit(&o_done[t]);
+            __syncwarp();
+          }
+          s_at(2 * j + t + 3);
+        }
+    } else {
+      for (int j = 0; j < n_tiles; ++j) {
+        mbar_wait(&k_full[j % NK], (j / NK) & 1);
+        tc_fence_after();
+        for (int t = 0; t < 2; ++t) {
+          if (j > 0) issue_pv(t, j - 1);
+          issue_s(t, j);
+        }
       }
-    }
-    for (int t = 0; t < 2; ++t) {
-      issue_pv(t, n_tiles - 1);
-      if (elect_one()) umma_commit(&o_done[t]);
-      __syncwarp();
+      for (int t = 0; t < 2; ++t) {
+        issue_pv(t, n_tiles - 1);
+        if (elect_one()) umma_commit(&o_done[t]);
+        __syncwarp();
+      }
     }
    }
   } else {
@@ -293,7 +332,6 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     const int wq = (warp - 4) & 3;
     const int row = wq * 32 + lane;
     const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
-    const uint32_t s_col = tmem + lane_base + t * 128;
     const uint32_t o_col = tmem + lane_base + C::O_COL + t * D;
     float m_ref = -FLT_MAX, l_sum = 0.f;
     auto hand_over = [&]() {   // P_t(j) is in TMEM: release it to the MMA warp
@@ -302,7 +340,11 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       mbar_arrive(&p_full[t]);   // (one arrival per warp after __syncwarp measured no faster)
     };
     for (int j = 0; j < n_tiles; ++j) {
-      mbar_wait(&s_full[t], j & 1);
+      // this tile's S (and then P) buffer: its own, or (RS) buffer (2 j + t) % 3, used for the
+      // ((2 j + t) / 3)-th time
+      const int sb = RS ? (2 * j + t) % 3 : t;
+      const uint32_t s_col = tmem + lane_base + sb * 128;
+      mbar_wait(&s_full[sb], (RS ? (2 * j + t) / 3 : j) & 1);
       tc_fence_after();
       uint32_t sr[4][32];
       const int kbase = (j0 + j) * AT_BN;
@@ -393,8 +435,14 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         }
       if (__any_sync(0xffffffffu, rescale)) {
         // S_t(j) complete => PV_t(j-1) complete (in-order pipe): O_t can be rescaled now, before
-        // P_t(j) is handed over.  tcgen05.ld/st are warp-collective: the whole warp's rows are
-        // rescaled together (alpha = 1 for rows that did not need it).
+        // P_t(j) is handed over.  RS issues S_t(j) ahead of PV_t(j-1), so it waits for PV_t(j-1)
+        // explicitly (the j-th completion of pv_done[t]; PV_t(j) cannot complete before P_t(j)).
+        // tcgen05.ld/st are warp-collective: the whole warp's rows are rescaled together (alpha = 1
+        // for rows that did not need it).
+        if (RS) {
+          mbar_wait(&pv_done[t], (j - 1) & 1);
+          tc_fence_after();
+        }
 #pragma unroll
         for (int c = 0; c < D / 32; ++c) {
           uint32_t ov[32];
@@ -558,7 +606,7 @@ static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L
   return r == CUDA_SUCCESS ? 0 : -2;
 }
 
-template <int D, int NP, int KV = 0>
+template <int D, int NP, int KV = 0, bool RS = false>
 static cudaError_t launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o,
                              long long ldo, int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s,
                              const AttnSplitArgs& sa) {
@@ -566,14 +614,14 @@ static cudaError_t launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const
   int dev = 0;
   cudaGetDevice(&dev);
   if (!(done >> dev & 1ull)) {
-    cudaError_t e = cudaFuncSetAttribute(attention_fa_kernel<D, NP, KV>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, FaCfg<D, KV>::SMEM);
+    cudaError_t e = cudaFuncSetAttribute(attention_fa_kernel<D, NP, KV, RS>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, FaCfg<D, KV, RS>::SMEM);
     if (e != cudaSuccess) return e;
     done |= 1ull << dev;
   }
   dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H, sa.nsplit);
-  return launch_pdl(attention_fa_kernel<D, NP, KV>, grid, dim3(FA_THREADS), FaCfg<D, KV>::SMEM, s, tq, tk, tv, o,
-                    ldo, L, scale_log2, sc, sa);
+  return launch_pdl(attention_fa_kernel<D, NP, KV, RS>, grid, dim3(FA_THREADS), FaCfg<D, KV, RS>::SMEM, s, tq, tk, tv,
+                    o, ldo, L, scale_log2, sc, sa);
 }
 
 // KV-split factor for a launch of C = ceil(L/256) x H CTAs: the S in 1..8 minimising the estimated
@@ -629,9 +677,10 @@ static int default_version(int D) {
   if (r < 0) {
     const char* e = getenv(D == 128 ? "TSV_ATTN_D128" : "TSV_ATTN_D64");
     // D = 128: separate K / V rings, 1 of 8 exp2 pairs by polynomial; D = 64: the joint ring (the split
-    // rings measured -2 % on the SD3 1024^2 step), 3 of 8 (round-2 sweeps, profiles/r02)
-    r = e ? atoi(e) : (D == 128 ? 51 : 83);
-    if (r < 50 || r > 89) r = D == 128 ? 51 : 83;
+    // rings measured -2 % on the SD3 1024^2 step) with rotating S buffers, 2 of 8 (round-2 sweeps,
+    // profiles/r02)
+    r = e ? atoi(e) : (D == 128 ? 51 : 92);
+    if (r < 50 || r > 99) r = D == 128 ? 51 : 92;
   }
   return r;
 }
@@ -646,8 +695,19 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     return -1;
   const float scale_log2 = (1.0f / sqrtf((float)D)) * 1.4426950408889634f;
   const AttnSplitArgs sa = plan_kv_split(L, H, D, spw);
-  // version = 50 + n: n of 8 exp2 pairs by polynomial
   cudaError_t e;
+  if constexpr (D == 64) {
+    // 90 + n (D = 64): rotating S buffers (RS) on the joint K+V ring, n of 8 exp2 pairs by polynomial
+    switch (version) {
+      case 91: return launch_fa<D, 1, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
+      case 92: return launch_fa<D, 2, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
+      case 93: return launch_fa<D, 3, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
+      case 94: return launch_fa<D, 4, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
+      case 99: return launch_fa<D, 9, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
+      default: break;
+    }
+  }
+  // version = 50 + n: n of 8 exp2 pairs by polynomial
   switch (version) {
     case 50: e = launch_fa<D, 0>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 51: e = launch_fa<D, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
