@@ -33,6 +33,7 @@
 // 192 B/clk); P handed over in two halves; CTA-pair (cta_group::2) tiles (-17 %: the pair couples
 // both CTAs' softmax chains); two softmax warps per row; packed ex2 (two MUFU ops per instruction).
 #include <cfloat>
+#include <cstdio>
 #include <cstdlib>
 #include <cudaTypedefs.h>
 
@@ -120,9 +121,9 @@ struct FaCfg {
   static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // NK stages
   static constexpr int OFF_V = OFF_K + NK * KV_TILE;     // NV stages
   static constexpr int OFF_BAR = OFF_V + NV * KV_TILE;
-  static constexpr int NBAR = 1 + 2 * NK + 2 * NV + 3 + 2 + 2 + 2 + 1;   // mbarriers + the TMEM address slot
-  static_assert(NBAR * 8 <= 256, "barrier region");
-  static constexpr int SMEM = OFF_BAR + 256 + 1024;      // barriers + 1 KB alignment slack
+  static constexpr int NBAR = 1 + 2 * NK + 2 * NV + 3 + 6 + 2 + 6 + 1;   // mbarriers + the TMEM address slot
+  static_assert(NBAR * 8 <= 512, "barrier region");
+  static constexpr int SMEM = OFF_BAR + 512 + 1024;      // barriers + 1 KB alignment slack
   static constexpr int NSB = RS ? 3 : 2;                 // S buffers
   static constexpr int O_COL = NSB * 128;
   static_assert(O_COL + 2 * D <= 512, "TMEM columns (RS needs D = 64)");
@@ -160,12 +161,19 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   uint64_t* k_empty = k_full + NK;                // [NK stages]
   uint64_t* v_full = k_empty + NK;                // [NV stages]
   uint64_t* v_empty = v_full + NV;                // [NV stages]
+  // RS lets the warps of one softmax warpgroup drift up to two tiles apart (S_t(j+1), S_t(j+2) can be
+  // ready before PV_t(j) consumed P_t(j)), so the per-tile barriers that see arrivals or waits from
+  // several of a warpgroup's tiles at once come in three copies, tile j using copy j % 3 (phase
+  // (j / 3) & 1): one barrier would mix a fast warp's arrival for tile j+1 into tile j's phase.
   uint64_t* s_full = v_empty + NV;                // [3: per S buffer (RS) / per q-tile]
-  uint64_t* p_full = s_full + 3;                  // [2 q-tiles]
-  uint64_t* o_done = p_full + 2;                  // [2 q-tiles]
-  uint64_t* pv_done = o_done + 2;                 // [2 q-tiles] RS: PV_t(j) complete (a rescale's wait)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pv_done + 2);
+  uint64_t* p_full = s_full + 3;                  // [2 q-tiles][3]
+  uint64_t* o_done = p_full + 6;                  // [2 q-tiles]
+  uint64_t* pv_done = o_done + 2;                 // [2 q-tiles][3] RS: PV_t(j) complete (a rescale's wait)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pv_done + 6);
 
+  // tile j's copy of a per-tile barrier of q-tile t, and the phase parity to wait for
+  auto tb = [](uint64_t* base, int t, int j) { return base + t * 3 + (RS ? j % 3 : 0); };
+  auto tpar = [](int j) { return (uint32_t)((RS ? j / 3 : j) & 1); };
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int head = blockIdx.y;
   const int q0 = blockIdx.x * 2 * AT_BM;
@@ -188,11 +196,11 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       mbar_init(&v_empty[i], 1);
     }
     for (int i = 0; i < 3; ++i) mbar_init(&s_full[i], 1);
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < 6; ++i) {
       mbar_init(&p_full[i], 128);
-      mbar_init(&o_done[i], 1);
       mbar_init(&pv_done[i], 1);
     }
+    for (int i = 0; i < 2; ++i) mbar_init(&o_done[i], 1);
     fence_mbar_init();
   }
   if (warp == 2) tmem_alloc<512>(tmem_slot);
@@ -273,16 +281,22 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     auto issue_pv = [&](int t, int j) {   // t == 0 waits for the V tile, t == 1 releases it
       const uint64_t dv = dv0 + (uint64_t)(((j % NV) * C::KV_TILE) >> 4);
       if (t == 0 && !JOINT) mbar_wait(&v_full[j % NV], (j / NV) & 1);
-      mbar_wait(&p_full[t], j & 1);
+#ifdef TSV_ATTN_DEBUG
+      if (!mbar_wait_bounded(tb(p_full, t, j), tpar(j), 1 << 22)) {
+        if (lane == 0) printf("p_full hang: blk %d head %d t %d j %d\n", blockIdx.x, head, t, j);
+        __trap();
+      }
+#else
+      mbar_wait(tb(p_full, t, j), tpar(j));
+#endif
       tc_fence_after();
       if (elect_one()) {
-#pragma unroll
         const int b = sbuf(t, j);
 #pragma unroll
         for (int kk = 0; kk < AT_BN / 16; ++kk)
           umma_bf16_ts(tmem + C::O_COL + t * D, tmem + b * 128 + kk * 8, dv + (uint64_t)(kk * (2048 >> 4)), idesc_o,
                        (j | kk) != 0);
-        if (RS) umma_commit(&pv_done[t]);
+        if (RS) umma_commit(tb(pv_done, t, j));
         if (t == 1) umma_commit(JOINT ? &k_empty[j % NK] : &v_empty[j % NV]);
       }
       __syncwarp();
@@ -334,17 +348,24 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
     const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
     const uint32_t o_col = tmem + lane_base + C::O_COL + t * D;
     float m_ref = -FLT_MAX, l_sum = 0.f;
-    auto hand_over = [&]() {   // P_t(j) is in TMEM: release it to the MMA warp
+    auto hand_over = [&](int j) {   // P_t(j) is in TMEM: release it to the MMA warp
       tmem_st_wait();
       tc_fence_before();
-      mbar_arrive(&p_full[t]);   // (one arrival per warp after __syncwarp measured no faster)
+      mbar_arrive(tb(p_full, t, j));   // (one arrival per warp after __syncwarp measured no faster)
     };
     for (int j = 0; j < n_tiles; ++j) {
       // this tile's S (and then P) buffer: its own, or (RS) buffer (2 j + t) % 3, used for the
       // ((2 j + t) / 3)-th time
       const int sb = RS ? (2 * j + t) % 3 : t;
       const uint32_t s_col = tmem + lane_base + sb * 128;
+#ifdef TSV_ATTN_DEBUG
+      if (!mbar_wait_bounded(&s_full[sb], (RS ? (2 * j + t) / 3 : j) & 1, 1 << 22)) {
+        if (lane == 0) printf("s_full hang: blk %d head %d t %d j %d sb %d\n", blockIdx.x, head, t, j, sb);
+        __trap();
+      }
+#else
       mbar_wait(&s_full[sb], (RS ? (2 * j + t) / 3 : j) & 1);
+#endif
       tc_fence_after();
       uint32_t sr[4][32];
       const int kbase = (j0 + j) * AT_BN;
@@ -387,7 +408,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
           l_sum += ts;
           tmem_st32(s_col, sr[0]);
           tmem_st32(s_col + 32, sr[1]);
-          hand_over();
+          hand_over(j);
           continue;
         }
       }
@@ -436,11 +457,18 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       if (__any_sync(0xffffffffu, rescale)) {
         // S_t(j) complete => PV_t(j-1) complete (in-order pipe): O_t can be rescaled now, before
         // P_t(j) is handed over.  RS issues S_t(j) ahead of PV_t(j-1), so it waits for PV_t(j-1)
-        // explicitly (the j-th completion of pv_done[t]; PV_t(j) cannot complete before P_t(j)).
+        // explicitly (pv_done copy (j - 1) % 3; PV_t(j+2) cannot complete before P_t(j+2)).
         // tcgen05.ld/st are warp-collective: the whole warp's rows are rescaled together (alpha = 1
         // for rows that did not need it).
         if (RS) {
-          mbar_wait(&pv_done[t], (j - 1) & 1);
+#ifdef TSV_ATTN_DEBUG
+          if (!mbar_wait_bounded(tb(pv_done, t, j - 1), tpar(j - 1), 1 << 22)) {
+            if (lane == 0) printf("RS pv_done hang: blk %d head %d t %d j %d\n", blockIdx.x, head, t, j);
+            __trap();
+          }
+#else
+          mbar_wait(tb(pv_done, t, j - 1), tpar(j - 1));
+#endif
           tc_fence_after();
         }
 #pragma unroll
@@ -455,7 +483,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       }
       tmem_st32(s_col, sr[0]);
       tmem_st32(s_col + 32, sr[1]);
-      hand_over();
+      hand_over(j);
       const float2 l01 = __fadd2_rn(lsum[0], lsum[1]), l23 = __fadd2_rn(lsum[2], lsum[3]);
       const float2 l4 = __fadd2_rn(l01, l23);
       l_sum += l4.x + l4.y;

@@ -50,6 +50,23 @@ TSV_DEV void mbar_wait(uint64_t* bar, uint32_t parity) {
       : "memory");
 }
 
+// Bounded wait (diagnostics): false after ~`tries` polls instead of hanging
+TSV_DEV bool mbar_wait_bounded(uint64_t* bar, uint32_t parity, long long tries) {
+  uint32_t addr = smem_u32(bar);
+  for (long long i = 0; i < tries; ++i) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred P1;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%1], %2, 1000;\n\t"
+        "selp.b32 %0, 1, 0, P1;\n\t}\n"
+        : "=r"(ok)
+        : "r"(addr), "r"(parity)
+        : "memory");
+    if (ok) return true;
+  }
+  return false;
+}
+
 // ------------------------------------------------------------------ TMA
 TSV_DEV void tma_prefetch_desc(const CUtensorMap* m) {
   asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(m)) : "memory");

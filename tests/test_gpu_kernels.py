@@ -423,3 +423,26 @@ def test_attention_score_jump(tsv, D, impl, jump):
     got = _np(o).reshape(L, H, D)
     assert np.all(np.isfinite(got))
     assert _rel(got, ref) < 2e-2
+
+
+@pytest.mark.parametrize("impl", [0, 83, 92, 51])
+def test_attention_large_logits_many_rescales(tsv, impl):
+    """Scores with a large spread (q, k ~ 8 N(0, 1)): most key tiles overflow the lazy bound and take
+    the exact path with an O rescale, so the softmax warps of a warpgroup drift apart by tiles -- the
+    case that exposed a barrier-phase race in the rotating-S variant (impl 92).  SD3 1024^2 shape
+    (L = 4429, H = 24), two heads checked against the float64 definition."""
+    L, H = 4429, 24
+    D = 128 if impl == 51 else 64
+    g = torch.Generator(device="cuda").manual_seed(impl)
+    qkv = (torch.randn(L, 3 * H * D, device="cuda", generator=g) * 8.0).to(torch.bfloat16)
+    o = torch.zeros(L, H * D, dtype=torch.bfloat16, device="cuda")
+    ld = 3 * H * D
+    tsv.op_attention(qkv, qkv[:, H * D:], qkv[:, 2 * H * D:], o, L, H, D, ldq=ld, ldk=ld, ldv=ld, impl=impl)
+    torch.cuda.synchronize()
+    t = qkv.view(L, 3, H, D)
+    for hh in (0, H - 1):
+        q, k, v = (t[:, i, hh].double().cpu().numpy()[:, None, :] for i in range(3))
+        ref = F.attention(q, k, v)[:, 0]
+        got = o.view(L, H, D)[:, hh].double().cpu().numpy()
+        assert _rel(got, ref) < 2e-2, hh
+        assert np.sum(got * ref) / np.linalg.norm(got) / np.linalg.norm(ref) > 0.999
