@@ -99,6 +99,7 @@ def main():
            "efficiency_range": {"low (450 GB/s, 20 us)": err_lo, "high (900 GB/s, 5 us)": err_hi},
            "a2a_model": {"bw_gbs": args.bw, "lat_us": args.lat_us, "overlap": "none (serial)"},
            "measured_virtual_ms": [[round(float(x), 4) for x in r] for r in ms],
+           "measured_cv": [[round(float(x), 5) for x in r] for r in cv],
            "note": "k=1 measured on one B200; k>1 = (k virtual ranks on one B200) / k + modeled NVLink all-to-all"
                    + ("; virtual ranks serialised on one stream (each kernel alone on the GPU, as on a rank's own "
                       "GPU)" if args.serial else "; virtual ranks on concurrent streams (overlap: optimistic for "
