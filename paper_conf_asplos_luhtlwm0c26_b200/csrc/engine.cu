@@ -308,6 +308,11 @@ struct Group {
   int win_evals = 0;
   DevBuf win_recv, win_cat, win_flags;
   bool ipc_failed = false;  // the device barrier gave up on a stalled member (check_ipc_barrier)
+  // multi-stream step graphs (several local ranks on their own streams): fork / join events per
+  // local member, and a switch-off if capturing this group's step ever failed
+  std::vector<cudaEvent_t> ev_pre, ev_join;
+  cudaEvent_t ev_fork = nullptr, ev_post = nullptr;
+  bool no_graph = false;
   std::vector<void*> peer_recv, peer_cat, peer_flags;  // by group rank (own entry = own window)
   std::vector<void*> opened;                           // IPC mappings to close
 };
@@ -1519,11 +1524,33 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
       CK(cudaMemcpyAsync(c.rdq[q]->step.p, &st, sizeof(int), cudaMemcpyHostToDevice, c.s->stream));
     }
   }
-  // one local rank, or several virtual ranks sharing one stream (TSV_VIRTUAL_SERIAL): replay (or
-  // capture once) the whole step as a CUDA graph on that stream
-  bool one_stream = true;
-  for (auto& c : E.rc) one_stream = one_stream && c.s->stream == E.rc[0].s->stream;
-  if (e->graphs && one_stream) {
+  // Replay (or capture once) the whole step as one CUDA graph launched on the first local rank's
+  // stream ("origin").  Local ranks on other streams (several ranks in this process: virtual ranks
+  // on one GPU, or GPUs of one process) are forked from and joined back to the origin inside the
+  // capture, so their kernels and the cross-rank event edges of the transports become one
+  // multi-stream (multi-device) graph; around the launch the other streams hand their order to the
+  // origin and take it back.
+  cudaStream_t origin = E.rc[0].s->stream;
+  std::vector<int> others;   // indices into E.rc of the ranks on streams other than the origin
+  for (size_t i = 0; i < E.rc.size(); ++i) {
+    bool seen = E.rc[i].s->stream == origin;
+    for (int o : others) seen = seen || E.rc[o].s->stream == E.rc[i].s->stream;
+    if (!seen) others.push_back((int)i);
+  }
+  const bool multi = !others.empty();
+  if (multi && g.ev_pre.empty()) {
+    g.ev_pre.assign(E.rc.size(), nullptr);
+    g.ev_join.assign(E.rc.size(), nullptr);
+    for (int o : others) {
+      CK(cudaSetDevice(E.rc[o].s->device));
+      CK(cudaEventCreateWithFlags(&g.ev_pre[o], cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&g.ev_join[o], cudaEventDisableTiming));
+    }
+    CK(cudaSetDevice(E.rc[0].s->device));
+    CK(cudaEventCreateWithFlags(&g.ev_fork, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&g.ev_post, cudaEventDisableTiming));
+  }
+  if (e->graphs && !g.no_graph) {
     // cached per (first) slot by every buffer the step references
     Slot& slot = *E.rc[0].s;
     uint64_t key = 1469598103934665603ull;
@@ -1566,9 +1593,42 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
       int64_t l0[8];
       for (int i = 0; i < 8; ++i) { f0[i] = e->prof_flops[i]; b0[i] = e->prof_bytes[i]; l0[i] = e->prof_launch[i]; }
       CK(cudaStreamBeginCapture(slot.stream, cudaStreamCaptureModeThreadLocal));
-      tsv_status st = run_step(E);
+      tsv_status st = TSV_OK;
+      cudaError_t fe = cudaSuccess;
+      if (multi) {   // fork the other ranks' streams into the capture
+        if ((fe = cudaEventRecord(g.ev_fork, origin)) == cudaSuccess)
+          for (int o : others)
+            if (fe == cudaSuccess) {
+              cudaSetDevice(E.rc[o].s->device);
+              fe = cudaStreamWaitEvent(E.rc[o].s->stream, g.ev_fork, 0);
+            }
+      }
+      if (fe == cudaSuccess) st = run_step(E);
+      if (multi && fe == cudaSuccess && st == TSV_OK) {   // join them back
+        for (int o : others)
+          if (fe == cudaSuccess) {
+            cudaSetDevice(E.rc[o].s->device);
+            if ((fe = cudaEventRecord(g.ev_join[o], E.rc[o].s->stream)) == cudaSuccess) {
+              cudaSetDevice(slot.device);
+              fe = cudaStreamWaitEvent(origin, g.ev_join[o], 0);
+            }
+          }
+      }
+      cudaSetDevice(slot.device);
       cudaGraph_t graph = nullptr;
       cudaError_t ce = cudaStreamEndCapture(slot.stream, &graph);
+      if (multi && (fe != cudaSuccess || ce != cudaSuccess)) {
+        // this group's step cannot be captured across its streams (e.g. a driver without
+        // multi-device capture): launch it directly from now on
+        if (graph) cudaGraphDestroy(graph);
+        cudaGetLastError();
+        e->prof_recs.resize(r0);
+        for (int i = 0; i < 8; ++i) { e->prof_flops[i] = f0[i]; e->prof_bytes[i] = b0[i]; e->prof_launch[i] = l0[i]; }
+        e->kernel_count = k0;
+        g.no_graph = true;
+        TRY(run_step(E));
+        goto stepped;
+      }
       // what ProfScope recorded during capture belongs to the graph: re-added at every replay
       gr.prof.assign(e->prof_recs.begin() + r0, e->prof_recs.end());
       e->prof_recs.resize(r0);
@@ -1589,7 +1649,22 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
     }
     StepGraph& gr = it->second;
     gr.last_use = ++e->graph_clock;
+    if (multi)   // the origin follows the other ranks' work so far (their step-index copies included)
+      for (int o : others) {
+        CK(cudaSetDevice(E.rc[o].s->device));
+        CK(cudaEventRecord(g.ev_pre[o], E.rc[o].s->stream));
+        CK(cudaSetDevice(slot.device));
+        CK(cudaStreamWaitEvent(origin, g.ev_pre[o], 0));
+      }
+    CK(cudaSetDevice(slot.device));
     CK(cudaGraphLaunch(gr.exec, slot.stream));
+    if (multi) {   // and the other ranks' streams follow the graph
+      CK(cudaEventRecord(g.ev_post, origin));
+      for (int o : others) {
+        CK(cudaSetDevice(E.rc[o].s->device));
+        CK(cudaStreamWaitEvent(E.rc[o].s->stream, g.ev_post, 0));
+      }
+    }
     e->kernel_count += gr.kernels;
     if (e->prof) {
       // the graph's event pairs now hold this replay's timestamps
@@ -1603,6 +1678,7 @@ static tsv_status do_step(tsv_engine* e, const std::vector<Request*>& Rs, int gi
   } else {
     TRY(run_step(E));
   }
+stepped:
   for (Request* R : Rs) {
     for (auto& c : E.rc) TRY(record_last(e, *R, c.si));
     R->next_step++;
@@ -1827,6 +1903,10 @@ void tsv_engine_destroy(tsv_engine* e) {
     if (g.comm) ncclCommDestroy(g.comm);
     for (auto ev : g.ev_a) cudaEventDestroy(ev);
     for (auto ev : g.ev_b) cudaEventDestroy(ev);
+    for (auto ev : g.ev_pre) if (ev) cudaEventDestroy(ev);
+    for (auto ev : g.ev_join) if (ev) cudaEventDestroy(ev);
+    if (g.ev_fork) cudaEventDestroy(g.ev_fork);
+    if (g.ev_post) cudaEventDestroy(g.ev_post);
   }
   if (e->world_comm) ncclCommDestroy(e->world_comm);
   for (auto& rec : e->events)

@@ -125,6 +125,24 @@ def test_sd3_512_golden(tsv, sd3_engine):
         eng.request_destroy(req)
 
 
+def test_sd3_1024_golden(tsv, sd3_engine):
+    """Config 5's 1024^2 SD3 request (L = 4096 + 333, CFG pair) at step 0 of 20 against the float64
+    oracle (tests/golden/sd3_1024_seed1000_S20.npz, tools/make_golden.py sd3_1024), SP = 1 and 8."""
+    p = os.path.join(ROOT, "tests", "golden", "sd3_1024_seed1000_S20.npz")
+    if not os.path.exists(p):
+        pytest.skip("golden sd3_1024_seed1000_S20.npz not generated (tools/make_golden.py sd3_1024)")
+    gold = np.load(p)
+    eng = sd3_engine
+    for ranks in ([0], [0, 1, 2, 3, 4, 5, 6, 7]):
+        g = eng.group_create(ranks)
+        req = eng.request_create(1024, 1024, num_steps=20, seed=1000)
+        eng.event_wait(eng.request_step(req, 0, g))
+        for got, ref in ((eng.read_velocity(req), gold["v"]), (eng.read_latent(req), gold["x_next"])):
+            rel, cos = _metrics(got.astype(np.float64), ref.astype(np.float64))
+            assert rel <= TOL_REL and cos >= TOL_COS, (ranks, rel, cos)
+        eng.request_destroy(req)
+
+
 def test_sd3_latency_table(tsv, sd3_engine):
     ms, cv = sd3_engine.latency_table([512, 1024], [1, 2], warmup=1, iters=3)
     assert ms.shape == (2, 2) and np.all(ms > 0)

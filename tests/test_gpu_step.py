@@ -230,6 +230,23 @@ def test_flux_2048_step_vs_golden(tsv, k):
     eng.close()
 
 
+def test_flux_1024_sp_degrees_vs_golden(tsv):
+    """BASELINE config 3 ("FLUX.1-dev shapes 1024x1024 = 4096 image tokens, one step at SP=1/2/4/8")
+    against the float64 oracle: step 0 of S = 20 (tests/golden/flux1024_seed1000_S20_step0.npz,
+    tools/make_golden.py flux1024) at SP = 1, 2, 4, 8 on virtual ranks of one GPU."""
+    gold = _golden("flux1024_seed1000_S20_step0.npz")
+    eng = tsv.Engine("flux", devices=[0] * 8)
+    for k in (1, 2, 4, 8):
+        g = eng.group_create(list(range(k)))
+        req = eng.request_create(1024, 1024, num_steps=20, seed=1000)
+        eng.event_wait(eng.request_step(req, 0, g))
+        for got, ref in ((eng.read_velocity(req), gold["v"]), (eng.read_latent(req), gold["x_next"])):
+            rel, cos = _metrics(got.astype(np.float64), ref.astype(np.float64))
+            assert rel <= TOL_REL and cos >= TOL_COS, (k, rel, cos)
+        eng.request_destroy(req)
+    eng.close()
+
+
 @pytest.mark.parametrize("model,res", [("tiny2", (208, 240)), ("tiny_sd3", (208, 240))])
 @pytest.mark.parametrize("k", [2, 4])
 def test_fused_transport_bitwise_equals_exchange(tsv, model, res, k):
@@ -381,3 +398,22 @@ def test_event_release_reuses_handles(tsv):
     eng.event_wait(e1)
     assert eng.event_query(e1)
     eng.close()
+
+
+@pytest.mark.parametrize("fused", [True, False])
+def test_multi_stream_graph_matches_direct(tsv, fused):
+    """Several local ranks on their own streams (concurrent virtual ranks) are captured as one
+    multi-stream step graph forked from / joined to the first rank's stream; its replays are
+    bit-identical to direct launches, for both transports, across a group change (re-capture)."""
+    outs = []
+    for graphs in (True, False):
+        eng = tsv.Engine("tiny2", devices=[0] * 4)
+        eng.set_transport(fused)
+        eng.set_graphs(graphs)
+        g2, g4 = eng.group_create([1, 0]), eng.group_create([0, 1, 2, 3])
+        r = eng.request_create(208, 240, num_steps=5, seed=1800)
+        for s, g in enumerate([g2, g2, g4, g4, g2]):
+            eng.request_step(r, s, g)
+        outs.append((eng.read_latent(r), eng.read_velocity(r)))
+        eng.close()
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])

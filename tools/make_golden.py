@@ -14,7 +14,12 @@ v, x_next stored as float32 (the oracle computes in float64; float32 storage kee
 8 MB and its rounding, 2^-24 relative, is far below the 2e-2 tolerance).  Runtime: ~1.5-2 h on
 8 cores (~418 TFLOP of fp64 plus 3.9e11 exponentials).
 
-Usage: python tools/make_golden.py [flux|sd3|flux2048 ...]   (default: flux sd3)
+flux1024_seed1000_S20_step0.npz: BASELINE config 3's resolution (1024x1024 = 4096 image + 512
+text tokens), step 0 of S = 20, float32 storage as above (~20 min).
+sd3_1024_seed1000_S20.npz: SD3-medium CFG step 0 of S = 20 at 1024x1024 (config 5's 1024^2
+request), float32 storage.
+
+Usage: python tools/make_golden.py [flux|sd3|flux2048|flux1024|sd3_1024 ...]   (default: flux sd3)
 """
 import os
 import sys
@@ -61,10 +66,30 @@ def flux2048():
     print(f"wrote {out} in {time.time() - t0:.1f} s; |v|max={np.abs(v).max():.4f}")
 
 
+def flux1024():
+    t0 = time.time()
+    x, T, y = request_inputs(FLUX, 1024, 1024, 1000)
+    W = Weights(FLUX, cache_bytes=0)
+    v, xn = F.request_step(FLUX, W, x, T, y, 0, 20, 3.5, 1024, 1024)
+    out = os.path.join(ROOT, "tests", "golden", "flux1024_seed1000_S20_step0.npz")
+    np.savez_compressed(out, v=v.astype(np.float32), x_next=xn.astype(np.float32))
+    print(f"wrote {out} in {time.time() - t0:.1f} s; |v|max={np.abs(v).max():.4f}")
+
+
+def sd3_1024():
+    t0 = time.time()
+    x, Tc, yc, Tu, yu = sd3_request_inputs(SD3, 1024, 1024, 1000)
+    W = Weights(SD3, cache_bytes=20 << 30)
+    v, xn = S3.request_step(SD3, W, x, Tc, yc, Tu, yu, 0, 20, 1024, 1024)
+    out = os.path.join(ROOT, "tests", "golden", "sd3_1024_seed1000_S20.npz")
+    np.savez_compressed(out, v=v.astype(np.float32), x_next=xn.astype(np.float32))
+    print(f"wrote {out} in {time.time() - t0:.1f} s; |v|max={np.abs(v).max():.4f}")
+
+
 def main():
     which = sys.argv[1:] or ["flux", "sd3"]
     for w in which:
-        {"flux": flux, "sd3": sd3, "flux2048": flux2048}[w]()
+        {"flux": flux, "sd3": sd3, "flux2048": flux2048, "flux1024": flux1024, "sd3_1024": sd3_1024}[w]()
 
 
 if __name__ == "__main__":
