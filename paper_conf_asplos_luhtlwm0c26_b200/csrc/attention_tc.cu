@@ -115,8 +115,8 @@ struct FaCfg {
   static constexpr int NSUB = D / 64;
   static constexpr int Q_TILE = AT_BM * D * 2;
   static constexpr int KV_TILE = AT_BN * D * 2;
-  static constexpr int NK = D == 64 ? (KV == 4 ? 6 : 4) : (KV == 1 ? 3 : 2);
-  static constexpr int NV = D == 64 ? (KV == 4 ? 6 : 4) : (KV == 2 ? 3 : 2);
+  static constexpr int NK = D == 64 ? 4 : (KV == 1 ? 3 : 2);
+  static constexpr int NV = D == 64 ? 4 : (KV == 2 ? 3 : 2);
   static constexpr int OFF_Q = 0;                        // 2 tiles
   static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // NK stages
   static constexpr int OFF_V = OFF_K + NK * KV_TILE;     // NV stages
@@ -151,7 +151,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
                         float scale_log2, const __grid_constant__ AttnScatter sc,
                         const __grid_constant__ AttnSplitArgs sa) {
   using C = FaCfg<D, KV, RS>;
-  constexpr bool JOINT = KV >= 3;   // K and V of a tile share one stage and one barrier pair (KV 4: 6 stages)
+  constexpr bool JOINT = KV == 3;   // K and V of a tile share one stage and one barrier pair
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
@@ -731,8 +731,6 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
       case 92: return launch_fa<D, 2, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       case 93: return launch_fa<D, 3, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       case 94: return launch_fa<D, 4, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
-      case 96: return launch_fa<D, 2, 4, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
-      case 97: return launch_fa<D, 3, 4, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       case 99: return launch_fa<D, 9, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       default: break;
     }
