@@ -95,6 +95,7 @@ def main():
         roof.append(rrow)
     out = {"model": args.model, "res": res_list, "ks": KS, "ms": table, "comm_model_ms": comm,
            "roofline_frac": roof, "roofline_peak_tflops": peak / 1e12,
+           "comm_share_model": [[round(c / m, 4) if m > 0 else 0.0 for c, m in zip(cr, mr)] for cr, mr in zip(comm, table)],
            "efficiency_vs_k1": [[round(row[0] / (k * row[j]), 4) for j, k in enumerate(KS)] for row in table],
            "efficiency_range": {"low (450 GB/s, 20 us)": err_lo, "high (900 GB/s, 5 us)": err_hi},
            "a2a_model": {"bw_gbs": args.bw, "lat_us": args.lat_us, "overlap": "none (serial)"},
