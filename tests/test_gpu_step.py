@@ -417,3 +417,55 @@ def test_multi_stream_graph_matches_direct(tsv, fused):
         outs.append((eng.read_latent(r), eng.read_velocity(r)))
         eng.close()
     assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+
+
+@pytest.mark.parametrize("model,seed", [("tiny2", 0), ("tiny2", 1), ("tiny_sd3", 2)])
+def test_randomized_serving_sequence(tsv, model, seed):
+    """Runtime fuzz: requests of mixed resolutions step on random groups (random k, random GPU
+    subsets and rank orders), sometimes batched, sometimes explicitly resharded, with events released
+    as they complete -- every request's trajectory must equal the same request stepped alone at
+    SP = 1 (bitwise where the arithmetic is identical, else within the SP tolerance), exercising the
+    step-graph cache keys, the per-layout shard state, stream-ordered releases and handle reuse."""
+    rng = np.random.default_rng(seed)
+    eng = tsv.Engine(model, devices=[0] * 4)
+    ref = tsv.Engine(model, devices=[0])
+    g_ref = ref.group_create([0])
+    shapes = [(256, 256), (208, 240), (320, 192)]
+    groups = []
+    for k in (1, 2, 4):
+        for _ in range(3):
+            groups.append(eng.group_create([int(x) for x in rng.permutation(4)[:k]]))
+    reqs = []
+    for i in range(5):
+        h, w = shapes[i % len(shapes)]
+        steps = int(rng.integers(3, 6))
+        reqs.append((eng.request_create(h, w, num_steps=steps, seed=1900 + i), ref.request_create(h, w, num_steps=steps, seed=1900 + i), steps, (h, w)))
+    done = {i: 0 for i in range(len(reqs))}
+    pending = []
+    while any(done[i] < reqs[i][2] for i in done):
+        live = [i for i in done if done[i] < reqs[i][2]]
+        g = groups[int(rng.integers(len(groups)))]
+        same = [i for i in live if reqs[i][3] == reqs[live[0]][3]]
+        if len(same) > 1 and rng.random() < 0.3:
+            ev = eng.request_step_batch([reqs[i][0] for i in same], g)
+            for i in same:
+                ref.event_wait(ref.request_step(reqs[i][1], done[i], g_ref))
+                done[i] += 1
+        else:
+            i = live[int(rng.integers(len(live)))]
+            if rng.random() < 0.3:
+                eng.request_reshard(reqs[i][0], groups[int(rng.integers(len(groups)))])
+            ev = eng.request_step(reqs[i][0], done[i], g)
+            ref.event_wait(ref.request_step(reqs[i][1], done[i], g_ref))
+            done[i] += 1
+        pending.append(ev)
+        if len(pending) > 3:
+            e0 = pending.pop(0)
+            eng.event_wait(e0)
+            eng.event_release(e0)
+    for r, rr, _, _ in reqs:
+        a, b = eng.read_latent(r).astype(np.float64), ref.read_latent(rr).astype(np.float64)
+        rel, cos = _metrics(a, b)
+        assert rel <= 1e-2 and cos >= 0.9999, (rel, cos)
+    eng.close()
+    ref.close()
