@@ -1,5 +1,5 @@
 # A/B of whole steps under two environments (same .so): alternate bench.py runs with ENV_A / ENV_B.
-# Env: ROUNDS, ARGS, ENV_A, ENV_B (e.g. ENV_A="TSV_ATTN_D128=3" ENV_B="TSV_ATTN_D128=52")
+# Env: ROUNDS, ARGS, ENV_A, ENV_B (e.g. ENV_A="TSV_ATTN_D128=51" ENV_B="TSV_ATTN_D128=52")
 cd $GRAFT_REPO_ROOT
 for i in $(seq ${ROUNDS:-3}); do
   for v in A B; do

@@ -1,5 +1,5 @@
 # Same-box A/B of two source trees: A = build/ab/old (an older checkout with its own libtsv.so), B = this tree.
-# Env: ROUNDS, ARGS, ENV_B (environment for B's runs, e.g. "TSV_SPLITK=0 TSV_ATTN_D128=11")
+# Env: ROUNDS, ARGS, ENV_B (environment for B's runs, e.g. "TSV_SPLITK=0 TSV_ATTN_D128=52")
 cd $GRAFT_REPO_ROOT
 for i in $(seq ${ROUNDS:-3}); do
   for v in A B; do
