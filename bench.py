@@ -457,7 +457,8 @@ def run_ours(args):
 
     # end to end through the public API with host buffers: H2D latent in, step, D2H latent out
     r0, r1 = tsv.shard_range(Li, world, rank)
-    host = np.empty((r1 - r0, 64), np.float32)
+    # pinned host buffer (the contract's "host->device copy from pinned host memory")
+    host = torch.empty((r1 - r0, 64), dtype=torch.float32, pin_memory=True).numpy()
     host[:] = eng.read_latent(req, r0, r1 - r0)
     barrier()
     e2e_times = []
