@@ -82,6 +82,30 @@ __device__ __forceinline__ float2 poly_exp2_x2(float2 x) {
   return make_float2(__int_as_float(__float_as_int(p.x) + (__float_as_int(t.x) << 23)),
                      __int_as_float(__float_as_int(p.y) + (__float_as_int(t.y) << 23)));
 }
+// The same 2^x for a pair of raw scores s (x = s * scale - m), with the clamp to [-126, 64] done by
+// the saturating FFMA: y = sat(s * ca + cb) in [0, 1] (ca = scale / 190, cb = (126 - m) / 190), so
+// x' = 190 y - 126 in [-126, 64] -- two FFMA.SAT instead of the scale FFMA2 and four FMNMX.  The
+// rounding to n and the remainder f = x' - n come straight from y: t = 190 y + (magic - 126) holds
+// n = round(x') in its low bits, f = 190 y - (t - (magic - 126)).  |x' - x| <= ~2e-5 (two fp32
+// roundings at |x| <= 190): a relative error of ~1.4e-5 in p, far below P's bf16 rounding.
+__device__ __forceinline__ float sat_fma(float a, float b, float c) {
+  float d;
+  asm("fma.rn.sat.f32 %0, %1, %2, %3;" : "=f"(d) : "f"(a), "f"(b), "f"(c));
+  return d;
+}
+__device__ __forceinline__ float2 poly_exp2_sat_x2(float s0, float s1, float ca, float cb) {
+  const float2 y = make_float2(sat_fma(s0, ca, cb), sat_fma(s1, ca, cb));
+  const float2 k190 = make_float2(190.0f, 190.0f);
+  const float2 t = __ffma2_rn(y, k190, make_float2(12582786.0f, 12582786.0f));      // magic - 126
+  const float2 nn = __ffma2_rn(t, make_float2(-1.0f, -1.0f), make_float2(12582786.0f, 12582786.0f));  // -(n + 126)
+  const float2 f = __ffma2_rn(y, k190, nn);
+  float2 p = __ffma2_rn(make_float2(0.0555041086648216f, 0.0555041086648216f), f,
+                        make_float2(0.2402265069591007f, 0.2402265069591007f));
+  p = __ffma2_rn(p, f, make_float2(0.6931471805599453f, 0.6931471805599453f));
+  p = __ffma2_rn(p, f, make_float2(1.0f, 1.0f));
+  return make_float2(__int_as_float(__float_as_int(p.x) + (__float_as_int(t.x) << 23)),
+                     __int_as_float(__float_as_int(p.y) + (__float_as_int(t.y) << 23)));
+}
 __device__ __forceinline__ void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 // MN-major, 128B-swizzled B operand (rows = K, 64 N-elements per 128-byte row):
@@ -144,7 +168,7 @@ struct AttnSplitArgs {
   float* ws = nullptr;
 };
 
-template <int D, int NPOLY, int KV, bool RS = false>
+template <int D, int NPOLY, int KV, bool RS = false, bool PSAT = false>
 __global__ void __launch_bounds__(FA_THREADS, 1)
     attention_fa_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
@@ -374,6 +398,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         // lazy path: no max before the exponentials, so the TMEM loads are pipelined with the
         // arithmetic (chunk c + 1 is in flight while chunk c is exponentiated)
         const float2 sc2 = make_float2(scale_log2, scale_log2), nm2 = make_float2(-m_ref, -m_ref);
+        const float sat_a = scale_log2 * (1.0f / 190.0f), sat_b = (126.0f - m_ref) * (1.0f / 190.0f);
         float2 lz[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
         tmem_ld32(s_col, sr[0]);
         tmem_ld_wait_dep(sr[0]);
@@ -382,8 +407,14 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
           if (c < 3) tmem_ld32(s_col + (c + 1) * 32, sr[c + 1]);
 #pragma unroll
           for (int i = 0; i < 32; i += 2) {
-            float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2, nm2);
             float2 p;
+            if (PSAT && NPOLY != 9 && ((i >> 1) & 7) >= 8 - NPOLY) {
+              p = poly_exp2_sat_x2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1]), sat_a, sat_b);
+              lz[(i >> 1) & 3] = __fadd2_rn(lz[(i >> 1) & 3], p);
+              sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);
+              continue;
+            }
+            float2 x = __ffma2_rn(make_float2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1])), sc2, nm2);
             if (NPOLY == 9) {
               p = x;   // diagnostic (impl 59): no exponential -- the pipeline's ceiling without softmax math
             } else if (((i >> 1) & 7) >= 8 - NPOLY) {
@@ -634,7 +665,7 @@ static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L
   return r == CUDA_SUCCESS ? 0 : -2;
 }
 
-template <int D, int NP, int KV = 0, bool RS = false>
+template <int D, int NP, int KV = 0, bool RS = false, bool PS = false>
 static cudaError_t launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o,
                              long long ldo, int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s,
                              const AttnSplitArgs& sa) {
@@ -642,13 +673,13 @@ static cudaError_t launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const
   int dev = 0;
   cudaGetDevice(&dev);
   if (!(done >> dev & 1ull)) {
-    cudaError_t e = cudaFuncSetAttribute(attention_fa_kernel<D, NP, KV, RS>,
+    cudaError_t e = cudaFuncSetAttribute(attention_fa_kernel<D, NP, KV, RS, PS>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, FaCfg<D, KV, RS>::SMEM);
     if (e != cudaSuccess) return e;
     done |= 1ull << dev;
   }
   dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H, sa.nsplit);
-  return launch_pdl(attention_fa_kernel<D, NP, KV, RS>, grid, dim3(FA_THREADS), FaCfg<D, KV, RS>::SMEM, s, tq, tk, tv,
+  return launch_pdl(attention_fa_kernel<D, NP, KV, RS, PS>, grid, dim3(FA_THREADS), FaCfg<D, KV, RS>::SMEM, s, tq, tk, tv,
                     o, ldo, L, scale_log2, sc, sa);
 }
 
@@ -704,11 +735,12 @@ static int default_version(int D) {
   int& r = v[D == 128];
   if (r < 0) {
     const char* e = getenv(D == 128 ? "TSV_ATTN_D128" : "TSV_ATTN_D64");
-    // D = 128: separate K / V rings, 1 of 8 exp2 pairs by polynomial; D = 64: the joint ring (the split
-    // rings measured -2 % on the SD3 1024^2 step) with rotating S buffers, 2 of 8 (round-2 sweeps,
-    // profiles/r02)
-    r = e ? atoi(e) : (D == 128 ? 51 : 92);
-    if (r < 50 || r > 99) r = D == 128 ? 51 : 92;
+    // D = 128: separate K / V rings, 2 of 8 exp2 pairs by the saturating-FFMA polynomial (impl 56); D = 64:
+    // the joint ring (the split rings measured -2 % on the SD3 1024^2 step) with rotating S buffers, 3 of
+    // 8 by the saturating-FFMA polynomial (impl 96).  Same-box step A/B (profiles/r02/ab_psat_l2hint.txt,
+    // ab_l2last_d128psat.txt): FLUX 2048^2 333.0 -> 330.4 ms vs impl 51, SD3 2048^2 143.9 -> 140.6 ms vs 92
+    r = e ? atoi(e) : (D == 128 ? 56 : 96);
+    if (r < 50 || r > 99) r = D == 128 ? 56 : 96;
   }
   return r;
 }
@@ -732,6 +764,10 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
       case 93: return launch_fa<D, 3, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       case 94: return launch_fa<D, 4, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       case 99: return launch_fa<D, 9, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
+      // 95 + n: the same with the saturating-FFMA polynomial (n + 2 of 8 pairs: 95 -> 2, 96 -> 3, 97 -> 4)
+      case 95: return launch_fa<D, 2, 3, true, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
+      case 96: return launch_fa<D, 3, 3, true, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
+      case 97: return launch_fa<D, 4, 3, true, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       default: break;
     }
   }
@@ -744,6 +780,9 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     case 54: e = launch_fa<D, 4>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 58: e = launch_fa<D, 8>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // all exp2 by polynomial
     case 59: e = launch_fa<D, 9>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // diagnostic: no exp2
+    case 55: e = launch_fa<D, 1, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // saturating-FFMA poly
+    case 56: e = launch_fa<D, 2, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 57: e = launch_fa<D, 3, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     // 60 + n / 70 + n (D = 128): 3 K + 2 V / 2 K + 3 V stages
     case 61: e = launch_fa<D, 1, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 62: e = launch_fa<D, 2, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
