@@ -93,16 +93,25 @@ __device__ __forceinline__ float sat_fma(float a, float b, float c) {
   asm("fma.rn.sat.f32 %0, %1, %2, %3;" : "=f"(d) : "f"(a), "f"(b), "f"(c));
   return d;
 }
+// DEG = 3: the cubic above; DEG = 2: the minimax quadratic for the relative error on |f| <= 1/2
+// (Remez: max 1.72e-3, P's bf16 rounding is 1.95e-3) -- one FFMA2 less per pair.
+template <int DEG = 3>
 __device__ __forceinline__ float2 poly_exp2_sat_x2(float s0, float s1, float ca, float cb) {
   const float2 y = make_float2(sat_fma(s0, ca, cb), sat_fma(s1, ca, cb));
   const float2 k190 = make_float2(190.0f, 190.0f);
   const float2 t = __ffma2_rn(y, k190, make_float2(12582786.0f, 12582786.0f));      // magic - 126
   const float2 nn = __ffma2_rn(t, make_float2(-1.0f, -1.0f), make_float2(12582786.0f, 12582786.0f));  // -(n + 126)
   const float2 f = __ffma2_rn(y, k190, nn);
-  float2 p = __ffma2_rn(make_float2(0.0555041086648216f, 0.0555041086648216f), f,
-                        make_float2(0.2402265069591007f, 0.2402265069591007f));
-  p = __ffma2_rn(p, f, make_float2(0.6931471805599453f, 0.6931471805599453f));
-  p = __ffma2_rn(p, f, make_float2(1.0f, 1.0f));
+  float2 p;
+  if constexpr (DEG == 2) {
+    p = __ffma2_rn(make_float2(0.23842894f, 0.23842894f), f, make_float2(0.703448f, 0.703448f));
+    p = __ffma2_rn(p, f, make_float2(1.0004431f, 1.0004431f));
+  } else {
+    p = __ffma2_rn(make_float2(0.0555041086648216f, 0.0555041086648216f), f,
+                   make_float2(0.2402265069591007f, 0.2402265069591007f));
+    p = __ffma2_rn(p, f, make_float2(0.6931471805599453f, 0.6931471805599453f));
+    p = __ffma2_rn(p, f, make_float2(1.0f, 1.0f));
+  }
   return make_float2(__int_as_float(__float_as_int(p.x) + (__float_as_int(t.x) << 23)),
                      __int_as_float(__float_as_int(p.y) + (__float_as_int(t.y) << 23)));
 }
@@ -168,7 +177,7 @@ struct AttnSplitArgs {
   float* ws = nullptr;
 };
 
-template <int D, int NPOLY, int KV, bool RS = false, bool PSAT = false>
+template <int D, int NPOLY, int KV, bool RS = false, int PSAT = 0>
 __global__ void __launch_bounds__(FA_THREADS, 1)
     attention_fa_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                         const __grid_constant__ CUtensorMap tmV, bf16* __restrict__ o, long long ldo, int L,
@@ -409,7 +418,8 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
           for (int i = 0; i < 32; i += 2) {
             float2 p;
             if (PSAT && NPOLY != 9 && ((i >> 1) & 7) >= 8 - NPOLY) {
-              p = poly_exp2_sat_x2(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1]), sat_a, sat_b);
+              p = poly_exp2_sat_x2<PSAT == 2 ? 2 : 3>(__uint_as_float(sr[c][i]), __uint_as_float(sr[c][i + 1]), sat_a,
+                                                      sat_b);
               lz[(i >> 1) & 3] = __fadd2_rn(lz[(i >> 1) & 3], p);
               sr[c >> 1][(c & 1) * 16 + i / 2] = pack_bf16x2(p.x, p.y);
               continue;
@@ -665,7 +675,7 @@ static int make_tmap_heads(CUtensorMap* m, const void* base, int D, int H, int L
   return r == CUDA_SUCCESS ? 0 : -2;
 }
 
-template <int D, int NP, int KV = 0, bool RS = false, bool PS = false>
+template <int D, int NP, int KV = 0, bool RS = false, int PS = 0>
 static cudaError_t launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const CUtensorMap& tv, bf16* o,
                              long long ldo, int L, int H, float scale_log2, const AttnScatter& sc, cudaStream_t s,
                              const AttnSplitArgs& sa) {
@@ -735,12 +745,13 @@ static int default_version(int D) {
   int& r = v[D == 128];
   if (r < 0) {
     const char* e = getenv(D == 128 ? "TSV_ATTN_D128" : "TSV_ATTN_D64");
-    // D = 128: separate K / V rings, 2 of 8 exp2 pairs by the saturating-FFMA polynomial (impl 56); D = 64:
-    // the joint ring (the split rings measured -2 % on the SD3 1024^2 step) with rotating S buffers, 3 of
-    // 8 by the saturating-FFMA polynomial (impl 96).  Same-box step A/B (profiles/r02/ab_psat_l2hint.txt,
-    // ab_l2last_d128psat.txt): FLUX 2048^2 333.0 -> 330.4 ms vs impl 51, SD3 2048^2 143.9 -> 140.6 ms vs 92
-    r = e ? atoi(e) : (D == 128 ? 56 : 96);
-    if (r < 50 || r > 99) r = D == 128 ? 56 : 96;
+    // D = 128: separate K / V rings, 2 of 8 exp2 pairs by the saturating-FFMA cubic (impl 56); D = 64: the
+    // joint ring (the split rings measured -2 % on the SD3 1024^2 step) with rotating S buffers, 3 of 8 by
+    // the saturating-FFMA quadratic (impl 103).  Same-box step A/B (profiles/r02/ab_psat_l2hint.txt,
+    // ab_l2last_d128psat.txt, ab_quad.txt): FLUX 2048^2 333.0 -> 330.4 ms vs impl 51 (the quadratic, 64:
+    // -0.15 %, noise), SD3 2048^2 143.9 -> 140.6 ms (96) vs 92, 140.1 -> 137.7 ms (103) vs 96
+    r = e ? atoi(e) : (D == 128 ? 56 : 103);
+    if (r < 50 || r > 109) r = D == 128 ? 56 : 103;
   }
   return r;
 }
@@ -768,6 +779,9 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
       case 95: return launch_fa<D, 2, 3, true, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       case 96: return launch_fa<D, 3, 3, true, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       case 97: return launch_fa<D, 4, 3, true, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
+      // 100 + n: the same with the quadratic polynomial (n of 8 pairs: 103 -> 3, 104 -> 4)
+      case 103: return launch_fa<D, 3, 3, true, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
+      case 104: return launch_fa<D, 4, 3, true, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       default: break;
     }
   }
@@ -783,6 +797,8 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
     case 55: e = launch_fa<D, 1, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // saturating-FFMA poly
     case 56: e = launch_fa<D, 2, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 57: e = launch_fa<D, 3, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 64: e = launch_fa<D, 2, 0, false, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // quadratic
+    case 65: e = launch_fa<D, 3, 0, false, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     // 60 + n / 70 + n (D = 128): 3 K + 2 V / 2 K + 3 V stages
     case 61: e = launch_fa<D, 1, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 62: e = launch_fa<D, 2, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
