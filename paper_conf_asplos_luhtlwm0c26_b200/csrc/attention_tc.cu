@@ -25,14 +25,18 @@
 // Without the max the four TMEM loads of S are pipelined under the exponentials.  NPOLY of every 8
 // exp2 pairs are evaluated on the FMA pipe (Cody-Waite split + cubic) to relieve MUFU.EX2.
 //
-// KV split (blockIdx.z): for launches with too few CTAs (SP = 4/8 head shards), each split covers
-// a key range and the last split of a 32-row warp merges the (O, m, l) partials in range order.
+// KV split (AttnSplitArgs): the last work items of a launch (or all of them: SP = 4/8 head shards) are
+// split into key ranges, and the last range of a 32-row warp merges the (O, m, l) partials in range order.
 //
 // Measured dead ends (profiles/README.md): one query tile per CTA with P in shared
 // memory; 64-key tiles with double-buffered S (the N = 64 S MMA re-reads Q from shared memory at
 // 192 B/clk); P handed over in two halves; CTA-pair (cta_group::2) tiles (-17 %: the pair couples
 // both CTAs' softmax chains); two softmax warps per row; packed ex2 (two MUFU ops per instruction).
+#include <algorithm>
 #include <cfloat>
+#include <map>
+#include <tuple>
+#include <vector>
 #include <cstdio>
 #include <cstdlib>
 #include <cudaTypedefs.h>
@@ -170,9 +174,14 @@ static_assert(FaCfg<128, 1>::SMEM <= 232448 && FaCfg<128, 2>::SMEM <= 232448 && 
               "attention shared memory > 227 KB");
 constexpr int FA_THREADS = 384;
 
-// KV split (blockIdx.z = split): see AttnSplitWs.  nsplit = 1: the whole key range, no workspace.
+// The launch is 1-D over work items i = query block + nqb * head: CTAs [0, n_plain) are items 0..n_plain-1
+// over all their keys; the remaining n_tail items ("the tail", dispatched last) are split into nsplit
+// key ranges, CTA n_plain + z * n_tail + u covering range z of item n_plain + u, z-major (every tail
+// item's first range before any second range).  n_plain = 0: every item split (the uniform KV split).
 struct AttnSplitArgs {
-  int nsplit = 1, tps = 0;   // splits, key tiles per split
+  int nsplit = 1, tps = 0;   // key ranges per tail item, tiles of the largest
+  int n_plain = 0, n_tail = 0, nqb = 1;
+  int bound[9] = {0};        // range z covers key tiles [bound[z], bound[z + 1])
   int* cnt = nullptr;
   float* ws = nullptr;
 };
@@ -208,12 +217,18 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   auto tb = [](uint64_t* base, int t, int j) { return base + t * 3 + (RS ? j % 3 : 0); };
   auto tpar = [](int j) { return (uint32_t)((RS ? j / 3 : j) & 1); };
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int head = blockIdx.y;
-  const int q0 = blockIdx.x * 2 * AT_BM;
+  // work item and key range of this CTA (see AttnSplitArgs)
+  const int bid = blockIdx.x;
+  const bool split = bid >= sa.n_plain && sa.nsplit > 1;
+  const int tail_u = split ? (bid - sa.n_plain) % sa.n_tail : 0;
+  const int zr = split ? (bid - sa.n_plain) / sa.n_tail : 0;
+  const int item = split ? sa.n_plain + tail_u : bid;
+  const int head = item / sa.nqb;
+  const int q0 = (item - head * sa.nqb) * 2 * AT_BM;
   // this CTA's key tiles: [j0, j0 + n_tiles) (all of them unless the launch splits the keys)
   const int n_all = (L + AT_BN - 1) / AT_BN;
-  const int j0 = sa.nsplit > 1 ? (int)blockIdx.z * sa.tps : 0;
-  const int n_tiles = sa.nsplit > 1 ? min(n_all - j0, sa.tps) : n_all;
+  const int j0 = split ? sa.bound[zr] : 0;
+  const int n_tiles = split ? sa.bound[zr + 1] - j0 : n_all;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tmQ);
@@ -316,7 +331,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       if (t == 0 && !JOINT) mbar_wait(&v_full[j % NV], (j / NV) & 1);
 #ifdef TSV_ATTN_DEBUG
       if (!mbar_wait_bounded(tb(p_full, t, j), tpar(j), 1 << 22)) {
-        if (lane == 0) printf("p_full hang: blk %d head %d t %d j %d\n", blockIdx.x, head, t, j);
+        if (lane == 0) printf("p_full hang: blk %d head %d t %d j %d\n", bid, head, t, j);
         __trap();
       }
 #else
@@ -393,7 +408,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       const uint32_t s_col = tmem + lane_base + sb * 128;
 #ifdef TSV_ATTN_DEBUG
       if (!mbar_wait_bounded(&s_full[sb], (RS ? (2 * j + t) / 3 : j) & 1, 1 << 22)) {
-        if (lane == 0) printf("s_full hang: blk %d head %d t %d j %d sb %d\n", blockIdx.x, head, t, j, sb);
+        if (lane == 0) printf("s_full hang: blk %d head %d t %d j %d sb %d\n", bid, head, t, j, sb);
         __trap();
       }
 #else
@@ -504,7 +519,7 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
         if (RS) {
 #ifdef TSV_ATTN_DEBUG
           if (!mbar_wait_bounded(tb(pv_done, t, j - 1), tpar(j - 1), 1 << 22)) {
-            if (lane == 0) printf("RS pv_done hang: blk %d head %d t %d j %d\n", blockIdx.x, head, t, j);
+            if (lane == 0) printf("RS pv_done hang: blk %d head %d t %d j %d\n", bid, head, t, j);
             __trap();
           }
 #else
@@ -548,15 +563,14 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
       }
       orow = sc.dst[p] + (long long)lr * sc.ld + sc.col0 + head * D;
     }
-    if (sa.nsplit > 1) {
+    if (split) {
       // KV split: unnormalised O_t (layout [D][128]: coalesced across the warp's rows), reference m
       // and sum l of this split -> ws; the last split of these 32 rows merges in split order:
       // O = sum_s 2^(m_s - M) O_s / sum_s 2^(m_s - M) l_s, M = max_s m_s
       const size_t slab = (size_t)AT_BM * (D + 2);
-      const int nqb = gridDim.x;
-      const size_t qt = ((size_t)head * nqb + blockIdx.x) * 2 + t;   // query tile
+      const size_t qt = (size_t)tail_u * 2 + t;   // query tile among the tail items'
       auto ws_at = [&](int s2) { return sa.ws + (qt * sa.nsplit + s2) * slab; };
-      float* mine = ws_at(blockIdx.z);
+      float* mine = ws_at(zr);
 #pragma unroll
       for (int c = 0; c < D / 32; ++c) {
         uint32_t ov[32];
@@ -688,51 +702,108 @@ static cudaError_t launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const
     if (e != cudaSuccess) return e;
     done |= 1ull << dev;
   }
-  dim3 grid((L + 2 * AT_BM - 1) / (2 * AT_BM), H, sa.nsplit);
+  dim3 grid(sa.n_plain + sa.n_tail * (sa.nsplit > 1 ? sa.nsplit : 0));
   return launch_pdl(attention_fa_kernel<D, NP, KV, RS, PS>, grid, dim3(FA_THREADS), FaCfg<D, KV, RS>::SMEM, s, tq, tk, tv,
                     o, ldo, L, scale_log2, sc, sa);
 }
 
-// KV-split factor for a launch of C = ceil(L/256) x H CTAs: the S in 1..8 minimising the estimated
-// makespan (below), each split >= 4 key tiles.
-static int KV_MIN_TILES = 4, KV_SPLIT_COST = 6;   // TSV_KV_MIN / TSV_KV_COST override (tuning)
+// KV split for a launch of C = ceil(L/256) x H work items (one per head and 256 queries, one CTA per
+// SM): the last T items (the tail) are split into S key ranges each, chosen by a list-scheduling
+// model of the launch.  CTAs are dispatched in block order to the first free SM; a CTA costs its key
+// tiles + a fixed cost (prologue, pipeline fill, epilogue: 2 tiles; + the merge when split: 6, fitted
+// to tools/microbench.py attnsplit).  The whole items come first in equal waves (closed form), then
+// the tail's S x T short CTAs fill the last wave's gaps.  T = C is the uniform split of round 1.
+// E.g. FLUX 2048^2 at SP = 8 (198 items of 132 tiles on 148 SMs): all items halved costs 218 tiles of
+// time, 148 whole + the last 50 in 5 ranges 200 (ideal 179).  TSV_KV_TAIL=0: uniform splits only.
+static int KV_MIN_TILES = 4, KV_SPLIT_COST = 6, KV_TAIL = 1;   // TSV_KV_MIN / _COST / _TAIL (tuning)
+static double kv_makespan(long long n_plain, int plain_cost, long long T, const int* sz, int S, int sms, int fixed) {
+  // n_plain equal CTAs first: q full rounds, r SMs one more; then the tail list-scheduled
+  std::vector<double> h(sms);
+  const long long q = n_plain / sms, r = n_plain % sms;
+  for (int i = 0; i < sms; ++i) h[i] = (double)(q + (i < r ? 1 : 0)) * plain_cost;
+  auto cmp = [](double x, double y) { return x > y; };
+  std::make_heap(h.begin(), h.end(), cmp);
+  for (int z = 0; z < S; ++z)
+    for (long long c = 0; c < T; ++c) {
+      std::pop_heap(h.begin(), h.end(), cmp);
+      h.back() += sz[z] + fixed;
+      std::push_heap(h.begin(), h.end(), cmp);
+    }
+  return *std::max_element(h.begin(), h.end());
+}
 static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
   static bool env_read = false;
   if (!env_read) {
     if (const char* v = getenv("TSV_KV_MIN")) KV_MIN_TILES = atoi(v);
     if (const char* v = getenv("TSV_KV_COST")) KV_SPLIT_COST = atoi(v);
+    if (const char* v = getenv("TSV_KV_TAIL")) KV_TAIL = atoi(v);
     env_read = true;
   }
+  const int n_all = (L + AT_BN - 1) / AT_BN;
+  const int nqb = (L + 2 * AT_BM - 1) / (2 * AT_BM);
+  const long long C = (long long)nqb * H;
   AttnSplitArgs a;
+  a.n_plain = (int)C;
+  a.nqb = nqb;
   if (!w || !w->cnt || !w->ws) return a;
   static int sms_of[64] = {0};
   int dev = 0;
   cudaGetDevice(&dev);
   if (!sms_of[dev & 63]) cudaDeviceGetAttribute(&sms_of[dev & 63], cudaDevAttrMultiProcessorCount, dev);
   const int sms = sms_of[dev & 63] ? sms_of[dev & 63] : 148;
-  const int n_all = (L + AT_BN - 1) / AT_BN;
-  const long long C = (long long)((L + 2 * AT_BM - 1) / (2 * AT_BM)) * H;
-  int best = 1;
+  // the workspace bounds the tail: T items x 2 query tiles x S ranges x (O, m, l) slabs; 4 counters each
+  const long long slab = (long long)AT_BM * (D + 2) * 4;
+  auto fits = [&](long long T, int S) { return T * 2 * S * slab <= w->ws_bytes && T * 2 * 4 <= w->cnt_ints; };
+  long long bestT = 0;
+  std::vector<int> sz;   // tiles per range (empty: no split)
   if (w->force > 0) {
-    best = w->force < n_all ? w->force : n_all;
+    const int f = w->force < n_all ? w->force : n_all;
+    const int tps = (n_all + f - 1) / f;
+    for (int j = 0; j < n_all; j += tps) sz.push_back(std::min(tps, n_all - j));
+    bestT = C;
   } else {
-    // makespan in key-tile units: waves x (tiles per split + fixed cost), the fixed cost (prologue,
-    // pipeline fill, epilogue; + the merge when split) fitted to tools/microbench.py attnsplit
-    double bestc = (double)((C + sms - 1) / sms) * (n_all + 2);
-    for (int S = 2; S <= 8; ++S) {
-      const int tps = (n_all + S - 1) / S;
-      if (tps < KV_MIN_TILES) break;
-      const double cost = (double)((C * S + sms - 1) / sms) * (tps + KV_SPLIT_COST);
-      if (cost < bestc * 0.95) { bestc = cost; best = S; }
+    // plans depend on (L, H, SMs, knobs) only: cached (each step graph captures a shape once anyway)
+    static std::map<std::tuple<int, int, int, int, int, int>, std::pair<long long, std::vector<int>>> cache;
+    const auto key = std::make_tuple(L, H, sms, KV_MIN_TILES, KV_SPLIT_COST, KV_TAIL);
+    auto it = cache.find(key);
+    if (it != cache.end()) {
+      bestT = it->second.first;
+      sz = it->second.second;
+    } else {
+      const double base = kv_makespan(C, n_all + 2, 0, nullptr, 0, sms, 0);
+      double bestc = base;
+      for (int S = 2; S <= 8; ++S) {
+        const int eq = (n_all + S - 1) / S;
+        if (eq < KV_MIN_TILES) break;
+        int t[8];
+        int left = n_all;
+        for (int z = 0; z < S; ++z) { t[z] = std::min(eq, left); left -= t[z]; }
+        if (t[S - 1] < 1) continue;
+        // tails: every item (the uniform split), or up to three waves' worth of the last items
+        const long long t_hi = KV_TAIL ? std::min<long long>(C, 3LL * sms) : 0;
+        for (long long T = t_hi; T >= 0; --T) {
+          const long long TT = T == 0 ? C : T;   // T = 0 encodes the uniform split (all C items)
+          if (T == 0 && t_hi == C) break;        // already evaluated
+          if (!fits(TT, S)) continue;
+          const double c = kv_makespan(C - TT, n_all + 2, TT, t, S, sms, KV_SPLIT_COST);
+          if (c < bestc && c < base * 0.97) {
+            bestc = c;
+            bestT = TT;
+            sz.assign(t, t + S);
+          }
+        }
+      }
+      cache[key] = std::make_pair(bestT, sz);
     }
   }
-  if (best < 2) return a;
-  const int tps = (n_all + best - 1) / best;
-  best = (n_all + tps - 1) / tps;   // no empty split
-  if (best < 2 || best > 8) return a;
-  if ((long long)C * 2 * best * AT_BM * (D + 2) * 4 > w->ws_bytes || C * 2 * 4 > w->cnt_ints) return a;
+  const int best = (int)sz.size();
+  if (best < 2 || best > 8 || bestT < 1 || !fits(bestT, best)) return a;
   a.nsplit = best;
-  a.tps = tps;
+  a.tps = *std::max_element(sz.begin(), sz.end());
+  a.n_plain = (int)(C - bestT);
+  a.n_tail = (int)bestT;
+  a.bound[0] = 0;
+  for (int z = 0; z < best; ++z) a.bound[z + 1] = a.bound[z] + sz[z];
   a.cnt = w->cnt;
   a.ws = w->ws;
   return a;

@@ -334,8 +334,36 @@ def test_attention_kv_split(tsv, L, H, D, nsplit):
     assert torch.count_nonzero(cnt) == 0
 
 
-@pytest.mark.parametrize("L,H,D,split", [(16896, 24, 128, False), (16896, 3, 128, True), (16717, 24, 64, False),
-                                         (4429, 3, 64, True)])
+@pytest.mark.parametrize("L,H,D", [(4608, 12, 128), (4429, 12, 64)])
+def test_attention_tail_split(tsv, L, H, D):
+    """Automatic KV split with a tail (FLUX / SD3 1024^2 at SP = 2: 216 work items on 148 SMs): the
+    first items run whole, the last ones in key ranges merged by their last range -- every head
+    against the float64 definition, deterministic run to run, counters re-armed."""
+    rng = np.random.default_rng(L + H)
+    qkv = rng.standard_normal((L, 3, H, D)).astype(np.float32) * np.float32(1.5)
+    qkv[L // 2:, 1] += 0.8
+    qkv = synth.bf16_bits_to_f32(synth.bf16_rne_bits(qkv)).astype(np.float64)
+    ref = F.attention(qkv[:, 0], qkv[:, 1], qkv[:, 2])
+    t = _bf16(qkv.reshape(L, 3 * H * D))
+    ld = 3 * H * D
+    cnt = torch.zeros(4096, dtype=torch.int32, device="cuda")
+    ws = torch.empty(32 << 20, dtype=torch.float32, device="cuda")
+    outs = []
+    for _ in range(2):
+        o = torch.zeros(L, H * D, dtype=torch.bfloat16, device="cuda")
+        tsv.op_attention_split(t, t[:, H * D:], t[:, 2 * H * D:], o, L, H, D, cnt, ws, nsplit=0, ldq=ld, ldk=ld,
+                               ldv=ld)
+        torch.cuda.synchronize()
+        outs.append(o.cpu())
+        got = _np(o).reshape(L, H, D)
+        assert _rel(got, ref) < 1.5e-2
+        assert np.sum(got * ref) / np.linalg.norm(got) / np.linalg.norm(ref) > 0.9999
+    assert torch.equal(outs[0], outs[1])
+    assert torch.count_nonzero(cnt) == 0
+
+
+@pytest.mark.parametrize("L,H,D,split", [(16896, 24, 128, False), (16896, 3, 128, True), (16896, 12, 128, True),
+                                         (16717, 24, 64, False), (16717, 6, 64, True), (4429, 3, 64, True)])
 def test_attention_sampled_full_size(tsv, L, H, D, split):
     """BASELINE sizes (FLUX 2048^2 joint L = 16 896, SD3 2048^2 / 1024^2 L = 16 717 / 4429; H = 3 is an
     SP = 8 head shard, run with the KV split): sampled query rows of sampled heads against the
