@@ -716,6 +716,7 @@ static cudaError_t launch_fa(const CUtensorMap& tq, const CUtensorMap& tk, const
 // E.g. FLUX 2048^2 at SP = 8 (198 items of 132 tiles on 148 SMs): all items halved costs 218 tiles of
 // time, 148 whole + the last 50 in 5 ranges 200 (ideal 179).  TSV_KV_TAIL=0: uniform splits only.
 static int KV_MIN_TILES = 4, KV_SPLIT_COST = 6, KV_TAIL = 1;   // TSV_KV_MIN / _COST / _TAIL (tuning)
+static double KV_GAIN = 0.97;   // a split plan must beat the unsplit launch's modeled makespan by 3 % (TSV_KV_GAIN)
 static double kv_makespan(long long n_plain, int plain_cost, long long T, const int* sz, int S, int sms, int fixed) {
   // n_plain equal CTAs first: q full rounds, r SMs one more; then the tail list-scheduled
   std::vector<double> h(sms);
@@ -737,6 +738,7 @@ static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
     if (const char* v = getenv("TSV_KV_MIN")) KV_MIN_TILES = atoi(v);
     if (const char* v = getenv("TSV_KV_COST")) KV_SPLIT_COST = atoi(v);
     if (const char* v = getenv("TSV_KV_TAIL")) KV_TAIL = atoi(v);
+    if (const char* v = getenv("TSV_KV_GAIN")) KV_GAIN = atof(v);
     env_read = true;
   }
   const int n_all = (L + AT_BN - 1) / AT_BN;
@@ -763,8 +765,8 @@ static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
     bestT = C;
   } else {
     // plans depend on (L, H, SMs, knobs) only: cached (each step graph captures a shape once anyway)
-    static std::map<std::tuple<int, int, int, int, int, int>, std::pair<long long, std::vector<int>>> cache;
-    const auto key = std::make_tuple(L, H, sms, KV_MIN_TILES, KV_SPLIT_COST, KV_TAIL);
+    static std::map<std::tuple<int, int, int, int, int, int, int>, std::pair<long long, std::vector<int>>> cache;
+    const auto key = std::make_tuple(L, H, sms, KV_MIN_TILES, KV_SPLIT_COST, KV_TAIL, (int)(KV_GAIN * 1000));
     auto it = cache.find(key);
     if (it != cache.end()) {
       bestT = it->second.first;
@@ -786,7 +788,7 @@ static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
           if (T == 0 && t_hi == C) break;        // already evaluated
           if (!fits(TT, S)) continue;
           const double c = kv_makespan(C - TT, n_all + 2, TT, t, S, sms, KV_SPLIT_COST);
-          if (c < bestc && c < base * 0.97) {
+          if (c < bestc && c < base * KV_GAIN) {
             bestc = c;
             bestT = TT;
             sz.assign(t, t + S);
