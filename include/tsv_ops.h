@@ -85,24 +85,27 @@ tsv_status tsv_op_qk_norm_rope(void* qkv, int64_t ld, int rows, int n_first, int
 
 /* a6: O = softmax(q k^T / sqrt(D)) v, non-causal, per head h < H; q(l, h) at q + l*ldq + h*D
  * (bf16, same for k, v, o).  D in {64, 128}.  Operands and row strides 16-byte aligned.
- * impl 0: the tcgen05/TMEM kernel the step uses (= impl 51 for D = 128, 92 for D = 64; the
+ * impl 0: the tcgen05/TMEM kernel the step uses (= impl 56 for D = 128, 103 for D = 64; the
  * environment variables TSV_ATTN_D128 / TSV_ATTN_D64 select another impl for the step);
- * 50..54: separate K and V TMA rings (2 + 2 stages at D = 128, 4 + 4 at D = 64) with 0..4 of
- * every 8 exp2 pairs evaluated by polynomial on the FMA pipe instead of MUFU.EX2; 58: all of them
- * by polynomial; 61, 62 / 71, 72 (D = 128): 3 K + 2 V / 2 K + 3 V stages, 1 or 2 poly pairs;
- * 81..83: one joint K+V ring, 1..3 poly pairs; 91..94 (D = 64): the joint ring with three rotating
- * S buffers shared by the two query tiles (S computed one ahead); 59, 69, 79, 99: DIAGNOSTIC ONLY, wrong results -- P = the
- * scaled score without any exponential (the pipeline's ceiling without the softmax arithmetic).
+ * 50 / 51 / 56: separate K and V TMA rings (2 + 2 stages at D = 128, 4 + 4 at D = 64) with 0 / 1 / 2
+ * of every 8 exp2 pairs evaluated by a polynomial on the FMA pipe instead of MUFU.EX2 (51: cubic with
+ * clamps, 56: cubic with the clamp folded into saturating FFMAs); 81 / 83: one joint K+V ring, 1 / 3
+ * polynomial pairs; D = 64 only, the joint ring with three rotating S buffers shared by the two query
+ * tiles (S computed one ahead): 92 (2 pairs, clamped cubic), 96 (3, saturating cubic), 103 (3,
+ * saturating minimax quadratic); 59, 99: DIAGNOSTIC ONLY, wrong results -- P = the scaled score without
+ * any exponential (the pipeline's ceiling without the softmax arithmetic).
  * Other values: TSV_E_INVAL. */
 tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
                             void* o, int64_t ldo, int L, int H, int D, int impl, void* stream);
 
 /* a6 with the key range split (flash-decoding style) for launches with too few CTAs (SP = 4/8 head
- * shards, small images): nsplit key ranges (0: the engine's automatic choice, possibly 1; capped at
- * 8 and by the workspace), each range's unnormalised O, reference and sum go to ws and the last
- * range to finish a query tile merges them in range order (deterministic).  The step's attention
- * kernel (impl 0).  cnt: zeroed device ints (>= 8 per 256-query block and head), left zero;
- * ws: fp32 device workspace (nsplit x 2 x 128 x (D + 2) floats per 256-query block and head).
+ * shards, small images): nsplit key ranges (0: the engine's automatic choice -- whole work items
+ * first, the launch's last items split into key ranges by a list-scheduling model, possibly none;
+ * > 0: every item in nsplit equal ranges; capped at 8 and by the workspace), each range's
+ * unnormalised O, reference and sum go to ws and the last range to finish a query tile merges them
+ * in range order (deterministic).  The step's attention kernel (impl 0).  cnt: zeroed device ints
+ * (>= 8 per split 256-query block and head), left zero; ws: fp32 device workspace (nsplit x 2 x 128
+ * x (D + 2) floats per split 256-query block and head).
  * Same operand rules as tsv_op_attention. */
 tsv_status tsv_op_attention_split(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
                                   void* o, int64_t ldo, int L, int H, int D, int nsplit, int* cnt, int cnt_ints,

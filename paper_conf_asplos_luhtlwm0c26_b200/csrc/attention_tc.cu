@@ -139,9 +139,9 @@ __host__ __device__ constexpr uint32_t make_idesc_bf16_bmn(int M, int N) {
 // stage is free as soon as both S MMAs of its tile completed, a V stage only after both PV MMAs, so
 // the next K load starts ~one tile of tensor time earlier than with one joint K/V stage (r02: the
 // MMA warp spent most of its stall samples waiting for K/V data with the joint 2-stage ring).
-// KV = 0: NK = NV = 2 (D = 128) / 4 (D = 64); KV = 1: NK = 3, NV = 2; KV = 2: NK = 2, NV = 3 (D = 128
-// fills the 227 KB of shared memory with 3 + 2 stages); KV = 3: one joint K+V ring (NK = NV stages,
-// one producer, a stage freed after both PV MMAs: round 1's design, kept where it measured better).
+// KV = 0: NK = NV = 2 (D = 128) / 4 (D = 64) (3 + 2 stages fill the 227 KB at D = 128 and measured
+// slower); KV = 3: one joint K+V ring (NK = NV stages, one producer, a stage freed after both PV MMAs:
+// round 1's design, kept at D = 64 where it measured better).
 // RS (rotating S buffers, D = 64 only): three 128-column S buffers shared by the two query tiles
 // (S index n = 2 j + t lives in buffer n % 3) instead of one per tile, so the MMA warp runs one S
 // ahead -- S_t(j+1) is computed while P_t(j) still waits for its PV MMA -- and a softmax warpgroup
@@ -152,8 +152,9 @@ struct FaCfg {
   static constexpr int NSUB = D / 64;
   static constexpr int Q_TILE = AT_BM * D * 2;
   static constexpr int KV_TILE = AT_BN * D * 2;
-  static constexpr int NK = D == 64 ? 4 : (KV == 1 ? 3 : 2);
-  static constexpr int NV = D == 64 ? 4 : (KV == 2 ? 3 : 2);
+  static_assert(KV == 0 || KV == 3, "K/V ring layout");
+  static constexpr int NK = D == 64 ? 4 : 2;
+  static constexpr int NV = D == 64 ? 4 : 2;
   static constexpr int OFF_Q = 0;                        // 2 tiles
   static constexpr int OFF_K = OFF_Q + 2 * Q_TILE;       // NK stages
   static constexpr int OFF_V = OFF_K + NK * KV_TILE;     // NV stages
@@ -170,7 +171,7 @@ struct FaCfg {
 // __launch_bounds__(384, 1) (64K / 384 rounded down to 8 = 168) -- and an .inc blocks until the pool
 // has the registers, so the split must fit that pool (a 4-tile variant that over-asked hung).
 static_assert(80 * 128 + 208 * 256 <= ((65536 / 384) & ~7) * 384, "setmaxnreg split exceeds the pool");
-static_assert(FaCfg<128, 1>::SMEM <= 232448 && FaCfg<128, 2>::SMEM <= 232448 && FaCfg<64>::SMEM <= 232448,
+static_assert(FaCfg<128>::SMEM <= 232448 && FaCfg<64>::SMEM <= 232448 && FaCfg<64, 3, true>::SMEM <= 232448,
               "attention shared memory > 227 KB");
 constexpr int FA_THREADS = 384;
 
@@ -840,48 +841,29 @@ static int launch_tc(const bf16* q, long long ldq, const bf16* k, long long ldk,
   const float scale_log2 = (1.0f / sqrtf((float)D)) * 1.4426950408889634f;
   const AttnSplitArgs sa = plan_kv_split(L, H, D, spw);
   cudaError_t e;
+  // Kept variants (the step's defaults, their round-2 predecessors, diagnostics); the other sweep points
+  // were removed after their measurements (profiles/README.md, profiles/r02/ab_*, mb_*).
   if constexpr (D == 64) {
-    // 90 + n (D = 64): rotating S buffers (RS) on the joint K+V ring, n of 8 exp2 pairs by polynomial
+    // rotating S buffers (RS) on the joint K+V ring: 92 = 2 of 8 exp2 pairs by the clamped cubic (round 2),
+    // 96 = 3 of 8 by the saturating-FFMA cubic, 103 = 3 of 8 by the saturating-FFMA quadratic (default),
+    // 99 = diagnostic without exponentials (wrong results: the pipeline's ceiling)
     switch (version) {
-      case 91: return launch_fa<D, 1, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       case 92: return launch_fa<D, 2, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
-      case 93: return launch_fa<D, 3, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
-      case 94: return launch_fa<D, 4, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
-      case 99: return launch_fa<D, 9, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
-      // 95 + n: the same with the saturating-FFMA polynomial (n + 2 of 8 pairs: 95 -> 2, 96 -> 3, 97 -> 4)
-      case 95: return launch_fa<D, 2, 3, true, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
-      case 96: return launch_fa<D, 3, 3, true, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
-      case 97: return launch_fa<D, 4, 3, true, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
-      // 100 + n: the same with the quadratic polynomial (n of 8 pairs: 103 -> 3, 104 -> 4)
+      case 96: return launch_fa<D, 3, 3, true, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       case 103: return launch_fa<D, 3, 3, true, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
-      case 104: return launch_fa<D, 4, 3, true, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
+      case 99: return launch_fa<D, 9, 3, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa) == cudaSuccess ? 0 : -5;
       default: break;
     }
   }
-  // version = 50 + n: n of 8 exp2 pairs by polynomial
+  // both head dims, one S buffer per query tile: 50 = all exp2 on MUFU, 51 = 1 of 8 pairs by the clamped
+  // cubic (round 2's D = 128 default), 56 = 2 of 8 by the saturating-FFMA cubic (D = 128 default), 59 =
+  // diagnostic without exponentials; 81 / 83 = the joint K+V ring (round 1's producer), 1 / 3 of 8
   switch (version) {
     case 50: e = launch_fa<D, 0>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 51: e = launch_fa<D, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 52: e = launch_fa<D, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 53: e = launch_fa<D, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 54: e = launch_fa<D, 4>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 58: e = launch_fa<D, 8>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // all exp2 by polynomial
-    case 59: e = launch_fa<D, 9>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // diagnostic: no exp2
-    case 55: e = launch_fa<D, 1, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // saturating-FFMA poly
-    case 56: e = launch_fa<D, 2, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 57: e = launch_fa<D, 3, 0, false, true>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 64: e = launch_fa<D, 2, 0, false, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;   // quadratic
-    case 65: e = launch_fa<D, 3, 0, false, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    // 60 + n / 70 + n (D = 128): 3 K + 2 V / 2 K + 3 V stages
-    case 61: e = launch_fa<D, 1, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 62: e = launch_fa<D, 2, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 69: e = launch_fa<D, 9, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 71: e = launch_fa<D, 1, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 72: e = launch_fa<D, 2, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 79: e = launch_fa<D, 9, 2>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    // 80 + n: the joint K+V ring (round 1's producer), n of 8 exp2 pairs by polynomial
+    case 56: e = launch_fa<D, 2, 0, false, 1>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
+    case 59: e = launch_fa<D, 9>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 81: e = launch_fa<D, 1, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
-    case 82: e = launch_fa<D, 2, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     case 83: e = launch_fa<D, 3, 3>(tq, tk, tv, o, ldo, L, H, scale_log2, sc, s, sa); break;
     default: return -3;
   }

@@ -282,7 +282,7 @@ def test_qk_norm_rope(tsv, H, D, rows, n_first):
 
 
 # ----------------------------------------------------------------------------- attention
-@pytest.mark.parametrize("impl", [0, 50, 51, 52, 53, 54, 55, 56, 61, 64, 65, 71, 81, 83, 92, 93, 95, 96, 97, 103, 104])
+@pytest.mark.parametrize("impl", [0, 50, 51, 56, 81, 83, 92, 96, 103])
 @pytest.mark.parametrize("L,H,D", [(1, 2, 64), (63, 4, 64), (320, 4, 64), (1000, 3, 128), (1536, 2, 128),
                                    (4700, 1, 128), (1357, 3, 64)])
 def test_attention(tsv, L, H, D, impl):
@@ -409,7 +409,7 @@ def test_attention_special_cases(tsv):
     assert np.max(np.abs(_np(o).reshape(L, H, D) - ref)) < 2e-2
 
 
-@pytest.mark.parametrize("impl", [0, 51, 52, 53, 55, 56, 61, 64, 81, 83])
+@pytest.mark.parametrize("impl", [0, 50, 51, 56, 81, 83])
 def test_attention_rescale_path(tsv, impl):
     """Scores growing along the key axis force the conditional O rescale (max grows by > 2^8)."""
     L, H, D = 700, 1, 128
@@ -429,7 +429,7 @@ def test_attention_rescale_path(tsv, impl):
     assert _rel(_np(o).reshape(L, H, D), ref) < 2e-2
 
 
-@pytest.mark.parametrize("D,impl", [(64, 0), (64, 51), (64, 83), (64, 93), (64, 96), (64, 103), (128, 0), (128, 52), (128, 56), (128, 81)])
+@pytest.mark.parametrize("D,impl", [(64, 0), (64, 51), (64, 83), (64, 92), (64, 96), (64, 103), (128, 0), (128, 51), (128, 56), (128, 81)])
 @pytest.mark.parametrize("jump", [3.0, 12.0, 200.0])
 def test_attention_score_jump(tsv, D, impl, jump):
     """A later key tile whose scores exceed the running maximum by `jump` (log2 units): small jumps
@@ -453,14 +453,14 @@ def test_attention_score_jump(tsv, D, impl, jump):
     assert _rel(got, ref) < 2e-2
 
 
-@pytest.mark.parametrize("impl", [0, 83, 92, 96, 103, 51, 56, 64])
+@pytest.mark.parametrize("impl", [0, 83, 92, 96, 103, 51, 56])
 def test_attention_large_logits_many_rescales(tsv, impl):
     """Scores with a large spread (q, k ~ 8 N(0, 1)): most key tiles overflow the lazy bound and take
     the exact path with an O rescale, so the softmax warps of a warpgroup drift apart by tiles -- the
     case that exposed a barrier-phase race in the rotating-S variant (impl 92).  SD3 1024^2 shape
     (L = 4429, H = 24), two heads checked against the float64 definition."""
     L, H = 4429, 24
-    D = 128 if impl in (51, 56, 64) else 64
+    D = 128 if impl in (51, 56) else 64
     g = torch.Generator(device="cuda").manual_seed(impl)
     qkv = (torch.randn(L, 3 * H * D, device="cuda", generator=g) * 8.0).to(torch.bfloat16)
     o = torch.zeros(L, H * D, dtype=torch.bfloat16, device="cuda")

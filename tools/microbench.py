@@ -117,13 +117,13 @@ def attn_split_cases():
 
 
 def attn_cases():
-    sweep = os.environ.get("ATTN_SWEEP")     # "1": also time the poly-share variants (impl 12..15)
+    sweep = os.environ.get("ATTN_SWEEP")     # "1": also time the kept exp2 variants
     for L, H, D in ((1536, 24, 128), (4608, 24, 128), (16896, 24, 128), (16896, 3, 128), (1357, 24, 64),
                     (4429, 24, 64), (16717, 24, 64)):
         qkv = torch.randn(L, 3 * H * D, device="cuda").to(torch.bfloat16)
         o = torch.empty(L, H * D, dtype=torch.bfloat16, device="cuda")
         ld = 3 * H * D
-        impls = (0,) + ((50, 51, 52, 53, 54) if sweep else ())
+        impls = (0,) + ((50, 51, 56, 92, 96, 103) if sweep else ())
         if os.environ.get("ATTN_IMPLS"):
             impls = tuple(int(x) for x in os.environ["ATTN_IMPLS"].split(","))
         impls = tuple(i for i in impls if not (i >= 90 and D != 64))   # RS variants: D = 64 only
