@@ -35,6 +35,7 @@
 #include <algorithm>
 #include <cfloat>
 #include <map>
+#include <mutex>
 #include <tuple>
 #include <vector>
 #include <cstdio>
@@ -767,6 +768,8 @@ static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
   } else {
     // plans depend on (L, H, SMs, knobs) only: cached (each step graph captures a shape once anyway)
     static std::map<std::tuple<int, int, int, int, int, int, int>, std::pair<long long, std::vector<int>>> cache;
+    static std::mutex cache_mu;   // launches may come from several host threads (one per engine / device)
+    std::lock_guard<std::mutex> lock(cache_mu);
     const auto key = std::make_tuple(L, H, sms, KV_MIN_TILES, KV_SPLIT_COST, KV_TAIL, (int)(KV_GAIN * 1000));
     auto it = cache.find(key);
     if (it != cache.end()) {
