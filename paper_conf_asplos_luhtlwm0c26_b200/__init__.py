@@ -327,7 +327,7 @@ def op_attention_split(q, k, v, o, L, H, D, cnt, ws, nsplit=0, ldq=None, ldk=Non
 
 
 def op_attention(q, k, v, o, L, H, D, ldq=None, ldk=None, ldv=None, ldo=None, impl=0, stream=None):
-    """impl 0: tcgen05 kernel (the step's); impl 1: mma.sync baseline (comparison only)."""
+    """impl 0: the step's tcgen05 kernel; other impl numbers: the kept variants (include/tsv_ops.h)."""
     check(lib.tsv_op_attention(_ptr(q), ldq or q.stride(0), _ptr(k), ldk or k.stride(0), _ptr(v), ldv or v.stride(0),
                                _ptr(o), ldo or o.stride(0), L, H, D, impl, _stream(stream)))
 

@@ -362,6 +362,34 @@ def test_attention_tail_split(tsv, L, H, D):
     assert torch.count_nonzero(cnt) == 0
 
 
+@pytest.mark.parametrize("ws_items", [1, 7, 40])
+def test_attention_split_workspace_bounds(tsv, ws_items):
+    """The automatic KV split stays inside the workspace it is given: a workspace for only ws_items
+    split 256-query blocks (2 splits each) and a counter array of 8 x ws_items ints, both followed by
+    guard regions (NaN / -1) that must stay untouched; the result still matches the float64 oracle."""
+    L, H, D = 4608, 12, 128
+    rng = np.random.default_rng(ws_items)
+    qkv = rng.standard_normal((L, 3, H, D)).astype(np.float32)
+    qkv = synth.bf16_bits_to_f32(synth.bf16_rne_bits(qkv)).astype(np.float64)
+    t = _bf16(qkv.reshape(L, 3 * H * D))
+    ld = 3 * H * D
+    n_ws = ws_items * 2 * 2 * 128 * (D + 2)
+    n_cnt = 8 * ws_items
+    ws_all = torch.full((n_ws + 65536,), float("nan"), dtype=torch.float32, device="cuda")
+    cnt_all = torch.zeros(n_cnt + 1024, dtype=torch.int32, device="cuda")
+    cnt_all[n_cnt:] = -1
+    o = torch.zeros(L, H * D, dtype=torch.bfloat16, device="cuda")
+    tsv.op_attention_split(t, t[:, H * D:], t[:, 2 * H * D:], o, L, H, D, cnt_all[:n_cnt], ws_all[:n_ws], nsplit=0,
+                           ldq=ld, ldk=ld, ldv=ld)
+    torch.cuda.synchronize()
+    assert torch.isnan(ws_all[n_ws:]).all()
+    assert (cnt_all[n_cnt:] == -1).all() and torch.count_nonzero(cnt_all[:n_cnt]) == 0
+    hh = [0, H - 1]
+    ref = F.attention(qkv[:, 0][:, hh], qkv[:, 1][:, hh], qkv[:, 2][:, hh])
+    got = _np(o).reshape(L, H, D)[:, hh]
+    assert _rel(got, ref) < 1.5e-2
+
+
 @pytest.mark.parametrize("L,H,D,split", [(16896, 24, 128, False), (16896, 3, 128, True), (16896, 12, 128, True),
                                          (16717, 24, 64, False), (16717, 6, 64, True), (4429, 3, 64, True)])
 def test_attention_sampled_full_size(tsv, L, H, D, split):

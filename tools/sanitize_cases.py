@@ -19,3 +19,19 @@ for model in ("tiny2", "tiny_sd3"):
         eng.event_wait(eng.request_step_batch(b, g2))
         print(model, fused, float(abs(eng.read_latent(r)).max()), flush=True)
         eng.close()
+
+# the attention's KV split with a tail (whole items first, the last items in key ranges: FLUX / SD3
+# 1024^2 at SP = 2 shapes) and the uniform split, kernel-level
+import torch  # noqa: E402
+
+for L, H, D in ((4608, 12, 128), (4429, 12, 64)):
+    for nsplit in (0, 3):
+        qkv = torch.randn(L, 3 * H * D, device="cuda").to(torch.bfloat16)
+        o = torch.zeros(L, H * D, dtype=torch.bfloat16, device="cuda")
+        cnt = torch.zeros(4096, dtype=torch.int32, device="cuda")
+        ws = torch.empty(32 << 20, dtype=torch.float32, device="cuda")
+        ld = 3 * H * D
+        tsv.op_attention_split(qkv, qkv[:, H * D:], qkv[:, 2 * H * D:], o, L, H, D, cnt, ws, nsplit=nsplit, ldq=ld,
+                               ldk=ld, ldv=ld)
+        torch.cuda.synchronize()
+        print("attention split", L, H, D, nsplit, float(o.float().abs().max()), int(torch.count_nonzero(cnt)), flush=True)
