@@ -107,6 +107,15 @@ tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t l
  * (>= 8 per split 256-query block and head), left zero; ws: fp32 device workspace (nsplit x 2 x 128
  * x (D + 2) floats per split 256-query block and head).
  * Same operand rules as tsv_op_attention. */
+/* Host only (no GPU needed): the KV-split plan tsv_op_attention_split(nsplit = 0 or the forced
+ * nsplit) and the step would use for (L, H, D) with a workspace of ws_bytes / cnt_ints on a GPU with
+ * `sms` SMs (<= 0: 148).  Work items = ceil(L / 256) x H; the first *n_plain run over all keys, the
+ * last *n_tail in *nsplit key ranges, range z = key tiles (of 128) [bounds[z], bounds[z + 1])
+ * (bounds: 9 ints, caller-owned).  *nsplit = 1: no split.  The same list-scheduling model as the
+ * launch.  Errors: TSV_E_INVAL. */
+tsv_status tsv_attention_split_plan(int L, int H, int D, int64_t ws_bytes, int cnt_ints, int nsplit, int sms,
+                                    int* n_plain, int* n_tail, int* nsplit_out, int* bounds);
+
 tsv_status tsv_op_attention_split(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
                                   void* o, int64_t ldo, int L, int H, int D, int nsplit, int* cnt, int cnt_ints,
                                   float* ws, int64_t ws_bytes, void* stream);

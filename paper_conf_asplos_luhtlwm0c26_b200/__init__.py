@@ -326,6 +326,15 @@ def op_attention_split(q, k, v, o, L, H, D, cnt, ws, nsplit=0, ldq=None, ldk=Non
                                      cnt.numel(), _ptr(ws), ws.numel() * 4, _stream(stream)))
 
 
+def attention_split_plan(L, H, D, ws_bytes, cnt_ints, nsplit=0, sms=148):
+    """The KV-split plan of an attention launch (host only): dict(n_plain, n_tail, nsplit, bounds)."""
+    n_plain, n_tail, ns = C.c_int(), C.c_int(), C.c_int()
+    b = (C.c_int * 9)()
+    check(lib.tsv_attention_split_plan(L, H, D, ws_bytes, cnt_ints, nsplit, sms, C.byref(n_plain), C.byref(n_tail),
+                                       C.byref(ns), b))
+    return {"n_plain": n_plain.value, "n_tail": n_tail.value, "nsplit": ns.value, "bounds": list(b)[:ns.value + 1]}
+
+
 def op_attention(q, k, v, o, L, H, D, ldq=None, ldk=None, ldv=None, ldo=None, impl=0, stream=None):
     """impl 0: the step's tcgen05 kernel; other impl numbers: the kept variants (include/tsv_ops.h)."""
     check(lib.tsv_op_attention(_ptr(q), ldq or q.stride(0), _ptr(k), ldk or k.stride(0), _ptr(v), ldv or v.stride(0),

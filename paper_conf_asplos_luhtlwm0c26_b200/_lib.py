@@ -93,6 +93,7 @@ _SIGS = {
                             _p]),
     "tsv_op_gemm_split": (_i32, [_p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p, _i64, _p, _p, _i32, _p, _i32, _p,
                                   _i64, _p]),
+    "tsv_attention_split_plan": (_i32, [_i32, _i32, _i32, _i64, _i32, _i32, _i32, _p, _p, _p, _p]),
     "tsv_op_attention_split": (_i32, [_p, _i64, _p, _i64, _p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p, _i32, _p,
                                        _i64, _p]),
     "tsv_op_gemm_qkv": (_i32, [_p, _i64, _p, _i64, _i32, _i32, _i32, _i32, _p, _i64, _p, _i64, _p, _i32, _i32,

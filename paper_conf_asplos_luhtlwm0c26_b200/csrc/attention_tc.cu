@@ -734,7 +734,7 @@ static double kv_makespan(long long n_plain, int plain_cost, long long T, const 
     }
   return *std::max_element(h.begin(), h.end());
 }
-static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
+static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w, int sms_override = 0) {
   static bool env_read = false;
   if (!env_read) {
     if (const char* v = getenv("TSV_KV_MIN")) KV_MIN_TILES = atoi(v);
@@ -752,9 +752,11 @@ static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
   if (!w || !w->cnt || !w->ws) return a;
   static int sms_of[64] = {0};
   int dev = 0;
-  cudaGetDevice(&dev);
-  if (!sms_of[dev & 63]) cudaDeviceGetAttribute(&sms_of[dev & 63], cudaDevAttrMultiProcessorCount, dev);
-  const int sms = sms_of[dev & 63] ? sms_of[dev & 63] : 148;
+  if (sms_override <= 0) {
+    cudaGetDevice(&dev);
+    if (!sms_of[dev & 63]) cudaDeviceGetAttribute(&sms_of[dev & 63], cudaDevAttrMultiProcessorCount, dev);
+  }
+  const int sms = sms_override > 0 ? sms_override : (sms_of[dev & 63] ? sms_of[dev & 63] : 148);
   // the workspace bounds the tail: T items x 2 query tiles x S ranges x (O, m, l) slabs; 4 counters each
   const long long slab = (long long)AT_BM * (D + 2) * 4;
   auto fits = [&](long long T, int S) { return T * 2 * S * slab <= w->ws_bytes && T * 2 * 4 <= w->cnt_ints; };
@@ -813,6 +815,25 @@ static AttnSplitArgs plan_kv_split(int L, int H, int D, const AttnSplitWs* w) {
   a.cnt = w->cnt;
   a.ws = w->ws;
   return a;
+}
+
+// host-only view of the planner (tsv_attention_split_plan): the plan a launch of (L, H, D) would use
+int attention_split_plan(int L, int H, int D, long long ws_bytes, int cnt_ints, int force, int sms, int* n_plain,
+                         int* n_tail, int* nsplit, int* bounds) {
+  static float dummy_ws;
+  static int dummy_cnt;
+  AttnSplitWs w;
+  w.cnt = &dummy_cnt;   // never dereferenced by the planner
+  w.cnt_ints = cnt_ints;
+  w.ws = &dummy_ws;
+  w.ws_bytes = ws_bytes;
+  w.force = force;
+  const AttnSplitArgs a = plan_kv_split(L, H, D, &w, sms > 0 ? sms : 148);
+  *n_plain = a.n_plain;
+  *n_tail = a.n_tail;
+  *nsplit = a.nsplit;
+  for (int z = 0; z < 9; ++z) bounds[z] = a.bound[z];
+  return 0;
 }
 
 // The step's variant per head dim (profiles/README.md, attention table); TSV_ATTN_D128 / TSV_ATTN_D64

@@ -2621,6 +2621,14 @@ tsv_status tsv_op_attention(const void* q, int64_t ldq, const void* k, int64_t l
   return TSV_OK;
 }
 
+tsv_status tsv_attention_split_plan(int L, int H, int D, int64_t ws_bytes, int cnt_ints, int nsplit, int sms,
+                                    int* n_plain, int* n_tail, int* nsplit_out, int* bounds) {
+  if (L <= 0 || H <= 0 || (D != 64 && D != 128)) return fail(TSV_E_INVAL, "split plan: L, H > 0 and D in {64, 128}");
+  if (nsplit < 0 || !n_plain || !n_tail || !nsplit_out || !bounds) return fail(TSV_E_INVAL, "split plan: bad arguments");
+  attention_split_plan(L, H, D, ws_bytes, cnt_ints, nsplit, sms, n_plain, n_tail, nsplit_out, bounds);
+  return TSV_OK;
+}
+
 tsv_status tsv_op_attention_split(const void* q, int64_t ldq, const void* k, int64_t ldk, const void* v, int64_t ldv,
                                   void* o, int64_t ldo, int L, int H, int D, int nsplit, int* cnt, int cnt_ints,
                                   float* ws, int64_t ws_bytes, void* stream) {

@@ -184,6 +184,9 @@ struct AttnSplitWs {
   long long ws_bytes = 0;
   int force = 0;        // > 0: this split factor (tests); 0: automatic
 };
+// the KV-split plan a launch would use (host only; sms <= 0: 148)
+int attention_split_plan(int L, int H, int D, long long ws_bytes, int cnt_ints, int force, int sms, int* n_plain,
+                         int* n_tail, int* nsplit, int* bounds);
 int attention_launch(const bf16* q, long long ldq, const bf16* k, long long ldk, const bf16* v, long long ldv,
                      bf16* o, long long ldo, int L, int H, int D, cudaStream_t s, int version = 3,
                      const AttnScatter* scatter = nullptr, const AttnSplitWs* split = nullptr);
