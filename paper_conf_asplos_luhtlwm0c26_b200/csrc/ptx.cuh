@@ -182,12 +182,16 @@ TSV_DEV uint32_t cluster_ctarank() {
 TSV_DEV void cluster_sync() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
-// arrive on the mbarrier at the same smem offset in CTA `cta` of the cluster
+// arrive on the mbarrier at the same smem offset in CTA `cta` of the cluster.  Default semantics
+// (release at CTA scope), as the tcgen05 consumer-release pattern needs: the caller's TMEM reads are
+// complete (tcgen05.wait::ld) and ordered by tcgen05.fence::before_thread_sync.  `.release.cluster`
+// compiles to MEMBAR.ALL.GPU, which made every epilogue warp wait for all its global stores before
+// freeing the accumulator (ncu: the MMA warp of short-K GEMMs stalled on the TMEM-empty barrier).
 TSV_DEV void mbar_arrive_remote(uint64_t* bar, uint32_t cta) {
   asm volatile(
       "{\n\t.reg .b32 ra;\n\t"
       "mapa.shared::cluster.u32 ra, %0, %1;\n\t"
-      "mbarrier.arrive.release.cluster.shared::cluster.b64 _, [ra];\n\t}" ::"r"(smem_u32(bar)),
+      "mbarrier.arrive.shared::cluster.b64 _, [ra];\n\t}" ::"r"(smem_u32(bar)),
       "r"(cta)
       : "memory");
 }

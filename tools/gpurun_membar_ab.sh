@@ -1,0 +1,10 @@
+# GEMM pair epilogue: remote TMEM-empty arrive without the cluster-scope release (no MEMBAR.ALL.GPU):
+# GEMM + step tests, then whole-step A/B (A = with the membar, B = without)
+cd $GRAFT_REPO_ROOT
+O=gpurun_out
+mkdir -p $O
+timeout -s KILL 1200 python -m pytest tests/test_gpu_kernels.py tests/test_gpu_step.py tests/test_gpu_sd3.py tests/test_gpu_batch.py -m gpu -q -x -p no:cacheprovider > $O/pytest_membar.log 2>&1; echo "pytest exit $?"
+tail -3 $O/pytest_membar.log
+for cfg in "--model sd3 --res 1024" "--model sd3 --res 2048" "--res 2048" "--res 512"; do
+  ARGS="$cfg --steps 10 --warmup 3" ROUNDS=3 bash tools/ab_bench.sh
+done
