@@ -197,7 +197,9 @@ __global__ void __launch_bounds__(FA_THREADS, 1)
   using C = FaCfg<D, KV, RS>;
   constexpr bool JOINT = KV == 3;   // K and V of a tile share one stage and one barrier pair
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1 KB alignment by pointer arithmetic on the shared array (an integer round trip would make the
+  // derived pointers generic: the epilogue's staging accesses compiled to LD.E / ST.E instead of LDS / STS)
+  uint8_t* sm = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
   constexpr int NK = C::NK, NV = C::NV;
   uint64_t* q_full = bars + 0;
