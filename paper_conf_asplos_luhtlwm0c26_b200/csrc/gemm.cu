@@ -242,12 +242,18 @@ __device__ __forceinline__ void stage_chunk(const uint32_t (&r)[32], float* stg,
 }
 
 // epilogue of one 32 x 32 chunk in the staged layout (bias, activation / fp32-stream update, stores)
-__device__ __forceinline__ void finish_chunk(const GemmEpi& e, int M, int row0, int n0, float4 (&a)[8], int lane) {
+// this lane's 4 bias values of the chunk at column n0 (bf16 pairs; zero when the GEMM has no bias)
+__device__ __forceinline__ uint2 load_bias4(const GemmEpi& e, int n0, int lane) {
+  return e.bias ? __ldg(reinterpret_cast<const uint2*>(e.bias + n0 + (lane & 7) * 4)) : make_uint2(0u, 0u);
+}
+// bpre: the chunk's bias values when the caller prefetched them (load_bias4), else read here
+__device__ __forceinline__ void finish_chunk(const GemmEpi& e, int M, int row0, int n0, float4 (&a)[8], int lane,
+                                             const uint2* bpre = nullptr) {
   const int c4 = lane & 7;
   const int col = n0 + c4 * 4;  // this lane's 4 columns for all 8 row groups
   float4 b = make_float4(0.f, 0.f, 0.f, 0.f);
   if (e.bias) {
-    const uint2 bu = __ldg(reinterpret_cast<const uint2*>(e.bias + col));
+    const uint2 bu = bpre ? *bpre : __ldg(reinterpret_cast<const uint2*>(e.bias + col));
     const float2 b0 = unpack_bf16x2(bu.x), b1 = unpack_bf16x2(bu.y);
     b = make_float4(b0.x, b0.y, b1.x, b1.y);
   }
@@ -525,6 +531,10 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       const int Mp = args.M[pr];
       const int acc = it & 1;
       const uint32_t acc_phase = (it >> 1) & 1;
+      // plain epilogues: the first chunk's bias is loaded while the MMAs still run, each next chunk's
+      // while the current one is finished (the load latency sat in front of every chunk)
+      uint2 bnext = make_uint2(0u, 0u);
+      if (!SPLITK) bnext = load_bias4(epi, n_blk * BN, lane);
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
       const int row0 = m_blk * BM + wq * 32;
@@ -540,8 +550,12 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
         for (int c = 0; c < BN / 32; ++c) {
           uint32_t r[32];
           tmem_ld32(tbase + c * 32, r);
+          const uint2 bcur = bnext;
+          if (c + 1 < BN / 32) bnext = load_bias4(epi, n_blk * BN + (c + 1) * 32, lane);
           tmem_ld_wait();
-          epilogue_chunk(epi, Mp, row0, n_blk * BN + c * 32, r, stg, lane);
+          float4 a[8];
+          stage_chunk(r, stg, lane, a);
+          finish_chunk(epi, Mp, row0, n_blk * BN + c * 32, a, lane, &bcur);
         }
       }
       tc_fence_before();
@@ -708,6 +722,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
       const int Mp = args.M[pr];
       const int acc = it & 1;
       const uint32_t acc_phase = (it >> 1) & 1;
+      // plain epilogues: bias prefetched one chunk ahead (see gemm_tc_kernel)
+      uint2 bnext = make_uint2(0u, 0u);
+      if (!SPLITK) bnext = load_bias4(epi, n_blk * BN, lane);
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
       const int row0 = m_blk * 256 + (int)rank * 128 + wq * 32;
@@ -723,8 +740,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GEMM_THREADS, 1)
         for (int c = 0; c < BN / 32; ++c) {
           uint32_t r[32];
           tmem_ld32(tbase + c * 32, r);
+          const uint2 bcur = bnext;
+          if (c + 1 < BN / 32) bnext = load_bias4(epi, n_blk * BN + (c + 1) * 32, lane);
           tmem_ld_wait();
-          epilogue_chunk(epi, Mp, row0, n_blk * BN + c * 32, r, stg, lane);
+          float4 a[8];
+          stage_chunk(r, stg, lane, a);
+          finish_chunk(epi, Mp, row0, n_blk * BN + c * 32, a, lane, &bcur);
         }
       }
       tc_fence_before();
